@@ -1,0 +1,106 @@
+"""Pins for oracle/coverage.py: exhaustive interleavings on tiny instances
+(Fig. 2's 2 SMs x 2 CTAs), hand-traced trajectories, a closed form for the final counter,
+temporal-equivalence of n >= num_sms, and a planted bug the checker must catch."""
+import itertools
+
+import pytest
+
+from oracle import coverage as cv
+
+
+def _cfg(**kw):
+    base = dict(n_blocks=5, chunk=1, poll=1, worker_sm=(0, 0, 1, 1), num_sms=2,
+                preempt_widths=(1, 2), max_events=2)
+    base.update(kw)
+    return cv.Config(**base)
+
+
+@pytest.mark.parametrize("C,K", list(itertools.product([1, 2], [1, 2])))
+def test_exhaustive_no_violations_fig2(C, K):
+    # Fig. 2: two SMs, two CTAs each; up to 2 preempt events (spatial 1 SM or temporal)
+    r = cv.explore(_cfg(n_blocks=5 if (C, K) != (1, 2) else 4, chunk=C, poll=K))
+    assert r.violations == set()
+    assert r.terminals > 0
+    assert r.preempted_epoch_ends > 0      # preempted epochs really are explored
+
+
+def test_exhaustive_with_clear_events():
+    r = cv.explore(_cfg(n_blocks=6, chunk=2, poll=2, allow_clear=True))
+    assert r.violations == set()
+
+
+def test_planted_bug_is_caught():
+    r = cv.explore(_cfg(bug_exit_holding_chunk=True))
+    assert any(v.startswith("I1") for v in r.violations)
+    assert any(v.startswith("I2") for v in r.violations)
+
+
+def test_final_counter_closed_form_without_preemption():
+    for n, C, ws in [(5, 1, (0, 0, 1, 1)), (5, 2, (0, 1)), (7, 3, (0, 0, 1)), (4, 4, (0,))]:
+        r = cv.explore(cv.Config(n_blocks=n, chunk=C, poll=1, worker_sm=ws, num_sms=2))
+        assert r.violations == set()
+        assert r.terminal_ctrs == {cv.final_counter_no_preempt(n, C, len(ws))}
+
+
+def test_temporal_equivalence_n_ge_num_sms():
+    # I4 / P:174: spa_P >= number of SMs behaves exactly as temporal preemption
+    a = cv.explore(_cfg(preempt_widths=(2,), max_events=1))
+    b = cv.explore(_cfg(preempt_widths=(7,), max_events=1))
+    assert (a.states, a.terminals, a.terminal_ctrs, a.preempted_epoch_ends) == \
+           (b.states, b.terminals, b.terminal_ctrs, b.preempted_epoch_ends)
+
+
+def _pick(seq):
+    """Choose successors by label prefix in order; falls back to the first successor."""
+    it = iter(seq)
+    want = [next(it, None)]
+
+    def choose(labels):
+        w = want[0]
+        if w is not None:
+            for i, lab in enumerate(labels):
+                if lab == w:
+                    want[0] = next(it, None)
+                    return i
+        return 0
+    return choose
+
+
+def test_hand_traced_temporal_preempt_after_one_chunk():
+    # one worker on SM0, N=3, C=1, K=1: poll, fetch b0, process, preempt, poll -> yield.
+    cfg = cv.Config(n_blocks=3, chunk=1, poll=1, worker_sm=(0,), num_sms=2,
+                    preempt_widths=(2,), max_events=1)
+    st = cv.initial_state(cfg)
+    for lab in ["w0.poll", "w0.fetch", "w0.proc", "preempt(2)", "w0.poll", "w0.exit"]:
+        st = dict(cv.successors(cfg, st))[lab]
+    ctr, ctrl, done, exited, cov, epoch, status, workers, ev = st
+    assert status == cv.ST_PREEMPTED and cov == (1, 0, 0) and ctr == 1 and done == 1
+    assert list(cov) == cv.expected_prefix(ctr, 3)
+    # resume: a fresh epoch ignores the stale request (gen 0) and finishes the rest
+    st = dict(cv.successors(cfg, st))["resume"]
+    for lab in ["w0.poll", "w0.fetch", "w0.proc", "w0.poll", "w0.fetch", "w0.proc", "w0.poll",
+                "w0.fetch", "w0.exit"]:
+        st = dict(cv.successors(cfg, st))[lab]
+    assert st[6] == cv.ST_DONE and st[4] == (1, 1, 1) and st[0] == 4
+
+
+def test_hand_traced_spatial_keeps_other_sm_running():
+    # workers on SM0 and SM1, spatial request n=1 yields SM0 only (rank = smid)
+    cfg = cv.Config(n_blocks=4, chunk=1, poll=1, worker_sm=(0, 1), num_sms=2,
+                    preempt_widths=(1,), max_events=1)
+    st = cv.initial_state(cfg)
+    for lab in ["preempt(1)", "w0.poll", "w1.poll", "w0.exit"]:
+        st = dict(cv.successors(cfg, st))[lab]
+    workers = st[7]
+    assert workers[0][3] == cv.R_YIELD and workers[1][0] == cv.FETCH
+    for lab in ["w1.fetch", "w1.proc", "w1.poll", "w1.fetch", "w1.proc", "w1.poll", "w1.fetch",
+                "w1.proc", "w1.poll", "w1.fetch", "w1.proc", "w1.poll", "w1.fetch", "w1.exit"]:
+        st = dict(cv.successors(cfg, st))[lab]
+    assert st[6] == cv.ST_DONE and st[4] == (1, 1, 1, 1)
+    assert st[7][1][3] == cv.R_EXHAUSTED
+
+
+def test_expected_prefix():
+    assert cv.expected_prefix(0, 3) == [0, 0, 0]
+    assert cv.expected_prefix(2, 3) == [1, 1, 0]
+    assert cv.expected_prefix(9, 3) == [1, 1, 1]
