@@ -1,0 +1,247 @@
+/*
+ * flep.h — C ABI of the B200-native FLEP runtime (preemptable persistent-CTA kernels).
+ *
+ * Paper: Wu, Liu, Zhou, Jiang, "FLEP: Enabling Flexible and Efficient Preemption on GPUs",
+ * ASPLOS'17. "P:N" = line N of the paper text.
+ *
+ * What the library does: a registered kernel is launched as a grid of
+ * resident worker CTAs (persistent threads) that pull chunks of C original
+ * block indices from a global atomic counter (pull_task, Fig. 4), run the
+ * original block body on each, and poll a 32-bit control word every K chunks (amortized check,
+ * Fig. 4(b)). On a preemption request either all workers exit (temporal, Fig. 4(a/b),
+ * P:164) or only those whose SM is among the n released ones (spatial, Fig. 4(c)).
+ * Progress lives in the counter, so a resume launch runs every original block exactly once
+ * (P:126). A host runtime intercepts launches and, in managed modes,
+ * decides who is preempted and when (HPF/SRPT, Fig. 6, §5.2; FIFO and kernel-slicing baselines).
+ *
+ * Conventions (all functions):
+ *   - Return flep_status: 0 = FLEP_OK, < 0 = error. Never throw, never abort. After an error,
+ *     flep_last_error() returns a thread-local human-readable message.
+ *   - A sticky CUDA error makes every later call return FLEP_ERR_CUDA; re-initialise.
+ *   - Device pointers passed inside argument structs belong to the caller and must stay valid
+ *     until flep_sync() has returned FLEP_OK for that launch. Argument structs are copied by
+ *     value at flep_launch().
+ *   - The runtime owns its control blocks, internal CUDA streams (one high-priority control
+ *     stream, a pool of execution streams) and pinned host status words.
+ *   - flep_launch / flep_preempt / flep_resume are asynchronous. Completion is observable
+ *     through flep_sync / flep_query. When flep_options.order_user_stream is set, work the
+ *     caller enqueues on `stream` after flep_launch waits for TRUE completion (every block done,
+ *     possibly after several preempt/resume cycles), via a stream wait on the done counter.
+ *   - Priority: larger value = higher priority (Fig. 6 line 1: Kr.priority < Kn.priority ->
+ *     preempt). The runtime maps it onto CUDA stream priorities internally.
+ *   - One runtime per device; all entry points are thread-safe (internal mutex).
+ */
+#ifndef FLEP_H
+#define FLEP_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  FLEP_OK = 0,
+  FLEP_ERR_INVALID = -1,      /* bad argument: n_sms == 0, empty grid, unknown body/kernel/handle */
+  FLEP_ERR_STATE = -2,        /* operation not allowed in the launch's current state / mode */
+  FLEP_ERR_CUDA = -3,         /* CUDA runtime/driver error (message in flep_last_error) */
+  FLEP_ERR_NOMEM = -4,        /* device or pinned host allocation failed */
+  FLEP_ERR_TIMEOUT = -5,      /* flep_sync timeout expired (launch still in flight) */
+  FLEP_ERR_UNSUPPORTED = -6   /* feature not available on this device/build */
+} flep_status;
+
+typedef struct flep_rt_s* flep_rt;   /* one runtime per GPU */
+typedef int32_t flep_kernel;          /* registered kernel id (>= 0) */
+typedef int64_t flep_launch_t;        /* one invocation (>= 1); handle for preempt/resume/sync */
+typedef void* flep_stream_t;          /* a cudaStream_t (NULL = legacy default stream) */
+
+typedef struct { uint32_t x, y, z; } flep_dim3;
+
+typedef enum {
+  FLEP_POLICY_MANUAL = 0,  /* caller issues preempt/resume itself (mechanism only) */
+  FLEP_POLICY_FIFO = 1,    /* interception, no preemption, arrival order (MPS co-run baseline) */
+  FLEP_POLICY_HPF = 2,     /* Fig. 6: priority preemption + SRPT within a priority (§5.2.1) */
+  FLEP_POLICY_SLICE = 3    /* HPF decisions on the kernel-slicing mechanism (P:96, P:391 baseline) */
+} flep_policy;
+
+typedef enum {
+  FLEP_FLAG_STREAM_MEMOP = 0,  /* ctrl word in device memory, written by cuStreamWriteValue32 on a
+                                  high-priority control stream (needs no SM) */
+  FLEP_FLAG_HOST_MAPPED = 1    /* ctrl word in mapped pinned host memory, written by a CPU store
+                                  (the paper's temp_P in pinned memory) */
+} flep_flag_transport;
+
+typedef enum {
+  FLEP_BODY_SAXPY_I32 = 1,     /* y <- a*x + y, int32, wraps mod 2^32; 256 elements per block */
+  FLEP_BODY_SAXPY_F32 = 2,     /* y <- a*x + y, fp32; 256 elements per block */
+  FLEP_BODY_SPMV_CSR_F32 = 3,  /* y = A x, CSR fp32; 32 rows per block */
+  FLEP_BODY_STENCIL5_F32 = 4,  /* 5-point out-of-place sweep, fp32; 64x64 cells per block */
+  FLEP_BODY_STENCIL5_I32 = 5,  /* 5-point integer sweep, wraps mod 2^32; 64x64 cells per block */
+  FLEP_BODY_GEMM_BF16 = 6      /* C = A B^T, bf16 in, fp32 accumulate (tcgen05), bf16 out;
+                                  128x256 output tile per block */
+} flep_body;
+
+/* Per-body argument structs (copied by value at launch). All pointers are device pointers. */
+typedef struct { int32_t* y; const int32_t* x; int32_t a; uint32_t n; } flep_saxpy_i32_args;
+typedef struct { float* y; const float* x; float a; uint32_t n; } flep_saxpy_f32_args;
+typedef struct {
+  float* y; const int32_t* rowptr; const int32_t* col; const float* val; const float* x;
+  uint32_t rows;
+} flep_spmv_args;
+/* in/out: n x n row-major, float (STENCIL5_F32) or int32 (STENCIL5_I32); out != in. */
+typedef struct { void* out; const void* in; uint32_t n; } flep_stencil_args;
+/* a: M x K row-major bf16, b: N x K row-major bf16 (K-major "TN"), c: M x N row-major bf16.
+   M % 128 == 0, N % 256 == 0, K % 64 == 0. */
+typedef struct { void* c; const void* a; const void* b; uint32_t m, n, k; } flep_gemm_args;
+
+typedef struct {
+  int32_t policy;              /* flep_policy */
+  int32_t flag;                /* flep_flag_transport */
+  uint32_t default_chunk;      /* C: original blocks per counter fetch (0 -> 8) */
+  uint32_t default_poll;       /* K: chunks between control-word polls (0 -> 1) */
+  uint32_t debug_coverage;     /* 1: keep a per-block execution count cov[N] (test builds) */
+  uint32_t order_user_stream;  /* 1: caller stream waits for true completion (see above) */
+  uint32_t slice_blocks;       /* SLICE policy: blocks per sub-kernel (0 -> W*C*K, A20) */
+} flep_options;
+
+typedef struct {
+  const char* name;
+  int32_t body;                /* flep_body */
+  uint32_t chunk, poll;        /* C, K (0 = runtime defaults) */
+  double model[5];             /* ridge model: T_e ns = m0*grid + m1*cta + m2*input
+                                  + m3*smem + m4, rounded once to integer ns */
+  int64_t preempt_overhead_ns; /* O: profiled mean preemption overhead */
+} flep_kernel_desc;
+
+typedef enum {
+  FLEP_STATE_QUEUED = 0,     /* intercepted, waiting for a scheduling decision (S2) */
+  FLEP_STATE_RUNNING = 1,    /* workers launched, no request pending (S3) */
+  FLEP_STATE_YIELDING = 2,   /* temporal request issued, epoch not yet drained */
+  FLEP_STATE_PREEMPTED = 3,  /* epoch drained with blocks left; resumable */
+  FLEP_STATE_PARTIAL = 4,    /* spatial request in force: running on the non-released SMs */
+  FLEP_STATE_DONE = 5        /* every original block executed exactly once */
+} flep_state;
+
+typedef struct {
+  int32_t state;               /* flep_state */
+  uint32_t epoch;              /* number of worker grids launched so far (1 after first launch) */
+  uint64_t blocks_total;       /* N */
+  uint64_t blocks_done;        /* done counter as of the last drained epoch */
+  uint64_t counter;            /* task counter value (may exceed N by <= W*C, A5) */
+  int64_t t_e, t_w, t_r;       /* execution-status triplet, ns (§5.1) */
+  int64_t t_arrive, t_first_start, t_finish;  /* host steady clock, ns */
+  uint32_t workers;            /* W: worker CTAs per epoch */
+  uint32_t n_yield;            /* yield width currently requested (0 = none) */
+} flep_launch_info;
+
+/* Per-worker event record of one epoch (device %globaltimer, ns). */
+typedef struct {
+  uint32_t smid;      /* %smid the worker ran on */
+  uint32_t reason;    /* 1 = yielded on request, 2 = counter exhausted */
+  uint32_t n_blocks;  /* original blocks this worker executed */
+  uint32_t epoch;     /* epoch the record belongs to */
+  uint64_t t_entry;   /* worker start */
+  uint64_t t_exit;    /* worker exit */
+} flep_worker_event;
+
+/* Per-epoch device summary. */
+typedef struct {
+  uint64_t t_trigger;      /* device self-trigger time (0 if none fired this epoch) */
+  uint64_t t_end;          /* last worker exit of the epoch */
+  uint32_t trigger_block;  /* block index that fired it */
+  uint32_t done;           /* done counter at epoch end */
+  uint32_t counter;        /* task counter at epoch end */
+  uint32_t state;          /* 3 = PREEMPTED, 5 = DONE */
+} flep_epoch_info;
+
+/* ---- lifecycle ------------------------------------------------------------------------ */
+/* Create the runtime for CUDA device `device`. opts may be NULL (defaults). */
+flep_status flep_init(int device, const flep_options* opts, flep_rt* out);
+/* Cancel every unfinished launch (unblocking waiting streams), synchronise, free everything. */
+flep_status flep_shutdown(flep_rt rt);
+/* num_sms = multiprocessor count; nsmid = %nsmid upper bound of %smid values. */
+flep_status flep_device_info(flep_rt rt, uint32_t* num_sms, uint32_t* nsmid);
+
+/* ---- kernels and launches ------------------------------------------------------------- */
+flep_status flep_register_kernel(flep_rt rt, const flep_kernel_desc* desc, flep_kernel* out);
+/* Intercepted launch: `grid` is the ORIGINAL grid in blocks; `args` points to the
+   body's argument struct of exactly `args_size` bytes. In MANUAL mode the workers are launched
+   immediately; in managed modes the policy decides (launch now, preempt the running kernel,
+   or queue). */
+flep_status flep_launch(flep_rt rt, flep_kernel k, flep_dim3 grid, const void* args,
+                        size_t args_size, int32_t priority, flep_stream_t stream,
+                        flep_launch_t* out);
+/* MANUAL mode only. Ask a running launch to yield n_sms SMs (n_sms >= num_sms: temporal,
+   P:174). Within one epoch a request can only widen. FLEP_ERR_INVALID if n_sms == 0. */
+flep_status flep_preempt(flep_rt rt, flep_launch_t h, uint32_t n_sms);
+/* MANUAL mode only. PREEMPTED: relaunch the workers on the same counter (stream-ordered after
+   the drained grid). PARTIAL: withdraw the spatial request (the remaining workers continue). */
+flep_status flep_resume(flep_rt rt, flep_launch_t h);
+/* Wait until the launch is DONE (timeout_ns < 0: forever). Also waits for its last grid. */
+flep_status flep_sync(flep_rt rt, flep_launch_t h, int64_t timeout_ns);
+/* Refresh and return the launch's state (never blocks). */
+flep_status flep_query(flep_rt rt, flep_launch_t h, flep_launch_info* out);
+/* Abandon a launch: temporal preempt, drain, mark done so no stream waits forever. */
+flep_status flep_cancel(flep_rt rt, flep_launch_t h);
+/* Wait for the current epoch of h to drain (state leaves RUNNING/YIELDING/PARTIAL). */
+flep_status flep_wait_epoch(flep_rt rt, flep_launch_t h, int64_t timeout_ns);
+
+/* ---- baselines (same bodies, no wrapper) ----------------------------------------------- */
+/* The original kernel: one CTA per original block (unwrapped twin, K7). */
+flep_status flep_launch_unwrapped(flep_rt rt, int32_t body, flep_dim3 grid, const void* args,
+                                  size_t args_size, flep_stream_t stream);
+/* Kernel slicing (K8): ceil(N/slice_blocks) back-to-back sub-kernels of slice_blocks. */
+flep_status flep_launch_sliced(flep_rt rt, int32_t body, flep_dim3 grid, const void* args,
+                               size_t args_size, uint32_t slice_blocks, flep_stream_t stream);
+/* Worker grid size W (= resident CTAs per SM x SMs) for a body / chunk. */
+flep_status flep_workers_for(flep_rt rt, int32_t body, uint32_t* ctas_per_sm, uint32_t* workers);
+
+/* ---- test / bench hooks (always compiled; cost nothing when unused) -------------------- */
+/* Device self-trigger: the worker that fetches the chunk holding `block_index` writes the
+   request (epoch, n_sms) itself. Applies to the launch's next epoch if it is not running. */
+flep_status flep_debug_trigger_at(flep_rt rt, flep_launch_t h, uint64_t block_index,
+                                  uint32_t n_sms);
+/* Arm a self-trigger for the NEXT flep_launch issued on this runtime. */
+flep_status flep_debug_arm_next_trigger(flep_rt rt, uint64_t block_index, uint32_t n_sms);
+/* Copy cov[0..n) (debug_coverage runtimes only). */
+flep_status flep_debug_copy_coverage(flep_rt rt, flep_launch_t h, uint32_t* host_out, size_t n);
+/* Copy the worker event records of epoch `epoch` (1-based; the last 8 epochs are kept). */
+flep_status flep_debug_copy_events(flep_rt rt, flep_launch_t h, uint32_t epoch,
+                                   flep_worker_event* host_out, size_t max_records,
+                                   size_t* n_out);
+flep_status flep_debug_epoch_info(flep_rt rt, flep_launch_t h, uint32_t epoch,
+                                  flep_epoch_info* out);
+/* Set the spatial rank table: rank[smid] for smid < nsmid (default rank = smid). */
+flep_status flep_set_rank_table(flep_rt rt, const uint16_t* rank, uint32_t n);
+/* Host steady-clock now, ns (the clock all host timestamps use). */
+int64_t flep_now_ns(void);
+/* Decision log of the managed runtime: n records of (t_ns, action, launch, n_sms) with
+   action 0 = LAUNCH, 1 = RESUME, 2 = PREEMPT; and the event log (t_ns, type, launch) with
+   type 0 = ARRIVE, 1 = FINISH, plus per-launch (priority, t_e, overhead). */
+flep_status flep_decision_log(flep_rt rt, int64_t* out4, size_t max_records, size_t* n_out);
+flep_status flep_event_log(flep_rt rt, int64_t* out6, size_t max_records, size_t* n_out);
+
+/* ---- pure policy engine (host only; no GPU needed) -------------------------------------
+   The exact decision logic the managed runtime uses (Fig. 6), exposed for replay parity with
+   the oracle's discrete-event simulation. kind: 1 FIFO, 2 HPF, 3 SLICE (= HPF decisions). */
+typedef struct flep_policy_s* flep_policy_t;
+flep_status flep_policy_create(int32_t kind, uint32_t num_sms, flep_policy_t* out);
+flep_status flep_policy_destroy(flep_policy_t p);
+flep_status flep_policy_arrive(flep_policy_t p, int64_t t_ns, int64_t id, int32_t priority,
+                               int64_t t_e_ns, int64_t overhead_ns);
+flep_status flep_policy_finish(flep_policy_t p, int64_t t_ns, int64_t id);
+/* Decisions emitted so far: records of 4 int64 (t_ns, action, id, n_sms). */
+flep_status flep_policy_decisions(flep_policy_t p, int64_t* out4, size_t max_records,
+                                  size_t* n_out);
+/* T_e ns from a 5-term model, rounded once (half away from zero), clamped >= 1. */
+int64_t flep_model_predict_ns(const double model[5], double grid, double cta, double input,
+                              double smem);
+
+const char* flep_last_error(void);
+const char* flep_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* FLEP_H */

@@ -1,0 +1,172 @@
+// bodies.cuh — original block bodies of the memory-bound workloads.
+//
+// Each body executes a contiguous range [b0, b1) of ORIGINAL block indices with all threads of
+// the CTA (the wrapper passes a chunk, the unwrapped twin passes one block). Per-block work is
+// identical in both, so wrapped, unwrapped, sliced and preempted-then-resumed runs produce
+// bit-identical outputs (SURVEY §8(c) "Parity criteria").
+//
+//   SAXPY  (VA-shaped, Table 1): block b = elements [256b, 256b+256); 128-bit ld/st.
+//   SpMV   (SPMV): block b = rows [32b, 32b+32); 8 lanes per row, fixed-order reduction.
+//   Stencil5 (BJ "2D stencil"; PF/CFD-shaped): block (tx, ty) = 64x64 output tile; each thread
+//          produces 4 contiguous cells per row pass with 128-bit loads; neighbours come from the
+//          L1/L2-resident rows of the same and adjacent tiles.
+#pragma once
+#include <cstdint>
+#include "../../include/flep.h"
+
+namespace flep {
+
+__device__ __forceinline__ int4 ldcs4(const int4* p) { return __ldcs(p); }
+__device__ __forceinline__ void stcs4(int4* p, int4 v) { __stcs(p, v); }
+
+// ---------------------------------------------------------------------------------------------
+// SAXPY: y <- a*x + y. int32 wraps modulo 2^32 (computed in uint32); fp32 uses one fma per element.
+template <bool kInt>
+struct SaxpyBody {
+  static constexpr int kThreads = 256;
+  static constexpr int kMinBlocks = 8;
+  static constexpr uint32_t kBlockElems = 256;
+  using Args = typename std::conditional<kInt, flep_saxpy_i32_args, flep_saxpy_f32_args>::type;
+
+  __device__ __forceinline__ static uint32_t op(uint32_t a, uint32_t x, uint32_t y, std::true_type) {
+    return a * x + y;
+  }
+  __device__ __forceinline__ static uint32_t op(uint32_t a, uint32_t x, uint32_t y, std::false_type) {
+    return __float_as_uint(fmaf(__uint_as_float(a), __uint_as_float(x), __uint_as_float(y)));
+  }
+  __device__ __forceinline__ static uint32_t f(uint32_t a, uint32_t x, uint32_t y) {
+    return op(a, x, y, std::integral_constant<bool, kInt>{});
+  }
+
+  __device__ static void run(const Args& g, uint32_t b0, uint32_t b1, uint32_t, uint32_t) {
+    const uint64_t e0 = (uint64_t)b0 * kBlockElems;
+    const uint64_t e1 = min((uint64_t)b1 * kBlockElems, (uint64_t)g.n);
+    if (e0 >= e1) return;
+    const uint32_t a = kInt ? (uint32_t)g.a : __float_as_uint((float)g.a);
+    const uint32_t* __restrict__ x = reinterpret_cast<const uint32_t*>(g.x) + e0;
+    uint32_t* __restrict__ y = reinterpret_cast<uint32_t*>(g.y) + e0;
+    const uint32_t nvec = (uint32_t)((e1 - e0) >> 2);
+    const int4* __restrict__ x4 = reinterpret_cast<const int4*>(x);
+    int4* __restrict__ y4 = reinterpret_cast<int4*>(y);
+    constexpr uint32_t U = 2;                    // 2 x 128-bit loads of x and of y in flight
+    uint32_t v = threadIdx.x;
+    for (; v + (U - 1) * kThreads < nvec; v += U * kThreads) {
+      int4 xv[U], yv[U];
+#pragma unroll
+      for (uint32_t u = 0; u < U; ++u) { xv[u] = ldcs4(x4 + v + u * kThreads); yv[u] = ldcs4(y4 + v + u * kThreads); }
+#pragma unroll
+      for (uint32_t u = 0; u < U; ++u) {
+        int4 r;
+        r.x = (int)f(a, (uint32_t)xv[u].x, (uint32_t)yv[u].x);
+        r.y = (int)f(a, (uint32_t)xv[u].y, (uint32_t)yv[u].y);
+        r.z = (int)f(a, (uint32_t)xv[u].z, (uint32_t)yv[u].z);
+        r.w = (int)f(a, (uint32_t)xv[u].w, (uint32_t)yv[u].w);
+        stcs4(y4 + v + u * kThreads, r);
+      }
+    }
+    for (; v < nvec; v += kThreads) {
+      const int4 xv = ldcs4(x4 + v), yv = ldcs4(y4 + v);
+      int4 r;
+      r.x = (int)f(a, (uint32_t)xv.x, (uint32_t)yv.x);
+      r.y = (int)f(a, (uint32_t)xv.y, (uint32_t)yv.y);
+      r.z = (int)f(a, (uint32_t)xv.z, (uint32_t)yv.z);
+      r.w = (int)f(a, (uint32_t)xv.w, (uint32_t)yv.w);
+      stcs4(y4 + v, r);
+    }
+    const uint64_t tail = e0 + ((uint64_t)nvec << 2);   // ragged tail (n % 4 != 0)
+    for (uint64_t e = tail + threadIdx.x; e < e1; e += kThreads) y[e - e0] = f(a, x[e - e0], y[e - e0]);
+  }
+};
+
+// ---------------------------------------------------------------------------------------------
+// SpMV-CSR fp32: y[r] = sum_p val[p] * x[col[p]]. 8 lanes per row: lane l accumulates
+// p = start+l, start+l+8, ... with fma in that order, then a fixed xor-butterfly over 8 lanes.
+struct SpmvBody {
+  static constexpr int kThreads = 256;
+  static constexpr int kMinBlocks = 8;
+  static constexpr uint32_t kRowsPerBlock = 32;
+  using Args = flep_spmv_args;
+
+  __device__ static void run(const Args& g, uint32_t b0, uint32_t b1, uint32_t, uint32_t) {
+    const uint32_t lane8 = threadIdx.x & 7u;
+    const uint32_t rloc = threadIdx.x >> 3;
+    for (uint32_t b = b0; b < b1; ++b) {
+      const uint32_t row = b * kRowsPerBlock + rloc;
+      float sum = 0.f;
+      if (row < g.rows) {
+        const int32_t s = __ldg(g.rowptr + row), e = __ldg(g.rowptr + row + 1);
+        for (int32_t p = s + (int32_t)lane8; p < e; p += 8)
+          sum = fmaf(__ldcs(g.val + p), __ldg(g.x + __ldcs(g.col + p)), sum);
+      }
+      sum += __shfl_xor_sync(0xffffffffu, sum, 4);
+      sum += __shfl_xor_sync(0xffffffffu, sum, 2);
+      sum += __shfl_xor_sync(0xffffffffu, sum, 1);
+      if (row < g.rows && lane8 == 0) __stcs(g.y + row, sum);
+    }
+  }
+};
+
+// ---------------------------------------------------------------------------------------------
+// 5-point stencil, out-of-place. Interior: fp32 0.5*c + 0.125*(n + s + w + e); int32
+// 4c - n - s - w - e (mod 2^32). Boundary rows/columns copied through.
+template <bool kInt>
+struct Stencil5Body {
+  static constexpr int kThreads = 256;
+  static constexpr int kMinBlocks = 6;
+  static constexpr uint32_t kTile = 64;
+  using Args = flep_stencil_args;
+
+  __device__ __forceinline__ static uint32_t cell(uint32_t c, uint32_t n, uint32_t s, uint32_t w, uint32_t e) {
+    if (kInt) return 4u * c - n - s - w - e;
+    const float fc = __uint_as_float(c), fn = __uint_as_float(n), fs = __uint_as_float(s),
+                fw = __uint_as_float(w), fe = __uint_as_float(e);
+    return __float_as_uint(0.5f * fc + 0.125f * (((fn + fs) + fw) + fe));
+  }
+
+  __device__ static void run(const Args& g, uint32_t b0, uint32_t b1, uint32_t gx, uint32_t) {
+    const uint32_t n = g.n;
+    const uint32_t* __restrict__ in = reinterpret_cast<const uint32_t*>(g.in);
+    uint32_t* __restrict__ out = reinterpret_cast<uint32_t*>(g.out);
+    for (uint32_t b = b0; b < b1; ++b) {
+      const uint32_t tx = b % gx, ty = b / gx;
+      const uint32_t r0 = ty * kTile, c0 = tx * kTile;
+      if ((n & 3u) == 0) {
+        const uint32_t q = threadIdx.x & 15u, rr = threadIdx.x >> 4;   // 16 float4 x 16 rows
+        const uint32_t c = c0 + 4u * q;
+#pragma unroll
+        for (uint32_t pass = 0; pass < kTile / 16; ++pass) {
+          const uint32_t r = r0 + rr + 16u * pass;
+          if (r >= n || c >= n) continue;
+          const size_t off = (size_t)r * n + c;
+          const uint4 C = __ldg(reinterpret_cast<const uint4*>(in + off));
+          uint4 O;
+          if (r == 0 || r == n - 1) {
+            O = C;
+          } else {
+            const uint4 N = __ldg(reinterpret_cast<const uint4*>(in + off - n));
+            const uint4 S = __ldg(reinterpret_cast<const uint4*>(in + off + n));
+            const uint32_t W = (c > 0) ? __ldg(in + off - 1) : 0u;
+            const uint32_t E = (c + 4 < n) ? __ldg(in + off + 4) : 0u;
+            O.x = (c == 0) ? C.x : cell(C.x, N.x, S.x, W, C.y);
+            O.y = cell(C.y, N.y, S.y, C.x, C.z);
+            O.z = cell(C.z, N.z, S.z, C.y, C.w);
+            O.w = (c + 3 == n - 1) ? C.w : cell(C.w, N.w, S.w, C.z, E);
+          }
+          __stcs(reinterpret_cast<uint4*>(out + off), O);
+        }
+      } else {
+        // scalar path for n % 4 != 0 (ragged rows)
+        for (uint32_t t = threadIdx.x; t < kTile * kTile; t += kThreads) {
+          const uint32_t r = r0 + t / kTile, c = c0 + t % kTile;
+          if (r >= n || c >= n) continue;
+          const size_t off = (size_t)r * n + c;
+          const uint32_t C = __ldg(in + off);
+          if (r == 0 || r == n - 1 || c == 0 || c == n - 1) { out[off] = C; continue; }
+          out[off] = cell(C, __ldg(in + off - n), __ldg(in + off + n), __ldg(in + off - 1), __ldg(in + off + 1));
+        }
+      }
+    }
+  }
+};
+
+}  // namespace flep

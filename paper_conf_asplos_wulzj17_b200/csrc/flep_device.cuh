@@ -1,0 +1,197 @@
+// flep_device.cuh — the preemptable persistent-CTA wrapper for sm_100a.
+//
+// Paper mapping (P:N = line N of the FLEP paper text):
+//   persistent threads, W = num_SMs x max_CTAs_per_SM resident workers ..... P:128
+//   pull_task(): global atomic task counter, one thread per CTA + smem bcast
+//   temporal check at the loop top, amortised over L tasks ................. Fig. 4(a)(b)
+//   spatial check hostSM_ID < spa_P (here: rank[%smid] < n) ................ Fig. 4(c)
+//   progress tracked in a global counter so a relaunch resumes ............. P:126
+//
+// B200 design: one 32-bit control word ctrl = epoch<<16 | n in device memory,
+// polled with ld.acquire.gpu (an L2 hit) once per K chunks; a chunk is C original blocks per
+// atomicAdd (the probe measured ~1.46 fetches/ns chip-wide on one address, so C amortises the
+// atomic); exits happen only at poll points or on exhaustion, never while holding a chunk
+// (exactly-once, reading A4). The last worker of an epoch publishes DONE/PREEMPTED to a pinned
+// host word with a system-scope release store.
+#pragma once
+#include <cstdint>
+
+namespace flep {
+
+constexpr uint32_t kReasonYield = 1;
+constexpr uint32_t kReasonExhausted = 2;
+constexpr uint32_t kStatePreempted = 3;
+constexpr uint32_t kStateDone = 5;
+constexpr uint32_t kEvEpochs = 8;       // event log ring: last 8 epochs per launch
+constexpr uint32_t kNoTrigger = 0xffffffffu;
+
+// Per-launch control block in device memory. Hot words on separate 128-B lines.
+struct alignas(128) ControlBlock {
+  uint32_t ctr;            // task counter: next original block index to hand out (D4)
+  uint32_t _p0[31];
+  uint32_t ctrl;           // epoch<<16 | n_yield (D1/D2); device copy for the memop transport
+  uint32_t _p1[31];
+  uint32_t done;           // original blocks executed (all epochs)
+  uint32_t exited;         // workers of the current epoch that have exited (reset by the last)
+  uint32_t _p2[30];
+  // per-epoch summaries (ring of kEvEpochs)
+  uint64_t ep_t_trigger[kEvEpochs];
+  uint64_t ep_t_end[kEvEpochs];
+  uint32_t ep_trigger_block[kEvEpochs];
+  uint32_t ep_done[kEvEpochs];
+  uint32_t ep_ctr[kEvEpochs];
+  uint32_t ep_state[kEvEpochs];
+};
+
+struct WorkerEvent {       // mirrors flep_worker_event
+  uint32_t smid, reason, n_blocks, epoch;
+  uint64_t t_entry, t_exit;
+};
+
+struct HostStatus {        // pinned, mapped; one 32-B slot per launch
+  uint32_t word;           // (epoch << 8) | state, epoch 1-based; written last (release.sys)
+  uint32_t done;           // done counter at the end of that epoch
+  uint32_t ctr;            // task counter at the end of that epoch
+  uint32_t ctrl;           // FLEP_FLAG_HOST_MAPPED: the control word itself (CPU-written)
+  uint64_t t_end;          // %globaltimer of the last exit
+  uint64_t _pad;
+};
+
+struct WorkerParams {
+  ControlBlock* cb;
+  uint32_t* ctrl;          // &cb->ctrl, or a mapped host word (FLEP_FLAG_HOST_MAPPED)
+  uint32_t* cov;           // per-block execution counts or nullptr
+  WorkerEvent* ev;         // [kEvEpochs][W]
+  HostStatus* status;      // device alias of the pinned status word
+  const uint16_t* rank;    // rank[smid]
+  uint32_t n_blocks;       // N
+  uint32_t chunk;          // C
+  uint32_t poll;           // K
+  uint32_t epoch;          // 1-based epoch number of this grid
+  uint32_t workers;        // W = gridDim.x of this epoch
+  uint32_t num_sms;
+  uint32_t gx, gy;         // original grid (x, y); z folded into the flat index
+  uint32_t trigger_block;  // device self-trigger for this epoch (kNoTrigger = none)
+  uint32_t trigger_n;      // its yield width
+};
+
+__device__ __forceinline__ uint32_t smid_reg() {
+  uint32_t r; asm volatile("mov.u32 %0, %%smid;" : "=r"(r)); return r;
+}
+__device__ __forceinline__ uint64_t gtimer() {
+  uint64_t r; asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(r)); return r;
+}
+__device__ __forceinline__ uint32_t ld_acquire_gpu(const uint32_t* p) {
+  uint32_t v; asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory"); return v;
+}
+__device__ __forceinline__ uint32_t ld_acquire_sys(const uint32_t* p) {
+  uint32_t v; asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory"); return v;
+}
+__device__ __forceinline__ uint32_t atom_add_acqrel_gpu(uint32_t* p, uint32_t v) {
+  uint32_t old; asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], %2;" : "=r"(old) : "l"(p), "r"(v) : "memory"); return old;
+}
+__device__ __forceinline__ void red_add_release_gpu(uint32_t* p, uint32_t v) {
+  asm volatile("red.release.gpu.global.add.u32 [%0], %1;" :: "l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ void st_release_sys(uint32_t* p, uint32_t v) {
+  asm volatile("st.release.sys.global.u32 [%0], %1;" :: "l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ void st_relaxed_gpu(uint32_t* p, uint32_t v) {
+  asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" :: "l"(p), "r"(v) : "memory");
+}
+
+// Does the control word ask the worker on `sm` to leave? (Fig. 4(c))
+__device__ __forceinline__ bool should_yield(uint32_t c, const WorkerParams& p, uint32_t sm) {
+  const uint32_t gen = c >> 16, n = c & 0xffffu;
+  if (gen != (p.epoch & 0xffffu) || n == 0) return false;
+  return n >= p.num_sms || p.rank[sm] < n;
+}
+
+// The worker. Body contract:
+//   Body::kThreads               CTA size of the original kernel
+//   Body::kMinBlocks             resident CTAs per SM the register budget is sized for
+//   Body::Args                   POD argument struct
+//   Body::run(args, b0, b1, gx, gy)  all threads of the CTA execute original blocks [b0, b1)
+//                                (flat indices b = x + gx*(y + gy*z)), leaving no pending smem
+//                                hazards (the wrapper barrier follows).
+template <class Body, bool kCoverage>
+__global__ void __launch_bounds__(Body::kThreads, Body::kMinBlocks)
+flep_worker(const typename Body::Args args, const WorkerParams p) {
+  __shared__ uint32_t s_slot[2];     // chunk base broadcast, double-buffered: 1 barrier per chunk
+  __shared__ uint64_t s_t_entry;     // worker bookkeeping kept out of registers (tid 0 only)
+  __shared__ uint32_t s_sm, s_blocks, s_reason;
+  const uint32_t tid = threadIdx.x;
+  if (tid == 0) { s_sm = smid_reg(); s_t_entry = gtimer(); s_blocks = 0; s_reason = 0; }
+  uint32_t k = 0;                    // chunk index within the current poll period
+  uint32_t parity = 0;
+  while (true) {
+    if (tid == 0) {
+      uint32_t base;
+      bool stop = false;
+      if (k == 0) {                                      // amortised poll (Fig. 4(b))
+        const uint32_t c = ld_acquire_gpu(p.ctrl);
+        if (should_yield(c, p, smid_reg())) stop = true;
+      }
+      if (stop) {
+        base = 0xffffffffu; s_reason = kReasonYield;
+      } else {
+        base = atomicAdd(&p.cb->ctr, p.chunk);          // pull_task
+        if (base >= p.n_blocks) { base = 0xffffffffu; s_reason = kReasonExhausted; }
+        else {
+          s_blocks += min(p.chunk, p.n_blocks - base);
+          if (p.trigger_block - base < p.chunk) {        // self-trigger inside this chunk
+            const uint32_t e = p.epoch % kEvEpochs;
+            p.cb->ep_t_trigger[e] = gtimer();
+            p.cb->ep_trigger_block[e] = p.trigger_block;
+            atomicExch(p.ctrl, ((p.epoch & 0xffffu) << 16) | (p.trigger_n & 0xffffu));
+          }
+        }
+      }
+      s_slot[parity] = base;
+    }
+    __syncthreads();
+    const uint32_t b0 = s_slot[parity];
+    parity ^= 1u;
+    if (b0 == 0xffffffffu) break;
+    const uint32_t b1 = min(b0 + p.chunk, p.n_blocks);
+    Body::run(args, b0, b1, p.gx, p.gy);
+    if (kCoverage && tid == 0)
+      for (uint32_t b = b0; b < b1; ++b) atomicAdd(&p.cov[b], 1u);
+    if (++k == p.poll) k = 0;
+  }
+  // exit path (a7). Every thread finished its last chunk before the barrier that broadcast the
+  // stop slot, so the release below (cumulative over the CTA barrier) publishes all of them.
+  if (tid == 0) {
+    const uint32_t my_blocks = s_blocks;
+    if (my_blocks) red_add_release_gpu(&p.cb->done, my_blocks);
+    WorkerEvent& e = p.ev[(p.epoch % kEvEpochs) * p.workers + blockIdx.x];
+    const uint64_t t_exit = gtimer();
+    e.smid = s_sm; e.reason = s_reason; e.n_blocks = my_blocks; e.epoch = p.epoch;
+    e.t_entry = s_t_entry; e.t_exit = t_exit;
+    const uint32_t old = atom_add_acqrel_gpu(&p.cb->exited, 1u);
+    if (old + 1 == p.workers) {                          // last worker of this epoch
+      const uint32_t d = ld_acquire_gpu(&p.cb->done);
+      const uint32_t c = ld_acquire_gpu(&p.cb->ctr);
+      const uint32_t st = (d >= p.n_blocks) ? kStateDone : kStatePreempted;
+      const uint32_t ei = p.epoch % kEvEpochs;
+      p.cb->ep_t_end[ei] = t_exit; p.cb->ep_done[ei] = d; p.cb->ep_ctr[ei] = c;
+      p.cb->ep_state[ei] = st;
+      p.cb->exited = 0;                                  // ready for the next epoch
+      p.status->t_end = t_exit;
+      p.status->done = d;
+      p.status->ctr = c;
+      __threadfence_system();
+      st_release_sys(&p.status->word, (p.epoch << 8) | st);
+    }
+  }
+}
+
+// The original kernel (unwrapped twin, K7): one CTA per original block, same body.
+template <class Body>
+__global__ void __launch_bounds__(Body::kThreads, Body::kMinBlocks)
+flep_unwrapped(const typename Body::Args args, uint32_t gx, uint32_t gy, uint32_t block_offset) {
+  const uint32_t b = block_offset + blockIdx.x + gx * (blockIdx.y + gy * blockIdx.z);
+  Body::run(args, b, b + 1, gx, gy);
+}
+
+}  // namespace flep

@@ -1,0 +1,81 @@
+// kernels.cu — instantiates the wrapper and the unwrapped twins for every body and exposes a
+// small dispatch table to the host runtime (runtime.cu). sm_100a only.
+#include <cuda_runtime.h>
+#include <type_traits>
+
+#include "flep_device.cuh"
+#include "bodies.cuh"
+#include "gemm_tcgen05.cuh"
+#include "kernels.hpp"
+
+namespace flep {
+
+namespace {
+
+template <class Body>
+struct Ops {
+  static cudaError_t worker(const void* args, const WorkerParams& p, uint32_t W, cudaStream_t s,
+                            bool cov) {
+    const typename Body::Args& a = *reinterpret_cast<const typename Body::Args*>(args);
+    if (cov) flep_worker<Body, true><<<W, Body::kThreads, Body::kDynSmem, s>>>(a, p);
+    else flep_worker<Body, false><<<W, Body::kThreads, Body::kDynSmem, s>>>(a, p);
+    return cudaGetLastError();
+  }
+  static cudaError_t unwrapped(const void* args, dim3 grid, uint32_t offset, uint32_t count,
+                               cudaStream_t s) {
+    const typename Body::Args& a = *reinterpret_cast<const typename Body::Args*>(args);
+    if (count == 0) flep_unwrapped<Body><<<grid, Body::kThreads, Body::kDynSmem, s>>>(a, grid.x, grid.y, 0);
+    else flep_unwrapped<Body><<<count, Body::kThreads, Body::kDynSmem, s>>>(a, grid.x, grid.y, offset);
+    return cudaGetLastError();
+  }
+  static cudaError_t occupancy(int* k, bool cov) {
+    cudaError_t e;
+    if (Body::kDynSmem > 48 * 1024) {
+      e = cudaFuncSetAttribute(flep_worker<Body, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, Body::kDynSmem);
+      if (e) return e;
+      e = cudaFuncSetAttribute(flep_worker<Body, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, Body::kDynSmem);
+      if (e) return e;
+      e = cudaFuncSetAttribute(flep_unwrapped<Body>, cudaFuncAttributeMaxDynamicSharedMemorySize, Body::kDynSmem);
+      if (e) return e;
+    }
+    if (cov) return cudaOccupancyMaxActiveBlocksPerMultiprocessor(k, flep_worker<Body, true>, Body::kThreads, Body::kDynSmem);
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(k, flep_worker<Body, false>, Body::kThreads, Body::kDynSmem);
+  }
+};
+
+// Adapter: bodies written without kDynSmem get 0.
+template <class B>
+struct WithSmem : B {
+  static constexpr size_t kDynSmem = 0;
+};
+
+using SaxpyI32 = WithSmem<SaxpyBody<true>>;
+using SaxpyF32 = WithSmem<SaxpyBody<false>>;
+using Spmv = WithSmem<SpmvBody>;
+using StencilF32 = WithSmem<Stencil5Body<false>>;
+using StencilI32 = WithSmem<Stencil5Body<true>>;
+
+const BodyOps kOps[] = {
+    {0, 0, 0, nullptr, nullptr, nullptr, nullptr},
+    {FLEP_BODY_SAXPY_I32, SaxpyI32::kThreads, sizeof(flep_saxpy_i32_args), &Ops<SaxpyI32>::worker,
+     &Ops<SaxpyI32>::unwrapped, &Ops<SaxpyI32>::occupancy, nullptr},
+    {FLEP_BODY_SAXPY_F32, SaxpyF32::kThreads, sizeof(flep_saxpy_f32_args), &Ops<SaxpyF32>::worker,
+     &Ops<SaxpyF32>::unwrapped, &Ops<SaxpyF32>::occupancy, nullptr},
+    {FLEP_BODY_SPMV_CSR_F32, Spmv::kThreads, sizeof(flep_spmv_args), &Ops<Spmv>::worker,
+     &Ops<Spmv>::unwrapped, &Ops<Spmv>::occupancy, nullptr},
+    {FLEP_BODY_STENCIL5_F32, StencilF32::kThreads, sizeof(flep_stencil_args), &Ops<StencilF32>::worker,
+     &Ops<StencilF32>::unwrapped, &Ops<StencilF32>::occupancy, nullptr},
+    {FLEP_BODY_STENCIL5_I32, StencilI32::kThreads, sizeof(flep_stencil_args), &Ops<StencilI32>::worker,
+     &Ops<StencilI32>::unwrapped, &Ops<StencilI32>::occupancy, nullptr},
+    {FLEP_BODY_GEMM_BF16, GemmBody::kThreads, sizeof(flep_gemm_args), &gemm_worker_launch,
+     &gemm_unwrapped_launch, &gemm_occupancy, &gemm_validate},
+};
+
+}  // namespace
+
+const BodyOps* body_ops(int32_t body) {
+  if (body < 1 || body > FLEP_BODY_GEMM_BF16) return nullptr;
+  return &kOps[body];
+}
+
+}  // namespace flep

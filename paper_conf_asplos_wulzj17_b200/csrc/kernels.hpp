@@ -1,0 +1,27 @@
+// kernels.hpp — host-side dispatch table over the instantiated device kernels.
+#pragma once
+#include <cuda_runtime.h>
+#include <cstdint>
+
+#include "../../include/flep.h"
+#include "flep_device.cuh"
+
+namespace flep {
+
+struct BodyOps {
+  int32_t body;
+  int threads;
+  size_t args_size;
+  // launch W worker CTAs of flep_worker<Body> on stream s
+  cudaError_t (*worker)(const void* args, const WorkerParams& p, uint32_t W, cudaStream_t s, bool cov);
+  // launch the original kernel: full grid (count == 0) or the 1-D slice [offset, offset+count)
+  cudaError_t (*unwrapped)(const void* args, dim3 grid, uint32_t offset, uint32_t count, cudaStream_t s);
+  // resident worker CTAs per SM
+  cudaError_t (*occupancy)(int* ctas_per_sm, bool cov);
+  // optional argument / grid validation (nullptr = none); returns a static message or nullptr
+  const char* (*validate)(const void* args, dim3 grid);
+};
+
+const BodyOps* body_ops(int32_t body);
+
+}  // namespace flep

@@ -1,0 +1,872 @@
+// runtime.cu — the FLEP host runtime behind include/flep.h (§8(b)).
+//
+// Paper mapping:
+//   interception of kernel invocations, name + config + priority to the runtime ... P:112
+//   CPU state machine S1 -> S2 (await decision) -> S3 (running) -> S2 on preempt ... Fig. 5
+//   preempt = set the shared variable; the GPU workers see it at their next poll ... P:164
+//   resume = relaunch "to finish the remaining tasks" ........................... P:126
+//   online decisions on arrive / finish, HPF + SRPT with overhead ................ §5, Fig. 6
+//   duration prediction (linear model) and execution logging (T_e, T_w, T_r) ..... §4.2, §5.1
+//
+// B200 choices: the control word lives in device memory and is written by
+// cuStreamWriteValue32 on a highest-priority control stream (executed by the GPU front end, so it
+// needs no SM while the victim occupies all of them; probe: ~9 us host round trip vs ~1 ms for a
+// mapped-host flag polled by 1184 CTAs). Completion / drain is published by the last exiting
+// worker into a pinned host slot that the host spins on.
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <array>
+#include <atomic>
+#include <chrono>
+#include <condition_variable>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <string>
+#include <thread>
+#include <vector>
+
+#include "../../include/flep.h"
+#include "flep_device.cuh"
+#include "kernels.hpp"
+#include "policy.hpp"
+
+namespace {
+
+using namespace flep;
+
+thread_local std::string g_err;
+
+flep_status fail(flep_status s, const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof(buf), fmt, ap);
+  va_end(ap);
+  g_err = buf;
+  return s;
+}
+
+#define CUDA_TRY(expr)                                                                        \
+  do {                                                                                        \
+    cudaError_t _e = (expr);                                                                  \
+    if (_e != cudaSuccess)                                                                    \
+      return fail(FLEP_ERR_CUDA, "%s failed: %s (%s:%d)", #expr, cudaGetErrorString(_e),      \
+                  __FILE__, __LINE__);                                                        \
+  } while (0)
+
+int64_t now_ns() {
+  return std::chrono::duration_cast<std::chrono::nanoseconds>(
+             std::chrono::steady_clock::now().time_since_epoch())
+      .count();
+}
+
+// Driver stream memory operations, resolved through the runtime (no link-time libcuda).
+typedef CUresult (*PFN_wv32)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+typedef CUresult (*PFN_wait32)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+PFN_wv32 p_write32 = nullptr;
+PFN_wait32 p_wait32 = nullptr;
+
+flep_status resolve_driver() {
+  if (p_write32 && p_wait32) return FLEP_OK;
+  cudaDriverEntryPointQueryResult q;
+  CUDA_TRY(cudaGetDriverEntryPoint("cuStreamWriteValue32", (void**)&p_write32, cudaEnableDefault, &q));
+  if (q != cudaDriverEntryPointSuccess || !p_write32)
+    return fail(FLEP_ERR_UNSUPPORTED, "cuStreamWriteValue32 not available");
+  CUDA_TRY(cudaGetDriverEntryPoint("cuStreamWaitValue32", (void**)&p_wait32, cudaEnableDefault, &q));
+  if (q != cudaDriverEntryPointSuccess || !p_wait32)
+    return fail(FLEP_ERR_UNSUPPORTED, "cuStreamWaitValue32 not available");
+  return FLEP_OK;
+}
+
+constexpr uint32_t kMaxSlots = 1u << 14;       // pinned status slots (recycled)
+constexpr uint32_t kMaxWorkersPerSm = 32;
+
+struct Launch {
+  int64_t id = 0;
+  int32_t kernel = -1;
+  int32_t body = 0;
+  const BodyOps* ops = nullptr;
+  std::vector<uint8_t> args;
+  dim3 grid;
+  uint32_t n_blocks = 0;
+  int32_t prio = 0;
+  cudaStream_t user = nullptr;
+  cudaStream_t exec = nullptr;
+  int exec_level = 0;
+  uint32_t chunk = 1, poll = 1, workers = 0;
+  void* dmem = nullptr;              // ControlBlock + event ring
+  ControlBlock* cb = nullptr;
+  WorkerEvent* ev = nullptr;
+  uint32_t* cov = nullptr;
+  size_t cov_cap = 0;
+  int slot = -1;
+  HostStatus* hs = nullptr;          // host view
+  HostStatus* ds = nullptr;          // device alias
+  uint32_t epoch = 0;
+  int32_t state = FLEP_STATE_QUEUED;
+  uint32_t n_yield = 0;
+  uint32_t trig_block = kNoTrigger, trig_n = 0;
+  int64_t t_arrive = 0, t_first_start = -1, t_finish = -1;
+  int64_t t_e = 0, overhead = 0;
+  uint32_t last_done = 0, last_ctr = 0;
+  cudaEvent_t user_after_wait = nullptr;   // recorded on the user stream after its done-wait
+  bool released = false;
+  bool cancelled = false;
+};
+
+struct KernelReg {
+  std::string name;
+  int32_t body;
+  uint32_t chunk, poll;
+  double model[5];
+  int64_t overhead;
+};
+
+}  // namespace
+
+struct flep_rt_s {
+  int device = 0;
+  flep_options opt{};
+  uint32_t num_sms = 0, nsmid = 0;
+  int prio_lo = 0, prio_hi = 0;            // CUDA stream priority range (lo = least)
+  cudaStream_t ctl = nullptr;              // highest-priority control stream
+  uint16_t* d_rank = nullptr;
+  HostStatus* h_slots = nullptr;
+  HostStatus* d_slots = nullptr;
+  std::vector<int> free_slots;
+  size_t dmem_bytes = 0;
+  uint32_t max_workers = 0;
+  std::vector<void*> free_dmem;
+  std::vector<std::pair<uint32_t*, size_t>> free_cov;
+  std::map<int, std::vector<cudaStream_t>> free_streams;
+  std::vector<cudaStream_t> all_streams;
+  std::vector<KernelReg> kernels;
+  std::map<int64_t, std::unique_ptr<Launch>> launches;
+  int64_t next_id = 1;
+  uint32_t arm_block = kNoTrigger, arm_n = 0;
+  std::mutex mu;
+  std::condition_variable cv;
+  // managed mode
+  std::unique_ptr<Policy> policy;
+  size_t applied = 0;
+  std::vector<std::array<int64_t, 6>> evlog;    // (t, type, id, prio, t_e, overhead)
+  std::thread monitor;
+  std::atomic<bool> stop{false};
+  std::map<std::pair<int32_t, bool>, int> occ_cache;
+  std::vector<int64_t> retained;   // finished launches whose logs are kept for debug copies
+};
+
+namespace {
+
+flep_status occupancy(flep_rt rt, const BodyOps* ops, bool cov, int* k) {
+  auto key = std::make_pair(ops->body, cov);
+  auto it = rt->occ_cache.find(key);
+  if (it != rt->occ_cache.end()) { *k = it->second; return FLEP_OK; }
+  CUDA_TRY(ops->occupancy(k, cov));
+  if (*k <= 0) return fail(FLEP_ERR_UNSUPPORTED, "body %d cannot be resident", ops->body);
+  rt->occ_cache[key] = *k;
+  return FLEP_OK;
+}
+
+int stream_level(flep_rt rt, int32_t prio) {
+  // FLEP priority (larger = higher) -> CUDA priority (numerically smaller = higher)
+  int cuda_p = rt->prio_lo - (prio > 0 ? prio : 0);
+  if (cuda_p < rt->prio_hi + 1) cuda_p = rt->prio_hi + 1;   // keep the top level for ctl
+  if (rt->prio_hi == rt->prio_lo) cuda_p = rt->prio_lo;
+  return cuda_p;
+}
+
+flep_status get_stream(flep_rt rt, int level, cudaStream_t* s) {
+  auto& v = rt->free_streams[level];
+  if (!v.empty()) { *s = v.back(); v.pop_back(); return FLEP_OK; }
+  CUDA_TRY(cudaStreamCreateWithPriority(s, cudaStreamNonBlocking, level));
+  rt->all_streams.push_back(*s);
+  return FLEP_OK;
+}
+
+flep_status write_ctrl(flep_rt rt, Launch& L, uint32_t value) {
+  if (rt->opt.flag == FLEP_FLAG_HOST_MAPPED) {
+    __atomic_store_n(&L.hs->ctrl, value, __ATOMIC_RELEASE);
+    return FLEP_OK;
+  }
+  CUresult r = p_write32((CUstream)rt->ctl, (CUdeviceptr)&L.cb->ctrl, value, 0);
+  if (r != CUDA_SUCCESS) return fail(FLEP_ERR_CUDA, "cuStreamWriteValue32 failed (%d)", (int)r);
+  return FLEP_OK;
+}
+
+flep_status start_epoch(flep_rt rt, Launch& L) {
+  L.epoch++;
+  WorkerParams p{};
+  p.cb = L.cb;
+  p.ctrl = rt->opt.flag == FLEP_FLAG_HOST_MAPPED ? &L.ds->ctrl : &L.cb->ctrl;
+  p.cov = L.cov;
+  p.ev = L.ev;
+  p.status = L.ds;
+  p.rank = rt->d_rank;
+  p.n_blocks = L.n_blocks;
+  p.chunk = L.chunk;
+  p.poll = L.poll;
+  p.epoch = L.epoch;
+  p.workers = L.workers;
+  p.num_sms = rt->num_sms;
+  p.gx = L.grid.x;
+  p.gy = L.grid.y;
+  p.trigger_block = L.trig_block;
+  p.trigger_n = L.trig_n;
+  L.trig_block = kNoTrigger;
+  L.trig_n = 0;
+  cudaError_t e = L.ops->worker(L.args.data(), p, L.workers, L.exec, L.cov != nullptr);
+  if (e != cudaSuccess) return fail(FLEP_ERR_CUDA, "worker launch failed: %s", cudaGetErrorString(e));
+  L.state = FLEP_STATE_RUNNING;
+  L.n_yield = 0;
+  if (L.t_first_start < 0) L.t_first_start = now_ns();
+  return FLEP_OK;
+}
+
+// Pull the pinned status slot; returns true if the launch's state changed to DONE.
+bool refresh(Launch& L) {
+  if (L.state != FLEP_STATE_RUNNING && L.state != FLEP_STATE_YIELDING && L.state != FLEP_STATE_PARTIAL)
+    return false;
+  const uint32_t w = __atomic_load_n(&L.hs->word, __ATOMIC_ACQUIRE);
+  if ((w >> 8) != L.epoch) return false;
+  L.last_done = L.hs->done;
+  L.last_ctr = L.hs->ctr;
+  if ((w & 0xffu) == kStateDone) {
+    L.state = FLEP_STATE_DONE;
+    L.t_finish = now_ns();
+    return true;
+  }
+  L.state = FLEP_STATE_PREEMPTED;
+  return false;
+}
+
+void release_resources(flep_rt rt, Launch& L) {
+  if (L.released) return;
+  // the launch's last grid has completed (caller synchronised the exec stream)
+  if (L.user_after_wait && cudaEventQuery(L.user_after_wait) != cudaSuccess) return;  // retry later
+  if (L.user_after_wait) { cudaEventDestroy(L.user_after_wait); L.user_after_wait = nullptr; }
+  if (L.dmem) rt->free_dmem.push_back(L.dmem);
+  if (L.cov) rt->free_cov.push_back({L.cov, L.cov_cap});
+  if (L.slot >= 0) rt->free_slots.push_back(L.slot);
+  if (L.exec) rt->free_streams[L.exec_level].push_back(L.exec);
+  L.dmem = nullptr; L.cov = nullptr; L.slot = -1; L.exec = nullptr;
+  L.released = true;
+}
+
+void apply_decisions(flep_rt rt) {
+  const auto& d = rt->policy->decisions();
+  for (; rt->applied < d.size(); ++rt->applied) {
+    const Decision& x = d[rt->applied];
+    auto it = rt->launches.find(x.id);
+    if (it == rt->launches.end()) continue;
+    Launch& L = *it->second;
+    if (x.action == kPreempt) {
+      if (L.state == FLEP_STATE_RUNNING || L.state == FLEP_STATE_PARTIAL) {
+        write_ctrl(rt, L, ((L.epoch & 0xffffu) << 16) | (uint32_t)std::min<int64_t>(x.n_sms, 0xffff));
+        L.state = FLEP_STATE_YIELDING;
+        L.n_yield = (uint32_t)x.n_sms;
+      }
+    } else {
+      if (L.state == FLEP_STATE_DONE) continue;   // finished while draining; FINISH pending
+      start_epoch(rt, L);
+    }
+  }
+}
+
+void monitor_loop(flep_rt rt) {
+  cudaSetDevice(rt->device);
+  while (!rt->stop.load(std::memory_order_relaxed)) {
+    bool active = false;
+    {
+      std::unique_lock<std::mutex> lk(rt->mu);
+      for (auto& kv : rt->launches) {
+        Launch& L = *kv.second;
+        if (L.state == FLEP_STATE_RUNNING || L.state == FLEP_STATE_YIELDING || L.state == FLEP_STATE_PARTIAL) {
+          active = true;
+          if (refresh(L)) {
+            const int64_t t = L.t_finish;
+            rt->evlog.push_back({t, 1, L.id, L.prio, L.t_e, L.overhead});
+            rt->policy->finish(t, L.id);
+            apply_decisions(rt);
+            rt->cv.notify_all();
+          } else if (L.state == FLEP_STATE_PREEMPTED) {
+            rt->cv.notify_all();
+          }
+        }
+      }
+      if (!active) {
+        rt->cv.wait_for(lk, std::chrono::milliseconds(1));
+        continue;
+      }
+    }
+    std::this_thread::yield();
+  }
+}
+
+Launch* find(flep_rt rt, flep_launch_t h) {
+  auto it = rt->launches.find(h);
+  return it == rt->launches.end() ? nullptr : it->second.get();
+}
+
+flep_status validate_grid(flep_dim3 g, uint64_t* n) {
+  if (g.x == 0 || g.y == 0 || g.z == 0) return fail(FLEP_ERR_INVALID, "empty grid");
+  const uint64_t N = (uint64_t)g.x * g.y * g.z;
+  if (N >= (1ull << 31)) return fail(FLEP_ERR_INVALID, "grid too large (%llu blocks)", (unsigned long long)N);
+  *n = N;
+  return FLEP_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char* flep_last_error(void) { return g_err.c_str(); }
+const char* flep_version(void) { return "flep-b200 0.1 (sm_100a)"; }
+int64_t flep_now_ns(void) { return now_ns(); }
+
+flep_status flep_init(int device, const flep_options* opts, flep_rt* out) {
+  if (!out) return fail(FLEP_ERR_INVALID, "out is NULL");
+  *out = nullptr;
+  int ndev = 0;
+  cudaError_t e = cudaGetDeviceCount(&ndev);
+  if (e != cudaSuccess || ndev == 0) return fail(FLEP_ERR_CUDA, "no CUDA device: %s", cudaGetErrorString(e));
+  if (device < 0 || device >= ndev) return fail(FLEP_ERR_INVALID, "bad device %d", device);
+  CUDA_TRY(cudaSetDevice(device));
+  flep_status s = resolve_driver();
+  if (s) return s;
+  std::unique_ptr<flep_rt_s> rt(new flep_rt_s());
+  rt->device = device;
+  if (opts) rt->opt = *opts;
+  if (rt->opt.default_chunk == 0) rt->opt.default_chunk = 8;
+  if (rt->opt.default_poll == 0) rt->opt.default_poll = 1;
+  if (rt->opt.policy < FLEP_POLICY_MANUAL || rt->opt.policy > FLEP_POLICY_SLICE)
+    return fail(FLEP_ERR_INVALID, "bad policy %d", rt->opt.policy);
+  if (rt->opt.policy == FLEP_POLICY_SLICE) return fail(FLEP_ERR_UNSUPPORTED, "SLICE runtime mode not built yet");
+  cudaDeviceProp prop;
+  CUDA_TRY(cudaGetDeviceProperties(&prop, device));
+  if (prop.major != 10) return fail(FLEP_ERR_UNSUPPORTED, "needs sm_100 (got %d.%d)", prop.major, prop.minor);
+  rt->num_sms = prop.multiProcessorCount;
+  rt->nsmid = prop.multiProcessorCount;   // probe: %nsmid == SM count, %smid dense on B200
+  CUDA_TRY(cudaDeviceGetStreamPriorityRange(&rt->prio_lo, &rt->prio_hi));
+  CUDA_TRY(cudaStreamCreateWithPriority(&rt->ctl, cudaStreamNonBlocking, rt->prio_hi));
+  std::vector<uint16_t> rank(256);
+  for (uint32_t i = 0; i < rank.size(); ++i) rank[i] = (uint16_t)i;
+  CUDA_TRY(cudaMalloc(&rt->d_rank, rank.size() * sizeof(uint16_t)));
+  CUDA_TRY(cudaMemcpy(rt->d_rank, rank.data(), rank.size() * sizeof(uint16_t), cudaMemcpyHostToDevice));
+  CUDA_TRY(cudaHostAlloc(&rt->h_slots, kMaxSlots * sizeof(HostStatus), cudaHostAllocMapped));
+  memset(rt->h_slots, 0, kMaxSlots * sizeof(HostStatus));
+  CUDA_TRY(cudaHostGetDevicePointer(&rt->d_slots, rt->h_slots, 0));
+  for (int i = kMaxSlots - 1; i >= 0; --i) rt->free_slots.push_back(i);
+  rt->max_workers = rt->num_sms * kMaxWorkersPerSm;
+  rt->dmem_bytes = sizeof(ControlBlock) + (size_t)kEvEpochs * rt->max_workers * sizeof(WorkerEvent);
+  if (rt->opt.policy != FLEP_POLICY_MANUAL) {
+    rt->policy.reset(new Policy(rt->opt.policy, rt->num_sms));
+    flep_rt raw = rt.get();
+    rt->monitor = std::thread([raw] { monitor_loop(raw); });
+  }
+  *out = rt.release();
+  return FLEP_OK;
+}
+
+flep_status flep_device_info(flep_rt rt, uint32_t* num_sms, uint32_t* nsmid) {
+  if (!rt) return fail(FLEP_ERR_INVALID, "rt is NULL");
+  if (num_sms) *num_sms = rt->num_sms;
+  if (nsmid) *nsmid = rt->nsmid;
+  return FLEP_OK;
+}
+
+flep_status flep_register_kernel(flep_rt rt, const flep_kernel_desc* d, flep_kernel* out) {
+  if (!rt || !d || !out) return fail(FLEP_ERR_INVALID, "NULL argument");
+  if (!body_ops(d->body)) return fail(FLEP_ERR_INVALID, "unknown body %d", d->body);
+  std::lock_guard<std::mutex> lk(rt->mu);
+  KernelReg k;
+  k.name = d->name ? d->name : "";
+  k.body = d->body;
+  k.chunk = d->chunk ? d->chunk : rt->opt.default_chunk;
+  k.poll = d->poll ? d->poll : rt->opt.default_poll;
+  memcpy(k.model, d->model, sizeof(k.model));
+  k.overhead = d->preempt_overhead_ns;
+  rt->kernels.push_back(k);
+  *out = (flep_kernel)rt->kernels.size() - 1;
+  return FLEP_OK;
+}
+
+flep_status flep_workers_for(flep_rt rt, int32_t body, uint32_t* ctas_per_sm, uint32_t* workers) {
+  if (!rt) return fail(FLEP_ERR_INVALID, "rt is NULL");
+  const BodyOps* ops = body_ops(body);
+  if (!ops) return fail(FLEP_ERR_INVALID, "unknown body %d", body);
+  int k = 0;
+  std::lock_guard<std::mutex> lk(rt->mu);
+  flep_status s = occupancy(rt, ops, rt->opt.debug_coverage != 0, &k);
+  if (s) return s;
+  if (ctas_per_sm) *ctas_per_sm = (uint32_t)k;
+  if (workers) *workers = (uint32_t)k * rt->num_sms;
+  return FLEP_OK;
+}
+
+flep_status flep_launch(flep_rt rt, flep_kernel kid, flep_dim3 grid, const void* args,
+                        size_t args_size, int32_t priority, flep_stream_t stream,
+                        flep_launch_t* out) {
+  if (!rt || !args || !out) return fail(FLEP_ERR_INVALID, "NULL argument");
+  std::unique_lock<std::mutex> lk(rt->mu);
+  if (kid < 0 || (size_t)kid >= rt->kernels.size()) return fail(FLEP_ERR_INVALID, "unknown kernel %d", kid);
+  const KernelReg& kr = rt->kernels[kid];
+  const BodyOps* ops = body_ops(kr.body);
+  if (args_size != ops->args_size) return fail(FLEP_ERR_INVALID, "args_size %zu != %zu", args_size, ops->args_size);
+  uint64_t N = 0;
+  flep_status s = validate_grid(grid, &N);
+  if (s) return s;
+  dim3 g(grid.x, grid.y, grid.z);
+  if (ops->validate) {
+    const char* m = ops->validate(args, g);
+    if (m) return fail(FLEP_ERR_INVALID, "%s", m);
+  }
+  const bool cov = rt->opt.debug_coverage != 0;
+  int k = 0;
+  s = occupancy(rt, ops, cov, &k);
+  if (s) return s;
+  if (rt->free_slots.empty()) return fail(FLEP_ERR_NOMEM, "out of status slots");
+
+  std::unique_ptr<Launch> Lp(new Launch());
+  Launch& L = *Lp;
+  L.id = rt->next_id++;
+  L.kernel = kid;
+  L.body = kr.body;
+  L.ops = ops;
+  L.args.assign((const uint8_t*)args, (const uint8_t*)args + args_size);
+  L.grid = g;
+  L.n_blocks = (uint32_t)N;
+  L.prio = priority;
+  L.user = (cudaStream_t)stream;
+  L.chunk = kr.chunk;
+  L.poll = kr.poll;
+  const uint64_t wmax = (uint64_t)k * rt->num_sms;
+  const uint64_t need = (N + L.chunk - 1) / L.chunk;
+  L.workers = (uint32_t)std::min<uint64_t>(std::min<uint64_t>(wmax, need), rt->max_workers);
+  L.t_arrive = now_ns();
+  L.t_e = flep_model_predict_ns(kr.model, (double)N, (double)ops->threads, (double)N, 0.0);
+  L.overhead = kr.overhead;
+  L.trig_block = rt->arm_block;
+  L.trig_n = rt->arm_n;
+  rt->arm_block = kNoTrigger;
+  rt->arm_n = 0;
+  // resources
+  L.exec_level = stream_level(rt, priority);
+  s = get_stream(rt, L.exec_level, &L.exec);
+  if (s) return s;
+  if (!rt->free_dmem.empty()) { L.dmem = rt->free_dmem.back(); rt->free_dmem.pop_back(); }
+  else CUDA_TRY(cudaMalloc(&L.dmem, rt->dmem_bytes));
+  L.cb = (ControlBlock*)L.dmem;
+  L.ev = (WorkerEvent*)((char*)L.dmem + sizeof(ControlBlock));
+  if (cov) {
+    for (size_t i = 0; i < rt->free_cov.size(); ++i) {
+      if (rt->free_cov[i].second >= N) {
+        L.cov = rt->free_cov[i].first; L.cov_cap = rt->free_cov[i].second;
+        rt->free_cov.erase(rt->free_cov.begin() + i);
+        break;
+      }
+    }
+    if (!L.cov) { L.cov_cap = std::max<size_t>(N, 4096); CUDA_TRY(cudaMalloc(&L.cov, L.cov_cap * 4)); }
+    CUDA_TRY(cudaMemsetAsync(L.cov, 0, N * 4, L.exec));
+  }
+  L.slot = rt->free_slots.back();
+  rt->free_slots.pop_back();
+  L.hs = rt->h_slots + L.slot;
+  L.ds = rt->d_slots + L.slot;
+  memset(L.hs, 0, sizeof(HostStatus));
+  // order: caller's prior work -> control-block reset -> workers; caller's later work waits for
+  // the done counter to reach N (true completion across preempt/resume cycles).
+  cudaEvent_t ev_u;
+  CUDA_TRY(cudaEventCreateWithFlags(&ev_u, cudaEventDisableTiming));
+  CUDA_TRY(cudaEventRecord(ev_u, L.user));
+  CUDA_TRY(cudaStreamWaitEvent(L.exec, ev_u, 0));
+  CUDA_TRY(cudaMemsetAsync(L.dmem, 0, rt->dmem_bytes, L.exec));
+  if (rt->opt.order_user_stream) {
+    CUDA_TRY(cudaEventRecord(ev_u, L.exec));
+    CUDA_TRY(cudaStreamWaitEvent(L.user, ev_u, 0));
+    CUresult r = p_wait32((CUstream)L.user, (CUdeviceptr)&L.cb->done, L.n_blocks, CU_STREAM_WAIT_VALUE_GEQ);
+    if (r != CUDA_SUCCESS) return fail(FLEP_ERR_CUDA, "cuStreamWaitValue32 failed (%d)", (int)r);
+    CUDA_TRY(cudaEventCreateWithFlags(&L.user_after_wait, cudaEventDisableTiming));
+    CUDA_TRY(cudaEventRecord(L.user_after_wait, L.user));
+  }
+  cudaEventDestroy(ev_u);
+  rt->launches[L.id] = std::move(Lp);
+  *out = L.id;
+  if (rt->opt.policy == FLEP_POLICY_MANUAL) return start_epoch(rt, L);
+  // managed: interception (S2) -> policy decides (Fig. 6 lines 0-15)
+  rt->evlog.push_back({L.t_arrive, 0, L.id, L.prio, L.t_e, L.overhead});
+  rt->policy->arrive(L.t_arrive, L.id, L.prio, L.t_e, L.overhead);
+  apply_decisions(rt);
+  rt->cv.notify_all();
+  return FLEP_OK;
+}
+
+flep_status flep_preempt(flep_rt rt, flep_launch_t h, uint32_t n_sms) {
+  if (!rt) return fail(FLEP_ERR_INVALID, "rt is NULL");
+  if (n_sms == 0) return fail(FLEP_ERR_INVALID, "n_sms == 0");
+  std::lock_guard<std::mutex> lk(rt->mu);
+  if (rt->opt.policy != FLEP_POLICY_MANUAL) return fail(FLEP_ERR_STATE, "preempt is policy-driven in managed mode");
+  Launch* L = find(rt, h);
+  if (!L) return fail(FLEP_ERR_INVALID, "unknown launch %lld", (long long)h);
+  refresh(*L);
+  if (L->state != FLEP_STATE_RUNNING && L->state != FLEP_STATE_PARTIAL)
+    return fail(FLEP_ERR_STATE, "launch %lld is not running (state %d)", (long long)h, L->state);
+  const uint32_t n = std::min<uint32_t>(n_sms, rt->num_sms);
+  if (L->state == FLEP_STATE_PARTIAL && n <= L->n_yield)
+    return fail(FLEP_ERR_INVALID, "a request can only widen within an epoch (%u <= %u)", n, L->n_yield);
+  flep_status s = write_ctrl(rt, *L, ((L->epoch & 0xffffu) << 16) | n);
+  if (s) return s;
+  L->n_yield = n;
+  L->state = n >= rt->num_sms ? FLEP_STATE_YIELDING : FLEP_STATE_PARTIAL;
+  return FLEP_OK;
+}
+
+flep_status flep_resume(flep_rt rt, flep_launch_t h) {
+  if (!rt) return fail(FLEP_ERR_INVALID, "rt is NULL");
+  std::lock_guard<std::mutex> lk(rt->mu);
+  if (rt->opt.policy != FLEP_POLICY_MANUAL) return fail(FLEP_ERR_STATE, "resume is policy-driven in managed mode");
+  Launch* L = find(rt, h);
+  if (!L) return fail(FLEP_ERR_INVALID, "unknown launch %lld", (long long)h);
+  refresh(*L);
+  if (L->state == FLEP_STATE_PREEMPTED) return start_epoch(rt, *L);
+  if (L->state == FLEP_STATE_PARTIAL) {
+    flep_status s = write_ctrl(rt, *L, (L->epoch & 0xffffu) << 16);
+    if (s) return s;
+    L->state = FLEP_STATE_RUNNING;
+    L->n_yield = 0;
+    return FLEP_OK;
+  }
+  return fail(FLEP_ERR_STATE, "launch %lld is not preempted (state %d)", (long long)h, L->state);
+}
+
+flep_status flep_wait_epoch(flep_rt rt, flep_launch_t h, int64_t timeout_ns) {
+  if (!rt) return fail(FLEP_ERR_INVALID, "rt is NULL");
+  const int64_t t0 = now_ns();
+  while (true) {
+    {
+      std::lock_guard<std::mutex> lk(rt->mu);
+      Launch* L = find(rt, h);
+      if (!L) return fail(FLEP_ERR_INVALID, "unknown launch %lld", (long long)h);
+      refresh(*L);
+      if (L->state == FLEP_STATE_PREEMPTED || L->state == FLEP_STATE_DONE || L->state == FLEP_STATE_QUEUED)
+        return FLEP_OK;
+    }
+    if (timeout_ns >= 0 && now_ns() - t0 > timeout_ns) return fail(FLEP_ERR_TIMEOUT, "epoch did not drain");
+    cudaError_t e = cudaPeekAtLastError();
+    if (e != cudaSuccess) return fail(FLEP_ERR_CUDA, "sticky CUDA error: %s", cudaGetErrorString(e));
+  }
+}
+
+flep_status flep_sync(flep_rt rt, flep_launch_t h, int64_t timeout_ns) {
+  if (!rt) return fail(FLEP_ERR_INVALID, "rt is NULL");
+  const int64_t t0 = now_ns();
+  cudaStream_t exec = nullptr;
+  while (true) {
+    {
+      std::lock_guard<std::mutex> lk(rt->mu);
+      Launch* L = find(rt, h);
+      if (!L) return fail(FLEP_ERR_INVALID, "unknown launch %lld", (long long)h);
+      if (rt->opt.policy == FLEP_POLICY_MANUAL) refresh(*L);
+      if (L->state == FLEP_STATE_DONE) { exec = L->exec; break; }
+      if (rt->opt.policy == FLEP_POLICY_MANUAL && L->state == FLEP_STATE_PREEMPTED)
+        return fail(FLEP_ERR_STATE, "launch %lld is preempted; resume it first", (long long)h);
+    }
+    if (timeout_ns >= 0 && now_ns() - t0 > timeout_ns) return fail(FLEP_ERR_TIMEOUT, "launch not done");
+    std::this_thread::yield();
+  }
+  if (exec) CUDA_TRY(cudaStreamSynchronize(exec));
+  std::lock_guard<std::mutex> lk(rt->mu);
+  Launch* L = find(rt, h);
+  // keep the newest finished launches' device logs (coverage, events) for debug copies
+  constexpr size_t kRetain = 64;
+  if (L && !L->released && std::find(rt->retained.begin(), rt->retained.end(), h) == rt->retained.end())
+    rt->retained.push_back(h);
+  while (rt->retained.size() > kRetain) {
+    Launch* old = find(rt, rt->retained.front());
+    rt->retained.erase(rt->retained.begin());
+    if (old) release_resources(rt, *old);
+  }
+  for (auto& kv : rt->launches)   // retry deferred releases
+    if (kv.second->state == FLEP_STATE_DONE && !kv.second->released &&
+        std::find(rt->retained.begin(), rt->retained.end(), kv.first) == rt->retained.end() &&
+        kv.second->exec && cudaStreamQuery(kv.second->exec) == cudaSuccess)
+      release_resources(rt, *kv.second);
+  return FLEP_OK;
+}
+
+flep_status flep_query(flep_rt rt, flep_launch_t h, flep_launch_info* out) {
+  if (!rt || !out) return fail(FLEP_ERR_INVALID, "NULL argument");
+  std::lock_guard<std::mutex> lk(rt->mu);
+  Launch* L = find(rt, h);
+  if (!L) return fail(FLEP_ERR_INVALID, "unknown launch %lld", (long long)h);
+  if (rt->opt.policy == FLEP_POLICY_MANUAL) refresh(*L);
+  memset(out, 0, sizeof(*out));
+  out->state = L->state;
+  out->epoch = L->epoch;
+  out->blocks_total = L->n_blocks;
+  out->blocks_done = L->last_done;
+  out->counter = L->last_ctr;
+  out->t_arrive = L->t_arrive;
+  out->t_first_start = L->t_first_start;
+  out->t_finish = L->t_finish;
+  out->workers = L->workers;
+  out->n_yield = L->n_yield;
+  out->t_e = L->t_e;
+  if (rt->policy) {
+    const Policy::Entry* e = rt->policy->entry(L->id);
+    if (e) { out->t_w = e->t_w; out->t_r = e->t_r; }
+  }
+  return FLEP_OK;
+}
+
+flep_status flep_cancel(flep_rt rt, flep_launch_t h) {
+  if (!rt) return fail(FLEP_ERR_INVALID, "rt is NULL");
+  {
+    std::lock_guard<std::mutex> lk(rt->mu);
+    Launch* L = find(rt, h);
+    if (!L) return fail(FLEP_ERR_INVALID, "unknown launch %lld", (long long)h);
+    refresh(*L);
+    if (L->state == FLEP_STATE_DONE) return FLEP_OK;
+    if (L->state == FLEP_STATE_RUNNING || L->state == FLEP_STATE_PARTIAL || L->state == FLEP_STATE_YIELDING) {
+      write_ctrl(rt, *L, ((L->epoch & 0xffffu) << 16) | 0xffffu);
+      L->state = FLEP_STATE_YIELDING;
+    }
+    L->cancelled = true;
+  }
+  for (;;) {
+    std::lock_guard<std::mutex> lk(rt->mu);
+    Launch* L = find(rt, h);
+    refresh(*L);
+    if (L->state != FLEP_STATE_YIELDING) break;
+  }
+  std::lock_guard<std::mutex> lk(rt->mu);
+  Launch* L = find(rt, h);
+  if (L->exec) CUDA_TRY(cudaStreamSynchronize(L->exec));
+  // unblock any stream waiting for true completion
+  CUresult r = p_write32((CUstream)rt->ctl, (CUdeviceptr)&L->cb->done, L->n_blocks, 0);
+  if (r != CUDA_SUCCESS) return fail(FLEP_ERR_CUDA, "cuStreamWriteValue32 failed (%d)", (int)r);
+  CUDA_TRY(cudaStreamSynchronize(rt->ctl));
+  L->state = FLEP_STATE_DONE;
+  L->t_finish = now_ns();
+  return FLEP_OK;
+}
+
+flep_status flep_shutdown(flep_rt rt) {
+  if (!rt) return FLEP_OK;
+  rt->stop = true;
+  if (rt->monitor.joinable()) rt->monitor.join();
+  std::vector<int64_t> ids;
+  for (auto& kv : rt->launches) if (kv.second->state != FLEP_STATE_DONE) ids.push_back(kv.first);
+  for (int64_t id : ids) flep_cancel(rt, id);
+  cudaDeviceSynchronize();
+  for (auto& kv : rt->launches) {
+    Launch& L = *kv.second;
+    if (L.user_after_wait) cudaEventDestroy(L.user_after_wait);
+    if (!L.released) {
+      if (L.dmem) cudaFree(L.dmem);
+      if (L.cov) cudaFree(L.cov);
+    }
+  }
+  for (void* p : rt->free_dmem) cudaFree(p);
+  for (auto& c : rt->free_cov) cudaFree(c.first);
+  for (cudaStream_t s : rt->all_streams) cudaStreamDestroy(s);
+  if (rt->ctl) cudaStreamDestroy(rt->ctl);
+  if (rt->d_rank) cudaFree(rt->d_rank);
+  if (rt->h_slots) cudaFreeHost(rt->h_slots);
+  delete rt;
+  return FLEP_OK;
+}
+
+flep_status flep_launch_unwrapped(flep_rt rt, int32_t body, flep_dim3 grid, const void* args,
+                                  size_t args_size, flep_stream_t stream) {
+  if (!rt || !args) return fail(FLEP_ERR_INVALID, "NULL argument");
+  const BodyOps* ops = body_ops(body);
+  if (!ops) return fail(FLEP_ERR_INVALID, "unknown body %d", body);
+  if (args_size != ops->args_size) return fail(FLEP_ERR_INVALID, "args_size mismatch");
+  uint64_t N = 0;
+  flep_status s = validate_grid(grid, &N);
+  if (s) return s;
+  dim3 g(grid.x, grid.y, grid.z);
+  if (ops->validate) { const char* m = ops->validate(args, g); if (m) return fail(FLEP_ERR_INVALID, "%s", m); }
+  { int k; std::lock_guard<std::mutex> lk(rt->mu); s = occupancy(rt, ops, false, &k); if (s) return s; }
+  CUDA_TRY(ops->unwrapped(args, g, 0, 0, (cudaStream_t)stream));
+  return FLEP_OK;
+}
+
+flep_status flep_launch_sliced(flep_rt rt, int32_t body, flep_dim3 grid, const void* args,
+                               size_t args_size, uint32_t slice_blocks, flep_stream_t stream) {
+  if (!rt || !args) return fail(FLEP_ERR_INVALID, "NULL argument");
+  if (slice_blocks == 0) return fail(FLEP_ERR_INVALID, "slice_blocks == 0");
+  const BodyOps* ops = body_ops(body);
+  if (!ops) return fail(FLEP_ERR_INVALID, "unknown body %d", body);
+  if (args_size != ops->args_size) return fail(FLEP_ERR_INVALID, "args_size mismatch");
+  uint64_t N = 0;
+  flep_status s = validate_grid(grid, &N);
+  if (s) return s;
+  dim3 g(grid.x, grid.y, grid.z);
+  if (ops->validate) { const char* m = ops->validate(args, g); if (m) return fail(FLEP_ERR_INVALID, "%s", m); }
+  { int k; std::lock_guard<std::mutex> lk(rt->mu); s = occupancy(rt, ops, false, &k); if (s) return s; }
+  for (uint64_t off = 0; off < N; off += slice_blocks) {
+    const uint32_t cnt = (uint32_t)std::min<uint64_t>(slice_blocks, N - off);
+    CUDA_TRY(ops->unwrapped(args, g, (uint32_t)off, cnt, (cudaStream_t)stream));
+  }
+  return FLEP_OK;
+}
+
+flep_status flep_debug_trigger_at(flep_rt rt, flep_launch_t h, uint64_t block_index, uint32_t n_sms) {
+  if (!rt) return fail(FLEP_ERR_INVALID, "rt is NULL");
+  if (n_sms == 0) return fail(FLEP_ERR_INVALID, "n_sms == 0");
+  std::lock_guard<std::mutex> lk(rt->mu);
+  Launch* L = find(rt, h);
+  if (!L) return fail(FLEP_ERR_INVALID, "unknown launch %lld", (long long)h);
+  refresh(*L);
+  if (L->state != FLEP_STATE_PREEMPTED && L->state != FLEP_STATE_QUEUED)
+    return fail(FLEP_ERR_STATE, "trigger can only be set for the next epoch of a launch that is not running");
+  L->trig_block = block_index >= 0xffffffffull ? kNoTrigger : (uint32_t)block_index;
+  L->trig_n = std::min<uint32_t>(n_sms, 0xffff);
+  return FLEP_OK;
+}
+
+flep_status flep_debug_arm_next_trigger(flep_rt rt, uint64_t block_index, uint32_t n_sms) {
+  if (!rt) return fail(FLEP_ERR_INVALID, "rt is NULL");
+  if (n_sms == 0) return fail(FLEP_ERR_INVALID, "n_sms == 0");
+  std::lock_guard<std::mutex> lk(rt->mu);
+  rt->arm_block = block_index >= 0xffffffffull ? kNoTrigger : (uint32_t)block_index;
+  rt->arm_n = std::min<uint32_t>(n_sms, 0xffff);
+  return FLEP_OK;
+}
+
+flep_status flep_debug_copy_coverage(flep_rt rt, flep_launch_t h, uint32_t* host_out, size_t n) {
+  if (!rt || !host_out) return fail(FLEP_ERR_INVALID, "NULL argument");
+  std::lock_guard<std::mutex> lk(rt->mu);
+  Launch* L = find(rt, h);
+  if (!L) return fail(FLEP_ERR_INVALID, "unknown launch %lld", (long long)h);
+  if (!L->cov) return fail(FLEP_ERR_STATE, "coverage log not enabled or already released");
+  if (n > L->n_blocks) return fail(FLEP_ERR_INVALID, "n > N");
+  CUDA_TRY(cudaMemcpyAsync(host_out, L->cov, n * 4, cudaMemcpyDeviceToHost, L->exec));
+  CUDA_TRY(cudaStreamSynchronize(L->exec));
+  return FLEP_OK;
+}
+
+flep_status flep_debug_copy_events(flep_rt rt, flep_launch_t h, uint32_t epoch,
+                                   flep_worker_event* host_out, size_t max_records, size_t* n_out) {
+  if (!rt || !host_out) return fail(FLEP_ERR_INVALID, "NULL argument");
+  std::lock_guard<std::mutex> lk(rt->mu);
+  Launch* L = find(rt, h);
+  if (!L) return fail(FLEP_ERR_INVALID, "unknown launch %lld", (long long)h);
+  if (!L->dmem) return fail(FLEP_ERR_STATE, "launch resources already released");
+  if (epoch == 0 || epoch > L->epoch || L->epoch - epoch >= kEvEpochs)
+    return fail(FLEP_ERR_INVALID, "epoch %u not in the log", epoch);
+  const size_t n = std::min<size_t>(max_records, L->workers);
+  CUDA_TRY(cudaMemcpyAsync(host_out, L->ev + (size_t)(epoch % kEvEpochs) * L->workers,
+                           n * sizeof(WorkerEvent), cudaMemcpyDeviceToHost, L->exec));
+  CUDA_TRY(cudaStreamSynchronize(L->exec));
+  if (n_out) *n_out = n;
+  return FLEP_OK;
+}
+
+flep_status flep_debug_epoch_info(flep_rt rt, flep_launch_t h, uint32_t epoch, flep_epoch_info* out) {
+  if (!rt || !out) return fail(FLEP_ERR_INVALID, "NULL argument");
+  std::lock_guard<std::mutex> lk(rt->mu);
+  Launch* L = find(rt, h);
+  if (!L) return fail(FLEP_ERR_INVALID, "unknown launch %lld", (long long)h);
+  if (!L->dmem) return fail(FLEP_ERR_STATE, "launch resources already released");
+  if (epoch == 0 || epoch > L->epoch || L->epoch - epoch >= kEvEpochs)
+    return fail(FLEP_ERR_INVALID, "epoch %u not in the log", epoch);
+  ControlBlock cb;
+  CUDA_TRY(cudaMemcpyAsync(&cb, L->cb, sizeof(cb), cudaMemcpyDeviceToHost, L->exec));
+  CUDA_TRY(cudaStreamSynchronize(L->exec));
+  const uint32_t e = epoch % kEvEpochs;
+  out->t_trigger = cb.ep_t_trigger[e];
+  out->t_end = cb.ep_t_end[e];
+  out->trigger_block = cb.ep_trigger_block[e];
+  out->done = cb.ep_done[e];
+  out->counter = cb.ep_ctr[e];
+  out->state = cb.ep_state[e];
+  return FLEP_OK;
+}
+
+flep_status flep_set_rank_table(flep_rt rt, const uint16_t* rank, uint32_t n) {
+  if (!rt || !rank) return fail(FLEP_ERR_INVALID, "NULL argument");
+  if (n < rt->nsmid || n > 256) return fail(FLEP_ERR_INVALID, "rank table needs %u entries", rt->nsmid);
+  std::lock_guard<std::mutex> lk(rt->mu);
+  CUDA_TRY(cudaMemcpyAsync(rt->d_rank, rank, n * sizeof(uint16_t), cudaMemcpyHostToDevice, rt->ctl));
+  CUDA_TRY(cudaStreamSynchronize(rt->ctl));
+  return FLEP_OK;
+}
+
+flep_status flep_decision_log(flep_rt rt, int64_t* out4, size_t max_records, size_t* n_out) {
+  if (!rt || !n_out) return fail(FLEP_ERR_INVALID, "NULL argument");
+  std::lock_guard<std::mutex> lk(rt->mu);
+  if (!rt->policy) { *n_out = 0; return FLEP_OK; }
+  const auto& d = rt->policy->decisions();
+  const size_t n = std::min(max_records, d.size());
+  for (size_t i = 0; i < n && out4; ++i) {
+    out4[4 * i] = d[i].t; out4[4 * i + 1] = d[i].action; out4[4 * i + 2] = d[i].id; out4[4 * i + 3] = d[i].n_sms;
+  }
+  *n_out = out4 ? n : d.size();
+  return FLEP_OK;
+}
+
+flep_status flep_event_log(flep_rt rt, int64_t* out6, size_t max_records, size_t* n_out) {
+  if (!rt || !n_out) return fail(FLEP_ERR_INVALID, "NULL argument");
+  std::lock_guard<std::mutex> lk(rt->mu);
+  const size_t n = std::min(max_records, rt->evlog.size());
+  for (size_t i = 0; i < n && out6; ++i)
+    for (int j = 0; j < 6; ++j) out6[6 * i + j] = rt->evlog[i][j];
+  *n_out = out6 ? n : rt->evlog.size();
+  return FLEP_OK;
+}
+
+// ---- pure policy engine --------------------------------------------------------------------
+struct flep_policy_s {
+  Policy p;
+  flep_policy_s(int32_t k, uint32_t n) : p(k, n) {}
+};
+
+flep_status flep_policy_create(int32_t kind, uint32_t num_sms, flep_policy_t* out) {
+  if (!out) return fail(FLEP_ERR_INVALID, "out is NULL");
+  if (kind < kPolicyFIFO || kind > kPolicySLICE) return fail(FLEP_ERR_INVALID, "bad policy kind %d", kind);
+  *out = new flep_policy_s(kind == kPolicySLICE ? kPolicyHPF : kind, num_sms);
+  return FLEP_OK;
+}
+flep_status flep_policy_destroy(flep_policy_t p) { delete p; return FLEP_OK; }
+flep_status flep_policy_arrive(flep_policy_t p, int64_t t, int64_t id, int32_t prio, int64_t t_e, int64_t o) {
+  if (!p) return fail(FLEP_ERR_INVALID, "NULL policy");
+  if (p->p.entry(id)) return fail(FLEP_ERR_INVALID, "duplicate id %lld", (long long)id);
+  p->p.arrive(t, id, prio, t_e, o);
+  return FLEP_OK;
+}
+flep_status flep_policy_finish(flep_policy_t p, int64_t t, int64_t id) {
+  if (!p) return fail(FLEP_ERR_INVALID, "NULL policy");
+  if (!p->p.entry(id)) return fail(FLEP_ERR_INVALID, "unknown id %lld", (long long)id);
+  p->p.finish(t, id);
+  return FLEP_OK;
+}
+flep_status flep_policy_decisions(flep_policy_t p, int64_t* out4, size_t max_records, size_t* n_out) {
+  if (!p || !n_out) return fail(FLEP_ERR_INVALID, "NULL argument");
+  const auto& d = p->p.decisions();
+  const size_t n = std::min(max_records, d.size());
+  for (size_t i = 0; i < n && out4; ++i) {
+    out4[4 * i] = d[i].t; out4[4 * i + 1] = d[i].action; out4[4 * i + 2] = d[i].id; out4[4 * i + 3] = d[i].n_sms;
+  }
+  *n_out = out4 ? n : d.size();
+  return FLEP_OK;
+}
+
+int64_t flep_model_predict_ns(const double m[5], double grid, double cta, double input, double smem) {
+  if (!m) return 1;
+  const double v = m[0] * grid + m[1] * cta + m[2] * input + m[3] * smem + m[4];
+  const double a = v < 0 ? -v : v;
+  int64_t r = (int64_t)(a + 0.5);
+  if (v < 0) r = -r;
+  return r < 1 ? 1 : r;
+}
+
+}  // extern "C"
