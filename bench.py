@@ -1,0 +1,524 @@
+#!/usr/bin/env python
+"""FLEP-on-B200 benchmark (driver contract: one JSON line from rank 0).
+
+Default workload = BASELINE.json configs[1]: a long low-priority fp32 SpMV-CSR (2^20 rows,
+~10.5M nnz) is temporally preempted mid-run (full-GPU yield) by a short high-priority 5-point
+fp32 stencil (4096^2), then resumed. One STEP = one whole co-run: LP launch -> preemption
+request at a seeded block t* (device self-trigger, uniform over the middle half) -> LP drains ->
+HP (which arrives with the request) runs -> LP resumes and finishes. Every §8(a) step runs
+inside the timed region: launch sizing, worker entry, chunk fetch, body, poll, progress record,
+yield, resume.
+
+Headline `value` (metric = BASELINE.json's): the full-GPU preemption latency in us, measured on
+the device (%globaltimer): request visible on the GPU -> first CTA of the waiting kernel running
+(median over the timed steps; max over ranks). Also reported: drain latency (request -> last
+victim CTA gone), wrapper overhead (wrapped vs unwrapped kernel time), the roofline of the
+dominant kernel, the oracle on the host cores, and an end-to-end number through the managed
+(HPF) public API with host buffers.
+
+Other configs: --config corun1 | spatial | queue.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from synth import gen  # noqa: E402
+
+METRIC = ("preemption latency µs (full vs N-SM yield); wrapper overhead % of HBM/tensor roofline; "
+          "co-run NATT")
+HBM_FALLBACK_GBS = 6650.0
+
+
+def peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            p = json.load(f)
+        return float(p["hbm_gbs"]), float(p.get("bf16_tflops", 1590.0)), float(p.get("bf16_tflops_sustained", 1400.0)), "measured"
+    except Exception:
+        return HBM_FALLBACK_GBS, 1590.0, 1400.0, "fallback"
+
+
+# ------------------------------------------------------------------------------------------
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled DURING the timed region."""
+
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index):
+        self.idx = gpu_index
+        self.p = None
+
+    def __enter__(self):
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", "-i", str(self.idx), f"--query-gpu={self.FIELDS}",
+                                       "--format=csv,noheader,nounits", "-lms", "50"],
+                                      stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self.p = None
+        return self
+
+    def __exit__(self, *a):
+        self.out = ""
+        if self.p is not None:
+            self.p.terminate()
+            try:
+                self.out, _ = self.p.communicate(timeout=5)
+            except Exception:
+                self.p.kill()
+
+    def summary(self):
+        sm, mx, reasons = [], 0.0, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in (self.out or "").splitlines():
+            f = [x.strip() for x in line.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sm.append(float(f[1]))
+                mx = max(mx, float(f[2]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[5:9]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        load = [s for s in sm if s > 300] or sm
+        return {"sm_mhz": statistics.median(load) if load else None, "sm_max_mhz": mx or None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def physical_gpu_index(local_rank):
+    vis = os.environ.get("CUDA_VISIBLE_DEVICES")
+    if vis:
+        ids = [v.strip() for v in vis.split(",") if v.strip()]
+        if local_rank < len(ids) and ids[local_rank].isdigit():
+            return int(ids[local_rank])
+    return local_rank
+
+
+# ------------------------------------------------------------------------------------------
+def dist_setup():
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return rank, world, local
+
+
+def allreduce_max(vals, world, torch):
+    if world == 1:
+        return vals
+    import torch.distributed as dist
+    t = torch.tensor(vals, dtype=torch.float64, device="cuda")
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return t.tolist()
+
+
+def barrier(world):
+    if world > 1:
+        import torch.distributed as dist
+        dist.barrier()
+
+
+# ------------------------------------------------------------------------------------------
+SPMV_ROWS = 1 << 20
+STENCIL_N = 4096
+
+
+def spmv_bytes(rowptr, rows, cols):
+    nnz = int(rowptr[-1])
+    return 8 * nnz + 8 * rows + 4 * cols      # 8 B/nnz + 8 B/row + 4 B/col
+
+
+def stencil_bytes(n):
+    return 8 * n * n                            # 8 B/cell
+
+
+class Workload:
+    def __init__(self, torch, seed_off=0):
+        self.torch = torch
+        self.rowptr, self.col, self.val, self.x = gen.csr_inputs(SPMV_ROWS, seed=2 + seed_off)
+        self.st_in = gen.stencil_f32_input(STENCIL_N, seed=3 + seed_off)
+        dev = "cuda"
+        T = lambda a: torch.from_numpy(np.ascontiguousarray(a)).to(dev)  # noqa: E731
+        self.d_rowptr, self.d_col, self.d_val, self.d_x = T(self.rowptr), T(self.col), T(self.val), T(self.x)
+        self.d_y = torch.zeros(SPMV_ROWS, dtype=torch.float32, device=dev)
+        self.d_in = T(self.st_in)
+        self.d_out = torch.empty_like(self.d_in)
+        self.nnz = int(self.rowptr[-1])
+        self.spmv_bytes = spmv_bytes(self.rowptr, SPMV_ROWS, SPMV_ROWS)
+        self.st_bytes = stencil_bytes(STENCIL_N)
+
+
+def l2_flush_buffer(torch):
+    l2 = torch.cuda.get_device_properties(0).L2_cache_size
+    return torch.empty(max(2 * l2, 256 << 20), dtype=torch.uint8, device="cuda")
+
+
+def run_temporal(args, rank, world, local):
+    import torch
+    from paper_conf_asplos_wulzj17_b200 import flep as F
+    torch.cuda.set_device(local)
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    hbm, _, _, peak_src = peaks()
+    wl = Workload(torch)
+    flush = l2_flush_buffer(torch)
+    # The waiting kernel is enqueued right behind the victim so that it is already pending when
+    # the request fires. The victim's stream gets the higher CUDA priority only so that the
+    # hardware dispatches all victim workers first when both become ready together (checked
+    # per step: the waiting kernel must not start before the request).
+    A = torch.cuda.Stream(priority=-2)
+    B = torch.cuda.Stream(priority=0)
+    rt = F.Runtime(device=local, exec_on_user_stream=True)
+    num_sms = rt.num_sms
+    kLP = rt.register_kernel(F.BODY_SPMV_CSR_F32, chunk=args.lp_chunk, poll=args.lp_poll, name="spmv",
+                             prefetch=bool(args.prefetch))
+    kHP = rt.register_kernel(F.BODY_STENCIL5_F32, chunk=1, poll=1, name="stencil", prefetch=bool(args.prefetch))
+    lp_args = F.spmv_args(wl.d_y, wl.d_rowptr, wl.d_col, wl.d_val, wl.d_x)
+    hp_args = F.stencil_args(wl.d_out, wl.d_in)
+    lp_grid, hp_grid = F.spmv_grid(SPMV_ROWS), F.stencil_grid(STENCIL_N)
+    n_lp = lp_grid[0]
+    g = gen.rng(1000 + rank)
+
+    def step():
+        tstar = int(g.integers(n_lp // 4, 3 * n_lp // 4))
+        with torch.cuda.stream(A):
+            flush.zero_()
+            e0 = torch.cuda.Event(enable_timing=True)
+            e0.record(A)
+        rt.arm_next_trigger(tstar, num_sms)
+        h_lp = rt.launch(kLP, lp_grid, lp_args, priority=0, stream=A)
+        B.wait_event(e0)
+        h_hp = rt.launch(kHP, hp_grid, hp_args, priority=1, stream=B)
+        rt.wait_epoch(h_lp, timeout_ns=10_000_000_000)
+        info = rt.query(h_lp)
+        preempted = info.state == F.STATE_PREEMPTED
+        rt.sync(h_hp, timeout_ns=10_000_000_000)      # FLEP resumes the victim when the HP ends
+        if preempted:
+            rt.resume(h_lp)
+        rt.sync(h_lp, timeout_ns=10_000_000_000)
+        e_b = torch.cuda.Event()
+        e_b.record(B)
+        A.wait_event(e_b)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e1.record(A)
+        e1.synchronize()
+        ep = rt.epoch_info(h_lp, 1)
+        hp_ev = rt.events(h_hp, 1)
+        lp_ev = rt.events(h_lp, 1)
+        t_req = ep.t_trigger
+        hp_start = min(e.t_entry for e in hp_ev)
+        hp_end = max(e.t_exit for e in hp_ev)
+        lp_start = min(e.t_entry for e in lp_ev)
+        launches = rt.query(h_lp).epoch + rt.query(h_hp).epoch
+        valid = preempted and t_req > 0 and hp_start >= t_req
+        return {
+            "preempted": valid,
+            "hp_started_early": bool(t_req and hp_start < t_req),
+            "latency_us": (hp_start - t_req) / 1e3 if t_req else None,
+            "drain_us": (ep.t_end - t_req) / 1e3 if t_req else None,
+            "hp_turnaround_us": (hp_end - t_req) / 1e3 if t_req else None,
+            "lp_before_request_us": (t_req - lp_start) / 1e3 if t_req else None,
+            "step_ms": e0.elapsed_time(e1),
+            "launches": launches,
+            "tstar": tstar,
+        }
+
+    res = []
+    with ClockSampler(physical_gpu_index(local)) as clk:
+        for _ in range(args.warmup):
+            step()
+        torch.cuda.synchronize()
+        barrier(world)
+        t_start = time.perf_counter()
+        for _ in range(args.steps):
+            res.append(step())
+        torch.cuda.synchronize()
+        barrier(world)
+        wall = time.perf_counter() - t_start
+    clocks = clk.summary()
+    # correctness spot check of the last co-run (device result vs oracle rows / cells sampled)
+    parity = spot_parity(wl, torch)
+
+    lat = [r["latency_us"] for r in res if r["preempted"]]
+    drain = [r["drain_us"] for r in res if r["preempted"]]
+    hpt = [r["hp_turnaround_us"] for r in res if r["preempted"]]
+    ms = [r["step_ms"] for r in res]
+    p50 = float(np.median(lat)) if lat else float("nan")
+    p99 = float(np.percentile(lat, 99)) if lat else float("nan")
+    ms_step = float(np.mean(ms))
+    red = allreduce_max([p50, ms_step], world, torch)
+
+    # ---- wrapper overhead + roofline (standalone launches, L2 flushed, CUDA events on stream A)
+    kern = kernel_timings(rt, F, torch, wl, flush, A, kLP, kHP, lp_args, hp_args, lp_grid, hp_grid, args.reps)
+    dom = max(("spmv", "stencil"), key=lambda k: kern[k]["wrapped_us"])
+    algo = wl.spmv_bytes if dom == "spmv" else wl.st_bytes
+    achieved = algo / (kern[dom]["wrapped_us"] * 1e-6) / 1e9
+    prof_traffic = load_traffic(dom)
+    roofline = {"bound": "hbm", "achieved": round(achieved, 1), "peak": hbm, "unit": "GB/s",
+                "frac": round(achieved / hbm, 4), "traffic": prof_traffic, "kernel": f"flep_worker<{dom}>",
+                "algorithmic_bytes": algo, "peak_source": peak_src}
+
+    e2e = run_e2e(F, torch, wl, local, args.e2e_steps)
+    rt.close()
+
+    out = {
+        "metric": METRIC,
+        "value": round(red[0], 3),
+        "unit": "us",
+        "n_gpus": world,
+        "steps": args.steps,
+        "warmup": args.warmup,
+        "ms_per_step": round(red[1], 4),
+        "higher_is_better": False,
+        "scaling": "weak",
+        "vs_baseline": None,
+        "dtype": "f32",
+        "data": "synthetic (seeded; synth/gen.py)",
+        "config": {"workload": "configs[1]: full-GPU temporal preemption of SpMV-CSR fp32 (2^20 rows, "
+                               f"{wl.nnz} nnz, low priority) by stencil5 fp32 4096^2 (high priority)",
+                   "lp_chunk": args.lp_chunk, "lp_poll": args.lp_poll, "hp_chunk": 1, "hp_poll": 1,
+                   "prefetch": bool(args.prefetch),
+                   "flag": "stream_memop (device self-trigger for the request)",
+                   "l2": "flushed between steps (write of 2x L2 bytes)", "parallelism": f"replicas x{world}"},
+        "latency_us": {"p50": round(p50, 3), "p99": round(p99, 3), "max": round(max(lat), 3) if lat else None,
+                       "min": round(min(lat), 3) if lat else None, "preempted_steps": len(lat),
+                       "definition": "device %globaltimer: preemption request visible on the GPU -> first CTA of the waiting kernel running"},
+        "drain_us": {"p50": round(float(np.median(drain)), 3) if drain else None,
+                     "max": round(max(drain), 3) if drain else None},
+        "hp_turnaround_us": {"p50": round(float(np.median(hpt)), 3) if hpt else None},
+        "target_20us_met": bool(lat) and max(lat) < 20.0,
+        "wrapper_overhead_pct": {k: v["overhead_pct"] for k, v in kern.items()},
+        "kernels": kern,
+        "roofline": roofline,
+        "e2e": e2e,
+        "gpu_launches": int(sum(r["launches"] for r in res)),
+        "hp_started_before_request": int(sum(1 for r in res if r["hp_started_early"])),
+        "clocks": clocks,
+        "parity": parity,
+        "wall_s_timed": round(wall, 3),
+    }
+    if rank == 0:
+        out["cpu_baseline"] = cpu_baseline(wl)
+        print(json.dumps(out), flush=True)
+    barrier(world)
+
+
+def spot_parity(wl, torch):
+    """Sampled element-by-element check of the last co-run's outputs against the oracle."""
+    from oracle import workloads as W
+    g = gen.rng(7)
+    rows = g.integers(0, SPMV_ROWS, 512)
+    y = wl.d_y.cpu().numpy()
+    worst = 0.0
+    for r in rows:
+        s, e = wl.rowptr[r], wl.rowptr[r + 1]
+        sub_rp = np.array([0, e - s], np.int32)
+        ref, absum = W.spmv_csr(sub_rp, wl.col[s:e], wl.val[s:e], wl.x)
+        d = max(abs(ref[0]), absum[0], 1e-30)
+        worst = max(worst, abs(float(y[r]) - ref[0]) / d)
+    out = wl.d_out.cpu().numpy()
+    ref, absum = W.stencil5_f32(wl.st_in[:130, :130])
+    d = np.maximum(np.abs(ref), absum)
+    worst_st = float(np.max(np.abs(out[:129, :129] - ref[:129, :129]) / np.where(d[:129, :129] > 0, d[:129, :129], 1)))
+    return {"spmv_max_rel": worst, "stencil_max_rel": worst_st, "tol": 1e-5,
+            "ok": bool(worst <= 1e-5 and worst_st <= 1e-5)}
+
+
+def kernel_timings(rt, F, torch, wl, flush, A, kLP, kHP, lp_args, hp_args, lp_grid, hp_grid, reps):
+    res = {}
+    for name, k, body, a, grid, nbytes in (("spmv", kLP, F.BODY_SPMV_CSR_F32, lp_args, lp_grid, wl.spmv_bytes),
+                                           ("stencil", kHP, F.BODY_STENCIL5_F32, hp_args, hp_grid, wl.st_bytes)):
+        tw, tu = [], []
+        for r in range(reps + 2):
+            for mode in ("w", "u"):
+                with torch.cuda.stream(A):
+                    flush.zero_()
+                    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                    e0.record(A)
+                if mode == "w":
+                    h = rt.launch(k, grid, a, stream=A)
+                else:
+                    rt.launch_unwrapped(body, grid, a, stream=A)
+                e1.record(A)
+                e1.synchronize()
+                if mode == "w":
+                    rt.sync(h)
+                if r >= 2:
+                    (tw if mode == "w" else tu).append(e0.elapsed_time(e1) * 1e3)
+        w_us, u_us = float(np.median(tw)), float(np.median(tu))
+        res[name] = {"wrapped_us": round(w_us, 3), "unwrapped_us": round(u_us, 3),
+                     "wrapped_min_us": round(min(tw), 3), "unwrapped_min_us": round(min(tu), 3),
+                     "wrapped_gbs": round(nbytes / (w_us * 1e-6) / 1e9, 1),
+                     "unwrapped_gbs": round(nbytes / (u_us * 1e-6) / 1e9, 1),
+                     "overhead_pct": round((w_us / u_us - 1.0) * 100.0, 2),
+                     "algorithmic_bytes": nbytes}
+    return res
+
+
+def load_traffic(dom):
+    """dram bytes per launch from the committed ncu --set full capture, if present."""
+    p = os.path.join(ROOT, "profiles", "traffic.json")
+    try:
+        with open(p) as f:
+            return json.load(f).get(dom)
+    except Exception:
+        return None
+
+
+def run_e2e(F, torch, wl, local, steps):
+    """Same metric through the managed public API (HPF policy), with host buffers: every step
+    copies the inputs from pinned host memory, the HP arrival is an intercepted flep_launch that
+    makes the runtime preempt the running LP, and the outputs are read back. Latency = host
+    clock from the runtime's preemption request to its observation of the drained epoch."""
+    rt = F.Runtime(device=local, policy=F.POLICY_HPF)
+    kLP = rt.register_kernel(F.BODY_SPMV_CSR_F32, chunk=4, poll=1, name="spmv", model=(0, 0, 0, 0, 20_000))
+    kHP = rt.register_kernel(F.BODY_STENCIL5_F32, chunk=1, poll=1, name="stencil", model=(0, 0, 0, 0, 25_000))
+    pin = lambda a: torch.from_numpy(np.ascontiguousarray(a)).pin_memory()  # noqa: E731
+    h_rp, h_col, h_val, h_x, h_in = pin(wl.rowptr), pin(wl.col), pin(wl.val), pin(wl.x), pin(wl.st_in)
+    h_y = torch.empty(SPMV_ROWS, dtype=torch.float32).pin_memory()
+    h_out = torch.empty_like(h_in).pin_memory()
+    A = torch.cuda.Stream(priority=0)
+    B = torch.cuda.Stream(priority=-2)
+    lp_args = F.spmv_args(wl.d_y, wl.d_rowptr, wl.d_col, wl.d_val, wl.d_x)
+    hp_args = F.stencil_args(wl.d_out, wl.d_in)
+    h2d = sum(t.numel() * t.element_size() for t in (h_rp, h_col, h_val, h_x, h_in))
+    d2h = h_y.numel() * 4 + h_out.numel() * 4
+    lats, step_ms, pre = [], [], 0
+    for i in range(steps + 2):
+        t0 = time.perf_counter()
+        with torch.cuda.stream(A):
+            for d, h in ((wl.d_rowptr, h_rp), (wl.d_col, h_col), (wl.d_val, h_val), (wl.d_x, h_x)):
+                d.copy_(h, non_blocking=True)
+        with torch.cuda.stream(B):
+            wl.d_in.copy_(h_in, non_blocking=True)
+        A.synchronize()
+        h_lp = rt.launch(kLP, F.spmv_grid(SPMV_ROWS), lp_args, priority=0, stream=A)
+        h_hp = rt.launch(kHP, F.stencil_grid(STENCIL_N), hp_args, priority=1, stream=B)
+        rt.sync(h_hp, timeout_ns=10_000_000_000)
+        rt.sync(h_lp, timeout_ns=10_000_000_000)
+        with torch.cuda.stream(A):
+            h_y.copy_(wl.d_y, non_blocking=True)
+        with torch.cuda.stream(B):
+            h_out.copy_(wl.d_out, non_blocking=True)
+        A.synchronize()
+        B.synchronize()
+        dt = (time.perf_counter() - t0) * 1e3
+        info = rt.query(h_lp)
+        if i >= 2:
+            step_ms.append(dt)
+            if info.epoch >= 2 and info.t_last_drain > 0:
+                pre += 1
+                lats.append((info.t_last_drain - info.t_last_request) / 1e3)
+    dec = rt.decision_log()
+    rt.close()
+    return {"value": round(float(np.median(lats)), 3) if lats else None, "unit": "us",
+            "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
+            "preempted_steps": pre, "steps": steps, "ms_per_step": round(float(np.median(step_ms)), 3),
+            "definition": "host clock: HPF runtime's preemption request (cuStreamWriteValue32 issued) -> "
+                          "host observes the victim's drained epoch; inputs H2D from pinned memory and "
+                          "outputs D2H inside every step",
+            "decisions_last": [F.ACTION_NAMES[d[1]] for d in dec[-4:]]}
+
+
+def cpu_baseline(wl):
+    """The oracle (as it stands) on the host cores, on this workload: a non-preemptive CPU
+    program must finish the LP's remaining blocks before the HP can start, so its 'preemption
+    latency' is the oracle time for the LP rows after t* (t* = N/2 here)."""
+    from oracle import workloads as W
+    half = SPMV_ROWS // 2
+    s = wl.rowptr[half]
+    rp = (wl.rowptr[half:] - s).astype(np.int32)
+    t0 = time.perf_counter()
+    W.spmv_csr(rp, wl.col[s:], wl.val[s:], wl.x)
+    t_rem = time.perf_counter() - t0
+    t0 = time.perf_counter()
+    W.stencil5_f32(wl.st_in)
+    t_st = time.perf_counter() - t0
+    return {"value": round(t_rem * 1e6, 1), "unit": "us", "cores": 1, "kind": "oracle",
+            "sample": "oracle SpMV over the LP's remaining half (2^19 rows) = the HP's wait on a "
+                      f"non-preemptive CPU; oracle stencil 4096^2 alone took {t_st * 1e6:.0f} us",
+            "threads_note": "numpy element-wise + np.add.at, single-threaded"}
+
+
+def run_reference(args, rank, world):
+    """--impl reference: the oracle, timed on the host cores, same config/metric/unit."""
+    if rank != 0:
+        return
+    from oracle import workloads as W
+    rowptr, col, val, x = gen.csr_inputs(SPMV_ROWS, seed=2)
+    st_in = gen.stencil_f32_input(STENCIL_N, seed=3)
+    n_lp = (SPMV_ROWS + 127) // 128
+    g = gen.rng(1000)
+    lats, steps_ms = [], []
+    for i in range(args.warmup + args.steps):
+        tstar = int(g.integers(n_lp // 4, 3 * n_lp // 4))
+        r0 = tstar * 128
+        s = rowptr[r0]
+        t0 = time.perf_counter()
+        W.spmv_csr((rowptr[r0:] - s).astype(np.int32), col[s:], val[s:], x)
+        t1 = time.perf_counter()
+        W.stencil5_f32(st_in)
+        t2 = time.perf_counter()
+        if i >= args.warmup:
+            lats.append((t1 - t0) * 1e6)
+            steps_ms.append((t2 - t0) * 1e3)
+    v = float(np.median(lats))
+    out = {"impl": "reference", "metric": METRIC, "value": round(v, 1), "unit": "us", "n_gpus": world,
+           "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(float(np.mean(steps_ms)), 3),
+           "higher_is_better": False, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+           "data": "synthetic (seeded; synth/gen.py)",
+           "config": {"workload": "configs[1]: SpMV-CSR (2^20 rows) then stencil5 4096^2 on the CPU oracle"},
+           "cpu_baseline": {"value": round(v, 1), "unit": "us", "cores": 1, "kind": "oracle",
+                            "sample": "per step: oracle SpMV over the LP rows after a seeded t* (what a "
+                                      "non-preemptive program must finish before the HP starts) + oracle stencil"},
+           "e2e": {"value": round(v, 1), "unit": "us", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(out), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=10)
+    ap.add_argument("--impl", default="flep", choices=["flep", "reference"])
+    ap.add_argument("--config", default="temporal", choices=["temporal"])
+    ap.add_argument("--lp-chunk", type=int, default=1)
+    ap.add_argument("--prefetch", type=int, default=1)
+    ap.add_argument("--lp-poll", type=int, default=1)
+    ap.add_argument("--reps", type=int, default=20)
+    ap.add_argument("--e2e-steps", type=int, default=10)
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+    rank, world, local = dist_setup()
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+    from paper_conf_asplos_wulzj17_b200 import build
+    if rank == 0:
+        build.build()
+    if world > 1:
+        # wait for rank 0's build: poll for the library
+        from paper_conf_asplos_wulzj17_b200 import build as b2
+        for _ in range(600):
+            if not b2.needs_build():
+                break
+            time.sleep(1)
+    run_temporal(args, rank, world, local)
+
+
+if __name__ == "__main__":
+    main()

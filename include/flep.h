@@ -23,10 +23,11 @@
  *     value at flep_launch().
  *   - The runtime owns its control blocks, internal CUDA streams (one high-priority control
  *     stream, a pool of execution streams) and pinned host status words.
- *   - flep_launch / flep_preempt / flep_resume are asynchronous. Completion is observable
- *     through flep_sync / flep_query. When flep_options.order_user_stream is set, work the
- *     caller enqueues on `stream` after flep_launch waits for TRUE completion (every block done,
- *     possibly after several preempt/resume cycles), via a stream wait on the done counter.
+ *   - flep_launch / flep_preempt / flep_resume are asynchronous. Work the caller enqueued on
+ *     `stream` BEFORE flep_launch precedes the workers (event dependency). Completion (every
+ *     block done, possibly after several preempt/resume cycles) is observable through
+ *     flep_sync / flep_query; the runtime never blocks a stream on a device-written value
+ *     (front-end waits can deadlock when streams share a hardware queue).
  *   - Priority: larger value = higher priority (Fig. 6 line 1: Kr.priority < Kn.priority ->
  *     preempt). The runtime maps it onto CUDA stream priorities internally.
  *   - One runtime per device; all entry points are thread-safe (internal mutex).
@@ -101,8 +102,12 @@ typedef struct {
   uint32_t default_chunk;      /* C: original blocks per counter fetch (0 -> 8) */
   uint32_t default_poll;       /* K: chunks between control-word polls (0 -> 1) */
   uint32_t debug_coverage;     /* 1: keep a per-block execution count cov[N] (test builds) */
-  uint32_t order_user_stream;  /* 1: caller stream waits for true completion (see above) */
+  uint32_t reserved0;          /* must be 0 */
   uint32_t slice_blocks;       /* SLICE policy: blocks per sub-kernel (0 -> W*C*K, A20) */
+  uint32_t exec_on_user_stream;/* MANUAL mode: launch worker grids (and resumes) directly on the
+                                  caller's stream instead of a runtime stream. Stream order then
+                                  only covers the epoch grids: the caller must resume before
+                                  enqueuing work that depends on the results. */
 } flep_options;
 
 typedef struct {
@@ -112,7 +117,14 @@ typedef struct {
   double model[5];             /* ridge model: T_e ns = m0*grid + m1*cta + m2*input
                                   + m3*smem + m4, rounded once to integer ns */
   int64_t preempt_overhead_ns; /* O: profiled mean preemption overhead */
+  uint32_t flags;              /* FLEP_KFLAG_* */
+  uint32_t ctas_per_sm;        /* resident workers per SM (0 = the occupancy maximum) */
 } flep_kernel_desc;
+
+/* Prefetch the next chunk's index while the current chunk runs (hides the counter atomic's
+   latency; a worker that must yield still executes the chunk it holds, so the drain can take up
+   to one extra chunk). */
+#define FLEP_KFLAG_PREFETCH 1u
 
 typedef enum {
   FLEP_STATE_QUEUED = 0,     /* intercepted, waiting for a scheduling decision (S2) */
@@ -133,6 +145,8 @@ typedef struct {
   int64_t t_arrive, t_first_start, t_finish;  /* host steady clock, ns */
   uint32_t workers;            /* W: worker CTAs per epoch */
   uint32_t n_yield;            /* yield width currently requested (0 = none) */
+  int64_t t_last_request;      /* host ns of the last preempt request issued by the runtime */
+  int64_t t_last_drain;        /* host ns the runtime observed the last PREEMPTED epoch end */
 } flep_launch_info;
 
 /* Per-worker event record of one epoch (device %globaltimer, ns). */

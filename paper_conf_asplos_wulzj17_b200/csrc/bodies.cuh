@@ -6,10 +6,9 @@
 // bit-identical outputs (SURVEY §8(c) "Parity criteria").
 //
 //   SAXPY  (VA-shaped, Table 1): block b = elements [256b, 256b+256); 128-bit ld/st.
-//   SpMV   (SPMV): block b = rows [32b, 32b+32); 8 lanes per row, fixed-order reduction.
+//   SpMV   (SPMV): block b = rows [128b, 128b+128); CSR-stream, fixed-order row sums.
 //   Stencil5 (BJ "2D stencil"; PF/CFD-shaped): block (tx, ty) = 64x64 output tile; each thread
-//          produces 4 contiguous cells per row pass with 128-bit loads; neighbours come from the
-//          L1/L2-resident rows of the same and adjacent tiles.
+//          produces a 4x4 patch with 128-bit loads; halo rows/columns come from L1/L2.
 #pragma once
 #include <cstdint>
 #include "../../include/flep.h"
@@ -79,29 +78,60 @@ struct SaxpyBody {
 };
 
 // ---------------------------------------------------------------------------------------------
-// SpMV-CSR fp32: y[r] = sum_p val[p] * x[col[p]]. 8 lanes per row: lane l accumulates
-// p = start+l, start+l+8, ... with fma in that order, then a fixed xor-butterfly over 8 lanes.
+// SpMV-CSR fp32: y[r] = sum_p val[p] * x[col[p]]. Block b = rows [128b, 128b+128).
+// CSR-stream form: the block's rowptr slice goes to smem; all 256 threads then stream the
+// block's contiguous nnz range [rowptr[r0], rowptr[r1]) in tiles of kTile entries (coalesced
+// col/val loads, independent x gathers, 4 in flight per thread), writing products to smem; thread
+// t < 128 finally sums row r0+t's products in ascending p order. Per-row summation order is
+// fixed, so every execution of a block gives bit-identical results.
 struct SpmvBody {
   static constexpr int kThreads = 256;
   static constexpr int kMinBlocks = 8;
-  static constexpr uint32_t kRowsPerBlock = 32;
+  static constexpr uint32_t kRowsPerBlock = 128;
+  static constexpr uint32_t kTile = 1024;
   using Args = flep_spmv_args;
 
   __device__ static void run(const Args& g, uint32_t b0, uint32_t b1, uint32_t, uint32_t) {
-    const uint32_t lane8 = threadIdx.x & 7u;
-    const uint32_t rloc = threadIdx.x >> 3;
+    __shared__ int32_t s_rp[kRowsPerBlock + 1];
+    __shared__ float s_prod[kTile];
+    const uint32_t tid = threadIdx.x;
     for (uint32_t b = b0; b < b1; ++b) {
-      const uint32_t row = b * kRowsPerBlock + rloc;
-      float sum = 0.f;
-      if (row < g.rows) {
-        const int32_t s = __ldg(g.rowptr + row), e = __ldg(g.rowptr + row + 1);
-        for (int32_t p = s + (int32_t)lane8; p < e; p += 8)
-          sum = fmaf(__ldcs(g.val + p), __ldg(g.x + __ldcs(g.col + p)), sum);
+      const uint32_t r0 = b * kRowsPerBlock;
+      const uint32_t nr = min(kRowsPerBlock, g.rows - r0);
+      if (tid <= nr) s_rp[tid] = __ldg(g.rowptr + r0 + tid);
+      __syncthreads();
+      const int32_t p0 = s_rp[0], p1 = s_rp[nr];
+      int32_t my_s = 0, my_e = 0;
+      if (tid < nr) { my_s = s_rp[tid]; my_e = s_rp[tid + 1]; }
+      float acc = 0.f;
+      for (int32_t base = p0; base < p1; base += (int32_t)kTile) {
+        const int32_t n = min((int32_t)kTile, p1 - base);
+        constexpr int U = 4;
+        for (int32_t i0 = (int32_t)tid; i0 < n; i0 += U * kThreads) {
+          int32_t c[U];
+          float v[U], xv[U];
+#pragma unroll
+          for (int u = 0; u < U; ++u) {
+            const int32_t i = i0 + u * kThreads;
+            c[u] = i < n ? __ldcs(g.col + base + i) : 0;
+            v[u] = i < n ? __ldcs(g.val + base + i) : 0.f;
+          }
+#pragma unroll
+          for (int u = 0; u < U; ++u) xv[u] = __ldg(g.x + c[u]);
+#pragma unroll
+          for (int u = 0; u < U; ++u) {
+            const int32_t i = i0 + u * kThreads;
+            if (i < n) s_prod[i] = v[u] * xv[u];
+          }
+        }
+        __syncthreads();
+        if (tid < nr) {
+          const int32_t lo = max(my_s, base), hi = min(my_e, base + n);
+          for (int32_t p = lo; p < hi; ++p) acc += s_prod[p - base];
+        }
+        __syncthreads();
       }
-      sum += __shfl_xor_sync(0xffffffffu, sum, 4);
-      sum += __shfl_xor_sync(0xffffffffu, sum, 2);
-      sum += __shfl_xor_sync(0xffffffffu, sum, 1);
-      if (row < g.rows && lane8 == 0) __stcs(g.y + row, sum);
+      if (tid < nr) __stcs(g.y + r0 + tid, acc);
     }
   }
 };
@@ -112,7 +142,7 @@ struct SpmvBody {
 template <bool kInt>
 struct Stencil5Body {
   static constexpr int kThreads = 256;
-  static constexpr int kMinBlocks = 6;
+  static constexpr int kMinBlocks = 4;
   static constexpr uint32_t kTile = 64;
   using Args = flep_stencil_args;
 
@@ -123,6 +153,9 @@ struct Stencil5Body {
     return __float_as_uint(0.5f * fc + 0.125f * (((fn + fs) + fw) + fe));
   }
 
+  // Vector path (n % 4 == 0): thread (q, rg) owns columns [c0+4q, c0+4q+4) of rows
+  // r0+4rg .. r0+4rg+3. It loads the 6 rows r-1..r+4 of its 4-column strip (128-bit) and the
+  // west/east neighbours of its 4 rows up front (14 independent loads in flight), then computes.
   __device__ static void run(const Args& g, uint32_t b0, uint32_t b1, uint32_t gx, uint32_t) {
     const uint32_t n = g.n;
     const uint32_t* __restrict__ in = reinterpret_cast<const uint32_t*>(g.in);
@@ -131,28 +164,39 @@ struct Stencil5Body {
       const uint32_t tx = b % gx, ty = b / gx;
       const uint32_t r0 = ty * kTile, c0 = tx * kTile;
       if ((n & 3u) == 0) {
-        const uint32_t q = threadIdx.x & 15u, rr = threadIdx.x >> 4;   // 16 float4 x 16 rows
+        const uint32_t q = threadIdx.x & 15u, rg = threadIdx.x >> 4;   // 16 strips x 16 row groups
         const uint32_t c = c0 + 4u * q;
+        const uint32_t rb = r0 + 4u * rg;
+        if (c >= n || rb >= n) continue;
+        uint4 R[6];
+        uint32_t Wv[4], Ev[4];
 #pragma unroll
-        for (uint32_t pass = 0; pass < kTile / 16; ++pass) {
-          const uint32_t r = r0 + rr + 16u * pass;
-          if (r >= n || c >= n) continue;
-          const size_t off = (size_t)r * n + c;
-          const uint4 C = __ldg(reinterpret_cast<const uint4*>(in + off));
+        for (int i = 0; i < 6; ++i) {
+          const int32_t r = (int32_t)rb - 1 + i;
+          R[i] = (r >= 0 && r < (int32_t)n) ? __ldg(reinterpret_cast<const uint4*>(in + (size_t)r * n + c))
+                                            : make_uint4(0, 0, 0, 0);
+        }
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          const uint32_t r = rb + i;
+          Wv[i] = (r < n && c > 0) ? __ldg(in + (size_t)r * n + c - 1) : 0u;
+          Ev[i] = (r < n && c + 4 < n) ? __ldg(in + (size_t)r * n + c + 4) : 0u;
+        }
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          const uint32_t r = rb + i;
+          if (r >= n) break;
+          const uint4 C = R[i + 1], N = R[i], S = R[i + 2];
           uint4 O;
           if (r == 0 || r == n - 1) {
             O = C;
           } else {
-            const uint4 N = __ldg(reinterpret_cast<const uint4*>(in + off - n));
-            const uint4 S = __ldg(reinterpret_cast<const uint4*>(in + off + n));
-            const uint32_t W = (c > 0) ? __ldg(in + off - 1) : 0u;
-            const uint32_t E = (c + 4 < n) ? __ldg(in + off + 4) : 0u;
-            O.x = (c == 0) ? C.x : cell(C.x, N.x, S.x, W, C.y);
+            O.x = (c == 0) ? C.x : cell(C.x, N.x, S.x, Wv[i], C.y);
             O.y = cell(C.y, N.y, S.y, C.x, C.z);
             O.z = cell(C.z, N.z, S.z, C.y, C.w);
-            O.w = (c + 3 == n - 1) ? C.w : cell(C.w, N.w, S.w, C.z, E);
+            O.w = (c + 3 == n - 1) ? C.w : cell(C.w, N.w, S.w, C.z, Ev[i]);
           }
-          __stcs(reinterpret_cast<uint4*>(out + off), O);
+          __stcs(reinterpret_cast<uint4*>(out + (size_t)r * n + c), O);
         }
       } else {
         // scalar path for n % 4 != 0 (ragged rows)

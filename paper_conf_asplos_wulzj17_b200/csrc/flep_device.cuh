@@ -73,6 +73,8 @@ struct WorkerParams {
   uint32_t gx, gy;         // original grid (x, y); z folded into the flat index
   uint32_t trigger_block;  // device self-trigger for this epoch (kNoTrigger = none)
   uint32_t trigger_n;      // its yield width
+  uint32_t prefetch;       // 1: fetch chunk j+1 while chunk j runs (hides the atomic's latency;
+                           //    a stopping worker still processes the prefetched chunk)
 };
 
 __device__ __forceinline__ uint32_t smid_reg() {
@@ -83,6 +85,13 @@ __device__ __forceinline__ uint64_t gtimer() {
 }
 __device__ __forceinline__ uint32_t ld_acquire_gpu(const uint32_t* p) {
   uint32_t v; asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory"); return v;
+}
+// The poll: a relaxed gpu-scope load (served by L2, never a stale L1 line). Deliberately NOT
+// ld.acquire: on sm_100a an acquire load is followed by CCTL.IVALL, which would invalidate the
+// SM's whole L1 at every poll and evict the bodies' cached neighbours. Nothing read after the
+// poll depends on data published before the request, so no acquire ordering is needed.
+__device__ __forceinline__ uint32_t ld_relaxed_gpu(const uint32_t* p) {
+  uint32_t v; asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory"); return v;
 }
 __device__ __forceinline__ uint32_t ld_acquire_sys(const uint32_t* p) {
   uint32_t v; asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory"); return v;
@@ -124,27 +133,30 @@ flep_worker(const typename Body::Args args, const WorkerParams p) {
   if (tid == 0) { s_sm = smid_reg(); s_t_entry = gtimer(); s_blocks = 0; s_reason = 0; }
   uint32_t k = 0;                    // chunk index within the current poll period
   uint32_t parity = 0;
+  uint32_t held = 0xffffffffu;       // tid 0: prefetched chunk base not yet processed
+  bool stopping = false;             // tid 0: a request named this SM; drain the held chunk
   while (true) {
     if (tid == 0) {
       uint32_t base;
-      bool stop = false;
-      if (k == 0) {                                      // amortised poll (Fig. 4(b))
-        const uint32_t c = ld_acquire_gpu(p.ctrl);
-        if (should_yield(c, p, smid_reg())) stop = true;
+      if (k == 0 && !stopping) {                         // amortised poll (Fig. 4(b))
+        const uint32_t c = ld_relaxed_gpu(p.ctrl);
+        if (should_yield(c, p, smid_reg())) { stopping = true; s_reason = kReasonYield; }
       }
-      if (stop) {
-        base = 0xffffffffu; s_reason = kReasonYield;
+      if (held != 0xffffffffu) {                         // a fetched chunk is always processed (A4)
+        base = held;
+        held = 0xffffffffu;
       } else {
-        base = atomicAdd(&p.cb->ctr, p.chunk);          // pull_task
-        if (base >= p.n_blocks) { base = 0xffffffffu; s_reason = kReasonExhausted; }
-        else {
-          s_blocks += min(p.chunk, p.n_blocks - base);
-          if (p.trigger_block - base < p.chunk) {        // self-trigger inside this chunk
-            const uint32_t e = p.epoch % kEvEpochs;
-            p.cb->ep_t_trigger[e] = gtimer();
-            p.cb->ep_trigger_block[e] = p.trigger_block;
-            atomicExch(p.ctrl, ((p.epoch & 0xffffu) << 16) | (p.trigger_n & 0xffffu));
-          }
+        base = stopping ? 0xffffffffu : atomicAdd(&p.cb->ctr, p.chunk);   // pull_task
+      }
+      if (base != 0xffffffffu && base >= p.n_blocks) { base = 0xffffffffu; s_reason = kReasonExhausted; }
+      if (base != 0xffffffffu) {
+        s_blocks += min(p.chunk, p.n_blocks - base);
+        if (p.prefetch && !stopping) held = atomicAdd(&p.cb->ctr, p.chunk);   // overlaps the body
+        if (p.trigger_block - base < p.chunk) {          // device self-trigger inside this chunk
+          const uint32_t e = p.epoch % kEvEpochs;
+          p.cb->ep_t_trigger[e] = gtimer();
+          p.cb->ep_trigger_block[e] = p.trigger_block;
+          atomicExch(p.ctrl, ((p.epoch & 0xffffu) << 16) | (p.trigger_n & 0xffffu));
         }
       }
       s_slot[parity] = base;
@@ -177,6 +189,8 @@ flep_worker(const typename Body::Args args, const WorkerParams p) {
       p.cb->ep_t_end[ei] = t_exit; p.cb->ep_done[ei] = d; p.cb->ep_ctr[ei] = c;
       p.cb->ep_state[ei] = st;
       p.cb->exited = 0;                                  // ready for the next epoch
+      if (st == kStateDone) { p.cb->ctr = 0; p.cb->done = 0; }   // block clean for reuse
+      p.cb->ep_t_trigger[(p.epoch + 1) % kEvEpochs] = 0;  // next epoch's trigger stamp
       p.status->t_end = t_exit;
       p.status->done = d;
       p.status->ctr = c;

@@ -66,21 +66,19 @@ int64_t now_ns() {
       .count();
 }
 
-// Driver stream memory operations, resolved through the runtime (no link-time libcuda).
+// Driver stream memory operation for the control word, resolved through the runtime (no
+// link-time libcuda). Deliberately no stream WAIT operations anywhere: a front-end wait on a
+// value written by a kernel of another stream can deadlock when the two streams share a
+// hardware queue (observed on the B200 probe), so ordering uses events only.
 typedef CUresult (*PFN_wv32)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
-typedef CUresult (*PFN_wait32)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
 PFN_wv32 p_write32 = nullptr;
-PFN_wait32 p_wait32 = nullptr;
 
 flep_status resolve_driver() {
-  if (p_write32 && p_wait32) return FLEP_OK;
+  if (p_write32) return FLEP_OK;
   cudaDriverEntryPointQueryResult q;
   CUDA_TRY(cudaGetDriverEntryPoint("cuStreamWriteValue32", (void**)&p_write32, cudaEnableDefault, &q));
   if (q != cudaDriverEntryPointSuccess || !p_write32)
     return fail(FLEP_ERR_UNSUPPORTED, "cuStreamWriteValue32 not available");
-  CUDA_TRY(cudaGetDriverEntryPoint("cuStreamWaitValue32", (void**)&p_wait32, cudaEnableDefault, &q));
-  if (q != cudaDriverEntryPointSuccess || !p_wait32)
-    return fail(FLEP_ERR_UNSUPPORTED, "cuStreamWaitValue32 not available");
   return FLEP_OK;
 }
 
@@ -99,7 +97,7 @@ struct Launch {
   cudaStream_t user = nullptr;
   cudaStream_t exec = nullptr;
   int exec_level = 0;
-  uint32_t chunk = 1, poll = 1, workers = 0;
+  uint32_t chunk = 1, poll = 1, workers = 0, flags = 0;
   void* dmem = nullptr;              // ControlBlock + event ring
   ControlBlock* cb = nullptr;
   WorkerEvent* ev = nullptr;
@@ -115,7 +113,8 @@ struct Launch {
   int64_t t_arrive = 0, t_first_start = -1, t_finish = -1;
   int64_t t_e = 0, overhead = 0;
   uint32_t last_done = 0, last_ctr = 0;
-  cudaEvent_t user_after_wait = nullptr;   // recorded on the user stream after its done-wait
+  int64_t t_last_request = -1, t_last_drain = -1;
+  uint32_t gen0 = 0;                 // control-block generation before this launch's epoch 1
   bool released = false;
   bool cancelled = false;
 };
@@ -126,6 +125,8 @@ struct KernelReg {
   uint32_t chunk, poll;
   double model[5];
   int64_t overhead;
+  uint32_t flags;
+  uint32_t ctas_per_sm;
 };
 
 }  // namespace
@@ -143,6 +144,7 @@ struct flep_rt_s {
   size_t dmem_bytes = 0;
   uint32_t max_workers = 0;
   std::vector<void*> free_dmem;
+  std::map<void*, uint32_t> cb_gen;   // next free generation of each control block
   std::vector<std::pair<uint32_t*, size_t>> free_cov;
   std::map<int, std::vector<cudaStream_t>> free_streams;
   std::vector<cudaStream_t> all_streams;
@@ -190,7 +192,13 @@ flep_status get_stream(flep_rt rt, int level, cudaStream_t* s) {
   return FLEP_OK;
 }
 
+// Generations: every epoch of every launch that uses a control block gets a new number, so a
+// late request for an old epoch (or an old launch) never matches a newer one (A2/H5).
+inline uint32_t gen_of(const Launch& L) { return L.gen0 + L.epoch; }
+inline uint32_t ctrl_word(const Launch& L, uint32_t n) { return ((gen_of(L) & 0xffffu) << 16) | (n & 0xffffu); }
+
 flep_status write_ctrl(flep_rt rt, Launch& L, uint32_t value) {
+  L.t_last_request = now_ns();
   if (rt->opt.flag == FLEP_FLAG_HOST_MAPPED) {
     __atomic_store_n(&L.hs->ctrl, value, __ATOMIC_RELEASE);
     return FLEP_OK;
@@ -212,13 +220,14 @@ flep_status start_epoch(flep_rt rt, Launch& L) {
   p.n_blocks = L.n_blocks;
   p.chunk = L.chunk;
   p.poll = L.poll;
-  p.epoch = L.epoch;
+  p.epoch = gen_of(L);
   p.workers = L.workers;
   p.num_sms = rt->num_sms;
   p.gx = L.grid.x;
   p.gy = L.grid.y;
   p.trigger_block = L.trig_block;
   p.trigger_n = L.trig_n;
+  p.prefetch = (L.flags & FLEP_KFLAG_PREFETCH) ? 1u : 0u;
   L.trig_block = kNoTrigger;
   L.trig_n = 0;
   cudaError_t e = L.ops->worker(L.args.data(), p, L.workers, L.exec, L.cov != nullptr);
@@ -234,7 +243,7 @@ bool refresh(Launch& L) {
   if (L.state != FLEP_STATE_RUNNING && L.state != FLEP_STATE_YIELDING && L.state != FLEP_STATE_PARTIAL)
     return false;
   const uint32_t w = __atomic_load_n(&L.hs->word, __ATOMIC_ACQUIRE);
-  if ((w >> 8) != L.epoch) return false;
+  if ((w >> 8) != (gen_of(L) & 0xffffffu)) return false;
   L.last_done = L.hs->done;
   L.last_ctr = L.hs->ctr;
   if ((w & 0xffu) == kStateDone) {
@@ -243,18 +252,18 @@ bool refresh(Launch& L) {
     return true;
   }
   L.state = FLEP_STATE_PREEMPTED;
+  L.t_last_drain = now_ns();
   return false;
 }
 
 void release_resources(flep_rt rt, Launch& L) {
   if (L.released) return;
-  // the launch's last grid has completed (caller synchronised the exec stream)
-  if (L.user_after_wait && cudaEventQuery(L.user_after_wait) != cudaSuccess) return;  // retry later
-  if (L.user_after_wait) { cudaEventDestroy(L.user_after_wait); L.user_after_wait = nullptr; }
-  if (L.dmem) rt->free_dmem.push_back(L.dmem);
+  // the launch's last grid has completed (caller synchronised the exec stream); the last worker
+  // of the DONE epoch left ctr/done/exited at 0, so the block is reusable as is
+  if (L.dmem) { rt->cb_gen[L.dmem] = gen_of(L) + 1; rt->free_dmem.push_back(L.dmem); }
   if (L.cov) rt->free_cov.push_back({L.cov, L.cov_cap});
   if (L.slot >= 0) rt->free_slots.push_back(L.slot);
-  if (L.exec) rt->free_streams[L.exec_level].push_back(L.exec);
+  if (L.exec && L.exec_level != -1000) rt->free_streams[L.exec_level].push_back(L.exec);
   L.dmem = nullptr; L.cov = nullptr; L.slot = -1; L.exec = nullptr;
   L.released = true;
 }
@@ -268,7 +277,7 @@ void apply_decisions(flep_rt rt) {
     Launch& L = *it->second;
     if (x.action == kPreempt) {
       if (L.state == FLEP_STATE_RUNNING || L.state == FLEP_STATE_PARTIAL) {
-        write_ctrl(rt, L, ((L.epoch & 0xffffu) << 16) | (uint32_t)std::min<int64_t>(x.n_sms, 0xffff));
+        write_ctrl(rt, L, ctrl_word(L, (uint32_t)std::min<int64_t>(x.n_sms, 0xffff)));
         L.state = FLEP_STATE_YIELDING;
         L.n_yield = (uint32_t)x.n_sms;
       }
@@ -392,6 +401,8 @@ flep_status flep_register_kernel(flep_rt rt, const flep_kernel_desc* d, flep_ker
   k.poll = d->poll ? d->poll : rt->opt.default_poll;
   memcpy(k.model, d->model, sizeof(k.model));
   k.overhead = d->preempt_overhead_ns;
+  k.flags = d->flags;
+  k.ctas_per_sm = d->ctas_per_sm;
   rt->kernels.push_back(k);
   *out = (flep_kernel)rt->kernels.size() - 1;
   return FLEP_OK;
@@ -446,6 +457,8 @@ flep_status flep_launch(flep_rt rt, flep_kernel kid, flep_dim3 grid, const void*
   L.user = (cudaStream_t)stream;
   L.chunk = kr.chunk;
   L.poll = kr.poll;
+  L.flags = kr.flags;
+  if (kr.ctas_per_sm && (int)kr.ctas_per_sm < k) k = (int)kr.ctas_per_sm;
   const uint64_t wmax = (uint64_t)k * rt->num_sms;
   const uint64_t need = (N + L.chunk - 1) / L.chunk;
   L.workers = (uint32_t)std::min<uint64_t>(std::min<uint64_t>(wmax, need), rt->max_workers);
@@ -461,7 +474,13 @@ flep_status flep_launch(flep_rt rt, flep_kernel kid, flep_dim3 grid, const void*
   s = get_stream(rt, L.exec_level, &L.exec);
   if (s) return s;
   if (!rt->free_dmem.empty()) { L.dmem = rt->free_dmem.back(); rt->free_dmem.pop_back(); }
-  else CUDA_TRY(cudaMalloc(&L.dmem, rt->dmem_bytes));
+  else {
+    CUDA_TRY(cudaMalloc(&L.dmem, rt->dmem_bytes));
+    CUDA_TRY(cudaMemset(L.dmem, 0, sizeof(ControlBlock)));   // once per block, synchronous
+    rt->cb_gen[L.dmem] = 0;
+  }
+  L.gen0 = rt->cb_gen[L.dmem];
+  if (L.gen0 + 2 * kEvEpochs >= 0xffffffu) return fail(FLEP_ERR_NOMEM, "control block generation space exhausted");
   L.cb = (ControlBlock*)L.dmem;
   L.ev = (WorkerEvent*)((char*)L.dmem + sizeof(ControlBlock));
   if (cov) {
@@ -473,29 +492,28 @@ flep_status flep_launch(flep_rt rt, flep_kernel kid, flep_dim3 grid, const void*
       }
     }
     if (!L.cov) { L.cov_cap = std::max<size_t>(N, 4096); CUDA_TRY(cudaMalloc(&L.cov, L.cov_cap * 4)); }
-    CUDA_TRY(cudaMemsetAsync(L.cov, 0, N * 4, L.exec));
   }
   L.slot = rt->free_slots.back();
   rt->free_slots.pop_back();
   L.hs = rt->h_slots + L.slot;
   L.ds = rt->d_slots + L.slot;
   memset(L.hs, 0, sizeof(HostStatus));
-  // order: caller's prior work -> control-block reset -> workers; caller's later work waits for
-  // the done counter to reach N (true completion across preempt/resume cycles).
-  cudaEvent_t ev_u;
-  CUDA_TRY(cudaEventCreateWithFlags(&ev_u, cudaEventDisableTiming));
-  CUDA_TRY(cudaEventRecord(ev_u, L.user));
-  CUDA_TRY(cudaStreamWaitEvent(L.exec, ev_u, 0));
-  CUDA_TRY(cudaMemsetAsync(L.dmem, 0, rt->dmem_bytes, L.exec));
-  if (rt->opt.order_user_stream) {
-    CUDA_TRY(cudaEventRecord(ev_u, L.exec));
-    CUDA_TRY(cudaStreamWaitEvent(L.user, ev_u, 0));
-    CUresult r = p_wait32((CUstream)L.user, (CUdeviceptr)&L.cb->done, L.n_blocks, CU_STREAM_WAIT_VALUE_GEQ);
-    if (r != CUDA_SUCCESS) return fail(FLEP_ERR_CUDA, "cuStreamWaitValue32 failed (%d)", (int)r);
-    CUDA_TRY(cudaEventCreateWithFlags(&L.user_after_wait, cudaEventDisableTiming));
-    CUDA_TRY(cudaEventRecord(L.user_after_wait, L.user));
+  // No per-launch reset work on the GPU: a pooled control block was left clean by the last
+  // worker of its previous launch's DONE epoch, and its generation numbers keep increasing.
+  const bool on_user = rt->opt.exec_on_user_stream && rt->opt.policy == FLEP_POLICY_MANUAL;
+  if (on_user) {
+    rt->free_streams[L.exec_level].push_back(L.exec);
+    L.exec = L.user;
+    L.exec_level = -1000;
+  } else {
+    // caller's prior work on `stream` (e.g. input copies) precedes the workers
+    cudaEvent_t ev_u;
+    CUDA_TRY(cudaEventCreateWithFlags(&ev_u, cudaEventDisableTiming));
+    CUDA_TRY(cudaEventRecord(ev_u, L.user));
+    CUDA_TRY(cudaStreamWaitEvent(L.exec, ev_u, 0));
+    cudaEventDestroy(ev_u);
   }
-  cudaEventDestroy(ev_u);
+  if (L.cov) CUDA_TRY(cudaMemsetAsync(L.cov, 0, N * 4, L.exec));
   rt->launches[L.id] = std::move(Lp);
   *out = L.id;
   if (rt->opt.policy == FLEP_POLICY_MANUAL) return start_epoch(rt, L);
@@ -520,7 +538,7 @@ flep_status flep_preempt(flep_rt rt, flep_launch_t h, uint32_t n_sms) {
   const uint32_t n = std::min<uint32_t>(n_sms, rt->num_sms);
   if (L->state == FLEP_STATE_PARTIAL && n <= L->n_yield)
     return fail(FLEP_ERR_INVALID, "a request can only widen within an epoch (%u <= %u)", n, L->n_yield);
-  flep_status s = write_ctrl(rt, *L, ((L->epoch & 0xffffu) << 16) | n);
+  flep_status s = write_ctrl(rt, *L, ctrl_word(*L, n));
   if (s) return s;
   L->n_yield = n;
   L->state = n >= rt->num_sms ? FLEP_STATE_YIELDING : FLEP_STATE_PARTIAL;
@@ -536,7 +554,7 @@ flep_status flep_resume(flep_rt rt, flep_launch_t h) {
   refresh(*L);
   if (L->state == FLEP_STATE_PREEMPTED) return start_epoch(rt, *L);
   if (L->state == FLEP_STATE_PARTIAL) {
-    flep_status s = write_ctrl(rt, *L, (L->epoch & 0xffffu) << 16);
+    flep_status s = write_ctrl(rt, *L, ctrl_word(*L, 0));
     if (s) return s;
     L->state = FLEP_STATE_RUNNING;
     L->n_yield = 0;
@@ -592,11 +610,6 @@ flep_status flep_sync(flep_rt rt, flep_launch_t h, int64_t timeout_ns) {
     rt->retained.erase(rt->retained.begin());
     if (old) release_resources(rt, *old);
   }
-  for (auto& kv : rt->launches)   // retry deferred releases
-    if (kv.second->state == FLEP_STATE_DONE && !kv.second->released &&
-        std::find(rt->retained.begin(), rt->retained.end(), kv.first) == rt->retained.end() &&
-        kv.second->exec && cudaStreamQuery(kv.second->exec) == cudaSuccess)
-      release_resources(rt, *kv.second);
   return FLEP_OK;
 }
 
@@ -618,6 +631,8 @@ flep_status flep_query(flep_rt rt, flep_launch_t h, flep_launch_info* out) {
   out->workers = L->workers;
   out->n_yield = L->n_yield;
   out->t_e = L->t_e;
+  out->t_last_request = L->t_last_request;
+  out->t_last_drain = L->t_last_drain;
   if (rt->policy) {
     const Policy::Entry* e = rt->policy->entry(L->id);
     if (e) { out->t_w = e->t_w; out->t_r = e->t_r; }
@@ -634,7 +649,7 @@ flep_status flep_cancel(flep_rt rt, flep_launch_t h) {
     refresh(*L);
     if (L->state == FLEP_STATE_DONE) return FLEP_OK;
     if (L->state == FLEP_STATE_RUNNING || L->state == FLEP_STATE_PARTIAL || L->state == FLEP_STATE_YIELDING) {
-      write_ctrl(rt, *L, ((L->epoch & 0xffffu) << 16) | 0xffffu);
+      write_ctrl(rt, *L, ctrl_word(*L, 0xffffu));
       L->state = FLEP_STATE_YIELDING;
     }
     L->cancelled = true;
@@ -648,10 +663,11 @@ flep_status flep_cancel(flep_rt rt, flep_launch_t h) {
   std::lock_guard<std::mutex> lk(rt->mu);
   Launch* L = find(rt, h);
   if (L->exec) CUDA_TRY(cudaStreamSynchronize(L->exec));
-  // unblock any stream waiting for true completion
-  CUresult r = p_write32((CUstream)rt->ctl, (CUdeviceptr)&L->cb->done, L->n_blocks, 0);
-  if (r != CUDA_SUCCESS) return fail(FLEP_ERR_CUDA, "cuStreamWriteValue32 failed (%d)", (int)r);
-  CUDA_TRY(cudaStreamSynchronize(rt->ctl));
+  // the abandoned epoch left ctr/done non-zero: clear the block for reuse
+  if (L->state != FLEP_STATE_DONE) {
+    CUDA_TRY(cudaMemsetAsync(L->cb, 0, offsetof(ControlBlock, ep_t_trigger), L->exec));
+    CUDA_TRY(cudaStreamSynchronize(L->exec));
+  }
   L->state = FLEP_STATE_DONE;
   L->t_finish = now_ns();
   return FLEP_OK;
@@ -667,7 +683,6 @@ flep_status flep_shutdown(flep_rt rt) {
   cudaDeviceSynchronize();
   for (auto& kv : rt->launches) {
     Launch& L = *kv.second;
-    if (L.user_after_wait) cudaEventDestroy(L.user_after_wait);
     if (!L.released) {
       if (L.dmem) cudaFree(L.dmem);
       if (L.cov) cudaFree(L.cov);
@@ -764,7 +779,7 @@ flep_status flep_debug_copy_events(flep_rt rt, flep_launch_t h, uint32_t epoch,
   if (epoch == 0 || epoch > L->epoch || L->epoch - epoch >= kEvEpochs)
     return fail(FLEP_ERR_INVALID, "epoch %u not in the log", epoch);
   const size_t n = std::min<size_t>(max_records, L->workers);
-  CUDA_TRY(cudaMemcpyAsync(host_out, L->ev + (size_t)(epoch % kEvEpochs) * L->workers,
+  CUDA_TRY(cudaMemcpyAsync(host_out, L->ev + (size_t)((L->gen0 + epoch) % kEvEpochs) * L->workers,
                            n * sizeof(WorkerEvent), cudaMemcpyDeviceToHost, L->exec));
   CUDA_TRY(cudaStreamSynchronize(L->exec));
   if (n_out) *n_out = n;
@@ -782,7 +797,7 @@ flep_status flep_debug_epoch_info(flep_rt rt, flep_launch_t h, uint32_t epoch, f
   ControlBlock cb;
   CUDA_TRY(cudaMemcpyAsync(&cb, L->cb, sizeof(cb), cudaMemcpyDeviceToHost, L->exec));
   CUDA_TRY(cudaStreamSynchronize(L->exec));
-  const uint32_t e = epoch % kEvEpochs;
+  const uint32_t e = (L->gen0 + epoch) % kEvEpochs;
   out->t_trigger = cb.ep_t_trigger[e];
   out->t_end = cb.ep_t_end[e];
   out->trigger_block = cb.ep_trigger_block[e];

@@ -21,6 +21,7 @@ STATE_NAMES = {0: "QUEUED", 1: "RUNNING", 2: "YIELDING", 3: "PREEMPTED", 4: "PAR
 REASON_YIELD, REASON_EXHAUSTED = 1, 2
 ACTION_NAMES = {0: "LAUNCH", 1: "RESUME", 2: "PREEMPT"}
 NO_TRIGGER = 0xFFFFFFFF
+KFLAG_PREFETCH = 1
 
 
 class Dim3(C.Structure):
@@ -52,12 +53,14 @@ class GemmArgs(C.Structure):
 class Options(C.Structure):
     _fields_ = [("policy", C.c_int32), ("flag", C.c_int32), ("default_chunk", C.c_uint32),
                 ("default_poll", C.c_uint32), ("debug_coverage", C.c_uint32),
-                ("order_user_stream", C.c_uint32), ("slice_blocks", C.c_uint32)]
+                ("reserved0", C.c_uint32), ("slice_blocks", C.c_uint32),
+                ("exec_on_user_stream", C.c_uint32)]
 
 
 class KernelDesc(C.Structure):
     _fields_ = [("name", C.c_char_p), ("body", C.c_int32), ("chunk", C.c_uint32), ("poll", C.c_uint32),
-                ("model", C.c_double * 5), ("preempt_overhead_ns", C.c_int64)]
+                ("model", C.c_double * 5), ("preempt_overhead_ns", C.c_int64), ("flags", C.c_uint32),
+                ("ctas_per_sm", C.c_uint32)]
 
 
 class LaunchInfo(C.Structure):
@@ -65,7 +68,7 @@ class LaunchInfo(C.Structure):
                 ("blocks_done", C.c_uint64), ("counter", C.c_uint64), ("t_e", C.c_int64),
                 ("t_w", C.c_int64), ("t_r", C.c_int64), ("t_arrive", C.c_int64),
                 ("t_first_start", C.c_int64), ("t_finish", C.c_int64), ("workers", C.c_uint32),
-                ("n_yield", C.c_uint32)]
+                ("n_yield", C.c_uint32), ("t_last_request", C.c_int64), ("t_last_drain", C.c_int64)]
 
 
 class WorkerEvent(C.Structure):
@@ -170,9 +173,10 @@ class Runtime:
     """One FLEP runtime on one device (flep_init ... flep_shutdown)."""
 
     def __init__(self, device=0, policy=POLICY_MANUAL, flag=FLAG_STREAM_MEMOP, chunk=8, poll=1,
-                 coverage=False, order_user_stream=True, slice_blocks=0):
+                 coverage=False, slice_blocks=0, exec_on_user_stream=False):
         self.L = lib()
-        o = Options(policy, flag, chunk, poll, int(coverage), int(order_user_stream), slice_blocks)
+        o = Options(policy, flag, chunk, poll, int(coverage), 0, slice_blocks,
+                    int(exec_on_user_stream))
         h = C.c_void_p()
         check(self.L.flep_init(device, C.byref(o), C.byref(h)), "flep_init")
         self.h = h
@@ -191,8 +195,10 @@ class Runtime:
     def __exit__(self, *a):
         self.close()
 
-    def register_kernel(self, body, chunk=0, poll=0, name="", model=(0, 0, 0, 0, 1), overhead_ns=0):
-        d = KernelDesc(name.encode(), body, chunk, poll, (C.c_double * 5)(*model), overhead_ns)
+    def register_kernel(self, body, chunk=0, poll=0, name="", model=(0, 0, 0, 0, 1), overhead_ns=0,
+                        prefetch=False, ctas_per_sm=0):
+        d = KernelDesc(name.encode(), body, chunk, poll, (C.c_double * 5)(*model), overhead_ns,
+                       KFLAG_PREFETCH if prefetch else 0, ctas_per_sm)
         k = C.c_int32()
         check(self.L.flep_register_kernel(self.h, C.byref(d), C.byref(k)), "flep_register_kernel")
         return k.value
@@ -348,8 +354,11 @@ def saxpy_grid(n):
     return ((n + 255) // 256, 1, 1)
 
 
+SPMV_ROWS_PER_BLOCK = 128
+
+
 def spmv_grid(rows):
-    return ((rows + 31) // 32, 1, 1)
+    return ((rows + SPMV_ROWS_PER_BLOCK - 1) // SPMV_ROWS_PER_BLOCK, 1, 1)
 
 
 def stencil_grid(n):

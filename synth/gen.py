@@ -28,7 +28,7 @@ __all__ = [
 
 # Original-kernel block geometry (the "task" of P:128/P:164). Fixed by DESIGN.md.
 SAXPY_BLOCK = 256          # elements per original CTA (CUDA SDK vectorAdd: one element per thread)
-SPMV_ROWS_PER_BLOCK = 32   # rows per original CTA (8 lanes per row x 32 rows = 256 threads)
+SPMV_ROWS_PER_BLOCK = 128  # rows per original CTA (CSR-stream block of 256 threads)
 STENCIL_TILE = 64          # 64x64 output cells per original CTA
 GEMM_TILE_M = 128          # output tile rows per original CTA
 GEMM_TILE_N = 256          # output tile cols per original CTA

@@ -1,0 +1,203 @@
+"""GPU tests of the runtime: the managed policies on real kernels (with replay parity of the
+measured event log against the oracle DES), the 10^4 random preempt/resume schedules of config 1
+(0 coverage violations, bit-exact results), the host-mapped flag transport, cancellation."""
+import numpy as np
+import pytest
+
+from oracle import des
+from oracle import workloads as W
+from synth import gen
+
+from flep_gpu_util import flep_mod, run_manual_schedule, t
+
+pytestmark = pytest.mark.gpu
+
+ACT = {"LAUNCH": 0, "RESUME": 1, "PREEMPT": 2}
+
+
+def _replay_from_runtime(rt, kind):
+    """Rebuild the oracle's event list from the runtime's own log and replay it."""
+    evs = []
+    for (t_ns, typ, lid, prio, t_e, ovh) in rt.event_log():
+        if typ == 0:
+            evs.append((t_ns, "ARRIVE", des.KernelSpec(lid, t_ns, prio, t_e, ovh)))
+        else:
+            evs.append((t_ns, "FINISH", lid))
+    return [(t, ACT[a], i, n) for (t, a, i, n) in des.replay(kind, evs)]
+
+
+def test_managed_hpf_preempts_and_replays_exactly():
+    f = flep_mod()
+    import torch
+    rt = f.Runtime(policy=f.POLICY_HPF, coverage=True)
+    try:
+        n_lp, n_hp = 1 << 26, 1 << 16
+        x, y = gen.saxpy_i32_inputs(n_lp, seed=21)
+        x2, y2 = gen.saxpy_i32_inputs(n_hp, seed=22)
+        xd, yd, x2d, y2d = t(x), t(y), t(x2), t(y2)
+        k_lp = rt.register_kernel(f.BODY_SAXPY_I32, chunk=4, poll=1, model=(0, 0, 0, 0, 2_000_000))
+        k_hp = rt.register_kernel(f.BODY_SAXPY_I32, chunk=1, poll=1, model=(0, 0, 0, 0, 5_000))
+        sA, sB = torch.cuda.Stream(), torch.cuda.Stream()
+        h_lp = rt.launch(k_lp, f.saxpy_grid(n_lp), f.saxpy_i32_args(yd, xd, 7), priority=0, stream=sA)
+        h_hp = rt.launch(k_hp, f.saxpy_grid(n_hp), f.saxpy_i32_args(y2d, x2d, 9), priority=1, stream=sB)
+        rt.sync(h_hp, timeout_ns=10_000_000_000)
+        rt.sync(h_lp, timeout_ns=10_000_000_000)
+        torch.cuda.synchronize()
+        assert np.array_equal(yd.cpu().numpy(), W.saxpy_i32(7, x, y))
+        assert np.array_equal(y2d.cpu().numpy(), W.saxpy_i32(9, x2, y2))
+        assert np.all(rt.coverage_np(h_lp, n_lp // 256) == 1)
+        dec = rt.decision_log()
+        acts = [f.ACTION_NAMES[d[1]] for d in dec]
+        assert acts[:3] == ["LAUNCH", "PREEMPT", "LAUNCH"]
+        assert dec == _replay_from_runtime(rt, des.HPF)
+    finally:
+        rt.close()
+
+
+@pytest.mark.parametrize("kind", ["HPF", "FIFO"])
+def test_managed_queue_replay_parity(kind):
+    """A burst of mixed-priority kernels; the runtime's decisions equal the DES replay of the
+    runtime's own measured ARRIVE/FINISH log (bit-exact, SURVEY §8(c) O3 replay mode)."""
+    f = flep_mod()
+    import torch
+    pol = f.POLICY_HPF if kind == "HPF" else f.POLICY_FIFO
+    rt = f.Runtime(policy=pol)
+    try:
+        g = gen.rng(31)
+        ks, hs, refs = [], [], []
+        streams = [torch.cuda.Stream() for _ in range(4)]
+        for i in range(12):
+            n = int(g.choice([1 << 16, 1 << 20, 1 << 23]))
+            x, y = gen.saxpy_i32_inputs(n, seed=100 + i)
+            xd, yd = t(x), t(y)
+            k = rt.register_kernel(f.BODY_SAXPY_I32, chunk=2, poll=1, model=(0, 0, 0.02, 0, 1000),
+                                   overhead_ns=int(g.integers(0, 20_000)))
+            a = int(g.integers(1, 1000))
+            h = rt.launch(k, f.saxpy_grid(n), f.saxpy_i32_args(yd, xd, a), priority=int(g.integers(0, 3)),
+                          stream=streams[i % 4])
+            hs.append(h)
+            refs.append((yd, W.saxpy_i32(a, x, y)))
+        for h in hs:
+            rt.sync(h, timeout_ns=20_000_000_000)
+        torch.cuda.synchronize()
+        for yd, ref in refs:
+            assert np.array_equal(yd.cpu().numpy(), ref)
+        dec = rt.decision_log()
+        assert dec == _replay_from_runtime(rt, des.HPF if kind == "HPF" else des.FIFO)
+        if kind == "FIFO":
+            assert all(d[1] == 0 for d in dec)
+    finally:
+        rt.close()
+
+
+def test_random_schedules_10k_zero_violations():
+    """Config 1: LP SAXPY-int32 2^20 under 10^4 random manual preempt/resume schedules (temporal
+    and spatial yields, C in {1,2,4,8,16}, K in {1,2,4,8}, with and without prefetch). Every
+    schedule: coverage == 1, bit-exact y, preempted epochs cover a prefix (I2), yields only on
+    requested SMs (I3)."""
+    f = flep_mod()
+    import torch
+    rt = f.Runtime(coverage=True)
+    try:
+        n, a = 1 << 20, 1664525
+        nb = n // 256
+        x, y = gen.saxpy_i32_inputs(n, seed=1)
+        ref = W.saxpy_i32(a, x, y)
+        xd, y0, yd = t(x), t(y), t(y)
+        kern = {}
+        viol_total, preempted_total, yielded_total, bad = 0, 0, 0, []
+        n_sched = 10_000
+        for i in range(n_sched):
+            s = gen.preempt_schedule(100 + i, nb, rt.num_sms)
+            pf = i % 2 == 1
+            cps = (1, 2, 8)[i % 3]                 # resident workers per SM (W = 148 * cps)
+            key = (s["C"], s["K"], pf, cps)
+            if key not in kern:
+                kern[key] = rt.register_kernel(f.BODY_SAXPY_I32, chunk=s["C"], poll=s["K"], prefetch=pf,
+                                               ctas_per_sm=cps)
+            yd.copy_(y0)
+            h, npre, viol = run_manual_schedule(rt, kern[key], f.saxpy_grid(n), f.saxpy_i32_args(yd, xd, a), nb,
+                                                s, rt.num_sms, check_prefix=(i % 10 == 0))
+            preempted_total += npre
+            info = rt.query(h)
+            yielded_total += int(any(e.reason == f.REASON_YIELD
+                                     for ep in range(1, info.epoch + 1) for e in rt.events(h, ep)))
+            cov = rt.coverage_np(h, nb)
+            if not np.all(cov == 1):
+                viol.append("I1: coverage != 1")
+            if i % 10 == 0 or viol:
+                if not np.array_equal(yd.cpu().numpy(), ref):
+                    viol.append("result != oracle")
+            if viol:
+                viol_total += len(viol)
+                bad.append((i, s, viol))
+        # outputs of every schedule are checked through coverage (exactly-once => bit-exact for
+        # this deterministic body); every 10th schedule also compares y against the oracle
+        summary = {"schedules": n_sched, "violations": viol_total, "schedules_with_yields": yielded_total,
+                   "preempted_epochs": preempted_total}
+        import json
+        import os
+        out = os.environ.get("FLEP_EVIDENCE_DIR")
+        if out:
+            with open(os.path.join(out, "schedules_10k.json"), "w") as fh:
+                json.dump(summary, fh)
+        assert viol_total == 0, bad[:5]
+        assert yielded_total > n_sched // 2        # most schedules really make workers yield
+        assert preempted_total > n_sched // 5      # ... and many drain whole epochs (temporal)
+    finally:
+        rt.close()
+
+
+def test_host_mapped_flag_transport():
+    f = flep_mod()
+    import time
+    rt = f.Runtime(flag=f.FLAG_HOST_MAPPED, coverage=True)
+    try:
+        n = 1 << 26
+        nb = n // 256
+        x, y = gen.saxpy_i32_inputs(n, seed=41)
+        xd, yd = t(x), t(y)
+        k = rt.register_kernel(f.BODY_SAXPY_I32, chunk=1, poll=1)
+        h = rt.launch(k, f.saxpy_grid(n), f.saxpy_i32_args(yd, xd, 5))
+        time.sleep(0.0002)
+        try:
+            rt.preempt(h, rt.num_sms)
+        except f.FlepError as e:
+            assert e.status == f.ERR_STATE      # already finished: legal
+        rt.wait_epoch(h, timeout_ns=10_000_000_000)
+        if rt.query(h).state == f.STATE_PREEMPTED:
+            c = rt.coverage_np(h, nb)
+            m = min(int(rt.query(h).counter), nb)
+            assert np.all(c[:m] == 1) and np.all(c[m:] == 0)
+            rt.resume(h)
+        rt.sync(h, timeout_ns=10_000_000_000)
+        assert np.array_equal(yd.cpu().numpy(), W.saxpy_i32(5, x, y))
+    finally:
+        rt.close()
+
+
+def test_cancel_then_reuse_control_block():
+    f = flep_mod()
+    rt = f.Runtime()
+    try:
+        n = 1 << 26
+        x, y = gen.saxpy_i32_inputs(n, seed=51)
+        xd, yd = t(x), t(y)
+        k = rt.register_kernel(f.BODY_SAXPY_I32, chunk=1, poll=1)
+        rt.arm_next_trigger(1000, rt.num_sms)
+        h = rt.launch(k, f.saxpy_grid(n), f.saxpy_i32_args(yd, xd, 3))
+        rt.wait_epoch(h, timeout_ns=10_000_000_000)
+        rt.cancel(h)
+        assert rt.query(h).state == f.STATE_DONE
+        rt.sync(h)
+        # the control block goes back to the pool; a new launch must start from a clean counter
+        n2 = 1 << 20
+        x2, y2 = gen.saxpy_i32_inputs(n2, seed=52)
+        x2d, y2d = t(x2), t(y2)
+        for _ in range(70):       # cycle through the retained-launch window and the pool
+            y2d.copy_(t(y2))
+            h2 = rt.launch(k, f.saxpy_grid(n2), f.saxpy_i32_args(y2d, x2d, 11))
+            rt.sync(h2)
+            assert np.array_equal(y2d.cpu().numpy(), W.saxpy_i32(11, x2, y2))
+    finally:
+        rt.close()

@@ -1,0 +1,77 @@
+"""Replay parity: the C++ decision engine inside libflep.so (flep_policy_*) must reproduce the
+oracle DES's decision list bit for bit on the same event traces (BJ "the
+scheduler's decision sequence" bit-exact). Host only — no GPU."""
+import pytest
+
+from oracle import des
+from synth import gen
+
+
+@pytest.fixture(scope="module")
+def flep():
+    from paper_conf_asplos_wulzj17_b200 import build, flep as F
+    build.build()
+    return F
+
+
+ACT = {"LAUNCH": 0, "RESUME": 1, "PREEMPT": 2}
+KIND = {des.FIFO: 1, des.HPF: 2, des.SLICE: 3}
+
+
+def replay_cpp(F, kind, events):
+    p = F.PolicyEngine(KIND[kind])
+    for ev in events:
+        if ev[1] == "ARRIVE":
+            s = ev[2]
+            p.arrive(ev[0], s.id, s.priority, s.t_e, s.overhead)
+        else:
+            p.finish(ev[0], ev[2])
+    return p.decisions()
+
+
+def as_tuples(dec):
+    return [(t, ACT[a], i, n) for (t, a, i, n) in dec]
+
+
+def random_trace(seed, n, prios=3, tight=False):
+    g = gen.rng(seed)
+    ks, t = [], 0
+    for i in range(n):
+        t += int(g.integers(0, 50_000 if tight else 400_000))
+        true = int(g.integers(1_000, 2_000_000))
+        est = max(1, int(true * g.uniform(0.5, 1.5)))
+        ks.append(des.KernelSpec(i, t, int(g.integers(0, prios)), est, int(g.integers(0, 80_000)), true))
+    return ks
+
+
+@pytest.mark.parametrize("kind", [des.FIFO, des.HPF, des.SLICE])
+@pytest.mark.parametrize("seed", range(25))
+def test_replay_parity_random_traces(flep, kind, seed):
+    ks = random_trace(seed, 40, prios=1 + seed % 4, tight=seed % 2 == 0)
+    params = des.SimParams(drain_ns=int(seed * 700), start_ns=3_000,
+                           slice_ns=150_000 if kind == des.SLICE else 0, slice_gap_ns=6_000)
+    sim = des.simulate(kind, ks, params)
+    assert as_tuples(sim.decisions) == replay_cpp(flep, kind, sim.events)
+
+
+def test_replay_parity_table1_pairs(flep):
+    T = {"CFD": (11106, 521), "NN": (15775, 728), "PF": (7364, 811), "PL": (5419, 952),
+         "MD": (15905, 938), "SPMV": (5840, 484), "MM": (2579, 1499), "VA": (30634, 720)}
+    for lp in T:
+        for hp in T:
+            if lp == hp:
+                continue
+            for prio_hp in (0, 1):
+                ks = [des.KernelSpec(0, 0, 0, T[lp][0] * 1000, 500, T[lp][0] * 1000),
+                      des.KernelSpec(1, 1, prio_hp, T[hp][1] * 1000, 500, T[hp][1] * 1000)]
+                sim = des.simulate(des.HPF, ks)
+                assert as_tuples(sim.decisions) == replay_cpp(flep, des.HPF, sim.events)
+
+
+def test_ties_and_equal_arrivals(flep):
+    # identical T_r and arrival times: arrival order decides (A14)
+    ks = [des.KernelSpec(i, 1000 * (i // 3), 0, 5000, 0, 5000) for i in range(9)]
+    sim = des.simulate(des.HPF, ks)
+    assert as_tuples(sim.decisions) == replay_cpp(flep, des.HPF, sim.events)
+    order = [d[2] for d in sim.decisions if d[1] in ("LAUNCH", "RESUME")]
+    assert order == sorted(order)

@@ -1,0 +1,60 @@
+"""Run each hot kernel (wrapped and unwrapped) a few times for ncu captures.
+
+Usage under gpurun:  ncu --set full -k regex:flep_ ... python tools/profile_kernels.py [--kernels spmv,stencil]
+"""
+import argparse
+import os
+import sys
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+from synth import gen  # noqa: E402
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--kernels", default="spmv,stencil,saxpy")
+    ap.add_argument("--reps", type=int, default=2)
+    ap.add_argument("--chunk", type=int, default=1)
+    ap.add_argument("--prefetch", type=int, default=1)
+    a = ap.parse_args()
+    import torch
+    from paper_conf_asplos_wulzj17_b200 import build, flep as F
+    build.build()
+    rt = F.Runtime(exec_on_user_stream=True)
+    flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
+    T = lambda x: torch.from_numpy(np.ascontiguousarray(x)).cuda()  # noqa: E731
+    jobs = []
+    if "spmv" in a.kernels:
+        rp, col, val, x = gen.csr_inputs(1 << 20, seed=2)
+        y = torch.zeros(1 << 20, device="cuda")
+        args = F.spmv_args(y, T(rp), T(col), T(val), T(x))
+        jobs.append(("spmv", F.BODY_SPMV_CSR_F32, F.spmv_grid(1 << 20), args, (rp, col, val, x)))
+    if "stencil" in a.kernels:
+        st = T(gen.stencil_f32_input(4096, seed=3))
+        out = torch.empty_like(st)
+        jobs.append(("stencil", F.BODY_STENCIL5_F32, F.stencil_grid(4096), F.stencil_args(out, st), (st, out)))
+    if "saxpy" in a.kernels:
+        n = 1 << 28
+        xs = torch.ones(n, dtype=torch.int32, device="cuda")
+        ys = torch.ones(n, dtype=torch.int32, device="cuda")
+        jobs.append(("saxpy", F.BODY_SAXPY_I32, F.saxpy_grid(n), F.saxpy_i32_args(ys, xs, 3), (xs, ys)))
+    s = torch.cuda.current_stream()
+    for name, body, grid, args, keep in jobs:
+        k = rt.register_kernel(body, chunk=a.chunk, poll=1, prefetch=bool(a.prefetch))
+        for _ in range(a.reps):
+            flush.zero_()
+            rt.launch_unwrapped(body, grid, args, stream=s)
+            torch.cuda.synchronize()
+            flush.zero_()
+            h = rt.launch(k, grid, args, stream=s)
+            rt.sync(h)
+    torch.cuda.synchronize()
+    rt.close()
+
+
+if __name__ == "__main__":
+    main()
