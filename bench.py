@@ -161,9 +161,26 @@ class Workload:
         self.st_bytes = stencil_bytes(STENCIL_N)
 
 
+class L2Flush:
+    """Evict L2 between timed iterations: write a buffer of 2x the L2 size (the contract's flush),
+    then read a second one so that the dirty lines the write left behind are written back by the
+    flush itself and not by the next timed kernel."""
+
+    def __init__(self, torch):
+        l2 = torch.cuda.get_device_properties(0).L2_cache_size
+        n = max(2 * l2, 256 << 20)
+        self.w = torch.empty(n, dtype=torch.uint8, device="cuda")
+        self.r = torch.zeros(n // 4, dtype=torch.int32, device="cuda")
+        self.out = torch.zeros((), dtype=torch.int64, device="cuda")
+        self.torch = torch
+
+    def zero_(self):
+        self.w.zero_()
+        self.r.sum()
+
+
 def l2_flush_buffer(torch):
-    l2 = torch.cuda.get_device_properties(0).L2_cache_size
-    return torch.empty(max(2 * l2, 256 << 20), dtype=torch.uint8, device="cuda")
+    return L2Flush(torch)
 
 
 def run_temporal(args, rank, world, local):
@@ -497,7 +514,7 @@ def main():
     ap.add_argument("--impl", default="flep", choices=["flep", "reference"])
     ap.add_argument("--config", default="temporal", choices=["temporal"])
     ap.add_argument("--lp-chunk", type=int, default=1)
-    ap.add_argument("--prefetch", type=int, default=1)
+    ap.add_argument("--prefetch", type=int, default=0)
     ap.add_argument("--lp-poll", type=int, default=1)
     ap.add_argument("--reps", type=int, default=20)
     ap.add_argument("--e2e-steps", type=int, default=10)

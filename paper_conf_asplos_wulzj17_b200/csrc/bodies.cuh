@@ -142,7 +142,7 @@ struct SpmvBody {
 template <bool kInt>
 struct Stencil5Body {
   static constexpr int kThreads = 256;
-  static constexpr int kMinBlocks = 4;
+  static constexpr int kMinBlocks = 3;
   static constexpr uint32_t kTile = 64;
   using Args = flep_stencil_args;
 

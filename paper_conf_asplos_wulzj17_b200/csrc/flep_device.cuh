@@ -12,7 +12,7 @@
 // atomicAdd (the probe measured ~1.46 fetches/ns chip-wide on one address, so C amortises the
 // atomic); exits happen only at poll points or on exhaustion, never while holding a chunk
 // (exactly-once, reading A4). The last worker of an epoch publishes DONE/PREEMPTED to a pinned
-// host word with a system-scope release store.
+// host slot with one relaxed system-scope 8-byte store.
 #pragma once
 #include <cstdint>
 
@@ -31,8 +31,9 @@ struct alignas(128) ControlBlock {
   uint32_t _p0[31];
   uint32_t ctrl;           // epoch<<16 | n_yield (D1/D2); device copy for the memop transport
   uint32_t _p1[31];
-  uint32_t done;           // original blocks executed (all epochs)
-  uint32_t exited;         // workers of the current epoch that have exited (reset by the last)
+  // one 64-bit word, one atomic per worker exit: low half = original blocks executed (all
+  // epochs), high half = workers of the current epoch that have exited (reset by the last)
+  unsigned long long done_exited;
   uint32_t _p2[30];
   // per-epoch summaries (ring of kEvEpochs)
   uint64_t ep_t_trigger[kEvEpochs];
@@ -49,11 +50,12 @@ struct WorkerEvent {       // mirrors flep_worker_event
 };
 
 struct HostStatus {        // pinned, mapped; one 32-B slot per launch
-  uint32_t word;           // (epoch << 8) | state, epoch 1-based; written last (release.sys)
-  uint32_t done;           // done counter at the end of that epoch
-  uint32_t ctr;            // task counter at the end of that epoch
+  uint32_t word;           // (generation << 8) | state of the last drained epoch   } one 8-byte
+  uint32_t done;           // done counter at the end of that epoch                 } store
+  uint32_t ctr;            // task counter at the end of that epoch (best effort; the device
+                           // copy in ControlBlock::ep_ctr is authoritative)
   uint32_t ctrl;           // FLEP_FLAG_HOST_MAPPED: the control word itself (CPU-written)
-  uint64_t t_end;          // %globaltimer of the last exit
+  uint64_t t_end;          // %globaltimer of the last exit (best effort)
   uint64_t _pad;
 };
 
@@ -104,6 +106,12 @@ __device__ __forceinline__ void red_add_release_gpu(uint32_t* p, uint32_t v) {
 }
 __device__ __forceinline__ void st_release_sys(uint32_t* p, uint32_t v) {
   asm volatile("st.release.sys.global.u32 [%0], %1;" :: "l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ void st_relaxed_sys(uint32_t* p, uint32_t v) {
+  asm volatile("st.relaxed.sys.global.u32 [%0], %1;" :: "l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ void st_relaxed_sys_u64(uint64_t* p, uint64_t v) {
+  asm volatile("st.relaxed.sys.global.u64 [%0], %1;" :: "l"(p), "l"(v) : "memory");
 }
 __device__ __forceinline__ void st_relaxed_gpu(uint32_t* p, uint32_t v) {
   asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" :: "l"(p), "r"(v) : "memory");
@@ -171,31 +179,30 @@ flep_worker(const typename Body::Args args, const WorkerParams p) {
       for (uint32_t b = b0; b < b1; ++b) atomicAdd(&p.cov[b], 1u);
     if (++k == p.poll) k = 0;
   }
-  // exit path (a7). Every thread finished its last chunk before the barrier that broadcast the
-  // stop slot, so the release below (cumulative over the CTA barrier) publishes all of them.
+  // exit path (a7). One relaxed 64-bit atomic adds this worker's block count and its exit; the
+  // worker that completes the epoch's exit count sees the exact total. No fences: the outputs
+  // are published by kernel completion (stream order), and the host status is a notification.
   if (tid == 0) {
     const uint32_t my_blocks = s_blocks;
-    if (my_blocks) red_add_release_gpu(&p.cb->done, my_blocks);
     WorkerEvent& e = p.ev[(p.epoch % kEvEpochs) * p.workers + blockIdx.x];
     const uint64_t t_exit = gtimer();
     e.smid = s_sm; e.reason = s_reason; e.n_blocks = my_blocks; e.epoch = p.epoch;
     e.t_entry = s_t_entry; e.t_exit = t_exit;
-    const uint32_t old = atom_add_acqrel_gpu(&p.cb->exited, 1u);
-    if (old + 1 == p.workers) {                          // last worker of this epoch
-      const uint32_t d = ld_acquire_gpu(&p.cb->done);
-      const uint32_t c = ld_acquire_gpu(&p.cb->ctr);
+    const unsigned long long old = atomicAdd(&p.cb->done_exited, (1ull << 32) | my_blocks);
+    if ((uint32_t)(old >> 32) + 1 == p.workers) {        // last worker of this epoch
+      const uint32_t d = (uint32_t)old + my_blocks;
+      const uint32_t c = ld_relaxed_gpu(&p.cb->ctr);     // every fetch has completed by now
       const uint32_t st = (d >= p.n_blocks) ? kStateDone : kStatePreempted;
       const uint32_t ei = p.epoch % kEvEpochs;
       p.cb->ep_t_end[ei] = t_exit; p.cb->ep_done[ei] = d; p.cb->ep_ctr[ei] = c;
       p.cb->ep_state[ei] = st;
-      p.cb->exited = 0;                                  // ready for the next epoch
-      if (st == kStateDone) { p.cb->ctr = 0; p.cb->done = 0; }   // block clean for reuse
       p.cb->ep_t_trigger[(p.epoch + 1) % kEvEpochs] = 0;  // next epoch's trigger stamp
-      p.status->t_end = t_exit;
-      p.status->done = d;
-      p.status->ctr = c;
-      __threadfence_system();
-      st_release_sys(&p.status->word, (p.epoch << 8) | st);
+      if (st == kStateDone) { p.cb->done_exited = 0ull; p.cb->ctr = 0; }   // clean for reuse
+      else p.cb->done_exited = (unsigned long long)d;    // exits reset, progress kept
+      st_relaxed_sys(&p.status->ctr, c);
+      st_relaxed_sys_u64(&p.status->t_end, t_exit);
+      st_relaxed_sys_u64(reinterpret_cast<uint64_t*>(&p.status->word),
+                         ((uint64_t)d << 32) | ((p.epoch << 8) | st));
     }
   }
 }

@@ -242,10 +242,11 @@ flep_status start_epoch(flep_rt rt, Launch& L) {
 bool refresh(Launch& L) {
   if (L.state != FLEP_STATE_RUNNING && L.state != FLEP_STATE_YIELDING && L.state != FLEP_STATE_PARTIAL)
     return false;
-  const uint32_t w = __atomic_load_n(&L.hs->word, __ATOMIC_ACQUIRE);
+  const uint64_t w64 = __atomic_load_n(reinterpret_cast<uint64_t*>(&L.hs->word), __ATOMIC_ACQUIRE);
+  const uint32_t w = (uint32_t)w64;
   if ((w >> 8) != (gen_of(L) & 0xffffffu)) return false;
-  L.last_done = L.hs->done;
-  L.last_ctr = L.hs->ctr;
+  L.last_done = (uint32_t)(w64 >> 32);
+  L.last_ctr = __atomic_load_n(&L.hs->ctr, __ATOMIC_ACQUIRE);
   if ((w & 0xffu) == kStateDone) {
     L.state = FLEP_STATE_DONE;
     L.t_finish = now_ns();
@@ -374,6 +375,13 @@ flep_status flep_init(int device, const flep_options* opts, flep_rt* out) {
   for (int i = kMaxSlots - 1; i >= 0; --i) rt->free_slots.push_back(i);
   rt->max_workers = rt->num_sms * kMaxWorkersPerSm;
   rt->dmem_bytes = sizeof(ControlBlock) + (size_t)kEvEpochs * rt->max_workers * sizeof(WorkerEvent);
+  for (int i = 0; i < 16; ++i) {             // warm pool: no allocation on the launch path
+    void* p = nullptr;
+    CUDA_TRY(cudaMalloc(&p, rt->dmem_bytes));
+    CUDA_TRY(cudaMemset(p, 0, sizeof(ControlBlock)));
+    rt->cb_gen[p] = 0;
+    rt->free_dmem.push_back(p);
+  }
   if (rt->opt.policy != FLEP_POLICY_MANUAL) {
     rt->policy.reset(new Policy(rt->opt.policy, rt->num_sms));
     flep_rt raw = rt.get();
@@ -473,11 +481,12 @@ flep_status flep_launch(flep_rt rt, flep_kernel kid, flep_dim3 grid, const void*
   L.exec_level = stream_level(rt, priority);
   s = get_stream(rt, L.exec_level, &L.exec);
   if (s) return s;
+  bool fresh_cb = false;
   if (!rt->free_dmem.empty()) { L.dmem = rt->free_dmem.back(); rt->free_dmem.pop_back(); }
   else {
     CUDA_TRY(cudaMalloc(&L.dmem, rt->dmem_bytes));
-    CUDA_TRY(cudaMemset(L.dmem, 0, sizeof(ControlBlock)));   // once per block, synchronous
     rt->cb_gen[L.dmem] = 0;
+    fresh_cb = true;             // zeroed below, on the stream the workers run on
   }
   L.gen0 = rt->cb_gen[L.dmem];
   if (L.gen0 + 2 * kEvEpochs >= 0xffffffu) return fail(FLEP_ERR_NOMEM, "control block generation space exhausted");
@@ -514,6 +523,7 @@ flep_status flep_launch(flep_rt rt, flep_kernel kid, flep_dim3 grid, const void*
     cudaEventDestroy(ev_u);
   }
   if (L.cov) CUDA_TRY(cudaMemsetAsync(L.cov, 0, N * 4, L.exec));
+  if (fresh_cb) CUDA_TRY(cudaMemsetAsync(L.dmem, 0, sizeof(ControlBlock), L.exec));
   rt->launches[L.id] = std::move(Lp);
   *out = L.id;
   if (rt->opt.policy == FLEP_POLICY_MANUAL) return start_epoch(rt, L);
@@ -602,7 +612,8 @@ flep_status flep_sync(flep_rt rt, flep_launch_t h, int64_t timeout_ns) {
   std::lock_guard<std::mutex> lk(rt->mu);
   Launch* L = find(rt, h);
   // keep the newest finished launches' device logs (coverage, events) for debug copies
-  constexpr size_t kRetain = 64;
+  // (64 with the coverage log, else the last 4; the warm pool keeps launches allocation-free)
+  const size_t kRetain = rt->opt.debug_coverage ? 64 : 4;
   if (L && !L->released && std::find(rt->retained.begin(), rt->retained.end(), h) == rt->retained.end())
     rt->retained.push_back(h);
   while (rt->retained.size() > kRetain) {

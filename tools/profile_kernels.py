@@ -25,7 +25,9 @@ def main():
     from paper_conf_asplos_wulzj17_b200 import build, flep as F
     build.build()
     rt = F.Runtime(exec_on_user_stream=True)
-    flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
+    sys.path.insert(0, ROOT)
+    from bench import L2Flush
+    flush = L2Flush(torch)
     T = lambda x: torch.from_numpy(np.ascontiguousarray(x)).cuda()  # noqa: E731
     jobs = []
     if "spmv" in a.kernels:
