@@ -12,6 +12,7 @@
 #pragma once
 #include <cstdint>
 #include "../../include/flep.h"
+#include "flep_device.cuh"
 
 namespace flep {
 
@@ -21,7 +22,7 @@ __device__ __forceinline__ void stcs4(int4* p, int4 v) { __stcs(p, v); }
 // ---------------------------------------------------------------------------------------------
 // SAXPY: y <- a*x + y. int32 wraps modulo 2^32 (computed in uint32); fp32 uses one fma per element.
 template <bool kInt>
-struct SaxpyBody {
+struct SaxpyBody : NoResources {
   static constexpr int kThreads = 256;
   static constexpr int kMinBlocks = 8;
   static constexpr uint32_t kBlockElems = 256;
@@ -84,7 +85,7 @@ struct SaxpyBody {
 // col/val loads, independent x gathers, 4 in flight per thread), writing products to smem; thread
 // t < 128 finally sums row r0+t's products in ascending p order. Per-row summation order is
 // fixed, so every execution of a block gives bit-identical results.
-struct SpmvBody {
+struct SpmvBody : NoResources {
   static constexpr int kThreads = 256;
   static constexpr int kMinBlocks = 8;
   static constexpr uint32_t kRowsPerBlock = 128;
@@ -140,7 +141,7 @@ struct SpmvBody {
 // 5-point stencil, out-of-place. Interior: fp32 0.5*c + 0.125*(n + s + w + e); int32
 // 4c - n - s - w - e (mod 2^32). Boundary rows/columns copied through.
 template <bool kInt>
-struct Stencil5Body {
+struct Stencil5Body : NoResources {
   static constexpr int kThreads = 256;
   static constexpr int kMinBlocks = 3;
   static constexpr uint32_t kTile = 64;

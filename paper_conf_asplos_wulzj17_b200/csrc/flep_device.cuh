@@ -133,12 +133,13 @@ __device__ __forceinline__ bool should_yield(uint32_t c, const WorkerParams& p, 
 //                                hazards (the wrapper barrier follows).
 template <class Body, bool kCoverage>
 __global__ void __launch_bounds__(Body::kThreads, Body::kMinBlocks)
-flep_worker(const typename Body::Args args, const WorkerParams p) {
+flep_worker(const __grid_constant__ typename Body::Args args, const WorkerParams p) {
   __shared__ uint32_t s_slot[2];     // chunk base broadcast, double-buffered: 1 barrier per chunk
   __shared__ uint64_t s_t_entry;     // worker bookkeeping kept out of registers (tid 0 only)
   __shared__ uint32_t s_sm, s_blocks, s_reason;
   const uint32_t tid = threadIdx.x;
   if (tid == 0) { s_sm = smid_reg(); s_t_entry = gtimer(); s_blocks = 0; s_reason = 0; }
+  Body::setup(args);                 // per-worker resources (e.g. TMEM, mbarriers); may sync
   uint32_t k = 0;                    // chunk index within the current poll period
   uint32_t parity = 0;
   uint32_t held = 0xffffffffu;       // tid 0: prefetched chunk base not yet processed
@@ -179,6 +180,7 @@ flep_worker(const typename Body::Args args, const WorkerParams p) {
       for (uint32_t b = b0; b < b1; ++b) atomicAdd(&p.cov[b], 1u);
     if (++k == p.poll) k = 0;
   }
+  Body::teardown(args);              // release per-worker resources before leaving the SM (a7)
   // exit path (a7). One relaxed 64-bit atomic adds this worker's block count and its exit; the
   // worker that completes the epoch's exit count sees the exact total. No fences: the outputs
   // are published by kernel completion (stream order), and the host status is a notification.
@@ -210,9 +212,17 @@ flep_worker(const typename Body::Args args, const WorkerParams p) {
 // The original kernel (unwrapped twin, K7): one CTA per original block, same body.
 template <class Body>
 __global__ void __launch_bounds__(Body::kThreads, Body::kMinBlocks)
-flep_unwrapped(const typename Body::Args args, uint32_t gx, uint32_t gy, uint32_t block_offset) {
+flep_unwrapped(const __grid_constant__ typename Body::Args args, uint32_t gx, uint32_t gy, uint32_t block_offset) {
   const uint32_t b = block_offset + blockIdx.x + gx * (blockIdx.y + gy * blockIdx.z);
+  Body::setup(args);
   Body::run(args, b, b + 1, gx, gy);
+  Body::teardown(args);
 }
+
+// Bodies without per-worker resources.
+struct NoResources {
+  template <class A> __device__ static void setup(const A&) {}
+  template <class A> __device__ static void teardown(const A&) {}
+};
 
 }  // namespace flep

@@ -1,22 +1,217 @@
-// gemm_tcgen05.cuh — placeholder until the tcgen05 GEMM body lands.
+// gemm_tcgen05.cuh — the dense-contraction body (MM, Table 1): C = A·Bᵀ with A
+// [M,K] and B [N,K] bf16 row-major (K-major "TN"), fp32 accumulation in TMEM, bf16 output.
+//
+// One original block = one 128x256 output tile. Inside the FLEP worker the CTA is warp-
+// specialised (sm_100a):
+//   warp 0 lane 0 : TMA producer — 128x64 A box + 256x64 B box per k-step, SWIZZLE_128B, into a
+//                   4-stage smem ring (full/empty mbarriers)
+//   warp 1 lane 0 : MMA issuer — tcgen05.mma.cta_group::1.kind::f16, M=128 N=256 K=16, four per
+//                   k-step, accumulator in TMEM (256 columns); tcgen05.commit frees smem stages
+//                   and finally signals the epilogue
+//   warp 2        : TMEM allocator (setup) / deallocator (teardown: before any exit, a7)
+//   warps 4..7    : epilogue — tcgen05.ld 32x32b.x32 → bf16 → global, then release the
+//                   accumulator (tmem_empty)
+// Pipeline phases persist in shared memory across chunks, so a worker's consecutive tasks share
+// one pipeline; the wrapper's barrier separates chunks (the poll point). Preemption is at tile
+// granularity (in-tile preemption is SURVEY f4).
 #pragma once
+#include <cuda.h>
+#include <cuda_bf16.h>
 #include <cuda_runtime.h>
+#include <cstdint>
+
+#include "../../include/flep.h"
 #include "flep_device.cuh"
 
 namespace flep {
 
+struct GemmArgsDev {
+  CUtensorMap tma_a;           // A [M,K] bf16, box {64, 128}, SWIZZLE_128B
+  CUtensorMap tma_b;           // B [N,K] bf16, box {64, 256}, SWIZZLE_128B
+  __nv_bfloat16* c;            // C [M,N] bf16 row-major
+  uint32_t m, n, k;
+};
+
 struct GemmBody {
   static constexpr int kThreads = 256;
   static constexpr int kMinBlocks = 1;
+  static constexpr uint32_t BM = 128, BN = 256, BK = 64, UMMA_K = 16, STAGES = 4;
+  static constexpr uint32_t kBytesA = BM * BK * 2, kBytesB = BN * BK * 2, kStage = kBytesA + kBytesB;
+  static constexpr uint32_t kTmemCols = 256;
+  static constexpr size_t kDynSmem = 1024 + STAGES * kStage + 256;
+  using Args = GemmArgsDev;
+
+  struct State {                      // lives after the stage ring
+    uint64_t full[STAGES], empty[STAGES], tmem_full, tmem_empty;
+    uint32_t tmem_base;
+    uint32_t p_stage, p_phase;        // producer
+    uint32_t m_stage, m_phase, m_acc; // MMA issuer
+    uint32_t e_acc;                   // epilogue
+  };
+
+  __device__ static uint8_t* ring() {
+    extern __shared__ uint8_t dsmem[];
+    const uint32_t a = static_cast<uint32_t>(__cvta_generic_to_shared(dsmem));
+    return dsmem + (((a + 1023u) & ~1023u) - a);
+  }
+  __device__ static State* state() { return reinterpret_cast<State*>(ring() + STAGES * kStage); }
+  __device__ static uint32_t smem_u32(const void* p) { return static_cast<uint32_t>(__cvta_generic_to_shared(p)); }
+
+  __device__ static void mbar_init(uint64_t* b, uint32_t n) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" :: "r"(smem_u32(b)), "r"(n) : "memory");
+  }
+  __device__ static void mbar_wait(uint64_t* b, uint32_t parity) {
+    asm volatile(
+        "{\n .reg .pred p;\n W: mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+        " @!p bra W;\n}\n" :: "r"(smem_u32(b)), "r"(parity) : "memory");
+  }
+  __device__ static void mbar_arrive(uint64_t* b) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" :: "r"(smem_u32(b)) : "memory");
+  }
+  __device__ static void mbar_expect_tx(uint64_t* b, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" :: "r"(smem_u32(b)), "r"(bytes) : "memory");
+  }
+  __device__ static void tma_2d(const CUtensorMap* map, void* dst, uint64_t* bar, int32_t x, int32_t y) {
+    asm volatile(
+        "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];"
+        :: "r"(smem_u32(dst)), "l"(reinterpret_cast<uint64_t>(map)), "r"(smem_u32(bar)), "r"(x), "r"(y)
+        : "memory");
+  }
+  // K-major, SWIZZLE_128B smem matrix descriptor (sm_100 UMMA): start>>4, LBO 16 B (unused for
+  // swizzled K-major), SBO 1024 B (8 rows x 128 B), version 1, layout SWIZZLE_128B (2).
+  __device__ static uint64_t sdesc(uint32_t saddr) {
+    return (uint64_t)((saddr >> 4) & 0x3FFFu) | ((uint64_t)1u << 16) | ((uint64_t)(1024u >> 4) << 32) |
+           ((uint64_t)1u << 46) | ((uint64_t)2u << 61);
+  }
+  // kind::f16 instruction descriptor: D f32, A/B bf16, both K-major, N = 256, M = 128.
+  static constexpr uint32_t kIdesc = (1u << 4) | (1u << 7) | (1u << 10) | ((BN >> 3) << 17) | ((BM >> 4) << 24);
+
+  __device__ static void setup(const Args&) {
+    State* s = state();
+    const uint32_t warp = threadIdx.x >> 5;
+    if (threadIdx.x == 0) {
+      for (uint32_t i = 0; i < STAGES; ++i) { mbar_init(&s->full[i], 1); mbar_init(&s->empty[i], 1); }
+      mbar_init(&s->tmem_full, 1);
+      mbar_init(&s->tmem_empty, 128);
+      s->p_stage = s->p_phase = s->m_stage = s->m_phase = s->m_acc = s->e_acc = 0;
+      asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    if (warp == 2) {
+      asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;"
+                   :: "r"(smem_u32(&s->tmem_base)), "r"(kTmemCols) : "memory");
+      asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+  }
+
+  __device__ static void teardown(const Args&) {
+    State* s = state();
+    __syncthreads();
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    if ((threadIdx.x >> 5) == 2)
+      asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" :: "r"(s->tmem_base), "r"(kTmemCols) : "memory");
+  }
+
+  __device__ static void run(const Args& g, uint32_t b0, uint32_t b1, uint32_t gx, uint32_t) {
+    State* s = state();
+    uint8_t* base = ring();
+    const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31u;
+    const uint32_t nk = g.k / BK;
+    if (warp == 0) {
+      if (lane == 0) {                                     // ---- TMA producer
+        uint32_t st = s->p_stage, ph = s->p_phase;
+        for (uint32_t b = b0; b < b1; ++b) {
+          const int32_t tm = (int32_t)(b / gx), tn = (int32_t)(b % gx);
+          for (uint32_t kb = 0; kb < nk; ++kb) {
+            mbar_wait(&s->empty[st], ph ^ 1u);
+            uint8_t* sa = base + st * kStage;
+            uint8_t* sb = sa + kBytesA;
+            mbar_expect_tx(&s->full[st], kStage);
+            tma_2d(&g.tma_a, sa, &s->full[st], (int32_t)(kb * BK), tm * (int32_t)BM);
+            tma_2d(&g.tma_b, sb, &s->full[st], (int32_t)(kb * BK), tn * (int32_t)BN);
+            if (++st == STAGES) { st = 0; ph ^= 1u; }
+          }
+        }
+        s->p_stage = st; s->p_phase = ph;
+      }
+    } else if (warp == 1) {
+      if (lane == 0) {                                     // ---- MMA issuer (one thread)
+        uint32_t st = s->m_stage, ph = s->m_phase, acc = s->m_acc;
+        const uint32_t tmem = s->tmem_base;
+        for (uint32_t b = b0; b < b1; ++b) {
+          mbar_wait(&s->tmem_empty, acc ^ 1u);             // epilogue drained the accumulator
+          asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+          for (uint32_t kb = 0; kb < nk; ++kb) {
+            mbar_wait(&s->full[st], ph);
+            asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+            const uint32_t sa = smem_u32(base + st * kStage), sb = sa + kBytesA;
+#pragma unroll
+            for (uint32_t k = 0; k < BK / UMMA_K; ++k) {
+              const uint64_t da = sdesc(sa + k * UMMA_K * 2), db = sdesc(sb + k * UMMA_K * 2);
+              const uint32_t accum = (kb | k) ? 1u : 0u;
+              asm volatile(
+                  "{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n"
+                  " tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n}\n"
+                  :: "r"(tmem), "l"(da), "l"(db), "r"(kIdesc), "r"(accum) : "memory");
+            }
+            asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];"
+                         :: "r"(smem_u32(&s->empty[st])) : "memory");
+            if (++st == STAGES) { st = 0; ph ^= 1u; }
+          }
+          asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];"
+                       :: "r"(smem_u32(&s->tmem_full)) : "memory");
+          acc ^= 1u;
+        }
+        s->m_stage = st; s->m_phase = ph; s->m_acc = acc;
+      }
+    } else if (warp >= 4) {                                // ---- epilogue (128 threads)
+      const uint32_t q = warp - 4;                         // TMEM lanes [32q, 32q+32)
+      uint32_t acc = s->e_acc;
+      const uint32_t tmem = s->tmem_base + ((q * 32u) << 16);
+      for (uint32_t b = b0; b < b1; ++b) {
+        const uint32_t tm = b / gx, tn = b % gx;
+        mbar_wait(&s->tmem_full, acc);
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        const uint32_t row = tm * BM + q * 32u + lane;
+        __nv_bfloat16* crow = g.c + (size_t)row * g.n + (size_t)tn * BN;
+#pragma unroll 1
+        for (uint32_t c0 = 0; c0 < BN; c0 += 32) {
+          uint32_t r[32];
+          asm volatile(
+              "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+              "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+              : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+                "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]),
+                "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]),
+                "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
+              : "r"(tmem + c0));
+          asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+          uint4 o[4];
+          uint32_t* ow = reinterpret_cast<uint32_t*>(o);
+#pragma unroll
+          for (int i = 0; i < 16; ++i) {
+            __nv_bfloat162 h = __floats2bfloat162_rn(__uint_as_float(r[2 * i]), __uint_as_float(r[2 * i + 1]));
+            ow[i] = *reinterpret_cast<uint32_t*>(&h);
+          }
+          uint4* dst = reinterpret_cast<uint4*>(crow + c0);
+#pragma unroll
+          for (int i = 0; i < 4; ++i) dst[i] = o[i];
+        }
+        asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+        mbar_arrive(&s->tmem_empty);
+        acc ^= 1u;
+      }
+      if (threadIdx.x == 128) s->e_acc = acc;
+    }
+  }
 };
 
-inline cudaError_t gemm_worker_launch(const void*, const WorkerParams&, uint32_t, cudaStream_t, bool) {
-  return cudaErrorNotSupported;
-}
-inline cudaError_t gemm_unwrapped_launch(const void*, dim3, uint32_t, uint32_t, cudaStream_t) {
-  return cudaErrorNotSupported;
-}
-inline cudaError_t gemm_occupancy(int* k, bool) { *k = 1; return cudaSuccess; }
-inline const char* gemm_validate(const void*, dim3) { return "GEMM body not built yet"; }
+// host side (gemm_tcgen05.cu)
+cudaError_t gemm_worker_launch(const void* user_args, const WorkerParams& p, uint32_t W, cudaStream_t s, bool cov);
+cudaError_t gemm_unwrapped_launch(const void* user_args, dim3 grid, uint32_t offset, uint32_t count, cudaStream_t s);
+cudaError_t gemm_occupancy(int* k, bool cov);
+const char* gemm_validate(const void* user_args, dim3 grid);
 
 }  // namespace flep

@@ -31,11 +31,11 @@ struct Ops {
   static cudaError_t occupancy(int* k, bool cov) {
     cudaError_t e;
     if (Body::kDynSmem > 48 * 1024) {
-      e = cudaFuncSetAttribute(flep_worker<Body, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, Body::kDynSmem);
+      e = cudaFuncSetAttribute(flep_worker<Body, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)Body::kDynSmem);
       if (e) return e;
-      e = cudaFuncSetAttribute(flep_worker<Body, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, Body::kDynSmem);
+      e = cudaFuncSetAttribute(flep_worker<Body, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)Body::kDynSmem);
       if (e) return e;
-      e = cudaFuncSetAttribute(flep_unwrapped<Body>, cudaFuncAttributeMaxDynamicSharedMemorySize, Body::kDynSmem);
+      e = cudaFuncSetAttribute(flep_unwrapped<Body>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)Body::kDynSmem);
       if (e) return e;
     }
     if (cov) return cudaOccupancyMaxActiveBlocksPerMultiprocessor(k, flep_worker<Body, true>, Body::kThreads, Body::kDynSmem);
@@ -48,6 +48,41 @@ template <class B>
 struct WithSmem : B {
   static constexpr size_t kDynSmem = 0;
 };
+
+}  // namespace
+
+// GEMM launchers live in gemm_tcgen05.cu (they need the tensor-map encoder); they use these.
+template <class Body>
+cudaError_t launch_worker_raw(const typename Body::Args& a, const WorkerParams& p, uint32_t W, cudaStream_t s, bool cov) {
+  if (cov) flep_worker<Body, true><<<W, Body::kThreads, Body::kDynSmem, s>>>(a, p);
+  else flep_worker<Body, false><<<W, Body::kThreads, Body::kDynSmem, s>>>(a, p);
+  return cudaGetLastError();
+}
+template <class Body>
+cudaError_t launch_unwrapped_raw(const typename Body::Args& a, dim3 grid, uint32_t offset, uint32_t count, cudaStream_t s) {
+  if (count == 0) flep_unwrapped<Body><<<grid, Body::kThreads, Body::kDynSmem, s>>>(a, grid.x, grid.y, 0);
+  else flep_unwrapped<Body><<<count, Body::kThreads, Body::kDynSmem, s>>>(a, grid.x, grid.y, offset);
+  return cudaGetLastError();
+}
+template <class Body>
+cudaError_t occupancy_raw(int* k, bool cov) {
+  cudaError_t e;
+  if (Body::kDynSmem > 48 * 1024) {
+    e = cudaFuncSetAttribute(flep_worker<Body, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)Body::kDynSmem);
+    if (e) return e;
+    e = cudaFuncSetAttribute(flep_worker<Body, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)Body::kDynSmem);
+    if (e) return e;
+    e = cudaFuncSetAttribute(flep_unwrapped<Body>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)Body::kDynSmem);
+    if (e) return e;
+  }
+  if (cov) return cudaOccupancyMaxActiveBlocksPerMultiprocessor(k, flep_worker<Body, true>, Body::kThreads, Body::kDynSmem);
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(k, flep_worker<Body, false>, Body::kThreads, Body::kDynSmem);
+}
+template cudaError_t launch_worker_raw<GemmBody>(const GemmBody::Args&, const WorkerParams&, uint32_t, cudaStream_t, bool);
+template cudaError_t launch_unwrapped_raw<GemmBody>(const GemmBody::Args&, dim3, uint32_t, uint32_t, cudaStream_t);
+template cudaError_t occupancy_raw<GemmBody>(int*, bool);
+
+namespace {
 
 using SaxpyI32 = WithSmem<SaxpyBody<true>>;
 using SaxpyF32 = WithSmem<SaxpyBody<false>>;

@@ -24,4 +24,11 @@ struct BodyOps {
 
 const BodyOps* body_ops(int32_t body);
 
+template <class Body>
+cudaError_t launch_worker_raw(const typename Body::Args& a, const WorkerParams& p, uint32_t W, cudaStream_t s, bool cov);
+template <class Body>
+cudaError_t launch_unwrapped_raw(const typename Body::Args& a, dim3 grid, uint32_t offset, uint32_t count, cudaStream_t s);
+template <class Body>
+cudaError_t occupancy_raw(int* k, bool cov);
+
 }  // namespace flep

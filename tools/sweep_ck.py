@@ -44,6 +44,24 @@ def main():
         st = torch.rand(16384, 16384, device="cuda")
         out = torch.empty_like(st)
         jobs["stencil16k"] = (F.BODY_STENCIL5_F32, F.stencil_grid(16384), F.stencil_args(out, st), 8 * 16384 ** 2, (st, out))
+    if "gemm" in a.bodies:
+        M = 8192
+        A = torch.randn(M, M, device="cuda").to(torch.bfloat16)
+        B = torch.randn(M, M, device="cuda").to(torch.bfloat16)
+        Cg = torch.empty(M, M, device="cuda", dtype=torch.bfloat16)
+        jobs["gemm"] = (F.BODY_GEMM_BF16, F.gemm_grid(M, M), F.gemm_args(Cg, A, B), 2 * M ** 3, (A, B, Cg))
+        for _ in range(3):
+            torch.matmul(A, B.t())
+        ts = []
+        for _ in range(10):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            torch.matmul(A, B.t())
+            e1.record()
+            e1.synchronize()
+            ts.append(e0.elapsed_time(e1) * 1e3)
+        print(json.dumps({"body": "gemm", "variant": "cublas(torch.matmul)", "us": round(float(np.median(ts)), 3),
+                          "tflops": round(2 * M ** 3 / float(np.median(ts)) / 1e6, 1)}), flush=True)
     if "saxpy" in a.bodies:
         n = 1 << 28
         xs = torch.ones(n, dtype=torch.int32, device="cuda")
@@ -69,7 +87,7 @@ def main():
     for name, (body, grid, args, nbytes, keep) in jobs.items():
         tu = timed(lambda: rt.launch_unwrapped(body, grid, args, stream=s))
         print(json.dumps({"body": name, "variant": "unwrapped", "us": round(tu, 3),
-                          "gbs": round(nbytes / tu / 1e3, 1)}), flush=True)
+                          ("tflops" if name == "gemm" else "gbs"): round(nbytes / tu / (1e6 if name == "gemm" else 1e3), 1)}), flush=True)
         for C in map(int, a.chunks.split(",")):
             for K in map(int, a.polls.split(",")):
                 for pf in map(int, a.prefetch.split(",")):
@@ -77,7 +95,8 @@ def main():
                         k = rt.register_kernel(body, chunk=C, poll=K, prefetch=bool(pf), ctas_per_sm=cps)
                         tw = timed(lambda: rt.launch(k, grid, args, stream=s))
                         print(json.dumps({"body": name, "C": C, "K": K, "prefetch": pf, "cps": cps,
-                                          "us": round(tw, 3), "gbs": round(nbytes / tw / 1e3, 1),
+                                          "us": round(tw, 3),
+                                          ("tflops" if name == "gemm" else "gbs"): round(nbytes / tw / (1e6 if name == "gemm" else 1e3), 1),
                                           "overhead_pct": round((tw / tu - 1) * 100, 2)}), flush=True)
     rt.close()
 
