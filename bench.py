@@ -512,7 +512,10 @@ def main():
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--impl", default="flep", choices=["flep", "reference"])
-    ap.add_argument("--config", default="temporal", choices=["temporal"])
+    ap.add_argument("--config", default="temporal", choices=["temporal", "corun1", "spatial", "queue"])
+    ap.add_argument("--corun-cps", type=int, default=2)
+    ap.add_argument("--queue-kernels", type=int, default=64)
+    ap.add_argument("--rho", type=float, default=1.0)
     ap.add_argument("--lp-chunk", type=int, default=1)
     ap.add_argument("--prefetch", type=int, default=0)
     ap.add_argument("--lp-poll", type=int, default=1)
@@ -534,7 +537,16 @@ def main():
             if not b2.needs_build():
                 break
             time.sleep(1)
-    run_temporal(args, rank, world, local)
+    if args.config == "temporal":
+        run_temporal(args, rank, world, local)
+    else:
+        import bench_configs
+        if args.config == "spatial":
+            bench_configs.run_spatial(args, rank, world, local)
+        elif args.config == "corun1":
+            bench_configs.run_corun1(args, rank, world, local)
+        else:
+            bench_configs.run_queue(args, rank, world, local)
 
 
 if __name__ == "__main__":

@@ -21,6 +21,7 @@
 #include <atomic>
 #include <chrono>
 #include <condition_variable>
+#include <deque>
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
@@ -115,6 +116,14 @@ struct Launch {
   uint32_t last_done = 0, last_ctr = 0;
   int64_t t_last_request = -1, t_last_drain = -1;
   uint32_t gen0 = 0;                 // control-block generation before this launch's epoch 1
+  // kernel-slicing baseline (FLEP_POLICY_SLICE): the original kernel as sub-grids of
+  // slice_blocks blocks, at most two in flight; a preemption stops issuing
+  bool sliced = false;
+  uint32_t slice_blocks = 0;
+  uint64_t next_block = 0, slice_done = 0;
+  std::deque<std::pair<cudaEvent_t, uint32_t>> inflight;
+  std::vector<cudaEvent_t> evpool;
+  cudaEvent_t fin_ev = nullptr;      // recorded after every grid of this launch (its last work)
   bool released = false;
   bool cancelled = false;
 };
@@ -162,9 +171,13 @@ struct flep_rt_s {
   std::atomic<bool> stop{false};
   std::map<std::pair<int32_t, bool>, int> occ_cache;
   std::vector<int64_t> retained;   // finished launches whose logs are kept for debug copies
+  std::vector<cudaEvent_t> event_pool;
+  std::vector<int64_t> to_release; // managed mode: DONE launches whose last grid may still run
 };
 
 namespace {
+
+Launch* find(flep_rt rt, flep_launch_t h);
 
 flep_status occupancy(flep_rt rt, const BodyOps* ops, bool cov, int* k) {
   auto key = std::make_pair(ops->body, cov);
@@ -208,7 +221,36 @@ flep_status write_ctrl(flep_rt rt, Launch& L, uint32_t value) {
   return FLEP_OK;
 }
 
+flep_status pooled_event(flep_rt rt, cudaEvent_t* e) {
+  if (!rt->event_pool.empty()) { *e = rt->event_pool.back(); rt->event_pool.pop_back(); return FLEP_OK; }
+  CUDA_TRY(cudaEventCreateWithFlags(e, cudaEventDisableTiming));
+  return FLEP_OK;
+}
+
+flep_status issue_slices(flep_rt rt, Launch& L) {
+  (void)rt;
+  while (L.state == FLEP_STATE_RUNNING && L.inflight.size() < 2 && L.next_block < L.n_blocks) {
+    const uint32_t cnt = (uint32_t)std::min<uint64_t>(L.slice_blocks, L.n_blocks - L.next_block);
+    CUDA_TRY(L.ops->unwrapped(L.args.data(), L.grid, (uint32_t)L.next_block, cnt, L.exec));
+    cudaEvent_t ev;
+    if (!L.evpool.empty()) { ev = L.evpool.back(); L.evpool.pop_back(); }
+    else CUDA_TRY(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
+    CUDA_TRY(cudaEventRecord(ev, L.exec));
+    L.inflight.push_back({ev, cnt});
+    L.next_block += cnt;
+    CUDA_TRY(cudaEventRecord(L.fin_ev, L.exec));
+  }
+  return FLEP_OK;
+}
+
 flep_status start_epoch(flep_rt rt, Launch& L) {
+  if (L.sliced) {
+    L.epoch++;
+    L.state = FLEP_STATE_RUNNING;
+    L.n_yield = 0;
+    if (L.t_first_start < 0) L.t_first_start = now_ns();
+    return issue_slices(rt, L);
+  }
   L.epoch++;
   WorkerParams p{};
   p.cb = L.cb;
@@ -232,6 +274,7 @@ flep_status start_epoch(flep_rt rt, Launch& L) {
   L.trig_n = 0;
   cudaError_t e = L.ops->worker(L.args.data(), p, L.workers, L.exec, L.cov != nullptr);
   if (e != cudaSuccess) return fail(FLEP_ERR_CUDA, "worker launch failed: %s", cudaGetErrorString(e));
+  CUDA_TRY(cudaEventRecord(L.fin_ev, L.exec));
   L.state = FLEP_STATE_RUNNING;
   L.n_yield = 0;
   if (L.t_first_start < 0) L.t_first_start = now_ns();
@@ -239,9 +282,27 @@ flep_status start_epoch(flep_rt rt, Launch& L) {
 }
 
 // Pull the pinned status slot; returns true if the launch's state changed to DONE.
-bool refresh(Launch& L) {
+bool refresh(flep_rt rt, Launch& L) {
   if (L.state != FLEP_STATE_RUNNING && L.state != FLEP_STATE_YIELDING && L.state != FLEP_STATE_PARTIAL)
     return false;
+  if (L.sliced) {
+    while (!L.inflight.empty() && cudaEventQuery(L.inflight.front().first) == cudaSuccess) {
+      L.slice_done += L.inflight.front().second;
+      L.evpool.push_back(L.inflight.front().first);
+      L.inflight.pop_front();
+    }
+    if (L.state == FLEP_STATE_RUNNING) issue_slices(rt, L);
+    if (!L.inflight.empty()) return false;
+    L.last_done = (uint32_t)L.slice_done;
+    L.last_ctr = (uint32_t)L.next_block;
+    if (L.slice_done >= L.n_blocks) {
+      L.state = FLEP_STATE_DONE;
+      L.t_finish = now_ns();
+      return true;
+    }
+    if (L.state == FLEP_STATE_YIELDING) { L.state = FLEP_STATE_PREEMPTED; L.t_last_drain = now_ns(); }
+    return false;
+  }
   const uint64_t w64 = __atomic_load_n(reinterpret_cast<uint64_t*>(&L.hs->word), __ATOMIC_ACQUIRE);
   const uint32_t w = (uint32_t)w64;
   if ((w >> 8) != (gen_of(L) & 0xffffffu)) return false;
@@ -265,6 +326,9 @@ void release_resources(flep_rt rt, Launch& L) {
   if (L.cov) rt->free_cov.push_back({L.cov, L.cov_cap});
   if (L.slot >= 0) rt->free_slots.push_back(L.slot);
   if (L.exec && L.exec_level != -1000) rt->free_streams[L.exec_level].push_back(L.exec);
+  for (cudaEvent_t e : L.evpool) rt->event_pool.push_back(e);
+  L.evpool.clear();
+  if (L.fin_ev) { rt->event_pool.push_back(L.fin_ev); L.fin_ev = nullptr; }
   L.dmem = nullptr; L.cov = nullptr; L.slot = -1; L.exec = nullptr;
   L.released = true;
 }
@@ -277,7 +341,11 @@ void apply_decisions(flep_rt rt) {
     if (it == rt->launches.end()) continue;
     Launch& L = *it->second;
     if (x.action == kPreempt) {
-      if (L.state == FLEP_STATE_RUNNING || L.state == FLEP_STATE_PARTIAL) {
+      if (L.sliced && L.state == FLEP_STATE_RUNNING) {   // slicing: stop issuing sub-kernels
+        L.t_last_request = now_ns();
+        L.state = FLEP_STATE_YIELDING;
+        L.n_yield = (uint32_t)x.n_sms;
+      } else if (L.state == FLEP_STATE_RUNNING || L.state == FLEP_STATE_PARTIAL) {
         write_ctrl(rt, L, ctrl_word(L, (uint32_t)std::min<int64_t>(x.n_sms, 0xffff)));
         L.state = FLEP_STATE_YIELDING;
         L.n_yield = (uint32_t)x.n_sms;
@@ -299,7 +367,8 @@ void monitor_loop(flep_rt rt) {
         Launch& L = *kv.second;
         if (L.state == FLEP_STATE_RUNNING || L.state == FLEP_STATE_YIELDING || L.state == FLEP_STATE_PARTIAL) {
           active = true;
-          if (refresh(L)) {
+          if (refresh(rt, L)) {
+            rt->to_release.push_back(L.id);
             const int64_t t = L.t_finish;
             rt->evlog.push_back({t, 1, L.id, L.prio, L.t_e, L.overhead});
             rt->policy->finish(t, L.id);
@@ -308,6 +377,25 @@ void monitor_loop(flep_rt rt) {
           } else if (L.state == FLEP_STATE_PREEMPTED) {
             rt->cv.notify_all();
           }
+        }
+      }
+      for (size_t i = 0; i < rt->to_release.size();) {      // recycle finished launches
+        Launch* R = find(rt, rt->to_release[i]);
+        if (R && cudaEventQuery(R->fin_ev) == cudaSuccess) {
+          if (rt->opt.debug_coverage) {                    // keep the newest 64 for debug copies
+            rt->retained.push_back(R->id);
+            while (rt->retained.size() > 64) {
+              Launch* old = find(rt, rt->retained.front());
+              rt->retained.erase(rt->retained.begin());
+              if (old) release_resources(rt, *old);
+            }
+          } else {
+            release_resources(rt, *R);
+          }
+          rt->to_release[i] = rt->to_release.back();
+          rt->to_release.pop_back();
+        } else {
+          ++i;
         }
       }
       if (!active) {
@@ -357,7 +445,6 @@ flep_status flep_init(int device, const flep_options* opts, flep_rt* out) {
   if (rt->opt.default_poll == 0) rt->opt.default_poll = 1;
   if (rt->opt.policy < FLEP_POLICY_MANUAL || rt->opt.policy > FLEP_POLICY_SLICE)
     return fail(FLEP_ERR_INVALID, "bad policy %d", rt->opt.policy);
-  if (rt->opt.policy == FLEP_POLICY_SLICE) return fail(FLEP_ERR_UNSUPPORTED, "SLICE runtime mode not built yet");
   cudaDeviceProp prop;
   CUDA_TRY(cudaGetDeviceProperties(&prop, device));
   if (prop.major != 10) return fail(FLEP_ERR_UNSUPPORTED, "needs sm_100 (got %d.%d)", prop.major, prop.minor);
@@ -381,6 +468,18 @@ flep_status flep_init(int device, const flep_options* opts, flep_rt* out) {
     CUDA_TRY(cudaMemset(p, 0, sizeof(ControlBlock)));
     rt->cb_gen[p] = 0;
     rt->free_dmem.push_back(p);
+  }
+  if (rt->opt.debug_coverage) {              // debug runtimes retain 64 launches' logs: warm more
+    for (int i = 0; i < 72; ++i) {
+      void* p = nullptr;
+      CUDA_TRY(cudaMalloc(&p, rt->dmem_bytes));
+      CUDA_TRY(cudaMemset(p, 0, sizeof(ControlBlock)));
+      rt->cb_gen[p] = 0;
+      rt->free_dmem.push_back(p);
+      uint32_t* c = nullptr;
+      CUDA_TRY(cudaMalloc(&c, (size_t)(1u << 20) * 4));
+      rt->free_cov.push_back({c, (size_t)1u << 20});
+    }
   }
   if (rt->opt.policy != FLEP_POLICY_MANUAL) {
     rt->policy.reset(new Policy(rt->opt.policy, rt->num_sms));
@@ -470,6 +569,11 @@ flep_status flep_launch(flep_rt rt, flep_kernel kid, flep_dim3 grid, const void*
   const uint64_t wmax = (uint64_t)k * rt->num_sms;
   const uint64_t need = (N + L.chunk - 1) / L.chunk;
   L.workers = (uint32_t)std::min<uint64_t>(std::min<uint64_t>(wmax, need), rt->max_workers);
+  if (rt->opt.policy == FLEP_POLICY_SLICE) {
+    L.sliced = true;                                  // R16: one slice = one wave of W*C*K blocks
+    L.slice_blocks = rt->opt.slice_blocks ? rt->opt.slice_blocks
+                                          : (uint32_t)std::min<uint64_t>(wmax * L.chunk * L.poll, 0x7fffffff);
+  }
   L.t_arrive = now_ns();
   L.t_e = flep_model_predict_ns(kr.model, (double)N, (double)ops->threads, (double)N, 0.0);
   L.overhead = kr.overhead;
@@ -517,11 +621,14 @@ flep_status flep_launch(flep_rt rt, flep_kernel kid, flep_dim3 grid, const void*
   } else {
     // caller's prior work on `stream` (e.g. input copies) precedes the workers
     cudaEvent_t ev_u;
-    CUDA_TRY(cudaEventCreateWithFlags(&ev_u, cudaEventDisableTiming));
+    s = pooled_event(rt, &ev_u);
+    if (s) return s;
     CUDA_TRY(cudaEventRecord(ev_u, L.user));
     CUDA_TRY(cudaStreamWaitEvent(L.exec, ev_u, 0));
-    cudaEventDestroy(ev_u);
+    rt->event_pool.push_back(ev_u);    // reusable once recorded (waits bind at enqueue time)
   }
+  s = pooled_event(rt, &L.fin_ev);
+  if (s) return s;
   if (L.cov) CUDA_TRY(cudaMemsetAsync(L.cov, 0, N * 4, L.exec));
   if (fresh_cb) CUDA_TRY(cudaMemsetAsync(L.dmem, 0, sizeof(ControlBlock), L.exec));
   rt->launches[L.id] = std::move(Lp);
@@ -542,7 +649,7 @@ flep_status flep_preempt(flep_rt rt, flep_launch_t h, uint32_t n_sms) {
   if (rt->opt.policy != FLEP_POLICY_MANUAL) return fail(FLEP_ERR_STATE, "preempt is policy-driven in managed mode");
   Launch* L = find(rt, h);
   if (!L) return fail(FLEP_ERR_INVALID, "unknown launch %lld", (long long)h);
-  refresh(*L);
+  refresh(rt, *L);
   if (L->state != FLEP_STATE_RUNNING && L->state != FLEP_STATE_PARTIAL)
     return fail(FLEP_ERR_STATE, "launch %lld is not running (state %d)", (long long)h, L->state);
   const uint32_t n = std::min<uint32_t>(n_sms, rt->num_sms);
@@ -561,7 +668,7 @@ flep_status flep_resume(flep_rt rt, flep_launch_t h) {
   if (rt->opt.policy != FLEP_POLICY_MANUAL) return fail(FLEP_ERR_STATE, "resume is policy-driven in managed mode");
   Launch* L = find(rt, h);
   if (!L) return fail(FLEP_ERR_INVALID, "unknown launch %lld", (long long)h);
-  refresh(*L);
+  refresh(rt, *L);
   if (L->state == FLEP_STATE_PREEMPTED) return start_epoch(rt, *L);
   if (L->state == FLEP_STATE_PARTIAL) {
     flep_status s = write_ctrl(rt, *L, ctrl_word(*L, 0));
@@ -581,7 +688,7 @@ flep_status flep_wait_epoch(flep_rt rt, flep_launch_t h, int64_t timeout_ns) {
       std::lock_guard<std::mutex> lk(rt->mu);
       Launch* L = find(rt, h);
       if (!L) return fail(FLEP_ERR_INVALID, "unknown launch %lld", (long long)h);
-      refresh(*L);
+      refresh(rt, *L);
       if (L->state == FLEP_STATE_PREEMPTED || L->state == FLEP_STATE_DONE || L->state == FLEP_STATE_QUEUED)
         return FLEP_OK;
     }
@@ -594,23 +701,24 @@ flep_status flep_wait_epoch(flep_rt rt, flep_launch_t h, int64_t timeout_ns) {
 flep_status flep_sync(flep_rt rt, flep_launch_t h, int64_t timeout_ns) {
   if (!rt) return fail(FLEP_ERR_INVALID, "rt is NULL");
   const int64_t t0 = now_ns();
-  cudaStream_t exec = nullptr;
+  cudaEvent_t fin = nullptr;
   while (true) {
     {
       std::lock_guard<std::mutex> lk(rt->mu);
       Launch* L = find(rt, h);
       if (!L) return fail(FLEP_ERR_INVALID, "unknown launch %lld", (long long)h);
-      if (rt->opt.policy == FLEP_POLICY_MANUAL) refresh(*L);
-      if (L->state == FLEP_STATE_DONE) { exec = L->exec; break; }
+      if (rt->opt.policy == FLEP_POLICY_MANUAL) refresh(rt, *L);
+      if (L->state == FLEP_STATE_DONE) { fin = L->released ? nullptr : L->fin_ev; break; }
       if (rt->opt.policy == FLEP_POLICY_MANUAL && L->state == FLEP_STATE_PREEMPTED)
         return fail(FLEP_ERR_STATE, "launch %lld is preempted; resume it first", (long long)h);
     }
     if (timeout_ns >= 0 && now_ns() - t0 > timeout_ns) return fail(FLEP_ERR_TIMEOUT, "launch not done");
     std::this_thread::yield();
   }
-  if (exec) CUDA_TRY(cudaStreamSynchronize(exec));
+  if (fin) CUDA_TRY(cudaEventSynchronize(fin));
   std::lock_guard<std::mutex> lk(rt->mu);
   Launch* L = find(rt, h);
+  if (rt->opt.policy != FLEP_POLICY_MANUAL) return FLEP_OK;   // the monitor releases at DONE
   // keep the newest finished launches' device logs (coverage, events) for debug copies
   // (64 with the coverage log, else the last 4; the warm pool keeps launches allocation-free)
   const size_t kRetain = rt->opt.debug_coverage ? 64 : 4;
@@ -629,7 +737,7 @@ flep_status flep_query(flep_rt rt, flep_launch_t h, flep_launch_info* out) {
   std::lock_guard<std::mutex> lk(rt->mu);
   Launch* L = find(rt, h);
   if (!L) return fail(FLEP_ERR_INVALID, "unknown launch %lld", (long long)h);
-  if (rt->opt.policy == FLEP_POLICY_MANUAL) refresh(*L);
+  if (rt->opt.policy == FLEP_POLICY_MANUAL) refresh(rt, *L);
   memset(out, 0, sizeof(*out));
   out->state = L->state;
   out->epoch = L->epoch;
@@ -657,7 +765,7 @@ flep_status flep_cancel(flep_rt rt, flep_launch_t h) {
     std::lock_guard<std::mutex> lk(rt->mu);
     Launch* L = find(rt, h);
     if (!L) return fail(FLEP_ERR_INVALID, "unknown launch %lld", (long long)h);
-    refresh(*L);
+    refresh(rt, *L);
     if (L->state == FLEP_STATE_DONE) return FLEP_OK;
     if (L->state == FLEP_STATE_RUNNING || L->state == FLEP_STATE_PARTIAL || L->state == FLEP_STATE_YIELDING) {
       write_ctrl(rt, *L, ctrl_word(*L, 0xffffu));
@@ -668,7 +776,7 @@ flep_status flep_cancel(flep_rt rt, flep_launch_t h) {
   for (;;) {
     std::lock_guard<std::mutex> lk(rt->mu);
     Launch* L = find(rt, h);
-    refresh(*L);
+    refresh(rt, *L);
     if (L->state != FLEP_STATE_YIELDING) break;
   }
   std::lock_guard<std::mutex> lk(rt->mu);
@@ -694,11 +802,14 @@ flep_status flep_shutdown(flep_rt rt) {
   cudaDeviceSynchronize();
   for (auto& kv : rt->launches) {
     Launch& L = *kv.second;
+    for (cudaEvent_t e : L.evpool) cudaEventDestroy(e);
+    for (auto& e : L.inflight) cudaEventDestroy(e.first);
     if (!L.released) {
       if (L.dmem) cudaFree(L.dmem);
       if (L.cov) cudaFree(L.cov);
     }
   }
+  for (cudaEvent_t e : rt->event_pool) cudaEventDestroy(e);
   for (void* p : rt->free_dmem) cudaFree(p);
   for (auto& c : rt->free_cov) cudaFree(c.first);
   for (cudaStream_t s : rt->all_streams) cudaStreamDestroy(s);
@@ -751,7 +862,7 @@ flep_status flep_debug_trigger_at(flep_rt rt, flep_launch_t h, uint64_t block_in
   std::lock_guard<std::mutex> lk(rt->mu);
   Launch* L = find(rt, h);
   if (!L) return fail(FLEP_ERR_INVALID, "unknown launch %lld", (long long)h);
-  refresh(*L);
+  refresh(rt, *L);
   if (L->state != FLEP_STATE_PREEMPTED && L->state != FLEP_STATE_QUEUED)
     return fail(FLEP_ERR_STATE, "trigger can only be set for the next epoch of a launch that is not running");
   L->trig_block = block_index >= 0xffffffffull ? kNoTrigger : (uint32_t)block_index;
