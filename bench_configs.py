@@ -214,6 +214,21 @@ def run_corun1(args, rank, world, local):
 
 
 # ------------------------------------------------------------------------------------------
+def assign_jobs(jobs, t_e_of, world):
+    """One job queue feeding `world` independent per-GPU schedulers (configs[4]): each arrival
+    goes to the GPU whose predicted backlog (sum of T_e of the work assigned to it that is not
+    yet predicted to be done) ends first; ties -> lowest index. Deterministic, so every rank
+    computes the same partition without communication. Returns one job list per GPU."""
+    backlog_end = [0] * world
+    out = [[] for _ in range(world)]
+    for j in jobs:
+        avail = [max(b, j["arrival_ns"]) for b in backlog_end]
+        r = min(range(world), key=lambda i: (avail[i], i))
+        backlog_end[r] = avail[r] + int(t_e_of(j))
+        out[r].append(j)
+    return out
+
+
 QUEUE_CHUNK = {"saxpy_f32": (8, False), "spmv": (2, True), "stencil_f32": (2, True), "gemm_bf16": (1, False)}
 
 
@@ -325,17 +340,7 @@ def run_queue(args, rank, world, local):
                                 for j in gen.queue_trace(5, n_total, 1)]))
     gap = int(mean_alone / args.rho)
     full = gen.queue_trace(6 if world > 1 else 5, n_total, gap)
-    # one job queue -> N schedulers: least predicted backlog (sum of T_e of assigned work not yet
-    # expected to be done), ties -> lowest index; every rank computes the same assignment
-    backlog_end = [0] * world
-    mine = []
-    for j in full:
-        te = t_alone[(j["type"], j["size_class"])]
-        avail = [max(b, j["arrival_ns"]) for b in backlog_end]
-        r = int(np.argmin(avail))
-        backlog_end[r] = avail[r] + te
-        if r == rank:
-            mine.append(j)
+    mine = assign_jobs(full, lambda j: t_alone[(j["type"], j["size_class"])], world)[rank]
     overhead_ns = 20_000
     res = {}
     debug = {}

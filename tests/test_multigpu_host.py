@@ -1,0 +1,68 @@
+"""Host-side logic of the N > 1 path on CPU with the gloo backend (world size 2): the one-queue
+-> N-schedulers partition is identical on every rank, disjoint and complete, and the timing
+reduction is a max over ranks (BASELINE configs[4]; replicas, no data-path
+collective)."""
+import os
+import socket
+
+import pytest
+
+from synth import gen
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _worker(rank, world, port, q):
+    import torch
+    import torch.distributed as dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    import bench_configs
+    jobs = gen.queue_trace(6, 128, 50_000)
+    te = {("saxpy_f32", 0): 10_000, ("saxpy_f32", 1): 80_000, ("saxpy_f32", 2): 900_000}
+    parts = bench_configs.assign_jobs(jobs, lambda j: te.get((j["type"], j["size_class"]),
+                                                              20_000 * (1 + j["size_class"])), world)
+    mine = [j["id"] for j in parts[rank]]
+    # the max-over-ranks timing reduction used by bench.py
+    t = torch.tensor([float(rank + 1), float(len(mine))], dtype=torch.float64)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    allparts = [None] * world
+    dist.all_gather_object(allparts, mine)
+    q.put((rank, [[j["id"] for j in p] for p in parts], allparts, t.tolist()))
+    dist.destroy_process_group()
+
+
+def test_job_queue_partition_gloo_world2():
+    import torch.multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=120) for _ in procs]
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    res.sort()
+    (r0, parts0, gathered0, red0), (r1, parts1, gathered1, red1) = res
+    assert parts0 == parts1                         # same partition computed on every rank
+    assert gathered0[0] == parts0[0] and gathered0[1] == parts0[1]
+    ids = sorted(parts0[0] + parts0[1])
+    assert ids == list(range(128))                  # complete and disjoint
+    assert len(parts0[0]) > 20 and len(parts0[1]) > 20
+    assert red0 == red1 and red0[0] == 2.0           # max over ranks
+
+
+def test_assign_jobs_single_gpu_keeps_order():
+    import bench_configs
+    jobs = gen.queue_trace(5, 40, 10_000)
+    parts = bench_configs.assign_jobs(jobs, lambda j: 1000, 1)
+    assert [j["id"] for j in parts[0]] == list(range(40))

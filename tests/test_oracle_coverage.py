@@ -24,6 +24,21 @@ def test_exhaustive_no_violations_fig2(C, K):
     assert r.preempted_epoch_ends > 0      # preempted epochs really are explored
 
 
+@pytest.mark.parametrize("C,K", [(1, 1), (1, 2), (2, 1)])
+def test_exhaustive_prefetch_no_violations(C, K):
+    # chunk prefetch (R3): a stopping worker still runs the chunk it holds
+    r = cv.explore(_cfg(n_blocks=4 if C == 1 else 5, chunk=C, poll=K, worker_sm=(0, 0, 1), prefetch=True))
+    assert r.violations == set()
+    assert r.preempted_epoch_ends > 0
+
+
+def test_prefetch_final_counter_closed_form():
+    for n, C, ws in [(5, 1, (0, 0, 1, 1)), (7, 2, (0, 1))]:
+        r = cv.explore(cv.Config(n_blocks=n, chunk=C, poll=1, worker_sm=ws, num_sms=2, prefetch=True))
+        assert r.violations == set()
+        assert r.terminal_ctrs == {cv.final_counter_no_preempt(n, C, len(ws))}
+
+
 def test_exhaustive_with_clear_events():
     r = cv.explore(_cfg(n_blocks=6, chunk=2, poll=2, allow_clear=True))
     assert r.violations == set()
