@@ -42,7 +42,8 @@ def needs_build() -> bool:
 def build(force: bool = False, verbose: bool = False) -> str:
     if not force and not needs_build():
         return LIB
-    cmd = [_nvcc()] + NVCC_FLAGS + ["-o", LIB + ".tmp"] + sources() + ["-lpthread"]
+    extra = os.environ.get("FLEP_NVCC_EXTRA", "").split()     # experiment hook (e.g. -DFLEP_SPMV_U=4)
+    cmd = [_nvcc()] + NVCC_FLAGS + extra + ["-o", LIB + ".tmp"] + sources() + ["-lpthread"]
     if verbose:
         print(" ".join(cmd), file=sys.stderr)
     r = subprocess.run(cmd, capture_output=True, text=True)

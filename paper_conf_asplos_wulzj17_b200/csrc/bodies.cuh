@@ -14,6 +14,10 @@
 #include "../../include/flep.h"
 #include "flep_device.cuh"
 
+#ifndef FLEP_SPMV_U
+#define FLEP_SPMV_U 4
+#endif
+
 namespace flep {
 
 __device__ __forceinline__ int4 ldcs4(const int4* p) { return __ldcs(p); }
@@ -107,7 +111,7 @@ struct SpmvBody : NoResources {
       float acc = 0.f;
       for (int32_t base = p0; base < p1; base += (int32_t)kTile) {
         const int32_t n = min((int32_t)kTile, p1 - base);
-        constexpr int U = 4;
+        constexpr int U = FLEP_SPMV_U;
         for (int32_t i0 = (int32_t)tid; i0 < n; i0 += U * kThreads) {
           int32_t c[U];
           float v[U], xv[U];
