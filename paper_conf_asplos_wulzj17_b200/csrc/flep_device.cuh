@@ -201,10 +201,12 @@ flep_worker(const __grid_constant__ typename Body::Args args, const WorkerParams
       p.cb->ep_t_trigger[(p.epoch + 1) % kEvEpochs] = 0;  // next epoch's trigger stamp
       if (st == kStateDone) { p.cb->done_exited = 0ull; p.cb->ctr = 0; }   // clean for reuse
       else p.cb->done_exited = (unsigned long long)d;    // exits reset, progress kept
-      st_relaxed_sys(&p.status->ctr, c);
-      st_relaxed_sys_u64(&p.status->t_end, t_exit);
-      st_relaxed_sys_u64(reinterpret_cast<uint64_t*>(&p.status->word),
-                         ((uint64_t)d << 32) | ((p.epoch << 8) | st));
+      if (p.status) {
+        st_relaxed_sys(&p.status->ctr, c);
+        st_relaxed_sys_u64(&p.status->t_end, t_exit);
+        st_relaxed_sys_u64(reinterpret_cast<uint64_t*>(&p.status->word),
+                           ((uint64_t)d << 32) | ((p.epoch << 8) | st));
+      }
     }
   }
 }

@@ -46,7 +46,7 @@ struct GemmBody {
     uint32_t tmem_base;
     uint32_t p_stage, p_phase;        // producer
     uint32_t m_stage, m_phase, m_acc; // MMA issuer
-    uint32_t e_acc;                   // epilogue
+    uint32_t e_acc[4];                // epilogue, one copy per epilogue warp (no cross-warp WAR)
   };
 
   __device__ static uint8_t* ring() {
@@ -93,7 +93,8 @@ struct GemmBody {
       for (uint32_t i = 0; i < STAGES; ++i) { mbar_init(&s->full[i], 1); mbar_init(&s->empty[i], 1); }
       mbar_init(&s->tmem_full, 1);
       mbar_init(&s->tmem_empty, 128);
-      s->p_stage = s->p_phase = s->m_stage = s->m_phase = s->m_acc = s->e_acc = 0;
+      s->p_stage = s->p_phase = s->m_stage = s->m_phase = s->m_acc = 0;
+      s->e_acc[0] = s->e_acc[1] = s->e_acc[2] = s->e_acc[3] = 0;
       asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     if (warp == 2) {
@@ -168,7 +169,7 @@ struct GemmBody {
       }
     } else if (warp >= 4) {                                // ---- epilogue (128 threads)
       const uint32_t q = warp - 4;                         // TMEM lanes [32q, 32q+32)
-      uint32_t acc = s->e_acc;
+      uint32_t acc = s->e_acc[q];
       const uint32_t tmem = s->tmem_base + ((q * 32u) << 16);
       for (uint32_t b = b0; b < b1; ++b) {
         const uint32_t tm = b / gx, tn = b % gx;
@@ -203,7 +204,8 @@ struct GemmBody {
         mbar_arrive(&s->tmem_empty);
         acc ^= 1u;
       }
-      if (threadIdx.x == 128) s->e_acc = acc;
+      __syncwarp();
+      if (lane == 0) s->e_acc[q] = acc;
     }
   }
 };

@@ -1,0 +1,50 @@
+"""Small wrapped launches for compute-sanitizer (memcheck / racecheck / synccheck): every body,
+one temporal and one spatial preemption with resume."""
+import os
+import sys
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+from synth import gen  # noqa: E402
+
+
+def main():
+    import torch
+    from paper_conf_asplos_wulzj17_b200 import build, flep as F
+    build.build()
+    T = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()  # noqa: E731
+    rt = F.Runtime(coverage=True)
+    n = 1 << 14
+    x, y = gen.saxpy_i32_inputs(n, 1)
+    xd, yd = T(x), T(y)
+    k = rt.register_kernel(F.BODY_SAXPY_I32, chunk=1, poll=1, ctas_per_sm=1)
+    for nsm in (rt.num_sms, 8):
+        rt.arm_next_trigger(n // 512, nsm)
+        h = rt.launch(k, F.saxpy_grid(n), F.saxpy_i32_args(yd, xd, 3))
+        rt.wait_epoch(h)
+        if rt.query(h).state == F.STATE_PREEMPTED:
+            rt.resume(h)
+        rt.sync(h)
+    rp, col, val, xv = gen.csr_inputs(2000, 2)
+    yv = torch.zeros(2000, device="cuda")
+    k2 = rt.register_kernel(F.BODY_SPMV_CSR_F32, chunk=2, poll=1, prefetch=True)
+    rt.sync(rt.launch(k2, F.spmv_grid(2000), F.spmv_args(yv, T(rp), T(col), T(val), T(xv))))
+    st = T(gen.stencil_f32_input(200, 3))
+    out = torch.empty_like(st)
+    k3 = rt.register_kernel(F.BODY_STENCIL5_F32, chunk=1, poll=1)
+    rt.sync(rt.launch(k3, F.stencil_grid(200), F.stencil_args(out, st)))
+    a_bits, b_bits = gen.gemm_bf16_inputs(256, 512, 128, 4)
+    A = torch.from_numpy(a_bits.view(np.int16)).cuda().view(torch.bfloat16)
+    B = torch.from_numpy(b_bits.view(np.int16)).cuda().view(torch.bfloat16)
+    C = torch.empty(256, 512, dtype=torch.bfloat16, device="cuda")
+    k4 = rt.register_kernel(F.BODY_GEMM_BF16, chunk=1, poll=1)
+    rt.sync(rt.launch(k4, F.gemm_grid(256, 512), F.gemm_args(C, A, B)))
+    torch.cuda.synchronize()
+    rt.close()
+    print("sanitizer case done")
+
+
+if __name__ == "__main__":
+    main()
