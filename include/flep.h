@@ -63,7 +63,10 @@ typedef enum {
   FLEP_POLICY_MANUAL = 0,  /* caller issues preempt/resume itself (mechanism only) */
   FLEP_POLICY_FIFO = 1,    /* interception, no preemption, arrival order (MPS co-run baseline) */
   FLEP_POLICY_HPF = 2,     /* Fig. 6: priority preemption + SRPT within a priority (§5.2.1) */
-  FLEP_POLICY_SLICE = 3    /* HPF decisions on the kernel-slicing mechanism (P:96, P:391 baseline) */
+  FLEP_POLICY_SLICE = 3,   /* HPF decisions on the kernel-slicing mechanism (P:96, P:391 baseline) */
+  FLEP_POLICY_FFS = 4      /* fairness first under an overhead constraint: weighted round robin,
+                              epoch T*W_i, W_i = priority+1, T minimal with
+                              sum O_i / (T sum W_i) <= max_overhead (§5.2.2) */
 } flep_policy;
 
 typedef enum {
@@ -108,6 +111,7 @@ typedef struct {
                                   caller's stream instead of a runtime stream. Stream order then
                                   only covers the epoch grids: the caller must resume before
                                   enqueuing work that depends on the results. */
+  uint32_t max_overhead_ppm;   /* FFS: max_overhead in parts per million (0 -> 100000 = 10%) */
 } flep_options;
 
 typedef struct {
@@ -232,13 +236,14 @@ flep_status flep_set_rank_table(flep_rt rt, const uint16_t* rank, uint32_t n);
 int64_t flep_now_ns(void);
 /* Decision log of the managed runtime: n records of (t_ns, action, launch, n_sms) with
    action 0 = LAUNCH, 1 = RESUME, 2 = PREEMPT; and the event log (t_ns, type, launch) with
-   type 0 = ARRIVE, 1 = FINISH, plus per-launch (priority, t_e, overhead). */
+   type 0 = ARRIVE, 1 = FINISH, 2 = TICK (FFS epoch expiry; launch = -1), plus per-launch
+   (priority, t_e, overhead). */
 flep_status flep_decision_log(flep_rt rt, int64_t* out4, size_t max_records, size_t* n_out);
 flep_status flep_event_log(flep_rt rt, int64_t* out6, size_t max_records, size_t* n_out);
 
 /* ---- pure policy engine (host only; no GPU needed) -------------------------------------
    The exact decision logic the managed runtime uses (Fig. 6), exposed for replay parity with
-   the oracle's discrete-event simulation. kind: 1 FIFO, 2 HPF, 3 SLICE (= HPF decisions). */
+   the oracle's discrete-event simulation. kind: 1 FIFO, 2 HPF, 3 SLICE (= HPF decisions), 4 FFS. */
 typedef struct flep_policy_s* flep_policy_t;
 flep_status flep_policy_create(int32_t kind, uint32_t num_sms, flep_policy_t* out);
 flep_status flep_policy_destroy(flep_policy_t p);
@@ -248,6 +253,11 @@ flep_status flep_policy_finish(flep_policy_t p, int64_t t_ns, int64_t id);
 /* Decisions emitted so far: records of 4 int64 (t_ns, action, id, n_sms). */
 flep_status flep_policy_decisions(flep_policy_t p, int64_t* out4, size_t max_records,
                                   size_t* n_out);
+/* FFS (kind 4): epoch-expiry check at time t; *acted = 1 iff it changed the schedule.
+   Other kinds: no-op. */
+flep_status flep_policy_tick(flep_policy_t p, int64_t t_ns, int32_t* acted);
+/* FFS max_overhead in ppm (default 100000). */
+flep_status flep_policy_set_max_overhead(flep_policy_t p, uint32_t ppm);
 /* T_e ns from a 5-term model, rounded once (half away from zero), clamped >= 1. */
 int64_t flep_model_predict_ns(const double model[5], double grid, double cta, double input,
                               double smem);

@@ -379,6 +379,13 @@ void monitor_loop(flep_rt rt) {
           }
         }
       }
+      if (rt->opt.policy == FLEP_POLICY_FFS) {               // FFS epochs are time-driven
+        const int64_t t = now_ns();
+        if (rt->policy->tick(t)) {
+          rt->evlog.push_back({t, 2, -1, 0, 0, 0});
+          apply_decisions(rt);
+        }
+      }
       for (size_t i = 0; i < rt->to_release.size();) {      // recycle finished launches
         Launch* R = find(rt, rt->to_release[i]);
         if (R && cudaEventQuery(R->fin_ev) == cudaSuccess) {
@@ -443,7 +450,7 @@ flep_status flep_init(int device, const flep_options* opts, flep_rt* out) {
   if (opts) rt->opt = *opts;
   if (rt->opt.default_chunk == 0) rt->opt.default_chunk = 8;
   if (rt->opt.default_poll == 0) rt->opt.default_poll = 1;
-  if (rt->opt.policy < FLEP_POLICY_MANUAL || rt->opt.policy > FLEP_POLICY_SLICE)
+  if (rt->opt.policy < FLEP_POLICY_MANUAL || rt->opt.policy > FLEP_POLICY_FFS)
     return fail(FLEP_ERR_INVALID, "bad policy %d", rt->opt.policy);
   cudaDeviceProp prop;
   CUDA_TRY(cudaGetDeviceProperties(&prop, device));
@@ -482,7 +489,8 @@ flep_status flep_init(int device, const flep_options* opts, flep_rt* out) {
     }
   }
   if (rt->opt.policy != FLEP_POLICY_MANUAL) {
-    rt->policy.reset(new Policy(rt->opt.policy, rt->num_sms));
+    rt->policy.reset(new Policy(rt->opt.policy == FLEP_POLICY_SLICE ? (int32_t)kPolicyHPF : rt->opt.policy,
+                                rt->num_sms, rt->opt.max_overhead_ppm ? rt->opt.max_overhead_ppm : 100000));
     flep_rt raw = rt.get();
     rt->monitor = std::thread([raw] { monitor_loop(raw); });
   }
@@ -967,9 +975,23 @@ struct flep_policy_s {
   flep_policy_s(int32_t k, uint32_t n) : p(k, n) {}
 };
 
+flep_status flep_policy_tick(flep_policy_t p, int64_t t, int32_t* acted) {
+  if (!p) return fail(FLEP_ERR_INVALID, "NULL policy");
+  const bool a = p->p.tick(t);
+  if (acted) *acted = a ? 1 : 0;
+  return FLEP_OK;
+}
+
+flep_status flep_policy_set_max_overhead(flep_policy_t p, uint32_t ppm) {
+  if (!p) return fail(FLEP_ERR_INVALID, "NULL policy");
+  if (ppm == 0) return fail(FLEP_ERR_INVALID, "max_overhead must be > 0");
+  p->p.set_max_overhead_ppm(ppm);
+  return FLEP_OK;
+}
+
 flep_status flep_policy_create(int32_t kind, uint32_t num_sms, flep_policy_t* out) {
   if (!out) return fail(FLEP_ERR_INVALID, "out is NULL");
-  if (kind < kPolicyFIFO || kind > kPolicySLICE) return fail(FLEP_ERR_INVALID, "bad policy kind %d", kind);
+  if (kind < kPolicyFIFO || kind > kPolicyFFS) return fail(FLEP_ERR_INVALID, "bad policy kind %d", kind);
   *out = new flep_policy_s(kind == kPolicySLICE ? kPolicyHPF : kind, num_sms);
   return FLEP_OK;
 }

@@ -13,7 +13,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(HERE, "libflep.so")
 
 OK, ERR_INVALID, ERR_STATE, ERR_CUDA, ERR_NOMEM, ERR_TIMEOUT, ERR_UNSUPPORTED = 0, -1, -2, -3, -4, -5, -6
-POLICY_MANUAL, POLICY_FIFO, POLICY_HPF, POLICY_SLICE = 0, 1, 2, 3
+POLICY_MANUAL, POLICY_FIFO, POLICY_HPF, POLICY_SLICE, POLICY_FFS = 0, 1, 2, 3, 4
 FLAG_STREAM_MEMOP, FLAG_HOST_MAPPED = 0, 1
 BODY_SAXPY_I32, BODY_SAXPY_F32, BODY_SPMV_CSR_F32, BODY_STENCIL5_F32, BODY_STENCIL5_I32, BODY_GEMM_BF16 = 1, 2, 3, 4, 5, 6
 STATE_QUEUED, STATE_RUNNING, STATE_YIELDING, STATE_PREEMPTED, STATE_PARTIAL, STATE_DONE = 0, 1, 2, 3, 4, 5
@@ -54,7 +54,7 @@ class Options(C.Structure):
     _fields_ = [("policy", C.c_int32), ("flag", C.c_int32), ("default_chunk", C.c_uint32),
                 ("default_poll", C.c_uint32), ("debug_coverage", C.c_uint32),
                 ("reserved0", C.c_uint32), ("slice_blocks", C.c_uint32),
-                ("exec_on_user_stream", C.c_uint32)]
+                ("exec_on_user_stream", C.c_uint32), ("max_overhead_ppm", C.c_uint32)]
 
 
 class KernelDesc(C.Structure):
@@ -116,6 +116,8 @@ _SIG = {
     "flep_policy_arrive": (C.c_int, [_P, C.c_int64, C.c_int64, C.c_int32, C.c_int64, C.c_int64]),
     "flep_policy_finish": (C.c_int, [_P, C.c_int64, C.c_int64]),
     "flep_policy_decisions": (C.c_int, [_P, C.POINTER(C.c_int64), C.c_size_t, C.POINTER(C.c_size_t)]),
+    "flep_policy_tick": (C.c_int, [_P, C.c_int64, C.POINTER(C.c_int32)]),
+    "flep_policy_set_max_overhead": (C.c_int, [_P, C.c_uint32]),
     "flep_model_predict_ns": (C.c_int64, [C.POINTER(C.c_double), C.c_double, C.c_double, C.c_double,
                                           C.c_double]),
     "flep_last_error": (C.c_char_p, []),
@@ -173,10 +175,10 @@ class Runtime:
     """One FLEP runtime on one device (flep_init ... flep_shutdown)."""
 
     def __init__(self, device=0, policy=POLICY_MANUAL, flag=FLAG_STREAM_MEMOP, chunk=8, poll=1,
-                 coverage=False, slice_blocks=0, exec_on_user_stream=False):
+                 coverage=False, slice_blocks=0, exec_on_user_stream=False, max_overhead_ppm=0):
         self.L = lib()
         o = Options(policy, flag, chunk, poll, int(coverage), 0, slice_blocks,
-                    int(exec_on_user_stream))
+                    int(exec_on_user_stream), max_overhead_ppm)
         h = C.c_void_p()
         check(self.L.flep_init(device, C.byref(o), C.byref(h)), "flep_init")
         self.h = h
@@ -315,6 +317,14 @@ class PolicyEngine:
 
     def finish(self, t, kid):
         check(self.L.flep_policy_finish(self.h, t, kid), "flep_policy_finish")
+
+    def tick(self, t):
+        a = C.c_int32()
+        check(self.L.flep_policy_tick(self.h, t, C.byref(a)), "flep_policy_tick")
+        return bool(a.value)
+
+    def set_max_overhead(self, ppm):
+        check(self.L.flep_policy_set_max_overhead(self.h, ppm), "flep_policy_set_max_overhead")
 
     def decisions(self):
         n = C.c_size_t()

@@ -201,3 +201,38 @@ def test_cancel_then_reuse_control_block():
             assert np.array_equal(y2d.cpu().numpy(), W.saxpy_i32(11, x2, y2))
     finally:
         rt.close()
+
+
+def test_managed_ffs_share_and_replay():
+    """FFS (§5.2.2): two long kernels of priorities 1 and 0 (weights 2:1) share the GPU in epochs;
+    the runtime's decisions replay exactly through the oracle FFS (TICK events logged)."""
+    f = flep_mod()
+    import torch
+    rt = f.Runtime(policy=f.POLICY_FFS, max_overhead_ppm=100_000)
+    try:
+        n = 1 << 28
+        x1, y1 = torch.ones(n, dtype=torch.int32, device="cuda"), torch.ones(n, dtype=torch.int32, device="cuda")
+        x2, y2 = torch.ones(n, dtype=torch.int32, device="cuda"), torch.ones(n, dtype=torch.int32, device="cuda")
+        k = rt.register_kernel(f.BODY_SAXPY_I32, chunk=8, poll=1, overhead_ns=20_000, model=(0, 0, 0, 0, 500_000))
+        sA, sB = torch.cuda.Stream(), torch.cuda.Stream()
+        h1 = rt.launch(k, f.saxpy_grid(n), f.saxpy_i32_args(y1, x1, 2), priority=1, stream=sA)
+        h2 = rt.launch(k, f.saxpy_grid(n), f.saxpy_i32_args(y2, x2, 3), priority=0, stream=sB)
+        rt.sync(h1, timeout_ns=20_000_000_000)
+        rt.sync(h2, timeout_ns=20_000_000_000)
+        torch.cuda.synchronize()
+        assert int(y1[0].item()) == 3 and int(y1[-1].item()) == 3
+        assert int(y2[12345].item()) == 4
+        dec = rt.decision_log()
+        assert sum(1 for d in dec if d[1] == 2) >= 2          # the epochs really alternated
+        evs = []
+        for (t_ns, typ, lid, prio, t_e, ovh) in rt.event_log():
+            if typ == 0:
+                evs.append((t_ns, "ARRIVE", des.KernelSpec(lid, t_ns, prio, t_e, ovh)))
+            elif typ == 1:
+                evs.append((t_ns, "FINISH", lid))
+            else:
+                evs.append((t_ns, "TICK", None))
+        rep = [(t, ACT[a], i, n_) for (t, a, i, n_) in des.replay_ffs(evs, 100_000)]
+        assert dec == rep
+    finally:
+        rt.close()

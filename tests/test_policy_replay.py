@@ -75,3 +75,27 @@ def test_ties_and_equal_arrivals(flep):
     assert as_tuples(sim.decisions) == replay_cpp(flep, des.HPF, sim.events)
     order = [d[2] for d in sim.decisions if d[1] in ("LAUNCH", "RESUME")]
     assert order == sorted(order)
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_ffs_replay_parity(flep, seed):
+    g = gen.rng(500 + seed)
+    ks, t = [], 0
+    for i in range(int(g.integers(2, 9))):
+        t += int(g.integers(0, 3_000_000))
+        true = int(g.integers(100_000, 20_000_000))
+        ks.append(des.KernelSpec(i, t, int(g.integers(0, 3)), true, int(g.integers(1_000, 200_000)), true))
+    ppm = int(g.choice([50_000, 100_000, 200_000]))
+    sim = des.simulate_ffs(ks, ppm, des.SimParams(drain_ns=int(g.integers(0, 20_000)), start_ns=5_000))
+    p = flep.PolicyEngine(4)
+    p.set_max_overhead(ppm)
+    for ev in sim.events:
+        if ev[1] == "ARRIVE":
+            s = ev[2]
+            p.arrive(ev[0], s.id, s.priority, s.t_e, s.overhead)
+        elif ev[1] == "FINISH":
+            p.finish(ev[0], ev[2])
+        else:
+            assert p.tick(ev[0])
+    assert as_tuples(sim.decisions) == p.decisions()
+    assert len(sim.finish) == len(ks)

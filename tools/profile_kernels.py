@@ -44,6 +44,12 @@ def main():
         xs = torch.ones(n, dtype=torch.int32, device="cuda")
         ys = torch.ones(n, dtype=torch.int32, device="cuda")
         jobs.append(("saxpy", F.BODY_SAXPY_I32, F.saxpy_grid(n), F.saxpy_i32_args(ys, xs, 3), (xs, ys)))
+    if "gemm" in a.kernels:
+        M = 8192
+        A = (torch.rand(M, M, device="cuda") * 2 - 1).to(torch.bfloat16)
+        B = (torch.rand(M, M, device="cuda") * 2 - 1).to(torch.bfloat16)
+        Cg = torch.empty(M, M, device="cuda", dtype=torch.bfloat16)
+        jobs.append(("gemm", F.BODY_GEMM_BF16, F.gemm_grid(M, M), F.gemm_args(Cg, A, B), (A, B, Cg)))
     s = torch.cuda.current_stream()
     for name, body, grid, args, keep in jobs:
         k = rt.register_kernel(body, chunk=a.chunk, poll=1, prefetch=bool(a.prefetch))
