@@ -517,7 +517,8 @@ def main():
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--impl", default="flep", choices=["flep", "reference"])
-    ap.add_argument("--config", default="temporal", choices=["temporal", "corun1", "spatial", "queue"])
+    ap.add_argument("--config", default="temporal", choices=["temporal", "corun1", "spatial", "queue", "ffs"])
+    ap.add_argument("--ffs-seconds", type=float, default=1.0)
     ap.add_argument("--corun-cps", type=int, default=2)
     ap.add_argument("--queue-kernels", type=int, default=64)
     ap.add_argument("--rho", type=float, default=1.0)
@@ -550,6 +551,8 @@ def main():
             bench_configs.run_spatial(args, rank, world, local)
         elif args.config == "corun1":
             bench_configs.run_corun1(args, rank, world, local)
+        elif args.config == "ffs":
+            bench_configs.run_ffs(args, rank, world, local)
         else:
             bench_configs.run_queue(args, rank, world, local)
 

@@ -396,3 +396,67 @@ def run_queue(args, rank, world, local):
             with open(os.path.join(dbg, "queue_debug.json"), "w") as fh:
                 json.dump(debug, fh)
     barrier(world)
+
+
+# ------------------------------------------------------------------------------------------
+def run_ffs(args, rank, world, local):
+    """FFS experiment (Figs. 13-14): two applications keep invoking the
+    same long kernel (SAXPY-int32 over 2^30 elements, ~2 ms) in a loop, priorities 1 and 0 (weights
+    2:1), max_overhead = 10%. Reports each application's GPU share and the throughput
+    degradation against one application running alone."""
+    import threading
+
+    import torch
+    from bench import barrier
+    from paper_conf_asplos_wulzj17_b200 import flep as F
+    torch.cuda.set_device(local)
+    n = 1 << 30
+    dur = args.ffs_seconds
+    bufs = [(torch.ones(n, dtype=torch.int32, device="cuda"), torch.ones(n, dtype=torch.int32, device="cuda"))
+            for _ in range(2)]
+
+    def loop(rt, k, app, prio, stop_at, counts):
+        x, y = bufs[app]
+        s = torch.cuda.Stream()
+        while F.now_ns() < stop_at:
+            h = rt.launch(k, F.saxpy_grid(n), F.saxpy_i32_args(y, x, 1), priority=prio, stream=s)
+            rt.sync(h, timeout_ns=5_000_000_000)
+            if F.now_ns() <= stop_at:
+                counts[app] += 1
+
+    def run(policy, apps):
+        rt = F.Runtime(device=local, policy=policy, max_overhead_ppm=100_000)
+        k = rt.register_kernel(F.BODY_SAXPY_I32, chunk=8, poll=1, overhead_ns=10_000,
+                               model=(0, 0, 0, 0, 2_000_000))
+        counts = [0, 0]
+        stop_at = F.now_ns() + int(dur * 1e9)
+        th = [threading.Thread(target=loop, args=(rt, k, a, 1 - a, stop_at, counts)) for a in apps]
+        for t_ in th:
+            t_.start()
+        for t_ in th:
+            t_.join()
+        dec = rt.decision_log()
+        evl = rt.event_log()
+        rt.close()
+        import os
+        dbg = os.environ.get("FLEP_EVIDENCE_DIR")
+        if dbg and policy == F.POLICY_FFS:
+            with open(os.path.join(dbg, "ffs_debug.json"), "w") as fh:
+                json.dump({"decisions": dec[-600:], "events": evl[-600:], "n_dec": len(dec), "n_ev": len(evl)}, fh)
+        return counts, sum(1 for d in dec if d[1] == 2)
+
+    alone, _ = run(F.POLICY_FIFO, [0])
+    shared, npre = run(F.POLICY_FFS, [0, 1])
+    tot = shared[0] + shared[1]
+    out = {"metric": METRIC, "value": round(shared[0] / tot, 4) if tot else None, "unit": "GPU share of the weight-2 app",
+           "value_definition": "FFS GPU share of the high-priority (weight 2) application; target 2/3 (P:363)",
+           "n_gpus": world, "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int32",
+           "data": "synthetic", "config": {"workload": "FFS pair: SAXPY-int32 2^30 invoked in a loop by two applications "
+                                                      "(priorities 1, 0), max_overhead 10%", "seconds": dur},
+           "kernels_completed": {"weight2": shared[0], "weight1": shared[1], "alone": alone[0]},
+           "share_weight1": round(shared[1] / tot, 4) if tot else None,
+           "throughput_degradation": round(1 - tot / alone[0], 4) if alone[0] else None,
+           "preemptions": npre}
+    if rank == 0:
+        print(json.dumps(out), flush=True)
+    barrier(world)

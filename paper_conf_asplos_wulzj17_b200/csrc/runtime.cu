@@ -173,11 +173,26 @@ struct flep_rt_s {
   std::vector<int64_t> retained;   // finished launches whose logs are kept for debug copies
   std::vector<cudaEvent_t> event_pool;
   std::vector<int64_t> to_release; // managed mode: DONE launches whose last grid may still run
+  std::atomic<int> waiters{0};      // API threads waiting for `mu`
+  std::vector<int64_t> active_ids;  // managed mode: launches whose state the monitor must poll
+  std::atomic<uint64_t> active_gen{0};   // bumped whenever active_ids grows (wakes the monitor)
 };
 
 namespace {
 
 Launch* find(flep_rt rt, flep_launch_t h);
+
+// Lock taken by API entry points. It announces itself so the spinning monitor thread backs off
+// instead of re-acquiring the (unfair) mutex immediately and starving application threads.
+struct ApiLock {
+  flep_rt rt;
+  std::unique_lock<std::mutex> u;
+  explicit ApiLock(flep_rt r) : rt(r) {
+    rt->waiters.fetch_add(1, std::memory_order_relaxed);
+    u = std::unique_lock<std::mutex>(rt->mu);
+    rt->waiters.fetch_sub(1, std::memory_order_relaxed);
+  }
+};
 
 flep_status occupancy(flep_rt rt, const BodyOps* ops, bool cov, int* k) {
   auto key = std::make_pair(ops->body, cov);
@@ -221,6 +236,13 @@ flep_status write_ctrl(flep_rt rt, Launch& L, uint32_t value) {
   return FLEP_OK;
 }
 
+void mark_active(flep_rt rt, Launch& L) {
+  if (rt->opt.policy == FLEP_POLICY_MANUAL) return;
+  if (std::find(rt->active_ids.begin(), rt->active_ids.end(), L.id) == rt->active_ids.end())
+    rt->active_ids.push_back(L.id);
+  rt->active_gen.fetch_add(1, std::memory_order_release);
+}
+
 flep_status pooled_event(flep_rt rt, cudaEvent_t* e) {
   if (!rt->event_pool.empty()) { *e = rt->event_pool.back(); rt->event_pool.pop_back(); return FLEP_OK; }
   CUDA_TRY(cudaEventCreateWithFlags(e, cudaEventDisableTiming));
@@ -249,6 +271,7 @@ flep_status start_epoch(flep_rt rt, Launch& L) {
     L.state = FLEP_STATE_RUNNING;
     L.n_yield = 0;
     if (L.t_first_start < 0) L.t_first_start = now_ns();
+    mark_active(rt, L);
     return issue_slices(rt, L);
   }
   L.epoch++;
@@ -278,6 +301,7 @@ flep_status start_epoch(flep_rt rt, Launch& L) {
   L.state = FLEP_STATE_RUNNING;
   L.n_yield = 0;
   if (L.t_first_start < 0) L.t_first_start = now_ns();
+  mark_active(rt, L);
   return FLEP_OK;
 }
 
@@ -357,60 +381,111 @@ void apply_decisions(flep_rt rt) {
   }
 }
 
+// One full pass over the active launches (caller holds rt->mu).
+void monitor_pass(flep_rt rt) {
+  bool changed = false;
+  for (int64_t id : rt->active_ids) {
+    Launch* Lp = find(rt, id);
+    if (!Lp) continue;
+    Launch& L = *Lp;
+    if (L.state != FLEP_STATE_RUNNING && L.state != FLEP_STATE_YIELDING && L.state != FLEP_STATE_PARTIAL) continue;
+    if (refresh(rt, L)) {
+      rt->to_release.push_back(L.id);
+      const int64_t t = L.t_finish;
+      rt->evlog.push_back({t, 1, L.id, L.prio, L.t_e, L.overhead});
+      rt->policy->finish(t, L.id);
+      apply_decisions(rt);
+      changed = true;
+    } else if (L.state == FLEP_STATE_PREEMPTED) {
+      changed = true;
+    }
+  }
+  if (rt->opt.policy == FLEP_POLICY_FFS) {               // FFS epochs are time-driven
+    const int64_t t = now_ns();
+    if (rt->policy->tick(t)) {
+      rt->evlog.push_back({t, 2, -1, 0, 0, 0});
+      apply_decisions(rt);
+      changed = true;
+    }
+  }
+  for (size_t i = 0; i < rt->to_release.size();) {      // recycle finished launches
+    Launch* R = find(rt, rt->to_release[i]);
+    if (R && cudaEventQuery(R->fin_ev) == cudaSuccess) {
+      if (rt->opt.debug_coverage) {                    // keep the newest 64 for debug copies
+        rt->retained.push_back(R->id);
+        while (rt->retained.size() > 64) {
+          Launch* old = find(rt, rt->retained.front());
+          rt->retained.erase(rt->retained.begin());
+          if (old) release_resources(rt, *old);
+        }
+      } else {
+        release_resources(rt, *R);
+      }
+      rt->to_release[i] = rt->to_release.back();
+      rt->to_release.pop_back();
+      changed = true;
+    } else {
+      ++i;
+    }
+  }
+  // rebuild the active list
+  std::vector<int64_t> keep;
+  for (int64_t id : rt->active_ids) {
+    Launch* L = find(rt, id);
+    if (L && L->state != FLEP_STATE_DONE && L->state != FLEP_STATE_QUEUED) keep.push_back(id);
+  }
+  rt->active_ids.swap(keep);
+  if (changed) rt->cv.notify_all();
+}
+
+// The completion monitor (a11). It polls the pinned status slots WITHOUT the runtime lock and
+// takes the lock only when something changed (a status word moved, a slice or a completion event
+// may have fired, an FFS epoch deadline passed), so application threads calling the API are
+// never starved by it.
 void monitor_loop(flep_rt rt) {
   cudaSetDevice(rt->device);
+  struct Watch { const uint64_t* word; uint64_t seen; bool sliced; };
+  std::vector<Watch> watch;
+  int64_t deadline = -1;
+  bool pending_release = false;
+  uint64_t gen_seen = ~0ull;
   while (!rt->stop.load(std::memory_order_relaxed)) {
-    bool active = false;
-    {
-      std::unique_lock<std::mutex> lk(rt->mu);
-      for (auto& kv : rt->launches) {
-        Launch& L = *kv.second;
-        if (L.state == FLEP_STATE_RUNNING || L.state == FLEP_STATE_YIELDING || L.state == FLEP_STATE_PARTIAL) {
-          active = true;
-          if (refresh(rt, L)) {
-            rt->to_release.push_back(L.id);
-            const int64_t t = L.t_finish;
-            rt->evlog.push_back({t, 1, L.id, L.prio, L.t_e, L.overhead});
-            rt->policy->finish(t, L.id);
-            apply_decisions(rt);
-            rt->cv.notify_all();
-          } else if (L.state == FLEP_STATE_PREEMPTED) {
-            rt->cv.notify_all();
-          }
-        }
-      }
-      if (rt->opt.policy == FLEP_POLICY_FFS) {               // FFS epochs are time-driven
-        const int64_t t = now_ns();
-        if (rt->policy->tick(t)) {
-          rt->evlog.push_back({t, 2, -1, 0, 0, 0});
-          apply_decisions(rt);
-        }
-      }
-      for (size_t i = 0; i < rt->to_release.size();) {      // recycle finished launches
-        Launch* R = find(rt, rt->to_release[i]);
-        if (R && cudaEventQuery(R->fin_ev) == cudaSuccess) {
-          if (rt->opt.debug_coverage) {                    // keep the newest 64 for debug copies
-            rt->retained.push_back(R->id);
-            while (rt->retained.size() > 64) {
-              Launch* old = find(rt, rt->retained.front());
-              rt->retained.erase(rt->retained.begin());
-              if (old) release_resources(rt, *old);
-            }
-          } else {
-            release_resources(rt, *R);
-          }
-          rt->to_release[i] = rt->to_release.back();
-          rt->to_release.pop_back();
-        } else {
-          ++i;
-        }
-      }
-      if (!active) {
-        rt->cv.wait_for(lk, std::chrono::milliseconds(1));
-        continue;
-      }
+    bool hit = false;
+    if (gen_seen != rt->active_gen.load(std::memory_order_acquire)) hit = true;   // new work
+    for (const Watch& w : watch) {
+      if (w.sliced || __atomic_load_n(w.word, __ATOMIC_ACQUIRE) != w.seen) { hit = true; break; }
     }
-    std::this_thread::yield();
+    if (deadline >= 0 && now_ns() >= deadline) hit = true;
+    if (pending_release) hit = true;
+    if (!hit) {
+      if (watch.empty() && deadline < 0) {
+        std::unique_lock<std::mutex> lk(rt->mu);
+        rt->cv.wait_for(lk, std::chrono::milliseconds(1));
+      } else {
+        for (int i = 0; i < 64; ++i) __builtin_ia32_pause();
+      }
+      continue;
+    }
+    std::unique_lock<std::mutex> lk(rt->mu);
+    gen_seen = rt->active_gen.load(std::memory_order_acquire);
+    // snapshot the status words BEFORE the pass: a word that moves after the pass read it is
+    // then seen as a change on the next poll (at worst one extra pass, never a missed event)
+    std::map<int64_t, uint64_t> snap;
+    for (int64_t id : rt->active_ids) {
+      Launch* L = find(rt, id);
+      if (L && L->hs) snap[id] = __atomic_load_n(reinterpret_cast<const uint64_t*>(&L->hs->word), __ATOMIC_ACQUIRE);
+    }
+    monitor_pass(rt);
+    watch.clear();
+    for (int64_t id : rt->active_ids) {
+      Launch* L = find(rt, id);
+      if (!L || !L->hs) continue;
+      const uint64_t* wp = reinterpret_cast<const uint64_t*>(&L->hs->word);
+      auto it = snap.find(id);
+      watch.push_back({wp, it != snap.end() ? it->second : ~0ull, L->sliced});
+    }
+    deadline = rt->policy->epoch_end();
+    pending_release = !rt->to_release.empty();
   }
 }
 
@@ -508,7 +583,7 @@ flep_status flep_device_info(flep_rt rt, uint32_t* num_sms, uint32_t* nsmid) {
 flep_status flep_register_kernel(flep_rt rt, const flep_kernel_desc* d, flep_kernel* out) {
   if (!rt || !d || !out) return fail(FLEP_ERR_INVALID, "NULL argument");
   if (!body_ops(d->body)) return fail(FLEP_ERR_INVALID, "unknown body %d", d->body);
-  std::lock_guard<std::mutex> lk(rt->mu);
+  ApiLock lk(rt);
   KernelReg k;
   k.name = d->name ? d->name : "";
   k.body = d->body;
@@ -528,7 +603,7 @@ flep_status flep_workers_for(flep_rt rt, int32_t body, uint32_t* ctas_per_sm, ui
   const BodyOps* ops = body_ops(body);
   if (!ops) return fail(FLEP_ERR_INVALID, "unknown body %d", body);
   int k = 0;
-  std::lock_guard<std::mutex> lk(rt->mu);
+  ApiLock lk(rt);
   flep_status s = occupancy(rt, ops, rt->opt.debug_coverage != 0, &k);
   if (s) return s;
   if (ctas_per_sm) *ctas_per_sm = (uint32_t)k;
@@ -540,7 +615,7 @@ flep_status flep_launch(flep_rt rt, flep_kernel kid, flep_dim3 grid, const void*
                         size_t args_size, int32_t priority, flep_stream_t stream,
                         flep_launch_t* out) {
   if (!rt || !args || !out) return fail(FLEP_ERR_INVALID, "NULL argument");
-  std::unique_lock<std::mutex> lk(rt->mu);
+  ApiLock lk(rt);
   if (kid < 0 || (size_t)kid >= rt->kernels.size()) return fail(FLEP_ERR_INVALID, "unknown kernel %d", kid);
   const KernelReg& kr = rt->kernels[kid];
   const BodyOps* ops = body_ops(kr.body);
@@ -653,7 +728,7 @@ flep_status flep_launch(flep_rt rt, flep_kernel kid, flep_dim3 grid, const void*
 flep_status flep_preempt(flep_rt rt, flep_launch_t h, uint32_t n_sms) {
   if (!rt) return fail(FLEP_ERR_INVALID, "rt is NULL");
   if (n_sms == 0) return fail(FLEP_ERR_INVALID, "n_sms == 0");
-  std::lock_guard<std::mutex> lk(rt->mu);
+  ApiLock lk(rt);
   if (rt->opt.policy != FLEP_POLICY_MANUAL) return fail(FLEP_ERR_STATE, "preempt is policy-driven in managed mode");
   Launch* L = find(rt, h);
   if (!L) return fail(FLEP_ERR_INVALID, "unknown launch %lld", (long long)h);
@@ -672,7 +747,7 @@ flep_status flep_preempt(flep_rt rt, flep_launch_t h, uint32_t n_sms) {
 
 flep_status flep_resume(flep_rt rt, flep_launch_t h) {
   if (!rt) return fail(FLEP_ERR_INVALID, "rt is NULL");
-  std::lock_guard<std::mutex> lk(rt->mu);
+  ApiLock lk(rt);
   if (rt->opt.policy != FLEP_POLICY_MANUAL) return fail(FLEP_ERR_STATE, "resume is policy-driven in managed mode");
   Launch* L = find(rt, h);
   if (!L) return fail(FLEP_ERR_INVALID, "unknown launch %lld", (long long)h);
@@ -693,7 +768,7 @@ flep_status flep_wait_epoch(flep_rt rt, flep_launch_t h, int64_t timeout_ns) {
   const int64_t t0 = now_ns();
   while (true) {
     {
-      std::lock_guard<std::mutex> lk(rt->mu);
+      ApiLock lk(rt);
       Launch* L = find(rt, h);
       if (!L) return fail(FLEP_ERR_INVALID, "unknown launch %lld", (long long)h);
       refresh(rt, *L);
@@ -709,22 +784,26 @@ flep_status flep_wait_epoch(flep_rt rt, flep_launch_t h, int64_t timeout_ns) {
 flep_status flep_sync(flep_rt rt, flep_launch_t h, int64_t timeout_ns) {
   if (!rt) return fail(FLEP_ERR_INVALID, "rt is NULL");
   const int64_t t0 = now_ns();
-  cudaEvent_t fin = nullptr;
+  const bool managed = rt->opt.policy != FLEP_POLICY_MANUAL;
   while (true) {
     {
-      std::lock_guard<std::mutex> lk(rt->mu);
+      ApiLock lk(rt);
       Launch* L = find(rt, h);
       if (!L) return fail(FLEP_ERR_INVALID, "unknown launch %lld", (long long)h);
-      if (rt->opt.policy == FLEP_POLICY_MANUAL) refresh(rt, *L);
-      if (L->state == FLEP_STATE_DONE) { fin = L->released ? nullptr : L->fin_ev; break; }
-      if (rt->opt.policy == FLEP_POLICY_MANUAL && L->state == FLEP_STATE_PREEMPTED)
+      if (!managed) refresh(rt, *L);
+      // DONE, and its last grid completed (queried under the lock: in managed mode the monitor
+      // recycles the completion event once it has fired, so never block on it unlocked)
+      if (L->state == FLEP_STATE_DONE && (L->released || cudaEventQuery(L->fin_ev) == cudaSuccess)) break;
+      if (!managed && L->state == FLEP_STATE_PREEMPTED)
         return fail(FLEP_ERR_STATE, "launch %lld is preempted; resume it first", (long long)h);
+      // managed: sleep until the monitor reports a state change (no lock spinning, which would
+      // starve the monitor and the other application threads)
+      if (managed) rt->cv.wait_for(lk.u, std::chrono::microseconds(200));
     }
     if (timeout_ns >= 0 && now_ns() - t0 > timeout_ns) return fail(FLEP_ERR_TIMEOUT, "launch not done");
-    std::this_thread::yield();
+    if (!managed) std::this_thread::yield();
   }
-  if (fin) CUDA_TRY(cudaEventSynchronize(fin));
-  std::lock_guard<std::mutex> lk(rt->mu);
+  ApiLock lk(rt);
   Launch* L = find(rt, h);
   if (rt->opt.policy != FLEP_POLICY_MANUAL) return FLEP_OK;   // the monitor releases at DONE
   // keep the newest finished launches' device logs (coverage, events) for debug copies
@@ -742,7 +821,7 @@ flep_status flep_sync(flep_rt rt, flep_launch_t h, int64_t timeout_ns) {
 
 flep_status flep_query(flep_rt rt, flep_launch_t h, flep_launch_info* out) {
   if (!rt || !out) return fail(FLEP_ERR_INVALID, "NULL argument");
-  std::lock_guard<std::mutex> lk(rt->mu);
+  ApiLock lk(rt);
   Launch* L = find(rt, h);
   if (!L) return fail(FLEP_ERR_INVALID, "unknown launch %lld", (long long)h);
   if (rt->opt.policy == FLEP_POLICY_MANUAL) refresh(rt, *L);
@@ -770,7 +849,7 @@ flep_status flep_query(flep_rt rt, flep_launch_t h, flep_launch_info* out) {
 flep_status flep_cancel(flep_rt rt, flep_launch_t h) {
   if (!rt) return fail(FLEP_ERR_INVALID, "rt is NULL");
   {
-    std::lock_guard<std::mutex> lk(rt->mu);
+    ApiLock lk(rt);
     Launch* L = find(rt, h);
     if (!L) return fail(FLEP_ERR_INVALID, "unknown launch %lld", (long long)h);
     refresh(rt, *L);
@@ -782,12 +861,12 @@ flep_status flep_cancel(flep_rt rt, flep_launch_t h) {
     L->cancelled = true;
   }
   for (;;) {
-    std::lock_guard<std::mutex> lk(rt->mu);
+    ApiLock lk(rt);
     Launch* L = find(rt, h);
     refresh(rt, *L);
     if (L->state != FLEP_STATE_YIELDING) break;
   }
-  std::lock_guard<std::mutex> lk(rt->mu);
+  ApiLock lk(rt);
   Launch* L = find(rt, h);
   if (L->exec) CUDA_TRY(cudaStreamSynchronize(L->exec));
   // the abandoned epoch left ctr/done non-zero: clear the block for reuse
@@ -839,7 +918,7 @@ flep_status flep_launch_unwrapped(flep_rt rt, int32_t body, flep_dim3 grid, cons
   if (s) return s;
   dim3 g(grid.x, grid.y, grid.z);
   if (ops->validate) { const char* m = ops->validate(args, g); if (m) return fail(FLEP_ERR_INVALID, "%s", m); }
-  { int k; std::lock_guard<std::mutex> lk(rt->mu); s = occupancy(rt, ops, false, &k); if (s) return s; }
+  { int k; ApiLock lk(rt); s = occupancy(rt, ops, false, &k); if (s) return s; }
   CUDA_TRY(ops->unwrapped(args, g, 0, 0, (cudaStream_t)stream));
   return FLEP_OK;
 }
@@ -856,7 +935,7 @@ flep_status flep_launch_sliced(flep_rt rt, int32_t body, flep_dim3 grid, const v
   if (s) return s;
   dim3 g(grid.x, grid.y, grid.z);
   if (ops->validate) { const char* m = ops->validate(args, g); if (m) return fail(FLEP_ERR_INVALID, "%s", m); }
-  { int k; std::lock_guard<std::mutex> lk(rt->mu); s = occupancy(rt, ops, false, &k); if (s) return s; }
+  { int k; ApiLock lk(rt); s = occupancy(rt, ops, false, &k); if (s) return s; }
   for (uint64_t off = 0; off < N; off += slice_blocks) {
     const uint32_t cnt = (uint32_t)std::min<uint64_t>(slice_blocks, N - off);
     CUDA_TRY(ops->unwrapped(args, g, (uint32_t)off, cnt, (cudaStream_t)stream));
@@ -867,7 +946,7 @@ flep_status flep_launch_sliced(flep_rt rt, int32_t body, flep_dim3 grid, const v
 flep_status flep_debug_trigger_at(flep_rt rt, flep_launch_t h, uint64_t block_index, uint32_t n_sms) {
   if (!rt) return fail(FLEP_ERR_INVALID, "rt is NULL");
   if (n_sms == 0) return fail(FLEP_ERR_INVALID, "n_sms == 0");
-  std::lock_guard<std::mutex> lk(rt->mu);
+  ApiLock lk(rt);
   Launch* L = find(rt, h);
   if (!L) return fail(FLEP_ERR_INVALID, "unknown launch %lld", (long long)h);
   refresh(rt, *L);
@@ -881,7 +960,7 @@ flep_status flep_debug_trigger_at(flep_rt rt, flep_launch_t h, uint64_t block_in
 flep_status flep_debug_arm_next_trigger(flep_rt rt, uint64_t block_index, uint32_t n_sms) {
   if (!rt) return fail(FLEP_ERR_INVALID, "rt is NULL");
   if (n_sms == 0) return fail(FLEP_ERR_INVALID, "n_sms == 0");
-  std::lock_guard<std::mutex> lk(rt->mu);
+  ApiLock lk(rt);
   rt->arm_block = block_index >= 0xffffffffull ? kNoTrigger : (uint32_t)block_index;
   rt->arm_n = std::min<uint32_t>(n_sms, 0xffff);
   return FLEP_OK;
@@ -889,7 +968,7 @@ flep_status flep_debug_arm_next_trigger(flep_rt rt, uint64_t block_index, uint32
 
 flep_status flep_debug_copy_coverage(flep_rt rt, flep_launch_t h, uint32_t* host_out, size_t n) {
   if (!rt || !host_out) return fail(FLEP_ERR_INVALID, "NULL argument");
-  std::lock_guard<std::mutex> lk(rt->mu);
+  ApiLock lk(rt);
   Launch* L = find(rt, h);
   if (!L) return fail(FLEP_ERR_INVALID, "unknown launch %lld", (long long)h);
   if (!L->cov) return fail(FLEP_ERR_STATE, "coverage log not enabled or already released");
@@ -902,7 +981,7 @@ flep_status flep_debug_copy_coverage(flep_rt rt, flep_launch_t h, uint32_t* host
 flep_status flep_debug_copy_events(flep_rt rt, flep_launch_t h, uint32_t epoch,
                                    flep_worker_event* host_out, size_t max_records, size_t* n_out) {
   if (!rt || !host_out) return fail(FLEP_ERR_INVALID, "NULL argument");
-  std::lock_guard<std::mutex> lk(rt->mu);
+  ApiLock lk(rt);
   Launch* L = find(rt, h);
   if (!L) return fail(FLEP_ERR_INVALID, "unknown launch %lld", (long long)h);
   if (!L->dmem) return fail(FLEP_ERR_STATE, "launch resources already released");
@@ -918,7 +997,7 @@ flep_status flep_debug_copy_events(flep_rt rt, flep_launch_t h, uint32_t epoch,
 
 flep_status flep_debug_epoch_info(flep_rt rt, flep_launch_t h, uint32_t epoch, flep_epoch_info* out) {
   if (!rt || !out) return fail(FLEP_ERR_INVALID, "NULL argument");
-  std::lock_guard<std::mutex> lk(rt->mu);
+  ApiLock lk(rt);
   Launch* L = find(rt, h);
   if (!L) return fail(FLEP_ERR_INVALID, "unknown launch %lld", (long long)h);
   if (!L->dmem) return fail(FLEP_ERR_STATE, "launch resources already released");
@@ -940,7 +1019,7 @@ flep_status flep_debug_epoch_info(flep_rt rt, flep_launch_t h, uint32_t epoch, f
 flep_status flep_set_rank_table(flep_rt rt, const uint16_t* rank, uint32_t n) {
   if (!rt || !rank) return fail(FLEP_ERR_INVALID, "NULL argument");
   if (n < rt->nsmid || n > 256) return fail(FLEP_ERR_INVALID, "rank table needs %u entries", rt->nsmid);
-  std::lock_guard<std::mutex> lk(rt->mu);
+  ApiLock lk(rt);
   CUDA_TRY(cudaMemcpyAsync(rt->d_rank, rank, n * sizeof(uint16_t), cudaMemcpyHostToDevice, rt->ctl));
   CUDA_TRY(cudaStreamSynchronize(rt->ctl));
   return FLEP_OK;
@@ -948,7 +1027,7 @@ flep_status flep_set_rank_table(flep_rt rt, const uint16_t* rank, uint32_t n) {
 
 flep_status flep_decision_log(flep_rt rt, int64_t* out4, size_t max_records, size_t* n_out) {
   if (!rt || !n_out) return fail(FLEP_ERR_INVALID, "NULL argument");
-  std::lock_guard<std::mutex> lk(rt->mu);
+  ApiLock lk(rt);
   if (!rt->policy) { *n_out = 0; return FLEP_OK; }
   const auto& d = rt->policy->decisions();
   const size_t n = std::min(max_records, d.size());
@@ -961,7 +1040,7 @@ flep_status flep_decision_log(flep_rt rt, int64_t* out4, size_t max_records, siz
 
 flep_status flep_event_log(flep_rt rt, int64_t* out6, size_t max_records, size_t* n_out) {
   if (!rt || !n_out) return fail(FLEP_ERR_INVALID, "NULL argument");
-  std::lock_guard<std::mutex> lk(rt->mu);
+  ApiLock lk(rt);
   const size_t n = std::min(max_records, rt->evlog.size());
   for (size_t i = 0; i < n && out6; ++i)
     for (int j = 0; j < 6; ++j) out6[6 * i + j] = rt->evlog[i][j];
