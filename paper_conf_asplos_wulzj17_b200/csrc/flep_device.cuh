@@ -124,72 +124,99 @@ __device__ __forceinline__ bool should_yield(uint32_t c, const WorkerParams& p, 
   return n >= p.num_sms || p.rank[sm] < n;
 }
 
+// Worker bookkeeping shared by every loop shape (kept in shared memory, written by the one
+// scheduling thread).
+struct WorkerShared {
+  uint64_t t_entry;
+  uint32_t sm, blocks, reason;
+};
+
+// The scheduling step of Fig. 4 (b)/(c), executed by ONE thread of the worker: the amortised
+// poll every K chunks, then the task fetch (pull_task) — or the chunk fetched
+// ahead by the previous step when prefetching. Returns the base block of the chunk to run, or
+// 0xffffffff when the worker must leave (yield on request, or counter exhausted). Never returns
+// "leave" while a fetched chunk is held (exactly-once, reading A4). Also fires the device
+// self-trigger of the test/bench hooks.
+struct SchedState {
+  uint32_t k = 0;                    // chunk index within the current poll period
+  uint32_t held = 0xffffffffu;       // prefetched chunk base not yet handed out
+  bool stopping = false;             // a request named this SM; drain the held chunk
+};
+
+__device__ __forceinline__ uint32_t next_chunk(const WorkerParams& p, SchedState& st, WorkerShared& ws) {
+  uint32_t base;
+  if (st.k == 0 && !st.stopping) {                   // amortised poll (Fig. 4(b))
+    const uint32_t c = ld_relaxed_gpu(p.ctrl);
+    if (should_yield(c, p, smid_reg())) { st.stopping = true; ws.reason = kReasonYield; }
+  }
+  if (st.held != 0xffffffffu) {                      // a fetched chunk is always processed (A4)
+    base = st.held;
+    st.held = 0xffffffffu;
+  } else {
+    base = st.stopping ? 0xffffffffu : atomicAdd(&p.cb->ctr, p.chunk);   // pull_task
+  }
+  if (base != 0xffffffffu && base >= p.n_blocks) { base = 0xffffffffu; ws.reason = kReasonExhausted; }
+  if (base != 0xffffffffu) {
+    ws.blocks += min(p.chunk, p.n_blocks - base);
+    if (p.prefetch && !st.stopping) st.held = atomicAdd(&p.cb->ctr, p.chunk);   // overlaps the body
+    if (p.trigger_block - base < p.chunk) {          // device self-trigger inside this chunk
+      const uint32_t e = p.epoch % kEvEpochs;
+      p.cb->ep_t_trigger[e] = gtimer();
+      p.cb->ep_trigger_block[e] = p.trigger_block;
+      atomicExch(p.ctrl, ((p.epoch & 0xffffu) << 16) | (p.trigger_n & 0xffffu));
+    }
+    if (++st.k == p.poll) st.k = 0;
+  }
+  return base;
+}
+
 // The worker. Body contract:
 //   Body::kThreads               CTA size of the original kernel
 //   Body::kMinBlocks             resident CTAs per SM the register budget is sized for
 //   Body::Args                   POD argument struct
-//   Body::run(args, b0, b1, gx, gy)  all threads of the CTA execute original blocks [b0, b1)
-//                                (flat indices b = x + gx*(y + gy*z)), leaving no pending smem
-//                                hazards (the wrapper barrier follows).
+//   Body::setup / teardown(args) per-worker resources (e.g. TMEM), all threads
+//   Body::kPersistent == false:  Body::run(args, b0, b1, gx, gy) — all threads of the CTA execute
+//                                original blocks [b0, b1) (flat b = x + gx*(y + gy*z)); the
+//                                wrapper broadcasts each chunk and keeps one barrier per chunk.
+//   Body::kPersistent == true:   Body::persistent(args, p, ws) owns the loop (warp-specialised
+//                                bodies): its scheduling thread (tid 0) calls next_chunk() and
+//                                hands chunks to the other warps itself, so chunk boundaries
+//                                do not drain its pipeline.
 template <class Body, bool kCoverage>
 __global__ void __launch_bounds__(Body::kThreads, Body::kMinBlocks)
 flep_worker(const __grid_constant__ typename Body::Args args, const WorkerParams p) {
   __shared__ uint32_t s_slot[2];     // chunk base broadcast, double-buffered: 1 barrier per chunk
-  __shared__ uint64_t s_t_entry;     // worker bookkeeping kept out of registers (tid 0 only)
-  __shared__ uint32_t s_sm, s_blocks, s_reason;
+  __shared__ WorkerShared ws;        // worker bookkeeping kept out of registers (tid 0 only)
   const uint32_t tid = threadIdx.x;
-  if (tid == 0) { s_sm = smid_reg(); s_t_entry = gtimer(); s_blocks = 0; s_reason = 0; }
+  if (tid == 0) { ws.sm = smid_reg(); ws.t_entry = gtimer(); ws.blocks = 0; ws.reason = 0; }
   Body::setup(args);                 // per-worker resources (e.g. TMEM, mbarriers); may sync
-  uint32_t k = 0;                    // chunk index within the current poll period
-  uint32_t parity = 0;
-  uint32_t held = 0xffffffffu;       // tid 0: prefetched chunk base not yet processed
-  bool stopping = false;             // tid 0: a request named this SM; drain the held chunk
-  while (true) {
-    if (tid == 0) {
-      uint32_t base;
-      if (k == 0 && !stopping) {                         // amortised poll (Fig. 4(b))
-        const uint32_t c = ld_relaxed_gpu(p.ctrl);
-        if (should_yield(c, p, smid_reg())) { stopping = true; s_reason = kReasonYield; }
-      }
-      if (held != 0xffffffffu) {                         // a fetched chunk is always processed (A4)
-        base = held;
-        held = 0xffffffffu;
-      } else {
-        base = stopping ? 0xffffffffu : atomicAdd(&p.cb->ctr, p.chunk);   // pull_task
-      }
-      if (base != 0xffffffffu && base >= p.n_blocks) { base = 0xffffffffu; s_reason = kReasonExhausted; }
-      if (base != 0xffffffffu) {
-        s_blocks += min(p.chunk, p.n_blocks - base);
-        if (p.prefetch && !stopping) held = atomicAdd(&p.cb->ctr, p.chunk);   // overlaps the body
-        if (p.trigger_block - base < p.chunk) {          // device self-trigger inside this chunk
-          const uint32_t e = p.epoch % kEvEpochs;
-          p.cb->ep_t_trigger[e] = gtimer();
-          p.cb->ep_trigger_block[e] = p.trigger_block;
-          atomicExch(p.ctrl, ((p.epoch & 0xffffu) << 16) | (p.trigger_n & 0xffffu));
-        }
-      }
-      s_slot[parity] = base;
+  if constexpr (Body::kPersistent) {
+    Body::persistent(args, p, ws);
+  } else {
+    SchedState st;
+    uint32_t parity = 0;
+    while (true) {
+      if (tid == 0) s_slot[parity] = next_chunk(p, st, ws);
+      __syncthreads();
+      const uint32_t b0 = s_slot[parity];
+      parity ^= 1u;
+      if (b0 == 0xffffffffu) break;
+      const uint32_t b1 = min(b0 + p.chunk, p.n_blocks);
+      Body::run(args, b0, b1, p.gx, p.gy);
+      if (kCoverage && tid == 0)
+        for (uint32_t b = b0; b < b1; ++b) atomicAdd(&p.cov[b], 1u);
     }
-    __syncthreads();
-    const uint32_t b0 = s_slot[parity];
-    parity ^= 1u;
-    if (b0 == 0xffffffffu) break;
-    const uint32_t b1 = min(b0 + p.chunk, p.n_blocks);
-    Body::run(args, b0, b1, p.gx, p.gy);
-    if (kCoverage && tid == 0)
-      for (uint32_t b = b0; b < b1; ++b) atomicAdd(&p.cov[b], 1u);
-    if (++k == p.poll) k = 0;
   }
   Body::teardown(args);              // release per-worker resources before leaving the SM (a7)
   // exit path (a7). One relaxed 64-bit atomic adds this worker's block count and its exit; the
   // worker that completes the epoch's exit count sees the exact total. No fences: the outputs
   // are published by kernel completion (stream order), and the host status is a notification.
   if (tid == 0) {
-    const uint32_t my_blocks = s_blocks;
+    const uint32_t my_blocks = ws.blocks;
     WorkerEvent& e = p.ev[(p.epoch % kEvEpochs) * p.workers + blockIdx.x];
     const uint64_t t_exit = gtimer();
-    e.smid = s_sm; e.reason = s_reason; e.n_blocks = my_blocks; e.epoch = p.epoch;
-    e.t_entry = s_t_entry; e.t_exit = t_exit;
+    e.smid = ws.sm; e.reason = ws.reason; e.n_blocks = my_blocks; e.epoch = p.epoch;
+    e.t_entry = ws.t_entry; e.t_exit = t_exit;
     const unsigned long long old = atomicAdd(&p.cb->done_exited, (1ull << 32) | my_blocks);
     if ((uint32_t)(old >> 32) + 1 == p.workers) {        // last worker of this epoch
       const uint32_t d = (uint32_t)old + my_blocks;
@@ -221,10 +248,12 @@ flep_unwrapped(const __grid_constant__ typename Body::Args args, uint32_t gx, ui
   Body::teardown(args);
 }
 
-// Bodies without per-worker resources.
+// Bodies without per-worker resources, run through the generic per-chunk loop.
 struct NoResources {
+  static constexpr bool kPersistent = false;
   template <class A> __device__ static void setup(const A&) {}
   template <class A> __device__ static void teardown(const A&) {}
+  template <class A> __device__ static void persistent(const A&, const WorkerParams&, WorkerShared&) {}
 };
 
 }  // namespace flep

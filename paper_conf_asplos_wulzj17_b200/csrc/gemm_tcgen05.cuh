@@ -23,6 +23,10 @@
 #include "../../include/flep.h"
 #include "flep_device.cuh"
 
+#ifndef FLEP_GEMM_GROUP
+#define FLEP_GEMM_GROUP 16
+#endif
+
 namespace flep {
 
 struct GemmArgsDev {
@@ -37,12 +41,17 @@ struct GemmBody {
   static constexpr int kMinBlocks = 1;
   static constexpr uint32_t BM = 128, BN = 256, BK = 64, UMMA_K = 16, STAGES = 4;
   static constexpr uint32_t kBytesA = BM * BK * 2, kBytesB = BN * BK * 2, kStage = kBytesA + kBytesB;
-  static constexpr uint32_t kTmemCols = 256;
-  static constexpr size_t kDynSmem = 1024 + STAGES * kStage + 256;
+  static constexpr uint32_t kTmemCols = 512;           // two 128x256 fp32 accumulators
+  static constexpr uint32_t QDEPTH = 4;                // tile queue: scheduler -> MMA / epilogue
+  static constexpr size_t kDynSmem = 1024 + STAGES * kStage + 512;
+  static constexpr bool kPersistent = true;
   using Args = GemmArgsDev;
 
   struct State {                      // lives after the stage ring
     uint64_t full[STAGES], empty[STAGES], tmem_full, tmem_empty;
+    uint64_t tfull[2], tempty[2];     // persistent loop: double-buffered accumulators
+    uint64_t qfull[QDEPTH], qempty[QDEPTH];
+    uint32_t tile_q[QDEPTH];
     uint32_t tmem_base;
     uint32_t p_stage, p_phase;        // producer
     uint32_t m_stage, m_phase, m_acc; // MMA issuer
@@ -77,6 +86,17 @@ struct GemmBody {
         :: "r"(smem_u32(dst)), "l"(reinterpret_cast<uint64_t>(map)), "r"(smem_u32(bar)), "r"(x), "r"(y)
         : "memory");
   }
+  // Original block b -> output tile (tm, tn). Blocks are numbered in bands of GROUP tile-rows,
+  // column by column inside a band, so the tiles that run concurrently share B panels in L2.
+  static constexpr uint32_t GROUP = FLEP_GEMM_GROUP;
+  __device__ static uint32_t p_gy(const Args& g) { return g.m / BM; }
+  __device__ static void tile_coords(uint32_t b, uint32_t gx, uint32_t gy, int32_t& tm, int32_t& tn) {
+    const uint32_t band = GROUP * gx;
+    const uint32_t grp = b / band, r = b % band;
+    const uint32_t rows = min(GROUP, gy - grp * GROUP);
+    tm = (int32_t)(grp * GROUP + r % rows);
+    tn = (int32_t)(r / rows);
+  }
   // K-major, SWIZZLE_128B smem matrix descriptor (sm_100 UMMA): start>>4, LBO 16 B (unused for
   // swizzled K-major), SBO 1024 B (8 rows x 128 B), version 1, layout SWIZZLE_128B (2).
   __device__ static uint64_t sdesc(uint32_t saddr) {
@@ -93,6 +113,8 @@ struct GemmBody {
       for (uint32_t i = 0; i < STAGES; ++i) { mbar_init(&s->full[i], 1); mbar_init(&s->empty[i], 1); }
       mbar_init(&s->tmem_full, 1);
       mbar_init(&s->tmem_empty, 128);
+      for (uint32_t i = 0; i < 2; ++i) { mbar_init(&s->tfull[i], 1); mbar_init(&s->tempty[i], 128); }
+      for (uint32_t i = 0; i < QDEPTH; ++i) { mbar_init(&s->qfull[i], 1); mbar_init(&s->qempty[i], 5); }
       s->p_stage = s->p_phase = s->m_stage = s->m_phase = s->m_acc = 0;
       s->e_acc[0] = s->e_acc[1] = s->e_acc[2] = s->e_acc[3] = 0;
       asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -124,7 +146,8 @@ struct GemmBody {
       if (lane == 0) {                                     // ---- TMA producer
         uint32_t st = s->p_stage, ph = s->p_phase;
         for (uint32_t b = b0; b < b1; ++b) {
-          const int32_t tm = (int32_t)(b / gx), tn = (int32_t)(b % gx);
+          int32_t tm, tn;
+          tile_coords(b, gx, p_gy(g), tm, tn);
           for (uint32_t kb = 0; kb < nk; ++kb) {
             mbar_wait(&s->empty[st], ph ^ 1u);
             uint8_t* sa = base + st * kStage;
@@ -172,7 +195,8 @@ struct GemmBody {
       uint32_t acc = s->e_acc[q];
       const uint32_t tmem = s->tmem_base + ((q * 32u) << 16);
       for (uint32_t b = b0; b < b1; ++b) {
-        const uint32_t tm = b / gx, tn = b % gx;
+        int32_t tm, tn;
+        tile_coords(b, gx, p_gy(g), tm, tn);
         mbar_wait(&s->tmem_full, acc);
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
         const uint32_t row = tm * BM + q * 32u + lane;
@@ -207,6 +231,135 @@ struct GemmBody {
       __syncwarp();
       if (lane == 0) s->e_acc[q] = acc;
     }
+  }
+
+  // ---- persistent FLEP worker loop (warp-specialised; chunk boundaries do not drain the
+  // pipeline). tid 0 is the scheduler AND the TMA producer: it runs the FLEP scheduling step
+  // (poll / fetch / trigger, next_chunk), pushes every tile of the fetched chunk into a 4-deep
+  // smem queue, then issues that tile's TMA loads; a STOP sentinel ends the loop. The MMA thread
+  // and the 4 epilogue warps consume the queue; accumulators alternate between two TMEM halves
+  // so tile t's epilogue overlaps tile t+1's MMAs. Every fetched tile is computed (A4).
+  __device__ static void persistent(const Args& g, const WorkerParams& p, WorkerShared& ws) {
+    State* s = state();
+    uint8_t* base = ring();
+    const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31u;
+    const uint32_t nk = g.k / BK;
+    const uint32_t gx = p.gx;
+    constexpr uint32_t STOP = 0xffffffffu;
+    if (warp == 0) {
+      if (lane == 0) {                                     // ---- scheduler + TMA producer
+        SchedState sch;
+        uint32_t qi = 0, qph = 0, st = 0, ph = 0;
+        while (true) {
+          const uint32_t b0 = next_chunk(p, sch, ws);
+          const uint32_t b1 = (b0 == STOP) ? b0 : min(b0 + p.chunk, p.n_blocks);
+          for (uint32_t b = b0; b != STOP && b < b1; ++b) {
+            mbar_wait(&s->qempty[qi], qph ^ 1u);
+            s->tile_q[qi] = b;
+            mbar_arrive(&s->qfull[qi]);
+            if (++qi == QDEPTH) { qi = 0; qph ^= 1u; }
+            if (p.cov) atomicAdd(&p.cov[b], 1u);
+            int32_t tm, tn;
+          tile_coords(b, gx, p_gy(g), tm, tn);
+            for (uint32_t kb = 0; kb < nk; ++kb) {
+              mbar_wait(&s->empty[st], ph ^ 1u);
+              uint8_t* sa = base + st * kStage;
+              uint8_t* sb = sa + kBytesA;
+              mbar_expect_tx(&s->full[st], kStage);
+              tma_2d(&g.tma_a, sa, &s->full[st], (int32_t)(kb * BK), tm * (int32_t)BM);
+              tma_2d(&g.tma_b, sb, &s->full[st], (int32_t)(kb * BK), tn * (int32_t)BN);
+              if (++st == STAGES) { st = 0; ph ^= 1u; }
+            }
+          }
+          if (b0 == STOP) {
+            mbar_wait(&s->qempty[qi], qph ^ 1u);
+            s->tile_q[qi] = STOP;
+            mbar_arrive(&s->qfull[qi]);
+            break;
+          }
+        }
+      }
+    } else if (warp == 1) {
+      if (lane == 0) {                                     // ---- MMA issuer
+        uint32_t qi = 0, qph = 0, st = 0, ph = 0, acc = 0, aph = 0;
+        const uint32_t tmem0 = s->tmem_base;
+        while (true) {
+          mbar_wait(&s->qfull[qi], qph);
+          const uint32_t b = s->tile_q[qi];
+          mbar_arrive(&s->qempty[qi]);
+          if (++qi == QDEPTH) { qi = 0; qph ^= 1u; }
+          if (b == STOP) break;
+          mbar_wait(&s->tempty[acc], aph ^ 1u);            // epilogue drained this half
+          asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+          const uint32_t tmem = tmem0 + acc * BN;
+          for (uint32_t kb = 0; kb < nk; ++kb) {
+            mbar_wait(&s->full[st], ph);
+            asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+            const uint32_t sa = smem_u32(base + st * kStage), sb = sa + kBytesA;
+#pragma unroll
+            for (uint32_t k = 0; k < BK / UMMA_K; ++k) {
+              const uint64_t da = sdesc(sa + k * UMMA_K * 2), db = sdesc(sb + k * UMMA_K * 2);
+              const uint32_t accum = (kb | k) ? 1u : 0u;
+              asm volatile(
+                  "{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n"
+                  " tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n}\n"
+                  :: "r"(tmem), "l"(da), "l"(db), "r"(kIdesc), "r"(accum) : "memory");
+            }
+            asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];"
+                         :: "r"(smem_u32(&s->empty[st])) : "memory");
+            if (++st == STAGES) { st = 0; ph ^= 1u; }
+          }
+          asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];"
+                       :: "r"(smem_u32(&s->tfull[acc])) : "memory");
+          if (++acc == 2) { acc = 0; aph ^= 1u; }
+        }
+      }
+    } else if (warp >= 4) {                                // ---- epilogue (128 threads)
+      const uint32_t q = warp - 4;
+      uint32_t qi = 0, qph = 0, acc = 0, aph = 0;
+      while (true) {
+        mbar_wait(&s->qfull[qi], qph);
+        const uint32_t b = s->tile_q[qi];
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&s->qempty[qi]);
+        if (++qi == QDEPTH) { qi = 0; qph ^= 1u; }
+        if (b == STOP) break;
+        int32_t tm, tn;
+        tile_coords(b, gx, p_gy(g), tm, tn);
+        mbar_wait(&s->tfull[acc], aph);
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        const uint32_t tmem = s->tmem_base + acc * BN + ((q * 32u) << 16);
+        const uint32_t row = tm * BM + q * 32u + lane;
+        __nv_bfloat16* crow = g.c + (size_t)row * g.n + (size_t)tn * BN;
+#pragma unroll 1
+        for (uint32_t c0 = 0; c0 < BN; c0 += 32) {
+          uint32_t r[32];
+          asm volatile(
+              "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+              "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+              : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+                "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]),
+                "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]),
+                "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
+              : "r"(tmem + c0));
+          asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+          uint4 o[4];
+          uint32_t* ow = reinterpret_cast<uint32_t*>(o);
+#pragma unroll
+          for (int i = 0; i < 16; ++i) {
+            __nv_bfloat162 h = __floats2bfloat162_rn(__uint_as_float(r[2 * i]), __uint_as_float(r[2 * i + 1]));
+            ow[i] = *reinterpret_cast<uint32_t*>(&h);
+          }
+          uint4* dst = reinterpret_cast<uint4*>(crow + c0);
+#pragma unroll
+          for (int i = 0; i < 4; ++i) dst[i] = o[i];
+        }
+        asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+        mbar_arrive(&s->tempty[acc]);
+        if (++acc == 2) { acc = 0; aph ^= 1u; }
+      }
+    }
+    __syncthreads();
   }
 };
 
