@@ -196,6 +196,12 @@ flep_status flep_preempt(flep_rt rt, flep_launch_t h, uint32_t n_sms);
 /* MANUAL mode only. PREEMPTED: relaunch the workers on the same counter (stream-ordered after
    the drained grid). PARTIAL: withdraw the spatial request (the remaining workers continue). */
 flep_status flep_resume(flep_rt rt, flep_launch_t h);
+/* MANUAL mode only. Spatial refill: for a PARTIAL launch, widen the request to the
+   whole GPU for the running epoch and queue a full-width epoch behind it, so the victim is
+   re-spread over every SM once the waiting kernel is done (the paper's baseline keeps it on the
+   remaining SMs). If the running epoch completes the launch first, the refill epoch
+   exits without work. PREEMPTED: same as flep_resume. */
+flep_status flep_refill(flep_rt rt, flep_launch_t h);
 /* Wait until the launch is DONE (timeout_ns < 0: forever). Also waits for its last grid. */
 flep_status flep_sync(flep_rt rt, flep_launch_t h, int64_t timeout_ns);
 /* Refresh and return the launch's state (never blocks). */

@@ -34,7 +34,9 @@ struct alignas(128) ControlBlock {
   // one 64-bit word, one atomic per worker exit: low half = original blocks executed (all
   // epochs), high half = workers of the current epoch that have exited (reset by the last)
   unsigned long long done_exited;
-  uint32_t _p2[30];
+  uint32_t done_gen;       // generation whose epoch completed the launch (0 = none yet); an
+                           // epoch launched after that (e.g. a refill) exits without fetching
+  uint32_t _p2[29];
   // per-epoch summaries (ring of kEvEpochs)
   uint64_t ep_t_trigger[kEvEpochs];
   uint64_t ep_t_end[kEvEpochs];
@@ -77,6 +79,7 @@ struct WorkerParams {
   uint32_t trigger_n;      // its yield width
   uint32_t prefetch;       // 1: fetch chunk j+1 while chunk j runs (hides the atomic's latency;
                            //    a stopping worker still processes the prefetched chunk)
+  uint32_t gen_first;      // generation of this launch's first epoch
 };
 
 __device__ __forceinline__ uint32_t smid_reg() {
@@ -141,10 +144,18 @@ struct SchedState {
   uint32_t k = 0;                    // chunk index within the current poll period
   uint32_t held = 0xffffffffu;       // prefetched chunk base not yet handed out
   bool stopping = false;             // a request named this SM; drain the held chunk
+  bool first = true;                 // first step of this worker
 };
 
 __device__ __forceinline__ uint32_t next_chunk(const WorkerParams& p, SchedState& st, WorkerShared& ws) {
   uint32_t base;
+  if (st.first) {                                    // the launch already completed in an earlier
+    st.first = false;                                // epoch (a refill raced with the last blocks):
+    if (ld_relaxed_gpu(&p.cb->done_gen) >= p.gen_first) {   // leave without touching the counter
+      ws.reason = kReasonExhausted;
+      return 0xffffffffu;
+    }
+  }
   if (st.k == 0 && !st.stopping) {                   // amortised poll (Fig. 4(b))
     const uint32_t c = ld_relaxed_gpu(p.ctrl);
     if (should_yield(c, p, smid_reg())) { st.stopping = true; ws.reason = kReasonYield; }
@@ -219,15 +230,20 @@ flep_worker(const __grid_constant__ typename Body::Args args, const WorkerParams
     e.t_entry = ws.t_entry; e.t_exit = t_exit;
     const unsigned long long old = atomicAdd(&p.cb->done_exited, (1ull << 32) | my_blocks);
     if ((uint32_t)(old >> 32) + 1 == p.workers) {        // last worker of this epoch
-      const uint32_t d = (uint32_t)old + my_blocks;
+      const bool already = ld_relaxed_gpu(&p.cb->done_gen) >= p.gen_first;
+      const uint32_t d = already ? p.n_blocks : (uint32_t)old + my_blocks;
       const uint32_t c = ld_relaxed_gpu(&p.cb->ctr);     // every fetch has completed by now
       const uint32_t st = (d >= p.n_blocks) ? kStateDone : kStatePreempted;
       const uint32_t ei = p.epoch % kEvEpochs;
       p.cb->ep_t_end[ei] = t_exit; p.cb->ep_done[ei] = d; p.cb->ep_ctr[ei] = c;
       p.cb->ep_state[ei] = st;
       p.cb->ep_t_trigger[(p.epoch + 1) % kEvEpochs] = 0;  // next epoch's trigger stamp
-      if (st == kStateDone) { p.cb->done_exited = 0ull; p.cb->ctr = 0; }   // clean for reuse
-      else p.cb->done_exited = (unsigned long long)d;    // exits reset, progress kept
+      if (st == kStateDone) {                            // clean for reuse; remember completion
+        p.cb->done_exited = 0ull; p.cb->ctr = 0;
+        if (!already) p.cb->done_gen = p.epoch;
+      } else {
+        p.cb->done_exited = (unsigned long long)d;       // exits reset, progress kept
+      }
       if (p.status) {
         st_relaxed_sys(&p.status->ctr, c);
         st_relaxed_sys_u64(&p.status->t_end, t_exit);

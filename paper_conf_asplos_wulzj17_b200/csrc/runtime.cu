@@ -293,6 +293,7 @@ flep_status start_epoch(flep_rt rt, Launch& L) {
   p.trigger_block = L.trig_block;
   p.trigger_n = L.trig_n;
   p.prefetch = (L.flags & FLEP_KFLAG_PREFETCH) ? 1u : 0u;
+  p.gen_first = L.gen0 + 1;
   L.trig_block = kNoTrigger;
   L.trig_n = 0;
   cudaError_t e = L.ops->worker(L.args.data(), p, L.workers, L.exec, L.cov != nullptr);
@@ -761,6 +762,23 @@ flep_status flep_resume(flep_rt rt, flep_launch_t h) {
     return FLEP_OK;
   }
   return fail(FLEP_ERR_STATE, "launch %lld is not preempted (state %d)", (long long)h, L->state);
+}
+
+flep_status flep_refill(flep_rt rt, flep_launch_t h) {
+  if (!rt) return fail(FLEP_ERR_INVALID, "rt is NULL");
+  ApiLock lk(rt);
+  if (rt->opt.policy != FLEP_POLICY_MANUAL) return fail(FLEP_ERR_STATE, "refill is policy-driven in managed mode");
+  Launch* L = find(rt, h);
+  if (!L) return fail(FLEP_ERR_INVALID, "unknown launch %lld", (long long)h);
+  refresh(rt, *L);
+  if (L->state == FLEP_STATE_PREEMPTED) return start_epoch(rt, *L);
+  if (L->state != FLEP_STATE_PARTIAL)
+    return fail(FLEP_ERR_STATE, "launch %lld is not partially preempted (state %d)", (long long)h, L->state);
+  // widen the request to the whole GPU for the running epoch, then queue a full-width epoch
+  // behind it (stream order): the victim is re-spread over every SM
+  flep_status s = write_ctrl(rt, *L, ctrl_word(*L, 0xffffu));
+  if (s) return s;
+  return start_epoch(rt, *L);
 }
 
 flep_status flep_wait_epoch(flep_rt rt, flep_launch_t h, int64_t timeout_ns) {

@@ -94,6 +94,7 @@ _SIG = {
     "flep_launch": (C.c_int, [_P, C.c_int32, Dim3, _P, C.c_size_t, C.c_int32, _P, C.POINTER(C.c_int64)]),
     "flep_preempt": (C.c_int, [_P, C.c_int64, C.c_uint32]),
     "flep_resume": (C.c_int, [_P, C.c_int64]),
+    "flep_refill": (C.c_int, [_P, C.c_int64]),
     "flep_sync": (C.c_int, [_P, C.c_int64, C.c_int64]),
     "flep_query": (C.c_int, [_P, C.c_int64, C.POINTER(LaunchInfo)]),
     "flep_cancel": (C.c_int, [_P, C.c_int64]),
@@ -216,6 +217,9 @@ class Runtime:
 
     def resume(self, launch):
         check(self.L.flep_resume(self.h, launch), "flep_resume")
+
+    def refill(self, launch):
+        check(self.L.flep_refill(self.h, launch), "flep_refill")
 
     def sync(self, launch, timeout_ns=-1):
         check(self.L.flep_sync(self.h, launch, timeout_ns), "flep_sync")

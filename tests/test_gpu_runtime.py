@@ -236,3 +236,52 @@ def test_managed_ffs_share_and_replay():
         assert dec == rep
     finally:
         rt.close()
+
+
+@pytest.mark.parametrize("tail", [False, True])
+def test_spatial_refill_exactly_once(tail):
+    """Spatial yield, then refill: the victim is re-spread over all SMs. With the
+    trigger near the end, the running epoch usually completes the launch before the refill epoch
+    starts; that epoch must not re-run anything (the control block was already reset)."""
+    f = flep_mod()
+    rt = f.Runtime(coverage=True)
+    try:
+        n = 1 << 22
+        nb = n // 256
+        x, y = gen.saxpy_i32_inputs(n, seed=81)
+        ref = W.saxpy_i32(13, x, y)
+        xd, y0 = t(x), t(y)
+        k = rt.register_kernel(f.BODY_SAXPY_I32, chunk=1, poll=1)
+        for rep in range(20):
+            yd = y0.clone()
+            tstar = nb - 40 if tail else nb // 4
+            rt.arm_next_trigger(tstar, 37)
+            h = rt.launch(k, f.saxpy_grid(n), f.saxpy_i32_args(yd, xd, 13))
+            # wait until the spatial request is in force (the trigger fired) or the epoch ended
+            import time
+            t0 = time.time()
+            while rt.query(h).state == f.STATE_RUNNING and time.time() - t0 < 5:
+                try:
+                    if rt.epoch_info(h, 1).t_trigger:
+                        break
+                except f.FlepError:
+                    pass
+            info = rt.query(h)
+            if info.state in (f.STATE_RUNNING, f.STATE_PARTIAL):
+                # the device trigger does not move the host state machine; mark the request
+                try:
+                    rt.preempt(h, 37)
+                except f.FlepError:
+                    pass
+            try:
+                rt.refill(h)
+            except f.FlepError as e:
+                assert e.status == f.ERR_STATE
+            rt.wait_epoch(h, timeout_ns=10_000_000_000)
+            if rt.query(h).state == f.STATE_PREEMPTED:
+                rt.resume(h)
+            rt.sync(h, timeout_ns=10_000_000_000)
+            assert np.all(rt.coverage_np(h, nb) == 1)
+            assert np.array_equal(yd.cpu().numpy(), ref)
+    finally:
+        rt.close()
