@@ -39,6 +39,34 @@ def test_prefetch_final_counter_closed_form():
         assert r.terminal_ctrs == {cv.final_counter_no_preempt(n, C, len(ws))}
 
 
+@pytest.mark.parametrize("C", [1, 2])
+def test_exhaustive_spatial_refill(C):
+    # flep_refill: widen a spatial request to temporal and queue a full-width epoch; when the
+    # running epoch completes the launch first (and the device cleans the block), the queued
+    # epoch must exit without fetching (completed-generation marker)
+    r = cv.explore(_cfg(n_blocks=4 if C == 1 else 5, chunk=C, poll=1, worker_sm=(0, 0, 1),
+                        preempt_widths=(1,), max_events=2, allow_refill=True))
+    assert r.violations == set()
+
+
+def test_refill_without_done_marker_double_executes():
+    # the same exploration with the marker check disabled finds double executions: the check is
+    # what keeps a refill that races the last blocks exactly-once
+    import oracle.coverage as m
+    orig = m.successors
+
+    def no_marker(cfg, st):
+        st2 = st[:9] + ((st[9][0], 0, st[9][2]),)   # pretend no epoch ever recorded completion
+        return [(lab, s[:9] + ((s[9][0], 0, s[9][2]),)) for lab, s in orig(cfg, st2)]
+    m.successors = no_marker
+    try:
+        r = cv.explore(_cfg(n_blocks=3, chunk=1, poll=1, worker_sm=(0, 1), preempt_widths=(1,),
+                            max_events=2, allow_refill=True))
+    finally:
+        m.successors = orig
+    assert any("more than once" in v for v in r.violations)
+
+
 def test_exhaustive_with_clear_events():
     r = cv.explore(_cfg(n_blocks=6, chunk=2, poll=2, allow_clear=True))
     assert r.violations == set()
@@ -88,7 +116,7 @@ def test_hand_traced_temporal_preempt_after_one_chunk():
     st = cv.initial_state(cfg)
     for lab in ["w0.poll", "w0.fetch", "w0.proc", "preempt(2)", "w0.poll", "w0.exit"]:
         st = dict(cv.successors(cfg, st))[lab]
-    ctr, ctrl, done, exited, cov, epoch, status, workers, ev = st
+    ctr, ctrl, done, exited, cov, epoch, status, workers, ev, extra = st
     assert status == cv.ST_PREEMPTED and cov == (1, 0, 0) and ctr == 1 and done == 1
     assert list(cov) == cv.expected_prefix(ctr, 3)
     # resume: a fresh epoch ignores the stale request (gen 0) and finishes the rest
@@ -96,7 +124,7 @@ def test_hand_traced_temporal_preempt_after_one_chunk():
     for lab in ["w0.poll", "w0.fetch", "w0.proc", "w0.poll", "w0.fetch", "w0.proc", "w0.poll",
                 "w0.fetch", "w0.exit"]:
         st = dict(cv.successors(cfg, st))[lab]
-    assert st[6] == cv.ST_DONE and st[4] == (1, 1, 1) and st[0] == 4
+    assert st[6] == cv.ST_DONE and st[4] == (1, 1, 1) and st[9][2] == 4 and st[0] == 0
 
 
 def test_hand_traced_spatial_keeps_other_sm_running():
