@@ -84,26 +84,30 @@ struct SaxpyBody : NoResources {
 
 // ---------------------------------------------------------------------------------------------
 // SpMV-CSR fp32: y[r] = sum_p val[p] * x[col[p]]. Block b = rows [128b, 128b+128).
-// CSR-stream form: the block's rowptr slice goes to smem; all 256 threads then stream the
-// block's contiguous nnz range [rowptr[r0], rowptr[r1]) in tiles of kTile entries (coalesced
-// col/val loads, independent x gathers, 4 in flight per thread), writing products to smem; thread
-// t < 128 finally sums row r0+t's products in ascending p order. Per-row summation order is
-// fixed, so every execution of a block gives bit-identical results.
+// CSR-stream form: the rowptr slice of up to 256 rows (two blocks of a chunk; one block in the
+// unwrapped kernel) goes to smem; all 256 threads then stream the rows' contiguous nnz range in
+// tiles of kTile entries (coalesced col/val loads, independent x gathers, U in flight per thread),
+// writing products to smem; thread t sums row r0+t's products in ascending p order. Per-row
+// summation order does not depend on the grouping, so every execution of a block (wrapped,
+// unwrapped, preempted and resumed) gives bit-identical results.
 struct SpmvBody : NoResources {
   static constexpr int kThreads = 256;
   static constexpr int kMinBlocks = 8;
   static constexpr uint32_t kRowsPerBlock = 128;
-  static constexpr uint32_t kTile = 1024;
+  static constexpr uint32_t kTile = 2048;
   using Args = flep_spmv_args;
 
+  static constexpr uint32_t kGroupRows = 256;     // rows streamed together (2 blocks of a chunk)
+
   __device__ static void run(const Args& g, uint32_t b0, uint32_t b1, uint32_t, uint32_t) {
-    __shared__ int32_t s_rp[kRowsPerBlock + 1];
+    __shared__ int32_t s_rp[kGroupRows + 1];
     __shared__ float s_prod[kTile];
     const uint32_t tid = threadIdx.x;
-    for (uint32_t b = b0; b < b1; ++b) {
-      const uint32_t r0 = b * kRowsPerBlock;
-      const uint32_t nr = min(kRowsPerBlock, g.rows - r0);
+    const uint32_t row_end = min(b1 * kRowsPerBlock, g.rows);
+    for (uint32_t r0 = b0 * kRowsPerBlock; r0 < row_end; r0 += kGroupRows) {
+      const uint32_t nr = min(kGroupRows, row_end - r0);
       if (tid <= nr) s_rp[tid] = __ldg(g.rowptr + r0 + tid);
+      if (tid == 0 && nr == kGroupRows) s_rp[kGroupRows] = __ldg(g.rowptr + r0 + kGroupRows);
       __syncthreads();
       const int32_t p0 = s_rp[0], p1 = s_rp[nr];
       int32_t my_s = 0, my_e = 0;
@@ -130,7 +134,7 @@ struct SpmvBody : NoResources {
           }
         }
         __syncthreads();
-        if (tid < nr) {
+        if (tid < nr) {                        // row r0+tid: its products in ascending p order
           const int32_t lo = max(my_s, base), hi = min(my_e, base + n);
           for (int32_t p = lo; p < hi; ++p) acc += s_prod[p - base];
         }
