@@ -151,6 +151,8 @@ typedef struct {
   uint32_t n_yield;            /* yield width currently requested (0 = none) */
   int64_t t_last_request;      /* host ns of the last preempt request issued by the runtime */
   int64_t t_last_drain;        /* host ns the runtime observed the last PREEMPTED epoch end */
+  uint32_t started_epoch;      /* newest epoch (1-based) whose first worker has begun running */
+  uint32_t reserved;
 } flep_launch_info;
 
 /* Per-worker event record of one epoch (device %globaltimer, ns). */

@@ -58,7 +58,8 @@ struct HostStatus {        // pinned, mapped; one 32-B slot per launch
                            // copy in ControlBlock::ep_ctr is authoritative)
   uint32_t ctrl;           // FLEP_FLAG_HOST_MAPPED: the control word itself (CPU-written)
   uint64_t t_end;          // %globaltimer of the last exit (best effort)
-  uint64_t _pad;
+  uint32_t started;        // generation of the newest epoch whose first worker has started
+  uint32_t _pad;
 };
 
 struct WorkerParams {
@@ -199,7 +200,10 @@ flep_worker(const __grid_constant__ typename Body::Args args, const WorkerParams
   __shared__ uint32_t s_slot[2];     // chunk base broadcast, double-buffered: 1 barrier per chunk
   __shared__ WorkerShared ws;        // worker bookkeeping kept out of registers (tid 0 only)
   const uint32_t tid = threadIdx.x;
-  if (tid == 0) { ws.sm = smid_reg(); ws.t_entry = gtimer(); ws.blocks = 0; ws.reason = 0; }
+  if (tid == 0) {
+    ws.sm = smid_reg(); ws.t_entry = gtimer(); ws.blocks = 0; ws.reason = 0;
+    if (blockIdx.x == 0 && p.status) st_relaxed_sys(&p.status->started, p.epoch);   // host hint
+  }
   Body::setup(args);                 // per-worker resources (e.g. TMEM, mbarriers); may sync
   if constexpr (Body::kPersistent) {
     Body::persistent(args, p, ws);

@@ -124,6 +124,7 @@ struct Launch {
   std::deque<std::pair<cudaEvent_t, uint32_t>> inflight;
   std::vector<cudaEvent_t> evpool;
   cudaEvent_t fin_ev = nullptr;      // recorded after every grid of this launch (its last work)
+  int64_t t_seen = 0;                // monitor: host time its status word was seen to move
   bool released = false;
   bool cancelled = false;
 };
@@ -333,13 +334,16 @@ bool refresh(flep_rt rt, Launch& L) {
   if ((w >> 8) != (gen_of(L) & 0xffffffu)) return false;
   L.last_done = (uint32_t)(w64 >> 32);
   L.last_ctr = __atomic_load_n(&L.hs->ctr, __ATOMIC_ACQUIRE);
+  // the monitor stamps the moment it saw the word move (before taking the lock)
+  const int64_t t_obs = L.t_seen > 0 ? L.t_seen : now_ns();
+  L.t_seen = 0;
   if ((w & 0xffu) == kStateDone) {
     L.state = FLEP_STATE_DONE;
-    L.t_finish = now_ns();
+    L.t_finish = t_obs;
     return true;
   }
   L.state = FLEP_STATE_PREEMPTED;
-  L.t_last_drain = now_ns();
+  L.t_last_drain = t_obs;
   return false;
 }
 
@@ -445,7 +449,8 @@ void monitor_pass(flep_rt rt) {
 // never starved by it.
 void monitor_loop(flep_rt rt) {
   cudaSetDevice(rt->device);
-  struct Watch { const uint64_t* word; uint64_t seen; bool sliced; };
+  struct Watch { const uint64_t* word; uint64_t seen; bool sliced; int64_t id; };
+  std::vector<std::pair<int64_t, int64_t>> moved;     // (launch, host time seen)
   std::vector<Watch> watch;
   int64_t deadline = -1;
   bool pending_release = false;
@@ -453,8 +458,10 @@ void monitor_loop(flep_rt rt) {
   while (!rt->stop.load(std::memory_order_relaxed)) {
     bool hit = false;
     if (gen_seen != rt->active_gen.load(std::memory_order_acquire)) hit = true;   // new work
+    moved.clear();
     for (const Watch& w : watch) {
-      if (w.sliced || __atomic_load_n(w.word, __ATOMIC_ACQUIRE) != w.seen) { hit = true; break; }
+      if (w.sliced) { hit = true; continue; }
+      if (__atomic_load_n(w.word, __ATOMIC_ACQUIRE) != w.seen) { hit = true; moved.push_back({w.id, now_ns()}); }
     }
     if (deadline >= 0 && now_ns() >= deadline) hit = true;
     if (pending_release) hit = true;
@@ -468,6 +475,10 @@ void monitor_loop(flep_rt rt) {
       continue;
     }
     std::unique_lock<std::mutex> lk(rt->mu);
+    for (auto& m : moved) {
+      Launch* L = find(rt, m.first);
+      if (L) L->t_seen = m.second;
+    }
     gen_seen = rt->active_gen.load(std::memory_order_acquire);
     // snapshot the status words BEFORE the pass: a word that moves after the pass read it is
     // then seen as a change on the next poll (at worst one extra pass, never a missed event)
@@ -483,7 +494,7 @@ void monitor_loop(flep_rt rt) {
       if (!L || !L->hs) continue;
       const uint64_t* wp = reinterpret_cast<const uint64_t*>(&L->hs->word);
       auto it = snap.find(id);
-      watch.push_back({wp, it != snap.end() ? it->second : ~0ull, L->sliced});
+      watch.push_back({wp, it != snap.end() ? it->second : ~0ull, L->sliced, id});
     }
     deadline = rt->policy->epoch_end();
     pending_release = !rt->to_release.empty();
@@ -857,6 +868,10 @@ flep_status flep_query(flep_rt rt, flep_launch_t h, flep_launch_info* out) {
   out->t_e = L->t_e;
   out->t_last_request = L->t_last_request;
   out->t_last_drain = L->t_last_drain;
+  if (L->hs) {
+    const uint32_t g = __atomic_load_n(&L->hs->started, __ATOMIC_ACQUIRE);
+    out->started_epoch = (g > L->gen0) ? g - L->gen0 : 0;
+  }
   if (rt->policy) {
     const Policy::Entry* e = rt->policy->entry(L->id);
     if (e) { out->t_w = e->t_w; out->t_r = e->t_r; }

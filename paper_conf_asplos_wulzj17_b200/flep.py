@@ -68,7 +68,8 @@ class LaunchInfo(C.Structure):
                 ("blocks_done", C.c_uint64), ("counter", C.c_uint64), ("t_e", C.c_int64),
                 ("t_w", C.c_int64), ("t_r", C.c_int64), ("t_arrive", C.c_int64),
                 ("t_first_start", C.c_int64), ("t_finish", C.c_int64), ("workers", C.c_uint32),
-                ("n_yield", C.c_uint32), ("t_last_request", C.c_int64), ("t_last_drain", C.c_int64)]
+                ("n_yield", C.c_uint32), ("t_last_request", C.c_int64), ("t_last_drain", C.c_int64),
+                ("started_epoch", C.c_uint32), ("reserved", C.c_uint32)]
 
 
 class WorkerEvent(C.Structure):

@@ -1,0 +1,54 @@
+"""Host-observed preemption latency breakdown (manual mode): flep_preempt() on a running wrapped
+kernel -> host sees the PREEMPTED status. Also reports the device-side drain from the worker log."""
+import json
+import os
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+
+def main():
+    import torch
+    from paper_conf_asplos_wulzj17_b200 import build, flep as F
+    build.build()
+    for flag in (F.FLAG_STREAM_MEMOP, F.FLAG_HOST_MAPPED):
+        rt = F.Runtime(exec_on_user_stream=False, flag=flag)
+        n = 1 << 28
+        x = torch.ones(n, dtype=torch.int32, device="cuda")
+        y = torch.ones(n, dtype=torch.int32, device="cuda")
+        k = rt.register_kernel(F.BODY_SAXPY_I32, chunk=8, poll=1)
+        lat, dev = [], []
+        for r in range(30):
+            h = rt.launch(k, F.saxpy_grid(n), F.saxpy_i32_args(y, x, 1))
+            t0 = time.perf_counter()
+            while rt.query(h).started_epoch < 1 and time.perf_counter() - t0 < 1:
+                pass
+            time.sleep(50e-6)
+            t1 = F.now_ns()
+            rt.preempt(h, rt.num_sms)
+            while rt.query(h).state not in (F.STATE_PREEMPTED, F.STATE_DONE):
+                pass
+            t2 = F.now_ns()
+            info = rt.query(h)
+            if info.state == F.STATE_PREEMPTED:
+                ev = rt.events(h, 1)
+                ys = [e.t_exit for e in ev if e.reason == F.REASON_YIELD]
+                if ys:
+                    dev.append((max(ys) - min(ys)) / 1e3)
+                lat.append((t2 - t1) / 1e3)
+                rt.resume(h)
+            rt.sync(h)
+        print(json.dumps({"flag": "stream_memop" if flag == F.FLAG_STREAM_MEMOP else "host_mapped",
+                          "host_latency_us_p50": round(float(np.median(lat)), 2) if lat else None,
+                          "min": round(min(lat), 2) if lat else None,
+                          "yield_exit_spread_us_p50": round(float(np.median(dev)), 2) if dev else None,
+                          "n": len(lat)}), flush=True)
+        rt.close()
+
+
+if __name__ == "__main__":
+    main()
