@@ -523,7 +523,10 @@ def main():
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--impl", default="flep", choices=["flep", "reference"])
-    ap.add_argument("--config", default="temporal", choices=["temporal", "corun1", "spatial", "queue", "ffs"])
+    ap.add_argument("--config", default="temporal", choices=["temporal", "corun1", "spatial", "queue", "ffs", "model"])
+    ap.add_argument("--model-train", type=int, default=100)
+    ap.add_argument("--model-test", type=int, default=30)
+    ap.add_argument("--overhead-runs", type=int, default=50)
     ap.add_argument("--ffs-seconds", type=float, default=1.0)
     ap.add_argument("--corun-cps", type=int, default=2)
     ap.add_argument("--queue-kernels", type=int, default=64)
@@ -561,6 +564,8 @@ def main():
             bench_configs.run_corun1(args, rank, world, local)
         elif args.config == "ffs":
             bench_configs.run_ffs(args, rank, world, local)
+        elif args.config == "model":
+            bench_configs.run_model(args, rank, world, local)
         else:
             bench_configs.run_queue(args, rank, world, local)
 

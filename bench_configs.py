@@ -487,3 +487,48 @@ def run_ffs(args, rank, world, local):
     if rank == 0:
         print(json.dumps(out), flush=True)
     barrier(world)
+
+
+# ------------------------------------------------------------------------------------------
+def run_model(args, rank, world, local):
+    """Offline phase (§4.2; Fig. 7): fit each body's duration model on
+    random inputs (100 per body), report the prediction error on held-out inputs, and the
+    profiled preemption overhead O."""
+    import torch
+    from bench import L2Flush, barrier
+    from paper_conf_asplos_wulzj17_b200 import calibrate, flep as F
+    torch.cuda.set_device(local)
+    wl = calibrate.Workloads(torch, seed=11 + rank)
+    fl = L2Flush(torch)
+    rt = F.Runtime(device=local, policy=F.POLICY_FIFO)
+    rows = {}
+    bodies = {"saxpy_f32": (F.BODY_SAXPY_F32, 8, False), "spmv": (F.BODY_SPMV_CSR_F32, 2, True),
+              "stencil_f32": (F.BODY_STENCIL5_F32, 2, True), "gemm_bf16": (F.BODY_GEMM_BF16, 1, False)}
+    for name, (body, chunk, pf) in bodies.items():
+        model, X, y = calibrate.fit_duration_model(rt, torch, wl, body, n_train=args.model_train, chunk=chunk,
+                                                   prefetch=pf, flush=fl.zero_)
+        k = rt.register_kernel(body, chunk=chunk, poll=1, prefetch=pf)
+        errs = []
+        for _ in range(args.model_test):
+            grid, a, feats = wl.case(body, wl.random_size(body))
+            t = calibrate.measure_duration(rt, k, grid, a, torch, fl.zero_, reps=1)
+            errs.append(abs(float(calibrate.predict(model, feats)) - t) / t)
+        size = {F.BODY_SAXPY_F32: 1 << 26, F.BODY_SPMV_CSR_F32: 1 << 22, F.BODY_STENCIL5_F32: 8192,
+                F.BODY_GEMM_BF16: 4096}[body]
+        o, t_alone = calibrate.preemption_overhead(torch, wl, body, size, runs=args.overhead_runs, chunk=chunk,
+                                                   prefetch=pf, flush=fl.zero_)
+        rows[name] = {"model": [round(v, 6) for v in model], "mean_abs_pct_error": round(100 * float(np.mean(errs)), 2),
+                      "max_abs_pct_error": round(100 * float(np.max(errs)), 2), "train": len(y), "test": len(errs),
+                      "preempt_overhead_ns": o, "overhead_reference_size": size,
+                      "standalone_span_us": round(t_alone / 1e3, 2)}
+    rt.close()
+    mean_err = float(np.mean([r["mean_abs_pct_error"] for r in rows.values()]))
+    out = {"metric": METRIC, "value": round(mean_err, 2), "unit": "% mean abs duration-prediction error",
+           "value_definition": "ridge duration model (P:192) on held-out random inputs, mean over bodies (paper: 6.9 % on K40)",
+           "n_gpus": world, "higher_is_better": False, "scaling": "weak", "vs_baseline": None, "dtype": "mixed",
+           "data": "synthetic (seeded)", "config": {"workload": "offline phase: model fit + O profiling per body",
+                                                      "train_per_body": args.model_train, "test_per_body": args.model_test},
+           "bodies": rows}
+    if rank == 0:
+        print(json.dumps(out), flush=True)
+    barrier(world)
