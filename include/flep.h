@@ -64,9 +64,11 @@ typedef enum {
   FLEP_POLICY_FIFO = 1,    /* interception, no preemption, arrival order (MPS co-run baseline) */
   FLEP_POLICY_HPF = 2,     /* Fig. 6: priority preemption + SRPT within a priority (§5.2.1) */
   FLEP_POLICY_SLICE = 3,   /* HPF decisions on the kernel-slicing mechanism (P:96, P:391 baseline) */
-  FLEP_POLICY_FFS = 4      /* fairness first under an overhead constraint: weighted round robin,
+  FLEP_POLICY_FFS = 4,     /* fairness first under an overhead constraint: weighted round robin,
                               epoch T*W_i, W_i = priority+1, T minimal with
                               sum O_i / (T sum W_i) <= max_overhead (§5.2.2) */
+  FLEP_POLICY_REORDER = 5  /* kernel-reordering baseline without preemption: shortest queued kernel
+                              of the highest priority runs next */
 } flep_policy;
 
 typedef enum {
@@ -251,7 +253,8 @@ flep_status flep_event_log(flep_rt rt, int64_t* out6, size_t max_records, size_t
 
 /* ---- pure policy engine (host only; no GPU needed) -------------------------------------
    The exact decision logic the managed runtime uses (Fig. 6), exposed for replay parity with
-   the oracle's discrete-event simulation. kind: 1 FIFO, 2 HPF, 3 SLICE (= HPF decisions), 4 FFS. */
+   the oracle's discrete-event simulation. kind: 1 FIFO, 2 HPF, 3 SLICE (= HPF decisions), 4 FFS,
+   5 REORDER. */
 typedef struct flep_policy_s* flep_policy_t;
 flep_status flep_policy_create(int32_t kind, uint32_t num_sms, flep_policy_t* out);
 flep_status flep_policy_destroy(flep_policy_t p);

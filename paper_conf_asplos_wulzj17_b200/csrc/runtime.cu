@@ -537,7 +537,7 @@ flep_status flep_init(int device, const flep_options* opts, flep_rt* out) {
   if (opts) rt->opt = *opts;
   if (rt->opt.default_chunk == 0) rt->opt.default_chunk = 8;
   if (rt->opt.default_poll == 0) rt->opt.default_poll = 1;
-  if (rt->opt.policy < FLEP_POLICY_MANUAL || rt->opt.policy > FLEP_POLICY_FFS)
+  if (rt->opt.policy < FLEP_POLICY_MANUAL || rt->opt.policy > FLEP_POLICY_REORDER)
     return fail(FLEP_ERR_INVALID, "bad policy %d", rt->opt.policy);
   cudaDeviceProp prop;
   CUDA_TRY(cudaGetDeviceProperties(&prop, device));
@@ -1103,7 +1103,7 @@ flep_status flep_policy_set_max_overhead(flep_policy_t p, uint32_t ppm) {
 
 flep_status flep_policy_create(int32_t kind, uint32_t num_sms, flep_policy_t* out) {
   if (!out) return fail(FLEP_ERR_INVALID, "out is NULL");
-  if (kind < kPolicyFIFO || kind > kPolicyFFS) return fail(FLEP_ERR_INVALID, "bad policy kind %d", kind);
+  if (kind < kPolicyFIFO || kind > kPolicyREORDER) return fail(FLEP_ERR_INVALID, "bad policy kind %d", kind);
   *out = new flep_policy_s(kind == kPolicySLICE ? kPolicyHPF : kind, num_sms);
   return FLEP_OK;
 }

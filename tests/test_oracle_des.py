@@ -240,3 +240,18 @@ def test_spatial_width_paper_example():
     assert des.spatial_width(ex["ctas"], ex["ctas_per_sm"], ex["num_sms"]) == ex["sms"]
     assert des.spatial_width(41, 8, 15) == 6
     assert des.spatial_width(10_000, 8, 148) == 148
+
+
+def test_reordering_baseline_triplet():
+    # reordering without preemption cannot help when the long kernel arrives first;
+    # it does reorder the queued kernels (shortest first) — VA_SPMV_MM with MM arriving before SPMV
+    va, spmv, mm = 30634_000, 484_000, 1499_000
+    ks = [des.KernelSpec(0, 0, 0, va, 0, va), des.KernelSpec(1, 1, 0, mm, 0, mm),
+          des.KernelSpec(2, 2, 0, spmv, 0, spmv)]
+    r = des.simulate(des.REORDER, ks)
+    assert [d[2] for d in r.decisions] == [0, 2, 1]          # VA, then SPMV before MM
+    assert all(d[1] == "LAUNCH" for d in r.decisions)
+    f = des.simulate(des.FIFO, ks)
+    alone = [va, mm, spmv]
+    g = M.antt([f.turnaround[i] for i in range(3)], alone) / M.antt([r.turnaround[i] for i in range(3)], alone)
+    assert 1.0 < g < 1.3                                       # a small gain, far below HPF's

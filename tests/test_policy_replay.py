@@ -15,7 +15,7 @@ def flep():
 
 
 ACT = {"LAUNCH": 0, "RESUME": 1, "PREEMPT": 2}
-KIND = {des.FIFO: 1, des.HPF: 2, des.SLICE: 3}
+KIND = {des.FIFO: 1, des.HPF: 2, des.SLICE: 3, des.REORDER: 5}
 
 
 def replay_cpp(F, kind, events):
@@ -44,7 +44,7 @@ def random_trace(seed, n, prios=3, tight=False):
     return ks
 
 
-@pytest.mark.parametrize("kind", [des.FIFO, des.HPF, des.SLICE])
+@pytest.mark.parametrize("kind", [des.FIFO, des.HPF, des.SLICE, des.REORDER])
 @pytest.mark.parametrize("seed", range(25))
 def test_replay_parity_random_traces(flep, kind, seed):
     ks = random_trace(seed, 40, prios=1 + seed % 4, tight=seed % 2 == 0)
