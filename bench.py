@@ -409,7 +409,7 @@ def run_e2e(F, torch, wl, local, steps, args):
     clock from the runtime's preemption request to its observation of the drained epoch."""
     rt = F.Runtime(device=local, policy=F.POLICY_HPF)
     kLP = rt.register_kernel(F.BODY_SPMV_CSR_F32, chunk=args.lp_chunk, poll=args.lp_poll, name="spmv",
-                             model=(0, 0, 0, 0, 70_000), prefetch=bool(args.prefetch))
+                             model=(0, 0, 0, 0, 70_000), prefetch=bool(args.prefetch), started_hint=True)
     kHP = rt.register_kernel(F.BODY_STENCIL5_F32, chunk=args.hp_chunk, poll=1, name="stencil",
                              model=(0, 0, 0, 0, 30_000), prefetch=bool(args.hp_prefetch))
     pin = lambda a: torch.from_numpy(np.ascontiguousarray(a)).pin_memory()  # noqa: E731

@@ -81,7 +81,7 @@ typedef enum {
 typedef enum {
   FLEP_BODY_SAXPY_I32 = 1,     /* y <- a*x + y, int32, wraps mod 2^32; 256 elements per block */
   FLEP_BODY_SAXPY_F32 = 2,     /* y <- a*x + y, fp32; 256 elements per block */
-  FLEP_BODY_SPMV_CSR_F32 = 3,  /* y = A x, CSR fp32; 32 rows per block */
+  FLEP_BODY_SPMV_CSR_F32 = 3,  /* y = A x, CSR fp32; 128 rows per block */
   FLEP_BODY_STENCIL5_F32 = 4,  /* 5-point out-of-place sweep, fp32; 64x64 cells per block */
   FLEP_BODY_STENCIL5_I32 = 5,  /* 5-point integer sweep, wraps mod 2^32; 64x64 cells per block */
   FLEP_BODY_GEMM_BF16 = 6      /* C = A B^T, bf16 in, fp32 accumulate (tcgen05), bf16 out;
@@ -131,6 +131,10 @@ typedef struct {
    latency; a worker that must yield still executes the chunk it holds, so the drain can take up
    to one extra chunk). */
 #define FLEP_KFLAG_PREFETCH 1u
+/* The first worker of every epoch publishes "epoch started" to the launch's pinned status slot
+   (flep_launch_info.started_epoch). Off by default: the system-scope store it needs delays the
+   grid's completion by about a microsecond. */
+#define FLEP_KFLAG_STARTED_HINT 2u
 
 typedef enum {
   FLEP_STATE_QUEUED = 0,     /* intercepted, waiting for a scheduling decision (S2) */
@@ -153,7 +157,8 @@ typedef struct {
   uint32_t n_yield;            /* yield width currently requested (0 = none) */
   int64_t t_last_request;      /* host ns of the last preempt request issued by the runtime */
   int64_t t_last_drain;        /* host ns the runtime observed the last PREEMPTED epoch end */
-  uint32_t started_epoch;      /* newest epoch (1-based) whose first worker has begun running */
+  uint32_t started_epoch;      /* newest epoch (1-based) whose first worker has begun running
+                                  (kernels registered with FLEP_KFLAG_STARTED_HINT; else 0) */
   uint32_t reserved;
 } flep_launch_info;
 

@@ -151,7 +151,7 @@ struct SpmvBody : NoResources {
 template <bool kInt>
 struct Stencil5Body : NoResources {
   static constexpr int kThreads = 256;
-  static constexpr int kMinBlocks = 3;
+  static constexpr int kMinBlocks = 4;
   static constexpr uint32_t kTile = 64;
   using Args = flep_stencil_args;
 

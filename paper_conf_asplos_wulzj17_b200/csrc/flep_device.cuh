@@ -81,6 +81,8 @@ struct WorkerParams {
   uint32_t prefetch;       // 1: fetch chunk j+1 while chunk j runs (hides the atomic's latency;
                            //    a stopping worker still processes the prefetched chunk)
   uint32_t gen_first;      // generation of this launch's first epoch
+  uint32_t started_hint;   // 1: worker 0 publishes "epoch started" to the host slot at entry (a
+                           //    system-scope store: the kernel's completion then waits for it)
 };
 
 __device__ __forceinline__ uint32_t smid_reg() {
@@ -148,29 +150,49 @@ struct SchedState {
   bool first = true;                 // first step of this worker
 };
 
+// pull_task. In the first epoch of a launch the counter hands out blocks after the W
+// static first chunks (reading R20), so the effective counter there is ctr + W*C.
+__device__ __forceinline__ uint32_t fetch_chunk(const WorkerParams& p) {
+  const uint32_t s = atomicAdd(&p.cb->ctr, p.chunk);
+  return p.epoch == p.gen_first ? s + p.workers * p.chunk : s;
+}
+
 __device__ __forceinline__ uint32_t next_chunk(const WorkerParams& p, SchedState& st, WorkerShared& ws) {
-  uint32_t base;
-  if (st.first) {                                    // the launch already completed in an earlier
-    st.first = false;                                // epoch (a refill raced with the last blocks):
-    if (ld_relaxed_gpu(&p.cb->done_gen) >= p.gen_first) {   // leave without touching the counter
-      ws.reason = kReasonExhausted;
-      return 0xffffffffu;
+  uint32_t base = 0xffffffffu;
+  bool have = false;
+  if (st.first) {
+    st.first = false;
+    if (p.epoch == p.gen_first) {
+      // First epoch: worker i starts on the static chunk [i*C, i*C + C) (R20): no poll and no
+      // atomic before the first body, so the grid starts moving data at once. A static chunk is
+      // "fetched" at launch and always processed (A4); the first poll comes at the next step.
+      base = blockIdx.x * p.chunk;
+      have = true;
+    } else {
+      // A later epoch: the launch may already have completed in an earlier one (a refill raced
+      // with the last blocks) -> leave without touching the counter. Both loads are issued back
+      // to back: one L2 round trip. The poll doubles as the entry check of a2 (Fig. 4(c)).
+      const uint32_t c = ld_relaxed_gpu(p.ctrl);
+      const uint32_t dg = ld_relaxed_gpu(&p.cb->done_gen);
+      if (dg >= p.gen_first) { ws.reason = kReasonExhausted; return 0xffffffffu; }
+      if (should_yield(c, p, smid_reg())) { ws.reason = kReasonYield; return 0xffffffffu; }
     }
-  }
-  if (st.k == 0 && !st.stopping) {                   // amortised poll (Fig. 4(b))
+  } else if (st.k == 0 && !st.stopping) {            // amortised poll (Fig. 4(b))
     const uint32_t c = ld_relaxed_gpu(p.ctrl);
     if (should_yield(c, p, smid_reg())) { st.stopping = true; ws.reason = kReasonYield; }
   }
-  if (st.held != 0xffffffffu) {                      // a fetched chunk is always processed (A4)
-    base = st.held;
-    st.held = 0xffffffffu;
-  } else {
-    base = st.stopping ? 0xffffffffu : atomicAdd(&p.cb->ctr, p.chunk);   // pull_task
+  if (!have) {
+    if (st.held != 0xffffffffu) {                    // a fetched chunk is always processed (A4)
+      base = st.held;
+      st.held = 0xffffffffu;
+    } else if (!st.stopping) {
+      base = fetch_chunk(p);
+    }
   }
   if (base != 0xffffffffu && base >= p.n_blocks) { base = 0xffffffffu; ws.reason = kReasonExhausted; }
   if (base != 0xffffffffu) {
     ws.blocks += min(p.chunk, p.n_blocks - base);
-    if (p.prefetch && !st.stopping) st.held = atomicAdd(&p.cb->ctr, p.chunk);   // overlaps the body
+    if (p.prefetch && !st.stopping) st.held = fetch_chunk(p);   // overlaps the body
     if (p.trigger_block - base < p.chunk) {          // device self-trigger inside this chunk
       const uint32_t e = p.epoch % kEvEpochs;
       p.cb->ep_t_trigger[e] = gtimer();
@@ -202,7 +224,7 @@ flep_worker(const __grid_constant__ typename Body::Args args, const WorkerParams
   const uint32_t tid = threadIdx.x;
   if (tid == 0) {
     ws.sm = smid_reg(); ws.t_entry = gtimer(); ws.blocks = 0; ws.reason = 0;
-    if (blockIdx.x == 0 && p.status) st_relaxed_sys(&p.status->started, p.epoch);   // host hint
+    if (blockIdx.x == 0 && p.started_hint && p.status) st_relaxed_sys(&p.status->started, p.epoch);
   }
   Body::setup(args);                 // per-worker resources (e.g. TMEM, mbarriers); may sync
   if constexpr (Body::kPersistent) {
@@ -234,9 +256,13 @@ flep_worker(const __grid_constant__ typename Body::Args args, const WorkerParams
     e.t_entry = ws.t_entry; e.t_exit = t_exit;
     const unsigned long long old = atomicAdd(&p.cb->done_exited, (1ull << 32) | my_blocks);
     if ((uint32_t)(old >> 32) + 1 == p.workers) {        // last worker of this epoch
-      const bool already = ld_relaxed_gpu(&p.cb->done_gen) >= p.gen_first;
+      // both loads issued back to back (one round trip); the first epoch of a launch cannot
+      // find it already complete
+      const bool first_epoch = p.epoch == p.gen_first;
+      const uint32_t raw = ld_relaxed_gpu(&p.cb->ctr);   // every fetch has completed by now
+      const bool already = !first_epoch && ld_relaxed_gpu(&p.cb->done_gen) >= p.gen_first;
+      const uint32_t c = first_epoch ? raw + p.workers * p.chunk : raw;   // effective counter (R20)
       const uint32_t d = already ? p.n_blocks : (uint32_t)old + my_blocks;
-      const uint32_t c = ld_relaxed_gpu(&p.cb->ctr);     // every fetch has completed by now
       const uint32_t st = (d >= p.n_blocks) ? kStateDone : kStatePreempted;
       const uint32_t ei = p.epoch % kEvEpochs;
       p.cb->ep_t_end[ei] = t_exit; p.cb->ep_done[ei] = d; p.cb->ep_ctr[ei] = c;
@@ -247,7 +273,8 @@ flep_worker(const __grid_constant__ typename Body::Args args, const WorkerParams
         if (!already) p.cb->done_gen = p.epoch;
       } else {
         p.cb->done_exited = (unsigned long long)d;       // exits reset, progress kept
-      }
+        p.cb->ctr = c;                                   // later epochs fetch from the effective
+      }                                                  // counter (no fetch is in flight now)
       if (p.status) {
         st_relaxed_sys(&p.status->ctr, c);
         st_relaxed_sys_u64(&p.status->t_end, t_exit);

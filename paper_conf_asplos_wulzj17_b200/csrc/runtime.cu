@@ -295,6 +295,7 @@ flep_status start_epoch(flep_rt rt, Launch& L) {
   p.trigger_n = L.trig_n;
   p.prefetch = (L.flags & FLEP_KFLAG_PREFETCH) ? 1u : 0u;
   p.gen_first = L.gen0 + 1;
+  p.started_hint = (L.flags & FLEP_KFLAG_STARTED_HINT) ? 1u : 0u;
   L.trig_block = kNoTrigger;
   L.trig_n = 0;
   cudaError_t e = L.ops->worker(L.args.data(), p, L.workers, L.exec, L.cov != nullptr);

@@ -22,6 +22,7 @@ REASON_YIELD, REASON_EXHAUSTED = 1, 2
 ACTION_NAMES = {0: "LAUNCH", 1: "RESUME", 2: "PREEMPT"}
 NO_TRIGGER = 0xFFFFFFFF
 KFLAG_PREFETCH = 1
+KFLAG_STARTED_HINT = 2
 
 
 class Dim3(C.Structure):
@@ -200,9 +201,10 @@ class Runtime:
         self.close()
 
     def register_kernel(self, body, chunk=0, poll=0, name="", model=(0, 0, 0, 0, 1), overhead_ns=0,
-                        prefetch=False, ctas_per_sm=0):
+                        prefetch=False, ctas_per_sm=0, started_hint=False):
+        flags = (KFLAG_PREFETCH if prefetch else 0) | (KFLAG_STARTED_HINT if started_hint else 0)
         d = KernelDesc(name.encode(), body, chunk, poll, (C.c_double * 5)(*model), overhead_ns,
-                       KFLAG_PREFETCH if prefetch else 0, ctas_per_sm)
+                       flags, ctas_per_sm)
         k = C.c_int32()
         check(self.L.flep_register_kernel(self.h, C.byref(d), C.byref(k)), "flep_register_kernel")
         return k.value

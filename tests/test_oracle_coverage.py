@@ -147,3 +147,58 @@ def test_expected_prefix():
     assert cv.expected_prefix(0, 3) == [0, 0, 0]
     assert cv.expected_prefix(2, 3) == [1, 1, 0]
     assert cv.expected_prefix(9, 3) == [1, 1, 1]
+
+
+# ---- static first chunks (R20): the product wrapper's first epoch -------------------
+
+@pytest.mark.parametrize("C,K,pf", [(1, 1, False), (1, 2, False), (2, 1, False), (1, 1, True), (2, 1, True)])
+def test_exhaustive_static_first_no_violations(C, K, pf):
+    ws = (0, 1) if pf else (0, 0, 1)
+    # enough blocks that a request can still find work after the static chunks (and the first
+    # K-chunk period, and a prefetched chunk)
+    r = cv.explore(_cfg(n_blocks=len(ws) * C * (K + pf) + 1, chunk=C, poll=K, worker_sm=ws,
+                        prefetch=pf, static_first=True))
+    assert r.violations == set()
+    assert r.preempted_epoch_ends > 0
+
+
+@pytest.mark.parametrize("n,C,ws", [(5, 1, (0, 0, 1, 1)), (7, 2, (0, 1)), (2, 1, (0, 0, 1, 1)),
+                                    (3, 2, (0, 0, 1)), (4, 4, (0,))])
+def test_static_first_final_counter_closed_form(n, C, ws):
+    # every worker holding a static chunk below N runs it and then fails exactly one fetch;
+    # workers whose static chunk starts at or beyond N leave at once: the effective counter is
+    # W*C + ceil(N/C)*C, the same closed form as with dynamic first fetches (A5)
+    for pf in (False, True):
+        r = cv.explore(cv.Config(n_blocks=n, chunk=C, poll=1, worker_sm=ws, num_sms=2, prefetch=pf,
+                                 static_first=True))
+        assert r.violations == set()
+        assert r.terminal_ctrs == {cv.final_counter_no_preempt(n, C, len(ws))}
+
+
+def test_static_first_spatial_refill():
+    r = cv.explore(_cfg(n_blocks=7, chunk=1, poll=1, worker_sm=(0, 0, 1), preempt_widths=(1,),
+                        max_events=2, allow_refill=True, static_first=True))
+    assert r.violations == set()
+
+
+def test_hand_traced_static_first_preempt():
+    # two workers, N=5, C=1: both run their static chunks (blocks 0 and 1) without polling; a
+    # temporal request then stops both at their first poll. The drained epoch covers [0, 2) and
+    # the counter (W*C = 2) names exactly that prefix; the resume finishes blocks 2..4.
+    cfg = cv.Config(n_blocks=5, chunk=1, poll=1, worker_sm=(0, 1), num_sms=2, preempt_widths=(2,),
+                    max_events=1, static_first=True)
+    st = cv.initial_state(cfg)
+    assert st[0] == 2
+    for lab in ["w0.fetch", "w1.fetch", "preempt(2)", "w0.proc", "w1.proc", "w0.poll", "w1.poll",
+                "w0.exit", "w1.exit"]:
+        st = dict(cv.successors(cfg, st))[lab]
+    ctr, ctrl, done, exited, cov, epoch, status, workers, ev, extra = st
+    assert status == cv.ST_PREEMPTED and cov == (1, 1, 0, 0, 0) and ctr == 2 and done == 2
+    st = dict(cv.successors(cfg, st))["resume"]
+    assert st[7][0][0] == cv.POLL and st[7][0][4] == cv.NOCHUNK     # later epochs poll first
+    while True:
+        succ = cv.successors(cfg, st)
+        if not succ:
+            break
+        st = succ[0][1]
+    assert st[6] == cv.ST_DONE and st[4] == (1, 1, 1, 1, 1)

@@ -20,7 +20,7 @@ def main():
         n = 1 << 28
         x = torch.ones(n, dtype=torch.int32, device="cuda")
         y = torch.ones(n, dtype=torch.int32, device="cuda")
-        k = rt.register_kernel(F.BODY_SAXPY_I32, chunk=8, poll=1)
+        k = rt.register_kernel(F.BODY_SAXPY_I32, chunk=8, poll=1, started_hint=True)
         lat, dev = [], []
         for r in range(30):
             h = rt.launch(k, F.saxpy_grid(n), F.saxpy_i32_args(y, x, 1))

@@ -20,6 +20,8 @@ def main():
     ap.add_argument("--reps", type=int, default=2)
     ap.add_argument("--chunk", type=int, default=1)
     ap.add_argument("--prefetch", type=int, default=1)
+    ap.add_argument("--poll", type=int, default=1)
+    ap.add_argument("--combos", default="", help="C:K:prefetch[,...] wrapped variants (overrides --chunk/--poll/--prefetch)")
     a = ap.parse_args()
     import torch
     from paper_conf_asplos_wulzj17_b200 import build, flep as F
@@ -51,15 +53,17 @@ def main():
         Cg = torch.empty(M, M, device="cuda", dtype=torch.bfloat16)
         jobs.append(("gemm", F.BODY_GEMM_BF16, F.gemm_grid(M, M), F.gemm_args(Cg, A, B), (A, B, Cg)))
     s = torch.cuda.current_stream()
+    combos = [tuple(map(int, c.split(":"))) for c in a.combos.split(",")] if a.combos else [(a.chunk, a.poll, a.prefetch)]
     for name, body, grid, args, keep in jobs:
-        k = rt.register_kernel(body, chunk=a.chunk, poll=1, prefetch=bool(a.prefetch))
+        ks = [rt.register_kernel(body, chunk=C, poll=K, prefetch=bool(pf)) for C, K, pf in combos]
         for _ in range(a.reps):
             flush.zero_()
             rt.launch_unwrapped(body, grid, args, stream=s)
             torch.cuda.synchronize()
-            flush.zero_()
-            h = rt.launch(k, grid, args, stream=s)
-            rt.sync(h)
+            for k in ks:
+                flush.zero_()
+                h = rt.launch(k, grid, args, stream=s)
+                rt.sync(h)
     torch.cuda.synchronize()
     rt.close()
 

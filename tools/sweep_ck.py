@@ -21,6 +21,8 @@ def main():
     ap.add_argument("--polls", default="1")
     ap.add_argument("--cps", default="0")
     ap.add_argument("--prefetch", default="0,1")
+    ap.add_argument("--gate-us", type=float, default=0.0,
+                    help="spin the stream this long before the start event (hides host submission latency)")
     a = ap.parse_args()
     import torch
     from paper_conf_asplos_wulzj17_b200 import build, flep as F
@@ -73,6 +75,8 @@ def main():
         ts = []
         for r in range(a.reps + 2):
             flush.zero_()
+            if a.gate_us > 0:
+                torch.cuda._sleep(int(a.gate_us * 2000))
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record(s)
             h = fn()
