@@ -232,11 +232,102 @@ def run_corun1(args, rank, world, local):
            "clocks": clk.summary()}
     if rank == 0:
         print(json.dumps(out), flush=True)
-        import os
-        dbg = os.environ.get("FLEP_EVIDENCE_DIR")
-        if dbg:
-            with open(os.path.join(dbg, "queue_debug.json"), "w") as fh:
-                json.dump(debug, fh)
+    barrier(world)
+
+
+# ------------------------------------------------------------------------------------------
+def run_gemm_preempt(args, rank, world, local):
+    """Full-GPU preemption of the dense contraction: LP bf16 GEMM 8192^3 (C = A B^T, tcgen05)
+    preempted at a random tile by HP stencil5 4096^2 (device self-trigger, temporal), then
+    resumed. Latency = request -> last GEMM CTA gone (device %globaltimer). Each step's result
+    must be bit-identical to an uninterrupted run of the same binary (SURVEY §8(c) parity), and a
+    sample of C is checked against the oracle (fp64 dot products, 2e-2 relative)."""
+    import torch
+    from bench import ClockSampler, L2Flush, barrier, physical_gpu_index
+    from oracle import workloads as W
+    from paper_conf_asplos_wulzj17_b200 import flep as F
+    torch.cuda.set_device(local)
+    rt = F.Runtime(device=local, exec_on_user_stream=True)
+    M = N = K = 8192
+    g = torch.Generator(device="cuda")
+    g.manual_seed(8 + rank)
+    A_ = (torch.rand(M, K, device="cuda", generator=g) * 2 - 1).to(torch.bfloat16)
+    B_ = (torch.rand(N, K, device="cuda", generator=g) * 2 - 1).to(torch.bfloat16)
+    C_ = torch.empty(M, N, device="cuda", dtype=torch.bfloat16)
+    st_in = torch.rand(4096, 4096, device="cuda", generator=g)
+    st_out = torch.empty_like(st_in)
+    in_tile = bool(args.gemm_in_tile)
+    k_lp = rt.register_kernel(F.BODY_GEMM_BF16, chunk=1, poll=1, name="gemm", in_tile=in_tile)
+    k_hp = rt.register_kernel(F.BODY_STENCIL5_F32, chunk=2, poll=1, prefetch=True, name="stencil")
+    lp_args, lp_grid = F.gemm_args(C_, A_, B_), F.gemm_grid(M, N)
+    hp_args, hp_grid = F.stencil_args(st_out, st_in), F.stencil_grid(4096)
+    nb = lp_grid[0] * lp_grid[1]
+    flush = L2Flush(torch)
+    SA = torch.cuda.Stream(priority=-2)
+    SB = torch.cuda.Stream(priority=0)
+    # uninterrupted reference of the same binary
+    h = rt.launch(k_lp, lp_grid, lp_args, stream=SA)
+    rt.sync(h)
+    torch.cuda.synchronize()
+    C_ref = C_.clone()
+    rng = gen.rng(5000 + rank)
+    lat, drain, hpt, bad, pre, epochs = [], [], [], 0, 0, []
+    with ClockSampler(physical_gpu_index(local)) as clk:
+        for i in range(args.warmup + args.steps):
+            C_.zero_()
+            flush.zero_()
+            torch.cuda.synchronize()
+            tstar = int(rng.integers(nb // 4, 3 * nb // 4))
+            rt.arm_next_trigger(tstar, rt.num_sms)
+            h = rt.launch(k_lp, lp_grid, lp_args, priority=0, stream=SA)
+            h2 = rt.launch(k_hp, hp_grid, hp_args, priority=1, stream=SB)
+            rt.wait_epoch(h, timeout_ns=20_000_000_000)
+            preempted = rt.query(h).state == F.STATE_PREEMPTED
+            rt.sync(h2, timeout_ns=20_000_000_000)
+            if preempted:
+                rt.resume(h)
+            rt.sync(h, timeout_ns=20_000_000_000)
+            torch.cuda.synchronize()
+            ep = rt.epoch_info(h, 1)
+            ev_hp = rt.events(h2, 1)
+            same = bool(torch.equal(C_, C_ref))
+            if i < args.warmup:
+                continue
+            bad += 0 if same else 1
+            if preempted and ep.t_trigger:
+                pre += 1
+                hs, he = _span(ev_hp)
+                lat.append((hs - ep.t_trigger) / 1e3)
+                drain.append((ep.t_end - ep.t_trigger) / 1e3)
+                hpt.append((he - ep.t_trigger) / 1e3)
+                epochs.append(rt.query(h).epoch)
+    # oracle spot check of the last result (rows x cols sampled; fp64 dot products of bf16 values)
+    r_idx = gen.rng(9).integers(0, M, 16)
+    c_idx = gen.rng(10).integers(0, N, 64)
+    a = A_[r_idx].view(torch.int16).cpu().numpy().view(np.uint16)
+    b = B_[c_idx].view(torch.int16).cpu().numpy().view(np.uint16)
+    ref = W.gemm_bf16(a, b)
+    got = C_[r_idx][:, c_idx].float().cpu().numpy()
+    rms = float(np.sqrt(np.mean(ref ** 2)))
+    worst = float(np.max(np.abs(got - ref) / (np.abs(ref) + rms)))
+    rt.close()
+    out = {"metric": METRIC, "value": round(float(np.median(drain)), 3) if drain else None, "unit": "us",
+           "value_definition": "full-GPU preemption latency of a bf16 GEMM 8192^3 victim: device request -> "
+                               "last GEMM CTA gone, p50",
+           "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "higher_is_better": False,
+           "scaling": "weak", "vs_baseline": None, "dtype": "bf16", "data": "synthetic (seeded)",
+           "config": {"workload": "LP GEMM bf16 8192^3 (tcgen05, 128x256 tiles) preempted by HP stencil5 4096^2",
+                      "chunk": 1, "poll": 1, "in_tile": in_tile},
+           "preempted_steps": pre, "not_bit_identical_to_uninterrupted": bad,
+           "oracle_sample_max_rel": worst, "tol": 2e-2,
+           "drain_us": {"p50": round(float(np.median(drain)), 3) if drain else None,
+                        "p99": round(float(np.percentile(drain, 99)), 3) if drain else None,
+                        "max": round(float(np.max(drain)), 3) if drain else None},
+           "waiting_start_us_p50": round(float(np.median(lat)), 3) if lat else None,
+           "hp_turnaround_us_p50": round(float(np.median(hpt)), 3) if hpt else None,
+           "clocks": clk.summary()}
+    if rank == 0:
+        print(json.dumps(out), flush=True)
     barrier(world)
 
 

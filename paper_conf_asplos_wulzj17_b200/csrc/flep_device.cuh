@@ -83,7 +83,24 @@ struct WorkerParams {
   uint32_t gen_first;      // generation of this launch's first epoch
   uint32_t started_hint;   // 1: worker 0 publishes "epoch started" to the host slot at entry (a
                            //    system-scope store: the kernel's completion then waits for it)
+  void* partial;           // in-tile preemption (FLEP_KFLAG_IN_TILE, GEMM): W partial-tile records
+                           // then W accumulator spill slots (layout: partial_bytes below), or nullptr
 };
+
+// In-tile preemption state: record i belongs to worker i of every epoch of a launch.
+struct PartialTile {
+  uint32_t valid;          // 1: worker i of the previous epoch stopped inside tile b
+  uint32_t b;              // original block (tile) in progress
+  uint32_t kb;             // first k-step not yet accumulated (0: nothing accumulated)
+  uint32_t b_end;          // end of the chunk the tile belongs to (tiles b+1..b_end-1 not started)
+};
+constexpr size_t kSpillBytes = 128u * 256u * 4u;          // one fp32 128x256 accumulator
+__host__ __device__ constexpr size_t partial_header_bytes(uint32_t workers) {
+  return ((size_t)workers * sizeof(PartialTile) + 1023u) & ~(size_t)1023u;
+}
+__host__ __device__ constexpr size_t partial_bytes(uint32_t workers) {
+  return partial_header_bytes(workers) + (size_t)workers * kSpillBytes;
+}
 
 __device__ __forceinline__ uint32_t smid_reg() {
   uint32_t r; asm volatile("mov.u32 %0, %%smid;" : "=r"(r)); return r;

@@ -12,8 +12,16 @@
 //   warps 4..7    : epilogue — tcgen05.ld 32x32b.x32 → bf16 → global, then release the
 //                   accumulator (tmem_empty)
 // Pipeline phases persist in shared memory across chunks, so a worker's consecutive tasks share
-// one pipeline; the wrapper's barrier separates chunks (the poll point). Preemption is at tile
-// granularity (in-tile preemption is SURVEY f4).
+// one pipeline; the wrapper's barrier separates chunks (the poll point).
+//
+// In-tile preemption (kernels registered with FLEP_KFLAG_IN_TILE): the producer also
+// polls the control word every kInTilePoll k-steps inside a tile. On a request naming its SM it
+// stops issuing k-steps and sends a stop marker through the stage ring; the MMA thread commits
+// the partial accumulator, the epilogue spills it (fp32, exact) to the worker's slot and the
+// producer records {tile, next k-step, chunk end}. Worker i of the next epoch restores the
+// accumulator into TMEM (tcgen05.st) and continues the same k-loop: every k-step of every tile is
+// accumulated exactly once, in the same order, so the result is bit-identical to an
+// uninterrupted run. Preemption latency drops from one tile (~55 us at 8192^3) to a few k-steps.
 #pragma once
 #include <cuda.h>
 #include <cuda_bf16.h>
@@ -25,6 +33,9 @@
 
 #ifndef FLEP_GEMM_GROUP
 #define FLEP_GEMM_GROUP 16
+#endif
+#ifndef FLEP_GEMM_KPOLL
+#define FLEP_GEMM_KPOLL 8         // k-steps (BK = 64 each) between in-tile polls
 #endif
 
 namespace flep {
@@ -51,7 +62,11 @@ struct GemmBody {
     uint64_t full[STAGES], empty[STAGES], tmem_full, tmem_empty;
     uint64_t tfull[2], tempty[2];     // persistent loop: double-buffered accumulators
     uint64_t qfull[QDEPTH], qempty[QDEPTH];
+    uint64_t trest[2];                // epilogue restored a spilled accumulator into this half
     uint32_t tile_q[QDEPTH];
+    uint32_t tile_kb0[QDEPTH];        // first k-step of the tile (> 0: continue a spilled tile)
+    uint32_t tile_kend[QDEPTH];       // k-step the producer stopped at (nk: runs to the end)
+    uint32_t acc_kend[2];             // MMA -> epilogue: k-steps accumulated in this half
     uint32_t tmem_base;
     uint32_t p_stage, p_phase;        // producer
     uint32_t m_stage, m_phase, m_acc; // MMA issuer
@@ -113,7 +128,10 @@ struct GemmBody {
       for (uint32_t i = 0; i < STAGES; ++i) { mbar_init(&s->full[i], 1); mbar_init(&s->empty[i], 1); }
       mbar_init(&s->tmem_full, 1);
       mbar_init(&s->tmem_empty, 128);
-      for (uint32_t i = 0; i < 2; ++i) { mbar_init(&s->tfull[i], 1); mbar_init(&s->tempty[i], 128); }
+      // tfull: the MMA's tcgen05.commit + a plain arrive of the MMA thread (publishes acc_kend)
+      for (uint32_t i = 0; i < 2; ++i) {
+        mbar_init(&s->tfull[i], 2); mbar_init(&s->tempty[i], 128); mbar_init(&s->trest[i], 128);
+      }
       for (uint32_t i = 0; i < QDEPTH; ++i) { mbar_init(&s->qfull[i], 1); mbar_init(&s->qempty[i], 5); }
       s->p_stage = s->p_phase = s->m_stage = s->m_phase = s->m_acc = 0;
       s->e_acc[0] = s->e_acc[1] = s->e_acc[2] = s->e_acc[3] = 0;
@@ -233,35 +251,114 @@ struct GemmBody {
     }
   }
 
+  static constexpr uint32_t kInTilePoll = FLEP_GEMM_KPOLL;
+  static constexpr uint32_t kMinLeft = 4;      // closer than this to the tile's end: finish it
+
+  __device__ static float4* spill_slot(const WorkerParams& p) {
+    return reinterpret_cast<float4*>(reinterpret_cast<uint8_t*>(p.partial) + partial_header_bytes(p.workers) +
+                                     (size_t)blockIdx.x * kSpillBytes);
+  }
+  // TMEM <-> registers, 32 lanes x 32 columns per warp
+  __device__ static void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+        "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+        : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+          "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]),
+          "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]),
+          "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
+        : "r"(taddr));
+    asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+  }
+  __device__ static void tmem_st32(uint32_t taddr, const uint32_t (&r)[32]) {
+    asm volatile(
+        "tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,"
+        "%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32};"
+        :: "r"(taddr), "r"(r[0]), "r"(r[1]), "r"(r[2]), "r"(r[3]), "r"(r[4]), "r"(r[5]), "r"(r[6]), "r"(r[7]),
+           "r"(r[8]), "r"(r[9]), "r"(r[10]), "r"(r[11]), "r"(r[12]), "r"(r[13]), "r"(r[14]), "r"(r[15]),
+           "r"(r[16]), "r"(r[17]), "r"(r[18]), "r"(r[19]), "r"(r[20]), "r"(r[21]), "r"(r[22]), "r"(r[23]),
+           "r"(r[24]), "r"(r[25]), "r"(r[26]), "r"(r[27]), "r"(r[28]), "r"(r[29]), "r"(r[30]), "r"(r[31])
+        : "memory");
+  }
+
   // ---- persistent FLEP worker loop (warp-specialised; chunk boundaries do not drain the
   // pipeline). tid 0 is the scheduler AND the TMA producer: it runs the FLEP scheduling step
   // (poll / fetch / trigger, next_chunk), pushes every tile of the fetched chunk into a 4-deep
   // smem queue, then issues that tile's TMA loads; a STOP sentinel ends the loop. The MMA thread
   // and the 4 epilogue warps consume the queue; accumulators alternate between two TMEM halves
-  // so tile t's epilogue overlaps tile t+1's MMAs. Every fetched tile is computed (A4).
+  // so tile t's epilogue overlaps tile t+1's MMAs. Every fetched tile is computed (A4) — with
+  // in-tile preemption, possibly across epochs (spill / restore, see the file header).
   __device__ static void persistent(const Args& g, const WorkerParams& p, WorkerShared& ws) {
     State* s = state();
     uint8_t* base = ring();
     const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31u;
     const uint32_t nk = g.k / BK;
     const uint32_t gx = p.gx;
+    const bool in_tile = p.partial != nullptr;
     constexpr uint32_t STOP = 0xffffffffu;
     if (warp == 0) {
       if (lane == 0) {                                     // ---- scheduler + TMA producer
         SchedState sch;
         uint32_t qi = 0, qph = 0, st = 0, ph = 0;
-        while (true) {
-          const uint32_t b0 = next_chunk(p, sch, ws);
-          const uint32_t b1 = (b0 == STOP) ? b0 : min(b0 + p.chunk, p.n_blocks);
-          for (uint32_t b = b0; b != STOP && b < b1; ++b) {
+        PartialTile* mine = in_tile ? reinterpret_cast<PartialTile*>(p.partial) + blockIdx.x : nullptr;
+        uint32_t rb0 = STOP, rb1 = 0, rkb = 0;             // a spilled tile to continue first
+        if (in_tile) {
+          if (p.epoch == p.gen_first) {
+            mine->valid = 0;                               // no record survives from another launch
+          } else {
+            const PartialTile e = *mine;                   // written by the previous grid
+            if (e.valid) {
+              sch.first = false;                           // (the launch is not complete)
+              const uint32_t c = ld_relaxed_gpu(p.ctrl);   // entry check (a2) before taking it
+              if (should_yield(c, p, smid_reg())) {
+                ws.reason = kReasonYield;                  // the record stays for a later epoch
+                rb0 = STOP; rb1 = 1;                       // (marker: leave at once)
+              } else {
+                rb0 = e.b; rb1 = e.b_end; rkb = e.kb;
+                mine->valid = 0;
+                ws.blocks += e.b_end - e.b;                // counted again when they complete
+              }
+            }
+          }
+        }
+        bool leave = (rb0 == STOP && rb1 == 1);
+        while (!leave) {
+          uint32_t b0, b1, kbs = 0;
+          bool restoring = false;
+          if (rb0 != STOP) {
+            b0 = rb0; b1 = rb1; kbs = rkb; restoring = true;
+            rb0 = STOP;
+          } else {
+            b0 = next_chunk(p, sch, ws);
+            if (b0 == STOP) break;
+            b1 = min(b0 + p.chunk, p.n_blocks);
+          }
+          for (uint32_t b = b0; b < b1; ++b) {
+            const bool cont = restoring && b == b0;        // continue a spilled tile
+            const uint32_t kb0 = cont ? kbs : 0u;
             mbar_wait(&s->qempty[qi], qph ^ 1u);
+            const uint32_t my_q = qi;
             s->tile_q[qi] = b;
+            s->tile_kb0[qi] = kb0;
+            s->tile_kend[qi] = nk;
             mbar_arrive(&s->qfull[qi]);
             if (++qi == QDEPTH) { qi = 0; qph ^= 1u; }
-            if (p.cov) atomicAdd(&p.cov[b], 1u);
+            // coverage log: a tile counts once, when its chunk is first handed out (the tiles of
+            // a chunk stopped in-tile are counted at the stop, not again when restored)
+            if (p.cov && !restoring) atomicAdd(&p.cov[b], 1u);
             int32_t tm, tn;
-          tile_coords(b, gx, p_gy(g), tm, tn);
-            for (uint32_t kb = 0; kb < nk; ++kb) {
+            tile_coords(b, gx, p_gy(g), tm, tn);
+            uint32_t kb = kb0, pend = 0;
+            bool pend_valid = false, stop = false;
+            for (; kb < nk; ++kb) {
+              if (in_tile) {                               // amortised in-tile poll, issued one
+                const uint32_t j = kb - kb0;               // half period before it is consumed
+                if (pend_valid && j % kInTilePoll == kInTilePoll / 2) {
+                  pend_valid = false;
+                  if (nk - kb > kMinLeft && should_yield(pend, p, smid_reg())) { stop = true; break; }
+                }
+                if (j % kInTilePoll == 0 && j > 0) { pend = ld_relaxed_gpu(p.ctrl); pend_valid = true; }
+              }
               mbar_wait(&s->empty[st], ph ^ 1u);
               uint8_t* sa = base + st * kStage;
               uint8_t* sb = sa + kBytesA;
@@ -270,36 +367,57 @@ struct GemmBody {
               tma_2d(&g.tma_b, sb, &s->full[st], (int32_t)(kb * BK), tn * (int32_t)BN);
               if (++st == STAGES) { st = 0; ph ^= 1u; }
             }
-          }
-          if (b0 == STOP) {
-            mbar_wait(&s->qempty[qi], qph ^ 1u);
-            s->tile_q[qi] = STOP;
-            mbar_arrive(&s->qfull[qi]);
-            break;
+            if (stop) {
+              // stop marker: the next stage carries no data; the MMA sees kend == kb and commits
+              mbar_wait(&s->empty[st], ph ^ 1u);
+              s->tile_kend[my_q] = kb;
+              mbar_arrive(&s->full[st]);
+              if (++st == STAGES) { st = 0; ph ^= 1u; }
+              mine->b = b; mine->kb = kb; mine->b_end = b1; mine->valid = 1;
+              if (p.cov && !restoring)
+                for (uint32_t bb = b + 1; bb < b1; ++bb) atomicAdd(&p.cov[bb], 1u);
+              ws.blocks -= b1 - b;                         // tiles b..b1-1 are not complete
+              ws.reason = kReasonYield;
+              leave = true;
+              break;
+            }
           }
         }
+        mbar_wait(&s->qempty[qi], qph ^ 1u);
+        s->tile_q[qi] = STOP;
+        mbar_arrive(&s->qfull[qi]);
       }
     } else if (warp == 1) {
       if (lane == 0) {                                     // ---- MMA issuer
         uint32_t qi = 0, qph = 0, st = 0, ph = 0, acc = 0, aph = 0;
+        uint32_t rph[2] = {0u, 0u};
         const uint32_t tmem0 = s->tmem_base;
         while (true) {
           mbar_wait(&s->qfull[qi], qph);
           const uint32_t b = s->tile_q[qi];
-          mbar_arrive(&s->qempty[qi]);
-          if (++qi == QDEPTH) { qi = 0; qph ^= 1u; }
+          const uint32_t kb0 = s->tile_kb0[qi];
+          const uint32_t my_q = qi;
+          mbar_arrive(&s->qempty[qi]);                     // (the slot is reused 4 tiles later:
+          if (++qi == QDEPTH) { qi = 0; qph ^= 1u; }       //  tile_kend[my_q] stays valid)
           if (b == STOP) break;
           mbar_wait(&s->tempty[acc], aph ^ 1u);            // epilogue drained this half
+          if (kb0 > 0) { mbar_wait(&s->trest[acc], rph[acc]); rph[acc] ^= 1u; }   // restored
           asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
           const uint32_t tmem = tmem0 + acc * BN;
-          for (uint32_t kb = 0; kb < nk; ++kb) {
+          uint32_t kb = kb0;
+          for (; kb < nk; ++kb) {
             mbar_wait(&s->full[st], ph);
+            if (kb >= s->tile_kend[my_q]) {                // stop marker: release it, commit
+              mbar_arrive(&s->empty[st]);
+              if (++st == STAGES) { st = 0; ph ^= 1u; }
+              break;
+            }
             asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
             const uint32_t sa = smem_u32(base + st * kStage), sb = sa + kBytesA;
 #pragma unroll
             for (uint32_t k = 0; k < BK / UMMA_K; ++k) {
               const uint64_t da = sdesc(sa + k * UMMA_K * 2), db = sdesc(sb + k * UMMA_K * 2);
-              const uint32_t accum = (kb | k) ? 1u : 0u;
+              const uint32_t accum = (kb | k) ? 1u : 0u;   // kb0 > 0: continue the restored sum
               asm volatile(
                   "{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n"
                   " tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n}\n"
@@ -309,50 +427,77 @@ struct GemmBody {
                          :: "r"(smem_u32(&s->empty[st])) : "memory");
             if (++st == STAGES) { st = 0; ph ^= 1u; }
           }
+          s->acc_kend[acc] = kb;
           asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];"
                        :: "r"(smem_u32(&s->tfull[acc])) : "memory");
+          mbar_arrive(&s->tfull[acc]);                     // publishes acc_kend (release)
           if (++acc == 2) { acc = 0; aph ^= 1u; }
         }
       }
     } else if (warp >= 4) {                                // ---- epilogue (128 threads)
       const uint32_t q = warp - 4;
+      const uint32_t rl = q * 32u + lane;                  // tile row (TMEM lane) of this thread
       uint32_t qi = 0, qph = 0, acc = 0, aph = 0;
       while (true) {
         mbar_wait(&s->qfull[qi], qph);
         const uint32_t b = s->tile_q[qi];
+        const uint32_t kb0 = s->tile_kb0[qi];
         __syncwarp();
         if (lane == 0) mbar_arrive(&s->qempty[qi]);
         if (++qi == QDEPTH) { qi = 0; qph ^= 1u; }
         if (b == STOP) break;
         int32_t tm, tn;
         tile_coords(b, gx, p_gy(g), tm, tn);
+        const uint32_t tmem = s->tmem_base + acc * BN + ((q * 32u) << 16);
+        if (kb0 > 0) {                                     // restore the spilled accumulator
+          const float4* src = spill_slot(p);               // layout [col/4][row]: coalesced
+#pragma unroll 1
+          for (uint32_t c0 = 0; c0 < BN; c0 += 32) {
+            uint32_t r[32];
+#pragma unroll
+            for (int j = 0; j < 8; ++j) {
+              const float4 v = __ldcs(src + (size_t)(c0 / 4 + j) * BM + rl);
+              r[4 * j] = __float_as_uint(v.x); r[4 * j + 1] = __float_as_uint(v.y);
+              r[4 * j + 2] = __float_as_uint(v.z); r[4 * j + 3] = __float_as_uint(v.w);
+            }
+            tmem_st32(tmem + c0, r);
+          }
+          asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+          asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+          mbar_arrive(&s->trest[acc]);
+        }
         mbar_wait(&s->tfull[acc], aph);
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-        const uint32_t tmem = s->tmem_base + acc * BN + ((q * 32u) << 16);
-        const uint32_t row = tm * BM + q * 32u + lane;
-        __nv_bfloat16* crow = g.c + (size_t)row * g.n + (size_t)tn * BN;
+        if (s->acc_kend[acc] < nk) {                       // stopped inside the tile: spill
+          float4* dst = spill_slot(p);
 #pragma unroll 1
-        for (uint32_t c0 = 0; c0 < BN; c0 += 32) {
-          uint32_t r[32];
-          asm volatile(
-              "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
-              "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
-              : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
-                "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]),
-                "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]),
-                "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
-              : "r"(tmem + c0));
-          asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
-          uint4 o[4];
-          uint32_t* ow = reinterpret_cast<uint32_t*>(o);
+          for (uint32_t c0 = 0; c0 < BN; c0 += 32) {
+            uint32_t r[32];
+            tmem_ld32(tmem + c0, r);
 #pragma unroll
-          for (int i = 0; i < 16; ++i) {
-            __nv_bfloat162 h = __floats2bfloat162_rn(__uint_as_float(r[2 * i]), __uint_as_float(r[2 * i + 1]));
-            ow[i] = *reinterpret_cast<uint32_t*>(&h);
+            for (int j = 0; j < 8; ++j)
+              __stcs(dst + (size_t)(c0 / 4 + j) * BM + rl,
+                     make_float4(__uint_as_float(r[4 * j]), __uint_as_float(r[4 * j + 1]),
+                                 __uint_as_float(r[4 * j + 2]), __uint_as_float(r[4 * j + 3])));
           }
-          uint4* dst = reinterpret_cast<uint4*>(crow + c0);
+        } else {
+          const uint32_t row = tm * BM + rl;
+          __nv_bfloat16* crow = g.c + (size_t)row * g.n + (size_t)tn * BN;
+#pragma unroll 1
+          for (uint32_t c0 = 0; c0 < BN; c0 += 32) {
+            uint32_t r[32];
+            tmem_ld32(tmem + c0, r);
+            uint4 o[4];
+            uint32_t* ow = reinterpret_cast<uint32_t*>(o);
 #pragma unroll
-          for (int i = 0; i < 4; ++i) dst[i] = o[i];
+            for (int i = 0; i < 16; ++i) {
+              __nv_bfloat162 h = __floats2bfloat162_rn(__uint_as_float(r[2 * i]), __uint_as_float(r[2 * i + 1]));
+              ow[i] = *reinterpret_cast<uint32_t*>(&h);
+            }
+            uint4* dst = reinterpret_cast<uint4*>(crow + c0);
+#pragma unroll
+            for (int i = 0; i < 4; ++i) dst[i] = o[i];
+          }
         }
         asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
         mbar_arrive(&s->tempty[acc]);

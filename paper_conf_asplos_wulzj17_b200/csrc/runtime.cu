@@ -104,6 +104,8 @@ struct Launch {
   WorkerEvent* ev = nullptr;
   uint32_t* cov = nullptr;
   size_t cov_cap = 0;
+  void* partial = nullptr;           // in-tile preemption records + spill slots (GEMM)
+  size_t partial_cap = 0;
   int slot = -1;
   HostStatus* hs = nullptr;          // host view
   HostStatus* ds = nullptr;          // device alias
@@ -151,6 +153,7 @@ struct flep_rt_s {
   HostStatus* h_slots = nullptr;
   HostStatus* d_slots = nullptr;
   std::vector<int> free_slots;
+  std::vector<std::pair<void*, size_t>> free_partial;
   size_t dmem_bytes = 0;
   uint32_t max_workers = 0;
   std::vector<void*> free_dmem;
@@ -296,6 +299,7 @@ flep_status start_epoch(flep_rt rt, Launch& L) {
   p.prefetch = (L.flags & FLEP_KFLAG_PREFETCH) ? 1u : 0u;
   p.gen_first = L.gen0 + 1;
   p.started_hint = (L.flags & FLEP_KFLAG_STARTED_HINT) ? 1u : 0u;
+  p.partial = L.partial;
   L.trig_block = kNoTrigger;
   L.trig_n = 0;
   cudaError_t e = L.ops->worker(L.args.data(), p, L.workers, L.exec, L.cov != nullptr);
@@ -354,6 +358,8 @@ void release_resources(flep_rt rt, Launch& L) {
   // of the DONE epoch left ctr/done/exited at 0, so the block is reusable as is
   if (L.dmem) { rt->cb_gen[L.dmem] = gen_of(L) + 1; rt->free_dmem.push_back(L.dmem); }
   if (L.cov) rt->free_cov.push_back({L.cov, L.cov_cap});
+  if (L.partial) rt->free_partial.push_back({L.partial, L.partial_cap});
+  L.partial = nullptr;
   if (L.slot >= 0) rt->free_slots.push_back(L.slot);
   if (L.exec && L.exec_level != -1000) rt->free_streams[L.exec_level].push_back(L.exec);
   for (cudaEvent_t e : L.evpool) rt->event_pool.push_back(e);
@@ -596,6 +602,10 @@ flep_status flep_device_info(flep_rt rt, uint32_t* num_sms, uint32_t* nsmid) {
 flep_status flep_register_kernel(flep_rt rt, const flep_kernel_desc* d, flep_kernel* out) {
   if (!rt || !d || !out) return fail(FLEP_ERR_INVALID, "NULL argument");
   if (!body_ops(d->body)) return fail(FLEP_ERR_INVALID, "unknown body %d", d->body);
+  if ((d->flags & FLEP_KFLAG_IN_TILE) && d->body != FLEP_BODY_GEMM_BF16)
+    return fail(FLEP_ERR_UNSUPPORTED, "in-tile preemption is implemented for the GEMM body only");
+  if ((d->flags & FLEP_KFLAG_IN_TILE) && (d->flags & FLEP_KFLAG_PREFETCH))
+    return fail(FLEP_ERR_UNSUPPORTED, "in-tile preemption does not combine with chunk prefetch");
   ApiLock lk(rt);
   KernelReg k;
   k.name = d->name ? d->name : "";
@@ -701,6 +711,19 @@ flep_status flep_launch(flep_rt rt, flep_kernel kid, flep_dim3 grid, const void*
       }
     }
     if (!L.cov) { L.cov_cap = std::max<size_t>(N, 4096); CUDA_TRY(cudaMalloc(&L.cov, L.cov_cap * 4)); }
+  }
+  if (L.flags & FLEP_KFLAG_IN_TILE) {
+    // per-worker partial-tile records and fp32 accumulator spill slots; no reset needed (the
+    // first epoch's workers clear their records)
+    const size_t need = partial_bytes(L.workers);
+    for (size_t i = 0; i < rt->free_partial.size(); ++i) {
+      if (rt->free_partial[i].second >= need) {
+        L.partial = rt->free_partial[i].first; L.partial_cap = rt->free_partial[i].second;
+        rt->free_partial.erase(rt->free_partial.begin() + i);
+        break;
+      }
+    }
+    if (!L.partial) { L.partial_cap = need; CUDA_TRY(cudaMalloc(&L.partial, need)); }
   }
   L.slot = rt->free_slots.back();
   rt->free_slots.pop_back();
@@ -928,11 +951,13 @@ flep_status flep_shutdown(flep_rt rt) {
     if (!L.released) {
       if (L.dmem) cudaFree(L.dmem);
       if (L.cov) cudaFree(L.cov);
+      if (L.partial) cudaFree(L.partial);
     }
   }
   for (cudaEvent_t e : rt->event_pool) cudaEventDestroy(e);
   for (void* p : rt->free_dmem) cudaFree(p);
   for (auto& c : rt->free_cov) cudaFree(c.first);
+  for (auto& c : rt->free_partial) cudaFree(c.first);
   for (cudaStream_t s : rt->all_streams) cudaStreamDestroy(s);
   if (rt->ctl) cudaStreamDestroy(rt->ctl);
   if (rt->d_rank) cudaFree(rt->d_rank);

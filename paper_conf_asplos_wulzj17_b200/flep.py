@@ -23,6 +23,7 @@ ACTION_NAMES = {0: "LAUNCH", 1: "RESUME", 2: "PREEMPT"}
 NO_TRIGGER = 0xFFFFFFFF
 KFLAG_PREFETCH = 1
 KFLAG_STARTED_HINT = 2
+KFLAG_IN_TILE = 4
 
 
 class Dim3(C.Structure):
@@ -201,8 +202,9 @@ class Runtime:
         self.close()
 
     def register_kernel(self, body, chunk=0, poll=0, name="", model=(0, 0, 0, 0, 1), overhead_ns=0,
-                        prefetch=False, ctas_per_sm=0, started_hint=False):
-        flags = (KFLAG_PREFETCH if prefetch else 0) | (KFLAG_STARTED_HINT if started_hint else 0)
+                        prefetch=False, ctas_per_sm=0, started_hint=False, in_tile=False):
+        flags = ((KFLAG_PREFETCH if prefetch else 0) | (KFLAG_STARTED_HINT if started_hint else 0)
+                 | (KFLAG_IN_TILE if in_tile else 0))
         d = KernelDesc(name.encode(), body, chunk, poll, (C.c_double * 5)(*model), overhead_ns,
                        flags, ctas_per_sm)
         k = C.c_int32()

@@ -39,7 +39,7 @@ def check_yield_events(rt, h, epoch, num_sms):
 
 
 def run_manual_schedule(rt, kernel, grid, args, n_blocks, schedule, num_sms, check_prefix=True,
-                        priority=0):
+                        priority=0, stats=None):
     """Execute one manual-mode preempt/resume schedule driven by device self-triggers.
 
     schedule = dict(cycles=[(t_star, n_sms), ...]). Returns (handle, n_preempted_epochs,
@@ -72,6 +72,8 @@ def run_manual_schedule(rt, kernel, grid, args, n_blocks, schedule, num_sms, che
             violations.append(f"unexpected state {info.state}")
             break
         preempted += 1
+        if stats is not None and info.blocks_done < min(int(info.counter), n_blocks):
+            stats["partial_epochs"] = stats.get("partial_epochs", 0) + 1   # fetched but unfinished
         if check_prefix:
             c = rt.coverage_np(h, n_blocks)
             exp = np.array(cov_oracle.expected_prefix(int(info.counter), n_blocks), dtype=np.uint32)

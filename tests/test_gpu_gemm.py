@@ -6,7 +6,7 @@ import pytest
 from oracle import workloads as W
 from synth import gen
 
-from flep_gpu_util import flep_mod
+from flep_gpu_util import flep_mod, run_manual_schedule
 
 pytestmark = pytest.mark.gpu
 
@@ -112,3 +112,64 @@ def test_gemm_full_size_sampled(rt):
     rms = float(np.sqrt(k / 9.0))       # rms of a sum of k products of U(-1,1) variables
     err = np.abs(Cn[rows, cols] - ref)
     assert np.all(err <= TOL * (np.abs(ref) + rms))
+
+
+@pytest.mark.parametrize("chunk", [1, 2])
+def test_gemm_in_tile_random_schedules_bitexact(rt, chunk):
+    """In-tile preemption: random temporal/spatial preempt/resume schedules stop
+    workers inside tiles (the accumulator is spilled and restored by the next epoch). Every
+    schedule: coverage == 1, yields only on requested SMs, drained epochs cover a counter prefix,
+    and C bit-identical to an uninterrupted run of the same binary."""
+    import torch
+    f = flep_mod()
+    m, n, k = 1024, 2048, 4096                      # 64 tiles, 64 k-steps per tile
+    ntiles = (m // 128) * (n // 256)
+    a_bits, b_bits = gen.gemm_bf16_inputs(m, n, k, seed=80 + chunk)
+    A, B = _bf16(a_bits), _bf16(b_bits)
+    kk = rt.register_kernel(f.BODY_GEMM_BF16, chunk=chunk, poll=1, ctas_per_sm=1, in_tile=True)
+    C0 = torch.empty((m, n), dtype=torch.bfloat16, device="cuda")
+    h0 = rt.launch(kk, f.gemm_grid(m, n), f.gemm_args(C0, A, B))
+    rt.sync(h0, timeout_ns=20_000_000_000)
+    _check(C0, W.gemm_bf16(a_bits, b_bits))
+    C1 = torch.empty((m, n), dtype=torch.bfloat16, device="cuda")
+    stats, bad = {}, []
+    for i in range(40):
+        s = gen.preempt_schedule(400 + i, ntiles, rt.num_sms)
+        C1.fill_(float("nan"))
+        h, npre, viol = run_manual_schedule(rt, kk, f.gemm_grid(m, n), f.gemm_args(C1, A, B), ntiles, s,
+                                            rt.num_sms, stats=stats)
+        if not np.all(rt.coverage_np(h, ntiles) == 1):
+            viol.append("I1: coverage != 1")
+        if not torch.equal(C0.view(torch.int16), C1.view(torch.int16)):
+            viol.append("C differs from the uninterrupted run")
+        if viol:
+            bad.append((i, s, viol))
+    assert not bad, bad[:3]
+    assert stats.get("partial_epochs", 0) > 5       # tiles really were stopped mid-way
+
+
+def test_gemm_in_tile_latency_below_tile_time(rt):
+    """A temporal request drains an in-tile GEMM in far less than one tile's compute time."""
+    import torch
+    f = flep_mod()
+    m = n = 4096
+    k = 8192                                        # 128 k-steps per tile
+    ntiles = (m // 128) * (n // 256)
+    a_bits, b_bits = gen.gemm_bf16_inputs(m, n, k, seed=90)
+    A, B = _bf16(a_bits), _bf16(b_bits)
+    C = torch.empty((m, n), dtype=torch.bfloat16, device="cuda")
+    out = {}
+    for in_tile in (False, True):
+        kk = rt.register_kernel(f.BODY_GEMM_BF16, chunk=1, poll=1, ctas_per_sm=1, in_tile=in_tile)
+        lat = []
+        for rep in range(3):
+            rt.arm_next_trigger(rt.num_sms + 20, rt.num_sms)    # after the static first wave
+            h = rt.launch(kk, f.gemm_grid(m, n), f.gemm_args(C, A, B))
+            rt.wait_epoch(h, timeout_ns=20_000_000_000)
+            assert rt.query(h).state == f.STATE_PREEMPTED
+            ep = rt.epoch_info(h, 1)
+            lat.append((ep.t_end - ep.t_trigger) / 1e3)
+            rt.resume(h)
+            rt.sync(h, timeout_ns=20_000_000_000)
+        out[in_tile] = float(np.median(lat))
+    assert out[True] < 0.5 * out[False], out

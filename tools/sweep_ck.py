@@ -21,6 +21,7 @@ def main():
     ap.add_argument("--polls", default="1")
     ap.add_argument("--cps", default="0")
     ap.add_argument("--prefetch", default="0,1")
+    ap.add_argument("--in-tile", default="0", help="GEMM: in-tile preemption variants (0,1)")
     ap.add_argument("--gate-us", type=float, default=0.0,
                     help="spin the stream this long before the start event (hides host submission latency)")
     a = ap.parse_args()
@@ -96,9 +97,13 @@ def main():
             for K in map(int, a.polls.split(",")):
                 for pf in map(int, a.prefetch.split(",")):
                     for cps in map(int, a.cps.split(",")):
-                        k = rt.register_kernel(body, chunk=C, poll=K, prefetch=bool(pf), ctas_per_sm=cps)
+                      for it_ in (map(int, a.in_tile.split(",")) if name == "gemm" else [0]):
+                        if it_ and pf:
+                            continue
+                        k = rt.register_kernel(body, chunk=C, poll=K, prefetch=bool(pf), ctas_per_sm=cps,
+                                               in_tile=bool(it_))
                         tw = timed(lambda: rt.launch(k, grid, args, stream=s))
-                        print(json.dumps({"body": name, "C": C, "K": K, "prefetch": pf, "cps": cps,
+                        print(json.dumps({"body": name, "C": C, "K": K, "prefetch": pf, "cps": cps, "in_tile": it_,
                                           "us": round(tw, 3),
                                           ("tflops" if name == "gemm" else "gbs"): round(nbytes / tw / (1e6 if name == "gemm" else 1e3), 1),
                                           "overhead_pct": round((tw / tu - 1) * 100, 2)}), flush=True)
