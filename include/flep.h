@@ -136,7 +136,7 @@ typedef struct {
    grid's completion by about a microsecond. */
 #define FLEP_KFLAG_STARTED_HINT 2u
 /* In-tile preemption (GEMM body only; not with FLEP_KFLAG_PREFETCH): workers also poll inside a
-   tile (every 8 k-steps) and, when asked to leave, spill the fp32 accumulator of the tile in
+   tile (every 4 k-steps) and, when asked to leave, spill the fp32 accumulator of the tile in
    progress to a per-worker slot; the next epoch's worker with the same index restores it and
    continues the k-loop. The result stays bit-identical to an uninterrupted run. Costs
    W x (16 B + 128 KiB) of device memory per launch (runtime-owned, pooled).

@@ -35,7 +35,7 @@
 #define FLEP_GEMM_GROUP 16
 #endif
 #ifndef FLEP_GEMM_KPOLL
-#define FLEP_GEMM_KPOLL 8         // k-steps (BK = 64 each) between in-tile polls
+#define FLEP_GEMM_KPOLL 4         // k-steps (BK = 64 each) between in-tile polls (sweep: 2 -> 7.4 us drain, +0.4 %; 4 -> 8.7 us, +0.1 %; 8 -> 11.9 us, +0.5 %)
 #endif
 
 namespace flep {
