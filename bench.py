@@ -206,7 +206,7 @@ def run_temporal(args, rank, world, local):
     # the waiting (high-priority) kernel is never preempted here: its chunking is tuned for
     # throughput (C = 2 with prefetch), the victim's for latency (C = K = 1)
     kHP = rt.register_kernel(F.BODY_STENCIL5_F32, chunk=args.hp_chunk, poll=1, name="stencil",
-                             prefetch=bool(args.hp_prefetch))
+                             prefetch=bool(args.hp_prefetch), async_poll=bool(args.hp_async))
     lp_args = F.spmv_args(wl.d_y, wl.d_rowptr, wl.d_col, wl.d_val, wl.d_x)
     hp_args = F.stencil_args(wl.d_out, wl.d_in)
     lp_grid, hp_grid = F.spmv_grid(SPMV_ROWS), F.stencil_grid(STENCIL_N)
@@ -312,6 +312,7 @@ def run_temporal(args, rank, world, local):
         "config": {"workload": "configs[1]: full-GPU temporal preemption of SpMV-CSR fp32 (2^20 rows, "
                                f"{wl.nnz} nnz, low priority) by stencil5 fp32 4096^2 (high priority)",
                    "lp_chunk": args.lp_chunk, "lp_poll": args.lp_poll, "hp_chunk": args.hp_chunk, "hp_poll": 1, "hp_prefetch": bool(args.hp_prefetch),
+                   "hp_async_poll": bool(args.hp_async),
                    "prefetch": bool(args.prefetch),
                    "flag": "stream_memop (device self-trigger for the request)",
                    "l2": "flushed between steps (write of 2x L2 bytes)", "parallelism": f"replicas x{world}"},
@@ -411,7 +412,7 @@ def run_e2e(F, torch, wl, local, steps, args):
     kLP = rt.register_kernel(F.BODY_SPMV_CSR_F32, chunk=args.lp_chunk, poll=args.lp_poll, name="spmv",
                              model=(0, 0, 0, 0, 70_000), prefetch=bool(args.prefetch), started_hint=True)
     kHP = rt.register_kernel(F.BODY_STENCIL5_F32, chunk=args.hp_chunk, poll=1, name="stencil",
-                             model=(0, 0, 0, 0, 30_000), prefetch=bool(args.hp_prefetch))
+                             model=(0, 0, 0, 0, 30_000), prefetch=bool(args.hp_prefetch), async_poll=bool(args.hp_async))
     pin = lambda a: torch.from_numpy(np.ascontiguousarray(a)).pin_memory()  # noqa: E731
     h_rp, h_col, h_val, h_x, h_in = pin(wl.rowptr), pin(wl.col), pin(wl.val), pin(wl.x), pin(wl.st_in)
     h_y = torch.empty(SPMV_ROWS, dtype=torch.float32).pin_memory()
@@ -535,6 +536,7 @@ def main():
     ap.add_argument("--prefetch", type=int, default=0)
     ap.add_argument("--hp-chunk", type=int, default=2)
     ap.add_argument("--hp-prefetch", type=int, default=1)
+    ap.add_argument("--hp-async", type=int, default=1, help="waiting kernel: async poll (R22)")
     ap.add_argument("--lp-poll", type=int, default=1)
     ap.add_argument("--reps", type=int, default=20)
     ap.add_argument("--e2e-steps", type=int, default=10)

@@ -142,6 +142,11 @@ typedef struct {
    W x (16 B + 128 KiB) of device memory per launch (runtime-owned, pooled).
    flep_register_kernel returns FLEP_ERR_UNSUPPORTED for other bodies or with prefetch. */
 #define FLEP_KFLAG_IN_TILE 4u
+/* Asynchronous poll: the control word a worker tests at a poll point was loaded at its previous
+   scheduling step, so no L2 round trip sits between two chunks; a request is acted on up to one
+   chunk later. For throughput-oriented kernels (with FLEP_KFLAG_PREFETCH the scheduling step then
+   waits on nothing). */
+#define FLEP_KFLAG_ASYNC_POLL 8u
 
 typedef enum {
   FLEP_STATE_QUEUED = 0,     /* intercepted, waiting for a scheduling decision (S2) */
@@ -252,6 +257,11 @@ flep_status flep_debug_copy_events(flep_rt rt, flep_launch_t h, uint32_t epoch,
                                    size_t* n_out);
 flep_status flep_debug_epoch_info(flep_rt rt, flep_launch_t h, uint32_t epoch,
                                   flep_epoch_info* out);
+/* Diagnostics builds (-DFLEP_TRACE) only, else FLEP_ERR_UNSUPPORTED: record per-chunk scheduling
+   timestamps of worker grids (device buffer [W][64][2] u64: tid 0 reaches the scheduling step,
+   the step returns) and entry/exit of every block of unwrapped grids ([N][2] u64). Buffers are
+   the caller's; NULL disables. */
+flep_status flep_debug_set_trace(flep_rt rt, void* worker_trace, void* unwrapped_trace);
 /* Set the spatial rank table: rank[smid] for smid < nsmid (default rank = smid). */
 flep_status flep_set_rank_table(flep_rt rt, const uint16_t* rank, uint32_t n);
 /* Host steady-clock now, ns (the clock all host timestamps use). */

@@ -81,11 +81,19 @@ struct WorkerParams {
   uint32_t prefetch;       // 1: fetch chunk j+1 while chunk j runs (hides the atomic's latency;
                            //    a stopping worker still processes the prefetched chunk)
   uint32_t gen_first;      // generation of this launch's first epoch
+  uint32_t async_poll;     // 1: the poll uses the control word copied one step earlier (R22);
+                           //    device-memory control word only (16-B aligned line)
   uint32_t started_hint;   // 1: worker 0 publishes "epoch started" to the host slot at entry (a
                            //    system-scope store: the kernel's completion then waits for it)
   void* partial;           // in-tile preemption (FLEP_KFLAG_IN_TILE, GEMM): W partial-tile records
                            // then W accumulator spill slots (layout: partial_bytes below), or nullptr
+#ifdef FLEP_TRACE
+  uint64_t* trace;         // diagnostics build only: [W][kTraceChunks][2] (see flep_worker)
+#endif
 };
+#ifdef FLEP_TRACE
+constexpr uint32_t kTraceChunks = 64;
+#endif
 
 // In-tile preemption state: record i belongs to worker i of every epoch of a launch.
 struct PartialTile {
@@ -149,10 +157,24 @@ __device__ __forceinline__ bool should_yield(uint32_t c, const WorkerParams& p, 
 
 // Worker bookkeeping shared by every loop shape (kept in shared memory, written by the one
 // scheduling thread).
-struct WorkerShared {
+struct alignas(16) WorkerShared {
+  uint32_t poll_buf[4];    // async poll: the control word's 16-B line, copied by cp.async.cg
   uint64_t t_entry;
   uint32_t sm, blocks, reason;
 };
+
+// Async poll (R22): copy the control word's 16 B from L2 (cp.async.cg bypasses L1, so it never
+// returns a stale line) into shared memory without a register destination: nothing waits for
+// it until the next scheduling step, and no register stays live across the body.
+__device__ __forceinline__ void poll_issue(WorkerShared& ws, const uint32_t* ctrl) {
+  const uint32_t dst = static_cast<uint32_t>(__cvta_generic_to_shared(ws.poll_buf));
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n cp.async.commit_group;"
+               :: "r"(dst), "l"(ctrl) : "memory");
+}
+__device__ __forceinline__ uint32_t poll_consume(const WorkerShared& ws) {
+  asm volatile("cp.async.wait_all;" ::: "memory");
+  return *reinterpret_cast<const volatile uint32_t*>(ws.poll_buf);
+}
 
 // The scheduling step of Fig. 4 (b)/(c), executed by ONE thread of the worker: the amortised
 // poll every K chunks, then the task fetch (pull_task) — or the chunk fetched
@@ -162,16 +184,33 @@ struct WorkerShared {
 // self-trigger of the test/bench hooks.
 struct SchedState {
   uint32_t k = 0;                    // chunk index within the current poll period
-  uint32_t held = 0xffffffffu;       // prefetched chunk base not yet handed out
+  uint32_t held = 0xffffffffu;       // prefetched counter value not yet handed out (raw: the
+                                     // first-epoch offset is added when it is consumed, so the
+                                     // atomic's round trip overlaps the body)
+  bool have_seen = false;            // async poll: a copy of the control word is in flight
   bool stopping = false;             // a request named this SM; drain the held chunk
   bool first = true;                 // first step of this worker
 };
 
 // pull_task. In the first epoch of a launch the counter hands out blocks after the W
 // static first chunks (reading R20), so the effective counter there is ctr + W*C.
+__device__ __forceinline__ uint32_t ctr_offset(const WorkerParams& p) {
+  return p.epoch == p.gen_first ? p.workers * p.chunk : 0u;
+}
+// The counter atomic as plain PTX: atomicAdd() lets nvcc emit a warp-aggregated sequence whose
+// SHFL consumes the result at once, which would make a prefetching thread wait for the whole L2
+// round trip right there; with atom.add the wait happens only where the value is used.
+__device__ __forceinline__ uint32_t atom_add_ctr(uint32_t* ctr, uint32_t v) {
+  uint32_t old;
+  // an opaque zero offset (ptxas cannot prove the address warp-uniform, so it emits no
+  // aggregation sequence around the atomic)
+  uint64_t z;
+  asm volatile("mov.u64 %0, 0;" : "=l"(z));
+  asm volatile("atom.relaxed.gpu.global.add.u32 %0, [%1], %2;" : "=r"(old) : "l"(ctr + z), "r"(v) : "memory");
+  return old;
+}
 __device__ __forceinline__ uint32_t fetch_chunk(const WorkerParams& p) {
-  const uint32_t s = atomicAdd(&p.cb->ctr, p.chunk);
-  return p.epoch == p.gen_first ? s + p.workers * p.chunk : s;
+  return atom_add_ctr(&p.cb->ctr, p.chunk) + ctr_offset(p);
 }
 
 __device__ __forceinline__ uint32_t next_chunk(const WorkerParams& p, SchedState& st, WorkerShared& ws) {
@@ -195,12 +234,14 @@ __device__ __forceinline__ uint32_t next_chunk(const WorkerParams& p, SchedState
       if (should_yield(c, p, smid_reg())) { ws.reason = kReasonYield; return 0xffffffffu; }
     }
   } else if (st.k == 0 && !st.stopping) {            // amortised poll (Fig. 4(b))
-    const uint32_t c = ld_relaxed_gpu(p.ctrl);
+    // async poll (FLEP_KFLAG_ASYNC_POLL, reading R22): use the word loaded at the previous step,
+    // so no round trip sits between two chunks; a request is then acted on one chunk later
+    const uint32_t c = (p.async_poll && st.have_seen) ? poll_consume(ws) : ld_relaxed_gpu(p.ctrl);
     if (should_yield(c, p, smid_reg())) { st.stopping = true; ws.reason = kReasonYield; }
   }
   if (!have) {
     if (st.held != 0xffffffffu) {                    // a fetched chunk is always processed (A4)
-      base = st.held;
+      base = st.held + ctr_offset(p);
       st.held = 0xffffffffu;
     } else if (!st.stopping) {
       base = fetch_chunk(p);
@@ -209,7 +250,7 @@ __device__ __forceinline__ uint32_t next_chunk(const WorkerParams& p, SchedState
   if (base != 0xffffffffu && base >= p.n_blocks) { base = 0xffffffffu; ws.reason = kReasonExhausted; }
   if (base != 0xffffffffu) {
     ws.blocks += min(p.chunk, p.n_blocks - base);
-    if (p.prefetch && !st.stopping) st.held = fetch_chunk(p);   // overlaps the body
+    if (p.prefetch && !st.stopping) st.held = atom_add_ctr(&p.cb->ctr, p.chunk);   // overlaps the body
     if (p.trigger_block - base < p.chunk) {          // device self-trigger inside this chunk
       const uint32_t e = p.epoch % kEvEpochs;
       p.cb->ep_t_trigger[e] = gtimer();
@@ -217,6 +258,10 @@ __device__ __forceinline__ uint32_t next_chunk(const WorkerParams& p, SchedState
       atomicExch(p.ctrl, ((p.epoch & 0xffffu) << 16) | (p.trigger_n & 0xffffu));
     }
     if (++st.k == p.poll) st.k = 0;
+    if (p.async_poll && st.k == 0 && !st.stopping) {  // the next step polls: load it now
+      poll_issue(ws, p.ctrl);
+      st.have_seen = true;
+    }
   }
   return base;
 }
@@ -249,8 +294,23 @@ flep_worker(const __grid_constant__ typename Body::Args args, const WorkerParams
   } else {
     SchedState st;
     uint32_t parity = 0;
+#ifdef FLEP_TRACE
+    uint32_t nchunk = 0;
+#endif
     while (true) {
+#ifdef FLEP_TRACE
+      // diagnostics: per chunk, when tid 0 reached the scheduling step (its share of the previous
+      // body done) and when the step returned (poll + fetch latency)
+      const uint64_t ta = (tid == 0 && p.trace) ? gtimer() : 0;
       if (tid == 0) s_slot[parity] = next_chunk(p, st, ws);
+      if (tid == 0 && p.trace && nchunk < kTraceChunks) {
+        uint64_t* t = p.trace + ((size_t)blockIdx.x * kTraceChunks + nchunk) * 2;
+        t[0] = ta; t[1] = gtimer();
+      }
+      ++nchunk;
+#else
+      if (tid == 0) s_slot[parity] = next_chunk(p, st, ws);
+#endif
       __syncthreads();
       const uint32_t b0 = s_slot[parity];
       parity ^= 1u;
@@ -303,13 +363,25 @@ flep_worker(const __grid_constant__ typename Body::Args args, const WorkerParams
 }
 
 // The original kernel (unwrapped twin, K7): one CTA per original block, same body.
+#ifdef FLEP_TRACE
+static __device__ uint64_t* g_unwrapped_trace;   // diagnostics build only: [N][2] entry/exit
+#endif
 template <class Body>
 __global__ void __launch_bounds__(Body::kThreads, Body::kMinBlocks)
 flep_unwrapped(const __grid_constant__ typename Body::Args args, uint32_t gx, uint32_t gy, uint32_t block_offset) {
   const uint32_t b = block_offset + blockIdx.x + gx * (blockIdx.y + gy * blockIdx.z);
+#ifdef FLEP_TRACE
+  const uint64_t t0 = gtimer();
+#endif
   Body::setup(args);
   Body::run(args, b, b + 1, gx, gy);
   Body::teardown(args);
+#ifdef FLEP_TRACE
+  if (g_unwrapped_trace) {
+    __syncthreads();
+    if (threadIdx.x == 0) { g_unwrapped_trace[2 * (size_t)b] = t0; g_unwrapped_trace[2 * (size_t)b + 1] = gtimer(); }
+  }
+#endif
 }
 
 // Bodies without per-worker resources, run through the generic per-chunk loop.

@@ -108,6 +108,12 @@ const BodyOps kOps[] = {
 
 }  // namespace
 
+#ifdef FLEP_TRACE
+cudaError_t set_unwrapped_trace(uint64_t* p) {
+  return cudaMemcpyToSymbol(g_unwrapped_trace, &p, sizeof(p));
+}
+#endif
+
 const BodyOps* body_ops(int32_t body) {
   if (body < 1 || body > FLEP_BODY_GEMM_BF16) return nullptr;
   return &kOps[body];

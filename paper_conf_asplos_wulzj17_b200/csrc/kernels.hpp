@@ -23,6 +23,9 @@ struct BodyOps {
 };
 
 const BodyOps* body_ops(int32_t body);
+#ifdef FLEP_TRACE
+cudaError_t set_unwrapped_trace(uint64_t* p);
+#endif
 
 template <class Body>
 cudaError_t launch_worker_raw(const typename Body::Args& a, const WorkerParams& p, uint32_t W, cudaStream_t s, bool cov);

@@ -154,6 +154,7 @@ struct flep_rt_s {
   HostStatus* d_slots = nullptr;
   std::vector<int> free_slots;
   std::vector<std::pair<void*, size_t>> free_partial;
+  uint64_t* trace = nullptr;        // FLEP_TRACE diagnostics builds: worker chunk trace buffer
   size_t dmem_bytes = 0;
   uint32_t max_workers = 0;
   std::vector<void*> free_dmem;
@@ -299,7 +300,11 @@ flep_status start_epoch(flep_rt rt, Launch& L) {
   p.prefetch = (L.flags & FLEP_KFLAG_PREFETCH) ? 1u : 0u;
   p.gen_first = L.gen0 + 1;
   p.started_hint = (L.flags & FLEP_KFLAG_STARTED_HINT) ? 1u : 0u;
+  p.async_poll = ((L.flags & FLEP_KFLAG_ASYNC_POLL) && rt->opt.flag != FLEP_FLAG_HOST_MAPPED) ? 1u : 0u;
   p.partial = L.partial;
+#ifdef FLEP_TRACE
+  p.trace = rt->trace;
+#endif
   L.trig_block = kNoTrigger;
   L.trig_n = 0;
   cudaError_t e = L.ops->worker(L.args.data(), p, L.workers, L.exec, L.cov != nullptr);
@@ -1164,6 +1169,19 @@ int64_t flep_model_predict_ns(const double m[5], double grid, double cta, double
   int64_t r = (int64_t)(a + 0.5);
   if (v < 0) r = -r;
   return r < 1 ? 1 : r;
+}
+
+flep_status flep_debug_set_trace(flep_rt rt, void* worker_trace, void* unwrapped_trace) {
+  if (!rt) return fail(FLEP_ERR_INVALID, "rt is NULL");
+#ifdef FLEP_TRACE
+  ApiLock lk(rt);
+  rt->trace = (uint64_t*)worker_trace;
+  CUDA_TRY(flep::set_unwrapped_trace((uint64_t*)unwrapped_trace));
+  return FLEP_OK;
+#else
+  (void)worker_trace; (void)unwrapped_trace;
+  return fail(FLEP_ERR_UNSUPPORTED, "built without FLEP_TRACE");
+#endif
 }
 
 }  // extern "C"

@@ -24,6 +24,7 @@ NO_TRIGGER = 0xFFFFFFFF
 KFLAG_PREFETCH = 1
 KFLAG_STARTED_HINT = 2
 KFLAG_IN_TILE = 4
+KFLAG_ASYNC_POLL = 8
 
 
 class Dim3(C.Structure):
@@ -111,6 +112,7 @@ _SIG = {
     "flep_debug_copy_events": (C.c_int, [_P, C.c_int64, C.c_uint32, C.POINTER(WorkerEvent), C.c_size_t,
                                          C.POINTER(C.c_size_t)]),
     "flep_debug_epoch_info": (C.c_int, [_P, C.c_int64, C.c_uint32, C.POINTER(EpochInfo)]),
+    "flep_debug_set_trace": (C.c_int, [_P, C.c_void_p, C.c_void_p]),
     "flep_set_rank_table": (C.c_int, [_P, C.POINTER(C.c_uint16), C.c_uint32]),
     "flep_now_ns": (C.c_int64, []),
     "flep_decision_log": (C.c_int, [_P, C.POINTER(C.c_int64), C.c_size_t, C.POINTER(C.c_size_t)]),
@@ -202,9 +204,9 @@ class Runtime:
         self.close()
 
     def register_kernel(self, body, chunk=0, poll=0, name="", model=(0, 0, 0, 0, 1), overhead_ns=0,
-                        prefetch=False, ctas_per_sm=0, started_hint=False, in_tile=False):
+                        prefetch=False, ctas_per_sm=0, started_hint=False, in_tile=False, async_poll=False):
         flags = ((KFLAG_PREFETCH if prefetch else 0) | (KFLAG_STARTED_HINT if started_hint else 0)
-                 | (KFLAG_IN_TILE if in_tile else 0))
+                 | (KFLAG_IN_TILE if in_tile else 0) | (KFLAG_ASYNC_POLL if async_poll else 0))
         d = KernelDesc(name.encode(), body, chunk, poll, (C.c_double * 5)(*model), overhead_ns,
                        flags, ctas_per_sm)
         k = C.c_int32()
@@ -283,6 +285,12 @@ class Runtime:
         e = EpochInfo()
         check(self.L.flep_debug_epoch_info(self.h, launch, epoch, C.byref(e)), "flep_debug_epoch_info")
         return e
+
+    def set_trace(self, worker_trace=None, unwrapped_trace=None):
+        """Diagnostics builds (-DFLEP_TRACE) only: device buffers (torch tensors) for the chunk /
+        block timestamp traces, or None."""
+        ptr = lambda t: None if t is None else C.c_void_p(t.data_ptr())  # noqa: E731
+        check(self.L.flep_debug_set_trace(self.h, ptr(worker_trace), ptr(unwrapped_trace)), "flep_debug_set_trace")
 
     def set_rank_table(self, rank):
         arr = (C.c_uint16 * len(rank))(*rank)

@@ -126,7 +126,8 @@ def test_gemm_in_tile_random_schedules_bitexact(rt, chunk):
     ntiles = (m // 128) * (n // 256)
     a_bits, b_bits = gen.gemm_bf16_inputs(m, n, k, seed=80 + chunk)
     A, B = _bf16(a_bits), _bf16(b_bits)
-    kk = rt.register_kernel(f.BODY_GEMM_BF16, chunk=chunk, poll=1, ctas_per_sm=1, in_tile=True)
+    kk = rt.register_kernel(f.BODY_GEMM_BF16, chunk=chunk, poll=1, ctas_per_sm=1, in_tile=True,
+                            async_poll=chunk == 2)
     C0 = torch.empty((m, n), dtype=torch.bfloat16, device="cuda")
     h0 = rt.launch(kk, f.gemm_grid(m, n), f.gemm_args(C0, A, B))
     rt.sync(h0, timeout_ns=20_000_000_000)

@@ -92,7 +92,8 @@ def test_managed_queue_replay_parity(kind):
 
 def test_random_schedules_10k_zero_violations():
     """Config 1: LP SAXPY-int32 2^20 under 10^4 random manual preempt/resume schedules (temporal
-    and spatial yields, C in {1,2,4,8,16}, K in {1,2,4,8}, with and without prefetch). Every
+    and spatial yields, C in {1,2,4,8,16}, K in {1,2,4,8}, with and without prefetch and async
+    poll). Every
     schedule: coverage == 1, bit-exact y, preempted epochs cover a prefix (I2), yields only on
     requested SMs (I3)."""
     f = flep_mod()
@@ -110,11 +111,12 @@ def test_random_schedules_10k_zero_violations():
         for i in range(n_sched):
             s = gen.preempt_schedule(100 + i, nb, rt.num_sms)
             pf = i % 2 == 1
+            ap = (i // 2) % 2 == 1                 # async poll (R22)
             cps = (1, 2, 8)[i % 3]                 # resident workers per SM (W = 148 * cps)
-            key = (s["C"], s["K"], pf, cps)
+            key = (s["C"], s["K"], pf, cps, ap)
             if key not in kern:
                 kern[key] = rt.register_kernel(f.BODY_SAXPY_I32, chunk=s["C"], poll=s["K"], prefetch=pf,
-                                               ctas_per_sm=cps)
+                                               ctas_per_sm=cps, async_poll=ap)
             yd.copy_(y0)
             h, npre, viol = run_manual_schedule(rt, kern[key], f.saxpy_grid(n), f.saxpy_i32_args(yd, xd, a), nb,
                                                 s, rt.num_sms, check_prefix=(i % 10 == 0))

@@ -202,3 +202,43 @@ def test_hand_traced_static_first_preempt():
             break
         st = succ[0][1]
     assert st[6] == cv.ST_DONE and st[4] == (1, 1, 1, 1, 1)
+
+
+# ---- async poll (R22): the poll tests the word copied when the previous chunk was taken
+
+@pytest.mark.parametrize("C,K,pf,sf", [(1, 1, False, False), (2, 1, False, True), (1, 2, False, True),
+                                       (1, 1, True, True), (2, 1, True, False)])
+def test_exhaustive_async_poll_no_violations(C, K, pf, sf):
+    ws = (0, 1) if pf else (0, 0, 1)
+    n = len(ws) * C * (K + pf) + 1 if sf else 4 + C
+    r = cv.explore(_cfg(n_blocks=n, chunk=C, poll=K, worker_sm=ws, prefetch=pf, static_first=sf,
+                        async_poll=True))
+    assert r.violations == set()
+    assert r.preempted_epoch_ends > 0
+
+
+def test_async_poll_refill_and_clear():
+    r = cv.explore(_cfg(n_blocks=5, chunk=1, poll=1, worker_sm=(0, 0, 1), preempt_widths=(1,),
+                        max_events=2, allow_refill=True, static_first=True, async_poll=True))
+    assert r.violations == set()
+    r = cv.explore(_cfg(n_blocks=6, chunk=2, poll=2, allow_clear=True, async_poll=True))
+    assert r.violations == set()
+
+
+def test_hand_traced_async_poll_acts_one_chunk_later():
+    # one worker, N=4, C=K=1: the request lands after the worker took block 0, so the copy taken
+    # with block 0 misses it: the worker still fetches block 1 and leaves at the poll after it
+    # (a synchronous poll would have left before block 1)
+    cfg = cv.Config(n_blocks=4, chunk=1, poll=1, worker_sm=(0,), num_sms=2, preempt_widths=(2,),
+                    max_events=1, async_poll=True)
+    st = cv.initial_state(cfg)
+    for lab in ["w0.poll", "w0.fetch", "preempt(2)", "w0.proc", "w0.poll", "w0.fetch", "w0.proc",
+                "w0.poll", "w0.exit"]:
+        st = dict(cv.successors(cfg, st))[lab]
+    assert st[6] == cv.ST_PREEMPTED and st[4] == (1, 1, 0, 0) and st[0] == 2
+    sync = cv.Config(n_blocks=4, chunk=1, poll=1, worker_sm=(0,), num_sms=2, preempt_widths=(2,),
+                     max_events=1)
+    st = cv.initial_state(sync)
+    for lab in ["w0.poll", "w0.fetch", "preempt(2)", "w0.proc", "w0.poll", "w0.exit"]:
+        st = dict(cv.successors(sync, st))[lab]
+    assert st[6] == cv.ST_PREEMPTED and st[4] == (1, 0, 0, 0)

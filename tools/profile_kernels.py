@@ -53,9 +53,10 @@ def main():
         Cg = torch.empty(M, M, device="cuda", dtype=torch.bfloat16)
         jobs.append(("gemm", F.BODY_GEMM_BF16, F.gemm_grid(M, M), F.gemm_args(Cg, A, B), (A, B, Cg)))
     s = torch.cuda.current_stream()
-    combos = [tuple(map(int, c.split(":"))) for c in a.combos.split(",")] if a.combos else [(a.chunk, a.poll, a.prefetch)]
+    combos = [(tuple(map(int, c.split(":"))) + (0,))[:4] for c in a.combos.split(",")] if a.combos else [(a.chunk, a.poll, a.prefetch)]
     for name, body, grid, args, keep in jobs:
-        ks = [rt.register_kernel(body, chunk=C, poll=K, prefetch=bool(pf)) for C, K, pf in combos]
+        ks = [rt.register_kernel(body, chunk=C, poll=K, prefetch=bool(pf), async_poll=bool(ap))
+              for C, K, pf, ap in combos]
         for _ in range(a.reps):
             flush.zero_()
             rt.launch_unwrapped(body, grid, args, stream=s)

@@ -22,6 +22,7 @@ def main():
     ap.add_argument("--cps", default="0")
     ap.add_argument("--prefetch", default="0,1")
     ap.add_argument("--in-tile", default="0", help="GEMM: in-tile preemption variants (0,1)")
+    ap.add_argument("--async-poll", default="0", help="async poll variants (0,1)")
     ap.add_argument("--gate-us", type=float, default=0.0,
                     help="spin the stream this long before the start event (hides host submission latency)")
     a = ap.parse_args()
@@ -98,12 +99,14 @@ def main():
                 for pf in map(int, a.prefetch.split(",")):
                     for cps in map(int, a.cps.split(",")):
                       for it_ in (map(int, a.in_tile.split(",")) if name == "gemm" else [0]):
+                       for ap_ in map(int, a.async_poll.split(",")):
                         if it_ and pf:
                             continue
                         k = rt.register_kernel(body, chunk=C, poll=K, prefetch=bool(pf), ctas_per_sm=cps,
-                                               in_tile=bool(it_))
+                                               in_tile=bool(it_), async_poll=bool(ap_))
                         tw = timed(lambda: rt.launch(k, grid, args, stream=s))
                         print(json.dumps({"body": name, "C": C, "K": K, "prefetch": pf, "cps": cps, "in_tile": it_,
+                                          "async_poll": ap_,
                                           "us": round(tw, 3),
                                           ("tflops" if name == "gemm" else "gbs"): round(nbytes / tw / (1e6 if name == "gemm" else 1e3), 1),
                                           "overhead_pct": round((tw / tu - 1) * 100, 2)}), flush=True)

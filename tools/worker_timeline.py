@@ -10,7 +10,7 @@ sys.path.insert(0, ROOT)
 from synth import gen  # noqa: E402
 
 
-COMBOS = [tuple(map(int, c.split(":"))) for c in
+COMBOS = [(tuple(map(int, c.split(":"))) + (0,))[:4] for c in
           (sys.argv[1] if len(sys.argv) > 1 else "1:1:0,2:1:1").split(",")]   # C:K:prefetch
 
 
@@ -48,8 +48,8 @@ def main():
         a = rt.events(h0, 1)[0]
         b = rt.events(h1, 1)[0]
         print(json.dumps({"body": name, "variant": "unwrapped", "stamp_gap_us": round((b.t_entry - a.t_exit) / 1e3, 2)}))
-        for C, K, pf in COMBOS:
-            k = rt.register_kernel(body, chunk=C, poll=K, prefetch=bool(pf))
+        for C, K, pf, ap in COMBOS:
+            k = rt.register_kernel(body, chunk=C, poll=K, prefetch=bool(pf), async_poll=bool(ap))
             for rep in range(3):
                 flush.zero_()
                 h0 = stamp()
@@ -67,7 +67,7 @@ def main():
             entry = np.array([e.t_entry - t0 for e in ev]) / 1e3
             exit_ = np.array([e.t_exit - t0 for e in ev]) / 1e3
             nb = np.array([e.n_blocks for e in ev])
-            print(json.dumps({"body": name, "C": C, "K": K, "prefetch": pf, "event_us": round(e0.elapsed_time(e1) * 1e3, 2),
+            print(json.dumps({"body": name, "C": C, "K": K, "prefetch": pf, "async_poll": ap, "event_us": round(e0.elapsed_time(e1) * 1e3, 2),
                               "stamp_gap_us": round((sb.t_entry - sa.t_exit) / 1e3, 2),
                               "gap_before_us": round((t0 - sa.t_exit) / 1e3, 2),
                               "gap_after_us": round((sb.t_entry - max(e.t_exit for e in ev)) / 1e3, 2),
