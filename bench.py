@@ -524,7 +524,7 @@ def main():
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--impl", default="flep", choices=["flep", "reference"])
-    ap.add_argument("--config", default="temporal", choices=["temporal", "corun1", "spatial", "queue", "ffs", "model", "gemm"])
+    ap.add_argument("--config", default="temporal", choices=["temporal", "corun1", "spatial", "queue", "ffs", "model", "gemm", "tune"])
     ap.add_argument("--model-train", type=int, default=100)
     ap.add_argument("--model-test", type=int, default=30)
     ap.add_argument("--overhead-runs", type=int, default=50)
@@ -540,6 +540,7 @@ def main():
     ap.add_argument("--lp-poll", type=int, default=1)
     ap.add_argument("--reps", type=int, default=20)
     ap.add_argument("--e2e-steps", type=int, default=10)
+    ap.add_argument("--tune-bound", type=float, default=0.04, help="config tune: overhead bound (P:166: 4 %%)")
     ap.add_argument("--gemm-in-tile", type=int, default=1, help="config gemm: in-tile preemption (1) or tile granularity (0)")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
@@ -567,6 +568,8 @@ def main():
             bench_configs.run_corun1(args, rank, world, local)
         elif args.config == "gemm":
             bench_configs.run_gemm_preempt(args, rank, world, local)
+        elif args.config == "tune":
+            bench_configs.run_tune(args, rank, world, local)
         elif args.config == "ffs":
             bench_configs.run_ffs(args, rank, world, local)
         elif args.config == "model":

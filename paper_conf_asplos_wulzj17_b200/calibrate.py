@@ -179,3 +179,79 @@ def preemption_overhead(torch, wl, body, size, runs=50, chunk=1, prefetch=False,
         return int(max(0.0, float(np.mean(over)))) if over else 0, t_alone
     finally:
         rt.close()
+
+
+# ---- amortizing factor ------------------------------------------------------------------
+# "FLEP can automatically find the smallest value for L through offline tuning (trying different
+# values from small to large) such that the runtime overhead introduced by the transformation is
+# less than 4%." On B200 L = C*K (reading R2): C blocks per counter fetch, a poll every K chunks.
+# For one L several variants exist (C vs K split, prefetch, async poll); the tuner tries them from
+# the latency-cheapest (no prefetch, synchronous poll) to the throughput-cheapest.
+
+DEFAULT_CANDIDATES = tuple(
+    (c, k, pf, ap)
+    for c, k in ((1, 1), (2, 1), (1, 2), (4, 1), (2, 2), (1, 4), (8, 1), (4, 2), (16, 1), (8, 2), (32, 1),
+                 (16, 2), (64, 1), (32, 4), (200, 1))
+    for pf, ap in ((False, False), (True, False), (True, True)))
+
+
+def select_amortizing_factor(table, bound=0.04):
+    """table: iterable of dicts {C, K, prefetch, async_poll, overhead} (overhead as a fraction of
+    the unwrapped time). Returns the entry with the smallest L = C*K whose overhead is below
+    `bound` (within one L: no prefetch before prefetch, synchronous before async poll — the order
+    of added preemption latency — then the lowest overhead), with met=True; if no entry meets the
+    bound, the entry with the lowest overhead, met=False."""
+    rows = list(table)
+    if not rows:
+        raise ValueError("empty tuning table")
+
+    def key(r):
+        return (r["C"] * r["K"], bool(r["prefetch"]) + bool(r["async_poll"]), r["overhead"])
+    ok = [r for r in rows if r["overhead"] < bound]
+    if ok:
+        best = min(ok, key=key)
+        return dict(best, L=best["C"] * best["K"], met=True)
+    best = min(rows, key=lambda r: (r["overhead"], r["C"] * r["K"]))
+    return dict(best, L=best["C"] * best["K"], met=False)
+
+
+def tune_amortizing_factor(rt, torch, body, grid, args, flush, bound=0.04, candidates=DEFAULT_CANDIDATES,
+                           reps=10, stream=None):
+    """Offline tuning of L for one kernel and input: time the unwrapped kernel and the
+    wrapped variants (CUDA events on `stream`, L2 flushed before each launch, median of `reps`),
+    trying L from small to large and stopping at the first L that has a variant under `bound`.
+    `rt` must be a MANUAL-mode runtime with exec_on_user_stream. Returns (choice, table)."""
+    s = stream or torch.cuda.current_stream()
+
+    def timed(fn):
+        ts = []
+        for r in range(reps + 2):
+            flush()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(s)
+            h = fn()
+            e1.record(s)
+            e1.synchronize()
+            if h is not None:
+                rt.sync(h)
+            if r >= 2:
+                ts.append(e0.elapsed_time(e1) * 1e3)
+        return float(np.median(ts))
+
+    t_u = timed(lambda: rt.launch_unwrapped(body, grid, args, stream=s))
+    table = []
+    by_l = {}
+    for c, k, pf, ap in candidates:
+        if body == F.BODY_GEMM_BF16 and pf:
+            continue                          # (in-tile GEMM: no prefetch, see flep.h)
+        by_l.setdefault(c * k, []).append((c, k, pf, ap))
+    for L in sorted(by_l):
+        for c, k, pf, ap in by_l[L]:
+            kk = rt.register_kernel(body, chunk=c, poll=k, prefetch=pf, async_poll=ap,
+                                    in_tile=body == F.BODY_GEMM_BF16)
+            t_w = timed(lambda: rt.launch(kk, grid, args, stream=s))
+            table.append({"C": c, "K": k, "prefetch": pf, "async_poll": ap, "wrapped_us": round(t_w, 3),
+                          "unwrapped_us": round(t_u, 3), "overhead": t_w / t_u - 1.0})
+        if any(r["overhead"] < bound for r in table if r["C"] * r["K"] == L):
+            break
+    return select_amortizing_factor(table, bound), table
