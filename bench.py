@@ -34,6 +34,7 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 from synth import gen  # noqa: E402
+from paper_conf_asplos_wulzj17_b200.calibrate import event_mean_us  # noqa: E402
 
 METRIC = ("preemption latency µs (full vs N-SM yield); wrapper overhead % of HBM/tensor roofline; "
           "co-run NATT")
@@ -383,8 +384,9 @@ def kernel_timings(rt, F, torch, wl, flush, A, kLP, kHP, lp_args, hp_args, lp_gr
                     rt.sync(h)
                 if r >= 2:
                     (tw if mode == "w" else tu).append(e0.elapsed_time(e1) * 1e3)
-        w_us, u_us = float(np.median(tw)), float(np.median(tu))
-        res[name] = {"wrapped_us": round(w_us, 3), "unwrapped_us": round(u_us, 3),
+        w_us, u_us = event_mean_us(tw), event_mean_us(tu)
+        res[name] = {"stat": "trimmed mean (middle 80 %) of CUDA-event durations",
+                     "wrapped_us": round(w_us, 3), "unwrapped_us": round(u_us, 3),
                      "wrapped_min_us": round(min(tw), 3), "unwrapped_min_us": round(min(tu), 3),
                      "wrapped_gbs": round(nbytes / (w_us * 1e-6) / 1e9, 1),
                      "unwrapped_gbs": round(nbytes / (u_us * 1e-6) / 1e9, 1),
@@ -538,7 +540,7 @@ def main():
     ap.add_argument("--hp-prefetch", type=int, default=1)
     ap.add_argument("--hp-async", type=int, default=1, help="waiting kernel: async poll (R22)")
     ap.add_argument("--lp-poll", type=int, default=1)
-    ap.add_argument("--reps", type=int, default=20)
+    ap.add_argument("--reps", type=int, default=40)
     ap.add_argument("--e2e-steps", type=int, default=10)
     ap.add_argument("--tune-bound", type=float, default=0.04, help="config tune: overhead bound (P:166: 4 %%)")
     ap.add_argument("--gemm-in-tile", type=int, default=1, help="config gemm: in-tile preemption (1) or tile granularity (0)")

@@ -681,7 +681,7 @@ def run_tune(args, rank, world, local):
     met = sum(1 for r in rows.values() if r["choice"]["met"])
     out = {"metric": METRIC, "value": met, "unit": f"kernels (of {len(rows)}) whose tuned L meets the overhead bound",
            "value_definition": "offline amortizing-factor tuning (P:166): smallest L = C*K with wrapped/unwrapped - 1 "
-                               f"< {args.tune_bound} (event-timed, L2 flushed, median of {args.reps})",
+                               f"< {args.tune_bound} (event-timed, L2 flushed, trimmed mean of {args.reps})",
            "n_gpus": world, "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "mixed",
            "data": "synthetic (seeded)", "config": {"workload": "amortizing-factor tuning at the BASELINE configs' sizes",
                                                       "bound": args.tune_bound},

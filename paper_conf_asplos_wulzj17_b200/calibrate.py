@@ -109,6 +109,15 @@ class Workloads:
         raise ValueError(body)
 
 
+def event_mean_us(ts):
+    """Summary of CUDA-event durations (us): events are stamped with a ~1 us quantum on this
+    system, so a median of a few samples sits on a quantum; the mean of the middle 80 % of the
+    samples averages over the kernel's random phase against the quantum instead."""
+    v = np.sort(np.asarray(ts, dtype=np.float64))
+    k = len(v) // 10
+    return float(np.mean(v[k:len(v) - k])) if len(v) > 2 * k else float(np.mean(v))
+
+
 def _flush(torch, buf):
     buf.zero_()
 
@@ -216,9 +225,9 @@ def select_amortizing_factor(table, bound=0.04):
 
 
 def tune_amortizing_factor(rt, torch, body, grid, args, flush, bound=0.04, candidates=DEFAULT_CANDIDATES,
-                           reps=10, stream=None):
+                           reps=30, stream=None):
     """Offline tuning of L for one kernel and input: time the unwrapped kernel and the
-    wrapped variants (CUDA events on `stream`, L2 flushed before each launch, median of `reps`),
+    wrapped variants (CUDA events on `stream`, L2 flushed before each launch, trimmed mean of `reps`),
     trying L from small to large and stopping at the first L that has a variant under `bound`.
     `rt` must be a MANUAL-mode runtime with exec_on_user_stream. Returns (choice, table)."""
     s = stream or torch.cuda.current_stream()
@@ -236,7 +245,7 @@ def tune_amortizing_factor(rt, torch, body, grid, args, flush, bound=0.04, candi
                 rt.sync(h)
             if r >= 2:
                 ts.append(e0.elapsed_time(e1) * 1e3)
-        return float(np.median(ts))
+        return event_mean_us(ts)
 
     t_u = timed(lambda: rt.launch_unwrapped(body, grid, args, stream=s))
     table = []

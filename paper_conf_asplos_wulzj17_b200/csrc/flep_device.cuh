@@ -11,8 +11,11 @@
 // polled with ld.acquire.gpu (an L2 hit) once per K chunks; a chunk is C original blocks per
 // atomicAdd (the probe measured ~1.46 fetches/ns chip-wide on one address, so C amortises the
 // atomic); exits happen only at poll points or on exhaustion, never while holding a chunk
-// (exactly-once, reading A4). The last worker of an epoch publishes DONE/PREEMPTED to a pinned
-// host slot with one relaxed system-scope 8-byte store.
+// (exactly-once, reading A4). Exit accounting (reading R23): the counter and the exit counts share
+// one 64-bit word; a worker's exit is counted by its exhausted fetch (the fetch that returns a
+// value >= N, which it makes anyway), or by one yield-exit increment if it never made one, so a
+// grid that runs to completion does no atomic at exit. The issuer of the W-th exit event
+// publishes DONE/PREEMPTED to a pinned host slot with one relaxed system-scope 8-byte store.
 #pragma once
 #include <cstdint>
 
@@ -27,16 +30,17 @@ constexpr uint32_t kNoTrigger = 0xffffffffu;
 
 // Per-launch control block in device memory. Hot words on separate 128-B lines.
 struct alignas(128) ControlBlock {
-  uint32_t ctr;            // task counter: next original block index to hand out (D4)
-  uint32_t _p0[31];
+  // the counter word (R23): bits 0-31 = task counter, the next original block index to hand out
+  // (D4; raw, see ctr_offset); bits 32-47 = yield exits of the current epoch; bits 48-63 =
+  // original blocks those exits left unfinished in partial tile records (in-tile preemption).
+  // The epoch's last worker resets the high half.
+  unsigned long long cx;
+  uint32_t _p0[30];
   uint32_t ctrl;           // epoch<<16 | n_yield (D1/D2); device copy for the memop transport
   uint32_t _p1[31];
-  // one 64-bit word, one atomic per worker exit: low half = original blocks executed (all
-  // epochs), high half = workers of the current epoch that have exited (reset by the last)
-  unsigned long long done_exited;
   uint32_t done_gen;       // generation whose epoch completed the launch (0 = none yet); an
                            // epoch launched after that (e.g. a refill) exits without fetching
-  uint32_t _p2[29];
+  uint32_t _p2[31];
   // per-epoch summaries (ring of kEvEpochs)
   uint64_t ep_t_trigger[kEvEpochs];
   uint64_t ep_t_end[kEvEpochs];
@@ -93,6 +97,7 @@ struct WorkerParams {
 };
 #ifdef FLEP_TRACE
 constexpr uint32_t kTraceChunks = 64;
+constexpr uint32_t kTraceWords = 4;    // per chunk: loop top, poll decided, step returned, after the barrier
 #endif
 
 // In-tile preemption state: record i belongs to worker i of every epoch of a launch.
@@ -161,6 +166,15 @@ struct alignas(16) WorkerShared {
   uint32_t poll_buf[4];    // async poll: the control word's 16-B line, copied by cp.async.cg
   uint64_t t_entry;
   uint32_t sm, blocks, reason;
+  // exit accounting (R23), written by the scheduling thread when its exit event happens
+  uint32_t counted;        // the exit event has happened (exhausted fetch or yield increment)
+  uint32_t last;           // ... and it was the epoch's W-th: this worker publishes the epoch
+  uint32_t ev_raw;         // raw counter after that event (no fetch follows the W-th event)
+  uint32_t ev_part;        // blocks left unfinished in partial tile records, including this one's
+  uint32_t partial;        // blocks this worker leaves unfinished in its partial tile record
+#ifdef FLEP_TRACE
+  uint64_t t_poll;         // diagnostics: when the scheduling step's poll decision was taken
+#endif
 };
 
 // Async poll (R22): copy the control word's 16 B from L2 (cp.async.cg bypasses L1, so it never
@@ -184,7 +198,7 @@ __device__ __forceinline__ uint32_t poll_consume(const WorkerShared& ws) {
 // self-trigger of the test/bench hooks.
 struct SchedState {
   uint32_t k = 0;                    // chunk index within the current poll period
-  uint32_t held = 0xffffffffu;       // prefetched counter value not yet handed out (raw: the
+  unsigned long long held = ~0ull;   // prefetched counter word not yet handed out (raw: the
                                      // first-epoch offset is added when it is consumed, so the
                                      // atomic's round trip overlaps the body)
   bool have_seen = false;            // async poll: a copy of the control word is in flight
@@ -200,17 +214,38 @@ __device__ __forceinline__ uint32_t ctr_offset(const WorkerParams& p) {
 // The counter atomic as plain PTX: atomicAdd() lets nvcc emit a warp-aggregated sequence whose
 // SHFL consumes the result at once, which would make a prefetching thread wait for the whole L2
 // round trip right there; with atom.add the wait happens only where the value is used.
-__device__ __forceinline__ uint32_t atom_add_ctr(uint32_t* ctr, uint32_t v) {
-  uint32_t old;
+__device__ __forceinline__ unsigned long long atom_add_cx(unsigned long long* cx, unsigned long long v) {
+  unsigned long long old;
   // an opaque zero offset (ptxas cannot prove the address warp-uniform, so it emits no
   // aggregation sequence around the atomic)
   uint64_t z;
   asm volatile("mov.u64 %0, 0;" : "=l"(z));
-  asm volatile("atom.relaxed.gpu.global.add.u32 %0, [%1], %2;" : "=r"(old) : "l"(ctr + z), "r"(v) : "memory");
+  asm volatile("atom.relaxed.gpu.global.add.u64 %0, [%1], %2;" : "=l"(old) : "l"(cx + z), "l"(v) : "memory");
   return old;
 }
-__device__ __forceinline__ uint32_t fetch_chunk(const WorkerParams& p) {
-  return atom_add_ctr(&p.cb->ctr, p.chunk) + ctr_offset(p);
+__device__ __forceinline__ unsigned long long fetch_chunk(const WorkerParams& p) {
+  return atom_add_cx(&p.cb->cx, p.chunk);
+}
+// First raw counter value whose fetch finds no work in this epoch (R23): the counter hands out
+// multiples of C from the epoch's start, which never exceeds ceil(N/C)*C (effective).
+__device__ __forceinline__ uint32_t first_exhausted_raw(const WorkerParams& p) {
+  const uint32_t off = ctr_offset(p);
+  const uint32_t cap = ((p.n_blocks + p.chunk - 1) / p.chunk) * p.chunk;
+  return cap > off ? cap - off : 0u;
+}
+// This worker's exit event (R23) happened with the counter word's old value `old` (the event
+// added `add_lo` to the counter): exhausted fetches before it = (raw - first exhausted) / C,
+// yield exits before it = bits 32-47; the event that makes W is the epoch's last.
+__device__ __forceinline__ void note_exit_event(const WorkerParams& p, WorkerShared& ws,
+                                                unsigned long long old, uint32_t add_lo, uint32_t own_partial) {
+  const uint32_t raw = (uint32_t)old;
+  const uint32_t t = first_exhausted_raw(p);
+  const uint32_t exh = raw >= t ? (raw - t) / p.chunk : 0u;
+  const uint32_t yields = (uint32_t)(old >> 32) & 0xffffu;
+  ws.counted = 1u;
+  ws.last = (exh + yields + 1u == p.workers) ? 1u : 0u;
+  ws.ev_raw = raw + add_lo;
+  ws.ev_part = (uint32_t)(old >> 48) + own_partial;
 }
 
 __device__ __forceinline__ uint32_t next_chunk(const WorkerParams& p, SchedState& st, WorkerShared& ws) {
@@ -239,18 +274,27 @@ __device__ __forceinline__ uint32_t next_chunk(const WorkerParams& p, SchedState
     const uint32_t c = (p.async_poll && st.have_seen) ? poll_consume(ws) : ld_relaxed_gpu(p.ctrl);
     if (should_yield(c, p, smid_reg())) { st.stopping = true; ws.reason = kReasonYield; }
   }
+#ifdef FLEP_TRACE
+  ws.t_poll = gtimer();
+#endif
   if (!have) {
-    if (st.held != 0xffffffffu) {                    // a fetched chunk is always processed (A4)
-      base = st.held + ctr_offset(p);
-      st.held = 0xffffffffu;
+    unsigned long long w = ~0ull;
+    if (st.held != ~0ull) {                          // a fetched chunk is always processed (A4)
+      w = st.held;
+      st.held = ~0ull;
     } else if (!st.stopping) {
-      base = fetch_chunk(p);
+      w = fetch_chunk(p);
+    }
+    if (w != ~0ull) {
+      base = (uint32_t)w + ctr_offset(p);
+      // an exhausted fetch is this worker's exit event (R23); nothing is fetched after it
+      if (base >= p.n_blocks) { note_exit_event(p, ws, w, p.chunk, 0u); base = 0xffffffffu; ws.reason = kReasonExhausted; }
     }
   }
   if (base != 0xffffffffu && base >= p.n_blocks) { base = 0xffffffffu; ws.reason = kReasonExhausted; }
   if (base != 0xffffffffu) {
     ws.blocks += min(p.chunk, p.n_blocks - base);
-    if (p.prefetch && !st.stopping) st.held = atom_add_ctr(&p.cb->ctr, p.chunk);   // overlaps the body
+    if (p.prefetch && !st.stopping) st.held = fetch_chunk(p);   // overlaps the body
     if (p.trigger_block - base < p.chunk) {          // device self-trigger inside this chunk
       const uint32_t e = p.epoch % kEvEpochs;
       p.cb->ep_t_trigger[e] = gtimer();
@@ -286,6 +330,7 @@ flep_worker(const __grid_constant__ typename Body::Args args, const WorkerParams
   const uint32_t tid = threadIdx.x;
   if (tid == 0) {
     ws.sm = smid_reg(); ws.t_entry = gtimer(); ws.blocks = 0; ws.reason = 0;
+    ws.counted = 0; ws.last = 0; ws.ev_raw = 0; ws.ev_part = 0; ws.partial = 0;
     if (blockIdx.x == 0 && p.started_hint && p.status) st_relaxed_sys(&p.status->started, p.epoch);
   }
   Body::setup(args);                 // per-worker resources (e.g. TMEM, mbarriers); may sync
@@ -300,18 +345,21 @@ flep_worker(const __grid_constant__ typename Body::Args args, const WorkerParams
     while (true) {
 #ifdef FLEP_TRACE
       // diagnostics: per chunk, when tid 0 reached the scheduling step (its share of the previous
-      // body done) and when the step returned (poll + fetch latency)
+      // body done), when the poll decision was taken, when the step returned (fetch done) and
+      // when the chunk barrier released it (the slowest warp of the previous body)
       const uint64_t ta = (tid == 0 && p.trace) ? gtimer() : 0;
       if (tid == 0) s_slot[parity] = next_chunk(p, st, ws);
+      const uint64_t tb = (tid == 0 && p.trace) ? gtimer() : 0;
+      __syncthreads();
       if (tid == 0 && p.trace && nchunk < kTraceChunks) {
-        uint64_t* t = p.trace + ((size_t)blockIdx.x * kTraceChunks + nchunk) * 2;
-        t[0] = ta; t[1] = gtimer();
+        uint64_t* t = p.trace + ((size_t)blockIdx.x * kTraceChunks + nchunk) * kTraceWords;
+        t[0] = ta; t[1] = ws.t_poll; t[2] = tb; t[3] = gtimer();
       }
       ++nchunk;
 #else
       if (tid == 0) s_slot[parity] = next_chunk(p, st, ws);
-#endif
       __syncthreads();
+#endif
       const uint32_t b0 = s_slot[parity];
       parity ^= 1u;
       if (b0 == 0xffffffffu) break;
@@ -322,39 +370,43 @@ flep_worker(const __grid_constant__ typename Body::Args args, const WorkerParams
     }
   }
   Body::teardown(args);              // release per-worker resources before leaving the SM (a7)
-  // exit path (a7). One relaxed 64-bit atomic adds this worker's block count and its exit; the
-  // worker that completes the epoch's exit count sees the exact total. No fences: the outputs
-  // are published by kernel completion (stream order), and the host status is a notification.
+  // exit path (a7). A worker whose exit was counted by its exhausted fetch does no atomic here;
+  // any other (yield, entry exit) makes its exit event now: one 64-bit increment of the yield
+  // count (R23). No fences: the outputs are published by kernel completion (stream order), and
+  // the host status is a notification (flep_sync also waits for the grid's completion event).
   if (tid == 0) {
-    const uint32_t my_blocks = ws.blocks;
     WorkerEvent& e = p.ev[(p.epoch % kEvEpochs) * p.workers + blockIdx.x];
     const uint64_t t_exit = gtimer();
-    e.smid = ws.sm; e.reason = ws.reason; e.n_blocks = my_blocks; e.epoch = p.epoch;
+    e.smid = ws.sm; e.reason = ws.reason; e.n_blocks = ws.blocks; e.epoch = p.epoch;
     e.t_entry = ws.t_entry; e.t_exit = t_exit;
-    const unsigned long long old = atomicAdd(&p.cb->done_exited, (1ull << 32) | my_blocks);
-    if ((uint32_t)(old >> 32) + 1 == p.workers) {        // last worker of this epoch
-      // both loads issued back to back (one round trip); the first epoch of a launch cannot
-      // find it already complete
+    if (!ws.counted) {
+      const unsigned long long inc = (1ull << 32) | ((unsigned long long)ws.partial << 48);
+      note_exit_event(p, ws, atom_add_cx(&p.cb->cx, inc), 0u, ws.partial);
+    }
+    if (ws.last) {                                       // the epoch's W-th exit event
+      // every worker has made its exit event: none fetches again (some may still run the chunk
+      // they hold, which they complete before the grid ends, A4)
       const bool first_epoch = p.epoch == p.gen_first;
-      const uint32_t raw = ld_relaxed_gpu(&p.cb->ctr);   // every fetch has completed by now
       const bool already = !first_epoch && ld_relaxed_gpu(&p.cb->done_gen) >= p.gen_first;
-      const uint32_t c = first_epoch ? raw + p.workers * p.chunk : raw;   // effective counter (R20)
-      const uint32_t d = already ? p.n_blocks : (uint32_t)old + my_blocks;
-      const uint32_t st = (d >= p.n_blocks) ? kStateDone : kStatePreempted;
+      const uint32_t c = ws.ev_raw + ctr_offset(p);      // effective counter (R20)
+      const bool done = already || (c >= p.n_blocks && ws.ev_part == 0u);
+      const uint32_t d = done ? p.n_blocks : min(c, p.n_blocks) - ws.ev_part;
+      const uint32_t st = done ? kStateDone : kStatePreempted;
       const uint32_t ei = p.epoch % kEvEpochs;
       p.cb->ep_t_end[ei] = t_exit; p.cb->ep_done[ei] = d; p.cb->ep_ctr[ei] = c;
       p.cb->ep_state[ei] = st;
       p.cb->ep_t_trigger[(p.epoch + 1) % kEvEpochs] = 0;  // next epoch's trigger stamp
-      if (st == kStateDone) {                            // clean for reuse; remember completion
-        p.cb->done_exited = 0ull; p.cb->ctr = 0;
+      if (done) {                                        // clean for reuse; remember completion
+        p.cb->cx = 0ull;
         if (!already) p.cb->done_gen = p.epoch;
       } else {
-        p.cb->done_exited = (unsigned long long)d;       // exits reset, progress kept
-        p.cb->ctr = c;                                   // later epochs fetch from the effective
-      }                                                  // counter (no fetch is in flight now)
+        // progress kept, exit counts reset; later epochs fetch from the effective counter,
+        // capped at ceil(N/C)*C (only reached when partial tiles remain)
+        const uint32_t cap = ((p.n_blocks + p.chunk - 1) / p.chunk) * p.chunk;
+        p.cb->cx = (unsigned long long)min(c, cap);
+      }
       if (p.status) {
         st_relaxed_sys(&p.status->ctr, c);
-        st_relaxed_sys_u64(&p.status->t_end, t_exit);
         st_relaxed_sys_u64(reinterpret_cast<uint64_t*>(&p.status->word),
                            ((uint64_t)d << 32) | ((p.epoch << 8) | st));
       }

@@ -312,6 +312,7 @@ struct GemmBody {
               const uint32_t c = ld_relaxed_gpu(p.ctrl);   // entry check (a2) before taking it
               if (should_yield(c, p, smid_reg())) {
                 ws.reason = kReasonYield;                  // the record stays for a later epoch
+                ws.partial = e.b_end - e.b;                // blocks still unfinished (R23)
                 rb0 = STOP; rb1 = 1;                       // (marker: leave at once)
               } else {
                 rb0 = e.b; rb1 = e.b_end; rkb = e.kb;
@@ -378,6 +379,7 @@ struct GemmBody {
                 for (uint32_t bb = b + 1; bb < b1; ++bb) atomicAdd(&p.cov[bb], 1u);
               ws.blocks -= b1 - b;                         // tiles b..b1-1 are not complete
               ws.reason = kReasonYield;
+              ws.partial = b1 - b;                         // the epoch cannot complete (R23)
               leave = true;
               break;
             }

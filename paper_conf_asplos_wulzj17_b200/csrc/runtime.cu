@@ -297,7 +297,9 @@ flep_status start_epoch(flep_rt rt, Launch& L) {
   p.gy = L.grid.y;
   p.trigger_block = L.trig_block;
   p.trigger_n = L.trig_n;
-  p.prefetch = (L.flags & FLEP_KFLAG_PREFETCH) ? 1u : 0u;
+  // no prefetch with in-tile preemption: a worker whose exhausted prefetch already counted its
+  // exit must not later leave a partial tile (R23)
+  p.prefetch = ((L.flags & FLEP_KFLAG_PREFETCH) && !(L.flags & FLEP_KFLAG_IN_TILE)) ? 1u : 0u;
   p.gen_first = L.gen0 + 1;
   p.started_hint = (L.flags & FLEP_KFLAG_STARTED_HINT) ? 1u : 0u;
   p.async_poll = ((L.flags & FLEP_KFLAG_ASYNC_POLL) && rt->opt.flag != FLEP_FLAG_HOST_MAPPED) ? 1u : 0u;
@@ -360,7 +362,7 @@ bool refresh(flep_rt rt, Launch& L) {
 void release_resources(flep_rt rt, Launch& L) {
   if (L.released) return;
   // the launch's last grid has completed (caller synchronised the exec stream); the last worker
-  // of the DONE epoch left ctr/done/exited at 0, so the block is reusable as is
+  // of the DONE epoch left the counter word at 0, so the block is reusable as is
   if (L.dmem) { rt->cb_gen[L.dmem] = gen_of(L) + 1; rt->free_dmem.push_back(L.dmem); }
   if (L.cov) rt->free_cov.push_back({L.cov, L.cov_cap});
   if (L.partial) rt->free_partial.push_back({L.partial, L.partial_cap});
@@ -1072,7 +1074,16 @@ flep_status flep_debug_epoch_info(flep_rt rt, flep_launch_t h, uint32_t epoch, f
   CUDA_TRY(cudaStreamSynchronize(L->exec));
   const uint32_t e = (L->gen0 + epoch) % kEvEpochs;
   out->t_trigger = cb.ep_t_trigger[e];
-  out->t_end = cb.ep_t_end[e];
+  // t_end = the epoch's last worker exit. The publishing worker is the last to stop taking work
+  // (R23), not necessarily the last to leave, so take the maximum over the epoch's worker log.
+  std::vector<WorkerEvent> ev(L->workers);
+  CUDA_TRY(cudaMemcpyAsync(ev.data(), L->ev + (size_t)e * L->workers, L->workers * sizeof(WorkerEvent),
+                           cudaMemcpyDeviceToHost, L->exec));
+  CUDA_TRY(cudaStreamSynchronize(L->exec));
+  uint64_t t_end = 0;
+  for (const WorkerEvent& w : ev)
+    if (w.epoch == L->gen0 + epoch && w.t_exit > t_end) t_end = w.t_exit;
+  out->t_end = t_end ? t_end : cb.ep_t_end[e];
   out->trigger_block = cb.ep_trigger_block[e];
   out->done = cb.ep_done[e];
   out->counter = cb.ep_ctr[e];

@@ -242,3 +242,45 @@ def test_hand_traced_async_poll_acts_one_chunk_later():
     for lab in ["w0.poll", "w0.fetch", "preempt(2)", "w0.proc", "w0.poll", "w0.exit"]:
         st = dict(cv.successors(sync, st))[lab]
     assert st[6] == cv.ST_PREEMPTED and st[4] == (1, 0, 0, 0)
+
+
+# ---- exit accounting by the exhausted fetch (R23) -----------------------------------
+
+def _early_done_states(cfg):
+    """Reachable states where DONE is published while some worker still runs a held chunk."""
+    start = cv._canon(cfg, cv.initial_state(cfg))
+    seen, stack, early = {start}, [start], 0
+    while stack:
+        st = stack.pop()
+        if st[6] == cv.ST_DONE and not cv._all_gone(st[7]) and any(w[0] == cv.PROC for w in st[7]):
+            early += 1
+        for _, s2 in cv.successors(cfg, st):
+            s2 = cv._canon(cfg, s2)
+            if s2 not in seen:
+                seen.add(s2)
+                stack.append(s2)
+    return early
+
+
+def test_done_published_early_is_reached_and_safe():
+    # with prefetch the W-th exit event can be an exhausted prefetch: DONE is then published
+    # while its issuer (and others) still run their last chunks; I6 holds in every such state
+    cfg = _cfg(n_blocks=5, chunk=1, poll=1, worker_sm=(0, 1), prefetch=True, static_first=True)
+    assert _early_done_states(cfg) > 0
+    assert cv.explore(cfg).violations == set()
+
+
+def test_first_exhausted_value_formula():
+    # the device formula: multiples of C from the epoch start (W*C with static first chunks)
+    cfg = cv.Config(n_blocks=7, chunk=2, poll=1, worker_sm=(0, 1), num_sms=2, static_first=True)
+    assert cv._first_exhausted(cfg, 0) == 8 and cv._first_exhausted(cfg, 1) == 8
+    cfg = cv.Config(n_blocks=3, chunk=2, poll=1, worker_sm=(0, 0, 1), num_sms=2, static_first=True)
+    assert cv._first_exhausted(cfg, 0) == 6 and cv._first_exhausted(cfg, 1) == 4
+
+
+def test_planted_double_count_is_caught():
+    # counting a worker's exit twice lets an early event look like the W-th: the epoch is
+    # published while a worker can still fetch (or never published at all)
+    for pf in (False, True):
+        cfg = _cfg(n_blocks=5, chunk=1, poll=1, worker_sm=(0, 0, 1), prefetch=pf, bug_count_twice=True)
+        assert cv.explore(cfg).violations

@@ -18,6 +18,7 @@ sys.path.insert(0, ROOT)
 from synth import gen  # noqa: E402
 
 KT = 64
+KW = 4      # words per chunk record (flep_device.cuh kTraceWords)
 
 
 def main():
@@ -59,7 +60,7 @@ def main():
         rt.set_trace(None, None)
         for C, K, pf, ap in combos:
             kk = rt.register_kernel(body, chunk=C, poll=K, prefetch=bool(pf), async_poll=bool(ap))
-            wt = torch.zeros(w * KT * 2, dtype=torch.int64, device="cuda")
+            wt = torch.zeros(w * KT * KW, dtype=torch.int64, device="cuda")
             rt.set_trace(wt, None)
             for rep in range(4):
                 wt.zero_()
@@ -69,25 +70,31 @@ def main():
                 rt.sync(h, timeout_ns=5_000_000_000)
                 torch.cuda.synchronize()
             rt.set_trace(None, None)
-            tr = wt.view(w, KT, 2).cpu().numpy().astype(np.int64)
+            tr = wt.view(w, KT, KW).cpu().numpy().astype(np.int64)
             ev = rt.events(h, 1)
             entry = np.array([e.t_entry for e in ev])
             exit_ = np.array([e.t_exit for e in ev])
             t0 = entry.min()
-            sched, bodyt, first = [], [], []
+            sched, bodyt, first, pollt, fetcht, bart = [], [], [], [], [], []
             for i in range(w):
-                ta, tb = tr[i, :, 0], tr[i, :, 1]
+                ta, tp, tb, tc = tr[i, :, 0], tr[i, :, 1], tr[i, :, 2], tr[i, :, 3]
                 n = int(np.count_nonzero(ta))
                 if n == 0:
                     continue
                 sched.extend((tb[:n] - ta[:n]) / 1e3)
-                bodyt.extend((ta[1:n] - tb[:n - 1]) / 1e3)
-                first.append((tb[0] - t0) / 1e3)
+                pollt.extend((tp[:n] - ta[:n]) / 1e3)
+                fetcht.extend((tb[:n] - tp[:n]) / 1e3)
+                bart.extend((tc[:n] - tb[:n]) / 1e3)
+                bodyt.extend((ta[1:n] - tc[:n - 1]) / 1e3)
+                first.append((tc[0] - t0) / 1e3)
+            m = lambda v: round(float(np.mean(v)), 3) if len(v) else None  # noqa: E731
             print(json.dumps({"body": name, "variant": "wrapped", "C": C, "K": K, "prefetch": pf, "async_poll": ap,
                               "span_us": round((exit_.max() - t0) / 1e3, 2),
-                              "sched_us_mean": round(float(np.mean(sched)), 3),
+                              "sched_us_mean": m(sched),
                               "sched_us_p50": round(float(np.median(sched)), 3),
-                              "body_us_mean": round(float(np.mean(bodyt)), 3),
+                              "poll_us_mean": m(pollt), "fetch_us_mean": m(fetcht),
+                              "barrier_wait_us_mean": m(bart),
+                              "body_us_mean": m(bodyt),
                               "body_us_p50": round(float(np.median(bodyt)), 3),
                               "first_chunk_ready_us_p50": round(float(np.median(first)), 3),
                               "exit_first_us": round((exit_.min() - t0) / 1e3, 2),
