@@ -34,7 +34,7 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 from synth import gen  # noqa: E402
-from paper_conf_asplos_wulzj17_b200.calibrate import event_mean_us  # noqa: E402
+from paper_conf_asplos_wulzj17_b200.calibrate import dither, event_mean_us  # noqa: E402
 
 METRIC = ("preemption latency µs (full vs N-SM yield); wrapper overhead % of HBM/tensor roofline; "
           "co-run NATT")
@@ -205,7 +205,8 @@ def run_temporal(args, rank, world, local):
     kLP = rt.register_kernel(F.BODY_SPMV_CSR_F32, chunk=args.lp_chunk, poll=args.lp_poll, name="spmv",
                              prefetch=bool(args.prefetch))
     # the waiting (high-priority) kernel is never preempted here: its chunking is tuned for
-    # throughput (C = 2 with prefetch), the victim's for latency (C = K = 1)
+    # throughput (C = 4, the tuned choice of tools/overhead_breakdown.py), the victim's for
+    # latency (C = K = 1)
     kHP = rt.register_kernel(F.BODY_STENCIL5_F32, chunk=args.hp_chunk, poll=1, name="stencil",
                              prefetch=bool(args.hp_prefetch), async_poll=bool(args.hp_async))
     lp_args = F.spmv_args(wl.d_y, wl.d_rowptr, wl.d_col, wl.d_val, wl.d_x)
@@ -372,6 +373,7 @@ def kernel_timings(rt, F, torch, wl, flush, A, kLP, kHP, lp_args, hp_args, lp_gr
             for mode in ("w", "u"):
                 with torch.cuda.stream(A):
                     flush.zero_()
+                    dither(torch)
                     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                     e0.record(A)
                 if mode == "w":
@@ -385,7 +387,7 @@ def kernel_timings(rt, F, torch, wl, flush, A, kLP, kHP, lp_args, hp_args, lp_gr
                 if r >= 2:
                     (tw if mode == "w" else tu).append(e0.elapsed_time(e1) * 1e3)
         w_us, u_us = event_mean_us(tw), event_mean_us(tu)
-        res[name] = {"stat": "trimmed mean (middle 80 %) of CUDA-event durations",
+        res[name] = {"stat": "trimmed mean (middle 80 %) of dithered CUDA-event durations",
                      "wrapped_us": round(w_us, 3), "unwrapped_us": round(u_us, 3),
                      "wrapped_min_us": round(min(tw), 3), "unwrapped_min_us": round(min(tu), 3),
                      "wrapped_gbs": round(nbytes / (w_us * 1e-6) / 1e9, 1),
@@ -536,9 +538,9 @@ def main():
     ap.add_argument("--rho", type=float, default=1.0)
     ap.add_argument("--lp-chunk", type=int, default=1)
     ap.add_argument("--prefetch", type=int, default=0)
-    ap.add_argument("--hp-chunk", type=int, default=2)
-    ap.add_argument("--hp-prefetch", type=int, default=1)
-    ap.add_argument("--hp-async", type=int, default=1, help="waiting kernel: async poll (R22)")
+    ap.add_argument("--hp-chunk", type=int, default=4)
+    ap.add_argument("--hp-prefetch", type=int, default=0)
+    ap.add_argument("--hp-async", type=int, default=0, help="waiting kernel: async poll (R22)")
     ap.add_argument("--lp-poll", type=int, default=1)
     ap.add_argument("--reps", type=int, default=40)
     ap.add_argument("--e2e-steps", type=int, default=10)

@@ -109,10 +109,21 @@ class Workloads:
         raise ValueError(body)
 
 
+_DITHER = np.random.default_rng(12345)
+
+
+def dither(torch, base_cycles=0):
+    """A spin of random length (0-4096 SM cycles, ~0-2 us) on the current stream before a timed
+    launch: CUDA events are stamped with a ~1 us quantum here, and right after the L2 flush the
+    launch's phase against that quantum is nearly fixed; the spin randomises it so that the mean
+    of the samples resolves well below the quantum (see event_mean_us)."""
+    torch.cuda._sleep(int(base_cycles) + int(_DITHER.integers(0, 4096)))
+
+
 def event_mean_us(ts):
     """Summary of CUDA-event durations (us): events are stamped with a ~1 us quantum on this
     system, so a median of a few samples sits on a quantum; the mean of the middle 80 % of the
-    samples averages over the kernel's random phase against the quantum instead."""
+    dithered samples (see dither) averages over the quantum instead."""
     v = np.sort(np.asarray(ts, dtype=np.float64))
     k = len(v) // 10
     return float(np.mean(v[k:len(v) - k])) if len(v) > 2 * k else float(np.mean(v))
@@ -235,7 +246,9 @@ def tune_amortizing_factor(rt, torch, body, grid, args, flush, bound=0.04, candi
     def timed(fn):
         ts = []
         for r in range(reps + 2):
-            flush()
+            with torch.cuda.stream(s):
+                flush()
+                dither(torch)
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record(s)
             h = fn()

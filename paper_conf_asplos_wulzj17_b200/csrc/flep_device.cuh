@@ -15,7 +15,8 @@
 // one 64-bit word; a worker's exit is counted by its exhausted fetch (the fetch that returns a
 // value >= N, which it makes anyway), or by one yield-exit increment if it never made one, so a
 // grid that runs to completion does no atomic at exit. The issuer of the W-th exit event
-// publishes DONE/PREEMPTED to a pinned host slot with one relaxed system-scope 8-byte store.
+// records the epoch; a PREEMPTED epoch is published to a pinned host slot with one relaxed
+// system-scope 8-byte store, a DONE epoch is seen by the host as the grid's completion (R24).
 #pragma once
 #include <cstdint>
 
@@ -97,7 +98,7 @@ struct WorkerParams {
 };
 #ifdef FLEP_TRACE
 constexpr uint32_t kTraceChunks = 64;
-constexpr uint32_t kTraceWords = 4;    // per chunk: loop top, poll decided, step returned, after the barrier
+constexpr uint32_t kTraceWords = 5;    // per chunk: loop top, poll decided, step returned, after the barrier, base known
 #endif
 
 // In-tile preemption state: record i belongs to worker i of every epoch of a launch.
@@ -174,6 +175,7 @@ struct alignas(16) WorkerShared {
   uint32_t partial;        // blocks this worker leaves unfinished in its partial tile record
 #ifdef FLEP_TRACE
   uint64_t t_poll;         // diagnostics: when the scheduling step's poll decision was taken
+  uint64_t t_base;         // diagnostics: when the chunk base was known (before the next prefetch)
 #endif
 };
 
@@ -216,11 +218,12 @@ __device__ __forceinline__ uint32_t ctr_offset(const WorkerParams& p) {
 // round trip right there; with atom.add the wait happens only where the value is used.
 __device__ __forceinline__ unsigned long long atom_add_cx(unsigned long long* cx, unsigned long long v) {
   unsigned long long old;
-  // an opaque zero offset (ptxas cannot prove the address warp-uniform, so it emits no
-  // aggregation sequence around the atomic)
-  uint64_t z;
-  asm volatile("mov.u64 %0, 0;" : "=l"(z));
-  asm volatile("atom.relaxed.gpu.global.add.u64 %0, [%1], %2;" : "=l"(old) : "l"(cx + z), "l"(v) : "memory");
+  // the address carries a lane-dependent offset that is zero for the one lane that executes it
+  // (the scheduling thread is lane 0): ptxas cannot prove it warp-uniform, so it emits no
+  // aggregation sequence around the atomic
+  uint32_t lane;
+  asm volatile("mov.u32 %0, %%laneid;" : "=r"(lane));
+  asm volatile("atom.relaxed.gpu.global.add.u64 %0, [%1], %2;" : "=l"(old) : "l"(cx + lane), "l"(v) : "memory");
   return old;
 }
 __device__ __forceinline__ unsigned long long fetch_chunk(const WorkerParams& p) {
@@ -292,6 +295,9 @@ __device__ __forceinline__ uint32_t next_chunk(const WorkerParams& p, SchedState
     }
   }
   if (base != 0xffffffffu && base >= p.n_blocks) { base = 0xffffffffu; ws.reason = kReasonExhausted; }
+#ifdef FLEP_TRACE
+  ws.t_base = gtimer();
+#endif
   if (base != 0xffffffffu) {
     ws.blocks += min(p.chunk, p.n_blocks - base);
     if (p.prefetch && !st.stopping) st.held = fetch_chunk(p);   // overlaps the body
@@ -353,7 +359,7 @@ flep_worker(const __grid_constant__ typename Body::Args args, const WorkerParams
       __syncthreads();
       if (tid == 0 && p.trace && nchunk < kTraceChunks) {
         uint64_t* t = p.trace + ((size_t)blockIdx.x * kTraceChunks + nchunk) * kTraceWords;
-        t[0] = ta; t[1] = ws.t_poll; t[2] = tb; t[3] = gtimer();
+        t[0] = ta; t[1] = ws.t_poll; t[2] = tb; t[3] = gtimer(); t[4] = ws.t_base;
       }
       ++nchunk;
 #else
@@ -405,7 +411,9 @@ flep_worker(const __grid_constant__ typename Body::Args args, const WorkerParams
         const uint32_t cap = ((p.n_blocks + p.chunk - 1) / p.chunk) * p.chunk;
         p.cb->cx = (unsigned long long)min(c, cap);
       }
-      if (p.status) {
+      // host notification only for a PREEMPTED epoch; DONE is seen as the grid's completion
+      // (a system-scope store delays the completion by a PCIe round trip, R24)
+      if (p.status && !done) {
         st_relaxed_sys(&p.status->ctr, c);
         st_relaxed_sys_u64(reinterpret_cast<uint64_t*>(&p.status->word),
                            ((uint64_t)d << 32) | ((p.epoch << 8) | st));

@@ -116,6 +116,7 @@ struct Launch {
   int64_t t_arrive = 0, t_first_start = -1, t_finish = -1;
   int64_t t_e = 0, overhead = 0;
   uint32_t last_done = 0, last_ctr = 0;
+  bool ctr_known = false;            // last_ctr is current (a silent DONE epoch leaves it on the device)
   int64_t t_last_request = -1, t_last_drain = -1;
   uint32_t gen0 = 0;                 // control-block generation before this launch's epoch 1
   // kernel-slicing baseline (FLEP_POLICY_SLICE): the original kernel as sub-grids of
@@ -341,11 +342,26 @@ bool refresh(flep_rt rt, Launch& L) {
     if (L.state == FLEP_STATE_YIELDING) { L.state = FLEP_STATE_PREEMPTED; L.t_last_drain = now_ns(); }
     return false;
   }
+  // A PREEMPTED epoch is published by its last worker to the pinned slot; a DONE epoch is silent
+  // on the device (a system-scope store would make the grid's completion wait for a PCIe round
+  // trip, R24) and is seen as the completion of the epoch's grid. Query the grid first: once it
+  // has completed, every store it made to the slot is visible, so a slot without this epoch's
+  // word then means DONE.
+  const bool grid_done = L.fin_ev && cudaEventQuery(L.fin_ev) == cudaSuccess;
   const uint64_t w64 = __atomic_load_n(reinterpret_cast<uint64_t*>(&L.hs->word), __ATOMIC_ACQUIRE);
   const uint32_t w = (uint32_t)w64;
-  if ((w >> 8) != (gen_of(L) & 0xffffffu)) return false;
+  if ((w >> 8) != (gen_of(L) & 0xffffffu)) {
+    if (!grid_done) return false;
+    L.last_done = L.n_blocks;
+    L.ctr_known = false;               // read lazily by flep_query (ControlBlock::ep_ctr)
+    L.t_finish = L.t_seen > 0 ? L.t_seen : now_ns();
+    L.t_seen = 0;
+    L.state = FLEP_STATE_DONE;
+    return true;
+  }
   L.last_done = (uint32_t)(w64 >> 32);
   L.last_ctr = __atomic_load_n(&L.hs->ctr, __ATOMIC_ACQUIRE);
+  L.ctr_known = true;
   // the monitor stamps the moment it saw the word move (before taking the lock)
   const int64_t t_obs = L.t_seen > 0 ? L.t_seen : now_ns();
   L.t_seen = 0;
@@ -463,7 +479,7 @@ void monitor_pass(flep_rt rt) {
 // never starved by it.
 void monitor_loop(flep_rt rt) {
   cudaSetDevice(rt->device);
-  struct Watch { const uint64_t* word; uint64_t seen; bool sliced; int64_t id; };
+  struct Watch { const uint64_t* word; uint64_t seen; bool sliced; int64_t id; cudaEvent_t ev; };
   std::vector<std::pair<int64_t, int64_t>> moved;     // (launch, host time seen)
   std::vector<Watch> watch;
   int64_t deadline = -1;
@@ -475,7 +491,10 @@ void monitor_loop(flep_rt rt) {
     moved.clear();
     for (const Watch& w : watch) {
       if (w.sliced) { hit = true; continue; }
-      if (__atomic_load_n(w.word, __ATOMIC_ACQUIRE) != w.seen) { hit = true; moved.push_back({w.id, now_ns()}); }
+      if (__atomic_load_n(w.word, __ATOMIC_ACQUIRE) != w.seen ||
+          (w.ev && cudaEventQuery(w.ev) == cudaSuccess)) {   // a DONE epoch is silent (R24)
+        hit = true; moved.push_back({w.id, now_ns()});
+      }
     }
     if (deadline >= 0 && now_ns() >= deadline) hit = true;
     if (pending_release) hit = true;
@@ -508,7 +527,10 @@ void monitor_loop(flep_rt rt) {
       if (!L || !L->hs) continue;
       const uint64_t* wp = reinterpret_cast<const uint64_t*>(&L->hs->word);
       auto it = snap.find(id);
-      watch.push_back({wp, it != snap.end() ? it->second : ~0ull, L->sliced, id});
+      const bool running = L->state == FLEP_STATE_RUNNING || L->state == FLEP_STATE_YIELDING ||
+                           L->state == FLEP_STATE_PARTIAL;
+      watch.push_back({wp, it != snap.end() ? it->second : ~0ull, L->sliced, id,
+                       (running && !L->sliced) ? L->fin_ev : nullptr});
     }
     deadline = rt->policy->epoch_end();
     pending_release = !rt->to_release.empty();
@@ -885,6 +907,15 @@ flep_status flep_query(flep_rt rt, flep_launch_t h, flep_launch_info* out) {
   Launch* L = find(rt, h);
   if (!L) return fail(FLEP_ERR_INVALID, "unknown launch %lld", (long long)h);
   if (rt->opt.policy == FLEP_POLICY_MANUAL) refresh(rt, *L);
+  if (L->state == FLEP_STATE_DONE && !L->ctr_known && !L->sliced && L->dmem && !L->released) {
+    // the final counter of a silent DONE epoch (R24): one small copy from the control block
+    uint32_t c = 0;
+    const uint32_t e = gen_of(*L) % kEvEpochs;
+    CUDA_TRY(cudaMemcpyAsync(&c, &L->cb->ep_ctr[e], 4, cudaMemcpyDeviceToHost, L->exec));
+    CUDA_TRY(cudaStreamSynchronize(L->exec));
+    L->last_ctr = c;
+    L->ctr_known = true;
+  }
   memset(out, 0, sizeof(*out));
   out->state = L->state;
   out->epoch = L->epoch;

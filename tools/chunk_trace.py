@@ -18,7 +18,7 @@ sys.path.insert(0, ROOT)
 from synth import gen  # noqa: E402
 
 KT = 64
-KW = 4      # words per chunk record (flep_device.cuh kTraceWords)
+KW = 5      # words per chunk record (flep_device.cuh kTraceWords)
 
 
 def main():
@@ -36,6 +36,9 @@ def main():
     y = torch.zeros(1 << 20, device="cuda")
     cases = [("stencil", F.BODY_STENCIL5_F32, F.stencil_grid(4096), F.stencil_args(out, st)),
              ("spmv", F.BODY_SPMV_CSR_F32, F.spmv_grid(1 << 20), F.spmv_args(y, T(rp), T(col), T(val), T(x)))]
+    only = os.environ.get("TRACE_BODIES")
+    if only:
+        cases = [c for c in cases if c[0] in only.split(",")]
     s = torch.cuda.current_stream()
     combos = [(tuple(map(int, c.split(":"))) + (0,))[:4] for c in (sys.argv[1] if len(sys.argv) > 1 else "1:1:0,1:1:1").split(",")]
     for name, body, grid, args in cases:
@@ -75,15 +78,16 @@ def main():
             entry = np.array([e.t_entry for e in ev])
             exit_ = np.array([e.t_exit for e in ev])
             t0 = entry.min()
-            sched, bodyt, first, pollt, fetcht, bart = [], [], [], [], [], []
+            sched, bodyt, first, pollt, fetcht, bart, issuet = [], [], [], [], [], [], []
             for i in range(w):
-                ta, tp, tb, tc = tr[i, :, 0], tr[i, :, 1], tr[i, :, 2], tr[i, :, 3]
+                ta, tp, tb, tc, tq = tr[i, :, 0], tr[i, :, 1], tr[i, :, 2], tr[i, :, 3], tr[i, :, 4]
                 n = int(np.count_nonzero(ta))
                 if n == 0:
                     continue
                 sched.extend((tb[:n] - ta[:n]) / 1e3)
                 pollt.extend((tp[:n] - ta[:n]) / 1e3)
-                fetcht.extend((tb[:n] - tp[:n]) / 1e3)
+                fetcht.extend((tq[:n] - tp[:n]) / 1e3)
+                issuet.extend((tb[:n] - tq[:n]) / 1e3)
                 bart.extend((tc[:n] - tb[:n]) / 1e3)
                 bodyt.extend((ta[1:n] - tc[:n - 1]) / 1e3)
                 first.append((tc[0] - t0) / 1e3)
@@ -92,7 +96,7 @@ def main():
                               "span_us": round((exit_.max() - t0) / 1e3, 2),
                               "sched_us_mean": m(sched),
                               "sched_us_p50": round(float(np.median(sched)), 3),
-                              "poll_us_mean": m(pollt), "fetch_us_mean": m(fetcht),
+                              "poll_us_mean": m(pollt), "fetch_us_mean": m(fetcht), "issue_us_mean": m(issuet),
                               "barrier_wait_us_mean": m(bart),
                               "body_us_mean": m(bodyt),
                               "body_us_p50": round(float(np.median(bodyt)), 3),

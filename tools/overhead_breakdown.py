@@ -20,7 +20,7 @@ from synth import gen  # noqa: E402
 def main():
     import torch
     from paper_conf_asplos_wulzj17_b200 import build, flep as F
-    from paper_conf_asplos_wulzj17_b200.calibrate import event_mean_us
+    from paper_conf_asplos_wulzj17_b200.calibrate import dither, event_mean_us
     from bench import L2Flush
     build.build()
     combos = [tuple(map(int, c.split(":"))) for c in
@@ -41,6 +41,7 @@ def main():
         ts, hs = [], []
         for r in range(reps + 2):
             flush.zero_()
+            dither(torch, int(os.environ.get("DITHER_BASE", "0")))
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record(s)
             h = fn()
