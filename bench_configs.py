@@ -336,6 +336,132 @@ def run_gemm_preempt(args, rank, world, local):
     barrier(world)
 
 
+def run_clc(args, rank, world, local):
+    """CLC task fetch vs the atomic counter (R25) on configs[1] kernels.
+
+    (1) Co-run: LP SpMV-CSR 2^20 rows on a low-priority stream; the HP stencil5 4096^2 is released
+        by the host ~20 us after the LP launch on a high-priority stream. Variants: CLC victim with
+        no request (the hardware's queue yields: try_cancel fails while a higher-priority grid is
+        pending), counter victim with the FLEP request issued by the host at the HP's release
+        (flep_preempt, then resume after the HP), counter victim without a request (the HP waits
+        for the whole LP). Per step (device %globaltimer): HP turnaround = HP last CTA exit - LP
+        first CTA entry, and LP span. Spot parity of the last LP result against the oracle.
+    (2) Wrapper overhead of both fetch variants against the unwrapped kernels (dithered CUDA
+        events, L2 flushed)."""
+    import torch
+    from bench import (ClockSampler, L2Flush, Workload, barrier, physical_gpu_index, spot_parity,
+                       STENCIL_N, SPMV_ROWS)
+    from paper_conf_asplos_wulzj17_b200 import flep as F
+    from paper_conf_asplos_wulzj17_b200.calibrate import dither, event_mean_us
+    torch.cuda.set_device(local)
+    rt = F.Runtime(device=local, exec_on_user_stream=True)
+    wl = Workload(torch)
+    flush = L2Flush(torch)
+    lo, hi = torch.cuda.Stream(priority=0), torch.cuda.Stream(priority=-2)
+    lp_args = F.spmv_args(wl.d_y, wl.d_rowptr, wl.d_col, wl.d_val, wl.d_x)
+    hp_args = F.stencil_args(wl.d_out, wl.d_in)
+    lp_grid, hp_grid = F.spmv_grid(SPMV_ROWS), F.stencil_grid(STENCIL_N)
+    k_clc = rt.register_kernel(F.BODY_SPMV_CSR_F32, poll=1, clc=True, name="spmv_clc")
+    k_ctr = rt.register_kernel(F.BODY_SPMV_CSR_F32, chunk=1, poll=1, name="spmv")
+    k_hp = rt.register_kernel(F.BODY_STENCIL5_F32, chunk=4, poll=1, name="stencil")
+    variants = [("clc_no_request", k_clc, False), ("counter_flep_request", k_ctr, True),
+                ("counter_no_request", k_ctr, False)]
+    res = {v[0]: {"hp_turnaround": [], "lp_span": [], "yields": []} for v in variants}
+
+    def spin_us(us):
+        t0 = time.perf_counter()
+        while time.perf_counter() - t0 < us * 1e-6:
+            pass
+    with ClockSampler(physical_gpu_index(local)) as clk:
+        for i in range(args.warmup + args.steps):
+            for name, k_lp, request in variants:
+                with torch.cuda.stream(lo):
+                    flush.zero_()
+                torch.cuda.synchronize()
+                h = rt.launch(k_lp, lp_grid, lp_args, priority=0, stream=lo)
+                spin_us(20)
+                if request:
+                    rt.preempt(h, rt.num_sms)
+                h2 = rt.launch(k_hp, hp_grid, hp_args, priority=1, stream=hi)
+                rt.sync(h2, timeout_ns=10_000_000_000)
+                if request:
+                    rt.wait_epoch(h, timeout_ns=10_000_000_000)
+                    if rt.query(h).state == F.STATE_PREEMPTED:
+                        rt.resume(h)
+                rt.sync(h, timeout_ns=10_000_000_000)
+                torch.cuda.synchronize()
+                if i < args.warmup:
+                    continue
+                lp_ev = rt.events(h, 1)
+                gen_now = max(e.epoch for e in lp_ev)    # stale slots of cancelled CTAs keep older gens
+                lp_ev = [e for e in lp_ev if e.epoch == gen_now]
+                lp0 = min(e.t_entry for e in lp_ev)
+                hp_ev = rt.events(h2, 1)
+                hp1 = max(e.t_exit for e in hp_ev)
+                q = rt.query(h)
+                lp_end = max(max(e.t_exit for e in lp_ev),
+                             max((e.t_exit for e in rt.events(h, q.epoch)), default=0))
+                r = res[name]
+                r["hp_turnaround"].append((hp1 - lp0) / 1e3)
+                r["lp_span"].append((lp_end - lp0) / 1e3)
+                r["yields"].append(sum(1 for e in lp_ev if e.reason == F.REASON_YIELD))
+    parity = spot_parity(wl, torch)
+    reps = max(args.reps, 20)
+
+    def timed(fn):
+        ts = []
+        for r in range(reps + 2):
+            with torch.cuda.stream(lo):
+                flush.zero_()
+                dither(torch)
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record(lo)
+            h = fn()
+            e1.record(lo)
+            e1.synchronize()
+            if h is not None:
+                rt.sync(h)
+            if r >= 2:
+                ts.append(e0.elapsed_time(e1) * 1e3)
+        return round(event_mean_us(ts), 3)
+    over = {}
+    n_sx = 1 << 20
+    xs = torch.randint(-2 ** 31, 2 ** 31 - 1, (n_sx,), dtype=torch.int32, device="cuda")
+    ys = torch.randint(-2 ** 31, 2 ** 31 - 1, (n_sx,), dtype=torch.int32, device="cuda")
+    cases = [("spmv", F.BODY_SPMV_CSR_F32, lp_grid, lp_args, dict(chunk=2, poll=2)),
+             ("stencil", F.BODY_STENCIL5_F32, hp_grid, hp_args, dict(chunk=4, poll=1)),
+             ("saxpy_i32_2^20", F.BODY_SAXPY_I32, F.saxpy_grid(n_sx), F.saxpy_i32_args(ys, xs, 3),
+              dict(chunk=16, poll=2, prefetch=True, async_poll=True))]
+    for name, body, grid, a, ckw in cases:
+        k_c = rt.register_kernel(body, poll=4, clc=True)
+        k_a = rt.register_kernel(body, **ckw)
+        t_u = timed(lambda: rt.launch_unwrapped(body, grid, a, stream=lo))
+        t_c = timed(lambda: rt.launch(k_c, grid, a, stream=lo))
+        t_a = timed(lambda: rt.launch(k_a, grid, a, stream=lo))
+        over[name] = {"unwrapped_us": t_u, "clc_us": t_c, "counter_us": t_a, "clc_poll": 4,
+                      "counter_config": ckw, "clc_overhead_pct": round((t_c / t_u - 1) * 100, 2),
+                      "counter_overhead_pct": round((t_a / t_u - 1) * 100, 2)}
+    rt.close()
+
+    def q(v, p):
+        return round(float(np.percentile(v, p)), 3) if v else None
+    summ = {k: {"hp_turnaround_us": {"p50": q(r["hp_turnaround"], 50), "p99": q(r["hp_turnaround"], 99)},
+                "lp_span_us": {"p50": q(r["lp_span"], 50)},
+                "first_wave_yield_exits_p50": q(r["yields"], 50)} for k, r in res.items()}
+    out = {"metric": METRIC, "value": summ["clc_no_request"]["hp_turnaround_us"]["p50"], "unit": "us",
+           "value_definition": "HP turnaround (HP last CTA exit - LP first CTA entry, device %globaltimer) with a CLC "
+                               "victim and no preemption request, p50; the HP is released ~20 us after the LP",
+           "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "higher_is_better": False,
+           "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic (seeded; synth/gen.py)",
+           "config": {"workload": "configs[1] kernels: LP SpMV-CSR 2^20 rows (low-priority stream) and HP stencil5 "
+                                  "4096^2 (high-priority stream, host-released ~20 us after the LP)",
+                      "l2": "flushed before every step"},
+           "variants": summ, "wrapper_overhead": over, "parity": parity, "clocks": clk.summary()}
+    if rank == 0:
+        print(json.dumps(out), flush=True)
+    barrier(world)
+
+
 # ------------------------------------------------------------------------------------------
 def assign_jobs(jobs, t_e_of, world):
     """One job queue feeding `world` independent per-GPU schedulers (configs[4]): each arrival

@@ -147,6 +147,15 @@ typedef struct {
    chunk later. For throughput-oriented kernels (with FLEP_KFLAG_PREFETCH the scheduling step then
    waits on nothing). */
 #define FLEP_KFLAG_ASYNC_POLL 8u
+/* CLC task fetch (R25; memory-bound bodies only, not GEMM): the launch runs
+   the original grid of N CTAs; a running CTA runs its own block and then takes pending CTAs'
+   blocks by cancelling them with the hardware's cluster launch control (try_cancel) instead of
+   an atomic counter. flep_preempt makes the named workers stop taking blocks at their next poll
+   (every K blocks) and leave; the rest of the grid waits in the hardware queue, where
+   higher-priority streams are served first. The launch goes to PREEMPTED (temporal) or PARTIAL
+   (spatial) at once; flep_resume withdraws the request (no relaunch); completion is the grid's
+   completion. The chunk C is 1; the worker event log covers the first W CTAs. */
+#define FLEP_KFLAG_CLC 16u
 
 typedef enum {
   FLEP_STATE_QUEUED = 0,     /* intercepted, waiting for a scheduling decision (S2) */

@@ -422,6 +422,99 @@ flep_worker(const __grid_constant__ typename Body::Args args, const WorkerParams
   }
 }
 
+// ---- CLC task fetch (reading R25) ----------------------------------------------
+// The same preemptable persistent form with the B200's cluster launch control instead of the
+// global counter: the grid is the original one (N CTAs, one per original block) and the work
+// queue is the hardware's queue of not-yet-launched CTAs. A running CTA runs its own block, then
+// asks the hardware to cancel a pending CTA (clusterlaunchcontrol.try_cancel) and runs that
+// CTA's block instead, until no CTA is left. Each original block therefore runs exactly once by
+// construction (launched and run by itself, or cancelled once and run by the canceller), with
+// no counter and no exit accounting.
+// Preemption withdraws the persistence: at a poll point a worker named by the request (temporal,
+// or rank[smid] < n) stops cancelling and leaves after the block it holds (A4: a cancelled CTA's
+// block is always run). The rest of the grid stays in the hardware queue, where the CTA scheduler
+// serves higher-priority streams first, so the waiting kernel gets the released SMs; an LP CTA
+// that the hardware still launches meanwhile runs its one block and leaves again. Resume only
+// clears the request: no relaunch, and the grid's completion is the launch's completion.
+__device__ __forceinline__ void clc_try_cancel(uint32_t resp, uint32_t mbar) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], 16;" :: "r"(mbar) : "memory");
+  asm volatile("clusterlaunchcontrol.try_cancel.async.shared::cta.mbarrier::complete_tx::bytes.b128 [%0], [%1];"
+               :: "r"(resp), "r"(mbar) : "memory");
+}
+// Waits for the response; returns the cancelled CTA's x index, or 0xffffffff if none was left.
+__device__ __forceinline__ uint32_t clc_response(uint32_t resp, uint32_t mbar, uint32_t phase) {
+  uint32_t done = 0;
+  while (!done)
+    asm volatile("{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
+                 : "=r"(done) : "r"(mbar), "r"(phase) : "memory");
+  uint32_t ok, x;
+  asm volatile("{ .reg .pred p; .reg .b128 q; ld.shared.b128 q, [%2];"
+               " clusterlaunchcontrol.query_cancel.is_canceled.pred.b128 p, q; selp.u32 %0, 1, 0, p;"
+               " @p clusterlaunchcontrol.query_cancel.get_first_ctaid::x.b32.b128 %1, q; }"
+               : "=r"(ok), "=r"(x) : "r"(resp) : "memory");
+  return ok ? x : 0xffffffffu;
+}
+
+template <class Body, bool kCoverage>
+__global__ void __launch_bounds__(Body::kThreads, Body::kMinBlocks)
+flep_clc_worker(const __grid_constant__ typename Body::Args args, const WorkerParams p) {
+  __shared__ alignas(16) uint32_t s_resp[4];
+  __shared__ alignas(8) uint64_t s_mbar;
+  __shared__ uint32_t s_next[2];     // double-buffered broadcast: one barrier per block
+  __shared__ WorkerShared ws;
+  const uint32_t tid = threadIdx.x;
+  const uint32_t resp = static_cast<uint32_t>(__cvta_generic_to_shared(s_resp));
+  const uint32_t mbar = static_cast<uint32_t>(__cvta_generic_to_shared(&s_mbar));
+  if (tid == 0) {
+    ws.sm = smid_reg(); ws.t_entry = gtimer(); ws.blocks = 0; ws.reason = kReasonExhausted;
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" :: "r"(mbar) : "memory");
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  Body::setup(args);
+  uint32_t b = blockIdx.x;           // this CTA's own original block (launched by the hardware)
+  uint32_t k = 0, phase = 0, parity = 0;
+  while (true) {
+    bool pending = false;
+    if (tid == 0) {
+      // amortised poll (every K blocks) before asking for more work; a request that names this
+      // SM ends the persistence after the block in hand
+      bool stop = false;
+      if (++k == p.poll) {
+        k = 0;
+        stop = should_yield(ld_relaxed_gpu(p.ctrl), p, smid_reg());
+      }
+      if (!stop) { clc_try_cancel(resp, mbar); pending = true; }   // overlaps the body
+      else ws.reason = kReasonYield;
+      if (p.trigger_block == b) {                        // device self-trigger (test/bench hook)
+        const uint32_t e = p.epoch % kEvEpochs;
+        p.cb->ep_t_trigger[e] = gtimer();
+        p.cb->ep_trigger_block[e] = p.trigger_block;
+        atomicExch(p.ctrl, ((p.epoch & 0xffffu) << 16) | (p.trigger_n & 0xffffu));
+      }
+    }
+    Body::run(args, b, b + 1, p.gx, p.gy);
+    if (tid == 0) {
+      if (kCoverage) atomicAdd(&p.cov[b], 1u);
+      ws.blocks += 1;
+      uint32_t nb = 0xffffffffu;
+      if (pending) { nb = clc_response(resp, mbar, phase); phase ^= 1u; }   // a cancelled CTA's block is always run
+      s_next[parity] = nb;
+    }
+    __syncthreads();
+    b = s_next[parity];
+    parity ^= 1u;
+    if (b == 0xffffffffu) break;
+  }
+  Body::teardown(args);
+  // event log: the first W CTAs (the first wave, which does nearly all the work) record their exit
+  if (tid == 0 && blockIdx.x < p.workers) {
+    WorkerEvent& e = p.ev[(p.epoch % kEvEpochs) * p.workers + blockIdx.x];
+    e.smid = ws.sm; e.reason = ws.reason; e.n_blocks = ws.blocks; e.epoch = p.epoch;
+    e.t_entry = ws.t_entry; e.t_exit = gtimer();
+  }
+}
+
 // The original kernel (unwrapped twin, K7): one CTA per original block, same body.
 #ifdef FLEP_TRACE
 static __device__ uint64_t* g_unwrapped_trace;   // diagnostics build only: [N][2] entry/exit

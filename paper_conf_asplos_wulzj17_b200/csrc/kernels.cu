@@ -21,6 +21,12 @@ struct Ops {
     else flep_worker<Body, false><<<W, Body::kThreads, Body::kDynSmem, s>>>(a, p);
     return cudaGetLastError();
   }
+  static cudaError_t clc(const void* args, const WorkerParams& p, uint32_t N, cudaStream_t s, bool cov) {
+    const typename Body::Args& a = *reinterpret_cast<const typename Body::Args*>(args);
+    if (cov) flep_clc_worker<Body, true><<<N, Body::kThreads, Body::kDynSmem, s>>>(a, p);
+    else flep_clc_worker<Body, false><<<N, Body::kThreads, Body::kDynSmem, s>>>(a, p);
+    return cudaGetLastError();
+  }
   static cudaError_t unwrapped(const void* args, dim3 grid, uint32_t offset, uint32_t count,
                                cudaStream_t s) {
     const typename Body::Args& a = *reinterpret_cast<const typename Body::Args*>(args);
@@ -91,19 +97,19 @@ using StencilF32 = WithSmem<Stencil5Body<false>>;
 using StencilI32 = WithSmem<Stencil5Body<true>>;
 
 const BodyOps kOps[] = {
-    {0, 0, 0, nullptr, nullptr, nullptr, nullptr},
+    {0, 0, 0, nullptr, nullptr, nullptr, nullptr, nullptr},
     {FLEP_BODY_SAXPY_I32, SaxpyI32::kThreads, sizeof(flep_saxpy_i32_args), &Ops<SaxpyI32>::worker,
-     &Ops<SaxpyI32>::unwrapped, &Ops<SaxpyI32>::occupancy, nullptr},
+     &Ops<SaxpyI32>::unwrapped, &Ops<SaxpyI32>::occupancy, nullptr, &Ops<SaxpyI32>::clc},
     {FLEP_BODY_SAXPY_F32, SaxpyF32::kThreads, sizeof(flep_saxpy_f32_args), &Ops<SaxpyF32>::worker,
-     &Ops<SaxpyF32>::unwrapped, &Ops<SaxpyF32>::occupancy, nullptr},
+     &Ops<SaxpyF32>::unwrapped, &Ops<SaxpyF32>::occupancy, nullptr, &Ops<SaxpyF32>::clc},
     {FLEP_BODY_SPMV_CSR_F32, Spmv::kThreads, sizeof(flep_spmv_args), &Ops<Spmv>::worker,
-     &Ops<Spmv>::unwrapped, &Ops<Spmv>::occupancy, nullptr},
+     &Ops<Spmv>::unwrapped, &Ops<Spmv>::occupancy, nullptr, &Ops<Spmv>::clc},
     {FLEP_BODY_STENCIL5_F32, StencilF32::kThreads, sizeof(flep_stencil_args), &Ops<StencilF32>::worker,
-     &Ops<StencilF32>::unwrapped, &Ops<StencilF32>::occupancy, nullptr},
+     &Ops<StencilF32>::unwrapped, &Ops<StencilF32>::occupancy, nullptr, &Ops<StencilF32>::clc},
     {FLEP_BODY_STENCIL5_I32, StencilI32::kThreads, sizeof(flep_stencil_args), &Ops<StencilI32>::worker,
-     &Ops<StencilI32>::unwrapped, &Ops<StencilI32>::occupancy, nullptr},
+     &Ops<StencilI32>::unwrapped, &Ops<StencilI32>::occupancy, nullptr, &Ops<StencilI32>::clc},
     {FLEP_BODY_GEMM_BF16, GemmBody::kThreads, sizeof(flep_gemm_args), &gemm_worker_launch,
-     &gemm_unwrapped_launch, &gemm_occupancy, &gemm_validate},
+     &gemm_unwrapped_launch, &gemm_occupancy, &gemm_validate, nullptr},
 };
 
 }  // namespace

@@ -20,6 +20,9 @@ struct BodyOps {
   cudaError_t (*occupancy)(int* ctas_per_sm, bool cov);
   // optional argument / grid validation (nullptr = none); returns a static message or nullptr
   const char* (*validate)(const void* args, dim3 grid);
+  // launch the CLC variant (flep_clc_worker<Body>) over the original grid of N blocks (1-D);
+  // nullptr for bodies that own their loop (GEMM)
+  cudaError_t (*clc)(const void* args, const WorkerParams& p, uint32_t N, cudaStream_t s, bool cov);
 };
 
 const BodyOps* body_ops(int32_t body);

@@ -122,6 +122,7 @@ struct Launch {
   // kernel-slicing baseline (FLEP_POLICY_SLICE): the original kernel as sub-grids of
   // slice_blocks blocks, at most two in flight; a preemption stops issuing
   bool sliced = false;
+  bool clc = false;                  // FLEP_KFLAG_CLC: hardware work queue, resume = clear (R25)
   uint32_t slice_blocks = 0;
   uint64_t next_block = 0, slice_done = 0;
   std::deque<std::pair<cudaEvent_t, uint32_t>> inflight;
@@ -280,6 +281,14 @@ flep_status start_epoch(flep_rt rt, Launch& L) {
     mark_active(rt, L);
     return issue_slices(rt, L);
   }
+  if (L.clc && L.epoch > 0) {        // R25: resume withdraws the request; no relaunch
+    flep_status s = write_ctrl(rt, L, ctrl_word(L, 0));
+    if (s) return s;
+    L.state = FLEP_STATE_RUNNING;
+    L.n_yield = 0;
+    mark_active(rt, L);
+    return FLEP_OK;
+  }
   L.epoch++;
   WorkerParams p{};
   p.cb = L.cb;
@@ -310,7 +319,8 @@ flep_status start_epoch(flep_rt rt, Launch& L) {
 #endif
   L.trig_block = kNoTrigger;
   L.trig_n = 0;
-  cudaError_t e = L.ops->worker(L.args.data(), p, L.workers, L.exec, L.cov != nullptr);
+  cudaError_t e = L.clc ? L.ops->clc(L.args.data(), p, L.n_blocks, L.exec, L.cov != nullptr)
+                        : L.ops->worker(L.args.data(), p, L.workers, L.exec, L.cov != nullptr);
   if (e != cudaSuccess) return fail(FLEP_ERR_CUDA, "worker launch failed: %s", cudaGetErrorString(e));
   CUDA_TRY(cudaEventRecord(L.fin_ev, L.exec));
   L.state = FLEP_STATE_RUNNING;
@@ -322,7 +332,8 @@ flep_status start_epoch(flep_rt rt, Launch& L) {
 
 // Pull the pinned status slot; returns true if the launch's state changed to DONE.
 bool refresh(flep_rt rt, Launch& L) {
-  if (L.state != FLEP_STATE_RUNNING && L.state != FLEP_STATE_YIELDING && L.state != FLEP_STATE_PARTIAL)
+  if (L.state != FLEP_STATE_RUNNING && L.state != FLEP_STATE_YIELDING && L.state != FLEP_STATE_PARTIAL &&
+      !(L.clc && L.state == FLEP_STATE_PREEMPTED))   // a preempted CLC grid still completes (R25)
     return false;
   if (L.sliced) {
     while (!L.inflight.empty() && cudaEventQuery(L.inflight.front().first) == cudaSuccess) {
@@ -408,6 +419,10 @@ void apply_decisions(flep_rt rt) {
         write_ctrl(rt, L, ctrl_word(L, (uint32_t)std::min<int64_t>(x.n_sms, 0xffff)));
         L.state = FLEP_STATE_YIELDING;
         L.n_yield = (uint32_t)x.n_sms;
+        if (L.clc) {                     // R25: no drain to wait for; the request is in force
+          L.t_last_request = now_ns();
+          L.state = x.n_sms >= rt->num_sms ? FLEP_STATE_PREEMPTED : FLEP_STATE_PARTIAL;
+        }
       }
     } else {
       if (L.state == FLEP_STATE_DONE) continue;   // finished while draining; FINISH pending
@@ -423,7 +438,8 @@ void monitor_pass(flep_rt rt) {
     Launch* Lp = find(rt, id);
     if (!Lp) continue;
     Launch& L = *Lp;
-    if (L.state != FLEP_STATE_RUNNING && L.state != FLEP_STATE_YIELDING && L.state != FLEP_STATE_PARTIAL) continue;
+    if (L.state != FLEP_STATE_RUNNING && L.state != FLEP_STATE_YIELDING && L.state != FLEP_STATE_PARTIAL &&
+        !(L.clc && L.state == FLEP_STATE_PREEMPTED)) continue;
     if (refresh(rt, L)) {
       rt->to_release.push_back(L.id);
       const int64_t t = L.t_finish;
@@ -528,7 +544,7 @@ void monitor_loop(flep_rt rt) {
       const uint64_t* wp = reinterpret_cast<const uint64_t*>(&L->hs->word);
       auto it = snap.find(id);
       const bool running = L->state == FLEP_STATE_RUNNING || L->state == FLEP_STATE_YIELDING ||
-                           L->state == FLEP_STATE_PARTIAL;
+                           L->state == FLEP_STATE_PARTIAL || (L->clc && L->state == FLEP_STATE_PREEMPTED);
       watch.push_back({wp, it != snap.end() ? it->second : ~0ull, L->sliced, id,
                        (running && !L->sliced) ? L->fin_ev : nullptr});
     }
@@ -700,6 +716,12 @@ flep_status flep_launch(flep_rt rt, flep_kernel kid, flep_dim3 grid, const void*
   L.chunk = kr.chunk;
   L.poll = kr.poll;
   L.flags = kr.flags;
+  if (kr.flags & FLEP_KFLAG_CLC) {
+    if (!ops->clc) return fail(FLEP_ERR_UNSUPPORTED, "body %d has no CLC variant", kr.body);
+    if (rt->opt.policy == FLEP_POLICY_SLICE) return fail(FLEP_ERR_UNSUPPORTED, "CLC kernels cannot be sliced");
+    L.clc = true;
+    L.chunk = 1;                                     // one original block per cancelled CTA
+  }
   if (kr.ctas_per_sm && (int)kr.ctas_per_sm < k) k = (int)kr.ctas_per_sm;
   const uint64_t wmax = (uint64_t)k * rt->num_sms;
   const uint64_t need = (N + L.chunk - 1) / L.chunk;
@@ -807,6 +829,7 @@ flep_status flep_preempt(flep_rt rt, flep_launch_t h, uint32_t n_sms) {
   if (s) return s;
   L->n_yield = n;
   L->state = n >= rt->num_sms ? FLEP_STATE_YIELDING : FLEP_STATE_PARTIAL;
+  if (L->clc && n >= rt->num_sms) L->state = FLEP_STATE_PREEMPTED;   // R25: in force at once
   return FLEP_OK;
 }
 
