@@ -204,11 +204,12 @@ def run_temporal(args, rank, world, local):
     num_sms = rt.num_sms
     kLP = rt.register_kernel(F.BODY_SPMV_CSR_F32, chunk=args.lp_chunk, poll=args.lp_poll, name="spmv",
                              prefetch=bool(args.prefetch))
-    # the waiting (high-priority) kernel is never preempted here: its chunking is tuned for
-    # throughput (C = 4, the tuned choice of tools/overhead_breakdown.py), the victim's for
-    # latency (C = K = 1)
-    kHP = rt.register_kernel(F.BODY_STENCIL5_F32, chunk=args.hp_chunk, poll=1, name="stencil",
-                             prefetch=bool(args.hp_prefetch), async_poll=bool(args.hp_async))
+    # the waiting (high-priority) kernel is never preempted here: it is tuned for throughput (CLC
+    # task fetch, C = 1, K = 4: 4.6 % over the unwrapped grid vs 19 % for the counter worker,
+    # profiles/r01_bench_clc.json), the victim for latency (atomic counter, C = K = 1)
+    kHP = rt.register_kernel(F.BODY_STENCIL5_F32, chunk=args.hp_chunk, poll=args.hp_poll, name="stencil",
+                             prefetch=bool(args.hp_prefetch), async_poll=bool(args.hp_async),
+                             clc=bool(args.hp_clc))
     lp_args = F.spmv_args(wl.d_y, wl.d_rowptr, wl.d_col, wl.d_val, wl.d_x)
     hp_args = F.stencil_args(wl.d_out, wl.d_in)
     lp_grid, hp_grid = F.spmv_grid(SPMV_ROWS), F.stencil_grid(STENCIL_N)
@@ -313,7 +314,7 @@ def run_temporal(args, rank, world, local):
         "data": "synthetic (seeded; synth/gen.py)",
         "config": {"workload": "configs[1]: full-GPU temporal preemption of SpMV-CSR fp32 (2^20 rows, "
                                f"{wl.nnz} nnz, low priority) by stencil5 fp32 4096^2 (high priority)",
-                   "lp_chunk": args.lp_chunk, "lp_poll": args.lp_poll, "hp_chunk": args.hp_chunk, "hp_poll": 1, "hp_prefetch": bool(args.hp_prefetch),
+                   "lp_chunk": args.lp_chunk, "lp_poll": args.lp_poll, "hp_chunk": args.hp_chunk, "hp_poll": args.hp_poll, "hp_clc": bool(args.hp_clc), "hp_prefetch": bool(args.hp_prefetch),
                    "hp_async_poll": bool(args.hp_async),
                    "prefetch": bool(args.prefetch),
                    "flag": "stream_memop (device self-trigger for the request)",
@@ -415,8 +416,9 @@ def run_e2e(F, torch, wl, local, steps, args):
     rt = F.Runtime(device=local, policy=F.POLICY_HPF)
     kLP = rt.register_kernel(F.BODY_SPMV_CSR_F32, chunk=args.lp_chunk, poll=args.lp_poll, name="spmv",
                              model=(0, 0, 0, 0, 70_000), prefetch=bool(args.prefetch), started_hint=True)
-    kHP = rt.register_kernel(F.BODY_STENCIL5_F32, chunk=args.hp_chunk, poll=1, name="stencil",
-                             model=(0, 0, 0, 0, 30_000), prefetch=bool(args.hp_prefetch), async_poll=bool(args.hp_async))
+    kHP = rt.register_kernel(F.BODY_STENCIL5_F32, chunk=args.hp_chunk, poll=args.hp_poll, name="stencil",
+                             model=(0, 0, 0, 0, 30_000), prefetch=bool(args.hp_prefetch), async_poll=bool(args.hp_async),
+                             clc=bool(args.hp_clc))
     pin = lambda a: torch.from_numpy(np.ascontiguousarray(a)).pin_memory()  # noqa: E731
     h_rp, h_col, h_val, h_x, h_in = pin(wl.rowptr), pin(wl.col), pin(wl.val), pin(wl.x), pin(wl.st_in)
     h_y = torch.empty(SPMV_ROWS, dtype=torch.float32).pin_memory()
@@ -538,7 +540,9 @@ def main():
     ap.add_argument("--rho", type=float, default=1.0)
     ap.add_argument("--lp-chunk", type=int, default=1)
     ap.add_argument("--prefetch", type=int, default=0)
-    ap.add_argument("--hp-chunk", type=int, default=4)
+    ap.add_argument("--hp-chunk", type=int, default=1)
+    ap.add_argument("--hp-poll", type=int, default=4)
+    ap.add_argument("--hp-clc", type=int, default=1, help="waiting kernel: CLC task fetch (R25)")
     ap.add_argument("--hp-prefetch", type=int, default=0)
     ap.add_argument("--hp-async", type=int, default=0, help="waiting kernel: async poll (R22)")
     ap.add_argument("--lp-poll", type=int, default=1)

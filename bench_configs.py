@@ -361,7 +361,7 @@ def run_clc(args, rank, world, local):
     lp_args = F.spmv_args(wl.d_y, wl.d_rowptr, wl.d_col, wl.d_val, wl.d_x)
     hp_args = F.stencil_args(wl.d_out, wl.d_in)
     lp_grid, hp_grid = F.spmv_grid(SPMV_ROWS), F.stencil_grid(STENCIL_N)
-    k_clc = rt.register_kernel(F.BODY_SPMV_CSR_F32, poll=1, clc=True, name="spmv_clc")
+    k_clc = rt.register_kernel(F.BODY_SPMV_CSR_F32, chunk=1, poll=1, clc=True, name="spmv_clc")
     k_ctr = rt.register_kernel(F.BODY_SPMV_CSR_F32, chunk=1, poll=1, name="spmv")
     k_hp = rt.register_kernel(F.BODY_STENCIL5_F32, chunk=4, poll=1, name="stencil")
     variants = [("clc_no_request", k_clc, False), ("counter_flep_request", k_ctr, True),
@@ -428,17 +428,17 @@ def run_clc(args, rank, world, local):
     n_sx = 1 << 20
     xs = torch.randint(-2 ** 31, 2 ** 31 - 1, (n_sx,), dtype=torch.int32, device="cuda")
     ys = torch.randint(-2 ** 31, 2 ** 31 - 1, (n_sx,), dtype=torch.int32, device="cuda")
-    cases = [("spmv", F.BODY_SPMV_CSR_F32, lp_grid, lp_args, dict(chunk=2, poll=2)),
-             ("stencil", F.BODY_STENCIL5_F32, hp_grid, hp_args, dict(chunk=4, poll=1)),
+    cases = [("spmv", F.BODY_SPMV_CSR_F32, lp_grid, lp_args, dict(chunk=2, poll=2), dict(chunk=2, poll=2)),
+             ("stencil", F.BODY_STENCIL5_F32, hp_grid, hp_args, dict(chunk=4, poll=1), dict(chunk=1, poll=4)),
              ("saxpy_i32_2^20", F.BODY_SAXPY_I32, F.saxpy_grid(n_sx), F.saxpy_i32_args(ys, xs, 3),
-              dict(chunk=16, poll=2, prefetch=True, async_poll=True))]
-    for name, body, grid, a, ckw in cases:
-        k_c = rt.register_kernel(body, poll=4, clc=True)
+              dict(chunk=16, poll=2, prefetch=True, async_poll=True), dict(chunk=8, poll=2))]
+    for name, body, grid, a, ckw, clkw in cases:
+        k_c = rt.register_kernel(body, clc=True, **clkw)
         k_a = rt.register_kernel(body, **ckw)
         t_u = timed(lambda: rt.launch_unwrapped(body, grid, a, stream=lo))
         t_c = timed(lambda: rt.launch(k_c, grid, a, stream=lo))
         t_a = timed(lambda: rt.launch(k_a, grid, a, stream=lo))
-        over[name] = {"unwrapped_us": t_u, "clc_us": t_c, "counter_us": t_a, "clc_poll": 4,
+        over[name] = {"unwrapped_us": t_u, "clc_us": t_c, "counter_us": t_a, "clc_config": clkw,
                       "counter_config": ckw, "clc_overhead_pct": round((t_c / t_u - 1) * 100, 2),
                       "counter_overhead_pct": round((t_a / t_u - 1) * 100, 2)}
     rt.close()

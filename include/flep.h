@@ -148,13 +148,13 @@ typedef struct {
    waits on nothing). */
 #define FLEP_KFLAG_ASYNC_POLL 8u
 /* CLC task fetch (R25; memory-bound bodies only, not GEMM): the launch runs
-   the original grid of N CTAs; a running CTA runs its own block and then takes pending CTAs'
-   blocks by cancelling them with the hardware's cluster launch control (try_cancel) instead of
+   the original grid in chunks (ceil(N/C) CTAs, CTA i = original blocks [iC, iC+C)); a running CTA
+   runs its own chunk and then takes pending CTAs' chunks by cancelling them with the hardware's cluster launch control (try_cancel) instead of
    an atomic counter. flep_preempt makes the named workers stop taking blocks at their next poll
    (every K blocks) and leave; the rest of the grid waits in the hardware queue, where
    higher-priority streams are served first. The launch goes to PREEMPTED (temporal) or PARTIAL
    (spatial) at once; flep_resume withdraws the request (no relaunch); completion is the grid's
-   completion. The chunk C is 1; the worker event log covers the first W CTAs. */
+   completion. The worker event log covers the first W CTAs. */
 #define FLEP_KFLAG_CLC 16u
 
 typedef enum {
@@ -260,15 +260,18 @@ flep_status flep_debug_trigger_at(flep_rt rt, flep_launch_t h, uint64_t block_in
 flep_status flep_debug_arm_next_trigger(flep_rt rt, uint64_t block_index, uint32_t n_sms);
 /* Copy cov[0..n) (debug_coverage runtimes only). */
 flep_status flep_debug_copy_coverage(flep_rt rt, flep_launch_t h, uint32_t* host_out, size_t n);
-/* Copy the worker event records of epoch `epoch` (1-based; the last 8 epochs are kept). */
+/* Copy the worker event records of epoch `epoch` (1-based; the last 8 epochs are kept): up to
+   max_records records written in that epoch, compacted to the front of host_out; *n_out = their
+   number (a CLC launch logs the first W CTAs of its grid that ran, R25). */
 flep_status flep_debug_copy_events(flep_rt rt, flep_launch_t h, uint32_t epoch,
                                    flep_worker_event* host_out, size_t max_records,
                                    size_t* n_out);
 flep_status flep_debug_epoch_info(flep_rt rt, flep_launch_t h, uint32_t epoch,
                                   flep_epoch_info* out);
 /* Diagnostics builds (-DFLEP_TRACE) only, else FLEP_ERR_UNSUPPORTED: record per-chunk scheduling
-   timestamps of worker grids (device buffer [W][64][2] u64: tid 0 reaches the scheduling step,
-   the step returns) and entry/exit of every block of unwrapped grids ([N][2] u64). Buffers are
+   timestamps of worker grids (device buffer [W][64][5] u64: tid 0 reaches the scheduling step,
+   the poll decision, the step returns, the chunk barrier releases, the chunk base is known) and
+   entry/exit of every block of unwrapped grids ([N][2] u64). Buffers are
    the caller's; NULL disables. */
 flep_status flep_debug_set_trace(flep_rt rt, void* worker_trace, void* unwrapped_trace);
 /* Set the spatial rank table: rank[smid] for smid < nsmid (default rank = smid). */

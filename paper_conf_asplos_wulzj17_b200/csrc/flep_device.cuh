@@ -424,8 +424,8 @@ flep_worker(const __grid_constant__ typename Body::Args args, const WorkerParams
 
 // ---- CLC task fetch (reading R25) ----------------------------------------------
 // The same preemptable persistent form with the B200's cluster launch control instead of the
-// global counter: the grid is the original one (N CTAs, one per original block) and the work
-// queue is the hardware's queue of not-yet-launched CTAs. A running CTA runs its own block, then
+// global counter: the grid is the original one in chunks (ceil(N/C) CTAs, CTA i = original blocks
+// [i*C, i*C + C)) and the work queue is the hardware's queue of not-yet-launched CTAs. A running CTA runs its own block, then
 // asks the hardware to cancel a pending CTA (clusterlaunchcontrol.try_cancel) and runs that
 // CTA's block instead, until no CTA is left. Each original block therefore runs exactly once by
 // construction (launched and run by itself, or cancelled once and run by the canceller), with
@@ -472,7 +472,9 @@ flep_clc_worker(const __grid_constant__ typename Body::Args args, const WorkerPa
   }
   __syncthreads();
   Body::setup(args);
-  uint32_t b = blockIdx.x;           // this CTA's own original block (launched by the hardware)
+  // CTA i of the CLC grid stands for the chunk of original blocks [i*C, i*C + C) (R25); it starts
+  // on its own chunk (launched by the hardware)
+  uint32_t b = blockIdx.x;
   uint32_t k = 0, phase = 0, parity = 0;
   while (true) {
     bool pending = false;
@@ -486,19 +488,21 @@ flep_clc_worker(const __grid_constant__ typename Body::Args args, const WorkerPa
       }
       if (!stop) { clc_try_cancel(resp, mbar); pending = true; }   // overlaps the body
       else ws.reason = kReasonYield;
-      if (p.trigger_block == b) {                        // device self-trigger (test/bench hook)
+      if (p.trigger_block - b * p.chunk < p.chunk) {     // device self-trigger (test/bench hook)
         const uint32_t e = p.epoch % kEvEpochs;
         p.cb->ep_t_trigger[e] = gtimer();
         p.cb->ep_trigger_block[e] = p.trigger_block;
         atomicExch(p.ctrl, ((p.epoch & 0xffffu) << 16) | (p.trigger_n & 0xffffu));
       }
     }
-    Body::run(args, b, b + 1, p.gx, p.gy);
+    const uint32_t b0 = b * p.chunk, b1 = min(b0 + p.chunk, p.n_blocks);
+    Body::run(args, b0, b1, p.gx, p.gy);
     if (tid == 0) {
-      if (kCoverage) atomicAdd(&p.cov[b], 1u);
-      ws.blocks += 1;
+      if (kCoverage)
+        for (uint32_t bb = b0; bb < b1; ++bb) atomicAdd(&p.cov[bb], 1u);
+      ws.blocks += b1 - b0;
       uint32_t nb = 0xffffffffu;
-      if (pending) { nb = clc_response(resp, mbar, phase); phase ^= 1u; }   // a cancelled CTA's block is always run
+      if (pending) { nb = clc_response(resp, mbar, phase); phase ^= 1u; }   // a cancelled CTA's chunk is always run
       s_next[parity] = nb;
     }
     __syncthreads();

@@ -319,7 +319,7 @@ flep_status start_epoch(flep_rt rt, Launch& L) {
 #endif
   L.trig_block = kNoTrigger;
   L.trig_n = 0;
-  cudaError_t e = L.clc ? L.ops->clc(L.args.data(), p, L.n_blocks, L.exec, L.cov != nullptr)
+  cudaError_t e = L.clc ? L.ops->clc(L.args.data(), p, (L.n_blocks + L.chunk - 1) / L.chunk, L.exec, L.cov != nullptr)
                         : L.ops->worker(L.args.data(), p, L.workers, L.exec, L.cov != nullptr);
   if (e != cudaSuccess) return fail(FLEP_ERR_CUDA, "worker launch failed: %s", cudaGetErrorString(e));
   CUDA_TRY(cudaEventRecord(L.fin_ev, L.exec));
@@ -719,8 +719,7 @@ flep_status flep_launch(flep_rt rt, flep_kernel kid, flep_dim3 grid, const void*
   if (kr.flags & FLEP_KFLAG_CLC) {
     if (!ops->clc) return fail(FLEP_ERR_UNSUPPORTED, "body %d has no CLC variant", kr.body);
     if (rt->opt.policy == FLEP_POLICY_SLICE) return fail(FLEP_ERR_UNSUPPORTED, "CLC kernels cannot be sliced");
-    L.clc = true;
-    L.chunk = 1;                                     // one original block per cancelled CTA
+    L.clc = true;                                    // CTA i of the CLC grid = chunk i (C blocks)
   }
   if (kr.ctas_per_sm && (int)kr.ctas_per_sm < k) k = (int)kr.ctas_per_sm;
   const uint64_t wmax = (uint64_t)k * rt->num_sms;
@@ -1111,7 +1110,14 @@ flep_status flep_debug_copy_events(flep_rt rt, flep_launch_t h, uint32_t epoch,
   CUDA_TRY(cudaMemcpyAsync(host_out, L->ev + (size_t)((L->gen0 + epoch) % kEvEpochs) * L->workers,
                            n * sizeof(WorkerEvent), cudaMemcpyDeviceToHost, L->exec));
   CUDA_TRY(cudaStreamSynchronize(L->exec));
-  if (n_out) *n_out = n;
+  // keep only this epoch's records: a slot nobody wrote in this epoch (a CLC CTA that was
+  // cancelled, R25) still holds an older generation's record
+  const uint32_t gen = L->gen0 + epoch;
+  WorkerEvent* r = reinterpret_cast<WorkerEvent*>(host_out);
+  size_t m = 0;
+  for (size_t i = 0; i < n; ++i)
+    if (r[i].epoch == gen) r[m++] = r[i];
+  if (n_out) *n_out = m;
   return FLEP_OK;
 }
 

@@ -39,11 +39,12 @@ def _rel_err(got, ref, denom):
 
 
 @pytest.mark.parametrize("n", [1, 255, 4099, (1 << 20) + 3])
-@pytest.mark.parametrize("poll", [1, 4])
-def test_clc_saxpy_i32_exact(rt, torch_mod, n, poll):
+@pytest.mark.parametrize("chunk,poll", [(1, 1), (1, 4), (3, 1), (16, 2)])
+def test_clc_saxpy_i32_exact(rt, torch_mod, n, chunk, poll):
+    # CTA i of the CLC grid = original blocks [iC, iC+C); ragged last chunk when C does not divide N
     f = flep_mod()
     x, y = gen.saxpy_i32_inputs(n, seed=31)
-    k = rt.register_kernel(f.BODY_SAXPY_I32, poll=poll, clc=True)
+    k = rt.register_kernel(f.BODY_SAXPY_I32, chunk=chunk, poll=poll, clc=True)
     xd, yd = t(x), t(y)
     h = rt.launch(k, f.saxpy_grid(n), f.saxpy_i32_args(yd, xd, 1664525))
     rt.sync(h, timeout_ns=10_000_000_000)
@@ -58,7 +59,7 @@ def test_clc_stencil_exact(rt, torch_mod, n, integer):
     f = flep_mod()
     a = gen.stencil_i32_input(n, seed=32) if integer else gen.stencil_f32_input(n, seed=32)
     body = f.BODY_STENCIL5_I32 if integer else f.BODY_STENCIL5_F32
-    k = rt.register_kernel(body, poll=1, clc=True)
+    k = rt.register_kernel(body, chunk=1, poll=1, clc=True)
     ind = t(a)
     outd = torch_mod.empty_like(ind)
     h = rt.launch(k, f.stencil_grid(n), f.stencil_args(outd, ind))
@@ -81,7 +82,7 @@ def test_clc_spmv_matches_counter_variant_bitwise(rt, torch_mod):
     y0 = torch_mod.zeros(rows, device="cuda")
     y1 = torch_mod.zeros(rows, device="cuda")
     k0 = rt.register_kernel(f.BODY_SPMV_CSR_F32, chunk=2, poll=1)
-    k1 = rt.register_kernel(f.BODY_SPMV_CSR_F32, poll=2, clc=True)
+    k1 = rt.register_kernel(f.BODY_SPMV_CSR_F32, chunk=3, poll=2, clc=True)
     for k, y in ((k0, y0), (k1, y1)):
         h = rt.launch(k, f.spmv_grid(rows), f.spmv_args(y, *args_in))
         rt.sync(h, timeout_ns=10_000_000_000)
@@ -94,7 +95,7 @@ def test_clc_spmv_matches_counter_variant_bitwise(rt, torch_mod):
 def _long_lp(rt, f, n_log2=27, seed=34, **kw):
     n = 1 << n_log2
     x, y = gen.saxpy_i32_inputs(n, seed=seed)
-    k = rt.register_kernel(f.BODY_SAXPY_I32, poll=1, clc=True, **kw)
+    k = rt.register_kernel(f.BODY_SAXPY_I32, chunk=kw.pop("chunk", 4), poll=1, clc=True, **kw)
     return n, x, y, k
 
 
@@ -180,7 +181,7 @@ def test_clc_managed_hpf(torch_mod):
         x, y = gen.saxpy_i32_inputs(n_lp, seed=38)
         x2, y2 = gen.saxpy_i32_inputs(n_hp, seed=39)
         xd, yd, x2d, y2d = t(x), t(y), t(x2), t(y2)
-        k_lp = rt.register_kernel(f.BODY_SAXPY_I32, poll=1, clc=True, model=(0, 0, 0, 0, 2_000_000))
+        k_lp = rt.register_kernel(f.BODY_SAXPY_I32, chunk=4, poll=1, clc=True, model=(0, 0, 0, 0, 2_000_000))
         k_hp = rt.register_kernel(f.BODY_SAXPY_I32, chunk=1, poll=1, model=(0, 0, 0, 0, 5_000))
         sA, sB = torch_mod.cuda.Stream(), torch_mod.cuda.Stream()
         h_lp = rt.launch(k_lp, f.saxpy_grid(n_lp), f.saxpy_i32_args(yd, xd, 7), priority=0, stream=sA)
