@@ -292,6 +292,15 @@ def run_temporal(args, rank, world, local):
     algo = wl.spmv_bytes if dom == "spmv" else wl.st_bytes
     achieved = algo / (kern[dom]["wrapped_us"] * 1e-6) / 1e9
     prof_traffic = load_traffic(dom)
+    # The SpMV's algorithmic bytes stream at a fraction of HBM speed because its x[col[p]] gathers
+    # are random 4-B reads of an L2-resident vector: one 32-B sector request per nonzero. Its real
+    # ceiling is the measured random-gather rate (probes/probe6.cu: same x size and nnz).
+    gpk = load_gather_peak()
+    g_ach = wl.nnz / (kern["spmv"]["wrapped_us"] * 1e-6)
+    gather_roofline = {"bound": "l1_gather", "kernel": "flep_worker<spmv>", "achieved": float(f"{g_ach:.4g}"),
+                       "peak": gpk, "unit": "gathers/s", "frac": round(g_ach / gpk, 4) if gpk else None,
+                       "unwrapped_frac": round(wl.nnz / (kern["spmv"]["unwrapped_us"] * 1e-6) / gpk, 4) if gpk else None,
+                       "peak_source": "measured: probes/probe6.cu (profiles/r01_probe_gather_ceiling.jsonl)"}
     roofline = {"bound": "hbm", "achieved": round(achieved, 1), "peak": hbm, "unit": "GB/s",
                 "frac": round(achieved / hbm, 4), "traffic": prof_traffic, "kernel": f"flep_worker<{dom}>",
                 "algorithmic_bytes": algo, "peak_source": peak_src}
@@ -331,6 +340,7 @@ def run_temporal(args, rank, world, local):
         "wrapper_overhead_pct": {k: v["overhead_pct"] for k, v in kern.items()},
         "kernels": kern,
         "roofline": roofline,
+        "gather_roofline": gather_roofline,
         "e2e": e2e,
         "gpu_launches": int(sum(r["launches"] for r in res)),
         "hp_started_before_request": int(sum(1 for r in res if r["hp_started_early"])),
@@ -396,6 +406,16 @@ def kernel_timings(rt, F, torch, wl, flush, A, kLP, kHP, lp_args, hp_args, lp_gr
                      "overhead_pct": round((w_us / u_us - 1.0) * 100.0, 2),
                      "algorithmic_bytes": nbytes}
     return res
+
+
+def load_gather_peak():
+    """Measured random-gather ceiling (gathers/s) of probes/probe6.cu, committed under profiles/."""
+    p = os.path.join(ROOT, "profiles", "r01_probe_gather_ceiling.jsonl")
+    try:
+        with open(p) as f:
+            return max(json.loads(l)["gathers_per_s"] for l in f if l.strip())
+    except Exception:
+        return None
 
 
 def load_traffic(dom):

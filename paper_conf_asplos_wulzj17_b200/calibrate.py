@@ -209,10 +209,11 @@ def preemption_overhead(torch, wl, body, size, runs=50, chunk=1, prefetch=False,
 # the latency-cheapest (no prefetch, synchronous poll) to the throughput-cheapest.
 
 DEFAULT_CANDIDATES = tuple(
-    (c, k, pf, ap)
+    (c, k, pf, ap, clc)
     for c, k in ((1, 1), (2, 1), (1, 2), (4, 1), (2, 2), (1, 4), (8, 1), (4, 2), (16, 1), (8, 2), (32, 1),
                  (16, 2), (64, 1), (32, 4), (200, 1))
-    for pf, ap in ((False, False), (True, False), (True, True)))
+    for pf, ap, clc in ((False, False, False), (True, False, False), (True, True, False),
+                        (False, False, True)))        # last: the CLC task fetch (R25)
 
 
 def select_amortizing_factor(table, bound=0.04):
@@ -227,6 +228,7 @@ def select_amortizing_factor(table, bound=0.04):
 
     def key(r):
         return (r["C"] * r["K"], bool(r["prefetch"]) + bool(r["async_poll"]), r["overhead"])
+    # (a CLC variant adds no preemption latency beyond its chunk: it ranks with the plain ones)
     ok = [r for r in rows if r["overhead"] < bound]
     if ok:
         best = min(ok, key=key)
@@ -263,17 +265,19 @@ def tune_amortizing_factor(rt, torch, body, grid, args, flush, bound=0.04, candi
     t_u = timed(lambda: rt.launch_unwrapped(body, grid, args, stream=s))
     table = []
     by_l = {}
-    for c, k, pf, ap in candidates:
-        if body == F.BODY_GEMM_BF16 and pf:
-            continue                          # (in-tile GEMM: no prefetch, see flep.h)
-        by_l.setdefault(c * k, []).append((c, k, pf, ap))
+    for cand in candidates:
+        c, k, pf, ap, clc = (tuple(cand) + (False,))[:5]
+        if body == F.BODY_GEMM_BF16 and (pf or clc):
+            continue                          # (in-tile GEMM: no prefetch, no CLC, see flep.h)
+        by_l.setdefault(c * k, []).append((c, k, pf, ap, clc))
     for L in sorted(by_l):
-        for c, k, pf, ap in by_l[L]:
+        for c, k, pf, ap, clc in by_l[L]:
             kk = rt.register_kernel(body, chunk=c, poll=k, prefetch=pf, async_poll=ap,
-                                    in_tile=body == F.BODY_GEMM_BF16)
+                                    in_tile=body == F.BODY_GEMM_BF16, clc=clc)
             t_w = timed(lambda: rt.launch(kk, grid, args, stream=s))
-            table.append({"C": c, "K": k, "prefetch": pf, "async_poll": ap, "wrapped_us": round(t_w, 3),
-                          "unwrapped_us": round(t_u, 3), "overhead": t_w / t_u - 1.0})
+            table.append({"C": c, "K": k, "prefetch": pf, "async_poll": ap, "clc": clc,
+                          "wrapped_us": round(t_w, 3), "unwrapped_us": round(t_u, 3),
+                          "overhead": t_w / t_u - 1.0})
         if any(r["overhead"] < bound for r in table if r["C"] * r["K"] == L):
             break
     return select_amortizing_factor(table, bound), table
