@@ -84,8 +84,11 @@ typedef enum {
   FLEP_BODY_SPMV_CSR_F32 = 3,  /* y = A x, CSR fp32; 128 rows per block */
   FLEP_BODY_STENCIL5_F32 = 4,  /* 5-point out-of-place sweep, fp32; 64x64 cells per block */
   FLEP_BODY_STENCIL5_I32 = 5,  /* 5-point integer sweep, wraps mod 2^32; 64x64 cells per block */
-  FLEP_BODY_GEMM_BF16 = 6      /* C = A B^T, bf16 in, fp32 accumulate (tcgen05), bf16 out;
+  FLEP_BODY_GEMM_BF16 = 6,     /* C = A B^T, bf16 in, fp32 accumulate (tcgen05), bf16 out;
                                   128x256 output tile per block */
+  FLEP_BODY_STENCIL5_F32_TMA = 7 /* STENCIL5_F32 with the tile and its halo staged in shared memory
+                                  by the TMA unit and the output tile written back by a bulk
+                                  tensor store; same args; n % 4 == 0, 16-byte aligned in/out */
 } flep_body;
 
 /* Per-body argument structs (copied by value at launch). All pointers are device pointers. */

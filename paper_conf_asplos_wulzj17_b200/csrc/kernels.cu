@@ -6,6 +6,7 @@
 #include "flep_device.cuh"
 #include "bodies.cuh"
 #include "gemm_tcgen05.cuh"
+#include "stencil_tma.cuh"
 #include "kernels.hpp"
 
 namespace flep {
@@ -58,16 +59,26 @@ struct WithSmem : B {
 }  // namespace
 
 // GEMM launchers live in gemm_tcgen05.cu (they need the tensor-map encoder); they use these.
+// dynamic shared memory of a launch whose chunks hold `chunk` blocks (bodies may size it by C)
+template <class B, class = void> struct HasDynSmemFn : std::false_type {};
+template <class B> struct HasDynSmemFn<B, std::void_t<decltype(B::dyn_smem(1u))>> : std::true_type {};
+template <class Body>
+constexpr size_t smem_for(uint32_t chunk) {
+  if constexpr (HasDynSmemFn<Body>::value) return Body::dyn_smem(chunk);
+  else return Body::kDynSmem;
+}
 template <class Body>
 cudaError_t launch_worker_raw(const typename Body::Args& a, const WorkerParams& p, uint32_t W, cudaStream_t s, bool cov) {
-  if (cov) flep_worker<Body, true><<<W, Body::kThreads, Body::kDynSmem, s>>>(a, p);
-  else flep_worker<Body, false><<<W, Body::kThreads, Body::kDynSmem, s>>>(a, p);
+  const size_t sm = smem_for<Body>(p.chunk);
+  if (cov) flep_worker<Body, true><<<W, Body::kThreads, sm, s>>>(a, p);
+  else flep_worker<Body, false><<<W, Body::kThreads, sm, s>>>(a, p);
   return cudaGetLastError();
 }
 template <class Body>
 cudaError_t launch_unwrapped_raw(const typename Body::Args& a, dim3 grid, uint32_t offset, uint32_t count, cudaStream_t s) {
-  if (count == 0) flep_unwrapped<Body><<<grid, Body::kThreads, Body::kDynSmem, s>>>(a, grid.x, grid.y, 0);
-  else flep_unwrapped<Body><<<count, Body::kThreads, Body::kDynSmem, s>>>(a, grid.x, grid.y, offset);
+  const size_t sm = smem_for<Body>(1);
+  if (count == 0) flep_unwrapped<Body><<<grid, Body::kThreads, sm, s>>>(a, grid.x, grid.y, 0);
+  else flep_unwrapped<Body><<<count, Body::kThreads, sm, s>>>(a, grid.x, grid.y, offset);
   return cudaGetLastError();
 }
 template <class Body>
@@ -80,10 +91,27 @@ cudaError_t occupancy_raw(int* k, bool cov) {
     if (e) return e;
     e = cudaFuncSetAttribute(flep_unwrapped<Body>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)Body::kDynSmem);
     if (e) return e;
+    if constexpr (!Body::kPersistent) {
+      e = cudaFuncSetAttribute(flep_clc_worker<Body, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)Body::kDynSmem);
+      if (e) return e;
+      e = cudaFuncSetAttribute(flep_clc_worker<Body, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)Body::kDynSmem);
+      if (e) return e;
+    }
   }
   if (cov) return cudaOccupancyMaxActiveBlocksPerMultiprocessor(k, flep_worker<Body, true>, Body::kThreads, Body::kDynSmem);
   return cudaOccupancyMaxActiveBlocksPerMultiprocessor(k, flep_worker<Body, false>, Body::kThreads, Body::kDynSmem);
 }
+template <class Body>
+cudaError_t launch_clc_raw(const typename Body::Args& a, const WorkerParams& p, uint32_t N, cudaStream_t s, bool cov) {
+  const size_t sm = smem_for<Body>(p.chunk);
+  if (cov) flep_clc_worker<Body, true><<<N, Body::kThreads, sm, s>>>(a, p);
+  else flep_clc_worker<Body, false><<<N, Body::kThreads, sm, s>>>(a, p);
+  return cudaGetLastError();
+}
+template cudaError_t launch_worker_raw<Stencil5TmaBody>(const Stencil5TmaBody::Args&, const WorkerParams&, uint32_t, cudaStream_t, bool);
+template cudaError_t launch_unwrapped_raw<Stencil5TmaBody>(const Stencil5TmaBody::Args&, dim3, uint32_t, uint32_t, cudaStream_t);
+template cudaError_t launch_clc_raw<Stencil5TmaBody>(const Stencil5TmaBody::Args&, const WorkerParams&, uint32_t, cudaStream_t, bool);
+template cudaError_t occupancy_raw<Stencil5TmaBody>(int*, bool);
 template cudaError_t launch_worker_raw<GemmBody>(const GemmBody::Args&, const WorkerParams&, uint32_t, cudaStream_t, bool);
 template cudaError_t launch_unwrapped_raw<GemmBody>(const GemmBody::Args&, dim3, uint32_t, uint32_t, cudaStream_t);
 template cudaError_t occupancy_raw<GemmBody>(int*, bool);
@@ -110,6 +138,8 @@ const BodyOps kOps[] = {
      &Ops<StencilI32>::unwrapped, &Ops<StencilI32>::occupancy, nullptr, &Ops<StencilI32>::clc},
     {FLEP_BODY_GEMM_BF16, GemmBody::kThreads, sizeof(flep_gemm_args), &gemm_worker_launch,
      &gemm_unwrapped_launch, &gemm_occupancy, &gemm_validate, nullptr},
+    {FLEP_BODY_STENCIL5_F32_TMA, Stencil5TmaBody::kThreads, sizeof(flep_stencil_args), &stencil_tma_worker_launch,
+     &stencil_tma_unwrapped_launch, &stencil_tma_occupancy, &stencil_tma_validate, &stencil_tma_clc_launch},
 };
 
 }  // namespace
@@ -121,7 +151,7 @@ cudaError_t set_unwrapped_trace(uint64_t* p) {
 #endif
 
 const BodyOps* body_ops(int32_t body) {
-  if (body < 1 || body > FLEP_BODY_GEMM_BF16) return nullptr;
+  if (body < 1 || body > FLEP_BODY_STENCIL5_F32_TMA) return nullptr;
   return &kOps[body];
 }
 

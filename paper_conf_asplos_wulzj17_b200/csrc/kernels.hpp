@@ -36,5 +36,14 @@ template <class Body>
 cudaError_t launch_unwrapped_raw(const typename Body::Args& a, dim3 grid, uint32_t offset, uint32_t count, cudaStream_t s);
 template <class Body>
 cudaError_t occupancy_raw(int* k, bool cov);
+template <class Body>
+cudaError_t launch_clc_raw(const typename Body::Args& a, const WorkerParams& p, uint32_t N, cudaStream_t s, bool cov);
+
+// TMA-staged stencil body (stencil_tma.cu)
+const char* stencil_tma_validate(const void* user, dim3 grid);
+cudaError_t stencil_tma_worker_launch(const void* user, const WorkerParams& p, uint32_t W, cudaStream_t s, bool cov);
+cudaError_t stencil_tma_unwrapped_launch(const void* user, dim3 grid, uint32_t offset, uint32_t count, cudaStream_t s);
+cudaError_t stencil_tma_clc_launch(const void* user, const WorkerParams& p, uint32_t N, cudaStream_t s, bool cov);
+cudaError_t stencil_tma_occupancy(int* k, bool cov);
 
 }  // namespace flep

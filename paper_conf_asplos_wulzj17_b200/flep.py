@@ -16,6 +16,7 @@ OK, ERR_INVALID, ERR_STATE, ERR_CUDA, ERR_NOMEM, ERR_TIMEOUT, ERR_UNSUPPORTED = 
 POLICY_MANUAL, POLICY_FIFO, POLICY_HPF, POLICY_SLICE, POLICY_FFS, POLICY_REORDER = 0, 1, 2, 3, 4, 5
 FLAG_STREAM_MEMOP, FLAG_HOST_MAPPED = 0, 1
 BODY_SAXPY_I32, BODY_SAXPY_F32, BODY_SPMV_CSR_F32, BODY_STENCIL5_F32, BODY_STENCIL5_I32, BODY_GEMM_BF16 = 1, 2, 3, 4, 5, 6
+BODY_STENCIL5_F32_TMA = 7
 STATE_QUEUED, STATE_RUNNING, STATE_YIELDING, STATE_PREEMPTED, STATE_PARTIAL, STATE_DONE = 0, 1, 2, 3, 4, 5
 STATE_NAMES = {0: "QUEUED", 1: "RUNNING", 2: "YIELDING", 3: "PREEMPTED", 4: "PARTIAL", 5: "DONE"}
 REASON_YIELD, REASON_EXHAUSTED = 1, 2
@@ -87,7 +88,8 @@ class EpochInfo(C.Structure):
 
 
 ARGS_FOR_BODY = {BODY_SAXPY_I32: SaxpyI32Args, BODY_SAXPY_F32: SaxpyF32Args, BODY_SPMV_CSR_F32: SpmvArgs,
-                 BODY_STENCIL5_F32: StencilArgs, BODY_STENCIL5_I32: StencilArgs, BODY_GEMM_BF16: GemmArgs}
+                 BODY_STENCIL5_F32: StencilArgs, BODY_STENCIL5_I32: StencilArgs, BODY_GEMM_BF16: GemmArgs,
+                 BODY_STENCIL5_F32_TMA: StencilArgs}
 
 # exported symbols: name -> (restype, argtypes)
 _P = C.c_void_p
