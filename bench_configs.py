@@ -462,6 +462,90 @@ def run_clc(args, rank, world, local):
     barrier(world)
 
 
+def run_delay(args, rank, world, local):
+    """Delay sweep (Fig. 9): the HP kernel (stencil5 4096^2) arrives when the
+    LP victim (SpMV-CSR 2^20 rows, counter worker C = K = 1) has handed out a fraction d of its
+    blocks (device self-trigger at block d*N), d = 0.1 .. 0.9. FLEP: the trigger is a temporal
+    request; FIFO: the same trigger only stamps the arrival (n = 0), the HP waits for the LP.
+    HP turnaround = HP last CTA exit - arrival (device %globaltimer); speedup = FIFO / FLEP, next
+    to the zero-overhead bound (T_LP (1 - d) + T_HP) / T_HP from the standalone times."""
+    import torch
+    from bench import (ClockSampler, L2Flush, Workload, barrier, physical_gpu_index, spot_parity,
+                       STENCIL_N, SPMV_ROWS)
+    from paper_conf_asplos_wulzj17_b200 import flep as F
+    torch.cuda.set_device(local)
+    rt = F.Runtime(device=local, exec_on_user_stream=True)
+    wl = Workload(torch)
+    flush = L2Flush(torch)
+    A, B = torch.cuda.Stream(priority=-2), torch.cuda.Stream(priority=0)
+    lp_args = F.spmv_args(wl.d_y, wl.d_rowptr, wl.d_col, wl.d_val, wl.d_x)
+    hp_args = F.stencil_args(wl.d_out, wl.d_in)
+    lp_grid, hp_grid = F.spmv_grid(SPMV_ROWS), F.stencil_grid(STENCIL_N)
+    n_lp = lp_grid[0]
+    k_lp = rt.register_kernel(F.BODY_SPMV_CSR_F32, chunk=1, poll=1, name="spmv")
+    k_hp = rt.register_kernel(F.BODY_STENCIL5_F32, chunk=1, poll=4, clc=True, name="stencil")
+
+    def alone(k, grid, a):
+        ts = []
+        for _ in range(12):
+            flush.zero_()
+            torch.cuda.synchronize()
+            h = rt.launch(k, grid, a, stream=A)
+            rt.sync(h)
+            ev = rt.events(h, 1)
+            ts.append((max(e.t_exit for e in ev) - min(e.t_entry for e in ev)) / 1e3)
+        return float(np.median(ts[2:]))
+    t_lp, t_hp = alone(k_lp, lp_grid, lp_args), alone(k_hp, hp_grid, hp_args)
+    reps = max(4, args.steps // 10)
+    points = []
+    with ClockSampler(physical_gpu_index(local)) as clk:
+        for d in [i / 10 for i in range(1, 10)]:
+            res = {}
+            for mode in ("fifo", "flep"):
+                tt = []
+                for r in range(reps + 1):
+                    with torch.cuda.stream(A):
+                        flush.zero_()
+                        e0 = torch.cuda.Event()
+                        e0.record(A)
+                    rt.arm_next_trigger(int(d * n_lp), rt.num_sms if mode == "flep" else 0)
+                    h = rt.launch(k_lp, lp_grid, lp_args, priority=0, stream=A)
+                    B.wait_event(e0)
+                    h2 = rt.launch(k_hp, hp_grid, hp_args, priority=1, stream=B)
+                    rt.wait_epoch(h, timeout_ns=10_000_000_000)
+                    pre = rt.query(h).state == F.STATE_PREEMPTED
+                    rt.sync(h2, timeout_ns=10_000_000_000)
+                    if pre:
+                        rt.resume(h)
+                    rt.sync(h, timeout_ns=10_000_000_000)
+                    torch.cuda.synchronize()
+                    ep = rt.epoch_info(h, 1)
+                    hp_end = max(e.t_exit for e in rt.events(h2, 1))
+                    if r >= 1 and ep.t_trigger:
+                        tt.append((hp_end - ep.t_trigger) / 1e3)
+                res[mode] = float(np.median(tt)) if tt else None
+            bound = (t_lp * (1 - d) + t_hp) / t_hp
+            points.append({"d": d, "hp_turnaround_fifo_us": round(res["fifo"], 3) if res["fifo"] else None,
+                           "hp_turnaround_flep_us": round(res["flep"], 3) if res["flep"] else None,
+                           "speedup": round(res["fifo"] / res["flep"], 3) if res["fifo"] and res["flep"] else None,
+                           "zero_overhead_bound": round(bound, 3)})
+    parity = spot_parity(wl, torch)
+    rt.close()
+    sp = [p["speedup"] for p in points if p["speedup"]]
+    out = {"metric": METRIC, "value": round(float(np.mean(sp)), 3) if sp else None, "unit": "x",
+           "value_definition": "HP turnaround speedup FIFO / FLEP averaged over arrival points d = 0.1..0.9 of the LP",
+           "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "higher_is_better": True,
+           "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic (seeded; synth/gen.py)",
+           "config": {"workload": "LP SpMV-CSR 2^20 rows (counter worker, C=K=1), HP stencil5 4096^2 (CLC), "
+                                  "HP arrival = device trigger at block d*N of the LP", "reps_per_point": reps,
+                      "l2": "flushed before every step"},
+           "standalone_us": {"lp": round(t_lp, 3), "hp": round(t_hp, 3)},
+           "points": points, "parity": parity, "clocks": clk.summary()}
+    if rank == 0:
+        print(json.dumps(out), flush=True)
+    barrier(world)
+
+
 # ------------------------------------------------------------------------------------------
 def assign_jobs(jobs, t_e_of, world):
     """One job queue feeding `world` independent per-GPU schedulers (configs[4]): each arrival

@@ -256,7 +256,9 @@ flep_status flep_workers_for(flep_rt rt, int32_t body, uint32_t* ctas_per_sm, ui
 
 /* ---- test / bench hooks (always compiled; cost nothing when unused) -------------------- */
 /* Device self-trigger: the worker that fetches the chunk holding `block_index` writes the
-   request (epoch, n_sms) itself. Applies to the launch's next epoch if it is not running. */
+   request (epoch, n_sms) itself and stamps the time (flep_epoch_info.t_trigger). n_sms == 0 only
+   stamps the time (an arrival marker, no request). Applies to the launch's next epoch if it is
+   not running. */
 flep_status flep_debug_trigger_at(flep_rt rt, flep_launch_t h, uint64_t block_index,
                                   uint32_t n_sms);
 /* Arm a self-trigger for the NEXT flep_launch issued on this runtime. */

@@ -1064,7 +1064,6 @@ flep_status flep_launch_sliced(flep_rt rt, int32_t body, flep_dim3 grid, const v
 
 flep_status flep_debug_trigger_at(flep_rt rt, flep_launch_t h, uint64_t block_index, uint32_t n_sms) {
   if (!rt) return fail(FLEP_ERR_INVALID, "rt is NULL");
-  if (n_sms == 0) return fail(FLEP_ERR_INVALID, "n_sms == 0");
   ApiLock lk(rt);
   Launch* L = find(rt, h);
   if (!L) return fail(FLEP_ERR_INVALID, "unknown launch %lld", (long long)h);
@@ -1078,7 +1077,6 @@ flep_status flep_debug_trigger_at(flep_rt rt, flep_launch_t h, uint64_t block_in
 
 flep_status flep_debug_arm_next_trigger(flep_rt rt, uint64_t block_index, uint32_t n_sms) {
   if (!rt) return fail(FLEP_ERR_INVALID, "rt is NULL");
-  if (n_sms == 0) return fail(FLEP_ERR_INVALID, "n_sms == 0");
   ApiLock lk(rt);
   rt->arm_block = block_index >= 0xffffffffull ? kNoTrigger : (uint32_t)block_index;
   rt->arm_n = std::min<uint32_t>(n_sms, 0xffff);
