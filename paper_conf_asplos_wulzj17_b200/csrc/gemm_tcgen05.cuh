@@ -65,7 +65,9 @@ struct GemmBody {
     uint64_t trest[2];                // epilogue restored a spilled accumulator into this half
     uint32_t tile_q[QDEPTH];
     uint32_t tile_kb0[QDEPTH];        // first k-step of the tile (> 0: continue a spilled tile)
-    uint32_t tile_kend[QDEPTH];       // k-step the producer stopped at (nk: runs to the end)
+    uint32_t stage_stop[STAGES];      // 1: this stage is a stop marker (no data): written by the
+                                      // producer after the stage's empty wait, read by the MMA
+                                      // after its full wait, so the ring orders every access
     uint32_t acc_kend[2];             // MMA -> epilogue: k-steps accumulated in this half
     uint32_t tmem_base;
     uint32_t p_stage, p_phase;        // producer
@@ -338,10 +340,8 @@ struct GemmBody {
             const bool cont = restoring && b == b0;        // continue a spilled tile
             const uint32_t kb0 = cont ? kbs : 0u;
             mbar_wait(&s->qempty[qi], qph ^ 1u);
-            const uint32_t my_q = qi;
             s->tile_q[qi] = b;
             s->tile_kb0[qi] = kb0;
-            s->tile_kend[qi] = nk;
             mbar_arrive(&s->qfull[qi]);
             if (++qi == QDEPTH) { qi = 0; qph ^= 1u; }
             // coverage log: a tile counts once, when its chunk is first handed out (the tiles of
@@ -361,6 +361,7 @@ struct GemmBody {
                 if (j % kInTilePoll == 0 && j > 0) { pend = ld_relaxed_gpu(p.ctrl); pend_valid = true; }
               }
               mbar_wait(&s->empty[st], ph ^ 1u);
+              s->stage_stop[st] = 0u;
               uint8_t* sa = base + st * kStage;
               uint8_t* sb = sa + kBytesA;
               mbar_expect_tx(&s->full[st], kStage);
@@ -369,9 +370,9 @@ struct GemmBody {
               if (++st == STAGES) { st = 0; ph ^= 1u; }
             }
             if (stop) {
-              // stop marker: the next stage carries no data; the MMA sees kend == kb and commits
+              // stop marker: the next stage carries no data; the MMA sees it and commits
               mbar_wait(&s->empty[st], ph ^ 1u);
-              s->tile_kend[my_q] = kb;
+              s->stage_stop[st] = 1u;
               mbar_arrive(&s->full[st]);
               if (++st == STAGES) { st = 0; ph ^= 1u; }
               mine->b = b; mine->kb = kb; mine->b_end = b1; mine->valid = 1;
@@ -398,9 +399,8 @@ struct GemmBody {
           mbar_wait(&s->qfull[qi], qph);
           const uint32_t b = s->tile_q[qi];
           const uint32_t kb0 = s->tile_kb0[qi];
-          const uint32_t my_q = qi;
-          mbar_arrive(&s->qempty[qi]);                     // (the slot is reused 4 tiles later:
-          if (++qi == QDEPTH) { qi = 0; qph ^= 1u; }       //  tile_kend[my_q] stays valid)
+          mbar_arrive(&s->qempty[qi]);
+          if (++qi == QDEPTH) { qi = 0; qph ^= 1u; }
           if (b == STOP) break;
           mbar_wait(&s->tempty[acc], aph ^ 1u);            // epilogue drained this half
           if (kb0 > 0) { mbar_wait(&s->trest[acc], rph[acc]); rph[acc] ^= 1u; }   // restored
@@ -409,7 +409,7 @@ struct GemmBody {
           uint32_t kb = kb0;
           for (; kb < nk; ++kb) {
             mbar_wait(&s->full[st], ph);
-            if (kb >= s->tile_kend[my_q]) {                // stop marker: release it, commit
+            if (s->stage_stop[st]) {                       // stop marker: release it, commit
               mbar_arrive(&s->empty[st]);
               if (++st == STAGES) { st = 0; ph ^= 1u; }
               break;

@@ -1,5 +1,7 @@
 """Small wrapped launches for compute-sanitizer (memcheck / racecheck / synccheck): every body,
-one temporal and one spatial preemption with resume."""
+one temporal and one spatial preemption with resume, the CLC task fetch (with a preempt/resume
+cycle), the TMA-staged stencil (counter and CLC workers, chunk 2 so the second input buffer is
+used) and in-tile GEMM preemption."""
 import os
 import sys
 
@@ -41,6 +43,35 @@ def main():
     C = torch.empty(256, 512, dtype=torch.bfloat16, device="cuda")
     k4 = rt.register_kernel(F.BODY_GEMM_BF16, chunk=1, poll=1)
     rt.sync(rt.launch(k4, F.gemm_grid(256, 512), F.gemm_args(C, A, B)))
+    # CLC task fetch: uninterrupted, then a host preempt/resume cycle
+    k5 = rt.register_kernel(F.BODY_SAXPY_I32, chunk=2, poll=1, clc=True)
+    rt.sync(rt.launch(k5, F.saxpy_grid(n), F.saxpy_i32_args(yd, xd, 5)))
+    h = rt.launch(k5, F.saxpy_grid(n), F.saxpy_i32_args(yd, xd, 7))
+    try:
+        rt.preempt(h, rt.num_sms)
+        rt.resume(h)
+    except F.FlepError:
+        pass                              # completed first
+    rt.sync(h)
+    # TMA-staged stencil: unwrapped, counter worker and CLC worker (chunk 2: double buffer)
+    st2 = T(gen.stencil_f32_input(260, 5))
+    out2 = torch.empty_like(st2)
+    rt.launch_unwrapped(F.BODY_STENCIL5_F32_TMA, F.stencil_grid(260), F.stencil_args(out2, st2))
+    for clc in (False, True):
+        k6 = rt.register_kernel(F.BODY_STENCIL5_F32_TMA, chunk=2, poll=1, clc=clc)
+        rt.sync(rt.launch(k6, F.stencil_grid(260), F.stencil_args(out2, st2)))
+    # in-tile GEMM preemption with resume
+    a_bits, b_bits = gen.gemm_bf16_inputs(256, 512, 1024, 6)
+    A = torch.from_numpy(a_bits.view(np.int16)).cuda().view(torch.bfloat16)
+    B = torch.from_numpy(b_bits.view(np.int16)).cuda().view(torch.bfloat16)
+    C = torch.empty(256, 512, dtype=torch.bfloat16, device="cuda")
+    k7 = rt.register_kernel(F.BODY_GEMM_BF16, chunk=1, poll=1, ctas_per_sm=1, in_tile=True)
+    rt.arm_next_trigger(1, rt.num_sms)
+    h = rt.launch(k7, F.gemm_grid(256, 512), F.gemm_args(C, A, B))
+    rt.wait_epoch(h)
+    if rt.query(h).state == F.STATE_PREEMPTED:
+        rt.resume(h)
+    rt.sync(h)
     torch.cuda.synchronize()
     rt.close()
     print("sanitizer case done")
