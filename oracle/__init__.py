@@ -14,6 +14,8 @@ Modules
   des        — discrete-event simulation of the runtime policies (Fig. 6, §5): FIFO, HPF(+SRPT),
                kernel slicing; simulate and replay modes
   estimates  — ridge-regression duration model (§4.2) and the preemption-overhead mean
+  intile     — k-step model of in-tile preemption of the contraction body (R21)
+  clc        — step model of the CLC task fetch (R25) with an exhaustive explorer
   metrics    — NTT / ANTT / STP / speedup / spatial-overhead definitions (§6.1)
 
 Parity status: every function is pinned by `tests/test_oracle_*.py`
