@@ -159,6 +159,11 @@ typedef struct {
    (spatial) at once; flep_resume withdraws the request (no relaunch); completion is the grid's
    completion. The worker event log covers the first W CTAs. */
 #define FLEP_KFLAG_CLC 16u
+/* Scheduling-warp worker (R26; bodies without whole-CTA barriers in run(): SAXPY, SpMV,
+   register stencils): the poll/fetch/exit step runs in one extra warp that keeps the next chunk in
+   a shared-memory ring, one chunk ahead (as FLEP_KFLAG_PREFETCH), so the body warps never wait
+   for it. The CTA is kThreads + 32 threads (fewer resident CTAs per SM may fit). */
+#define FLEP_KFLAG_SCHED_WARP 32u
 
 typedef enum {
   FLEP_STATE_QUEUED = 0,     /* intercepted, waiting for a scheduling decision (S2) */

@@ -209,11 +209,13 @@ def preemption_overhead(torch, wl, body, size, runs=50, chunk=1, prefetch=False,
 # the latency-cheapest (no prefetch, synchronous poll) to the throughput-cheapest.
 
 DEFAULT_CANDIDATES = tuple(
-    (c, k, pf, ap, clc)
+    (c, k, pf, ap, clc, sw)
     for c, k in ((1, 1), (2, 1), (1, 2), (4, 1), (2, 2), (1, 4), (8, 1), (4, 2), (16, 1), (8, 2), (32, 1),
                  (16, 2), (64, 1), (32, 4), (200, 1))
-    for pf, ap, clc in ((False, False, False), (True, False, False), (True, True, False),
-                        (False, False, True)))        # last: the CLC task fetch (R25)
+    for pf, ap, clc, sw in ((False, False, False, False), (True, False, False, False),
+                            (True, True, False, False),
+                            (False, False, True, False),     # the CLC task fetch (R25)
+                            (False, False, False, True)))    # the scheduling-warp worker (R26)
 
 
 def select_amortizing_factor(table, bound=0.04):
@@ -266,16 +268,17 @@ def tune_amortizing_factor(rt, torch, body, grid, args, flush, bound=0.04, candi
     table = []
     by_l = {}
     for cand in candidates:
-        c, k, pf, ap, clc = (tuple(cand) + (False,))[:5]
-        if body == F.BODY_GEMM_BF16 and (pf or clc):
-            continue                          # (in-tile GEMM: no prefetch, no CLC, see flep.h)
-        by_l.setdefault(c * k, []).append((c, k, pf, ap, clc))
+        c, k, pf, ap, clc, sw = (tuple(cand) + (False, False))[:6]
+        if body in (F.BODY_GEMM_BF16, F.BODY_STENCIL5_F32_TMA) and (pf or clc or sw) and \
+                not (body == F.BODY_STENCIL5_F32_TMA and clc):
+            continue                          # (in-tile GEMM: no prefetch/CLC; TMA stencil: no sched warp)
+        by_l.setdefault(c * k, []).append((c, k, pf, ap, clc, sw))
     for L in sorted(by_l):
-        for c, k, pf, ap, clc in by_l[L]:
+        for c, k, pf, ap, clc, sw in by_l[L]:
             kk = rt.register_kernel(body, chunk=c, poll=k, prefetch=pf, async_poll=ap,
-                                    in_tile=body == F.BODY_GEMM_BF16, clc=clc)
+                                    in_tile=body == F.BODY_GEMM_BF16, clc=clc, sched_warp=sw)
             t_w = timed(lambda: rt.launch(kk, grid, args, stream=s))
-            table.append({"C": c, "K": k, "prefetch": pf, "async_poll": ap, "clc": clc,
+            table.append({"C": c, "K": k, "prefetch": pf, "async_poll": ap, "clc": clc, "sched_warp": sw,
                           "wrapped_us": round(t_w, 3), "unwrapped_us": round(t_u, 3),
                           "overhead": t_w / t_u - 1.0})
         if any(r["overhead"] < bound for r in table if r["C"] * r["K"] == L):

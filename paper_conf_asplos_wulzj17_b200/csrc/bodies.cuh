@@ -108,7 +108,7 @@ struct SpmvBody : NoResources {
       const uint32_t nr = min(kGroupRows, row_end - r0);
       if (tid <= nr) s_rp[tid] = __ldg(g.rowptr + r0 + tid);
       if (tid == 0 && nr == kGroupRows) s_rp[kGroupRows] = __ldg(g.rowptr + r0 + kGroupRows);
-      __syncthreads();
+      body_sync<kThreads>();
       const int32_t p0 = s_rp[0], p1 = s_rp[nr];
       int32_t my_s = 0, my_e = 0;
       if (tid < nr) { my_s = s_rp[tid]; my_e = s_rp[tid + 1]; }
@@ -133,12 +133,12 @@ struct SpmvBody : NoResources {
             if (i < n) s_prod[i] = v[u] * xv[u];
           }
         }
-        __syncthreads();
+        body_sync<kThreads>();
         if (tid < nr) {                        // row r0+tid: its products in ascending p order
           const int32_t lo = max(my_s, base), hi = min(my_e, base + n);
           for (int32_t p = lo; p < hi; ++p) acc += s_prod[p - base];
         }
-        __syncthreads();
+        body_sync<kThreads>();
       }
       if (tid < nr) __stcs(g.y + r0 + tid, acc);
     }

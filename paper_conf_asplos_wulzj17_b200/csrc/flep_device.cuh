@@ -154,6 +154,14 @@ __device__ __forceinline__ void st_relaxed_gpu(uint32_t* p, uint32_t v) {
   asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" :: "l"(p), "r"(v) : "memory");
 }
 
+// CTA-wide barrier for original block bodies: named barrier 1 over the body's kThreads threads.
+// In the unwrapped grid and the plain worker that is every thread (same as __syncthreads); in the
+// scheduling-warp worker (flep_worker_sw) the extra scheduling warp does not take part.
+template <int kThreads>
+__device__ __forceinline__ void body_sync() {
+  asm volatile("bar.sync 1, %0;" :: "n"(kThreads) : "memory");
+}
+
 // Does the control word ask the worker on `sm` to leave? (Fig. 4(c))
 __device__ __forceinline__ bool should_yield(uint32_t c, const WorkerParams& p, uint32_t sm) {
   const uint32_t gen = c >> 16, n = c & 0xffffu;
@@ -316,6 +324,52 @@ __device__ __forceinline__ uint32_t next_chunk(const WorkerParams& p, SchedState
   return base;
 }
 
+// Exit path (a7), run by the worker's scheduling thread after the body's last chunk. A worker
+// whose exit was counted by its exhausted fetch does no atomic here;
+// any other (yield, entry exit) makes its exit event now: one 64-bit increment of the yield
+// count (R23). No fences: the outputs are published by kernel completion (stream order), and
+// the host status is a notification (flep_sync also waits for the grid's completion event).
+__device__ __forceinline__ void worker_exit(const WorkerParams& p, WorkerShared& ws) {
+  WorkerEvent& e = p.ev[(p.epoch % kEvEpochs) * p.workers + blockIdx.x];
+  const uint64_t t_exit = gtimer();
+  e.smid = ws.sm; e.reason = ws.reason; e.n_blocks = ws.blocks; e.epoch = p.epoch;
+  e.t_entry = ws.t_entry; e.t_exit = t_exit;
+  if (!ws.counted) {
+    const unsigned long long inc = (1ull << 32) | ((unsigned long long)ws.partial << 48);
+    note_exit_event(p, ws, atom_add_cx(&p.cb->cx, inc), 0u, ws.partial);
+  }
+  if (ws.last) {                                       // the epoch's W-th exit event
+    // every worker has made its exit event: none fetches again (some may still run the chunk
+    // they hold, which they complete before the grid ends, A4)
+    const bool first_epoch = p.epoch == p.gen_first;
+    const bool already = !first_epoch && ld_relaxed_gpu(&p.cb->done_gen) >= p.gen_first;
+    const uint32_t c = ws.ev_raw + ctr_offset(p);      // effective counter (R20)
+    const bool done = already || (c >= p.n_blocks && ws.ev_part == 0u);
+    const uint32_t d = done ? p.n_blocks : min(c, p.n_blocks) - ws.ev_part;
+    const uint32_t st = done ? kStateDone : kStatePreempted;
+    const uint32_t ei = p.epoch % kEvEpochs;
+    p.cb->ep_t_end[ei] = t_exit; p.cb->ep_done[ei] = d; p.cb->ep_ctr[ei] = c;
+    p.cb->ep_state[ei] = st;
+    p.cb->ep_t_trigger[(p.epoch + 1) % kEvEpochs] = 0;  // next epoch's trigger stamp
+    if (done) {                                        // clean for reuse; remember completion
+      p.cb->cx = 0ull;
+      if (!already) p.cb->done_gen = p.epoch;
+    } else {
+      // progress kept, exit counts reset; later epochs fetch from the effective counter,
+      // capped at ceil(N/C)*C (only reached when partial tiles remain)
+      const uint32_t cap = ((p.n_blocks + p.chunk - 1) / p.chunk) * p.chunk;
+      p.cb->cx = (unsigned long long)min(c, cap);
+    }
+    // host notification only for a PREEMPTED epoch; DONE is seen as the grid's completion
+    // (a system-scope store delays the completion by a PCIe round trip, R24)
+    if (p.status && !done) {
+      st_relaxed_sys(&p.status->ctr, c);
+      st_relaxed_sys_u64(reinterpret_cast<uint64_t*>(&p.status->word),
+                         ((uint64_t)d << 32) | ((p.epoch << 8) | st));
+    }
+  }
+}
+
 // The worker. Body contract:
 //   Body::kThreads               CTA size of the original kernel
 //   Body::kMinBlocks             resident CTAs per SM the register budget is sized for
@@ -376,50 +430,79 @@ flep_worker(const __grid_constant__ typename Body::Args args, const WorkerParams
     }
   }
   Body::teardown(args);              // release per-worker resources before leaving the SM (a7)
-  // exit path (a7). A worker whose exit was counted by its exhausted fetch does no atomic here;
-  // any other (yield, entry exit) makes its exit event now: one 64-bit increment of the yield
-  // count (R23). No fences: the outputs are published by kernel completion (stream order), and
-  // the host status is a notification (flep_sync also waits for the grid's completion event).
-  if (tid == 0) {
-    WorkerEvent& e = p.ev[(p.epoch % kEvEpochs) * p.workers + blockIdx.x];
-    const uint64_t t_exit = gtimer();
-    e.smid = ws.sm; e.reason = ws.reason; e.n_blocks = ws.blocks; e.epoch = p.epoch;
-    e.t_entry = ws.t_entry; e.t_exit = t_exit;
-    if (!ws.counted) {
-      const unsigned long long inc = (1ull << 32) | ((unsigned long long)ws.partial << 48);
-      note_exit_event(p, ws, atom_add_cx(&p.cb->cx, inc), 0u, ws.partial);
+  if (tid == 0) worker_exit(p, ws);
+}
+
+// ---- scheduling-warp worker (FLEP_KFLAG_SCHED_WARP, reading R26) ------------------------------
+// The same protocol as flep_worker, with the scheduling step (poll, fetch, exit accounting) run by
+// one extra warp instead of thread 0 of the body: the scheduler fills a two-slot ring in shared
+// memory one chunk ahead and the body warps only wait on an mbarrier, so the step's serial
+// instruction chain and its round trips leave the body warps' critical path. Holding one chunk
+// ahead is the prefetch of reading R3 (a stopping worker still runs the chunk it holds, A4).
+__device__ __forceinline__ void sw_mbar_wait(uint32_t bar, uint32_t parity) {
+  asm volatile("{\n .reg .pred p;\n W: mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n @!p bra W;\n}\n"
+               :: "r"(bar), "r"(parity) : "memory");
+}
+__device__ __forceinline__ void sw_mbar_arrive(uint32_t bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" :: "r"(bar) : "memory");
+}
+template <class Body>
+struct SwMinBlocks {                 // resident CTAs per SM the register budget is sized for
+  static constexpr int value = (Body::kMinBlocks * Body::kThreads) / (Body::kThreads + 32) > 0
+                                   ? (Body::kMinBlocks * Body::kThreads) / (Body::kThreads + 32) : 1;
+};
+
+template <class Body, bool kCoverage>
+__global__ void __launch_bounds__(Body::kThreads + 32, SwMinBlocks<Body>::value)
+flep_worker_sw(const __grid_constant__ typename Body::Args args, const WorkerParams p) {
+  __shared__ uint32_t s_ring[2];
+  __shared__ alignas(8) uint64_t s_full[2], s_empty[2];
+  __shared__ WorkerShared ws;
+  constexpr uint32_t kT = Body::kThreads;
+  const uint32_t tid = threadIdx.x;
+  const uint32_t full0 = static_cast<uint32_t>(__cvta_generic_to_shared(&s_full[0]));
+  const uint32_t empty0 = static_cast<uint32_t>(__cvta_generic_to_shared(&s_empty[0]));
+  if (tid == kT) {
+    ws.sm = smid_reg(); ws.t_entry = gtimer(); ws.blocks = 0; ws.reason = 0;
+    ws.counted = 0; ws.last = 0; ws.ev_raw = 0; ws.ev_part = 0; ws.partial = 0;
+    if (blockIdx.x == 0 && p.started_hint && p.status) st_relaxed_sys(&p.status->started, p.epoch);
+    for (uint32_t i = 0; i < 2; ++i) {
+      asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" :: "r"(full0 + 8 * i) : "memory");
+      asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" :: "r"(empty0 + 8 * i) : "memory");
     }
-    if (ws.last) {                                       // the epoch's W-th exit event
-      // every worker has made its exit event: none fetches again (some may still run the chunk
-      // they hold, which they complete before the grid ends, A4)
-      const bool first_epoch = p.epoch == p.gen_first;
-      const bool already = !first_epoch && ld_relaxed_gpu(&p.cb->done_gen) >= p.gen_first;
-      const uint32_t c = ws.ev_raw + ctr_offset(p);      // effective counter (R20)
-      const bool done = already || (c >= p.n_blocks && ws.ev_part == 0u);
-      const uint32_t d = done ? p.n_blocks : min(c, p.n_blocks) - ws.ev_part;
-      const uint32_t st = done ? kStateDone : kStatePreempted;
-      const uint32_t ei = p.epoch % kEvEpochs;
-      p.cb->ep_t_end[ei] = t_exit; p.cb->ep_done[ei] = d; p.cb->ep_ctr[ei] = c;
-      p.cb->ep_state[ei] = st;
-      p.cb->ep_t_trigger[(p.epoch + 1) % kEvEpochs] = 0;  // next epoch's trigger stamp
-      if (done) {                                        // clean for reuse; remember completion
-        p.cb->cx = 0ull;
-        if (!already) p.cb->done_gen = p.epoch;
-      } else {
-        // progress kept, exit counts reset; later epochs fetch from the effective counter,
-        // capped at ceil(N/C)*C (only reached when partial tiles remain)
-        const uint32_t cap = ((p.n_blocks + p.chunk - 1) / p.chunk) * p.chunk;
-        p.cb->cx = (unsigned long long)min(c, cap);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  Body::setup(args);
+  if (tid >= kT) {
+    if (tid == kT) {                 // the scheduling lane: one chunk ahead of the body warps
+      SchedState st;
+      for (uint32_t j = 0;; ++j) {
+        const uint32_t i = j & 1u, ph = (j >> 1) & 1u;
+        if (j >= 2) sw_mbar_wait(empty0 + 8 * i, ph ^ 1u);   // slot i consumed (round j-2)
+        const uint32_t b = next_chunk(p, st, ws);
+        s_ring[i] = b;
+        sw_mbar_arrive(full0 + 8 * i);                      // release: the body warps read s_ring[i]
+        if (b == 0xffffffffu) break;
       }
-      // host notification only for a PREEMPTED epoch; DONE is seen as the grid's completion
-      // (a system-scope store delays the completion by a PCIe round trip, R24)
-      if (p.status && !done) {
-        st_relaxed_sys(&p.status->ctr, c);
-        st_relaxed_sys_u64(reinterpret_cast<uint64_t*>(&p.status->word),
-                           ((uint64_t)d << 32) | ((p.epoch << 8) | st));
-      }
+    }
+  } else {
+    for (uint32_t j = 0;; ++j) {
+      const uint32_t i = j & 1u, ph = (j >> 1) & 1u;
+      sw_mbar_wait(full0 + 8 * i, ph);
+      const uint32_t b0 = s_ring[i];
+      if (b0 == 0xffffffffu) break;
+      const uint32_t b1 = min(b0 + p.chunk, p.n_blocks);
+      Body::run(args, b0, b1, p.gx, p.gy);
+      if (kCoverage && tid == 0)
+        for (uint32_t b = b0; b < b1; ++b) atomicAdd(&p.cov[b], 1u);
+      body_sync<kT>();               // every body thread is past s_ring[i] and the chunk's smem
+      if (tid == 0) sw_mbar_arrive(empty0 + 8 * i);
     }
   }
+  __syncthreads();
+  Body::teardown(args);
+  if (tid == kT) worker_exit(p, ws);
 }
 
 // ---- CLC task fetch (reading R25) ----------------------------------------------

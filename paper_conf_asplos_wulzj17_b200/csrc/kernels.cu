@@ -28,6 +28,16 @@ struct Ops {
     else flep_clc_worker<Body, false><<<N, Body::kThreads, Body::kDynSmem, s>>>(a, p);
     return cudaGetLastError();
   }
+  static cudaError_t worker_sw(const void* args, const WorkerParams& p, uint32_t W, cudaStream_t s, bool cov) {
+    const typename Body::Args& a = *reinterpret_cast<const typename Body::Args*>(args);
+    if (cov) flep_worker_sw<Body, true><<<W, Body::kThreads + 32, Body::kDynSmem, s>>>(a, p);
+    else flep_worker_sw<Body, false><<<W, Body::kThreads + 32, Body::kDynSmem, s>>>(a, p);
+    return cudaGetLastError();
+  }
+  static cudaError_t occupancy_sw(int* k, bool cov) {
+    if (cov) return cudaOccupancyMaxActiveBlocksPerMultiprocessor(k, flep_worker_sw<Body, true>, Body::kThreads + 32, Body::kDynSmem);
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(k, flep_worker_sw<Body, false>, Body::kThreads + 32, Body::kDynSmem);
+  }
   static cudaError_t unwrapped(const void* args, dim3 grid, uint32_t offset, uint32_t count,
                                cudaStream_t s) {
     const typename Body::Args& a = *reinterpret_cast<const typename Body::Args*>(args);
@@ -125,21 +135,27 @@ using StencilF32 = WithSmem<Stencil5Body<false>>;
 using StencilI32 = WithSmem<Stencil5Body<true>>;
 
 const BodyOps kOps[] = {
-    {0, 0, 0, nullptr, nullptr, nullptr, nullptr, nullptr},
+    {0, 0, 0, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr},
     {FLEP_BODY_SAXPY_I32, SaxpyI32::kThreads, sizeof(flep_saxpy_i32_args), &Ops<SaxpyI32>::worker,
-     &Ops<SaxpyI32>::unwrapped, &Ops<SaxpyI32>::occupancy, nullptr, &Ops<SaxpyI32>::clc},
+     &Ops<SaxpyI32>::unwrapped, &Ops<SaxpyI32>::occupancy, nullptr, &Ops<SaxpyI32>::clc,
+     &Ops<SaxpyI32>::worker_sw, &Ops<SaxpyI32>::occupancy_sw},
     {FLEP_BODY_SAXPY_F32, SaxpyF32::kThreads, sizeof(flep_saxpy_f32_args), &Ops<SaxpyF32>::worker,
-     &Ops<SaxpyF32>::unwrapped, &Ops<SaxpyF32>::occupancy, nullptr, &Ops<SaxpyF32>::clc},
+     &Ops<SaxpyF32>::unwrapped, &Ops<SaxpyF32>::occupancy, nullptr, &Ops<SaxpyF32>::clc,
+     &Ops<SaxpyF32>::worker_sw, &Ops<SaxpyF32>::occupancy_sw},
     {FLEP_BODY_SPMV_CSR_F32, Spmv::kThreads, sizeof(flep_spmv_args), &Ops<Spmv>::worker,
-     &Ops<Spmv>::unwrapped, &Ops<Spmv>::occupancy, nullptr, &Ops<Spmv>::clc},
+     &Ops<Spmv>::unwrapped, &Ops<Spmv>::occupancy, nullptr, &Ops<Spmv>::clc,
+     &Ops<Spmv>::worker_sw, &Ops<Spmv>::occupancy_sw},
     {FLEP_BODY_STENCIL5_F32, StencilF32::kThreads, sizeof(flep_stencil_args), &Ops<StencilF32>::worker,
-     &Ops<StencilF32>::unwrapped, &Ops<StencilF32>::occupancy, nullptr, &Ops<StencilF32>::clc},
+     &Ops<StencilF32>::unwrapped, &Ops<StencilF32>::occupancy, nullptr, &Ops<StencilF32>::clc,
+     &Ops<StencilF32>::worker_sw, &Ops<StencilF32>::occupancy_sw},
     {FLEP_BODY_STENCIL5_I32, StencilI32::kThreads, sizeof(flep_stencil_args), &Ops<StencilI32>::worker,
-     &Ops<StencilI32>::unwrapped, &Ops<StencilI32>::occupancy, nullptr, &Ops<StencilI32>::clc},
+     &Ops<StencilI32>::unwrapped, &Ops<StencilI32>::occupancy, nullptr, &Ops<StencilI32>::clc,
+     &Ops<StencilI32>::worker_sw, &Ops<StencilI32>::occupancy_sw},
     {FLEP_BODY_GEMM_BF16, GemmBody::kThreads, sizeof(flep_gemm_args), &gemm_worker_launch,
-     &gemm_unwrapped_launch, &gemm_occupancy, &gemm_validate, nullptr},
+     &gemm_unwrapped_launch, &gemm_occupancy, &gemm_validate, nullptr, nullptr, nullptr},
     {FLEP_BODY_STENCIL5_F32_TMA, Stencil5TmaBody::kThreads, sizeof(flep_stencil_args), &stencil_tma_worker_launch,
-     &stencil_tma_unwrapped_launch, &stencil_tma_occupancy, &stencil_tma_validate, &stencil_tma_clc_launch},
+     &stencil_tma_unwrapped_launch, &stencil_tma_occupancy, &stencil_tma_validate, &stencil_tma_clc_launch,
+     nullptr, nullptr},
 };
 
 }  // namespace

@@ -23,6 +23,10 @@ struct BodyOps {
   // launch the CLC variant (flep_clc_worker<Body>) over the original grid of N blocks (1-D);
   // nullptr for bodies that own their loop (GEMM)
   cudaError_t (*clc)(const void* args, const WorkerParams& p, uint32_t N, cudaStream_t s, bool cov);
+  // launch W CTAs of the scheduling-warp worker (flep_worker_sw<Body>, R26) and its occupancy;
+  // nullptr for bodies that own their loop or synchronise the whole CTA inside run()
+  cudaError_t (*worker_sw)(const void* args, const WorkerParams& p, uint32_t W, cudaStream_t s, bool cov);
+  cudaError_t (*occupancy_sw)(int* ctas_per_sm, bool cov);
 };
 
 const BodyOps* body_ops(int32_t body);

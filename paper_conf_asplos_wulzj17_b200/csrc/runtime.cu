@@ -123,6 +123,7 @@ struct Launch {
   // slice_blocks blocks, at most two in flight; a preemption stops issuing
   bool sliced = false;
   bool clc = false;                  // FLEP_KFLAG_CLC: hardware work queue, resume = clear (R25)
+  bool sw = false;                   // FLEP_KFLAG_SCHED_WARP: scheduling-warp worker (R26)
   uint32_t slice_blocks = 0;
   uint64_t next_block = 0, slice_done = 0;
   std::deque<std::pair<cudaEvent_t, uint32_t>> inflight;
@@ -201,11 +202,12 @@ struct ApiLock {
   }
 };
 
-flep_status occupancy(flep_rt rt, const BodyOps* ops, bool cov, int* k) {
-  auto key = std::make_pair(ops->body, cov);
+flep_status occupancy(flep_rt rt, const BodyOps* ops, bool cov, int* k, bool sw = false) {
+  auto key = std::make_pair(ops->body * 2 + (sw ? 1 : 0), cov);
   auto it = rt->occ_cache.find(key);
   if (it != rt->occ_cache.end()) { *k = it->second; return FLEP_OK; }
-  CUDA_TRY(ops->occupancy(k, cov));
+  if (sw) CUDA_TRY(ops->occupancy_sw(k, cov));
+  else CUDA_TRY(ops->occupancy(k, cov));
   if (*k <= 0) return fail(FLEP_ERR_UNSUPPORTED, "body %d cannot be resident", ops->body);
   rt->occ_cache[key] = *k;
   return FLEP_OK;
@@ -320,6 +322,7 @@ flep_status start_epoch(flep_rt rt, Launch& L) {
   L.trig_block = kNoTrigger;
   L.trig_n = 0;
   cudaError_t e = L.clc ? L.ops->clc(L.args.data(), p, (L.n_blocks + L.chunk - 1) / L.chunk, L.exec, L.cov != nullptr)
+                 : L.sw ? L.ops->worker_sw(L.args.data(), p, L.workers, L.exec, L.cov != nullptr)
                         : L.ops->worker(L.args.data(), p, L.workers, L.exec, L.cov != nullptr);
   if (e != cudaSuccess) return fail(FLEP_ERR_CUDA, "worker launch failed: %s", cudaGetErrorString(e));
   CUDA_TRY(cudaEventRecord(L.fin_ev, L.exec));
@@ -697,8 +700,10 @@ flep_status flep_launch(flep_rt rt, flep_kernel kid, flep_dim3 grid, const void*
     if (m) return fail(FLEP_ERR_INVALID, "%s", m);
   }
   const bool cov = rt->opt.debug_coverage != 0;
+  const bool sw = (kr.flags & FLEP_KFLAG_SCHED_WARP) && !(kr.flags & FLEP_KFLAG_CLC);
+  if (sw && !ops->worker_sw) return fail(FLEP_ERR_UNSUPPORTED, "body %d has no scheduling-warp worker", kr.body);
   int k = 0;
-  s = occupancy(rt, ops, cov, &k);
+  s = occupancy(rt, ops, cov, &k, sw);
   if (s) return s;
   if (rt->free_slots.empty()) return fail(FLEP_ERR_NOMEM, "out of status slots");
 
@@ -716,6 +721,7 @@ flep_status flep_launch(flep_rt rt, flep_kernel kid, flep_dim3 grid, const void*
   L.chunk = kr.chunk;
   L.poll = kr.poll;
   L.flags = kr.flags;
+  L.sw = sw;
   if (kr.flags & FLEP_KFLAG_CLC) {
     if (!ops->clc) return fail(FLEP_ERR_UNSUPPORTED, "body %d has no CLC variant", kr.body);
     if (rt->opt.policy == FLEP_POLICY_SLICE) return fail(FLEP_ERR_UNSUPPORTED, "CLC kernels cannot be sliced");

@@ -23,7 +23,8 @@ def main():
     from paper_conf_asplos_wulzj17_b200.calibrate import dither, event_mean_us
     from bench import L2Flush
     build.build()
-    combos = [tuple(map(int, c.split(":"))) for c in
+    # C:K:prefetch:async[:sched_warp]
+    combos = [(tuple(map(int, c.split(":"))) + (0,))[:5] for c in
               (sys.argv[1] if len(sys.argv) > 1 else "1:1:0:0,2:1:1:1,4:1:0:0,8:1:0:0").split(",")]
     rt = F.Runtime(exec_on_user_stream=True)
     flush = L2Flush(torch)
@@ -58,8 +59,8 @@ def main():
         tu, _ = timed(lambda: rt.launch_unwrapped(body, grid, args, stream=s))
         print(json.dumps({"body": name, "variant": "unwrapped", "event_us": round(event_mean_us(tu), 3),
                           "event_min_us": round(min(tu), 3)}), flush=True)
-        for C, K, pf, ap in combos:
-            kk = rt.register_kernel(body, chunk=C, poll=K, prefetch=bool(pf), async_poll=bool(ap))
+        for C, K, pf, ap, sw in combos:
+            kk = rt.register_kernel(body, chunk=C, poll=K, prefetch=bool(pf), async_poll=bool(ap), sched_warp=bool(sw))
             tw, hs = timed(lambda: rt.launch(kk, grid, args, stream=s))
             ev = rt.events(hs[-1], 1)
             ent = np.array([e.t_entry for e in ev], dtype=np.int64)
@@ -67,7 +68,7 @@ def main():
             nb = np.array([e.n_blocks for e in ev])
             t0 = ent.min()
             print(json.dumps({
-                "body": name, "variant": "wrapped", "C": C, "K": K, "prefetch": pf, "async_poll": ap,
+                "body": name, "variant": "wrapped", "C": C, "K": K, "prefetch": pf, "async_poll": ap, "sched_warp": sw,
                 "workers": len(ev), "event_us": round(event_mean_us(tw), 3), "event_min_us": round(min(tw), 3),
                 "ramp_us": round((ent.max() - t0) / 1e3, 3),
                 "span_us": round((ext.max() - t0) / 1e3, 3),
