@@ -269,9 +269,10 @@ def tune_amortizing_factor(rt, torch, body, grid, args, flush, bound=0.04, candi
     by_l = {}
     for cand in candidates:
         c, k, pf, ap, clc, sw = (tuple(cand) + (False, False))[:6]
-        if body in (F.BODY_GEMM_BF16, F.BODY_STENCIL5_F32_TMA) and (pf or clc or sw) and \
-                not (body == F.BODY_STENCIL5_F32_TMA and clc):
-            continue                          # (in-tile GEMM: no prefetch/CLC; TMA stencil: no sched warp)
+        if body == F.BODY_GEMM_BF16 and (pf or clc or sw):
+            continue                          # in-tile GEMM: no prefetch, CLC or scheduling warp
+        if body == F.BODY_STENCIL5_F32_TMA and sw:
+            continue                          # the TMA stencil synchronises the whole CTA in run()
         by_l.setdefault(c * k, []).append((c, k, pf, ap, clc, sw))
     for L in sorted(by_l):
         for c, k, pf, ap, clc, sw in by_l[L]:
