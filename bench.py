@@ -516,7 +516,8 @@ def run_reference(args, rank, world):
     from oracle import workloads as W
     rowptr, col, val, x = gen.csr_inputs(SPMV_ROWS, seed=2)
     st_in = gen.stencil_f32_input(STENCIL_N, seed=3)
-    n_lp = (SPMV_ROWS + 127) // 128
+    from paper_conf_asplos_wulzj17_b200.flep import SPMV_ROWS_PER_BLOCK
+    n_lp = (SPMV_ROWS + SPMV_ROWS_PER_BLOCK - 1) // SPMV_ROWS_PER_BLOCK
     g = gen.rng(1000)
     lats, steps_ms = [], []
     for i in range(args.warmup + args.steps):

@@ -17,6 +17,9 @@
 #ifndef FLEP_SPMV_U
 #define FLEP_SPMV_U 4
 #endif
+#ifndef FLEP_SPMV_ROWS
+#define FLEP_SPMV_ROWS 128           // rows per original block (flep.py SPMV_ROWS_PER_BLOCK)
+#endif
 
 namespace flep {
 
@@ -93,7 +96,7 @@ struct SaxpyBody : NoResources {
 struct SpmvBody : NoResources {
   static constexpr int kThreads = 256;
   static constexpr int kMinBlocks = 8;
-  static constexpr uint32_t kRowsPerBlock = 128;
+  static constexpr uint32_t kRowsPerBlock = FLEP_SPMV_ROWS;
   static constexpr uint32_t kTile = 2048;
   using Args = flep_spmv_args;
 

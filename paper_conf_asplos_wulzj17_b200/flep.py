@@ -387,7 +387,7 @@ def saxpy_grid(n):
     return ((n + 255) // 256, 1, 1)
 
 
-SPMV_ROWS_PER_BLOCK = 128
+SPMV_ROWS_PER_BLOCK = int(os.environ.get("FLEP_SPMV_ROWS", "128"))   # = FLEP_SPMV_ROWS of the build
 
 
 def spmv_grid(rows):
