@@ -504,14 +504,19 @@ void monitor_loop(flep_rt rt) {
   int64_t deadline = -1;
   bool pending_release = false;
   uint64_t gen_seen = ~0ull;
+  uint32_t spin = 0;
   while (!rt->stop.load(std::memory_order_relaxed)) {
     bool hit = false;
     if (gen_seen != rt->active_gen.load(std::memory_order_acquire)) hit = true;   // new work
     moved.clear();
+    // the pinned words every pass (a plain load); the completion events of silent DONE epochs
+    // (R24) every 8th pass: cudaEventQuery takes a driver lock that the application's launches
+    // also need, and the PREEMPTED word is the latency-critical notification
+    const bool query_events = (++spin & 7u) == 0;
     for (const Watch& w : watch) {
       if (w.sliced) { hit = true; continue; }
       if (__atomic_load_n(w.word, __ATOMIC_ACQUIRE) != w.seen ||
-          (w.ev && cudaEventQuery(w.ev) == cudaSuccess)) {   // a DONE epoch is silent (R24)
+          (query_events && w.ev && cudaEventQuery(w.ev) == cudaSuccess)) {
         hit = true; moved.push_back({w.id, now_ns()});
       }
     }
