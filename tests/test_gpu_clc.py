@@ -92,6 +92,15 @@ def test_clc_spmv_matches_counter_variant_bitwise(rt, torch_mod):
     assert _rel_err(y1.cpu().numpy(), ref, absum) <= REL_FP32
 
 
+def _resume_unless_done(rt, f, h):
+    # a preempted CLC grid keeps completing chunks (its queued CTAs still start), so it may finish
+    # between a state query and the resume
+    try:
+        rt.resume(h)
+    except f.FlepError:
+        assert rt.query(h).state == f.STATE_DONE
+
+
 def _long_lp(rt, f, n_log2=27, seed=34, **kw):
     n = 1 << n_log2
     x, y = gen.saxpy_i32_inputs(n, seed=seed)
@@ -112,12 +121,10 @@ def test_clc_temporal_preempt_hands_sms_to_waiting_kernel(rt, torch_mod):
     h = rt.launch(k, f.saxpy_grid(n), f.saxpy_i32_args(yd, xd, 3), priority=0)
     time.sleep(50e-6)
     rt.preempt(h, rt.num_sms)
-    assert rt.query(h).state == f.STATE_PREEMPTED          # in force at once (R25)
+    assert rt.query(h).state in (f.STATE_PREEMPTED, f.STATE_DONE)   # in force at once (R25)
     h2 = rt.launch(k_hp, f.saxpy_grid(n2), f.saxpy_i32_args(y2d, x2d, 5), priority=1)
     rt.sync(h2, timeout_ns=10_000_000_000)
-    st = rt.query(h).state
-    if st != f.STATE_DONE:
-        rt.resume(h)
+    _resume_unless_done(rt, f, h)
     rt.sync(h, timeout_ns=20_000_000_000)
     torch_mod.cuda.synchronize()
     nb = n // 256
@@ -138,8 +145,7 @@ def test_clc_spatial_request_yields_only_named_sms(rt, torch_mod):
     rt.preempt(h, nsm)
     assert rt.query(h).state in (f.STATE_PARTIAL, f.STATE_DONE)
     time.sleep(200e-6)
-    if rt.query(h).state != f.STATE_DONE:
-        rt.resume(h)
+    _resume_unless_done(rt, f, h)
     rt.sync(h, timeout_ns=20_000_000_000)
     ev = rt.events(h, 1)
     yielded = [e for e in ev if e.reason == f.REASON_YIELD]
