@@ -295,6 +295,16 @@ def run_temporal(args, rank, world, local):
     # The SpMV's algorithmic bytes stream at a fraction of HBM speed because its x[col[p]] gathers
     # are random 4-B reads of an L2-resident vector: one 32-B sector request per nonzero. Its real
     # ceiling is the measured random-gather rate (probes/probe6.cu: same x size and nnz).
+    # latency budget: the drain against one chunk of the victim (a worker stops at
+    # its next poll, i.e. after the chunk it is running: at C = K = 1 the drain is bounded by one
+    # chunk's execution time plus the exit), with the chunk time from the standalone wrapped run
+    _, w_lp = rt.workers_for(F.BODY_SPMV_CSR_F32)
+    chunk_us = kern["spmv"]["wrapped_us"] * w_lp * args.lp_chunk / n_lp
+    latency_budget = {"drain_p50_us": round(d50, 3), "victim_chunk_us": round(chunk_us, 3),
+                      "drain_over_chunk": round(d50 / chunk_us, 3) if chunk_us else None,
+                      "definition": "victim chunk time = standalone wrapped SpMV time x W x C / N (each of "
+                                    "the W workers runs N/(W C) chunks back to back)",
+                      "kernel_boundary_us": 2.36, "kernel_boundary_source": "profiles/r01_probe_exit_accounting.jsonl (empty grid, back to back)"}
     gpk = load_gather_peak()
     g_ach = wl.nnz / (kern["spmv"]["wrapped_us"] * 1e-6)
     gather_roofline = {"bound": "l1_gather", "kernel": "flep_worker<spmv>", "achieved": float(f"{g_ach:.4g}"),
@@ -337,6 +347,7 @@ def run_temporal(args, rank, world, local):
                      "max": round(max(drain), 3) if drain else None},
         "hp_turnaround_us": {"p50": round(float(np.median(hpt)), 3) if hpt else None},
         "target_20us_met": bool(drain) and max(drain) < 20.0,
+        "latency_budget": latency_budget,
         "wrapper_overhead_pct": {k: v["overhead_pct"] for k, v in kern.items()},
         "kernels": kern,
         "roofline": roofline,
