@@ -562,7 +562,7 @@ def main():
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--impl", default="flep", choices=["flep", "reference"])
-    ap.add_argument("--config", default="temporal", choices=["temporal", "corun1", "spatial", "queue", "ffs", "model", "gemm", "tune", "clc", "delay"])
+    ap.add_argument("--config", default="temporal", choices=["temporal", "corun1", "spatial", "queue", "ffs", "model", "gemm", "tune", "clc", "delay", "spatial_f1"])
     ap.add_argument("--model-train", type=int, default=100)
     ap.add_argument("--model-test", type=int, default=30)
     ap.add_argument("--overhead-runs", type=int, default=50)
@@ -618,6 +618,8 @@ def main():
             bench_configs.run_clc(args, rank, world, local)
         elif args.config == "delay":
             bench_configs.run_delay(args, rank, world, local)
+        elif args.config == "spatial_f1":
+            bench_configs.run_spatial_f1(args, rank, world, local)
         else:
             bench_configs.run_queue(args, rank, world, local)
 

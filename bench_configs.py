@@ -156,11 +156,160 @@ def run_spatial(args, rank, world, local):
            "clocks": clocks}
     if rank == 0:
         print(json.dumps(out), flush=True)
-        import os
-        dbg = os.environ.get("FLEP_EVIDENCE_DIR")
-        if dbg:
-            with open(os.path.join(dbg, "queue_debug.json"), "w") as fh:
-                json.dump(debug, fh)
+    barrier(world)
+
+
+def _rank_tables(num_sms, die):
+    """Yield orders (rank[smid]; a spatial request for n releases the SMs with rank < n):
+    ascending smid (the paper's ID < spa_P), die-packed (one die's SMs first) and die-balanced
+    (the dies alternate), from a measured smid -> die map (probes/probe7.cu)."""
+    tables = {"ascending": list(range(num_sms))}
+    if die is None or len(die) < num_sms:
+        return tables
+    d0 = [s for s in range(num_sms) if die[s] == 0]
+    d1 = [s for s in range(num_sms) if die[s] == 1]
+    packed = d0 + d1
+    balanced = [x for pair in zip(d0, d1) for x in pair] + d0[len(d1):] + d1[len(d0):]
+    for name, order in (("die_packed", packed), ("die_balanced", balanced)):
+        r = [0] * num_sms
+        for k, smid in enumerate(order):
+            r[smid] = k
+        tables[name] = r
+    return tables
+
+
+def run_spatial_f1(args, rank, world, local):
+    """SURVEY f1 beyond refill (Fig. 16): a 16384^2 stencil victim (counter worker,
+    C = K = 1) yields n SMs to a SAXPY-f32 waiting kernel.
+    (A) "More than enough SMs": the waiting kernel is sized for n_need = 8 SMs (8 x k_wait CTAs)
+        and the request yields n = 8, 12, 16, 24, 32: waiting-kernel turnaround (request -> its
+        last CTA), co-run time T_FLEP and its overhead over T_org.
+    (B) Which SMs: rank tables ascending smid (paper), die-packed and die-balanced (measured
+        smid -> die map, FLEP_DIE_MAP or profiles/r01_sm_die_map.json) at n = 16, 32, 74 with the
+        waiting kernel sized for n SMs: yield latency, waiting turnaround, overhead; I3 checked
+        against each table."""
+    import os
+    import torch
+    from bench import ClockSampler, L2Flush, barrier, physical_gpu_index, ROOT
+    from paper_conf_asplos_wulzj17_b200 import flep as F
+    torch.cuda.set_device(local)
+    rt = F.Runtime(device=local, exec_on_user_stream=True)
+    die_path = os.environ.get("FLEP_DIE_MAP") or os.path.join(ROOT, "profiles", "r01_sm_die_map.json")
+    try:
+        with open(die_path) as fh:
+            die = json.load(fh)["die"]
+    except Exception:
+        die = None
+    n_st = 16384
+    g = torch.Generator(device="cuda")
+    g.manual_seed(4 + rank)
+    v_in = torch.rand(n_st, n_st, device="cuda", generator=g)
+    v_out = torch.empty_like(v_in)
+    k_v = rt.register_kernel(F.BODY_STENCIL5_F32, chunk=1, poll=1, name="victim")
+    k_w = rt.register_kernel(F.BODY_SAXPY_F32, chunk=1, poll=1, name="waiting")
+    cps_w, _ = rt.workers_for(F.BODY_SAXPY_F32)
+    n_max = 74 * cps_w * 256
+    wx = torch.rand(n_max, device="cuda", generator=g)
+    wy = torch.rand(n_max, device="cuda", generator=g)
+    flush = L2Flush(torch)
+    A = torch.cuda.Stream(priority=-2)
+    B = torch.cuda.Stream(priority=0)
+    v_args, v_grid = F.stencil_args(v_out, v_in), F.stencil_grid(n_st)
+    n_v = v_grid[0] * v_grid[1]
+    rng = gen.rng(3000 + rank)
+
+    def w_args(n):
+        elems = n * cps_w * 256
+        return F.saxpy_f32_args(wy[:elems], wx[:elems], 0.5), F.saxpy_grid(elems)
+
+    def alone(k, grid, a):
+        flush.zero_()
+        torch.cuda.synchronize()
+        h = rt.launch(k, grid, a, stream=A)
+        rt.sync(h)
+        t0, t1 = _span(rt.events(h, 1))
+        return (t1 - t0) / 1e3
+
+    def trials(n, wa, wg, table, reps):
+        lat, wturn, tflep, viol = [], [], [], 0
+        for trial in range(reps + 2):
+            tstar = int(rng.integers(n_v // 4, n_v // 2))
+            flush.zero_()
+            torch.cuda.synchronize()
+            rt.arm_next_trigger(tstar, n)
+            h_v = rt.launch(k_v, v_grid, v_args, priority=0, stream=A)
+            h_w = rt.launch(k_w, wg, wa, priority=1, stream=B)
+            rt.wait_epoch(h_v, timeout_ns=10_000_000_000)
+            if rt.query(h_v).state == F.STATE_PREEMPTED:
+                rt.sync(h_w, timeout_ns=10_000_000_000)
+                rt.resume(h_v)
+            rt.sync(h_v, timeout_ns=10_000_000_000)
+            rt.sync(h_w, timeout_ns=10_000_000_000)
+            info = rt.query(h_v)
+            ep = rt.epoch_info(h_v, 1)
+            ev1 = rt.events(h_v, 1)
+            evs = list(ev1)
+            for e_ in range(2, info.epoch + 1):
+                evs += list(rt.events(h_v, e_))
+            evw = rt.events(h_w, 1)
+            if trial < 2 or ep.t_trigger == 0:
+                continue
+            viol += sum(1 for e in ev1 if (e.reason == F.REASON_YIELD) != (table[e.smid] < n))
+            y = [e.t_exit for e in ev1 if e.reason == F.REASON_YIELD]
+            if y:
+                lat.append((max(y) - ep.t_trigger) / 1e3)
+            v0, v1 = _span(evs)
+            w0, w1 = _span(evw)
+            wturn.append((w1 - ep.t_trigger) / 1e3)
+            tflep.append((max(v1, w1) - v0) / 1e3)
+        med = lambda v: round(float(np.median(v)), 3) if v else None  # noqa: E731
+        return {"yield_latency_us_p50": med(lat), "waiting_turnaround_us_p50": med(wturn),
+                "t_flep_us": med(tflep), "I3_violations": viol, "trials": len(tflep)}
+
+    for _ in range(2):
+        alone(k_v, v_grid, v_args)
+    t_v = float(np.median([alone(k_v, v_grid, v_args) for _ in range(5)]))
+    reps = max(10, args.steps // 4)
+    more, which = [], []
+    tables = _rank_tables(rt.num_sms, die)
+    with ClockSampler(physical_gpu_index(local)) as clk:
+        rt.set_rank_table(tables["ascending"])
+        wa, wg = w_args(8)
+        t_w8 = float(np.median([alone(k_w, wg, wa) for _ in range(5)]))
+        for n in (8, 12, 16, 24, 32):
+            r = trials(n, wa, wg, tables["ascending"], reps)
+            t_org = t_v + t_w8
+            r.update({"n_need": 8, "n_sms": n, "t_org_us": round(t_org, 2), "t_waiting_alone_us": round(t_w8, 2),
+                      "overhead": round((r["t_flep_us"] - t_org) / t_org, 4) if r["t_flep_us"] else None})
+            more.append(r)
+        for name, table in tables.items():
+            rt.set_rank_table(table)
+            for n in (16, 32, 74):
+                wa, wg = w_args(n)
+                t_w = float(np.median([alone(k_w, wg, wa) for _ in range(3)]))
+                r = trials(n, wa, wg, table, reps)
+                t_org = t_v + t_w
+                r.update({"table": name, "n_sms": n, "t_org_us": round(t_org, 2),
+                          "overhead": round((r["t_flep_us"] - t_org) / t_org, 4) if r["t_flep_us"] else None})
+                which.append(r)
+        rt.set_rank_table(tables["ascending"])
+    rt.close()
+    base = more[0]["waiting_turnaround_us_p50"]
+    for r in more:
+        r["waiting_speedup_vs_n_need"] = round(base / r["waiting_turnaround_us_p50"], 3) \
+            if base and r["waiting_turnaround_us_p50"] else None
+    best = max((r["waiting_speedup_vs_n_need"] or 0) for r in more)
+    out = {"metric": METRIC, "value": best, "unit": "x",
+           "value_definition": "largest waiting-kernel turnaround speedup from yielding more SMs than its grid "
+                               "needs (n_need = 8), P:383 Fig. 16",
+           "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "higher_is_better": True,
+           "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic (seeded)",
+           "config": {"workload": "stencil5 fp32 16384^2 victim (C=K=1) spatially preempted by SAXPY-f32",
+                      "die_map": die_path if die else None, "trials_per_point": reps,
+                      "l2": "flushed between trials"},
+           "more_than_enough": more, "rank_tables": which, "clocks": clk.summary()}
+    if rank == 0:
+        print(json.dumps(out), flush=True)
     barrier(world)
 
 

@@ -287,3 +287,33 @@ def test_spatial_refill_exactly_once(tail):
             assert np.array_equal(yd.cpu().numpy(), ref)
     finally:
         rt.close()
+
+
+def test_custom_rank_table_spatial_yield():
+    """flep_set_rank_table: a spatial request for n SMs releases exactly the SMs whose
+    rank is below n, for a non-identity table; then the identity table is restored."""
+    f = flep_mod()
+    import torch
+    rt = f.Runtime(coverage=True)
+    try:
+        S = rt.num_sms
+        table = [(S - 1 - s) for s in range(S)]          # reversed: the highest smids yield first
+        rt.set_rank_table(table + list(range(S, rt.nsmid)) if rt.nsmid > S else table)
+        n = 4096
+        a = gen.stencil_f32_input(n, seed=61)
+        ind = t(a)
+        outd = torch.empty_like(ind)
+        k = rt.register_kernel(f.BODY_STENCIL5_F32, chunk=1, poll=1)
+        nb = (n // 64) ** 2
+        for nsm in (8, 37):
+            rt.arm_next_trigger(nb // 4, nsm)
+            h = rt.launch(k, f.stencil_grid(n), f.stencil_args(outd, ind))
+            rt.sync(h)
+            ev = rt.events(h, 1)
+            assert any(e.reason == f.REASON_YIELD for e in ev)
+            for e in ev:
+                assert (e.reason == f.REASON_YIELD) == (table[e.smid] < nsm)
+            assert np.all(rt.coverage_np(h, nb) == 1)
+        rt.set_rank_table(list(range(max(S, rt.nsmid))))
+    finally:
+        rt.close()

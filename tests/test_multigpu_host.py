@@ -66,3 +66,18 @@ def test_assign_jobs_single_gpu_keeps_order():
     jobs = gen.queue_trace(5, 40, 10_000)
     parts = bench_configs.assign_jobs(jobs, lambda j: 1000, 1)
     assert [j["id"] for j in parts[0]] == list(range(40))
+
+
+def test_rank_tables_are_permutations_and_follow_the_die_map():
+    import bench_configs as bc
+    die = [0, 1, 1, 0, 0, 1, 0, 1]
+    t = bc._rank_tables(8, die)
+    for name, r in t.items():
+        assert sorted(r) == list(range(8)), name
+    # die-packed: every die-0 SM ranks before every die-1 SM (a request for <= 4 SMs takes die 0)
+    assert max(t["die_packed"][s] for s in range(8) if die[s] == 0) < min(t["die_packed"][s] for s in range(8) if die[s] == 1)
+    # die-balanced: any even prefix of ranks holds as many SMs of each die
+    inv = sorted(range(8), key=lambda s: t["die_balanced"][s])
+    for k in (2, 4, 6, 8):
+        assert sum(die[s] for s in inv[:k]) == k // 2
+    assert bc._rank_tables(8, None) == {"ascending": list(range(8))}
