@@ -6,7 +6,8 @@
 // bit-identical outputs (SURVEY §8(c) "Parity criteria").
 //
 //   SAXPY  (VA-shaped, Table 1): block b = elements [256b, 256b+256); 128-bit ld/st.
-//   SpMV   (SPMV): block b = rows [128b, 128b+128); CSR-stream, fixed-order row sums.
+//   SpMV   (SPMV): block b = rows [128b, 128b+128); CSR-stream, fixed-order row sums (a
+//          CSR-vector form with 4 lanes per row is FLEP_SPMV_VECTOR=1).
 //   Stencil5 (BJ "2D stencil"; PF/CFD-shaped): block (tx, ty) = 64x64 output tile; each thread
 //          produces a 4x4 patch with 128-bit loads; halo rows/columns come from L1/L2.
 #pragma once
@@ -16,6 +17,10 @@
 
 #ifndef FLEP_SPMV_U
 #define FLEP_SPMV_U 4
+#endif
+#ifndef FLEP_SPMV_VECTOR
+#define FLEP_SPMV_VECTOR 0           // 0: CSR-stream body (products staged in shared memory);
+                                     // 1: CSR-vector body (4 lanes per row, shuffle reduction)
 #endif
 #ifndef FLEP_SPMV_ROWS
 #define FLEP_SPMV_ROWS 128           // rows per original block (flep.py SPMV_ROWS_PER_BLOCK)
@@ -87,7 +92,10 @@ struct SaxpyBody : NoResources {
 
 // ---------------------------------------------------------------------------------------------
 // SpMV-CSR fp32: y[r] = sum_p val[p] * x[col[p]]. Block b = rows [128b, 128b+128).
-// CSR-stream form: the rowptr slice of up to 256 rows (two blocks of a chunk; one block in the
+// Default: the CSR-stream form. The CSR-vector form (FLEP_SPMV_VECTOR=1) is 4 % faster unwrapped
+// and 2.5 % as the C = 1 worker (profiles/r01_spmv_vector.jsonl) but its warps finish a block at
+// more spread-out times (rows of different lengths per warp), which lengthened the victim's
+// drain from 9.1 to 10.2 us p50 (r01_bench_spmv_vector.json): latency wins here. CSR-stream: the rowptr slice of up to 256 rows (two blocks of a chunk; one block in the
 // unwrapped kernel) goes to smem; all 256 threads then stream the rows' contiguous nnz range in
 // tiles of kTile entries (coalesced col/val loads, independent x gathers, U in flight per thread),
 // writing products to smem; thread t sums row r0+t's products in ascending p order. Per-row
@@ -102,6 +110,43 @@ struct SpmvBody : NoResources {
 
   static constexpr uint32_t kGroupRows = 256;     // rows streamed together (2 blocks of a chunk)
 
+#if FLEP_SPMV_VECTOR
+  // CSR-vector form: 4 lanes per row (8 rows per warp, 64 rows per CTA pass); lane l of a row's
+  // group takes the row's nonzeros p = s+l, s+l+4, ... in ascending order (U in flight), and the
+  // group's 4 partial sums are combined by two butterfly shuffles (every lane ends with the same
+  // bits). No shared memory and no CTA barrier; the order is fixed, so wrapped, unwrapped and
+  // resumed runs stay bit-identical.
+  __device__ static void run(const Args& g, uint32_t b0, uint32_t b1, uint32_t, uint32_t) {
+    constexpr int U = FLEP_SPMV_U;
+    const uint32_t tid = threadIdx.x;
+    const int32_t sub = (int32_t)(tid & 3u);
+    const uint32_t row_end = min(b1 * kRowsPerBlock, g.rows);
+    for (uint32_t r0 = b0 * kRowsPerBlock; r0 < row_end; r0 += kThreads / 4) {
+      const uint32_t r = r0 + (tid >> 2);
+      const bool valid = r < row_end;
+      const int32_t s = valid ? __ldg(g.rowptr + r) : 0, e = valid ? __ldg(g.rowptr + r + 1) : 0;
+      float acc = 0.f;
+      for (int32_t p = s + sub; p < e; p += 4 * U) {
+        int32_t c[U];
+        float v[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+          const int32_t q = p + 4 * u;
+          c[u] = q < e ? __ldcs(g.col + q) : 0;
+          v[u] = q < e ? __ldcs(g.val + q) : 0.f;
+        }
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+          const float xv = __ldg(g.x + c[u]);
+          if (p + 4 * u < e) acc += v[u] * xv;
+        }
+      }
+      acc += __shfl_xor_sync(0xffffffffu, acc, 1);
+      acc += __shfl_xor_sync(0xffffffffu, acc, 2);
+      if (valid && sub == 0) __stcs(g.y + r, acc);
+    }
+  }
+#else
   __device__ static void run(const Args& g, uint32_t b0, uint32_t b1, uint32_t, uint32_t) {
     __shared__ int32_t s_rp[kGroupRows + 1];
     __shared__ float s_prod[kTile];
@@ -146,6 +191,7 @@ struct SpmvBody : NoResources {
       if (tid < nr) __stcs(g.y + r0 + tid, acc);
     }
   }
+#endif
 };
 
 // ---------------------------------------------------------------------------------------------
