@@ -107,7 +107,8 @@ def test_random_schedules_10k_zero_violations():
         xd, y0, yd = t(x), t(y), t(y)
         kern = {}
         viol_total, preempted_total, yielded_total, bad = 0, 0, 0, []
-        n_sched = 10_000
+        import os
+        n_sched = int(os.environ.get("FLEP_SCHEDULES", "10000"))   # evidence runs use 10^5
         for i in range(n_sched):
             s = gen.preempt_schedule(100 + i, nb, rt.num_sms)
             pf = i % 2 == 1
