@@ -316,6 +316,9 @@ def run_temporal(args, rank, world, local):
                 "algorithmic_bytes": algo, "peak_source": peak_src}
 
     e2e = run_e2e(F, torch, wl, local, args.e2e_steps, args)
+    _diag = run_e2e(F, torch, wl, local, args.e2e_steps, args, diag=True)
+    e2e["breakdown_us_p50"] = _diag.get("breakdown_us_p50")
+    e2e["breakdown_steps"] = _diag.get("diag_points")
     rt.close()
 
     out = {
@@ -439,7 +442,7 @@ def load_traffic(dom):
         return None
 
 
-def run_e2e(F, torch, wl, local, steps, args):
+def run_e2e(F, torch, wl, local, steps, args, diag=False):
     """Same metric through the managed public API (HPF policy), with host buffers: every step
     copies the inputs from pinned host memory, the HP arrival is an intercepted flep_launch that
     makes the runtime preempt the running LP, and the outputs are read back. Latency = host
@@ -460,7 +463,7 @@ def run_e2e(F, torch, wl, local, steps, args):
     hp_args = F.stencil_args(wl.d_out, wl.d_in)
     h2d = sum(t.numel() * t.element_size() for t in (h_rp, h_col, h_val, h_x, h_in))
     d2h = h_y.numel() * 4 + h_out.numel() * 4
-    lats, step_ms, pre = [], [], 0
+    lats, step_ms, pre, parts, dev = [], [], 0, [], []
     for i in range(steps + 2):
         t0 = time.perf_counter()
         with torch.cuda.stream(A):
@@ -473,7 +476,20 @@ def run_e2e(F, torch, wl, local, steps, args):
         t_w = time.perf_counter()
         while rt.query(h_lp).started_epoch < 1 and time.perf_counter() - t_w < 1.0:
             pass                                   # the HP arrives while the LP is running
+        t_started_seen = F.now_ns()
+        t_l0 = F.now_ns()
         h_hp = rt.launch(kHP, F.stencil_grid(STENCIL_N), hp_args, priority=1, stream=B)
+        t_l1 = F.now_ns()
+        ev = []
+        if diag:      # read the victim's first-epoch worker log while it is preempted (before release)
+            t_d = time.perf_counter()
+            while rt.query(h_lp).state not in (F.STATE_PREEMPTED, F.STATE_DONE) and time.perf_counter() - t_d < 1.0:
+                pass
+            if rt.query(h_lp).state == F.STATE_PREEMPTED:
+                try:
+                    ev = rt.events(h_lp, 1)
+                except F.FlepError:
+                    ev = []
         rt.sync(h_hp, timeout_ns=10_000_000_000)
         rt.sync(h_lp, timeout_ns=10_000_000_000)
         with torch.cuda.stream(A):
@@ -489,6 +505,17 @@ def run_e2e(F, torch, wl, local, steps, args):
             if info.epoch >= 2 and info.t_last_drain > 0:
                 pre += 1
                 lats.append((info.t_last_drain - info.t_last_request) / 1e3)
+                parts.append(((info.t_last_request - t_l0) / 1e3, (t_l1 - info.t_last_request) / 1e3))
+                # device <-> host clock: worker 0 publishes "started" right after stamping t_entry,
+                # and the host saw it at t_started_seen (offset error: one PCIe write + a poll)
+                w0 = [e for e in ev if e.t_entry > 0]
+                if w0:
+                    off = t_started_seen - min(e.t_entry for e in w0)      # host - device
+                    ys = [e.t_exit for e in ev if e.reason == F.REASON_YIELD]
+                    if ys:
+                        dev.append(((min(ys) + off - info.t_last_request) / 1e3,
+                                    (max(ys) - min(ys)) / 1e3,
+                                    (info.t_last_drain - (max(ys) + off)) / 1e3))
     dec = rt.decision_log()
     rt.close()
     return {"value": round(float(np.median(lats)), 3) if lats else None, "unit": "us",
@@ -497,7 +524,15 @@ def run_e2e(F, torch, wl, local, steps, args):
             "definition": "host clock: HPF runtime's preemption request (cuStreamWriteValue32 issued) -> "
                           "host observes the victim's drained epoch; inputs H2D from pinned memory and "
                           "outputs D2H inside every step",
-            "decisions_last": [F.ACTION_NAMES[d[1]] for d in dec[-4:]]}
+            "decisions_last": [F.ACTION_NAMES[d[1]] for d in dec[-4:]],
+            "host_path_us_p50": {"launch_call_to_request": round(float(np.median([a for a, _ in parts])), 3) if parts else None,
+                                 "request_to_launch_return": round(float(np.median([b for _, b in parts])), 3) if parts else None},
+            "diag_points": [len(dev), pre],
+            "breakdown_us_p50": ({"request_to_first_yield": round(float(np.median([a for a, _, _ in dev])), 3),
+                                  "yield_spread": round(float(np.median([b for _, b, _ in dev])), 3),
+                                  "last_yield_to_host_seen": round(float(np.median([c for _, _, c in dev])), 3),
+                                  "note": "device times mapped to the host clock through the started hint "
+                                          "(error ~ one PCIe write + one poll)"} if dev else None)}
 
 
 def cpu_baseline(wl):

@@ -15,15 +15,27 @@ def main():
     import torch
     from paper_conf_asplos_wulzj17_b200 import build, flep as F
     build.build()
-    for flag in (F.FLAG_STREAM_MEMOP, F.FLAG_HOST_MAPPED):
+    body = os.environ.get("BODY", "saxpy")
+    flags = (F.FLAG_STREAM_MEMOP,) if body == "spmv" else (F.FLAG_STREAM_MEMOP, F.FLAG_HOST_MAPPED)
+    for flag in flags:
         rt = F.Runtime(exec_on_user_stream=False, flag=flag)
-        n = 1 << 28
-        x = torch.ones(n, dtype=torch.int32, device="cuda")
-        y = torch.ones(n, dtype=torch.int32, device="cuda")
-        k = rt.register_kernel(F.BODY_SAXPY_I32, chunk=8, poll=1, started_hint=True)
+        if body == "spmv":                       # the bench's victim: SpMV-CSR 2^22 rows, C = K = 1
+            from synth import gen
+            rows = 1 << 22
+            rp, col, val, xv = gen.csr_inputs(rows, seed=2)
+            T = lambda a: torch.from_numpy(a).cuda()  # noqa: E731
+            yv = torch.zeros(rows, device="cuda")
+            k = rt.register_kernel(F.BODY_SPMV_CSR_F32, chunk=1, poll=1, started_hint=True)
+            grid, kargs = F.spmv_grid(rows), F.spmv_args(yv, T(rp), T(col), T(val), T(xv))
+        else:
+            n = 1 << 28
+            x = torch.ones(n, dtype=torch.int32, device="cuda")
+            y = torch.ones(n, dtype=torch.int32, device="cuda")
+            k = rt.register_kernel(F.BODY_SAXPY_I32, chunk=8, poll=1, started_hint=True)
+            grid, kargs = F.saxpy_grid(n), F.saxpy_i32_args(y, x, 1)
         lat, dev = [], []
         for r in range(30):
-            h = rt.launch(k, F.saxpy_grid(n), F.saxpy_i32_args(y, x, 1))
+            h = rt.launch(k, grid, kargs)
             t0 = time.perf_counter()
             while rt.query(h).started_epoch < 1 and time.perf_counter() - t0 < 1:
                 pass
@@ -42,7 +54,7 @@ def main():
                 lat.append((t2 - t1) / 1e3)
                 rt.resume(h)
             rt.sync(h)
-        print(json.dumps({"flag": "stream_memop" if flag == F.FLAG_STREAM_MEMOP else "host_mapped",
+        print(json.dumps({"body": body, "flag": "stream_memop" if flag == F.FLAG_STREAM_MEMOP else "host_mapped",
                           "host_latency_us_p50": round(float(np.median(lat)), 2) if lat else None,
                           "min": round(min(lat), 2) if lat else None,
                           "yield_exit_spread_us_p50": round(float(np.median(dev)), 2) if dev else None,
