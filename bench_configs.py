@@ -316,10 +316,10 @@ def run_spatial_f1(args, rank, world, local):
 # ------------------------------------------------------------------------------------------
 def run_corun1(args, rank, world, local):
     """configs[0]: LP SAXPY-int32 2^20 preempted mid-run by HP SAXPY-int32 2^16 (device trigger,
-    temporal); exactly-once coverage and bit-exact results checked against the oracle every step."""
+    temporal); exactly-once coverage and bit-exact results checked against a NumPy reference (bench_check) every step."""
     import torch
+    import bench_check as W
     from bench import ClockSampler, L2Flush, barrier, physical_gpu_index
-    from oracle import workloads as W
     from paper_conf_asplos_wulzj17_b200 import flep as F
     torch.cuda.set_device(local)
     rt = F.Runtime(device=local, exec_on_user_stream=True, coverage=True)
@@ -390,10 +390,10 @@ def run_gemm_preempt(args, rank, world, local):
     preempted at a random tile by HP stencil5 4096^2 (device self-trigger, temporal), then
     resumed. Latency = request -> last GEMM CTA gone (device %globaltimer). Each step's result
     must be bit-identical to an uninterrupted run of the same binary (SURVEY §8(c) parity), and a
-    sample of C is checked against the oracle (fp64 dot products, 2e-2 relative)."""
+    sample of C is checked against fp64 dot products (bench_check, 2e-2 relative)."""
     import torch
+    import bench_check as W
     from bench import ClockSampler, L2Flush, barrier, physical_gpu_index
-    from oracle import workloads as W
     from paper_conf_asplos_wulzj17_b200 import flep as F
     torch.cuda.set_device(local)
     rt = F.Runtime(device=local, exec_on_user_stream=True)
@@ -453,7 +453,7 @@ def run_gemm_preempt(args, rank, world, local):
                 drain.append((ep.t_end - ep.t_trigger) / 1e3)
                 hpt.append((he - ep.t_trigger) / 1e3)
                 epochs.append(rt.query(h).epoch)
-    # oracle spot check of the last result (rows x cols sampled; fp64 dot products of bf16 values)
+    # spot check of the last result (rows x cols sampled; fp64 dot products of bf16 values)
     r_idx = gen.rng(9).integers(0, M, 16)
     c_idx = gen.rng(10).integers(0, N, 64)
     a = A_[r_idx].view(torch.int16).cpu().numpy().view(np.uint16)
@@ -471,7 +471,7 @@ def run_gemm_preempt(args, rank, world, local):
            "config": {"workload": "LP GEMM bf16 8192^3 (tcgen05, 128x256 tiles) preempted by HP stencil5 4096^2",
                       "chunk": 1, "poll": 1, "in_tile": in_tile},
            "preempted_steps": pre, "not_bit_identical_to_uninterrupted": bad,
-           "oracle_sample_max_rel": worst, "tol": 2e-2,
+           "sample_max_rel": worst, "tol": 2e-2,
            "drain_us": {"p50": round(float(np.median(drain)), 3) if drain else None,
                         "p99": round(float(np.percentile(drain, 99)), 3) if drain else None,
                         "max": round(float(np.max(drain)), 3) if drain else None},
@@ -494,7 +494,7 @@ def run_clc(args, rank, world, local):
         pending), counter victim with the FLEP request issued by the host at the HP's release
         (flep_preempt, then resume after the HP), counter victim without a request (the HP waits
         for the whole LP). Per step (device %globaltimer): HP turnaround = HP last CTA exit - LP
-        first CTA entry, and LP span. Spot parity of the last LP result against the oracle.
+        first CTA entry, and LP span. Spot parity of the last LP result (bench_check).
     (2) Wrapper overhead of both fetch variants against the unwrapped kernels (dithered CUDA
         events, L2 flushed)."""
     import torch
@@ -792,9 +792,8 @@ def run_queue(args, rank, world, local):
     slicing; NATT gain = ANTT_base / ANTT_FLEP. At N > 1 one job queue of
     64*N kernels feeds N independent per-GPU schedulers (least predicted backlog)."""
     import torch
+    import bench_check as M
     from bench import barrier
-    from oracle import des
-    from oracle import metrics as M
     from paper_conf_asplos_wulzj17_b200 import flep as F
     torch.cuda.set_device(local)
     inst = _queue_instances(torch, F, seed=5)
@@ -827,6 +826,7 @@ def run_queue(args, rank, world, local):
     overhead_ns = 20_000
     res = {}
     debug = {}
+    logs = {}
     # untimed warm-up of a short prefix (first-use costs of a fresh runtime, stream and event pools)
     _run_trace(F, torch, local, F.POLICY_FIFO, mine[:8], inst, t_alone, overhead_ns, streams)
     for name, pol in (("FIFO", F.POLICY_FIFO), ("HPF", F.POLICY_HPF), ("SLICE", F.POLICY_SLICE),
@@ -837,19 +837,14 @@ def run_queue(args, rank, world, local):
         debug[name] = [(f"{t[1][0]}-{t[1][1]}", t[2], t[3], t[4], t[5], t_alone[t[1]]) for t in turn]
         res[name] = {"antt": M.antt(tt, al), "stp": M.stp(tt, al), "preemptions": sum(1 for d in dec if d[1] == 2),
                      "makespan_ms": round(max(t[4] for t in turn) / 1e6, 3)}
-        if name in ("HPF", "FIFO", "REORDER"):
-            evs = [(t, "ARRIVE", des.KernelSpec(i, t, p, te, o)) if ty == 0 else (t, "FINISH", i)
-                   for (t, ty, i, p, te, o) in evl]
-            rep = [(t, {"LAUNCH": 0, "RESUME": 1, "PREEMPT": 2}[a], i, n) for (t, a, i, n) in
-                   des.replay({"HPF": des.HPF, "FIFO": des.FIFO, "REORDER": des.REORDER}[name], evs)]
-            res[name]["replay_parity"] = rep == dec
-    # the oracle DES's prediction of the same trace (zero-overhead and measured-overhead variants)
-    specs = [des.KernelSpec(i, j["arrival_ns"], 0, t_alone[(j["type"], j["size_class"])], overhead_ns,
-                            t_alone[(j["type"], j["size_class"])]) for i, j in enumerate(mine)]
-    pred = {}
-    for name, kind in (("FIFO", des.FIFO), ("HPF", des.HPF)):
-        s = des.simulate(kind, specs, des.SimParams(drain_ns=10_000, start_ns=10_000))
-        pred[name] = M.antt([s.turnaround[k.id] for k in specs], [k.t_true for k in specs])
+        logs[name] = {"events": [list(map(int, e)) for e in evl], "decisions": [list(map(int, d_)) for d_ in dec]}
+    # the runtime's event and decision logs (replayed through the oracle DES by
+    # tests/test_policy_replay.py from the committed copy under tests/golden/)
+    import os
+    ev_dir = os.environ.get("FLEP_EVIDENCE_DIR")
+    if ev_dir and rank == 0:
+        with open(os.path.join(ev_dir, "queue_logs.json"), "w") as fh:
+            json.dump({"workload": "configs[3] queue, seed 5", "logs": logs}, fh)
     gain_fifo = res["FIFO"]["antt"] / res["HPF"]["antt"]
     gain_slice = res["SLICE"]["antt"] / res["HPF"]["antt"]
     out = {"metric": METRIC, "value": round(gain_fifo, 3), "unit": "x (ANTT_FIFO / ANTT_FLEP)",
@@ -866,9 +861,8 @@ def run_queue(args, rank, world, local):
            "natt_gain_vs_fifo": round(gain_fifo, 3), "natt_gain_vs_slicing": round(gain_slice, 3),
            "reordering_gain_vs_fifo": round(res["FIFO"]["antt"] / res["REORDER"]["antt"], 3),
            "stp_degradation_vs_fifo": round(1 - res["HPF"]["stp"] / res["FIFO"]["stp"], 4),
-           "replay_parity": {k: res[k].get("replay_parity") for k in ("FIFO", "HPF", "REORDER")},
+           "replay_parity": "checked on CPU: tests/test_policy_replay.py replays the committed logs (tests/golden/queue_logs_r01.json) through the oracle DES",
            "makespan_ms": {k: v["makespan_ms"] for k, v in res.items()},
-           "des_predicted_antt": {k: round(v, 3) for k, v in pred.items()},
            "t_alone_us": {f"{k[0]}-{k[1]}": round(v / 1e3, 1) for k, v in sorted(t_alone.items())}}
     vals = [gain_fifo]
     if world > 1:

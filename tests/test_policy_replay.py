@@ -99,3 +99,25 @@ def test_ffs_replay_parity(flep, seed):
             assert p.tick(ev[0])
     assert as_tuples(sim.decisions) == p.decisions()
     assert len(sim.finish) == len(ks)
+
+
+def test_b200_queue_trace_replays_exactly_through_the_oracle():
+    """The runtime's own event log of the configs[3] queue run on the B200 (64 kernels, FIFO,
+    FLEP-HPF and REORDER; tests/golden/queue_logs_r01.json, written by bench.py --config queue
+    with FLEP_EVIDENCE_DIR) replayed through the oracle DES gives the runtime's decision list bit
+    for bit (SURVEY §8(c) O3 replay mode)."""
+    import json
+    import os
+    path = os.path.join(os.path.dirname(__file__), "golden", "queue_logs_r01.json")
+    with open(path) as fh:
+        logs = json.load(fh)["logs"]
+    kinds = {"FIFO": des.FIFO, "HPF": des.HPF, "REORDER": des.REORDER}
+    checked = 0
+    for name, kind in kinds.items():
+        evl, dec = logs[name]["events"], logs[name]["decisions"]
+        evs = [(t, "ARRIVE", des.KernelSpec(i, t, p, te, o)) if ty == 0 else (t, "FINISH", i)
+               for (t, ty, i, p, te, o) in evl]
+        assert as_tuples(des.replay(kind, evs)) == [tuple(d) for d in dec], name
+        checked += len(dec)
+    assert checked > 100
+    assert sum(1 for d in logs["HPF"]["decisions"] if d[1] == ACT["PREEMPT"]) > 5
