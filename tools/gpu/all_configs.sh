@@ -1,7 +1,7 @@
 #!/bin/bash
 # Every bench configuration once (round-end evidence refresh); one JSON line per file.
 mkdir -p gpurun_out/cfg
-for c in corun1 spatial gemm ffs model queue; do
+for c in corun1 spatial gemm ffs model clc delay; do
   timeout 900 python bench.py --config $c > gpurun_out/cfg/$c.json 2> gpurun_out/cfg/$c.err
   echo "$c rc=$?"
 done
