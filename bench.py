@@ -448,7 +448,8 @@ def run_e2e(F, torch, wl, local, steps, args, diag=False):
     clock from the runtime's preemption request to its observation of the drained epoch."""
     rt = F.Runtime(device=local, policy=F.POLICY_HPF)
     kLP = rt.register_kernel(F.BODY_SPMV_CSR_F32, chunk=args.lp_chunk, poll=args.lp_poll, name="spmv",
-                             model=(0, 0, 0, 0, 70_000), prefetch=bool(args.prefetch), started_hint=True)
+                             model=(0, 0, 0, 0, 70_000), prefetch=bool(args.prefetch), started_hint=True,
+                             host_relay=bool(args.e2e_relay))
     kHP = rt.register_kernel(F.BODY_STENCIL5_F32, chunk=args.hp_chunk, poll=args.hp_poll, name="stencil",
                              model=(0, 0, 0, 0, 30_000), prefetch=bool(args.hp_prefetch), async_poll=bool(args.hp_async),
                              clc=bool(args.hp_clc))
@@ -471,7 +472,8 @@ def run_e2e(F, torch, wl, local, steps, args, diag=False):
         with torch.cuda.stream(B):
             wl.d_in.copy_(h_in, non_blocking=True)
         A.synchronize()
-        B.synchronize()        # both inputs resident: no DMA runs beside the co-run
+        if not args.e2e_overlap_copy:
+            B.synchronize()    # both inputs resident: no DMA runs beside the co-run
         h_lp = rt.launch(kLP, F.spmv_grid(SPMV_ROWS), lp_args, priority=0, stream=A)
         t_w = time.perf_counter()
         while rt.query(h_lp).started_epoch < 1 and time.perf_counter() - t_w < 1.0:
@@ -524,9 +526,10 @@ def run_e2e(F, torch, wl, local, steps, args, diag=False):
             "definition": "host clock: HPF runtime's preemption request (cuStreamWriteValue32 issued) -> "
                           "host observes the victim's drained epoch; inputs H2D from pinned memory (both "
                           "copies complete before the victim starts) and outputs D2H inside every step",
-            "note": "a stream memop issued while a large H2D copy is in flight on another stream reaches "
-                    "the GPU ~20 us later (measured: 38.6 us with the waiting kernel's 67 MB input copy "
-                    "overlapping the co-run, 19 us without)",
+            "note": "the victim uses the request-relay CTA (R28): without it a stream memop issued while a "
+                    "large H2D copy is in flight reaches the GPU ~20 us later (39 us with the waiting "
+                    "kernel's 67 MB input copy overlapping the co-run vs 19.6 us with the relay)",
+            "relay": bool(args.e2e_relay), "overlap_copy": bool(args.e2e_overlap_copy),
             "decisions_last": [F.ACTION_NAMES[d[1]] for d in dec[-4:]],
             "host_path_us_p50": {"launch_call_to_request": round(float(np.median([a for a, _ in parts])), 3) if parts else None,
                                  "request_to_launch_return": round(float(np.median([b for _, b in parts])), 3) if parts else None},
@@ -617,6 +620,8 @@ def main():
     ap.add_argument("--hp-async", type=int, default=0, help="waiting kernel: async poll (R22)")
     ap.add_argument("--lp-poll", type=int, default=1)
     ap.add_argument("--reps", type=int, default=40)
+    ap.add_argument("--e2e-relay", type=int, default=1, help="e2e victim with the request-relay CTA (R28)")
+    ap.add_argument("--e2e-overlap-copy", type=int, default=0, help="e2e: let the HP's input copy overlap the co-run")
     ap.add_argument("--e2e-steps", type=int, default=10)
     ap.add_argument("--tune-bound", type=float, default=0.04, help="config tune: overhead bound (P:166: 4 %%)")
     ap.add_argument("--gemm-in-tile", type=int, default=1, help="config gemm: in-tile preemption (1) or tile granularity (0)")

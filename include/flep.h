@@ -164,6 +164,12 @@ typedef struct {
    a shared-memory ring, one chunk ahead (as FLEP_KFLAG_PREFETCH), so the body warps never wait
    for it. The CTA is kThreads + 32 threads (fewer resident CTAs per SM may fit). */
 #define FLEP_KFLAG_SCHED_WARP 32u
+/* Request relay (R28; plain counter worker of the memory-bound bodies, stream-memop
+   transport): the grid gets one extra CTA that is not a worker; its thread polls the launch's
+   pinned slot, where every request is also stored, and copies each new value into the device
+   control word, so a request reaches the workers in ~1 us instead of waiting for the stream memop
+   (~5 us, tens of us behind copy-engine work). Takes one resident slot (W = k x SMs - 1). */
+#define FLEP_KFLAG_HOST_RELAY 64u
 
 typedef enum {
   FLEP_STATE_QUEUED = 0,     /* intercepted, waiting for a scheduling decision (S2) */

@@ -41,7 +41,8 @@ struct alignas(128) ControlBlock {
   uint32_t _p1[31];
   uint32_t done_gen;       // generation whose epoch completed the launch (0 = none yet); an
                            // epoch launched after that (e.g. a refill) exits without fetching
-  uint32_t _p2[31];
+  uint32_t pub_gen;        // generation of the last published epoch (the relay CTA's exit cue, R28)
+  uint32_t _p2[30];
   // per-epoch summaries (ring of kEvEpochs)
   uint64_t ep_t_trigger[kEvEpochs];
   uint64_t ep_t_end[kEvEpochs];
@@ -88,6 +89,8 @@ struct WorkerParams {
   uint32_t gen_first;      // generation of this launch's first epoch
   uint32_t async_poll;     // 1: the poll uses the control word copied one step earlier (R22);
                            //    device-memory control word only (16-B aligned line)
+  uint32_t relay_block;    // blockIdx of the request-relay CTA (R28), 0xffffffff = none; the
+                           // relay is not a worker (W excludes it)
   uint32_t started_hint;   // 1: worker 0 publishes "epoch started" to the host slot at entry (a
                            //    system-scope store: the kernel's completion then waits for it)
   void* partial;           // in-tile preemption (FLEP_KFLAG_IN_TILE, GEMM): W partial-tile records
@@ -351,6 +354,7 @@ __device__ __forceinline__ void worker_exit(const WorkerParams& p, WorkerShared&
     p.cb->ep_t_end[ei] = t_exit; p.cb->ep_done[ei] = d; p.cb->ep_ctr[ei] = c;
     p.cb->ep_state[ei] = st;
     p.cb->ep_t_trigger[(p.epoch + 1) % kEvEpochs] = 0;  // next epoch's trigger stamp
+    st_relaxed_gpu(&p.cb->pub_gen, p.epoch);            // the relay CTA may leave (R28)
     if (done) {                                        // clean for reuse; remember completion
       p.cb->cx = 0ull;
       if (!already) p.cb->done_gen = p.epoch;
@@ -367,6 +371,28 @@ __device__ __forceinline__ void worker_exit(const WorkerParams& p, WorkerShared&
       st_relaxed_sys_u64(reinterpret_cast<uint64_t*>(&p.status->word),
                          ((uint64_t)d << 32) | ((p.epoch << 8) | st));
     }
+  }
+}
+
+// Request relay (reading R28): one extra CTA of the grid, not a worker, whose thread 0 polls the
+// host-written request word in the pinned slot and copies each new value into the device control
+// word the workers poll. A single GPU thread sees a host store in ~1 us even while copy-engine
+// work is in flight, where the stream memop takes ~5 us and tens of us behind a large H2D copy
+// (probes/probe8.cu). It leaves once the epoch is published (or a temporal request was relayed:
+// every worker then leaves at its next poll).
+__device__ __forceinline__ void request_relay(const WorkerParams& p) {
+  if (threadIdx.x != 0) return;
+  uint32_t last;
+  asm volatile("ld.relaxed.sys.global.u32 %0, [%1];" : "=r"(last) : "l"(&p.status->ctrl) : "memory");
+  while (true) {
+    uint32_t h;
+    asm volatile("ld.relaxed.sys.global.u32 %0, [%1];" : "=r"(h) : "l"(&p.status->ctrl) : "memory");
+    if (h != last) {
+      last = h;
+      atomicExch(p.ctrl, h);
+      if ((h >> 16) == (p.epoch & 0xffffu) && (h & 0xffffu) >= p.num_sms) return;
+    }
+    if (ld_relaxed_gpu(&p.cb->pub_gen) == p.epoch) return;
   }
 }
 
@@ -388,6 +414,7 @@ flep_worker(const __grid_constant__ typename Body::Args args, const WorkerParams
   __shared__ uint32_t s_slot[2];     // chunk base broadcast, double-buffered: 1 barrier per chunk
   __shared__ WorkerShared ws;        // worker bookkeeping kept out of registers (tid 0 only)
   const uint32_t tid = threadIdx.x;
+  if (blockIdx.x == p.relay_block) { request_relay(p); return; }   // R28: not a worker
   if (tid == 0) {
     ws.sm = smid_reg(); ws.t_entry = gtimer(); ws.blocks = 0; ws.reason = 0;
     ws.counted = 0; ws.last = 0; ws.ev_raw = 0; ws.ev_part = 0; ws.partial = 0;

@@ -124,6 +124,7 @@ struct Launch {
   bool sliced = false;
   bool clc = false;                  // FLEP_KFLAG_CLC: hardware work queue, resume = clear (R25)
   bool sw = false;                   // FLEP_KFLAG_SCHED_WARP: scheduling-warp worker (R26)
+  bool relay = false;                // FLEP_KFLAG_HOST_RELAY: one request-relay CTA (R28)
   uint32_t slice_blocks = 0;
   uint64_t next_block = 0, slice_done = 0;
   std::deque<std::pair<cudaEvent_t, uint32_t>> inflight;
@@ -240,6 +241,9 @@ flep_status write_ctrl(flep_rt rt, Launch& L, uint32_t value) {
     __atomic_store_n(&L.hs->ctrl, value, __ATOMIC_RELEASE);
     return FLEP_OK;
   }
+  // R28: the relay CTA reads the pinned slot; written before the memop is issued, so the host
+  // word is never older than the device word it feeds
+  if (L.relay) __atomic_store_n(&L.hs->ctrl, value, __ATOMIC_RELEASE);
   CUresult r = p_write32((CUstream)rt->ctl, (CUdeviceptr)&L.cb->ctrl, value, 0);
   if (r != CUDA_SUCCESS) return fail(FLEP_ERR_CUDA, "cuStreamWriteValue32 failed (%d)", (int)r);
   return FLEP_OK;
@@ -314,6 +318,7 @@ flep_status start_epoch(flep_rt rt, Launch& L) {
   p.prefetch = ((L.flags & FLEP_KFLAG_PREFETCH) && !(L.flags & FLEP_KFLAG_IN_TILE)) ? 1u : 0u;
   p.gen_first = L.gen0 + 1;
   p.started_hint = (L.flags & FLEP_KFLAG_STARTED_HINT) ? 1u : 0u;
+  p.relay_block = L.relay ? L.workers : 0xffffffffu;
   p.async_poll = ((L.flags & FLEP_KFLAG_ASYNC_POLL) && rt->opt.flag != FLEP_FLAG_HOST_MAPPED) ? 1u : 0u;
   p.partial = L.partial;
 #ifdef FLEP_TRACE
@@ -323,7 +328,7 @@ flep_status start_epoch(flep_rt rt, Launch& L) {
   L.trig_n = 0;
   cudaError_t e = L.clc ? L.ops->clc(L.args.data(), p, (L.n_blocks + L.chunk - 1) / L.chunk, L.exec, L.cov != nullptr)
                  : L.sw ? L.ops->worker_sw(L.args.data(), p, L.workers, L.exec, L.cov != nullptr)
-                        : L.ops->worker(L.args.data(), p, L.workers, L.exec, L.cov != nullptr);
+                        : L.ops->worker(L.args.data(), p, L.workers + (L.relay ? 1u : 0u), L.exec, L.cov != nullptr);
   if (e != cudaSuccess) return fail(FLEP_ERR_CUDA, "worker launch failed: %s", cudaGetErrorString(e));
   CUDA_TRY(cudaEventRecord(L.fin_ev, L.exec));
   L.state = FLEP_STATE_RUNNING;
@@ -735,7 +740,10 @@ flep_status flep_launch(flep_rt rt, flep_kernel kid, flep_dim3 grid, const void*
   if (kr.ctas_per_sm && (int)kr.ctas_per_sm < k) k = (int)kr.ctas_per_sm;
   const uint64_t wmax = (uint64_t)k * rt->num_sms;
   const uint64_t need = (N + L.chunk - 1) / L.chunk;
-  L.workers = (uint32_t)std::min<uint64_t>(std::min<uint64_t>(wmax, need), rt->max_workers);
+  // R28: the relay CTA takes one resident slot (plain counter worker, stream-memop transport)
+  L.relay = (kr.flags & FLEP_KFLAG_HOST_RELAY) && !L.sw && !L.clc && !ops->validate &&
+            rt->opt.flag != FLEP_FLAG_HOST_MAPPED && wmax > 1;
+  L.workers = (uint32_t)std::min<uint64_t>(std::min<uint64_t>(wmax - (L.relay ? 1 : 0), need), rt->max_workers);
   if (rt->opt.policy == FLEP_POLICY_SLICE) {
     L.sliced = true;                                  // R16: one slice = one wave of W*C*K blocks
     L.slice_blocks = rt->opt.slice_blocks ? rt->opt.slice_blocks

@@ -43,6 +43,17 @@ def main():
     C = torch.empty(256, 512, dtype=torch.bfloat16, device="cuda")
     k4 = rt.register_kernel(F.BODY_GEMM_BF16, chunk=1, poll=1)
     rt.sync(rt.launch(k4, F.gemm_grid(256, 512), F.gemm_args(C, A, B)))
+    # request-relay CTA (R28): a host preempt/resume cycle through the relay
+    k8 = rt.register_kernel(F.BODY_SAXPY_I32, chunk=1, poll=1, host_relay=True)
+    h = rt.launch(k8, F.saxpy_grid(n), F.saxpy_i32_args(yd, xd, 9))
+    try:
+        rt.preempt(h, rt.num_sms)
+        rt.wait_epoch(h)
+        if rt.query(h).state == F.STATE_PREEMPTED:
+            rt.resume(h)
+    except F.FlepError:
+        pass
+    rt.sync(h)
     # CLC task fetch: uninterrupted, then a host preempt/resume cycle
     k5 = rt.register_kernel(F.BODY_SAXPY_I32, chunk=2, poll=1, clc=True)
     rt.sync(rt.launch(k5, F.saxpy_grid(n), F.saxpy_i32_args(yd, xd, 5)))
