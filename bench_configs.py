@@ -513,8 +513,8 @@ def run_clc(args, rank, world, local):
     k_clc = rt.register_kernel(F.BODY_SPMV_CSR_F32, chunk=1, poll=1, clc=True, name="spmv_clc")
     k_ctr = rt.register_kernel(F.BODY_SPMV_CSR_F32, chunk=1, poll=1, name="spmv")
     k_hp = rt.register_kernel(F.BODY_STENCIL5_F32, chunk=4, poll=1, name="stencil")
-    variants = [("clc_no_request", k_clc, False), ("counter_flep_request", k_ctr, True),
-                ("counter_no_request", k_ctr, False)]
+    variants = [("clc_no_request", k_clc, False), ("clc_flep_request", k_clc, True),
+                ("counter_flep_request", k_ctr, True), ("counter_no_request", k_ctr, False)]
     res = {v[0]: {"hp_turnaround": [], "lp_span": [], "yields": []} for v in variants}
 
     def spin_us(us):
@@ -533,7 +533,14 @@ def run_clc(args, rank, world, local):
                     rt.preempt(h, rt.num_sms)
                 h2 = rt.launch(k_hp, hp_grid, hp_args, priority=1, stream=hi)
                 rt.sync(h2, timeout_ns=10_000_000_000)
-                if request:
+                if request and name.startswith("clc"):
+                    # a CLC request is in force at once; resume withdraws it (the preempted grid
+                    # may have completed meanwhile: its queued CTAs still start, R25)
+                    try:
+                        rt.resume(h)
+                    except F.FlepError:
+                        assert rt.query(h).state == F.STATE_DONE
+                elif request:
                     rt.wait_epoch(h, timeout_ns=10_000_000_000)
                     if rt.query(h).state == F.STATE_PREEMPTED:
                         rt.resume(h)
@@ -578,6 +585,7 @@ def run_clc(args, rank, world, local):
     xs = torch.randint(-2 ** 31, 2 ** 31 - 1, (n_sx,), dtype=torch.int32, device="cuda")
     ys = torch.randint(-2 ** 31, 2 ** 31 - 1, (n_sx,), dtype=torch.int32, device="cuda")
     cases = [("spmv", F.BODY_SPMV_CSR_F32, lp_grid, lp_args, dict(chunk=2, poll=2), dict(chunk=2, poll=2)),
+             ("spmv_c1k1", F.BODY_SPMV_CSR_F32, lp_grid, lp_args, dict(chunk=1, poll=1), dict(chunk=1, poll=1)),
              ("stencil", F.BODY_STENCIL5_F32, hp_grid, hp_args, dict(chunk=4, poll=1), dict(chunk=1, poll=4)),
              ("saxpy_i32_2^20", F.BODY_SAXPY_I32, F.saxpy_grid(n_sx), F.saxpy_i32_args(ys, xs, 3),
               dict(chunk=16, poll=2, prefetch=True, async_poll=True), dict(chunk=8, poll=2))]
