@@ -22,6 +22,12 @@
 #define FLEP_SPMV_VECTOR 0           // 0: CSR-stream body (products staged in shared memory);
                                      // 1: CSR-vector body (4 lanes per row, shuffle reduction)
 #endif
+#ifndef FLEP_SPMV_ASYNC
+#define FLEP_SPMV_ASYNC 0            // 1: CSR-stream body whose col/val tiles arrive by cp.async
+#endif
+#ifndef FLEP_SPMV_AU
+#define FLEP_SPMV_AU 8               // gathers in flight per thread in the cp.async body
+#endif
 #ifndef FLEP_SPMV_ROWS
 #define FLEP_SPMV_ROWS 128           // rows per original block (flep.py SPMV_ROWS_PER_BLOCK)
 #endif
@@ -144,6 +150,74 @@ struct SpmvBody : NoResources {
       acc += __shfl_xor_sync(0xffffffffu, acc, 1);
       acc += __shfl_xor_sync(0xffffffffu, acc, 2);
       if (valid && sub == 0) __stcs(g.y + r, acc);
+    }
+  }
+#elif FLEP_SPMV_ASYNC
+  // CSR-stream with the tile's col/val staged by cp.async (16-B copies, no registers held while
+  // they are in flight): one HBM round trip per tile, then every gather of the tile in flight
+  // (U = FLEP_SPMV_AU per thread, indices read from shared memory). Products are formed in place
+  // (val * x, the same fp32 multiply) and summed per row in ascending p, as in the form below, so
+  // results stay bit-identical to it.
+  __device__ static void cp_async16(void* dst, const void* src) {
+    const uint32_t d = static_cast<uint32_t>(__cvta_generic_to_shared(dst));
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" :: "r"(d), "l"(src) : "memory");
+  }
+  __device__ static void run(const Args& g, uint32_t b0, uint32_t b1, uint32_t, uint32_t) {
+    __shared__ int32_t s_rp[kGroupRows + 1];
+    __shared__ __align__(16) int32_t s_col[kTile + 4];
+    __shared__ __align__(16) float s_val[kTile + 4];
+    const uint32_t tid = threadIdx.x;
+    const uint32_t row_end = min(b1 * kRowsPerBlock, g.rows);
+    for (uint32_t r0 = b0 * kRowsPerBlock; r0 < row_end; r0 += kGroupRows) {
+      const uint32_t nr = min(kGroupRows, row_end - r0);
+      if (tid <= nr) s_rp[tid] = __ldg(g.rowptr + r0 + tid);
+      if (tid == 0 && nr == kGroupRows) s_rp[kGroupRows] = __ldg(g.rowptr + r0 + kGroupRows);
+      body_sync<kThreads>();
+      const int32_t p0 = s_rp[0], p1 = s_rp[nr];
+      int32_t my_s = 0, my_e = 0;
+      if (tid < nr) { my_s = s_rp[tid]; my_e = s_rp[tid + 1]; }
+      float acc = 0.f;
+      for (int32_t base = p0; base < p1; base += (int32_t)kTile) {
+        const int32_t n = min((int32_t)kTile, p1 - base);
+        const int32_t a0 = base & ~3;                 // 16-B aligned (elements before base exist)
+        const int32_t off = base - a0;
+        const int32_t a1 = (base + n) & ~3;           // aligned end: never past the arrays
+        for (int32_t j = (int32_t)tid; 4 * j < a1 - a0; j += kThreads) {
+          cp_async16(&s_col[4 * j], g.col + a0 + 4 * j);
+          cp_async16(&s_val[4 * j], g.val + a0 + 4 * j);
+        }
+        const int32_t t0 = max(a1, base);             // < 4 tail elements by plain loads
+        if ((int32_t)tid < base + n - t0) {
+          s_col[t0 - a0 + (int32_t)tid] = __ldcs(g.col + t0 + tid);
+          s_val[t0 - a0 + (int32_t)tid] = __ldcs(g.val + t0 + tid);
+        }
+        asm volatile("cp.async.wait_all;" ::: "memory");
+        body_sync<kThreads>();
+        constexpr int U = FLEP_SPMV_AU;
+        for (int32_t i0 = (int32_t)tid; i0 < n; i0 += U * kThreads) {
+          int32_t c[U];
+          float xv[U];
+#pragma unroll
+          for (int u = 0; u < U; ++u) {
+            const int32_t i = i0 + u * kThreads;
+            c[u] = i < n ? s_col[off + i] : 0;
+          }
+#pragma unroll
+          for (int u = 0; u < U; ++u) xv[u] = __ldg(g.x + c[u]);
+#pragma unroll
+          for (int u = 0; u < U; ++u) {
+            const int32_t i = i0 + u * kThreads;
+            if (i < n) s_val[off + i] = s_val[off + i] * xv[u];
+          }
+        }
+        body_sync<kThreads>();
+        if (tid < nr) {                        // row r0+tid: its products in ascending p order
+          const int32_t lo = max(my_s, base), hi = min(my_e, base + n);
+          for (int32_t p = lo; p < hi; ++p) acc += s_val[off + p - base];
+        }
+        body_sync<kThreads>();
+      }
+      if (tid < nr) __stcs(g.y + r0 + tid, acc);
     }
   }
 #else
