@@ -571,7 +571,12 @@ def run_reference(args, rank, world):
     from paper_conf_asplos_wulzj17_b200.flep import SPMV_ROWS_PER_BLOCK
     n_lp = (SPMV_ROWS + SPMV_ROWS_PER_BLOCK - 1) // SPMV_ROWS_PER_BLOCK
     g = gen.rng(1000)
-    lats, steps_ms = [], []
+    lats = []
+    # the oracle stencil (~0.6 s) is timed once, so that any --steps K stays within a few
+    # minutes; every step times the SpMV the HP must wait for (the line's value)
+    ts0 = time.perf_counter()
+    W.stencil5_f32(st_in)
+    t_st = time.perf_counter() - ts0
     for i in range(args.warmup + args.steps):
         tstar = int(g.integers(n_lp // 4, 3 * n_lp // 4))
         r0 = tstar * 128
@@ -579,11 +584,9 @@ def run_reference(args, rank, world):
         t0 = time.perf_counter()
         W.spmv_csr((rowptr[r0:] - s).astype(np.int32), col[s:], val[s:], x)
         t1 = time.perf_counter()
-        W.stencil5_f32(st_in)
-        t2 = time.perf_counter()
         if i >= args.warmup:
             lats.append((t1 - t0) * 1e6)
-            steps_ms.append((t2 - t0) * 1e3)
+    steps_ms = [lt / 1e3 + t_st * 1e3 for lt in lats]
     v = float(np.median(lats))
     out = {"impl": "reference", "metric": METRIC, "value": round(v, 1), "unit": "us", "n_gpus": world,
            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(float(np.mean(steps_ms)), 3),
@@ -592,7 +595,8 @@ def run_reference(args, rank, world):
            "config": {"workload": "configs[1]: SpMV-CSR (2^20 rows) then stencil5 4096^2 on the CPU oracle"},
            "cpu_baseline": {"value": round(v, 1), "unit": "us", "cores": 1, "kind": "oracle",
                             "sample": "per step: oracle SpMV over the LP rows after a seeded t* (what a "
-                                      "non-preemptive program must finish before the HP starts) + oracle stencil"},
+                                      "non-preemptive program must finish before the HP starts); ms_per_step adds the oracle "
+                                      "stencil, timed once per run"},
            "e2e": {"value": round(v, 1), "unit": "us", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(out), flush=True)
 
