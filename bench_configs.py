@@ -515,7 +515,8 @@ def run_clc(args, rank, world, local):
     k_hp = rt.register_kernel(F.BODY_STENCIL5_F32, chunk=4, poll=1, name="stencil")
     variants = [("clc_no_request", k_clc, False), ("clc_flep_request", k_clc, True),
                 ("counter_flep_request", k_ctr, True), ("counter_no_request", k_ctr, False)]
-    res = {v[0]: {"hp_turnaround": [], "lp_span": [], "yields": []} for v in variants}
+    res = {v[0]: {"hp_turnaround": [], "lp_span": [], "yields": [], "lp_after_hp": [], "hp_start": []}
+           for v in variants}
 
     def spin_us(us):
         t0 = time.perf_counter()
@@ -554,6 +555,7 @@ def run_clc(args, rank, world, local):
                 lp0 = min(e.t_entry for e in lp_ev)
                 hp_ev = rt.events(h2, 1)
                 hp1 = max(e.t_exit for e in hp_ev)
+                hp0 = min(e.t_entry for e in hp_ev)
                 q = rt.query(h)
                 lp_end = max(max(e.t_exit for e in lp_ev),
                              max((e.t_exit for e in rt.events(h, q.epoch)), default=0))
@@ -561,6 +563,10 @@ def run_clc(args, rank, world, local):
                 r["hp_turnaround"].append((hp1 - lp0) / 1e3)
                 r["lp_span"].append((lp_end - lp0) / 1e3)
                 r["yields"].append(sum(1 for e in lp_ev if e.reason == F.REASON_YIELD))
+                # victim CTAs that started after the waiting kernel's first CTA (refills of freed
+                # slots by the victim's own pending CTAs) and the HP's start after the LP's
+                r["lp_after_hp"].append(sum(1 for e in lp_ev if e.t_entry > hp0))
+                r["hp_start"].append((hp0 - lp0) / 1e3)
     parity = spot_parity(wl, torch)
     reps = max(args.reps, 20)
 
@@ -604,7 +610,9 @@ def run_clc(args, rank, world, local):
         return round(float(np.percentile(v, p)), 3) if v else None
     summ = {k: {"hp_turnaround_us": {"p50": q(r["hp_turnaround"], 50), "p99": q(r["hp_turnaround"], 99)},
                 "lp_span_us": {"p50": q(r["lp_span"], 50)},
-                "first_wave_yield_exits_p50": q(r["yields"], 50)} for k, r in res.items()}
+                "first_wave_yield_exits_p50": q(r["yields"], 50),
+                "hp_first_cta_us_p50": q(r["hp_start"], 50),
+                "lp_ctas_started_after_hp_p50": q(r["lp_after_hp"], 50)} for k, r in res.items()}
     out = {"metric": METRIC, "value": summ["clc_no_request"]["hp_turnaround_us"]["p50"], "unit": "us",
            "value_definition": "HP turnaround (HP last CTA exit - LP first CTA entry, device %globaltimer) with a CLC "
                                "victim and no preemption request, p50; the HP is released ~20 us after the LP",
