@@ -110,7 +110,12 @@ typedef struct {
   uint32_t default_chunk;      /* C: original blocks per counter fetch (0 -> 8) */
   uint32_t default_poll;       /* K: chunks between control-word polls (0 -> 1) */
   uint32_t debug_coverage;     /* 1: keep a per-block execution count cov[N] (test builds) */
-  uint32_t reserved0;          /* must be 0 */
+  uint32_t spatial;            /* HPF only: 1 = the runtime decides how far to preempt: a
+                                  higher-priority arrival that needs n < num_sms SMs
+                                  (n = ceil(workers / resident CTAs per SM), A9)
+                                  gets a spatial yield of n SMs and runs beside the victim, which
+                                  is refilled to every SM when it finishes (R29);
+                                  0 = always temporal (Fig. 6 as printed) */
   uint32_t slice_blocks;       /* SLICE policy: blocks per sub-kernel (0 -> W*C*K, A20) */
   uint32_t exec_on_user_stream;/* MANUAL mode: launch worker grids (and resumes) directly on the
                                   caller's stream instead of a runtime stream. Stream order then
@@ -295,11 +300,16 @@ flep_status flep_set_rank_table(flep_rt rt, const uint16_t* rank, uint32_t n);
 /* Host steady-clock now, ns (the clock all host timestamps use). */
 int64_t flep_now_ns(void);
 /* Decision log of the managed runtime: n records of (t_ns, action, launch, n_sms) with
-   action 0 = LAUNCH, 1 = RESUME, 2 = PREEMPT; and the event log (t_ns, type, launch) with
-   type 0 = ARRIVE, 1 = FINISH, 2 = TICK (FFS epoch expiry; launch = -1), plus per-launch
-   (priority, t_e, overhead). */
+   action 0 = LAUNCH, 1 = RESUME, 2 = PREEMPT (n_sms = yield width: num_sms temporal, fewer
+   spatial), 3 = REFILL (a spatially preempted launch back on every SM); and the event log
+   (t_ns, type, launch) with type 0 = ARRIVE, 1 = FINISH, 2 = TICK (FFS epoch expiry;
+   launch = -1), plus per-launch (priority, t_e, overhead). out4 / out6 may be NULL: *n_out is
+   then the number of records available. */
 flep_status flep_decision_log(flep_rt rt, int64_t* out4, size_t max_records, size_t* n_out);
 flep_status flep_event_log(flep_rt rt, int64_t* out6, size_t max_records, size_t* n_out);
+/* The event log with a 7th field per record: the SMs the launch needs (ARRIVE records; the
+   spatial HPF input, A9), else 0. */
+flep_status flep_event_log_ex(flep_rt rt, int64_t* out7, size_t max_records, size_t* n_out);
 
 /* ---- pure policy engine (host only; no GPU needed) -------------------------------------
    The exact decision logic the managed runtime uses (Fig. 6), exposed for replay parity with
@@ -310,8 +320,14 @@ flep_status flep_policy_create(int32_t kind, uint32_t num_sms, flep_policy_t* ou
 flep_status flep_policy_destroy(flep_policy_t p);
 flep_status flep_policy_arrive(flep_policy_t p, int64_t t_ns, int64_t id, int32_t priority,
                                int64_t t_e_ns, int64_t overhead_ns);
+/* Same, with the SMs the kernel needs (spatial HPF input; 0 = the whole GPU). */
+flep_status flep_policy_arrive_ex(flep_policy_t p, int64_t t_ns, int64_t id, int32_t priority,
+                                  int64_t t_e_ns, int64_t overhead_ns, int64_t sms_need);
+/* HPF (kind 2): 1 = spatial preemption decisions (R29), 0 = temporal only (default). */
+flep_status flep_policy_set_spatial(flep_policy_t p, int32_t on);
 flep_status flep_policy_finish(flep_policy_t p, int64_t t_ns, int64_t id);
-/* Decisions emitted so far: records of 4 int64 (t_ns, action, id, n_sms). */
+/* Decisions emitted so far: records of 4 int64 (t_ns, action, id, n_sms); action as in
+   flep_decision_log. */
 flep_status flep_policy_decisions(flep_policy_t p, int64_t* out4, size_t max_records,
                                   size_t* n_out);
 /* FFS (kind 4): epoch-expiry check at time t; *acted = 1 iff it changed the schedule.

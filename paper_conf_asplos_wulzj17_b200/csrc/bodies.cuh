@@ -176,6 +176,9 @@ struct SpmvBody : NoResources {
       const int32_t p0 = s_rp[0], p1 = s_rp[nr];
       int32_t my_s = 0, my_e = 0;
       if (tid < nr) { my_s = s_rp[tid]; my_e = s_rp[tid + 1]; }
+      // An all-empty group runs no tile (whose barriers order these s_rp reads before the next
+      // group's s_rp writes): order them here. p0/p1 are the same in every thread (uniform).
+      if (p0 >= p1) body_sync<kThreads>();
       float acc = 0.f;
       for (int32_t base = p0; base < p1; base += (int32_t)kTile) {
         const int32_t n = min((int32_t)kTile, p1 - base);
@@ -234,6 +237,9 @@ struct SpmvBody : NoResources {
       const int32_t p0 = s_rp[0], p1 = s_rp[nr];
       int32_t my_s = 0, my_e = 0;
       if (tid < nr) { my_s = s_rp[tid]; my_e = s_rp[tid + 1]; }
+      // An all-empty group runs no tile (whose barriers order these s_rp reads before the next
+      // group's s_rp writes): order them here. p0/p1 are the same in every thread (uniform).
+      if (p0 >= p1) body_sync<kThreads>();
       float acc = 0.f;
       for (int32_t base = p0; base < p1; base += (int32_t)kTile) {
         const int32_t n = min((int32_t)kTile, p1 - base);

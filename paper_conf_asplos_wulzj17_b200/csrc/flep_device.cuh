@@ -7,7 +7,9 @@
 //   spatial check hostSM_ID < spa_P (here: rank[%smid] < n) ................ Fig. 4(c)
 //   progress tracked in a global counter so a relaunch resumes ............. P:126
 //
-// B200 design: one 32-bit control word ctrl = epoch<<16 | n in device memory,
+// B200 design: one 32-bit control word ctrl = epoch<<8 | n in device memory (24
+// generation bits, the same width as the host status word, so a late request never matches a
+// later epoch of a pooled control block; n <= 255 covers the 148 SMs, n >= #SMs = temporal),
 // polled with ld.acquire.gpu (an L2 hit) once per K chunks; a chunk is C original blocks per
 // atomicAdd (the probe measured ~1.46 fetches/ns chip-wide on one address, so C amortises the
 // atomic); exits happen only at poll points or on exhaustion, never while holding a chunk
@@ -29,6 +31,16 @@ constexpr uint32_t kStateDone = 5;
 constexpr uint32_t kEvEpochs = 8;       // event log ring: last 8 epochs per launch
 constexpr uint32_t kNoTrigger = 0xffffffffu;
 
+// The control word (reading R2): generation in bits 8-31 (24 bits, as in HostStatus::word), the
+// yield width n in bits 0-7 (0 = no request, n >= #SMs = temporal; kCtrlAll asks every SM).
+constexpr uint32_t kCtrlGenMask = 0xffffffu;
+constexpr uint32_t kCtrlAll = 0xffu;
+__host__ __device__ __forceinline__ uint32_t ctrl_word(uint32_t gen, uint32_t n) {
+  return ((gen & kCtrlGenMask) << 8) | (n < kCtrlAll ? n : kCtrlAll);
+}
+__host__ __device__ __forceinline__ uint32_t ctrl_gen(uint32_t c) { return c >> 8; }
+__host__ __device__ __forceinline__ uint32_t ctrl_n(uint32_t c) { return c & kCtrlAll; }
+
 // Per-launch control block in device memory. Hot words on separate 128-B lines.
 struct alignas(128) ControlBlock {
   // the counter word (R23): bits 0-31 = task counter, the next original block index to hand out
@@ -37,7 +49,7 @@ struct alignas(128) ControlBlock {
   // The epoch's last worker resets the high half.
   unsigned long long cx;
   uint32_t _p0[30];
-  uint32_t ctrl;           // epoch<<16 | n_yield (D1/D2); device copy for the memop transport
+  uint32_t ctrl;           // epoch<<8 | n_yield (D1/D2, ctrl_word()); device copy for the memop transport
   uint32_t _p1[31];
   uint32_t done_gen;       // generation whose epoch completed the launch (0 = none yet); an
                            // epoch launched after that (e.g. a refill) exits without fetching
@@ -93,6 +105,9 @@ struct WorkerParams {
                            // relay is not a worker (W excludes it)
   uint32_t started_hint;   // 1: worker 0 publishes "epoch started" to the host slot at entry (a
                            //    system-scope store: the kernel's completion then waits for it)
+  uint32_t ctrl_sys;       // 1: `ctrl` is a CPU-written mapped host word (FLEP_FLAG_HOST_MAPPED):
+                           //    polled with a system-scope load (a gpu-scope load is not
+                           //    guaranteed to observe a CPU store)
   void* partial;           // in-tile preemption (FLEP_KFLAG_IN_TILE, GEMM): W partial-tile records
                            // then W accumulator spill slots (layout: partial_bytes below), or nullptr
 #ifdef FLEP_TRACE
@@ -135,6 +150,9 @@ __device__ __forceinline__ uint32_t ld_acquire_gpu(const uint32_t* p) {
 __device__ __forceinline__ uint32_t ld_relaxed_gpu(const uint32_t* p) {
   uint32_t v; asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory"); return v;
 }
+__device__ __forceinline__ uint32_t ld_relaxed_sys(const uint32_t* p) {
+  uint32_t v; asm volatile("ld.relaxed.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory"); return v;
+}
 __device__ __forceinline__ uint32_t ld_acquire_sys(const uint32_t* p) {
   uint32_t v; asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory"); return v;
 }
@@ -167,9 +185,20 @@ __device__ __forceinline__ void body_sync() {
 
 // Does the control word ask the worker on `sm` to leave? (Fig. 4(c))
 __device__ __forceinline__ bool should_yield(uint32_t c, const WorkerParams& p, uint32_t sm) {
-  const uint32_t gen = c >> 16, n = c & 0xffffu;
-  if (gen != (p.epoch & 0xffffu) || n == 0) return false;
+  const uint32_t n = ctrl_n(c);
+  if (ctrl_gen(c) != (p.epoch & kCtrlGenMask) || n == 0) return false;
   return n >= p.num_sms || p.rank[sm] < n;
+}
+// The poll's load of the control word: device word (stream memop / relay) -> gpu scope; mapped
+// host word written by the CPU -> system scope.
+__device__ __forceinline__ uint32_t poll_ctrl(const WorkerParams& p) {
+  return p.ctrl_sys ? ld_relaxed_sys(p.ctrl) : ld_relaxed_gpu(p.ctrl);
+}
+// Device-side store of a request (self-trigger test hook, relay): a plain system-scope store to a
+// mapped host word, an L2 exchange for the device word.
+__device__ __forceinline__ void store_ctrl(const WorkerParams& p, uint32_t v) {
+  if (p.ctrl_sys) st_relaxed_sys(p.ctrl, v);
+  else atomicExch(p.ctrl, v);
 }
 
 // Worker bookkeeping shared by every loop shape (kept in shared memory, written by the one
@@ -277,7 +306,7 @@ __device__ __forceinline__ uint32_t next_chunk(const WorkerParams& p, SchedState
       // A later epoch: the launch may already have completed in an earlier one (a refill raced
       // with the last blocks) -> leave without touching the counter. Both loads are issued back
       // to back: one L2 round trip. The poll doubles as the entry check of a2 (Fig. 4(c)).
-      const uint32_t c = ld_relaxed_gpu(p.ctrl);
+      const uint32_t c = poll_ctrl(p);
       const uint32_t dg = ld_relaxed_gpu(&p.cb->done_gen);
       if (dg >= p.gen_first) { ws.reason = kReasonExhausted; return 0xffffffffu; }
       if (should_yield(c, p, smid_reg())) { ws.reason = kReasonYield; return 0xffffffffu; }
@@ -285,7 +314,7 @@ __device__ __forceinline__ uint32_t next_chunk(const WorkerParams& p, SchedState
   } else if (st.k == 0 && !st.stopping) {            // amortised poll (Fig. 4(b))
     // async poll (FLEP_KFLAG_ASYNC_POLL, reading R22): use the word loaded at the previous step,
     // so no round trip sits between two chunks; a request is then acted on one chunk later
-    const uint32_t c = (p.async_poll && st.have_seen) ? poll_consume(ws) : ld_relaxed_gpu(p.ctrl);
+    const uint32_t c = (p.async_poll && st.have_seen) ? poll_consume(ws) : poll_ctrl(p);
     if (should_yield(c, p, smid_reg())) { st.stopping = true; ws.reason = kReasonYield; }
   }
 #ifdef FLEP_TRACE
@@ -316,7 +345,7 @@ __device__ __forceinline__ uint32_t next_chunk(const WorkerParams& p, SchedState
       const uint32_t e = p.epoch % kEvEpochs;
       p.cb->ep_t_trigger[e] = gtimer();
       p.cb->ep_trigger_block[e] = p.trigger_block;
-      atomicExch(p.ctrl, ((p.epoch & 0xffffu) << 16) | (p.trigger_n & 0xffffu));
+      store_ctrl(p, ctrl_word(p.epoch, p.trigger_n));
     }
     if (++st.k == p.poll) st.k = 0;
     if (p.async_poll && st.k == 0 && !st.stopping) {  // the next step polls: load it now
@@ -390,7 +419,7 @@ __device__ __forceinline__ void request_relay(const WorkerParams& p) {
     if (h != last) {
       last = h;
       atomicExch(p.ctrl, h);
-      if ((h >> 16) == (p.epoch & 0xffffu) && (h & 0xffffu) >= p.num_sms) return;
+      if (ctrl_gen(h) == (p.epoch & kCtrlGenMask) && ctrl_n(h) >= p.num_sms) return;
     }
     if (ld_relaxed_gpu(&p.cb->pub_gen) == p.epoch) return;
   }
@@ -594,7 +623,7 @@ flep_clc_worker(const __grid_constant__ typename Body::Args args, const WorkerPa
       bool stop = false;
       if (++k == p.poll) {
         k = 0;
-        stop = should_yield(ld_relaxed_gpu(p.ctrl), p, smid_reg());
+        stop = should_yield(poll_ctrl(p), p, smid_reg());
       }
       if (!stop) { clc_try_cancel(resp, mbar); pending = true; }   // overlaps the body
       else ws.reason = kReasonYield;
@@ -602,7 +631,7 @@ flep_clc_worker(const __grid_constant__ typename Body::Args args, const WorkerPa
         const uint32_t e = p.epoch % kEvEpochs;
         p.cb->ep_t_trigger[e] = gtimer();
         p.cb->ep_trigger_block[e] = p.trigger_block;
-        atomicExch(p.ctrl, ((p.epoch & 0xffffu) << 16) | (p.trigger_n & 0xffffu));
+        store_ctrl(p, ctrl_word(p.epoch, p.trigger_n));
       }
     }
     const uint32_t b0 = b * p.chunk, b1 = min(b0 + p.chunk, p.n_blocks);

@@ -311,7 +311,7 @@ struct GemmBody {
             const PartialTile e = *mine;                   // written by the previous grid
             if (e.valid) {
               sch.first = false;                           // (the launch is not complete)
-              const uint32_t c = ld_relaxed_gpu(p.ctrl);   // entry check (a2) before taking it
+              const uint32_t c = poll_ctrl(p);   // entry check (a2) before taking it
               if (should_yield(c, p, smid_reg())) {
                 ws.reason = kReasonYield;                  // the record stays for a later epoch
                 ws.partial = e.b_end - e.b;                // blocks still unfinished (R23)
@@ -358,7 +358,7 @@ struct GemmBody {
                   pend_valid = false;
                   if (nk - kb > kMinLeft && should_yield(pend, p, smid_reg())) { stop = true; break; }
                 }
-                if (j % kInTilePoll == 0 && j > 0) { pend = ld_relaxed_gpu(p.ctrl); pend_valid = true; }
+                if (j % kInTilePoll == 0 && j > 0) { pend = poll_ctrl(p); pend_valid = true; }
               }
               mbar_wait(&s->empty[st], ph ^ 1u);
               s->stage_stop[st] = 0u;

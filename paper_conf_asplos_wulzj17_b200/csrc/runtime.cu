@@ -99,6 +99,7 @@ struct Launch {
   cudaStream_t exec = nullptr;
   int exec_level = 0;
   uint32_t chunk = 1, poll = 1, workers = 0, flags = 0;
+  int64_t sms_need = 0;              // SMs that host all its workers (A9), the spatial HPF input
   void* dmem = nullptr;              // ControlBlock + event ring
   ControlBlock* cb = nullptr;
   WorkerEvent* ev = nullptr;
@@ -175,7 +176,7 @@ struct flep_rt_s {
   // managed mode
   std::unique_ptr<Policy> policy;
   size_t applied = 0;
-  std::vector<std::array<int64_t, 6>> evlog;    // (t, type, id, prio, t_e, overhead)
+  std::vector<std::array<int64_t, 7>> evlog;    // (t, type, id, prio, t_e, overhead, sms_need)
   std::thread monitor;
   std::atomic<bool> stop{false};
   std::map<std::pair<int32_t, bool>, int> occ_cache;
@@ -233,7 +234,7 @@ flep_status get_stream(flep_rt rt, int level, cudaStream_t* s) {
 // Generations: every epoch of every launch that uses a control block gets a new number, so a
 // late request for an old epoch (or an old launch) never matches a newer one (A2/H5).
 inline uint32_t gen_of(const Launch& L) { return L.gen0 + L.epoch; }
-inline uint32_t ctrl_word(const Launch& L, uint32_t n) { return ((gen_of(L) & 0xffffu) << 16) | (n & 0xffffu); }
+inline uint32_t ctrl_word(const Launch& L, uint32_t n) { return flep::ctrl_word(gen_of(L), n); }
 
 flep_status write_ctrl(flep_rt rt, Launch& L, uint32_t value) {
   L.t_last_request = now_ns();
@@ -320,6 +321,7 @@ flep_status start_epoch(flep_rt rt, Launch& L) {
   p.started_hint = (L.flags & FLEP_KFLAG_STARTED_HINT) ? 1u : 0u;
   p.relay_block = L.relay ? L.workers : 0xffffffffu;
   p.async_poll = ((L.flags & FLEP_KFLAG_ASYNC_POLL) && rt->opt.flag != FLEP_FLAG_HOST_MAPPED) ? 1u : 0u;
+  p.ctrl_sys = rt->opt.flag == FLEP_FLAG_HOST_MAPPED ? 1u : 0u;
   p.partial = L.partial;
 #ifdef FLEP_TRACE
   p.trace = rt->trace;
@@ -419,18 +421,35 @@ void apply_decisions(flep_rt rt) {
     if (it == rt->launches.end()) continue;
     Launch& L = *it->second;
     if (x.action == kPreempt) {
+      const bool spatial = x.n_sms < (int64_t)rt->num_sms;
       if (L.sliced && L.state == FLEP_STATE_RUNNING) {   // slicing: stop issuing sub-kernels
         L.t_last_request = now_ns();
         L.state = FLEP_STATE_YIELDING;
         L.n_yield = (uint32_t)x.n_sms;
       } else if (L.state == FLEP_STATE_RUNNING || L.state == FLEP_STATE_PARTIAL) {
-        write_ctrl(rt, L, ctrl_word(L, (uint32_t)std::min<int64_t>(x.n_sms, 0xffff)));
-        L.state = FLEP_STATE_YIELDING;
+        write_ctrl(rt, L, ctrl_word(L, (uint32_t)std::min<int64_t>(x.n_sms, kCtrlAll)));
+        // spatial (R29): the launch keeps running on the SMs it was not asked to release
+        L.state = spatial ? FLEP_STATE_PARTIAL : FLEP_STATE_YIELDING;
         L.n_yield = (uint32_t)x.n_sms;
         if (L.clc) {                     // R25: no drain to wait for; the request is in force
           L.t_last_request = now_ns();
-          L.state = x.n_sms >= rt->num_sms ? FLEP_STATE_PREEMPTED : FLEP_STATE_PARTIAL;
+          L.state = spatial ? FLEP_STATE_PARTIAL : FLEP_STATE_PREEMPTED;
         }
+      }
+    } else if (x.action == kRefill) {
+      // the guest of a spatial co-run finished: the victim goes back to every SM (f1): a CLC grid
+      // just loses its request; a counter launch widens the request for its running epoch and
+      // queues a full-width epoch behind it (flep_refill)
+      if (L.state == FLEP_STATE_DONE) continue;       // finished meanwhile; FINISH pending
+      if (L.clc) {
+        write_ctrl(rt, L, ctrl_word(L, 0));
+        L.state = FLEP_STATE_RUNNING;
+        L.n_yield = 0;
+      } else if (L.state == FLEP_STATE_PARTIAL) {
+        write_ctrl(rt, L, ctrl_word(L, kCtrlAll));
+        start_epoch(rt, L);
+      } else if (L.state == FLEP_STATE_PREEMPTED) {
+        start_epoch(rt, L);
       }
     } else {
       if (L.state == FLEP_STATE_DONE) continue;   // finished while draining; FINISH pending
@@ -451,7 +470,7 @@ void monitor_pass(flep_rt rt) {
     if (refresh(rt, L)) {
       rt->to_release.push_back(L.id);
       const int64_t t = L.t_finish;
-      rt->evlog.push_back({t, 1, L.id, L.prio, L.t_e, L.overhead});
+      rt->evlog.push_back({t, 1, L.id, L.prio, L.t_e, L.overhead, 0});
       rt->policy->finish(t, L.id);
       apply_decisions(rt);
       changed = true;
@@ -462,7 +481,7 @@ void monitor_pass(flep_rt rt) {
   if (rt->opt.policy == FLEP_POLICY_FFS) {               // FFS epochs are time-driven
     const int64_t t = now_ns();
     if (rt->policy->tick(t)) {
-      rt->evlog.push_back({t, 2, -1, 0, 0, 0});
+      rt->evlog.push_back({t, 2, -1, 0, 0, 0, 0});
       apply_decisions(rt);
       changed = true;
     }
@@ -604,6 +623,8 @@ flep_status flep_init(int device, const flep_options* opts, flep_rt* out) {
   if (rt->opt.default_poll == 0) rt->opt.default_poll = 1;
   if (rt->opt.policy < FLEP_POLICY_MANUAL || rt->opt.policy > FLEP_POLICY_REORDER)
     return fail(FLEP_ERR_INVALID, "bad policy %d", rt->opt.policy);
+  if (rt->opt.spatial && rt->opt.policy != FLEP_POLICY_HPF)
+    return fail(FLEP_ERR_INVALID, "spatial decisions need the HPF policy");
   cudaDeviceProp prop;
   CUDA_TRY(cudaGetDeviceProperties(&prop, device));
   if (prop.major != 10) return fail(FLEP_ERR_UNSUPPORTED, "needs sm_100 (got %d.%d)", prop.major, prop.minor);
@@ -643,6 +664,9 @@ flep_status flep_init(int device, const flep_options* opts, flep_rt* out) {
   if (rt->opt.policy != FLEP_POLICY_MANUAL) {
     rt->policy.reset(new Policy(rt->opt.policy == FLEP_POLICY_SLICE ? (int32_t)kPolicyHPF : rt->opt.policy,
                                 rt->num_sms, rt->opt.max_overhead_ppm ? rt->opt.max_overhead_ppm : 100000));
+    // spatial decisions (R29): HPF on the persistent-worker mechanism only (a sliced kernel has no
+    // per-SM yield)
+    rt->policy->set_spatial(rt->opt.spatial != 0 && rt->opt.policy == FLEP_POLICY_HPF);
     flep_rt raw = rt.get();
     rt->monitor = std::thread([raw] { monitor_loop(raw); });
   }
@@ -744,6 +768,12 @@ flep_status flep_launch(flep_rt rt, flep_kernel kid, flep_dim3 grid, const void*
   L.relay = (kr.flags & FLEP_KFLAG_HOST_RELAY) && !L.sw && !L.clc && !ops->validate &&
             rt->opt.flag != FLEP_FLAG_HOST_MAPPED && wmax > 1;
   L.workers = (uint32_t)std::min<uint64_t>(std::min<uint64_t>(wmax - (L.relay ? 1 : 0), need), rt->max_workers);
+  {
+    // SMs that host every CTA of this launch (A9: n = ceil(grid / k)): the workers
+    // (+ the relay CTA), or the CLC grid's resident part
+    const uint64_t ctas = L.clc ? std::min<uint64_t>(need, wmax) : (uint64_t)L.workers + (L.relay ? 1u : 0u);
+    L.sms_need = (int64_t)std::min<uint64_t>(rt->num_sms, (ctas + (uint64_t)k - 1) / (uint64_t)k);
+  }
   if (rt->opt.policy == FLEP_POLICY_SLICE) {
     L.sliced = true;                                  // R16: one slice = one wave of W*C*K blocks
     L.slice_blocks = rt->opt.slice_blocks ? rt->opt.slice_blocks
@@ -823,8 +853,8 @@ flep_status flep_launch(flep_rt rt, flep_kernel kid, flep_dim3 grid, const void*
   *out = L.id;
   if (rt->opt.policy == FLEP_POLICY_MANUAL) return start_epoch(rt, L);
   // managed: interception (S2) -> policy decides (Fig. 6 lines 0-15)
-  rt->evlog.push_back({L.t_arrive, 0, L.id, L.prio, L.t_e, L.overhead});
-  rt->policy->arrive(L.t_arrive, L.id, L.prio, L.t_e, L.overhead);
+  rt->evlog.push_back({L.t_arrive, 0, L.id, L.prio, L.t_e, L.overhead, L.sms_need});
+  rt->policy->arrive(L.t_arrive, L.id, L.prio, L.t_e, L.overhead, L.sms_need);
   apply_decisions(rt);
   rt->cv.notify_all();
   return FLEP_OK;
@@ -881,7 +911,7 @@ flep_status flep_refill(flep_rt rt, flep_launch_t h) {
     return fail(FLEP_ERR_STATE, "launch %lld is not partially preempted (state %d)", (long long)h, L->state);
   // widen the request to the whole GPU for the running epoch, then queue a full-width epoch
   // behind it (stream order): the victim is re-spread over every SM
-  flep_status s = write_ctrl(rt, *L, ctrl_word(*L, 0xffffu));
+  flep_status s = write_ctrl(rt, *L, ctrl_word(*L, kCtrlAll));
   if (s) return s;
   return start_epoch(rt, *L);
 }
@@ -984,6 +1014,7 @@ flep_status flep_query(flep_rt rt, flep_launch_t h, flep_launch_info* out) {
 
 flep_status flep_cancel(flep_rt rt, flep_launch_t h) {
   if (!rt) return fail(FLEP_ERR_INVALID, "rt is NULL");
+  const bool managed = rt->opt.policy != FLEP_POLICY_MANUAL;
   {
     ApiLock lk(rt);
     Launch* L = find(rt, h);
@@ -991,27 +1022,41 @@ flep_status flep_cancel(flep_rt rt, flep_launch_t h) {
     refresh(rt, *L);
     if (L->state == FLEP_STATE_DONE) return FLEP_OK;
     if (L->state == FLEP_STATE_RUNNING || L->state == FLEP_STATE_PARTIAL || L->state == FLEP_STATE_YIELDING) {
-      write_ctrl(rt, *L, ctrl_word(*L, 0xffffu));
+      write_ctrl(rt, *L, ctrl_word(*L, kCtrlAll));
       L->state = FLEP_STATE_YIELDING;
     }
     L->cancelled = true;
   }
-  for (;;) {
+  for (;;) {                               // wait for the running epoch to drain (or complete)
     ApiLock lk(rt);
     Launch* L = find(rt, h);
     refresh(rt, *L);
-    if (L->state != FLEP_STATE_YIELDING) break;
+    if (L->state != FLEP_STATE_YIELDING && !(L->clc && L->state == FLEP_STATE_PREEMPTED && L->epoch > 0 &&
+                                             cudaEventQuery(L->fin_ev) != cudaSuccess))
+      break;
+    if (managed) rt->cv.wait_for(lk.u, std::chrono::microseconds(200));
   }
   ApiLock lk(rt);
   Launch* L = find(rt, h);
+  if (L->state == FLEP_STATE_DONE) return FLEP_OK;    // completed while draining (the monitor
+                                                      // already told the policy, managed mode)
   if (L->exec) CUDA_TRY(cudaStreamSynchronize(L->exec));
-  // the abandoned epoch left ctr/done non-zero: clear the block for reuse
-  if (L->state != FLEP_STATE_DONE) {
+  // the abandoned epoch left the counter word non-zero: clear the block for reuse
+  if (L->epoch > 0 && L->cb && !L->sliced) {
     CUDA_TRY(cudaMemsetAsync(L->cb, 0, offsetof(ControlBlock, ep_t_trigger), L->exec));
     CUDA_TRY(cudaStreamSynchronize(L->exec));
   }
   L->state = FLEP_STATE_DONE;
   L->t_finish = now_ns();
+  if (managed) {
+    // the policy must forget it (it may think the launch runs, or hold it in a queue): a FINISH
+    // event, the decisions that follow, and the launch's resources go back to the pools
+    rt->evlog.push_back({L->t_finish, 1, L->id, L->prio, L->t_e, L->overhead, 0});
+    rt->policy->finish(L->t_finish, L->id);
+    apply_decisions(rt);
+    rt->to_release.push_back(L->id);
+    rt->cv.notify_all();
+  }
   return FLEP_OK;
 }
 
@@ -1090,7 +1135,7 @@ flep_status flep_debug_trigger_at(flep_rt rt, flep_launch_t h, uint64_t block_in
   if (L->state != FLEP_STATE_PREEMPTED && L->state != FLEP_STATE_QUEUED)
     return fail(FLEP_ERR_STATE, "trigger can only be set for the next epoch of a launch that is not running");
   L->trig_block = block_index >= 0xffffffffull ? kNoTrigger : (uint32_t)block_index;
-  L->trig_n = std::min<uint32_t>(n_sms, 0xffff);
+  L->trig_n = std::min<uint32_t>(n_sms, kCtrlAll);
   return FLEP_OK;
 }
 
@@ -1098,7 +1143,7 @@ flep_status flep_debug_arm_next_trigger(flep_rt rt, uint64_t block_index, uint32
   if (!rt) return fail(FLEP_ERR_INVALID, "rt is NULL");
   ApiLock lk(rt);
   rt->arm_block = block_index >= 0xffffffffull ? kNoTrigger : (uint32_t)block_index;
-  rt->arm_n = std::min<uint32_t>(n_sms, 0xffff);
+  rt->arm_n = std::min<uint32_t>(n_sms, kCtrlAll);
   return FLEP_OK;
 }
 
@@ -1200,6 +1245,16 @@ flep_status flep_event_log(flep_rt rt, int64_t* out6, size_t max_records, size_t
   return FLEP_OK;
 }
 
+flep_status flep_event_log_ex(flep_rt rt, int64_t* out7, size_t max_records, size_t* n_out) {
+  if (!rt || !n_out) return fail(FLEP_ERR_INVALID, "NULL argument");
+  ApiLock lk(rt);
+  const size_t n = std::min(max_records, rt->evlog.size());
+  for (size_t i = 0; i < n && out7; ++i)
+    for (int j = 0; j < 7; ++j) out7[7 * i + j] = rt->evlog[i][j];
+  *n_out = out7 ? n : rt->evlog.size();
+  return FLEP_OK;
+}
+
 // ---- pure policy engine --------------------------------------------------------------------
 struct flep_policy_s {
   Policy p;
@@ -1231,6 +1286,19 @@ flep_status flep_policy_arrive(flep_policy_t p, int64_t t, int64_t id, int32_t p
   if (!p) return fail(FLEP_ERR_INVALID, "NULL policy");
   if (p->p.entry(id)) return fail(FLEP_ERR_INVALID, "duplicate id %lld", (long long)id);
   p->p.arrive(t, id, prio, t_e, o);
+  return FLEP_OK;
+}
+flep_status flep_policy_arrive_ex(flep_policy_t p, int64_t t, int64_t id, int32_t prio, int64_t t_e, int64_t o,
+                                  int64_t sms_need) {
+  if (!p) return fail(FLEP_ERR_INVALID, "NULL policy");
+  if (p->p.entry(id)) return fail(FLEP_ERR_INVALID, "duplicate id %lld", (long long)id);
+  if (sms_need < 0) return fail(FLEP_ERR_INVALID, "sms_need < 0");
+  p->p.arrive(t, id, prio, t_e, o, sms_need);
+  return FLEP_OK;
+}
+flep_status flep_policy_set_spatial(flep_policy_t p, int32_t on) {
+  if (!p) return fail(FLEP_ERR_INVALID, "NULL policy");
+  p->p.set_spatial(on != 0);
   return FLEP_OK;
 }
 flep_status flep_policy_finish(flep_policy_t p, int64_t t, int64_t id) {

@@ -20,7 +20,7 @@ BODY_STENCIL5_F32_TMA = 7
 STATE_QUEUED, STATE_RUNNING, STATE_YIELDING, STATE_PREEMPTED, STATE_PARTIAL, STATE_DONE = 0, 1, 2, 3, 4, 5
 STATE_NAMES = {0: "QUEUED", 1: "RUNNING", 2: "YIELDING", 3: "PREEMPTED", 4: "PARTIAL", 5: "DONE"}
 REASON_YIELD, REASON_EXHAUSTED = 1, 2
-ACTION_NAMES = {0: "LAUNCH", 1: "RESUME", 2: "PREEMPT"}
+ACTION_NAMES = {0: "LAUNCH", 1: "RESUME", 2: "PREEMPT", 3: "REFILL"}
 NO_TRIGGER = 0xFFFFFFFF
 KFLAG_PREFETCH = 1
 KFLAG_STARTED_HINT = 2
@@ -60,7 +60,7 @@ class GemmArgs(C.Structure):
 class Options(C.Structure):
     _fields_ = [("policy", C.c_int32), ("flag", C.c_int32), ("default_chunk", C.c_uint32),
                 ("default_poll", C.c_uint32), ("debug_coverage", C.c_uint32),
-                ("reserved0", C.c_uint32), ("slice_blocks", C.c_uint32),
+                ("spatial", C.c_uint32), ("slice_blocks", C.c_uint32),
                 ("exec_on_user_stream", C.c_uint32), ("max_overhead_ppm", C.c_uint32)]
 
 
@@ -122,9 +122,12 @@ _SIG = {
     "flep_now_ns": (C.c_int64, []),
     "flep_decision_log": (C.c_int, [_P, C.POINTER(C.c_int64), C.c_size_t, C.POINTER(C.c_size_t)]),
     "flep_event_log": (C.c_int, [_P, C.POINTER(C.c_int64), C.c_size_t, C.POINTER(C.c_size_t)]),
+    "flep_event_log_ex": (C.c_int, [_P, C.POINTER(C.c_int64), C.c_size_t, C.POINTER(C.c_size_t)]),
     "flep_policy_create": (C.c_int, [C.c_int32, C.c_uint32, C.POINTER(_P)]),
     "flep_policy_destroy": (C.c_int, [_P]),
     "flep_policy_arrive": (C.c_int, [_P, C.c_int64, C.c_int64, C.c_int32, C.c_int64, C.c_int64]),
+    "flep_policy_arrive_ex": (C.c_int, [_P, C.c_int64, C.c_int64, C.c_int32, C.c_int64, C.c_int64, C.c_int64]),
+    "flep_policy_set_spatial": (C.c_int, [_P, C.c_int32]),
     "flep_policy_finish": (C.c_int, [_P, C.c_int64, C.c_int64]),
     "flep_policy_decisions": (C.c_int, [_P, C.POINTER(C.c_int64), C.c_size_t, C.POINTER(C.c_size_t)]),
     "flep_policy_tick": (C.c_int, [_P, C.c_int64, C.POINTER(C.c_int32)]),
@@ -186,9 +189,9 @@ class Runtime:
     """One FLEP runtime on one device (flep_init ... flep_shutdown)."""
 
     def __init__(self, device=0, policy=POLICY_MANUAL, flag=FLAG_STREAM_MEMOP, chunk=8, poll=1,
-                 coverage=False, slice_blocks=0, exec_on_user_stream=False, max_overhead_ppm=0):
+                 coverage=False, slice_blocks=0, exec_on_user_stream=False, max_overhead_ppm=0, spatial=False):
         self.L = lib()
-        o = Options(policy, flag, chunk, poll, int(coverage), 0, slice_blocks,
+        o = Options(policy, flag, chunk, poll, int(coverage), int(spatial), slice_blocks,
                     int(exec_on_user_stream), max_overhead_ppm)
         h = C.c_void_p()
         check(self.L.flep_init(device, C.byref(o), C.byref(h)), "flep_init")
@@ -318,6 +321,14 @@ class Runtime:
         check(self.L.flep_event_log(self.h, buf, n.value, C.byref(n)), "flep_event_log")
         return [tuple(buf[6 * i:6 * i + 6]) for i in range(n.value)]
 
+    def event_log_ex(self):
+        """(t, type, launch, priority, t_e, overhead, sms_need) records."""
+        n = C.c_size_t()
+        check(self.L.flep_event_log_ex(self.h, None, 0, C.byref(n)), "flep_event_log_ex")
+        buf = (C.c_int64 * (7 * max(1, n.value)))()
+        check(self.L.flep_event_log_ex(self.h, buf, n.value, C.byref(n)), "flep_event_log_ex")
+        return [tuple(buf[7 * i:7 * i + 7]) for i in range(n.value)]
+
 
 def now_ns():
     return lib().flep_now_ns()
@@ -326,19 +337,21 @@ def now_ns():
 class PolicyEngine:
     """The runtime's pure decision engine (flep_policy_*), host only."""
 
-    def __init__(self, kind, num_sms=148):
+    def __init__(self, kind, num_sms=148, spatial=False):
         self.L = lib()
         h = C.c_void_p()
         check(self.L.flep_policy_create(kind, num_sms, C.byref(h)), "flep_policy_create")
         self.h = h
+        if spatial:
+            check(self.L.flep_policy_set_spatial(self.h, 1), "flep_policy_set_spatial")
 
     def __del__(self):
         if getattr(self, "h", None):
             self.L.flep_policy_destroy(self.h)
             self.h = None
 
-    def arrive(self, t, kid, prio, t_e, overhead):
-        check(self.L.flep_policy_arrive(self.h, t, kid, prio, t_e, overhead), "flep_policy_arrive")
+    def arrive(self, t, kid, prio, t_e, overhead, sms_need=0):
+        check(self.L.flep_policy_arrive_ex(self.h, t, kid, prio, t_e, overhead, sms_need), "flep_policy_arrive_ex")
 
     def finish(self, t, kid):
         check(self.L.flep_policy_finish(self.h, t, kid), "flep_policy_finish")

@@ -54,13 +54,17 @@ def saxpy_f32_inputs(n: int, seed: int):
     return x, y
 
 
-def csr_inputs(rows: int, seed: int, max_row_len: int = 20, cols: int | None = None):
+def csr_inputs(rows: int, seed: int, max_row_len: int = 20, cols: int | None = None,
+               empty_runs=()):
     """CSR matrix with row length uniform in {0..max_row_len}, columns uniform with replacement
     and sorted within each row (duplicates allowed), val and x uniform on [-1, 1) fp32.
-    SURVEY §8(c) A28 / §8(d) C2 (1M rows, ~10.5M nnz at seed 2)."""
+    SURVEY §8(c) A28 / §8(d) C2 (1M rows, ~10.5M nnz at seed 2). `empty_runs` = [(r0, r1), ...]
+    forces rows r0..r1-1 empty (edge-case inputs: whole empty row groups)."""
     g = rng(seed)
     ncols = rows if cols is None else cols
     lens = g.integers(0, max_row_len + 1, size=rows, dtype=np.int64)
+    for r0, r1 in empty_runs:
+        lens[r0:r1] = 0
     rowptr = np.zeros(rows + 1, dtype=np.int64)
     np.cumsum(lens, out=rowptr[1:])
     nnz = int(rowptr[-1])

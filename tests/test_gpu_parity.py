@@ -90,6 +90,58 @@ def test_spmv_wrapped_unwrapped(rt, torch_mod, rows, chunk):
     assert np.array_equal(yd2.cpu().numpy(), got)
 
 
+@pytest.mark.parametrize("chunk", [1, 3, 8])
+@pytest.mark.parametrize("variant", ["counter", "clc", "sched_warp"])
+def test_spmv_empty_row_groups(rt, torch_mod, chunk, variant):
+    """Runs of >= 256 consecutive empty rows (whole CSR-stream row groups without a nonzero) at
+    the start, in the middle and at the end, at chunks that put several groups in one run (the
+    ADVICE r1 race: an all-empty group skipped every barrier of the tile loop)."""
+    f = flep_mod()
+    rows = 6000
+    runs = [(0, 300), (1000, 1800), (2304, 2816), (5600, 6000)]
+    rowptr, col, val, x = gen.csr_inputs(rows, seed=13, empty_runs=runs)
+    ref, absum = W.spmv_csr(rowptr, col, val, x)
+    k = rt.register_kernel(f.BODY_SPMV_CSR_F32, chunk=chunk, poll=1, clc=variant == "clc",
+                           sched_warp=variant == "sched_warp")
+    dr, dc, dv, dx = t(rowptr), t(col), t(val), t(x)
+    for _ in range(3):
+        yd = torch_mod.full((rows,), float("nan"), device="cuda")
+        h = rt.launch(k, f.spmv_grid(rows), f.spmv_args(yd, dr, dc, dv, dx))
+        rt.sync(h)
+        got = yd.cpu().numpy()
+        assert _rel_err(got, ref, absum) <= REL_FP32
+        for r0, r1 in runs:
+            assert np.all(got[r0:r1] == 0.0)
+
+
+@pytest.mark.parametrize("body", ["f32", "f32_tma"])
+def test_stencil_16384_sampled_rows_vs_oracle(rt, torch_mod, body):
+    """configs[2]'s victim size (16384^2, 2 GB in + out): every cell of sampled rows against the
+    oracle, computed row by row on 3-row slabs (the middle row of a slab is an interior row with
+    the same neighbours as in the full field; boundary rows are copied through)."""
+    f = flep_mod()
+    n = 16384
+    a = gen.stencil_f32_input(n, seed=4)
+    kb = f.BODY_STENCIL5_F32 if body == "f32" else f.BODY_STENCIL5_F32_TMA
+    k = rt.register_kernel(kb, chunk=2, poll=1)
+    ind = t(a)
+    outd = torch_mod.empty_like(ind)
+    h = rt.launch(k, f.stencil_grid(n), f.stencil_args(outd, ind))
+    rt.sync(h)
+    g = gen.rng(99)
+    rows = sorted(set([1, 63, 64, 65, n - 2] + [int(r) for r in g.integers(1, n - 1, 40)]))
+    for r in rows:
+        ref, absum = W.stencil5_f32(a[r - 1:r + 2])
+        got = outd[r].cpu().numpy()
+        assert _rel_err(got, ref[1], absum[1]) <= REL_FP32, r
+    for r in (0, n - 1):                                   # boundary rows: copied through
+        assert np.array_equal(outd[r].cpu().numpy(), a[r])
+    out2 = torch_mod.empty_like(ind)
+    rt.launch_unwrapped(kb, f.stencil_grid(n), f.stencil_args(out2, ind))
+    torch_mod.cuda.synchronize()
+    assert torch_mod.equal(out2, outd)                      # wrapped == unwrapped, bit for bit
+
+
 @pytest.mark.parametrize("n", [3, 64, 130, 257, 1000, 4096])
 @pytest.mark.parametrize("integer", [False, True])
 def test_stencil_wrapped_unwrapped(rt, torch_mod, n, integer):

@@ -14,16 +14,16 @@ def flep():
     return F
 
 
-ACT = {"LAUNCH": 0, "RESUME": 1, "PREEMPT": 2}
+ACT = {"LAUNCH": 0, "RESUME": 1, "PREEMPT": 2, "REFILL": 3}
 KIND = {des.FIFO: 1, des.HPF: 2, des.SLICE: 3, des.REORDER: 5}
 
 
-def replay_cpp(F, kind, events):
-    p = F.PolicyEngine(KIND[kind])
+def replay_cpp(F, kind, events, spatial=False):
+    p = F.PolicyEngine(KIND[kind], spatial=spatial)
     for ev in events:
         if ev[1] == "ARRIVE":
             s = ev[2]
-            p.arrive(ev[0], s.id, s.priority, s.t_e, s.overhead)
+            p.arrive(ev[0], s.id, s.priority, s.t_e, s.overhead, s.sms_need)
         else:
             p.finish(ev[0], ev[2])
     return p.decisions()
@@ -52,6 +52,27 @@ def test_replay_parity_random_traces(flep, kind, seed):
                            slice_ns=150_000 if kind == des.SLICE else 0, slice_gap_ns=6_000)
     sim = des.simulate(kind, ks, params)
     assert as_tuples(sim.decisions) == replay_cpp(flep, kind, sim.events)
+
+
+@pytest.mark.parametrize("seed", range(25))
+def test_replay_parity_spatial_hpf(flep, seed):
+    """Spatial HPF (R29): decision lists with n_sms < 148 and REFILLs replay bit-exactly."""
+    g = gen.rng(500 + seed)
+    ks = random_trace(seed, 40, prios=1 + seed % 4, tight=seed % 2 == 0)
+    for k in ks:
+        k.sms_need = int(g.integers(0, 160))
+    sim = des.simulate_rates(ks, des.SimParams(drain_ns=seed * 500, start_ns=2_500), spatial=True)
+    assert as_tuples(sim.decisions) == replay_cpp(flep, des.HPF, sim.events, spatial=True)
+
+
+def test_replay_parity_spatial_hand_trace(flep):
+    ks = [des.KernelSpec(0, 0, 0, 5_000_000, 0, 5_000_000, 0),
+          des.KernelSpec(1, 10, 2, 100_000, 0, 100_000, 8),
+          des.KernelSpec(2, 20, 3, 100_000, 0, 100_000, 16),
+          des.KernelSpec(3, 30, 0, 10, 0, 10, 1)]
+    sim = des.simulate_rates(ks, spatial=True)
+    assert sum(1 for d in sim.decisions if d[1] == "REFILL") == 2
+    assert as_tuples(sim.decisions) == replay_cpp(flep, des.HPF, sim.events, spatial=True)
 
 
 def test_replay_parity_table1_pairs(flep):
