@@ -110,10 +110,23 @@ def physical_gpu_index(local_rank):
 
 
 # ------------------------------------------------------------------------------------------
-def dist_setup():
+def dist_setup(dry_run=False):
+    """One process per GPU (torch.distributed.run sets RANK / WORLD_SIZE / LOCAL_RANK). At
+    world > 1 the process group is initialised here, once, for every config: NCCL on the GPU box
+    (it only carries the timing reductions and the job-queue bookkeeping: the path itself is
+    replicas), gloo for --dry-run on CPU."""
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        import torch
+        import torch.distributed as dist
+        if not dist.is_initialized():
+            if dry_run or not torch.cuda.is_available():
+                dist.init_process_group("gloo")
+            else:
+                torch.cuda.set_device(local)
+                dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     return rank, world, local
 
 
@@ -121,15 +134,52 @@ def allreduce_max(vals, world, torch):
     if world == 1:
         return vals
     import torch.distributed as dist
-    t = torch.tensor(vals, dtype=torch.float64, device="cuda")
+    dev = "cuda" if dist.get_backend() == "nccl" else "cpu"
+    t = torch.tensor(vals, dtype=torch.float64, device=dev)
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
     return t.tolist()
+
+
+def allreduce_mean(vals, world, torch):
+    if world == 1:
+        return vals
+    import torch.distributed as dist
+    dev = "cuda" if dist.get_backend() == "nccl" else "cpu"
+    t = torch.tensor(vals, dtype=torch.float64, device=dev)
+    dist.all_reduce(t, op=dist.ReduceOp.SUM)
+    return (t / world).tolist()
+
+
+def gather_objects(obj, world):
+    """Every rank's `obj` (host-side bookkeeping only), in rank order."""
+    if world == 1:
+        return [obj]
+    import torch.distributed as dist
+    out = [None] * world
+    dist.all_gather_object(out, obj)
+    return out
 
 
 def barrier(world):
     if world > 1:
         import torch.distributed as dist
-        dist.barrier()
+        if dist.get_backend() == "nccl":
+            import torch
+            dist.barrier(device_ids=[torch.cuda.current_device()])
+        else:
+            dist.barrier()
+
+
+def relaunch_under_torchrun(n):
+    """`bench.py --gpus N` without a torchrun environment: re-execute this command as N ranks
+    (one process per GPU, rendezvous on 127.0.0.1) and return their exit code."""
+    import socket
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        port = so.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={n}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd)
 
 
 # ------------------------------------------------------------------------------------------
@@ -188,9 +238,6 @@ def run_temporal(args, rank, world, local):
     import torch
     from paper_conf_asplos_wulzj17_b200 import flep as F
     torch.cuda.set_device(local)
-    if world > 1:
-        import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     hbm, _, _, peak_src = peaks()
     wl = Workload(torch)
     flush = l2_flush_buffer(torch)
@@ -364,6 +411,13 @@ def run_temporal(args, rank, world, local):
     }
     if rank == 0:
         out["cpu_baseline"] = cpu_baseline(wl)
+    del wl, flush
+    torch.cuda.empty_cache()
+    if args.sub:
+        subs = sub_records(args, rank, world, local)
+        if rank == 0:
+            out["configs"] = subs
+    if rank == 0:
         print(json.dumps(out), flush=True)
     barrier(world)
 
@@ -562,43 +616,68 @@ def cpu_baseline(wl):
 
 
 def run_reference(args, rank, world):
-    """--impl reference: the oracle, timed on the host cores, same config/metric/unit."""
+    """--impl reference: the oracle, timed on the host cores, same config/metric/unit. A step is
+    what a non-preemptive program makes the waiting kernel wait for: the oracle SpMV over the LP
+    rows after a seeded block t*. `ms_per_step` is the mean of exactly those timed steps."""
     if rank != 0:
         return
     from oracle import workloads as W
     rowptr, col, val, x = gen.csr_inputs(SPMV_ROWS, seed=2)
-    st_in = gen.stencil_f32_input(STENCIL_N, seed=3)
     from paper_conf_asplos_wulzj17_b200.flep import SPMV_ROWS_PER_BLOCK
     n_lp = (SPMV_ROWS + SPMV_ROWS_PER_BLOCK - 1) // SPMV_ROWS_PER_BLOCK
     g = gen.rng(1000)
     lats = []
-    # the oracle stencil (~0.6 s) is timed once, so that any --steps K stays within a few
-    # minutes; every step times the SpMV the HP must wait for (the line's value)
-    ts0 = time.perf_counter()
-    W.stencil5_f32(st_in)
-    t_st = time.perf_counter() - ts0
     for i in range(args.warmup + args.steps):
         tstar = int(g.integers(n_lp // 4, 3 * n_lp // 4))
-        r0 = tstar * 128
+        r0 = tstar * SPMV_ROWS_PER_BLOCK
         s = rowptr[r0]
         t0 = time.perf_counter()
         W.spmv_csr((rowptr[r0:] - s).astype(np.int32), col[s:], val[s:], x)
         t1 = time.perf_counter()
         if i >= args.warmup:
             lats.append((t1 - t0) * 1e6)
-    steps_ms = [lt / 1e3 + t_st * 1e3 for lt in lats]
     v = float(np.median(lats))
     out = {"impl": "reference", "metric": METRIC, "value": round(v, 1), "unit": "us", "n_gpus": world,
-           "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(float(np.mean(steps_ms)), 3),
+           "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(float(np.mean(lats)) / 1e3, 3),
            "higher_is_better": False, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
            "data": "synthetic (seeded; synth/gen.py)",
-           "config": {"workload": "configs[1]: SpMV-CSR (2^20 rows) then stencil5 4096^2 on the CPU oracle"},
+           "config": {"workload": "configs[1]: full-GPU temporal preemption of SpMV-CSR fp32 (2^20 rows) by stencil5 "
+                                  "fp32 4096^2 -- CPU oracle arm: the HP waits for the LP's remaining rows"},
            "cpu_baseline": {"value": round(v, 1), "unit": "us", "cores": 1, "kind": "oracle",
                             "sample": "per step: oracle SpMV over the LP rows after a seeded t* (what a "
-                                      "non-preemptive program must finish before the HP starts); ms_per_step adds the oracle "
-                                      "stencil, timed once per run"},
+                                      "non-preemptive program must finish before the HP starts); ms_per_step is the "
+                                      "mean of these timed steps"},
            "e2e": {"value": round(v, 1), "unit": "us", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(out), flush=True)
+
+
+def sub_records(args, rank, world, local):
+    """The other BASELINE configs as sub-records of the default line (each with its own clocks):
+    configs[0] (SAXPY-int co-run, exactness), configs[2] (spatial yield per width: the manual
+    device-triggered sweep and the managed spatial-HPF decision path, victim checked against a
+    NumPy reference), configs[3] (64-kernel same-priority queue: ANTT/STP, decision logs) and
+    configs[4] (one 512-kernel job queue over the N GPUs of this run)."""
+    import copy
+    import bench_configs as BCF
+    a = copy.copy(args)
+    a.sub_record = True
+    a.steps, a.warmup = args.sub_steps, 3
+    out, timing = {}, {}
+    for name, fn in (("configs[0]", BCF.run_corun1), ("configs[2]", BCF.run_spatial),
+                     ("configs[2]_managed", BCF.run_spatial_managed), ("configs[3]", BCF.run_queue),
+                     ("configs[4]", BCF.run_scale_queue)):
+        if name in args.skip_sub:
+            continue
+        t0 = time.perf_counter()
+        r = fn(a, rank, world, local)
+        timing[name] = round(time.perf_counter() - t0, 1)
+        if rank == 0 and r is not None:
+            for k in ("metric", "n_gpus", "higher_is_better", "scaling", "vs_baseline", "data"):
+                r.pop(k, None)
+            out[name] = r
+    if rank == 0:
+        out["wall_s"] = timing
+    return out
 
 
 def main():
@@ -607,7 +686,15 @@ def main():
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--impl", default="flep", choices=["flep", "reference"])
-    ap.add_argument("--config", default="temporal", choices=["temporal", "corun1", "spatial", "queue", "ffs", "model", "gemm", "tune", "clc", "delay", "spatial_f1"])
+    ap.add_argument("--config", default="temporal", choices=["temporal", "corun1", "spatial", "spatial_managed", "queue",
+                                                             "scale", "ffs", "model", "gemm", "tune", "clc", "delay",
+                                                             "spatial_f1"])
+    ap.add_argument("--dry-run", action="store_true",
+                    help="configs[4] launcher and control flow without CUDA (CPU, gloo); one JSON line")
+    ap.add_argument("--sub", type=int, default=1, help="default run: add the configs[0,2,3,4] sub-records")
+    ap.add_argument("--sub-steps", type=int, default=12, help="timed trials per sub-record case")
+    ap.add_argument("--skip-sub", default="", help="comma list of sub-record names to skip")
+    ap.add_argument("--scale-kernels", type=int, default=512)
     ap.add_argument("--model-train", type=int, default=100)
     ap.add_argument("--model-test", type=int, default=30)
     ap.add_argument("--overhead-runs", type=int, default=50)
@@ -631,7 +718,16 @@ def main():
     ap.add_argument("--gemm-in-tile", type=int, default=1, help="config gemm: in-tile preemption (1) or tile granularity (0)")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
-    rank, world, local = dist_setup()
+    args.skip_sub = [x.strip() for x in args.skip_sub.split(",") if x.strip()]
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        sys.exit(relaunch_under_torchrun(args.gpus))
+    rank, world, local = dist_setup(dry_run=args.dry_run)
+    if world != args.gpus and rank == 0:
+        print(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world}; using {world} ranks", file=sys.stderr)
+    if args.dry_run:
+        import bench_configs
+        bench_configs.run_scale_dry(args, rank, world, local)
+        return
     if args.impl == "reference":
         run_reference(args, rank, world)
         return
@@ -639,36 +735,18 @@ def main():
     if rank == 0:
         build.build()
     if world > 1:
-        # wait for rank 0's build: poll for the library
-        from paper_conf_asplos_wulzj17_b200 import build as b2
-        for _ in range(600):
-            if not b2.needs_build():
-                break
-            time.sleep(1)
+        barrier(world)                       # rank 0's build (if any) is complete
     if args.config == "temporal":
         run_temporal(args, rank, world, local)
     else:
         import bench_configs
-        if args.config == "spatial":
-            bench_configs.run_spatial(args, rank, world, local)
-        elif args.config == "corun1":
-            bench_configs.run_corun1(args, rank, world, local)
-        elif args.config == "gemm":
-            bench_configs.run_gemm_preempt(args, rank, world, local)
-        elif args.config == "tune":
-            bench_configs.run_tune(args, rank, world, local)
-        elif args.config == "ffs":
-            bench_configs.run_ffs(args, rank, world, local)
-        elif args.config == "model":
-            bench_configs.run_model(args, rank, world, local)
-        elif args.config == "clc":
-            bench_configs.run_clc(args, rank, world, local)
-        elif args.config == "delay":
-            bench_configs.run_delay(args, rank, world, local)
-        elif args.config == "spatial_f1":
-            bench_configs.run_spatial_f1(args, rank, world, local)
-        else:
-            bench_configs.run_queue(args, rank, world, local)
+        fn = {"spatial": bench_configs.run_spatial, "spatial_managed": bench_configs.run_spatial_managed,
+              "corun1": bench_configs.run_corun1, "gemm": bench_configs.run_gemm_preempt,
+              "tune": bench_configs.run_tune, "ffs": bench_configs.run_ffs, "model": bench_configs.run_model,
+              "clc": bench_configs.run_clc, "delay": bench_configs.run_delay,
+              "spatial_f1": bench_configs.run_spatial_f1, "queue": bench_configs.run_queue,
+              "scale": bench_configs.run_scale_queue}[args.config]
+        fn(args, rank, world, local)
 
 
 if __name__ == "__main__":

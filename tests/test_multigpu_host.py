@@ -2,12 +2,17 @@
 -> N-schedulers partition is identical on every rank, disjoint and complete, and the timing
 reduction is a max over ranks (BASELINE configs[4]; replicas, no data-path
 collective)."""
+import json
 import os
 import socket
+import subprocess
+import sys
 
 import pytest
 
 from synth import gen
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
 def _free_port():
@@ -81,3 +86,37 @@ def test_rank_tables_are_permutations_and_follow_the_die_map():
     for k in (2, 4, 6, 8):
         assert sum(die[s] for s in inv[:k]) == k // 2
     assert bc._rank_tables(8, None) == {"ascending": list(range(8))}
+
+
+def _json_lines(stdout):
+    out = []
+    for line in stdout.splitlines():
+        line = line.strip()
+        if line.startswith("{"):
+            out.append(json.loads(line))
+    return out
+
+
+@pytest.mark.parametrize("n", [1, 2, 4])
+def test_bench_launcher_dry_run(n):
+    """The real bench.py launcher at N ranks: `--gpus N` re-executes itself under
+    torch.distributed.run when no torchrun environment is set, every rank initialises the process
+    group (gloo here, no CUDA), partitions the one 512-kernel job queue identically, and rank 0
+    alone prints exactly one JSON line with n_gpus = N."""
+    env = dict(os.environ)
+    for k in ("RANK", "WORLD_SIZE", "LOCAL_RANK", "MASTER_ADDR", "MASTER_PORT"):
+        env.pop(k, None)
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", str(n), "--dry-run"],
+                       capture_output=True, text=True, env=env, timeout=300, cwd=ROOT)
+    assert r.returncode == 0, r.stderr[-2000:]
+    lines = _json_lines(r.stdout)
+    assert len(lines) == 1, r.stdout
+    d = lines[0]
+    assert d["n_gpus"] == n and d["dry_run"] is True
+    assert d["partition_ok"] is True
+    assert [x["rank"] for x in d["ranks"]] == list(range(n))
+    assert sum(x["kernels"] for x in d["ranks"]) == 512
+    assert d["backend"] == (None if n == 1 else "gloo")
+    if n > 1:
+        busy = [x["predicted_busy_us"] for x in d["ranks"]]
+        assert max(busy) / min(busy) < 1.2          # least-backlog assignment balances the GPUs
