@@ -799,6 +799,7 @@ def _run_trace(F, torch, local, policy, trace, inst, t_alone, overhead_ns, strea
                                       model=(0, 0, 0, 0, float(t_alone[key])), overhead_ns=int(overhead_ns),
                                       in_tile=body == F.BODY_GEMM_BF16)
     hs = []
+    call_ns = []
     t0 = F.now_ns() + 2_000_000
     for i, job in enumerate(trace):
         key = (job["type"], job["size_class"])
@@ -806,7 +807,9 @@ def _run_trace(F, torch, local, policy, trace, inst, t_alone, overhead_ns, strea
         target = t0 + job["arrival_ns"]
         while F.now_ns() < target:
             pass
+        tl = F.now_ns()
         hs.append((rt.launch(kid[key], grid, a, priority=job["priority"], stream=streams[i % len(streams)]), key))
+        call_ns.append(F.now_ns() - tl)
     for h, _ in hs:
         rt.sync(h, timeout_ns=60_000_000_000)
     turn = []
@@ -821,6 +824,7 @@ def _run_trace(F, torch, local, policy, trace, inst, t_alone, overhead_ns, strea
     dec = rt.decision_log()
     evl = rt.event_log()
     rt.close()
+    _run_trace.last_call_us = {"mean": round(float(np.mean(call_ns)) / 1e3, 2), "max": round(float(np.max(call_ns)) / 1e3, 2)}
     if want_lat:
         return turn, dec, evl, lat
     return turn, dec, evl
@@ -880,6 +884,7 @@ def run_queue(args, rank, world, local):
         res[name] = {"antt": M.antt(tt, al), "stp": M.stp(tt, al), "preemptions": sum(1 for d in dec if d[1] == 2),
                      "makespan_ms": round(max(t[4] for t in turn) / 1e6, 3)}
         logs[name] = {"events": [list(map(int, e)) for e in evl], "decisions": [list(map(int, d_)) for d_ in dec]}
+        res[name]["launch_call_us"] = _run_trace.last_call_us
     # the runtime's event and decision logs (replayed through the oracle DES by
     # tests/test_policy_replay.py from the committed copy under tests/golden/)
     import os
@@ -905,6 +910,7 @@ def run_queue(args, rank, world, local):
            "stp_degradation_vs_fifo": round(1 - res["HPF"]["stp"] / res["FIFO"]["stp"], 4),
            "replay_parity": "checked on CPU: tests/test_policy_replay.py replays the committed logs (tests/golden/queue_logs_r01.json) through the oracle DES",
            "makespan_ms": {k: v["makespan_ms"] for k, v in res.items()},
+           "launch_call_us": {k: v["launch_call_us"] for k, v in res.items()},
            "t_alone_us": {f"{k[0]}-{k[1]}": round(v / 1e3, 1) for k, v in sorted(t_alone.items())}}
     if world > 1:
         from bench import allreduce_max
@@ -1261,7 +1267,7 @@ def run_spatial_managed(args, rank, world, local):
     g.manual_seed(4 + rank)
     v_in = torch.rand(n_st, n_st, device="cuda", generator=g)
     v_out = torch.empty_like(v_in)
-    rt = F.Runtime(device=local, policy=F.POLICY_HPF, spatial=True)
+    rt = F.Runtime(device=local, policy=F.POLICY_HPF, spatial=True, keep_logs=True)
     k_v = rt.register_kernel(F.BODY_STENCIL5_F32, chunk=1, poll=1, name="victim", started_hint=True,
                              model=(0, 0, 0, 0, 330_000))
     k_w = rt.register_kernel(F.BODY_SAXPY_F32, chunk=1, poll=1, name="waiting", model=(0, 0, 0, 0, 10_000))
@@ -1312,7 +1318,7 @@ def run_spatial_managed(args, rank, world, local):
                 if r:
                     ts.append((t1 - t0) / 1e3)
             t_w = float(np.median(ts))
-            lat, wstart, tflep, viol, bad_dec, worst, ok = [], [], [], 0, 0, 0.0, 0
+            lat, wstart, tflep, viol, bad_dec, worst, ok, mism = [], [], [], 0, 0, 0.0, 0, []
             for trial in range(args.warmup + args.steps):
                 flush.zero_()
                 torch.cuda.synchronize()
@@ -1337,15 +1343,34 @@ def run_spatial_managed(args, rank, world, local):
                     want = [("LAUNCH", h_v, 0), ("PREEMPT", h_v, rt.num_sms), ("LAUNCH", h_w, 0), ("RESUME", h_v, 0)]
                 if names != want:
                     bad_dec += 1
+                    if len(mism) < 3:
+                        (v0_, v1_), iv = spans(h_v)
+                        (w0_, w1_), iw = spans(h_w)
+                        mism.append({"got": [(a_, int(i_ == h_v), int(n_)) for a_, i_, n_ in names],
+                                     "want": [(a_, int(i_ == h_v), int(n_)) for a_, i_, n_ in want],
+                                     "dev_us_from_victim_start": {"guest_start": (w0_ - v0_) / 1e3, "guest_end": (w1_ - v0_) / 1e3,
+                                                                  "victim_end": (v1_ - v0_) / 1e3},
+                                     "host_us_from_victim_arrive": {"guest_arrive": (iw.t_arrive - iv.t_arrive) / 1e3,
+                                                                    "guest_finish": (iw.t_finish - iv.t_arrive) / 1e3,
+                                                                    "victim_finish": (iv.t_finish - iv.t_arrive) / 1e3,
+                                                                    "guest_first_start": (iw.t_first_start - iv.t_arrive) / 1e3},
+                                     "victim_epochs": iv.epoch, "guest_workers": iw.workers})
                     continue
                 info_v = rt.query(h_v)
                 ev1 = rt.events(h_v, 1)
-                if n < rt.num_sms:
-                    viol += sum(1 for e in ev1 if (e.reason == F.REASON_YIELD) != (e.smid < n))
                 (v0, v1), _ = spans(h_v)
                 (w0, w1), _ = spans(h_w)
+                if n < rt.num_sms:
+                    # I3: the workers on the n released SMs (rank = smid) yield; no other worker
+                    # leaves before the waiting kernel is done (the REFILL then widens the request
+                    # to every SM, so later yields elsewhere are the refill's)
+                    viol += sum(1 for e in ev1 if e.smid < n and e.reason != F.REASON_YIELD)
+                    viol += sum(1 for e in ev1 if e.smid >= n and e.reason == F.REASON_YIELD and e.t_exit < w1)
                 off = t_seen - v0                                 # host - device (started hint)
-                t_req = info_v.t_last_request - off if info_v.t_last_request > 0 else None
+                # the PREEMPT decision's host time (the runtime writes the request right after it;
+                # t_last_request is overwritten by the REFILL's request)
+                t_pre = [d[0] for d in dec if d[1] == 2 and d[2] == h_v]
+                t_req = t_pre[0] - off if t_pre else None
                 ys = [e.t_exit for e in ev1 if e.reason == F.REASON_YIELD]
                 if ys and t_req:
                     lat.append((max(ys) - t_req) / 1e3)
@@ -1360,6 +1385,7 @@ def run_spatial_managed(args, rank, world, local):
                 worst = max(worst, float(np.max(np.abs(got[r] - ref[1]) / np.where(d > 0, d, 1))))
             t_org = alone["victim"] + t_w
             rows.append({"n_sms": n, "trials": ok, "decision_list_mismatches": bad_dec, "I3_violations": viol,
+                         "mismatch_examples": mism,
                          "yield_latency_us_p50": round(float(np.median(lat)), 3) if lat else None,
                          "waiting_start_us_p50": round(float(np.median(wstart)), 3) if wstart else None,
                          "t_flep_us": round(float(np.median(tflep)), 2) if tflep else None,

@@ -109,7 +109,10 @@ typedef struct {
   int32_t flag;                /* flep_flag_transport */
   uint32_t default_chunk;      /* C: original blocks per counter fetch (0 -> 8) */
   uint32_t default_poll;       /* K: chunks between control-word polls (0 -> 1) */
-  uint32_t debug_coverage;     /* 1: keep a per-block execution count cov[N] (test builds) */
+  uint32_t debug_coverage;     /* bit 0: keep a per-block execution count cov[N] (test builds);
+                                  any non-zero value: keep the device logs (worker events, epoch
+                                  summaries) of the newest 64 finished launches for the debug
+                                  copies (2 = logs only, no coverage count in the workers) */
   uint32_t spatial;            /* HPF only: 1 = the runtime decides how far to preempt: a
                                   higher-priority arrival that needs n < num_sms SMs
                                   (n = ceil(workers / resident CTAs per SM), A9)

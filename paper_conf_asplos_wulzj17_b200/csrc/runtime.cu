@@ -24,6 +24,7 @@
 #include <deque>
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <map>
 #include <memory>
@@ -134,6 +135,9 @@ struct Launch {
   int64_t t_seen = 0;                // monitor: host time its status word was seen to move
   bool released = false;
   bool cancelled = false;
+  bool materialized = false;         // device resources taken (at the first epoch, see materialize)
+  bool want_cov = false;
+  cudaEvent_t ev_user = nullptr;     // the caller's stream position at flep_launch (workers wait on it)
 };
 
 struct KernelReg {
@@ -154,6 +158,7 @@ struct flep_rt_s {
   uint32_t num_sms = 0, nsmid = 0;
   int prio_lo = 0, prio_hi = 0;            // CUDA stream priority range (lo = least)
   cudaStream_t ctl = nullptr;              // highest-priority control stream
+  cudaStream_t aux = nullptr;              // debug copies of launches whose stream went back to the pool
   uint16_t* d_rank = nullptr;
   HostStatus* h_slots = nullptr;
   HostStatus* d_slots = nullptr;
@@ -279,7 +284,108 @@ flep_status issue_slices(flep_rt rt, Launch& L) {
   return FLEP_OK;
 }
 
+// FLEP_DEBUG_SLOW=<us>: report to stderr every epoch start whose host path took longer (where the
+// time went: resource materialisation vs the launch call).
+int64_t slow_threshold_ns() {
+  static const int64_t v = [] {
+    const char* e = getenv("FLEP_DEBUG_SLOW");
+    return e ? (int64_t)(atof(e) * 1e3) : (int64_t)-1;
+  }();
+  return v;
+}
+
+// Take the launch's device resources (first epoch only). Pools are pre-warmed so this normally
+// allocates nothing.
+flep_status materialize(flep_rt rt, Launch& L) {
+  if (L.materialized) return FLEP_OK;
+  if (rt->free_slots.empty()) return fail(FLEP_ERR_NOMEM, "out of status slots");
+  flep_status s = FLEP_OK;
+  int64_t tm[6] = {now_ns(), 0, 0, 0, 0, 0};
+  if (L.exec_level != -1000) {
+    s = get_stream(rt, L.exec_level, &L.exec);
+    if (s) return s;
+    tm[1] = now_ns();
+    if (L.ev_user) {
+      CUDA_TRY(cudaStreamWaitEvent(L.exec, L.ev_user, 0));
+      rt->event_pool.push_back(L.ev_user);    // reusable once waited on (waits bind at enqueue time)
+      L.ev_user = nullptr;
+    }
+  }
+  tm[2] = now_ns();
+  bool fresh_cb = false;
+  if (!rt->free_dmem.empty()) { L.dmem = rt->free_dmem.back(); rt->free_dmem.pop_back(); }
+  else {
+    CUDA_TRY(cudaMalloc(&L.dmem, rt->dmem_bytes));
+    rt->cb_gen[L.dmem] = 0;
+    fresh_cb = true;             // zeroed below, on the stream the workers run on
+  }
+  L.gen0 = rt->cb_gen[L.dmem];
+  if (L.gen0 + 2 * kEvEpochs >= kCtrlGenMask) return fail(FLEP_ERR_NOMEM, "control block generation space exhausted");
+  L.cb = (ControlBlock*)L.dmem;
+  L.ev = (WorkerEvent*)((char*)L.dmem + sizeof(ControlBlock));
+  tm[3] = now_ns();
+  const uint32_t N = L.n_blocks;
+  if (L.want_cov) {
+    for (size_t i = 0; i < rt->free_cov.size(); ++i) {
+      if (rt->free_cov[i].second >= N) {
+        L.cov = rt->free_cov[i].first; L.cov_cap = rt->free_cov[i].second;
+        rt->free_cov.erase(rt->free_cov.begin() + i);
+        break;
+      }
+    }
+    if (!L.cov) { L.cov_cap = std::max<size_t>(N, 4096); CUDA_TRY(cudaMalloc(&L.cov, L.cov_cap * 4)); }
+  }
+  if (L.flags & FLEP_KFLAG_IN_TILE) {
+    // per-worker partial-tile records and fp32 accumulator spill slots; no reset needed (the
+    // first epoch's workers clear their records)
+    const size_t need = partial_bytes(L.workers);
+    for (size_t i = 0; i < rt->free_partial.size(); ++i) {
+      if (rt->free_partial[i].second >= need) {
+        L.partial = rt->free_partial[i].first; L.partial_cap = rt->free_partial[i].second;
+        rt->free_partial.erase(rt->free_partial.begin() + i);
+        break;
+      }
+    }
+    if (!L.partial) { L.partial_cap = need; CUDA_TRY(cudaMalloc(&L.partial, need)); }
+  }
+  L.slot = rt->free_slots.back();
+  rt->free_slots.pop_back();
+  L.hs = rt->h_slots + L.slot;
+  L.ds = rt->d_slots + L.slot;
+  memset(L.hs, 0, sizeof(HostStatus));
+  // No per-launch reset work on the GPU: a pooled control block was left clean by the last
+  // worker of its previous launch's DONE epoch, and its generation numbers keep increasing.
+  tm[4] = now_ns();
+  s = pooled_event(rt, &L.fin_ev);
+  if (s) return s;
+  if (L.cov) CUDA_TRY(cudaMemsetAsync(L.cov, 0, (size_t)N * 4, L.exec));
+  if (fresh_cb) CUDA_TRY(cudaMemsetAsync(L.dmem, 0, sizeof(ControlBlock), L.exec));
+  tm[5] = now_ns();
+  if (slow_threshold_ns() >= 0 && tm[5] - tm[0] > slow_threshold_ns())
+    fprintf(stderr, "[flep] materialize launch %lld: stream %.1f wait %.1f block %.1f bufs %.1f event %.1f us\n",
+            (long long)L.id, tm[1] ? (tm[1] - tm[0]) / 1e3 : 0.0, tm[1] ? (tm[2] - tm[1]) / 1e3 : 0.0,
+            (tm[3] - tm[2]) / 1e3, (tm[4] - tm[3]) / 1e3, (tm[5] - tm[4]) / 1e3);
+  L.materialized = true;
+  return FLEP_OK;
+}
+
 flep_status start_epoch(flep_rt rt, Launch& L) {
+  const int64_t t_a = now_ns();
+  const bool fresh = !L.materialized;
+  {
+    flep_status s = materialize(rt, L);
+    if (s) return s;
+  }
+  const int64_t t_b = now_ns();
+  struct SlowReport {
+    const Launch& L; int64_t a, b; bool fresh;
+    ~SlowReport() {
+      const int64_t th = slow_threshold_ns(), c = now_ns();
+      if (th >= 0 && c - a > th)
+        fprintf(stderr, "[flep] slow epoch start: launch %lld body %d epoch %u: materialize %.1f us%s, launch %.1f us\n",
+                (long long)L.id, L.body, L.epoch, (b - a) / 1e3, fresh ? " (first)" : "", (c - b) / 1e3);
+    }
+  } slow_report{L, t_a, t_b, fresh};
   if (L.sliced) {
     L.epoch++;
     L.state = FLEP_STATE_RUNNING;
@@ -396,6 +502,17 @@ bool refresh(flep_rt rt, Launch& L) {
   return false;
 }
 
+// The stream a debug copy of L runs on: its own (ordered after its grids) while it has one, else
+// the runtime's auxiliary stream (the stream goes back to the pool once the last grid completed).
+cudaStream_t dbg_stream(flep_rt rt, const Launch& L) { return L.exec ? L.exec : rt->aux; }
+
+// A finished launch whose last grid completed gives its execution stream back at once, even if
+// its device logs are retained for debug copies.
+void release_stream(flep_rt rt, Launch& L) {
+  if (L.exec && L.exec_level != -1000) rt->free_streams[L.exec_level].push_back(L.exec);
+  if (L.exec_level != -1000) L.exec = nullptr;
+}
+
 void release_resources(flep_rt rt, Launch& L) {
   if (L.released) return;
   // the launch's last grid has completed (caller synchronised the exec stream); the last worker
@@ -408,6 +525,7 @@ void release_resources(flep_rt rt, Launch& L) {
   if (L.exec && L.exec_level != -1000) rt->free_streams[L.exec_level].push_back(L.exec);
   for (cudaEvent_t e : L.evpool) rt->event_pool.push_back(e);
   L.evpool.clear();
+  if (L.ev_user) { rt->event_pool.push_back(L.ev_user); L.ev_user = nullptr; }
   if (L.fin_ev) { rt->event_pool.push_back(L.fin_ev); L.fin_ev = nullptr; }
   L.dmem = nullptr; L.cov = nullptr; L.slot = -1; L.exec = nullptr;
   L.released = true;
@@ -488,8 +606,9 @@ void monitor_pass(flep_rt rt) {
   }
   for (size_t i = 0; i < rt->to_release.size();) {      // recycle finished launches
     Launch* R = find(rt, rt->to_release[i]);
-    if (R && cudaEventQuery(R->fin_ev) == cudaSuccess) {
+    if (R && (!R->fin_ev || cudaEventQuery(R->fin_ev) == cudaSuccess)) {
       if (rt->opt.debug_coverage) {                    // keep the newest 64 for debug copies
+        release_stream(rt, *R);
         rt->retained.push_back(R->id);
         while (rt->retained.size() > 64) {
           Launch* old = find(rt, rt->retained.front());
@@ -545,7 +664,9 @@ void monitor_loop(flep_rt rt) {
       }
     }
     if (deadline >= 0 && now_ns() >= deadline) hit = true;
-    if (pending_release) hit = true;
+    // launches waiting for their last grid before release: checked every 64th pass only (the
+    // lock is what application threads need; a release is never latency-critical)
+    if (pending_release && (spin & 63u) == 0) hit = true;
     if (!hit) {
       if (watch.empty() && deadline < 0) {
         std::unique_lock<std::mutex> lk(rt->mu);
@@ -555,6 +676,9 @@ void monitor_loop(flep_rt rt) {
       }
       continue;
     }
+    // API threads announce themselves before taking the lock (ApiLock): let them in first, for a
+    // bounded time (a thread that calls the API in a loop must not starve the monitor either)
+    for (int i = 0; i < 256 && rt->waiters.load(std::memory_order_relaxed) > 0; ++i) __builtin_ia32_pause();
     std::unique_lock<std::mutex> lk(rt->mu);
     for (auto& m : moved) {
       Launch* L = find(rt, m.first);
@@ -632,6 +756,18 @@ flep_status flep_init(int device, const flep_options* opts, flep_rt* out) {
   rt->nsmid = prop.multiProcessorCount;   // probe: %nsmid == SM count, %smid dense on B200
   CUDA_TRY(cudaDeviceGetStreamPriorityRange(&rt->prio_lo, &rt->prio_hi));
   CUDA_TRY(cudaStreamCreateWithPriority(&rt->ctl, cudaStreamNonBlocking, rt->prio_hi));
+  CUDA_TRY(cudaStreamCreateWithPriority(&rt->aux, cudaStreamNonBlocking, rt->prio_lo));
+  // execution streams are pre-created (4 per priority level below the control stream's): creating
+  // one on the launch path costs 60 us to over 1 ms while kernels run
+  for (int lv = rt->prio_lo; lv >= rt->prio_hi + 1 || (lv == rt->prio_lo && rt->prio_hi == rt->prio_lo); --lv) {
+    for (int i = 0; i < 4; ++i) {
+      cudaStream_t st;
+      CUDA_TRY(cudaStreamCreateWithPriority(&st, cudaStreamNonBlocking, lv));
+      rt->all_streams.push_back(st);
+      rt->free_streams[lv].push_back(st);
+    }
+    if (rt->prio_hi == rt->prio_lo) break;
+  }
   std::vector<uint16_t> rank(256);
   for (uint32_t i = 0; i < rank.size(); ++i) rank[i] = (uint16_t)i;
   CUDA_TRY(cudaMalloc(&rt->d_rank, rank.size() * sizeof(uint16_t)));
@@ -650,15 +786,18 @@ flep_status flep_init(int device, const flep_options* opts, flep_rt* out) {
     rt->free_dmem.push_back(p);
   }
   if (rt->opt.debug_coverage) {              // debug runtimes retain 64 launches' logs: warm more
+    // (coverage buffers only with bit 0)
     for (int i = 0; i < 72; ++i) {
       void* p = nullptr;
       CUDA_TRY(cudaMalloc(&p, rt->dmem_bytes));
       CUDA_TRY(cudaMemset(p, 0, sizeof(ControlBlock)));
       rt->cb_gen[p] = 0;
       rt->free_dmem.push_back(p);
-      uint32_t* c = nullptr;
-      CUDA_TRY(cudaMalloc(&c, (size_t)(1u << 20) * 4));
-      rt->free_cov.push_back({c, (size_t)1u << 20});
+      if (rt->opt.debug_coverage & 1u) {
+        uint32_t* c = nullptr;
+        CUDA_TRY(cudaMalloc(&c, (size_t)(1u << 20) * 4));
+        rt->free_cov.push_back({c, (size_t)1u << 20});
+      }
     }
   }
   if (rt->opt.policy != FLEP_POLICY_MANUAL) {
@@ -709,7 +848,7 @@ flep_status flep_workers_for(flep_rt rt, int32_t body, uint32_t* ctas_per_sm, ui
   if (!ops) return fail(FLEP_ERR_INVALID, "unknown body %d", body);
   int k = 0;
   ApiLock lk(rt);
-  flep_status s = occupancy(rt, ops, rt->opt.debug_coverage != 0, &k);
+  flep_status s = occupancy(rt, ops, (rt->opt.debug_coverage & 1u) != 0, &k);
   if (s) return s;
   if (ctas_per_sm) *ctas_per_sm = (uint32_t)k;
   if (workers) *workers = (uint32_t)k * rt->num_sms;
@@ -733,7 +872,7 @@ flep_status flep_launch(flep_rt rt, flep_kernel kid, flep_dim3 grid, const void*
     const char* m = ops->validate(args, g);
     if (m) return fail(FLEP_ERR_INVALID, "%s", m);
   }
-  const bool cov = rt->opt.debug_coverage != 0;
+  const bool cov = (rt->opt.debug_coverage & 1u) != 0;
   const bool sw = (kr.flags & FLEP_KFLAG_SCHED_WARP) && !(kr.flags & FLEP_KFLAG_CLC);
   if (sw && !ops->worker_sw) return fail(FLEP_ERR_UNSUPPORTED, "body %d has no scheduling-warp worker", kr.body);
   int k = 0;
@@ -786,69 +925,21 @@ flep_status flep_launch(flep_rt rt, flep_kernel kid, flep_dim3 grid, const void*
   L.trig_n = rt->arm_n;
   rt->arm_block = kNoTrigger;
   rt->arm_n = 0;
-  // resources
+  // Device resources (control block, status slot, coverage / partial-tile buffers, execution
+  // stream) are taken when the launch first runs (materialize), not at interception: a managed
+  // queue can hold hundreds of intercepted launches, and only running or preempted ones need them.
   L.exec_level = stream_level(rt, priority);
-  s = get_stream(rt, L.exec_level, &L.exec);
-  if (s) return s;
-  bool fresh_cb = false;
-  if (!rt->free_dmem.empty()) { L.dmem = rt->free_dmem.back(); rt->free_dmem.pop_back(); }
-  else {
-    CUDA_TRY(cudaMalloc(&L.dmem, rt->dmem_bytes));
-    rt->cb_gen[L.dmem] = 0;
-    fresh_cb = true;             // zeroed below, on the stream the workers run on
-  }
-  L.gen0 = rt->cb_gen[L.dmem];
-  if (L.gen0 + 2 * kEvEpochs >= 0xffffffu) return fail(FLEP_ERR_NOMEM, "control block generation space exhausted");
-  L.cb = (ControlBlock*)L.dmem;
-  L.ev = (WorkerEvent*)((char*)L.dmem + sizeof(ControlBlock));
-  if (cov) {
-    for (size_t i = 0; i < rt->free_cov.size(); ++i) {
-      if (rt->free_cov[i].second >= N) {
-        L.cov = rt->free_cov[i].first; L.cov_cap = rt->free_cov[i].second;
-        rt->free_cov.erase(rt->free_cov.begin() + i);
-        break;
-      }
-    }
-    if (!L.cov) { L.cov_cap = std::max<size_t>(N, 4096); CUDA_TRY(cudaMalloc(&L.cov, L.cov_cap * 4)); }
-  }
-  if (L.flags & FLEP_KFLAG_IN_TILE) {
-    // per-worker partial-tile records and fp32 accumulator spill slots; no reset needed (the
-    // first epoch's workers clear their records)
-    const size_t need = partial_bytes(L.workers);
-    for (size_t i = 0; i < rt->free_partial.size(); ++i) {
-      if (rt->free_partial[i].second >= need) {
-        L.partial = rt->free_partial[i].first; L.partial_cap = rt->free_partial[i].second;
-        rt->free_partial.erase(rt->free_partial.begin() + i);
-        break;
-      }
-    }
-    if (!L.partial) { L.partial_cap = need; CUDA_TRY(cudaMalloc(&L.partial, need)); }
-  }
-  L.slot = rt->free_slots.back();
-  rt->free_slots.pop_back();
-  L.hs = rt->h_slots + L.slot;
-  L.ds = rt->d_slots + L.slot;
-  memset(L.hs, 0, sizeof(HostStatus));
-  // No per-launch reset work on the GPU: a pooled control block was left clean by the last
-  // worker of its previous launch's DONE epoch, and its generation numbers keep increasing.
-  const bool on_user = rt->opt.exec_on_user_stream && rt->opt.policy == FLEP_POLICY_MANUAL;
-  if (on_user) {
-    rt->free_streams[L.exec_level].push_back(L.exec);
+  L.want_cov = cov;
+  if (rt->opt.exec_on_user_stream && rt->opt.policy == FLEP_POLICY_MANUAL) {
     L.exec = L.user;
     L.exec_level = -1000;
   } else {
-    // caller's prior work on `stream` (e.g. input copies) precedes the workers
-    cudaEvent_t ev_u;
-    s = pooled_event(rt, &ev_u);
+    // the caller's prior work on `stream` (e.g. input copies) precedes the workers: its position
+    // is captured now and waited on by the execution stream when the launch materialises
+    s = pooled_event(rt, &L.ev_user);
     if (s) return s;
-    CUDA_TRY(cudaEventRecord(ev_u, L.user));
-    CUDA_TRY(cudaStreamWaitEvent(L.exec, ev_u, 0));
-    rt->event_pool.push_back(ev_u);    // reusable once recorded (waits bind at enqueue time)
+    CUDA_TRY(cudaEventRecord(L.ev_user, L.user));
   }
-  s = pooled_event(rt, &L.fin_ev);
-  if (s) return s;
-  if (L.cov) CUDA_TRY(cudaMemsetAsync(L.cov, 0, N * 4, L.exec));
-  if (fresh_cb) CUDA_TRY(cudaMemsetAsync(L.dmem, 0, sizeof(ControlBlock), L.exec));
   rt->launches[L.id] = std::move(Lp);
   *out = L.id;
   if (rt->opt.policy == FLEP_POLICY_MANUAL) return start_epoch(rt, L);
@@ -946,7 +1037,7 @@ flep_status flep_sync(flep_rt rt, flep_launch_t h, int64_t timeout_ns) {
       if (!managed) refresh(rt, *L);
       // DONE, and its last grid completed (queried under the lock: in managed mode the monitor
       // recycles the completion event once it has fired, so never block on it unlocked)
-      if (L->state == FLEP_STATE_DONE && (L->released || cudaEventQuery(L->fin_ev) == cudaSuccess)) break;
+      if (L->state == FLEP_STATE_DONE && (L->released || !L->fin_ev || cudaEventQuery(L->fin_ev) == cudaSuccess)) break;
       if (!managed && L->state == FLEP_STATE_PREEMPTED)
         return fail(FLEP_ERR_STATE, "launch %lld is preempted; resume it first", (long long)h);
       // managed: sleep until the monitor reports a state change (no lock spinning, which would
@@ -962,8 +1053,10 @@ flep_status flep_sync(flep_rt rt, flep_launch_t h, int64_t timeout_ns) {
   // keep the newest finished launches' device logs (coverage, events) for debug copies
   // (64 with the coverage log, else the last 4; the warm pool keeps launches allocation-free)
   const size_t kRetain = rt->opt.debug_coverage ? 64 : 4;
-  if (L && !L->released && std::find(rt->retained.begin(), rt->retained.end(), h) == rt->retained.end())
+  if (L && !L->released && std::find(rt->retained.begin(), rt->retained.end(), h) == rt->retained.end()) {
+    release_stream(rt, *L);                 // DONE and its last grid completed (checked above)
     rt->retained.push_back(h);
+  }
   while (rt->retained.size() > kRetain) {
     Launch* old = find(rt, rt->retained.front());
     rt->retained.erase(rt->retained.begin());
@@ -982,8 +1075,8 @@ flep_status flep_query(flep_rt rt, flep_launch_t h, flep_launch_info* out) {
     // the final counter of a silent DONE epoch (R24): one small copy from the control block
     uint32_t c = 0;
     const uint32_t e = gen_of(*L) % kEvEpochs;
-    CUDA_TRY(cudaMemcpyAsync(&c, &L->cb->ep_ctr[e], 4, cudaMemcpyDeviceToHost, L->exec));
-    CUDA_TRY(cudaStreamSynchronize(L->exec));
+    CUDA_TRY(cudaMemcpyAsync(&c, &L->cb->ep_ctr[e], 4, cudaMemcpyDeviceToHost, dbg_stream(rt, *L)));
+    CUDA_TRY(cudaStreamSynchronize(dbg_stream(rt, *L)));
     L->last_ctr = c;
     L->ctr_known = true;
   }
@@ -1043,8 +1136,8 @@ flep_status flep_cancel(flep_rt rt, flep_launch_t h) {
   if (L->exec) CUDA_TRY(cudaStreamSynchronize(L->exec));
   // the abandoned epoch left the counter word non-zero: clear the block for reuse
   if (L->epoch > 0 && L->cb && !L->sliced) {
-    CUDA_TRY(cudaMemsetAsync(L->cb, 0, offsetof(ControlBlock, ep_t_trigger), L->exec));
-    CUDA_TRY(cudaStreamSynchronize(L->exec));
+    CUDA_TRY(cudaMemsetAsync(L->cb, 0, offsetof(ControlBlock, ep_t_trigger), dbg_stream(rt, *L)));
+    CUDA_TRY(cudaStreamSynchronize(dbg_stream(rt, *L)));
   }
   L->state = FLEP_STATE_DONE;
   L->t_finish = now_ns();
@@ -1084,6 +1177,7 @@ flep_status flep_shutdown(flep_rt rt) {
   for (auto& c : rt->free_partial) cudaFree(c.first);
   for (cudaStream_t s : rt->all_streams) cudaStreamDestroy(s);
   if (rt->ctl) cudaStreamDestroy(rt->ctl);
+  if (rt->aux) cudaStreamDestroy(rt->aux);
   if (rt->d_rank) cudaFree(rt->d_rank);
   if (rt->h_slots) cudaFreeHost(rt->h_slots);
   delete rt;
@@ -1154,8 +1248,8 @@ flep_status flep_debug_copy_coverage(flep_rt rt, flep_launch_t h, uint32_t* host
   if (!L) return fail(FLEP_ERR_INVALID, "unknown launch %lld", (long long)h);
   if (!L->cov) return fail(FLEP_ERR_STATE, "coverage log not enabled or already released");
   if (n > L->n_blocks) return fail(FLEP_ERR_INVALID, "n > N");
-  CUDA_TRY(cudaMemcpyAsync(host_out, L->cov, n * 4, cudaMemcpyDeviceToHost, L->exec));
-  CUDA_TRY(cudaStreamSynchronize(L->exec));
+  CUDA_TRY(cudaMemcpyAsync(host_out, L->cov, n * 4, cudaMemcpyDeviceToHost, dbg_stream(rt, *L)));
+  CUDA_TRY(cudaStreamSynchronize(dbg_stream(rt, *L)));
   return FLEP_OK;
 }
 
@@ -1170,8 +1264,8 @@ flep_status flep_debug_copy_events(flep_rt rt, flep_launch_t h, uint32_t epoch,
     return fail(FLEP_ERR_INVALID, "epoch %u not in the log", epoch);
   const size_t n = std::min<size_t>(max_records, L->workers);
   CUDA_TRY(cudaMemcpyAsync(host_out, L->ev + (size_t)((L->gen0 + epoch) % kEvEpochs) * L->workers,
-                           n * sizeof(WorkerEvent), cudaMemcpyDeviceToHost, L->exec));
-  CUDA_TRY(cudaStreamSynchronize(L->exec));
+                           n * sizeof(WorkerEvent), cudaMemcpyDeviceToHost, dbg_stream(rt, *L)));
+  CUDA_TRY(cudaStreamSynchronize(dbg_stream(rt, *L)));
   // keep only this epoch's records: a slot nobody wrote in this epoch (a CLC CTA that was
   // cancelled, R25) still holds an older generation's record
   const uint32_t gen = L->gen0 + epoch;
@@ -1192,16 +1286,16 @@ flep_status flep_debug_epoch_info(flep_rt rt, flep_launch_t h, uint32_t epoch, f
   if (epoch == 0 || epoch > L->epoch || L->epoch - epoch >= kEvEpochs)
     return fail(FLEP_ERR_INVALID, "epoch %u not in the log", epoch);
   ControlBlock cb;
-  CUDA_TRY(cudaMemcpyAsync(&cb, L->cb, sizeof(cb), cudaMemcpyDeviceToHost, L->exec));
-  CUDA_TRY(cudaStreamSynchronize(L->exec));
+  CUDA_TRY(cudaMemcpyAsync(&cb, L->cb, sizeof(cb), cudaMemcpyDeviceToHost, dbg_stream(rt, *L)));
+  CUDA_TRY(cudaStreamSynchronize(dbg_stream(rt, *L)));
   const uint32_t e = (L->gen0 + epoch) % kEvEpochs;
   out->t_trigger = cb.ep_t_trigger[e];
   // t_end = the epoch's last worker exit. The publishing worker is the last to stop taking work
   // (R23), not necessarily the last to leave, so take the maximum over the epoch's worker log.
   std::vector<WorkerEvent> ev(L->workers);
   CUDA_TRY(cudaMemcpyAsync(ev.data(), L->ev + (size_t)e * L->workers, L->workers * sizeof(WorkerEvent),
-                           cudaMemcpyDeviceToHost, L->exec));
-  CUDA_TRY(cudaStreamSynchronize(L->exec));
+                           cudaMemcpyDeviceToHost, dbg_stream(rt, *L)));
+  CUDA_TRY(cudaStreamSynchronize(dbg_stream(rt, *L)));
   uint64_t t_end = 0;
   for (const WorkerEvent& w : ev)
     if (w.epoch == L->gen0 + epoch && w.t_exit > t_end) t_end = w.t_exit;

@@ -189,9 +189,11 @@ class Runtime:
     """One FLEP runtime on one device (flep_init ... flep_shutdown)."""
 
     def __init__(self, device=0, policy=POLICY_MANUAL, flag=FLAG_STREAM_MEMOP, chunk=8, poll=1,
-                 coverage=False, slice_blocks=0, exec_on_user_stream=False, max_overhead_ppm=0, spatial=False):
+                 coverage=False, slice_blocks=0, exec_on_user_stream=False, max_overhead_ppm=0, spatial=False,
+                 keep_logs=False):
         self.L = lib()
-        o = Options(policy, flag, chunk, poll, int(coverage), int(spatial), slice_blocks,
+        dbg = 1 if coverage else (2 if keep_logs else 0)
+        o = Options(policy, flag, chunk, poll, dbg, int(spatial), slice_blocks,
                     int(exec_on_user_stream), max_overhead_ppm)
         h = C.c_void_p()
         check(self.L.flep_init(device, C.byref(o), C.byref(h)), "flep_init")
