@@ -1112,7 +1112,9 @@ flep_status flep_cancel(flep_rt rt, flep_launch_t h) {
     ApiLock lk(rt);
     Launch* L = find(rt, h);
     if (!L) return fail(FLEP_ERR_INVALID, "unknown launch %lld", (long long)h);
-    refresh(rt, *L);
+    // managed modes: the monitor owns the state transitions (a DONE seen here would never reach
+    // the policy); it refreshes the launch and signals the condition variable
+    if (!managed) refresh(rt, *L);
     if (L->state == FLEP_STATE_DONE) return FLEP_OK;
     if (L->state == FLEP_STATE_RUNNING || L->state == FLEP_STATE_PARTIAL || L->state == FLEP_STATE_YIELDING) {
       write_ctrl(rt, *L, ctrl_word(*L, kCtrlAll));
@@ -1123,7 +1125,7 @@ flep_status flep_cancel(flep_rt rt, flep_launch_t h) {
   for (;;) {                               // wait for the running epoch to drain (or complete)
     ApiLock lk(rt);
     Launch* L = find(rt, h);
-    refresh(rt, *L);
+    if (!managed) refresh(rt, *L);
     if (L->state != FLEP_STATE_YIELDING && !(L->clc && L->state == FLEP_STATE_PREEMPTED && L->epoch > 0 &&
                                              cudaEventQuery(L->fin_ev) != cudaSuccess))
       break;

@@ -318,3 +318,95 @@ def test_custom_rank_table_spatial_yield():
         rt.set_rank_table(list(range(max(S, rt.nsmid))))
     finally:
         rt.close()
+
+
+def _replay_ex(rt, spatial):
+    evs = []
+    for (t_ns, typ, lid, prio, t_e, ovh, need) in rt.event_log_ex():
+        if typ == 0:
+            evs.append((t_ns, "ARRIVE", des.KernelSpec(lid, t_ns, prio, t_e, ovh, 0, need)))
+        else:
+            evs.append((t_ns, "FINISH", lid))
+    acts = {"LAUNCH": 0, "RESUME": 1, "PREEMPT": 2, "REFILL": 3}
+    return [(t_, acts[a], i, n) for (t_, a, i, n) in des.replay(des.HPF, evs, num_sms=rt.num_sms, spatial=spatial)]
+
+
+@pytest.mark.parametrize("n_sms", [5, 16, 74])
+def test_managed_spatial_hpf_decides_how_far(n_sms):
+    """Spatial HPF (R29): a high-priority SAXPY-int32 whose workers fit on n SMs
+    arrives while an int32 stencil 8192^2 runs; the runtime yields exactly n SMs (rank < n), runs
+    the waiting kernel beside the victim, refills the victim at its end. Checked: decision list
+    (and its oracle replay), I3 on the victim's worker log, every block exactly once, both
+    outputs bit-exact vs the oracle."""
+    f = flep_mod()
+    import torch
+    rt = f.Runtime(policy=f.POLICY_HPF, spatial=True, coverage=True)
+    try:
+        nst = 8192
+        a = gen.stencil_i32_input(nst, seed=61)
+        ind = t(a)
+        outd = torch.empty_like(ind)
+        k_v = rt.register_kernel(f.BODY_STENCIL5_I32, chunk=1, poll=1, model=(0, 0, 0, 0, 400_000))
+        cps, _ = rt.workers_for(f.BODY_SAXPY_I32)
+        n_hp = n_sms * cps * 256 - 77                      # ragged tail, still n_sms * cps blocks
+        x2, y2 = gen.saxpy_i32_inputs(n_hp, seed=62)
+        x2d, y2d = t(x2), t(y2)
+        k_w = rt.register_kernel(f.BODY_SAXPY_I32, chunk=1, poll=1, model=(0, 0, 0, 0, 5_000))
+        sA, sB = torch.cuda.Stream(), torch.cuda.Stream()
+        h_v = rt.launch(k_v, f.stencil_grid(nst), f.stencil_args(outd, ind), priority=0, stream=sA)
+        h_w = rt.launch(k_w, f.saxpy_grid(n_hp), f.saxpy_i32_args(y2d, x2d, 5), priority=1, stream=sB)
+        rt.sync(h_w, timeout_ns=10_000_000_000)
+        rt.sync(h_v, timeout_ns=10_000_000_000)
+        torch.cuda.synchronize()
+        assert np.array_equal(y2d.cpu().numpy(), W.saxpy_i32(5, x2, y2))
+        assert np.array_equal(outd.cpu().numpy(), W.stencil5_i32(a))
+        nb = (nst // 64) ** 2
+        assert np.all(rt.coverage_np(h_v, nb) == 1)
+        dec = rt.decision_log()
+        names = [(f.ACTION_NAMES[d[1]], d[2], d[3]) for d in dec]
+        assert names[:3] == [("LAUNCH", h_v, 0), ("PREEMPT", h_v, n_sms), ("LAUNCH", h_w, 0)]
+        # the guest ends long before the victim: REFILL (if both completions land in one monitor
+        # pass the victim may be seen first; the replay below checks that order too)
+        if len(names) == 4:
+            assert names[3] == ("REFILL", h_v, rt.num_sms)
+        ev1 = rt.events(h_v, 1)
+        w_end = max(e.t_exit for e in rt.events(h_w, 1))
+        assert all(e.reason == f.REASON_YIELD for e in ev1 if e.smid < n_sms)
+        assert not any(e.reason == f.REASON_YIELD and e.t_exit < w_end for e in ev1 if e.smid >= n_sms)
+        assert dec == _replay_ex(rt, True)
+    finally:
+        rt.close()
+
+
+def test_managed_cancel_releases_the_policy():
+    """flep_cancel in a managed mode: the policy forgets the cancelled launch, so the
+    kernels behind it still run, and its resources go back to the pools."""
+    f = flep_mod()
+    import torch
+    rt = f.Runtime(policy=f.POLICY_FIFO)
+    try:
+        n = 1 << 26
+        x, y = gen.saxpy_i32_inputs(n, seed=71)
+        xd, yd = t(x), t(y)
+        k = rt.register_kernel(f.BODY_SAXPY_I32, chunk=1, poll=1)
+        n2 = 1 << 18
+        x2, y2 = gen.saxpy_i32_inputs(n2, seed=72)
+        x2d, y2d = t(x2), t(y2)
+        h1 = rt.launch(k, f.saxpy_grid(n), f.saxpy_i32_args(yd, xd, 3))        # running
+        h2 = rt.launch(k, f.saxpy_grid(n), f.saxpy_i32_args(yd, xd, 3))        # queued behind it
+        h3 = rt.launch(k, f.saxpy_grid(n2), f.saxpy_i32_args(y2d, x2d, 11))    # queued
+        rt.cancel(h2)                                                           # a queued one
+        rt.cancel(h1)                                                           # the running one
+        rt.sync(h3, timeout_ns=10_000_000_000)
+        torch.cuda.synchronize()
+        assert np.array_equal(y2d.cpu().numpy(), W.saxpy_i32(11, x2, y2))
+        for h in (h1, h2, h3):
+            assert rt.query(h).state == f.STATE_DONE
+        for _ in range(20):                                                     # pools still work
+            y2d.copy_(t(y2))
+            h = rt.launch(k, f.saxpy_grid(n2), f.saxpy_i32_args(y2d, x2d, 11))
+            rt.sync(h, timeout_ns=10_000_000_000)
+            torch.cuda.synchronize()
+            assert np.array_equal(y2d.cpu().numpy(), W.saxpy_i32(11, x2, y2))
+    finally:
+        rt.close()

@@ -142,3 +142,39 @@ def test_b200_queue_trace_replays_exactly_through_the_oracle():
         checked += len(dec)
     assert checked > 100
     assert sum(1 for d in logs["HPF"]["decisions"] if d[1] == ACT["PREEMPT"]) > 5
+
+
+def test_b200_slice_queue_log_replays_exactly():
+    """Round-2 B200 queue run (configs[3], tests/golden/queue_logs_r02.json): every policy's log,
+    including kernel slicing (SLICE takes HPF's decisions, R16), replays bit for bit."""
+    import json
+    import os
+    path = os.path.join(os.path.dirname(__file__), "golden", "queue_logs_r02.json")
+    with open(path) as fh:
+        logs = json.load(fh)["logs"]
+    kinds = {"FIFO": des.FIFO, "HPF": des.HPF, "SLICE": des.SLICE, "REORDER": des.REORDER}
+    for name, kind in kinds.items():
+        evl, dec = logs[name]["events"], logs[name]["decisions"]
+        evs = [(t, "ARRIVE", des.KernelSpec(i, t, p, te, o)) if ty == 0 else (t, "FINISH", i)
+               for (t, ty, i, p, te, o) in evl]
+        assert as_tuples(des.replay(kind, evs)) == [tuple(d) for d in dec], name
+    assert sum(1 for d in logs["SLICE"]["decisions"] if d[1] == ACT["PREEMPT"]) > 0
+
+
+def test_b200_managed_spatial_log_replays_exactly():
+    """The managed spatial-HPF run of configs[2] on the B200 (tests/golden/spatial_managed_logs_r02.json,
+    written by bench.py --config spatial_managed): the runtime's event log (with each launch's
+    sms_need) replayed through the oracle DES with spatial decisions gives its decision list bit
+    for bit, including PREEMPT widths 8/16/32/74 (< 148) and the REFILLs (R29)."""
+    import json
+    import os
+    path = os.path.join(os.path.dirname(__file__), "golden", "spatial_managed_logs_r02.json")
+    with open(path) as fh:
+        d = json.load(fh)
+    evs = [(t, "ARRIVE", des.KernelSpec(i, t, p, te, o, 0, need)) if ty == 0 else (t, "FINISH", i)
+           for (t, ty, i, p, te, o, need) in d["events"]]
+    got = as_tuples(des.replay(des.HPF, evs, num_sms=d["num_sms"], spatial=True))
+    assert got == [tuple(x) for x in d["decisions"]]
+    widths = sorted({x[3] for x in d["decisions"] if x[1] == ACT["PREEMPT"]})
+    assert widths == [8, 16, 32, 74, 148]
+    assert sum(1 for x in d["decisions"] if x[1] == ACT["REFILL"]) >= 40
