@@ -86,9 +86,12 @@ typedef enum {
   FLEP_BODY_STENCIL5_I32 = 5,  /* 5-point integer sweep, wraps mod 2^32; 64x64 cells per block */
   FLEP_BODY_GEMM_BF16 = 6,     /* C = A B^T, bf16 in, fp32 accumulate (tcgen05), bf16 out;
                                   128x256 output tile per block */
-  FLEP_BODY_STENCIL5_F32_TMA = 7 /* STENCIL5_F32 with the tile and its halo staged in shared memory
+  FLEP_BODY_STENCIL5_F32_TMA = 7, /* STENCIL5_F32 with the tile and its halo staged in shared memory
                                   by the TMA unit and the output tile written back by a bulk
                                   tensor store; same args; n % 4 == 0, 16-byte aligned in/out */
+  FLEP_BODY_SPMV_CSR_F32_VEC = 8 /* y = A x, CSR fp32, CSR-vector form (4 lanes per row, shuffle
+                                  reduction, no shared memory); same args; 128 rows per block,
+                                  each warp owns 16 of them (warp-task capable, R30) */
 } flep_body;
 
 /* Per-body argument structs (copied by value at launch). All pointers are device pointers. */
@@ -178,6 +181,15 @@ typedef struct {
    control word, so a request reaches the workers in ~1 us instead of waiting for the stream memop
    (~5 us, tens of us behind copy-engine work). Takes one resident slot (W = k x SMs - 1). */
 #define FLEP_KFLAG_HOST_RELAY 64u
+/* Warp-task worker (R30; STENCIL5_F32/I32 and SPMV_CSR_F32_VEC, not with CLC,
+   scheduling warp, in-tile or the SLICE policy): the unit of work is one warp's share of an
+   original block (task = block x 8 + warp) and every warp of a worker CTA fetches, polls and
+   exits on its own, so no warp waits for another at a chunk boundary and a request is acted on
+   after one warp task. For these launches the counter, the coverage log, the done count
+   (flep_launch_info.blocks_total / blocks_done / counter), the chunk C and the debug trigger's
+   block index are in tasks (flep_launch_info.tasks_per_block = 8; the trigger index given in
+   blocks is converted); worker records are per warp. */
+#define FLEP_KFLAG_WARP_TASKS 128u
 
 typedef enum {
   FLEP_STATE_QUEUED = 0,     /* intercepted, waiting for a scheduling decision (S2) */
@@ -202,7 +214,7 @@ typedef struct {
   int64_t t_last_drain;        /* host ns the runtime observed the last PREEMPTED epoch end */
   uint32_t started_epoch;      /* newest epoch (1-based) whose first worker has begun running
                                   (kernels registered with FLEP_KFLAG_STARTED_HINT; else 0) */
-  uint32_t reserved;
+  uint32_t tasks_per_block;    /* 1, or 8 for FLEP_KFLAG_WARP_TASKS launches (counts are in tasks) */
 } flep_launch_info;
 
 /* Per-worker event record of one epoch (device %globaltimer, ns). */
@@ -223,6 +235,10 @@ typedef struct {
   uint32_t done;           /* done counter at epoch end */
   uint32_t counter;        /* task counter at epoch end */
   uint32_t state;          /* 3 = PREEMPTED, 5 = DONE */
+  uint32_t relay_smid;     /* FLEP_KFLAG_HOST_RELAY: SM of the epoch's relay CTA */
+  uint32_t relay_reason;   /* why it left: 1 = a spatial request released its SM, 2 = it relayed
+                              a temporal request, 3 = the epoch was published; 0 = no relay */
+  uint64_t relay_t_exit;   /* when it left (%globaltimer) */
 } flep_epoch_info;
 
 /* ---- lifecycle ------------------------------------------------------------------------ */

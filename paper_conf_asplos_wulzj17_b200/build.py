@@ -40,6 +40,8 @@ def needs_build() -> bool:
 
 
 def build(force: bool = False, verbose: bool = False) -> str:
+    if os.environ.get("FLEP_LIB_PATH"):          # an experiment's prebuilt variant (flep.py loads it)
+        return os.environ["FLEP_LIB_PATH"]
     if not force and not needs_build():
         return LIB
     extra = os.environ.get("FLEP_NVCC_EXTRA", "").split()     # experiment hook (e.g. -DFLEP_SPMV_U=4)

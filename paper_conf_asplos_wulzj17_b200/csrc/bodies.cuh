@@ -294,60 +294,118 @@ struct Stencil5Body : NoResources {
   // Vector path (n % 4 == 0): thread (q, rg) owns columns [c0+4q, c0+4q+4) of rows
   // r0+4rg .. r0+4rg+3. It loads the 6 rows r-1..r+4 of its 4-column strip (128-bit) and the
   // west/east neighbours of its 4 rows up front (14 independent loads in flight), then computes.
-  __device__ static void run(const Args& g, uint32_t b0, uint32_t b1, uint32_t gx, uint32_t) {
+  // Thread tid's work depends on (b, tid) only, so warp w of a block (threads 32w..32w+31, rows
+  // r0+8w..r0+8w+7) is an independent task of the warp-task worker (R30).
+  static constexpr uint32_t kWarpTasks = kThreads / 32;
+  __device__ __forceinline__ static void run_thread(const Args& g, uint32_t b, uint32_t tid, uint32_t gx) {
     const uint32_t n = g.n;
     const uint32_t* __restrict__ in = reinterpret_cast<const uint32_t*>(g.in);
     uint32_t* __restrict__ out = reinterpret_cast<uint32_t*>(g.out);
-    for (uint32_t b = b0; b < b1; ++b) {
-      const uint32_t tx = b % gx, ty = b / gx;
-      const uint32_t r0 = ty * kTile, c0 = tx * kTile;
-      if ((n & 3u) == 0) {
-        const uint32_t q = threadIdx.x & 15u, rg = threadIdx.x >> 4;   // 16 strips x 16 row groups
-        const uint32_t c = c0 + 4u * q;
-        const uint32_t rb = r0 + 4u * rg;
-        if (c >= n || rb >= n) continue;
-        uint4 R[6];
-        uint32_t Wv[4], Ev[4];
+    const uint32_t tx = b % gx, ty = b / gx;
+    const uint32_t r0 = ty * kTile, c0 = tx * kTile;
+    if ((n & 3u) == 0) {
+      const uint32_t q = tid & 15u, rg = tid >> 4;   // 16 strips x 16 row groups
+      const uint32_t c = c0 + 4u * q;
+      const uint32_t rb = r0 + 4u * rg;
+      if (c >= n || rb >= n) return;
+      uint4 R[6];
+      uint32_t Wv[4], Ev[4];
 #pragma unroll
-        for (int i = 0; i < 6; ++i) {
-          const int32_t r = (int32_t)rb - 1 + i;
-          R[i] = (r >= 0 && r < (int32_t)n) ? __ldg(reinterpret_cast<const uint4*>(in + (size_t)r * n + c))
-                                            : make_uint4(0, 0, 0, 0);
-        }
+      for (int i = 0; i < 6; ++i) {
+        const int32_t r = (int32_t)rb - 1 + i;
+        R[i] = (r >= 0 && r < (int32_t)n) ? __ldg(reinterpret_cast<const uint4*>(in + (size_t)r * n + c))
+                                          : make_uint4(0, 0, 0, 0);
+      }
 #pragma unroll
-        for (int i = 0; i < 4; ++i) {
-          const uint32_t r = rb + i;
-          Wv[i] = (r < n && c > 0) ? __ldg(in + (size_t)r * n + c - 1) : 0u;
-          Ev[i] = (r < n && c + 4 < n) ? __ldg(in + (size_t)r * n + c + 4) : 0u;
-        }
+      for (int i = 0; i < 4; ++i) {
+        const uint32_t r = rb + i;
+        Wv[i] = (r < n && c > 0) ? __ldg(in + (size_t)r * n + c - 1) : 0u;
+        Ev[i] = (r < n && c + 4 < n) ? __ldg(in + (size_t)r * n + c + 4) : 0u;
+      }
 #pragma unroll
-        for (int i = 0; i < 4; ++i) {
-          const uint32_t r = rb + i;
-          if (r >= n) break;
-          const uint4 C = R[i + 1], N = R[i], S = R[i + 2];
-          uint4 O;
-          if (r == 0 || r == n - 1) {
-            O = C;
-          } else {
-            O.x = (c == 0) ? C.x : cell(C.x, N.x, S.x, Wv[i], C.y);
-            O.y = cell(C.y, N.y, S.y, C.x, C.z);
-            O.z = cell(C.z, N.z, S.z, C.y, C.w);
-            O.w = (c + 3 == n - 1) ? C.w : cell(C.w, N.w, S.w, C.z, Ev[i]);
-          }
-          __stcs(reinterpret_cast<uint4*>(out + (size_t)r * n + c), O);
+      for (int i = 0; i < 4; ++i) {
+        const uint32_t r = rb + i;
+        if (r >= n) break;
+        const uint4 C = R[i + 1], N = R[i], S = R[i + 2];
+        uint4 O;
+        if (r == 0 || r == n - 1) {
+          O = C;
+        } else {
+          O.x = (c == 0) ? C.x : cell(C.x, N.x, S.x, Wv[i], C.y);
+          O.y = cell(C.y, N.y, S.y, C.x, C.z);
+          O.z = cell(C.z, N.z, S.z, C.y, C.w);
+          O.w = (c + 3 == n - 1) ? C.w : cell(C.w, N.w, S.w, C.z, Ev[i]);
         }
-      } else {
-        // scalar path for n % 4 != 0 (ragged rows)
-        for (uint32_t t = threadIdx.x; t < kTile * kTile; t += kThreads) {
-          const uint32_t r = r0 + t / kTile, c = c0 + t % kTile;
-          if (r >= n || c >= n) continue;
-          const size_t off = (size_t)r * n + c;
-          const uint32_t C = __ldg(in + off);
-          if (r == 0 || r == n - 1 || c == 0 || c == n - 1) { out[off] = C; continue; }
-          out[off] = cell(C, __ldg(in + off - n), __ldg(in + off + n), __ldg(in + off - 1), __ldg(in + off + 1));
-        }
+        __stcs(reinterpret_cast<uint4*>(out + (size_t)r * n + c), O);
+      }
+    } else {
+      // scalar path for n % 4 != 0 (ragged rows)
+      for (uint32_t t = tid; t < kTile * kTile; t += kThreads) {
+        const uint32_t r = r0 + t / kTile, c = c0 + t % kTile;
+        if (r >= n || c >= n) continue;
+        const size_t off = (size_t)r * n + c;
+        const uint32_t C = __ldg(in + off);
+        if (r == 0 || r == n - 1 || c == 0 || c == n - 1) { out[off] = C; continue; }
+        out[off] = cell(C, __ldg(in + off - n), __ldg(in + off + n), __ldg(in + off - 1), __ldg(in + off + 1));
       }
     }
+  }
+  __device__ static void run(const Args& g, uint32_t b0, uint32_t b1, uint32_t gx, uint32_t) {
+    for (uint32_t b = b0; b < b1; ++b) run_thread(g, b, threadIdx.x, gx);
+  }
+  __device__ static void run_warp(const Args& g, uint32_t task, uint32_t gx, uint32_t) {
+    run_thread(g, task / kWarpTasks, (task % kWarpTasks) * 32u + (threadIdx.x & 31u), gx);
+  }
+};
+
+// ---------------------------------------------------------------------------------------------
+// SpMV-CSR fp32, CSR-vector form (FLEP_BODY_SPMV_CSR_F32_VEC): block b = rows [128b, 128b+128),
+// 4 lanes per row, 8 rows per warp per pass, 2 passes: warp w of block b owns rows
+// 128b + 64*pass + 8w + lane/4. Lane l of a row's group sums the row's nonzeros p = s+l, s+l+4,
+// ... in ascending order (U in flight) and the group's 4 partial sums are combined by two
+// butterfly shuffles. No shared memory and no CTA barrier: warp w's rows are an independent task
+// of the warp-task worker (R30); every execution of a row is the same arithmetic in the same order.
+struct SpmvVecBody : NoResources {
+  static constexpr int kThreads = 256;
+  static constexpr int kMinBlocks = 8;
+  static constexpr uint32_t kRowsPerBlock = 128;
+  static constexpr uint32_t kWarpTasks = kThreads / 32;
+  using Args = flep_spmv_args;
+
+  __device__ __forceinline__ static void rows_of_warp(const Args& g, uint32_t b, uint32_t w, uint32_t lane) {
+    constexpr int U = FLEP_SPMV_U;
+    const int32_t sub = (int32_t)(lane & 3u);
+#pragma unroll 1
+    for (uint32_t pass = 0; pass < 2; ++pass) {
+      const uint32_t r = b * kRowsPerBlock + pass * 64u + w * 8u + (lane >> 2);
+      const bool valid = r < g.rows;
+      const int32_t s = valid ? __ldg(g.rowptr + r) : 0, e = valid ? __ldg(g.rowptr + r + 1) : 0;
+      float acc = 0.f;
+      for (int32_t p = s + sub; p < e; p += 4 * U) {
+        int32_t c[U];
+        float v[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+          const int32_t q = p + 4 * u;
+          c[u] = q < e ? __ldcs(g.col + q) : 0;
+          v[u] = q < e ? __ldcs(g.val + q) : 0.f;
+        }
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+          const float xv = __ldg(g.x + c[u]);
+          if (p + 4 * u < e) acc += v[u] * xv;
+        }
+      }
+      acc += __shfl_xor_sync(0xffffffffu, acc, 1);
+      acc += __shfl_xor_sync(0xffffffffu, acc, 2);
+      if (valid && sub == 0) __stcs(g.y + r, acc);
+    }
+  }
+  __device__ static void run(const Args& g, uint32_t b0, uint32_t b1, uint32_t, uint32_t) {
+    for (uint32_t b = b0; b < b1; ++b) rows_of_warp(g, b, threadIdx.x >> 5, threadIdx.x & 31u);
+  }
+  __device__ static void run_warp(const Args& g, uint32_t task, uint32_t, uint32_t) {
+    rows_of_warp(g, task / kWarpTasks, task % kWarpTasks, threadIdx.x & 31u);
   }
 };
 

@@ -62,7 +62,12 @@ struct alignas(128) ControlBlock {
   uint32_t ep_done[kEvEpochs];
   uint32_t ep_ctr[kEvEpochs];
   uint32_t ep_state[kEvEpochs];
+  uint32_t ep_relay[kEvEpochs];     // request-relay CTA of the epoch (R28): smid << 8 | why it left
+  uint64_t ep_relay_t[kEvEpochs];   // ... and when (%globaltimer)
 };
+constexpr uint32_t kRelayLeftOwnSm = 1;     // a spatial request released the relay's own SM (I3)
+constexpr uint32_t kRelayLeftTemporal = 2;  // it relayed a temporal request
+constexpr uint32_t kRelayLeftPublished = 3; // the epoch was published
 
 struct WorkerEvent {       // mirrors flep_worker_event
   uint32_t smid, reason, n_blocks, epoch;
@@ -291,7 +296,8 @@ __device__ __forceinline__ void note_exit_event(const WorkerParams& p, WorkerSha
   ws.ev_part = (uint32_t)(old >> 48) + own_partial;
 }
 
-__device__ __forceinline__ uint32_t next_chunk(const WorkerParams& p, SchedState& st, WorkerShared& ws) {
+__device__ __forceinline__ uint32_t next_chunk(const WorkerParams& p, SchedState& st, WorkerShared& ws,
+                                               uint32_t wid = blockIdx.x) {
   uint32_t base = 0xffffffffu;
   bool have = false;
   if (st.first) {
@@ -300,7 +306,7 @@ __device__ __forceinline__ uint32_t next_chunk(const WorkerParams& p, SchedState
       // First epoch: worker i starts on the static chunk [i*C, i*C + C) (R20): no poll and no
       // atomic before the first body, so the grid starts moving data at once. A static chunk is
       // "fetched" at launch and always processed (A4); the first poll comes at the next step.
-      base = blockIdx.x * p.chunk;
+      base = wid * p.chunk;
       have = true;
     } else {
       // A later epoch: the launch may already have completed in an earlier one (a refill raced
@@ -361,11 +367,13 @@ __device__ __forceinline__ uint32_t next_chunk(const WorkerParams& p, SchedState
 // any other (yield, entry exit) makes its exit event now: one 64-bit increment of the yield
 // count (R23). No fences: the outputs are published by kernel completion (stream order), and
 // the host status is a notification (flep_sync also waits for the grid's completion event).
-__device__ __forceinline__ void worker_exit(const WorkerParams& p, WorkerShared& ws) {
-  WorkerEvent& e = p.ev[(p.epoch % kEvEpochs) * p.workers + blockIdx.x];
+__device__ __forceinline__ void worker_exit(const WorkerParams& p, WorkerShared& ws, uint32_t wid = blockIdx.x) {
   const uint64_t t_exit = gtimer();
+#ifndef FLEP_NO_EVLOG          // experiment knob: no per-worker record (measures its cost)
+  WorkerEvent& e = p.ev[(p.epoch % kEvEpochs) * p.workers + wid];
   e.smid = ws.sm; e.reason = ws.reason; e.n_blocks = ws.blocks; e.epoch = p.epoch;
   e.t_entry = ws.t_entry; e.t_exit = t_exit;
+#endif
   if (!ws.counted) {
     const unsigned long long inc = (1ull << 32) | ((unsigned long long)ws.partial << 48);
     note_exit_event(p, ws, atom_add_cx(&p.cb->cx, inc), 0u, ws.partial);
@@ -411,18 +419,28 @@ __device__ __forceinline__ void worker_exit(const WorkerParams& p, WorkerShared&
 // every worker then leaves at its next poll).
 __device__ __forceinline__ void request_relay(const WorkerParams& p) {
   if (threadIdx.x != 0) return;
-  uint32_t last;
+  const uint32_t sm = smid_reg();
+  uint32_t last, why = 0;
   asm volatile("ld.relaxed.sys.global.u32 %0, [%1];" : "=r"(last) : "l"(&p.status->ctrl) : "memory");
-  while (true) {
+  while (!why) {
     uint32_t h;
     asm volatile("ld.relaxed.sys.global.u32 %0, [%1];" : "=r"(h) : "l"(&p.status->ctrl) : "memory");
     if (h != last) {
       last = h;
       atomicExch(p.ctrl, h);
-      if (ctrl_gen(h) == (p.epoch & kCtrlGenMask) && ctrl_n(h) >= p.num_sms) return;
+      if (ctrl_gen(h) == (p.epoch & kCtrlGenMask) && ctrl_n(h) > 0) {
+        // a temporal request: every worker leaves at its next poll; a spatial one that releases
+        // this SM: the relay leaves it too (I3 covers every CTA of the grid; later requests still
+        // arrive by the stream memop)
+        if (ctrl_n(h) >= p.num_sms) why = kRelayLeftTemporal;
+        else if (p.rank[sm] < ctrl_n(h)) why = kRelayLeftOwnSm;
+      }
     }
-    if (ld_relaxed_gpu(&p.cb->pub_gen) == p.epoch) return;
+    if (!why && ld_relaxed_gpu(&p.cb->pub_gen) == p.epoch) why = kRelayLeftPublished;
   }
+  const uint32_t e = p.epoch % kEvEpochs;
+  p.cb->ep_relay[e] = (sm << 8) | why;
+  p.cb->ep_relay_t[e] = gtimer();
 }
 
 // The worker. Body contract:
@@ -559,6 +577,43 @@ flep_worker_sw(const __grid_constant__ typename Body::Args args, const WorkerPar
   __syncthreads();
   Body::teardown(args);
   if (tid == kT) worker_exit(p, ws);
+}
+
+// ---- warp-task worker (FLEP_KFLAG_WARP_TASKS, reading R30) ---------------------------------
+// For bodies whose warps never communicate (no shared memory between warps, no CTA barrier in
+// run()): a task is one warp's share of an original block (task t = b * kWarpTasks + w, run by
+// Body::run_warp with the 32 lanes of one warp, exactly what warp w of the original CTA computes)
+// and every warp of a worker CTA is a worker of its own: its lane 0 polls, fetches and makes its
+// exit event (the same scheduling step as flep_worker, with the worker index wid = CTA * warps +
+// warp), the chunk base reaches the other lanes by a shuffle, and no warp ever waits for another
+// at a chunk boundary. A request is seen by each warp at its own next poll, so the drain is one
+// warp task (a fraction of a block) instead of the slowest warp of a whole chunk.
+template <class Body, bool kCoverage>
+__global__ void __launch_bounds__(Body::kThreads, Body::kMinBlocks)
+flep_warp_worker(const __grid_constant__ typename Body::Args args, const WorkerParams p) {
+  constexpr uint32_t kWarps = Body::kThreads / 32;
+  __shared__ WorkerShared wss[kWarps];
+  if (blockIdx.x == p.relay_block) { request_relay(p); return; }   // R28: not a worker
+  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31u;
+  const uint32_t wid = blockIdx.x * kWarps + warp;
+  WorkerShared& ws = wss[warp];
+  if (lane == 0) {
+    ws.sm = smid_reg(); ws.t_entry = gtimer(); ws.blocks = 0; ws.reason = 0;
+    ws.counted = 0; ws.last = 0; ws.ev_raw = 0; ws.ev_part = 0; ws.partial = 0;
+    if (wid == 0 && p.started_hint && p.status) st_relaxed_sys(&p.status->started, p.epoch);
+  }
+  SchedState st;                     // used by lane 0 only
+  while (true) {
+    uint32_t base = 0;
+    if (lane == 0) base = next_chunk(p, st, ws, wid);
+    base = __shfl_sync(0xffffffffu, base, 0);
+    if (base == 0xffffffffu) break;
+    const uint32_t end = min(base + p.chunk, p.n_blocks);
+    for (uint32_t t = base; t < end; ++t) Body::run_warp(args, t, p.gx, p.gy);
+    if (kCoverage && lane == 0)
+      for (uint32_t t = base; t < end; ++t) atomicAdd(&p.cov[t], 1u);
+  }
+  if (lane == 0) worker_exit(p, ws, wid);
 }
 
 // ---- CLC task fetch (reading R25) ----------------------------------------------

@@ -38,6 +38,16 @@ struct Ops {
     if (cov) return cudaOccupancyMaxActiveBlocksPerMultiprocessor(k, flep_worker_sw<Body, true>, Body::kThreads + 32, Body::kDynSmem);
     return cudaOccupancyMaxActiveBlocksPerMultiprocessor(k, flep_worker_sw<Body, false>, Body::kThreads + 32, Body::kDynSmem);
   }
+  static cudaError_t warp_worker(const void* args, const WorkerParams& p, uint32_t G, cudaStream_t s, bool cov) {
+    const typename Body::Args& a = *reinterpret_cast<const typename Body::Args*>(args);
+    if (cov) flep_warp_worker<Body, true><<<G, Body::kThreads, Body::kDynSmem, s>>>(a, p);
+    else flep_warp_worker<Body, false><<<G, Body::kThreads, Body::kDynSmem, s>>>(a, p);
+    return cudaGetLastError();
+  }
+  static cudaError_t occupancy_warp(int* k, bool cov) {
+    if (cov) return cudaOccupancyMaxActiveBlocksPerMultiprocessor(k, flep_warp_worker<Body, true>, Body::kThreads, Body::kDynSmem);
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(k, flep_warp_worker<Body, false>, Body::kThreads, Body::kDynSmem);
+  }
   static cudaError_t unwrapped(const void* args, dim3 grid, uint32_t offset, uint32_t count,
                                cudaStream_t s) {
     const typename Body::Args& a = *reinterpret_cast<const typename Body::Args*>(args);
@@ -131,6 +141,7 @@ namespace {
 using SaxpyI32 = WithSmem<SaxpyBody<true>>;
 using SaxpyF32 = WithSmem<SaxpyBody<false>>;
 using Spmv = WithSmem<SpmvBody>;
+using SpmvVec = WithSmem<SpmvVecBody>;
 using StencilF32 = WithSmem<Stencil5Body<false>>;
 using StencilI32 = WithSmem<Stencil5Body<true>>;
 
@@ -147,15 +158,21 @@ const BodyOps kOps[] = {
      &Ops<Spmv>::worker_sw, &Ops<Spmv>::occupancy_sw},
     {FLEP_BODY_STENCIL5_F32, StencilF32::kThreads, sizeof(flep_stencil_args), &Ops<StencilF32>::worker,
      &Ops<StencilF32>::unwrapped, &Ops<StencilF32>::occupancy, nullptr, &Ops<StencilF32>::clc,
-     &Ops<StencilF32>::worker_sw, &Ops<StencilF32>::occupancy_sw},
+     &Ops<StencilF32>::worker_sw, &Ops<StencilF32>::occupancy_sw, &Ops<StencilF32>::warp_worker,
+     &Ops<StencilF32>::occupancy_warp, StencilF32::kWarpTasks},
     {FLEP_BODY_STENCIL5_I32, StencilI32::kThreads, sizeof(flep_stencil_args), &Ops<StencilI32>::worker,
      &Ops<StencilI32>::unwrapped, &Ops<StencilI32>::occupancy, nullptr, &Ops<StencilI32>::clc,
-     &Ops<StencilI32>::worker_sw, &Ops<StencilI32>::occupancy_sw},
+     &Ops<StencilI32>::worker_sw, &Ops<StencilI32>::occupancy_sw, &Ops<StencilI32>::warp_worker,
+     &Ops<StencilI32>::occupancy_warp, StencilI32::kWarpTasks},
     {FLEP_BODY_GEMM_BF16, GemmBody::kThreads, sizeof(flep_gemm_args), &gemm_worker_launch,
      &gemm_unwrapped_launch, &gemm_occupancy, &gemm_validate, nullptr, nullptr, nullptr},
     {FLEP_BODY_STENCIL5_F32_TMA, Stencil5TmaBody::kThreads, sizeof(flep_stencil_args), &stencil_tma_worker_launch,
      &stencil_tma_unwrapped_launch, &stencil_tma_occupancy, &stencil_tma_validate, &stencil_tma_clc_launch,
      nullptr, nullptr},
+    {FLEP_BODY_SPMV_CSR_F32_VEC, SpmvVec::kThreads, sizeof(flep_spmv_args), &Ops<SpmvVec>::worker,
+     &Ops<SpmvVec>::unwrapped, &Ops<SpmvVec>::occupancy, nullptr, &Ops<SpmvVec>::clc,
+     &Ops<SpmvVec>::worker_sw, &Ops<SpmvVec>::occupancy_sw, &Ops<SpmvVec>::warp_worker,
+     &Ops<SpmvVec>::occupancy_warp, SpmvVec::kWarpTasks},
 };
 
 }  // namespace
@@ -167,7 +184,7 @@ cudaError_t set_unwrapped_trace(uint64_t* p) {
 #endif
 
 const BodyOps* body_ops(int32_t body) {
-  if (body < 1 || body > FLEP_BODY_STENCIL5_F32_TMA) return nullptr;
+  if (body < 1 || body > FLEP_BODY_SPMV_CSR_F32_VEC) return nullptr;
   return &kOps[body];
 }
 

@@ -27,6 +27,11 @@ struct BodyOps {
   // nullptr for bodies that own their loop or synchronise the whole CTA inside run()
   cudaError_t (*worker_sw)(const void* args, const WorkerParams& p, uint32_t W, cudaStream_t s, bool cov);
   cudaError_t (*occupancy_sw)(int* ctas_per_sm, bool cov);
+  // warp-task worker (flep_warp_worker<Body>, R30): launch G CTAs (G x threads/32 warp workers)
+  // and its occupancy; warp_tasks = tasks per original block (0 = the body does not decompose)
+  cudaError_t (*warp_worker)(const void* args, const WorkerParams& p, uint32_t G, cudaStream_t s, bool cov);
+  cudaError_t (*occupancy_warp)(int* ctas_per_sm, bool cov);
+  uint32_t warp_tasks;
 };
 
 const BodyOps* body_ops(int32_t body);

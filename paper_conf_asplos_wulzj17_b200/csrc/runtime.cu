@@ -85,7 +85,7 @@ flep_status resolve_driver() {
 }
 
 constexpr uint32_t kMaxSlots = 1u << 14;       // pinned status slots (recycled)
-constexpr uint32_t kMaxWorkersPerSm = 32;
+constexpr uint32_t kMaxWorkersPerSm = 64;     // warp workers: 8 CTAs x 8 warps
 
 struct Launch {
   int64_t id = 0;
@@ -127,6 +127,9 @@ struct Launch {
   bool clc = false;                  // FLEP_KFLAG_CLC: hardware work queue, resume = clear (R25)
   bool sw = false;                   // FLEP_KFLAG_SCHED_WARP: scheduling-warp worker (R26)
   bool relay = false;                // FLEP_KFLAG_HOST_RELAY: one request-relay CTA (R28)
+  bool warp = false;                 // FLEP_KFLAG_WARP_TASKS: warp workers, counts in tasks (R30)
+  uint32_t tasks_per_block = 1;
+  uint32_t ctas = 0;                 // worker CTAs per epoch (= workers, or workers / warps per CTA)
   uint32_t slice_blocks = 0;
   uint64_t next_block = 0, slice_done = 0;
   std::deque<std::pair<cudaEvent_t, uint32_t>> inflight;
@@ -209,11 +212,12 @@ struct ApiLock {
   }
 };
 
-flep_status occupancy(flep_rt rt, const BodyOps* ops, bool cov, int* k, bool sw = false) {
-  auto key = std::make_pair(ops->body * 2 + (sw ? 1 : 0), cov);
+flep_status occupancy(flep_rt rt, const BodyOps* ops, bool cov, int* k, bool sw = false, bool warp = false) {
+  auto key = std::make_pair(ops->body * 4 + (sw ? 1 : 0) + (warp ? 2 : 0), cov);
   auto it = rt->occ_cache.find(key);
   if (it != rt->occ_cache.end()) { *k = it->second; return FLEP_OK; }
   if (sw) CUDA_TRY(ops->occupancy_sw(k, cov));
+  else if (warp) CUDA_TRY(ops->occupancy_warp(k, cov));
   else CUDA_TRY(ops->occupancy(k, cov));
   if (*k <= 0) return fail(FLEP_ERR_UNSUPPORTED, "body %d cannot be resident", ops->body);
   rt->occ_cache[key] = *k;
@@ -425,7 +429,7 @@ flep_status start_epoch(flep_rt rt, Launch& L) {
   p.prefetch = ((L.flags & FLEP_KFLAG_PREFETCH) && !(L.flags & FLEP_KFLAG_IN_TILE)) ? 1u : 0u;
   p.gen_first = L.gen0 + 1;
   p.started_hint = (L.flags & FLEP_KFLAG_STARTED_HINT) ? 1u : 0u;
-  p.relay_block = L.relay ? L.workers : 0xffffffffu;
+  p.relay_block = L.relay ? L.ctas : 0xffffffffu;
   p.async_poll = ((L.flags & FLEP_KFLAG_ASYNC_POLL) && rt->opt.flag != FLEP_FLAG_HOST_MAPPED) ? 1u : 0u;
   p.ctrl_sys = rt->opt.flag == FLEP_FLAG_HOST_MAPPED ? 1u : 0u;
   p.partial = L.partial;
@@ -436,6 +440,7 @@ flep_status start_epoch(flep_rt rt, Launch& L) {
   L.trig_n = 0;
   cudaError_t e = L.clc ? L.ops->clc(L.args.data(), p, (L.n_blocks + L.chunk - 1) / L.chunk, L.exec, L.cov != nullptr)
                  : L.sw ? L.ops->worker_sw(L.args.data(), p, L.workers, L.exec, L.cov != nullptr)
+                 : L.warp ? L.ops->warp_worker(L.args.data(), p, L.ctas + (L.relay ? 1u : 0u), L.exec, L.cov != nullptr)
                         : L.ops->worker(L.args.data(), p, L.workers + (L.relay ? 1u : 0u), L.exec, L.cov != nullptr);
   if (e != cudaSuccess) return fail(FLEP_ERR_CUDA, "worker launch failed: %s", cudaGetErrorString(e));
   CUDA_TRY(cudaEventRecord(L.fin_ev, L.exec));
@@ -875,8 +880,16 @@ flep_status flep_launch(flep_rt rt, flep_kernel kid, flep_dim3 grid, const void*
   const bool cov = (rt->opt.debug_coverage & 1u) != 0;
   const bool sw = (kr.flags & FLEP_KFLAG_SCHED_WARP) && !(kr.flags & FLEP_KFLAG_CLC);
   if (sw && !ops->worker_sw) return fail(FLEP_ERR_UNSUPPORTED, "body %d has no scheduling-warp worker", kr.body);
+  // R30: warp tasks (not under SLICE, whose sub-kernels are the unwrapped original grid)
+  const bool warp = (kr.flags & FLEP_KFLAG_WARP_TASKS) && rt->opt.policy != FLEP_POLICY_SLICE;
+  if (warp && (!ops->warp_worker || !ops->warp_tasks))
+    return fail(FLEP_ERR_UNSUPPORTED, "body %d has no warp-task worker", kr.body);
+  if (warp && (sw || (kr.flags & (FLEP_KFLAG_CLC | FLEP_KFLAG_IN_TILE))))
+    return fail(FLEP_ERR_UNSUPPORTED, "warp tasks do not combine with CLC, the scheduling warp or in-tile preemption");
+  const uint32_t tpb = warp ? ops->warp_tasks : 1u;
+  if (N * tpb >= (1ull << 31)) return fail(FLEP_ERR_INVALID, "grid too large for warp tasks");
   int k = 0;
-  s = occupancy(rt, ops, cov, &k, sw);
+  s = occupancy(rt, ops, cov, &k, sw, warp);
   if (s) return s;
   if (rt->free_slots.empty()) return fail(FLEP_ERR_NOMEM, "out of status slots");
 
@@ -888,7 +901,9 @@ flep_status flep_launch(flep_rt rt, flep_kernel kid, flep_dim3 grid, const void*
   L.ops = ops;
   L.args.assign((const uint8_t*)args, (const uint8_t*)args + args_size);
   L.grid = g;
-  L.n_blocks = (uint32_t)N;
+  L.warp = warp;
+  L.tasks_per_block = tpb;
+  L.n_blocks = (uint32_t)(N * tpb);          // the runtime's unit: tasks (= blocks unless R30)
   L.prio = priority;
   L.user = (cudaStream_t)stream;
   L.chunk = kr.chunk;
@@ -902,15 +917,24 @@ flep_status flep_launch(flep_rt rt, flep_kernel kid, flep_dim3 grid, const void*
   }
   if (kr.ctas_per_sm && (int)kr.ctas_per_sm < k) k = (int)kr.ctas_per_sm;
   const uint64_t wmax = (uint64_t)k * rt->num_sms;
-  const uint64_t need = (N + L.chunk - 1) / L.chunk;
+  const uint64_t need = ((uint64_t)L.n_blocks + L.chunk - 1) / L.chunk;
   // R28: the relay CTA takes one resident slot (plain counter worker, stream-memop transport)
   L.relay = (kr.flags & FLEP_KFLAG_HOST_RELAY) && !L.sw && !L.clc && !ops->validate &&
             rt->opt.flag != FLEP_FLAG_HOST_MAPPED && wmax > 1;
-  L.workers = (uint32_t)std::min<uint64_t>(std::min<uint64_t>(wmax - (L.relay ? 1 : 0), need), rt->max_workers);
+  if (warp) {
+    // R30: worker CTAs of threads/32 warp workers each
+    const uint64_t wpc = (uint64_t)ops->threads / 32u;
+    const uint64_t g_need = (need + wpc - 1) / wpc;
+    L.ctas = (uint32_t)std::min<uint64_t>(std::min<uint64_t>(wmax - (L.relay ? 1 : 0), g_need), rt->max_workers / wpc);
+    L.workers = (uint32_t)(L.ctas * wpc);
+  } else {
+    L.workers = (uint32_t)std::min<uint64_t>(std::min<uint64_t>(wmax - (L.relay ? 1 : 0), need), rt->max_workers);
+    L.ctas = L.workers;
+  }
   {
     // SMs that host every CTA of this launch (A9: n = ceil(grid / k)): the workers
     // (+ the relay CTA), or the CLC grid's resident part
-    const uint64_t ctas = L.clc ? std::min<uint64_t>(need, wmax) : (uint64_t)L.workers + (L.relay ? 1u : 0u);
+    const uint64_t ctas = L.clc ? std::min<uint64_t>(need, wmax) : (uint64_t)L.ctas + (L.relay ? 1u : 0u);
     L.sms_need = (int64_t)std::min<uint64_t>(rt->num_sms, (ctas + (uint64_t)k - 1) / (uint64_t)k);
   }
   if (rt->opt.policy == FLEP_POLICY_SLICE) {
@@ -921,7 +945,8 @@ flep_status flep_launch(flep_rt rt, flep_kernel kid, flep_dim3 grid, const void*
   L.t_arrive = now_ns();
   L.t_e = flep_model_predict_ns(kr.model, (double)N, (double)ops->threads, (double)N, 0.0);
   L.overhead = kr.overhead;
-  L.trig_block = rt->arm_block;
+  // the debug trigger names an original block: its first task (R30)
+  L.trig_block = rt->arm_block == kNoTrigger ? kNoTrigger : rt->arm_block * tpb;
   L.trig_n = rt->arm_n;
   rt->arm_block = kNoTrigger;
   rt->arm_n = 0;
@@ -1098,6 +1123,7 @@ flep_status flep_query(flep_rt rt, flep_launch_t h, flep_launch_info* out) {
     const uint32_t g = __atomic_load_n(&L->hs->started, __ATOMIC_ACQUIRE);
     out->started_epoch = (g > L->gen0) ? g - L->gen0 : 0;
   }
+  out->tasks_per_block = L->tasks_per_block;
   if (rt->policy) {
     const Policy::Entry* e = rt->policy->entry(L->id);
     if (e) { out->t_w = e->t_w; out->t_r = e->t_r; }
@@ -1230,7 +1256,7 @@ flep_status flep_debug_trigger_at(flep_rt rt, flep_launch_t h, uint64_t block_in
   refresh(rt, *L);
   if (L->state != FLEP_STATE_PREEMPTED && L->state != FLEP_STATE_QUEUED)
     return fail(FLEP_ERR_STATE, "trigger can only be set for the next epoch of a launch that is not running");
-  L->trig_block = block_index >= 0xffffffffull ? kNoTrigger : (uint32_t)block_index;
+  L->trig_block = block_index >= 0xffffffffull ? kNoTrigger : (uint32_t)(block_index * L->tasks_per_block);
   L->trig_n = std::min<uint32_t>(n_sms, kCtrlAll);
   return FLEP_OK;
 }
@@ -1306,6 +1332,9 @@ flep_status flep_debug_epoch_info(flep_rt rt, flep_launch_t h, uint32_t epoch, f
   out->done = cb.ep_done[e];
   out->counter = cb.ep_ctr[e];
   out->state = cb.ep_state[e];
+  out->relay_smid = L->relay ? cb.ep_relay[e] >> 8 : 0;
+  out->relay_reason = L->relay ? cb.ep_relay[e] & 0xffu : 0;
+  out->relay_t_exit = L->relay ? cb.ep_relay_t[e] : 0;
   return FLEP_OK;
 }
 

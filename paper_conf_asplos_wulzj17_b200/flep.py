@@ -10,16 +10,18 @@ import ctypes as C
 import os
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "libflep.so")
+LIB_PATH = os.environ.get("FLEP_LIB_PATH") or os.path.join(HERE, "libflep.so")   # override: A/B builds
 
 OK, ERR_INVALID, ERR_STATE, ERR_CUDA, ERR_NOMEM, ERR_TIMEOUT, ERR_UNSUPPORTED = 0, -1, -2, -3, -4, -5, -6
 POLICY_MANUAL, POLICY_FIFO, POLICY_HPF, POLICY_SLICE, POLICY_FFS, POLICY_REORDER = 0, 1, 2, 3, 4, 5
 FLAG_STREAM_MEMOP, FLAG_HOST_MAPPED = 0, 1
 BODY_SAXPY_I32, BODY_SAXPY_F32, BODY_SPMV_CSR_F32, BODY_STENCIL5_F32, BODY_STENCIL5_I32, BODY_GEMM_BF16 = 1, 2, 3, 4, 5, 6
 BODY_STENCIL5_F32_TMA = 7
+BODY_SPMV_CSR_F32_VEC = 8
 STATE_QUEUED, STATE_RUNNING, STATE_YIELDING, STATE_PREEMPTED, STATE_PARTIAL, STATE_DONE = 0, 1, 2, 3, 4, 5
 STATE_NAMES = {0: "QUEUED", 1: "RUNNING", 2: "YIELDING", 3: "PREEMPTED", 4: "PARTIAL", 5: "DONE"}
 REASON_YIELD, REASON_EXHAUSTED = 1, 2
+RELAY_LEFT_OWN_SM, RELAY_LEFT_TEMPORAL, RELAY_LEFT_PUBLISHED = 1, 2, 3
 ACTION_NAMES = {0: "LAUNCH", 1: "RESUME", 2: "PREEMPT", 3: "REFILL"}
 NO_TRIGGER = 0xFFFFFFFF
 KFLAG_PREFETCH = 1
@@ -29,6 +31,8 @@ KFLAG_ASYNC_POLL = 8
 KFLAG_CLC = 16
 KFLAG_SCHED_WARP = 32
 KFLAG_HOST_RELAY = 64
+KFLAG_WARP_TASKS = 128
+WARP_TASKS_PER_BLOCK = 8
 
 
 class Dim3(C.Structure):
@@ -76,7 +80,7 @@ class LaunchInfo(C.Structure):
                 ("t_w", C.c_int64), ("t_r", C.c_int64), ("t_arrive", C.c_int64),
                 ("t_first_start", C.c_int64), ("t_finish", C.c_int64), ("workers", C.c_uint32),
                 ("n_yield", C.c_uint32), ("t_last_request", C.c_int64), ("t_last_drain", C.c_int64),
-                ("started_epoch", C.c_uint32), ("reserved", C.c_uint32)]
+                ("started_epoch", C.c_uint32), ("tasks_per_block", C.c_uint32)]
 
 
 class WorkerEvent(C.Structure):
@@ -86,12 +90,13 @@ class WorkerEvent(C.Structure):
 
 class EpochInfo(C.Structure):
     _fields_ = [("t_trigger", C.c_uint64), ("t_end", C.c_uint64), ("trigger_block", C.c_uint32),
-                ("done", C.c_uint32), ("counter", C.c_uint32), ("state", C.c_uint32)]
+                ("done", C.c_uint32), ("counter", C.c_uint32), ("state", C.c_uint32),
+                ("relay_smid", C.c_uint32), ("relay_reason", C.c_uint32), ("relay_t_exit", C.c_uint64)]
 
 
 ARGS_FOR_BODY = {BODY_SAXPY_I32: SaxpyI32Args, BODY_SAXPY_F32: SaxpyF32Args, BODY_SPMV_CSR_F32: SpmvArgs,
                  BODY_STENCIL5_F32: StencilArgs, BODY_STENCIL5_I32: StencilArgs, BODY_GEMM_BF16: GemmArgs,
-                 BODY_STENCIL5_F32_TMA: StencilArgs}
+                 BODY_STENCIL5_F32_TMA: StencilArgs, BODY_SPMV_CSR_F32_VEC: SpmvArgs}
 
 # exported symbols: name -> (restype, argtypes)
 _P = C.c_void_p
@@ -215,11 +220,11 @@ class Runtime:
 
     def register_kernel(self, body, chunk=0, poll=0, name="", model=(0, 0, 0, 0, 1), overhead_ns=0,
                         prefetch=False, ctas_per_sm=0, started_hint=False, in_tile=False, async_poll=False,
-                        clc=False, sched_warp=False, host_relay=False):
+                        clc=False, sched_warp=False, host_relay=False, warp_tasks=False):
         flags = ((KFLAG_PREFETCH if prefetch else 0) | (KFLAG_STARTED_HINT if started_hint else 0)
                  | (KFLAG_IN_TILE if in_tile else 0) | (KFLAG_ASYNC_POLL if async_poll else 0)
                  | (KFLAG_CLC if clc else 0) | (KFLAG_SCHED_WARP if sched_warp else 0)
-                 | (KFLAG_HOST_RELAY if host_relay else 0))
+                 | (KFLAG_HOST_RELAY if host_relay else 0) | (KFLAG_WARP_TASKS if warp_tasks else 0))
         d = KernelDesc(name.encode(), body, chunk, poll, (C.c_double * 5)(*model), overhead_ns,
                        flags, ctas_per_sm)
         k = C.c_int32()

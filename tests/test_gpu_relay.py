@@ -80,3 +80,39 @@ def test_relay_host_request_preempts_and_resumes(rt):
     got = y.cpu().numpy().astype(np.float64)
     d = np.maximum(np.abs(ref), absum)
     assert float(np.max(np.abs(got - ref) / np.where(d > 0, d, 1.0))) <= 1e-5
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_relay_leaves_a_released_sm(rt, seed):
+    """I3 for every CTA of the grid: a host spatial request of n SMs makes the relay
+    CTA leave if its own SM is among the released ones (rank = smid < n), before the epoch ends;
+    otherwise it stays until the epoch is published. Workers yield only on the released SMs."""
+    f = flep_mod()
+    import torch
+    rows = 1 << 22
+    rp, col, val, xv = gen.csr_inputs(rows, seed=74)
+    y = torch.zeros(rows, device="cuda")
+    k = rt.register_kernel(f.BODY_SPMV_CSR_F32, chunk=1, poll=1, host_relay=True, started_hint=True)
+    g = gen.rng(4000 + seed)
+    n = int(g.integers(1, rt.num_sms))
+    h = rt.launch(k, f.spmv_grid(rows), f.spmv_args(y, t(rp), t(col), t(val), t(xv)))
+    t0 = time.perf_counter()
+    while rt.query(h).started_epoch < 1 and time.perf_counter() - t0 < 1:
+        pass
+    try:
+        rt.preempt(h, n)
+    except f.FlepError:
+        pytest.skip("the launch completed before the request")
+    rt.sync(h, timeout_ns=10_000_000_000)           # spatial: the rest of the workers finish it
+    ep = rt.epoch_info(h, 1)
+    assert ep.relay_reason in (f.RELAY_LEFT_OWN_SM, f.RELAY_LEFT_PUBLISHED)
+    if ep.relay_smid < n:
+        assert ep.relay_reason == f.RELAY_LEFT_OWN_SM
+        assert ep.relay_t_exit <= ep.t_end
+    else:
+        assert ep.relay_reason == f.RELAY_LEFT_PUBLISHED
+    for e in rt.events(h, 1):
+        if e.reason == f.REASON_YIELD:
+            assert e.smid < n
+    nb = f.spmv_grid(rows)[0]
+    assert np.all(rt.coverage_np(h, nb) == 1)

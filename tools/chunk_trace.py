@@ -34,8 +34,10 @@ def main():
     out = torch.empty_like(st)
     rp, col, val, x = gen.csr_inputs(1 << 20, seed=2)
     y = torch.zeros(1 << 20, device="cuda")
+    dev = [T(rp), T(col), T(val), T(x)]         # kept alive: the args structs hold raw pointers
     cases = [("stencil", F.BODY_STENCIL5_F32, F.stencil_grid(4096), F.stencil_args(out, st)),
-             ("spmv", F.BODY_SPMV_CSR_F32, F.spmv_grid(1 << 20), F.spmv_args(y, T(rp), T(col), T(val), T(x)))]
+             ("spmv", F.BODY_SPMV_CSR_F32, F.spmv_grid(1 << 20), F.spmv_args(y, *dev)),
+             ("spmvvec", F.BODY_SPMV_CSR_F32_VEC, F.spmv_grid(1 << 20), F.spmv_args(y, *dev))]
     only = os.environ.get("TRACE_BODIES")
     if only:
         cases = [c for c in cases if c[0] in only.split(",")]

@@ -23,6 +23,7 @@ def main():
     ap.add_argument("--prefetch", default="0,1")
     ap.add_argument("--in-tile", default="0", help="GEMM: in-tile preemption variants (0,1)")
     ap.add_argument("--async-poll", default="0", help="async poll variants (0,1)")
+    ap.add_argument("--warp", default="0", help="warp-task worker variants (0,1; R30)")
     ap.add_argument("--gate-us", type=float, default=0.0,
                     help="spin the stream this long before the start event (hides host submission latency)")
     a = ap.parse_args()
@@ -40,7 +41,12 @@ def main():
         y = torch.zeros(1 << 20, device="cuda")
         jobs["spmv"] = (F.BODY_SPMV_CSR_F32, F.spmv_grid(1 << 20), F.spmv_args(y, T(rp), T(col), T(val), T(x)),
                         8 * int(rp[-1]) + 12 * (1 << 20), (rp, col, val, x, y))
-    if "stencil" in a.bodies:
+    if "spmvvec" in a.bodies:
+        rp, col, val, x = gen.csr_inputs(1 << 20, seed=2)
+        y = torch.zeros(1 << 20, device="cuda")
+        jobs["spmvvec"] = (F.BODY_SPMV_CSR_F32_VEC, F.spmv_grid(1 << 20), F.spmv_args(y, T(rp), T(col), T(val), T(x)),
+                           8 * int(rp[-1]) + 12 * (1 << 20), (rp, col, val, x, y))
+    if "stencil" in a.bodies.split(","):
         st = T(gen.stencil_f32_input(4096, seed=3))
         out = torch.empty_like(st)
         jobs["stencil"] = (F.BODY_STENCIL5_F32, F.stencil_grid(4096), F.stencil_args(out, st), 8 * 4096 * 4096, (st, out))
@@ -100,13 +106,16 @@ def main():
                     for cps in map(int, a.cps.split(",")):
                       for it_ in (map(int, a.in_tile.split(",")) if name == "gemm" else [0]):
                        for ap_ in map(int, a.async_poll.split(",")):
-                        if it_ and pf:
+                        for wp in map(int, a.warp.split(",")):
+                         if it_ and pf:
                             continue
-                        k = rt.register_kernel(body, chunk=C, poll=K, prefetch=bool(pf), ctas_per_sm=cps,
-                                               in_tile=bool(it_), async_poll=bool(ap_))
-                        tw = timed(lambda: rt.launch(k, grid, args, stream=s))
-                        print(json.dumps({"body": name, "C": C, "K": K, "prefetch": pf, "cps": cps, "in_tile": it_,
-                                          "async_poll": ap_,
+                         if wp and body not in (F.BODY_SPMV_CSR_F32_VEC, F.BODY_STENCIL5_F32):
+                            continue
+                         k = rt.register_kernel(body, chunk=C, poll=K, prefetch=bool(pf), ctas_per_sm=cps,
+                                               in_tile=bool(it_), async_poll=bool(ap_), warp_tasks=bool(wp))
+                         tw = timed(lambda: rt.launch(k, grid, args, stream=s))
+                         print(json.dumps({"body": name, "C": C, "K": K, "prefetch": pf, "cps": cps, "in_tile": it_,
+                                          "async_poll": ap_, "warp": wp,
                                           "us": round(tw, 3),
                                           ("tflops" if name == "gemm" else "gbs"): round(nbytes / tw / (1e6 if name == "gemm" else 1e3), 1),
                                           "overhead_pct": round((tw / tu - 1) * 100, 2)}), flush=True)
