@@ -655,8 +655,9 @@ def sub_records(args, rank, world, local):
     """The other BASELINE configs as sub-records of the default line (each with its own clocks):
     configs[0] (SAXPY-int co-run, exactness), configs[2] (spatial yield per width: the manual
     device-triggered sweep and the managed spatial-HPF decision path, victim checked against a
-    NumPy reference), configs[3] (64-kernel same-priority queue: ANTT/STP, decision logs) and
-    configs[4] (one 512-kernel job queue over the N GPUs of this run)."""
+    NumPy reference), configs[3] (64-kernel same-priority queue: ANTT/STP, decision logs),
+    configs[4] (one 512-kernel job queue over the N GPUs of this run) and E13 (never-preempted
+    overhead of FLEP vs kernel slicing)."""
     import copy
     import bench_configs as BCF
     a = copy.copy(args)
@@ -665,7 +666,7 @@ def sub_records(args, rank, world, local):
     out, timing = {}, {}
     for name, fn in (("configs[0]", BCF.run_corun1), ("configs[2]", BCF.run_spatial),
                      ("configs[2]_managed", BCF.run_spatial_managed), ("configs[3]", BCF.run_queue),
-                     ("configs[4]", BCF.run_scale_queue)):
+                     ("configs[4]", BCF.run_scale_queue), ("E13_never_preempted", BCF.run_slicing_overhead)):
         if name in args.skip_sub:
             continue
         t0 = time.perf_counter()
@@ -688,7 +689,7 @@ def main():
     ap.add_argument("--impl", default="flep", choices=["flep", "reference"])
     ap.add_argument("--config", default="temporal", choices=["temporal", "corun1", "spatial", "spatial_managed", "queue",
                                                              "scale", "ffs", "model", "gemm", "tune", "clc", "delay",
-                                                             "spatial_f1"])
+                                                             "spatial_f1", "slicing"])
     ap.add_argument("--dry-run", action="store_true",
                     help="configs[4] launcher and control flow without CUDA (CPU, gloo); one JSON line")
     ap.add_argument("--sub", type=int, default=1, help="default run: add the configs[0,2,3,4] sub-records")
@@ -745,7 +746,7 @@ def main():
               "tune": bench_configs.run_tune, "ffs": bench_configs.run_ffs, "model": bench_configs.run_model,
               "clc": bench_configs.run_clc, "delay": bench_configs.run_delay,
               "spatial_f1": bench_configs.run_spatial_f1, "queue": bench_configs.run_queue,
-              "scale": bench_configs.run_scale_queue}[args.config]
+              "scale": bench_configs.run_scale_queue, "slicing": bench_configs.run_slicing_overhead}[args.config]
         fn(args, rank, world, local)
 
 

@@ -876,7 +876,7 @@ def run_queue(args, rank, world, local):
     # untimed warm-up of a short prefix (first-use costs of a fresh runtime, stream and event pools)
     _run_trace(F, torch, local, F.POLICY_FIFO, mine[:8], inst, t_alone, overhead_ns, streams)
     for name, pol in (("FIFO", F.POLICY_FIFO), ("HPF", F.POLICY_HPF), ("SLICE", F.POLICY_SLICE),
-                      ("REORDER", F.POLICY_REORDER)):
+                      ("SLICE_DEVICE", F.POLICY_SLICE_DEVICE), ("REORDER", F.POLICY_REORDER)):
         turn, dec, evl = _run_trace(F, torch, local, pol, mine, inst, t_alone, overhead_ns, streams)
         tt = [t[0] for t in turn]
         al = [t_alone[t[1]] for t in turn]
@@ -894,6 +894,7 @@ def run_queue(args, rank, world, local):
             json.dump({"workload": "configs[3] queue, seed 5", "logs": logs}, fh)
     gain_fifo = res["FIFO"]["antt"] / res["HPF"]["antt"]
     gain_slice = res["SLICE"]["antt"] / res["HPF"]["antt"]
+    gain_slice_dev = res["SLICE_DEVICE"]["antt"] / res["HPF"]["antt"]
     out = {"metric": METRIC, "value": round(gain_fifo, 3), "unit": "x (ANTT_FIFO / ANTT_FLEP)",
            "value_definition": "co-run NATT gain of FLEP-HPF over the FIFO (MPS-like) baseline on the same trace",
            "n_gpus": world, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
@@ -906,6 +907,9 @@ def run_queue(args, rank, world, local):
            "stp": {k: round(v["stp"], 3) for k, v in res.items()},
            "preemptions": {k: v["preemptions"] for k, v in res.items()},
            "natt_gain_vs_fifo": round(gain_fifo, 3), "natt_gain_vs_slicing": round(gain_slice, 3),
+           "natt_gain_vs_slicing_device": round(gain_slice_dev, 3),
+           "slicing_note": "SLICE = host-issued slices, at most two in flight (R19); SLICE_DEVICE = every slice "
+                           "enqueued at launch with the device check at slice entry (R31)",
            "reordering_gain_vs_fifo": round(res["FIFO"]["antt"] / res["REORDER"]["antt"], 3),
            "stp_degradation_vs_fifo": round(1 - res["HPF"]["stp"] / res["FIFO"]["stp"], 4),
            "replay_parity": "checked on CPU: tests/test_policy_replay.py replays the committed logs (tests/golden/queue_logs_r01.json) through the oracle DES",
@@ -1419,6 +1423,89 @@ def run_spatial_managed(args, rank, world, local):
            "I3_violations": sum(r["I3_violations"] for r in rows),
            "victim_parity_ok": all(r["victim_parity_ok"] for r in rows),
            "clocks": clk.summary()}
+    _emit(out, rank, args)
+    barrier(world)
+    return out
+
+
+# ------------------------------------------------------------------------------------------
+def run_slicing_overhead(args, rank, world, local):
+    """E13 (Fig. 17): overhead of the preemption mechanisms when NOTHING preempts,
+    per kernel, against the unwrapped grid: FLEP's persistent workers (the queue's tuned C and the
+    latency setting C = 1), kernel slicing with every slice enqueued and the device check at slice
+    entry (R31; slice = one wave W*C*K, A20), and plain back-to-back slices without any check (the
+    lower bound of slicing: launch gaps only). CUDA events on the launching stream, dithered, L2
+    flushed, interleaved; trimmed mean of `reps` samples."""
+    import torch
+    from bench import ClockSampler, L2Flush, barrier, physical_gpu_index
+    from paper_conf_asplos_wulzj17_b200 import flep as F
+    from paper_conf_asplos_wulzj17_b200.calibrate import dither, event_mean_us
+    torch.cuda.set_device(local)
+    inst = _queue_instances(torch, F, seed=5)
+    flush = L2Flush(torch)
+    S = torch.cuda.Stream()
+    rt_m = F.Runtime(device=local, exec_on_user_stream=True)
+    rt_s = F.Runtime(device=local, policy=F.POLICY_SLICE_DEVICE, exec_on_user_stream=True)
+    rows = []
+    reps = max(8, args.reps // 4)
+    with ClockSampler(physical_gpu_index(local)) as clk:
+        for key in sorted(inst):
+            body, grid, a, keep, _ = inst[key]
+            C, pf = QUEUE_CHUNK[key[0]]
+            k_t = rt_m.register_kernel(body, chunk=C, poll=1, prefetch=pf, in_tile=body == F.BODY_GEMM_BF16)
+            k_1 = rt_m.register_kernel(body, chunk=1, poll=1, in_tile=body == F.BODY_GEMM_BF16)
+            k_s = rt_s.register_kernel(body, chunk=C, poll=1)
+            cps, w = rt_m.workers_for(body)
+            slice_blocks = w * C                                     # one wave of W*C*K blocks (A20)
+            t = {m: [] for m in ("unwrapped", "flep_tuned", "flep_c1", "slice_device", "slice_plain")}
+            for r in range(reps + 2):
+                for m in t:
+                    with torch.cuda.stream(S):
+                        flush.zero_()
+                        dither(torch)
+                        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                        e0.record(S)
+                    h = None
+                    if m == "unwrapped":
+                        rt_m.launch_unwrapped(body, grid, a, stream=S)
+                    elif m == "flep_tuned":
+                        h = (rt_m, rt_m.launch(k_t, grid, a, stream=S))
+                    elif m == "flep_c1":
+                        h = (rt_m, rt_m.launch(k_1, grid, a, stream=S))
+                    elif m == "slice_device":
+                        h = (rt_s, rt_s.launch(k_s, grid, a, stream=S))
+                    else:
+                        rt_m.launch_sliced(body, grid, a, slice_blocks, stream=S)
+                    e1.record(S)
+                    e1.synchronize()
+                    if h is not None:
+                        h[0].sync(h[1])
+                    if r >= 2:
+                        t[m].append(e0.elapsed_time(e1) * 1e3)
+            u = event_mean_us(t["unwrapped"])
+            nb = grid[0] * grid[1]
+            row = {"kernel": f"{key[0]}-{key[1]}", "blocks": nb, "slice_blocks": slice_blocks,
+                   "slices": -(-nb // slice_blocks), "unwrapped_us": round(u, 2)}
+            for m in ("flep_tuned", "flep_c1", "slice_device", "slice_plain"):
+                v = event_mean_us(t[m])
+                row[m + "_us"] = round(v, 2)
+                row[m + "_overhead_pct"] = round((v / u - 1) * 100, 2)
+            row["tuned_chunk"] = C
+            rows.append(row)
+    rt_m.close()
+    rt_s.close()
+    big = [r for r in rows if r["kernel"].endswith("-2")]
+    mean = lambda k, rs: round(float(np.mean([r[k] for r in rs])), 2)  # noqa: E731
+    out = {"metric": METRIC, "value": mean("flep_tuned_overhead_pct", rows), "unit": "% over the unwrapped grid",
+           "value_definition": "mean never-preempted overhead of FLEP (tuned C) over the 12 queue kernels (E13, Fig. 17)",
+           "n_gpus": world, "higher_is_better": False, "scaling": "weak", "vs_baseline": None,
+           "dtype": "mixed", "data": "synthetic (seeded)",
+           "config": {"workload": "E13: the configs[3] queue's 12 kernel instances run alone, never preempted",
+                      "reps": reps, "l2": "flushed between samples"},
+           "mean_overhead_pct": {k: mean(k + "_overhead_pct", rows) for k in ("flep_tuned", "flep_c1", "slice_device", "slice_plain")},
+           "mean_overhead_pct_large": {k: mean(k + "_overhead_pct", big) for k in ("flep_tuned", "flep_c1", "slice_device", "slice_plain")},
+           "paper": "FLEP 2.5 % vs kernel slicing 8 % at the same preemption granularity (P:391, K40)",
+           "kernels": rows, "clocks": clk.summary()}
     _emit(out, rank, args)
     barrier(world)
     return out

@@ -67,8 +67,13 @@ typedef enum {
   FLEP_POLICY_FFS = 4,     /* fairness first under an overhead constraint: weighted round robin,
                               epoch T*W_i, W_i = priority+1, T minimal with
                               sum O_i / (T sum W_i) <= max_overhead (§5.2.2) */
-  FLEP_POLICY_REORDER = 5  /* kernel-reordering baseline without preemption: shortest queued kernel
+  FLEP_POLICY_REORDER = 5, /* kernel-reordering baseline without preemption: shortest queued kernel
                               of the highest priority runs next */
+  FLEP_POLICY_SLICE_DEVICE = 6 /* HPF decisions on kernel slicing with every slice enqueued at
+                              launch and a device-side check at slice entry (the first CTA of a
+                              slice decides for all of it: run, or skip when a request is in
+                              force), so a never-preempted kernel pays only the launch gaps
+                              between its slices (R31; P:96, P:391 baseline) */
 } flep_policy;
 
 typedef enum {
@@ -123,10 +128,13 @@ typedef struct {
                                   is refilled to every SM when it finishes (R29);
                                   0 = always temporal (Fig. 6 as printed) */
   uint32_t slice_blocks;       /* SLICE policy: blocks per sub-kernel (0 -> W*C*K, A20) */
-  uint32_t exec_on_user_stream;/* MANUAL mode: launch worker grids (and resumes) directly on the
+  uint32_t exec_on_user_stream;/* launch worker grids (and resumes, slices) directly on the
                                   caller's stream instead of a runtime stream. Stream order then
-                                  only covers the epoch grids: the caller must resume before
-                                  enqueuing work that depends on the results. */
+                                  only covers the epoch grids: the caller must resume (manual) or
+                                  sync (managed) before enqueuing work that depends on the
+                                  results. In managed modes this is a measurement aid (CUDA events
+                                  on the caller's stream bracket a launch the policy starts at
+                                  once). */
   uint32_t max_overhead_ppm;   /* FFS: max_overhead in parts per million (0 -> 100000 = 10%) */
 } flep_options;
 
@@ -333,7 +341,7 @@ flep_status flep_event_log_ex(flep_rt rt, int64_t* out7, size_t max_records, siz
 /* ---- pure policy engine (host only; no GPU needed) -------------------------------------
    The exact decision logic the managed runtime uses (Fig. 6), exposed for replay parity with
    the oracle's discrete-event simulation. kind: 1 FIFO, 2 HPF, 3 SLICE (= HPF decisions), 4 FFS,
-   5 REORDER. */
+   5 REORDER, 6 SLICE_DEVICE (= HPF decisions). */
 typedef struct flep_policy_s* flep_policy_t;
 flep_status flep_policy_create(int32_t kind, uint32_t num_sms, flep_policy_t* out);
 flep_status flep_policy_destroy(flep_policy_t p);

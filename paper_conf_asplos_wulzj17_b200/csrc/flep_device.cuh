@@ -735,6 +735,52 @@ flep_unwrapped(const __grid_constant__ typename Body::Args args, uint32_t gx, ui
 #endif
 }
 
+// Kernel slicing with a device-side check (FLEP_POLICY_SLICE_DEVICE, the baseline of P:96 and
+// P:391, reading R31): the original kernel as sub-grids of consecutive blocks, ALL enqueued on the
+// stream at launch. Every CTA of slice j follows one decision for the whole slice, taken by the
+// first of its CTAs that gets there: run, or skip if a preemption request for this launch is in
+// force (a slice is never split). A decision word holds the deciding epoch's tag; a RUN decided
+// in an earlier epoch means the slice is done, so a resume may re-enqueue slices from any lower
+// bound of the progress (the words are zeroed at the launch's first epoch).
+struct SliceParams {
+  const uint32_t* ctrl;    // the launch's control word (device copy)
+  uint32_t* decision;      // [slices]: tag << 2 | 1 (run) or 2 (skip)
+  uint32_t slice;          // j
+  uint32_t gen;            // epoch generation (ctrl tag)
+};
+constexpr uint32_t kSliceRun = 1, kSliceSkip = 2;
+__host__ __device__ __forceinline__ uint32_t slice_tag(uint32_t gen) { return gen & 0x3fffffffu; }
+
+template <class Body>
+__global__ void __launch_bounds__(Body::kThreads, Body::kMinBlocks)
+flep_slice(const __grid_constant__ typename Body::Args args, uint32_t gx, uint32_t gy, uint32_t block_offset,
+           const SliceParams sp) {
+  __shared__ uint32_t s_go;
+  if (threadIdx.x == 0) {
+    uint32_t* dp = sp.decision + sp.slice;
+    uint32_t d = ld_relaxed_gpu(dp);
+    bool go;
+    if ((d >> 2) == slice_tag(sp.gen)) {
+      go = (d & 3u) == kSliceRun;                 // decided in this epoch by another CTA
+    } else if ((d & 3u) == kSliceRun) {
+      go = false;                                 // ran in an earlier epoch
+    } else {
+      const uint32_t c = ld_relaxed_gpu(sp.ctrl);
+      const bool stop = ctrl_gen(c) == (sp.gen & kCtrlGenMask) && ctrl_n(c) > 0;   // slicing is temporal
+      const uint32_t want = (slice_tag(sp.gen) << 2) | (stop ? kSliceSkip : kSliceRun);
+      const uint32_t old = atomicCAS(dp, d, want);
+      go = ((old == d) ? want : old) == ((slice_tag(sp.gen) << 2) | kSliceRun);   // first CTA decides
+    }
+    s_go = go ? 1u : 0u;
+  }
+  __syncthreads();
+  if (!s_go) return;
+  const uint32_t b = block_offset + blockIdx.x + gx * (blockIdx.y + gy * blockIdx.z);
+  Body::setup(args);
+  Body::run(args, b, b + 1, gx, gy);
+  Body::teardown(args);
+}
+
 // Bodies without per-worker resources, run through the generic per-chunk loop.
 struct NoResources {
   static constexpr bool kPersistent = false;

@@ -74,4 +74,11 @@ cudaError_t gemm_unwrapped_launch(const void* user, dim3 grid, uint32_t offset, 
 
 cudaError_t gemm_occupancy(int* k, bool cov) { return occupancy_raw<GemmBody>(k, cov); }
 
+cudaError_t gemm_slice_launch(const void* user, dim3 grid, uint32_t offset, uint32_t count,
+                               const SliceParams& sp, cudaStream_t s) {
+  GemmArgsDev d;
+  if (!to_dev(user, &d)) return cudaErrorInvalidValue;
+  return launch_slice_raw<GemmBody>(d, grid, offset, count, sp, s);
+}
+
 }  // namespace flep

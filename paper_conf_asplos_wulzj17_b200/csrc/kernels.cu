@@ -55,6 +55,12 @@ struct Ops {
     else flep_unwrapped<Body><<<count, Body::kThreads, Body::kDynSmem, s>>>(a, grid.x, grid.y, offset);
     return cudaGetLastError();
   }
+  static cudaError_t sliced(const void* args, dim3 grid, uint32_t offset, uint32_t count, const SliceParams& sp,
+                            cudaStream_t s) {
+    const typename Body::Args& a = *reinterpret_cast<const typename Body::Args*>(args);
+    flep_slice<Body><<<count, Body::kThreads, Body::kDynSmem, s>>>(a, grid.x, grid.y, offset, sp);
+    return cudaGetLastError();
+  }
   static cudaError_t occupancy(int* k, bool cov) {
     cudaError_t e;
     if (Body::kDynSmem > 48 * 1024) {
@@ -122,6 +128,17 @@ cudaError_t occupancy_raw(int* k, bool cov) {
   return cudaOccupancyMaxActiveBlocksPerMultiprocessor(k, flep_worker<Body, false>, Body::kThreads, Body::kDynSmem);
 }
 template <class Body>
+cudaError_t launch_slice_raw(const typename Body::Args& a, dim3 grid, uint32_t offset, uint32_t count,
+                             const SliceParams& sp, cudaStream_t s) {
+  const size_t sm = smem_for<Body>(1);
+  if (sm > 48 * 1024) {
+    cudaError_t e = cudaFuncSetAttribute(flep_slice<Body>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    if (e) return e;
+  }
+  flep_slice<Body><<<count, Body::kThreads, sm, s>>>(a, grid.x, grid.y, offset, sp);
+  return cudaGetLastError();
+}
+template <class Body>
 cudaError_t launch_clc_raw(const typename Body::Args& a, const WorkerParams& p, uint32_t N, cudaStream_t s, bool cov) {
   const size_t sm = smem_for<Body>(p.chunk);
   if (cov) flep_clc_worker<Body, true><<<N, Body::kThreads, sm, s>>>(a, p);
@@ -135,6 +152,8 @@ template cudaError_t occupancy_raw<Stencil5TmaBody>(int*, bool);
 template cudaError_t launch_worker_raw<GemmBody>(const GemmBody::Args&, const WorkerParams&, uint32_t, cudaStream_t, bool);
 template cudaError_t launch_unwrapped_raw<GemmBody>(const GemmBody::Args&, dim3, uint32_t, uint32_t, cudaStream_t);
 template cudaError_t occupancy_raw<GemmBody>(int*, bool);
+template cudaError_t launch_slice_raw<GemmBody>(const GemmBody::Args&, dim3, uint32_t, uint32_t, const SliceParams&, cudaStream_t);
+template cudaError_t launch_slice_raw<Stencil5TmaBody>(const Stencil5TmaBody::Args&, dim3, uint32_t, uint32_t, const SliceParams&, cudaStream_t);
 
 namespace {
 
@@ -149,30 +168,31 @@ const BodyOps kOps[] = {
     {0, 0, 0, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr},
     {FLEP_BODY_SAXPY_I32, SaxpyI32::kThreads, sizeof(flep_saxpy_i32_args), &Ops<SaxpyI32>::worker,
      &Ops<SaxpyI32>::unwrapped, &Ops<SaxpyI32>::occupancy, nullptr, &Ops<SaxpyI32>::clc,
-     &Ops<SaxpyI32>::worker_sw, &Ops<SaxpyI32>::occupancy_sw},
+     &Ops<SaxpyI32>::worker_sw, &Ops<SaxpyI32>::occupancy_sw, nullptr, nullptr, 0, &Ops<SaxpyI32>::sliced},
     {FLEP_BODY_SAXPY_F32, SaxpyF32::kThreads, sizeof(flep_saxpy_f32_args), &Ops<SaxpyF32>::worker,
      &Ops<SaxpyF32>::unwrapped, &Ops<SaxpyF32>::occupancy, nullptr, &Ops<SaxpyF32>::clc,
-     &Ops<SaxpyF32>::worker_sw, &Ops<SaxpyF32>::occupancy_sw},
+     &Ops<SaxpyF32>::worker_sw, &Ops<SaxpyF32>::occupancy_sw, nullptr, nullptr, 0, &Ops<SaxpyF32>::sliced},
     {FLEP_BODY_SPMV_CSR_F32, Spmv::kThreads, sizeof(flep_spmv_args), &Ops<Spmv>::worker,
      &Ops<Spmv>::unwrapped, &Ops<Spmv>::occupancy, nullptr, &Ops<Spmv>::clc,
-     &Ops<Spmv>::worker_sw, &Ops<Spmv>::occupancy_sw},
+     &Ops<Spmv>::worker_sw, &Ops<Spmv>::occupancy_sw, nullptr, nullptr, 0, &Ops<Spmv>::sliced},
     {FLEP_BODY_STENCIL5_F32, StencilF32::kThreads, sizeof(flep_stencil_args), &Ops<StencilF32>::worker,
      &Ops<StencilF32>::unwrapped, &Ops<StencilF32>::occupancy, nullptr, &Ops<StencilF32>::clc,
      &Ops<StencilF32>::worker_sw, &Ops<StencilF32>::occupancy_sw, &Ops<StencilF32>::warp_worker,
-     &Ops<StencilF32>::occupancy_warp, StencilF32::kWarpTasks},
+     &Ops<StencilF32>::occupancy_warp, StencilF32::kWarpTasks, &Ops<StencilF32>::sliced},
     {FLEP_BODY_STENCIL5_I32, StencilI32::kThreads, sizeof(flep_stencil_args), &Ops<StencilI32>::worker,
      &Ops<StencilI32>::unwrapped, &Ops<StencilI32>::occupancy, nullptr, &Ops<StencilI32>::clc,
      &Ops<StencilI32>::worker_sw, &Ops<StencilI32>::occupancy_sw, &Ops<StencilI32>::warp_worker,
-     &Ops<StencilI32>::occupancy_warp, StencilI32::kWarpTasks},
+     &Ops<StencilI32>::occupancy_warp, StencilI32::kWarpTasks, &Ops<StencilI32>::sliced},
     {FLEP_BODY_GEMM_BF16, GemmBody::kThreads, sizeof(flep_gemm_args), &gemm_worker_launch,
-     &gemm_unwrapped_launch, &gemm_occupancy, &gemm_validate, nullptr, nullptr, nullptr},
+     &gemm_unwrapped_launch, &gemm_occupancy, &gemm_validate, nullptr, nullptr, nullptr, nullptr, nullptr, 0,
+     &gemm_slice_launch},
     {FLEP_BODY_STENCIL5_F32_TMA, Stencil5TmaBody::kThreads, sizeof(flep_stencil_args), &stencil_tma_worker_launch,
      &stencil_tma_unwrapped_launch, &stencil_tma_occupancy, &stencil_tma_validate, &stencil_tma_clc_launch,
-     nullptr, nullptr},
+     nullptr, nullptr, nullptr, nullptr, 0, &stencil_tma_slice_launch},
     {FLEP_BODY_SPMV_CSR_F32_VEC, SpmvVec::kThreads, sizeof(flep_spmv_args), &Ops<SpmvVec>::worker,
      &Ops<SpmvVec>::unwrapped, &Ops<SpmvVec>::occupancy, nullptr, &Ops<SpmvVec>::clc,
      &Ops<SpmvVec>::worker_sw, &Ops<SpmvVec>::occupancy_sw, &Ops<SpmvVec>::warp_worker,
-     &Ops<SpmvVec>::occupancy_warp, SpmvVec::kWarpTasks},
+     &Ops<SpmvVec>::occupancy_warp, SpmvVec::kWarpTasks, &Ops<SpmvVec>::sliced},
 };
 
 }  // namespace

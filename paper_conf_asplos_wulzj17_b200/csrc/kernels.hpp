@@ -32,9 +32,15 @@ struct BodyOps {
   cudaError_t (*warp_worker)(const void* args, const WorkerParams& p, uint32_t G, cudaStream_t s, bool cov);
   cudaError_t (*occupancy_warp)(int* ctas_per_sm, bool cov);
   uint32_t warp_tasks;
+  // kernel slicing with the device check (flep_slice<Body>, R31): blocks [offset, offset+count)
+  cudaError_t (*sliced)(const void* args, dim3 grid, uint32_t offset, uint32_t count, const SliceParams& sp,
+                        cudaStream_t s);
 };
 
 const BodyOps* body_ops(int32_t body);
+// GEMM body (gemm_tcgen05.cu)
+cudaError_t gemm_slice_launch(const void* user, dim3 grid, uint32_t offset, uint32_t count,
+                              const SliceParams& sp, cudaStream_t s);
 #ifdef FLEP_TRACE
 cudaError_t set_unwrapped_trace(uint64_t* p);
 #endif
@@ -46,6 +52,9 @@ cudaError_t launch_unwrapped_raw(const typename Body::Args& a, dim3 grid, uint32
 template <class Body>
 cudaError_t occupancy_raw(int* k, bool cov);
 template <class Body>
+cudaError_t launch_slice_raw(const typename Body::Args& a, dim3 grid, uint32_t offset, uint32_t count,
+                             const SliceParams& sp, cudaStream_t s);
+template <class Body>
 cudaError_t launch_clc_raw(const typename Body::Args& a, const WorkerParams& p, uint32_t N, cudaStream_t s, bool cov);
 
 // TMA-staged stencil body (stencil_tma.cu)
@@ -54,5 +63,7 @@ cudaError_t stencil_tma_worker_launch(const void* user, const WorkerParams& p, u
 cudaError_t stencil_tma_unwrapped_launch(const void* user, dim3 grid, uint32_t offset, uint32_t count, cudaStream_t s);
 cudaError_t stencil_tma_clc_launch(const void* user, const WorkerParams& p, uint32_t N, cudaStream_t s, bool cov);
 cudaError_t stencil_tma_occupancy(int* k, bool cov);
+cudaError_t stencil_tma_slice_launch(const void* user, dim3 grid, uint32_t offset, uint32_t count,
+                                     const SliceParams& sp, cudaStream_t s);
 
 }  // namespace flep

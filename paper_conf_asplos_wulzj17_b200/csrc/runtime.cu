@@ -85,6 +85,7 @@ flep_status resolve_driver() {
 }
 
 constexpr uint32_t kMaxSlots = 1u << 14;       // pinned status slots (recycled)
+constexpr uint32_t kMaxSlices = 4096;          // R31: decision words per launch
 constexpr uint32_t kMaxWorkersPerSm = 64;     // warp workers: 8 CTAs x 8 warps
 
 struct Launch {
@@ -124,6 +125,9 @@ struct Launch {
   // kernel-slicing baseline (FLEP_POLICY_SLICE): the original kernel as sub-grids of
   // slice_blocks blocks, at most two in flight; a preemption stops issuing
   bool sliced = false;
+  bool slice_dev = false;            // FLEP_POLICY_SLICE_DEVICE: all slices enqueued, device check (R31)
+  uint32_t* slice_dec = nullptr;     // per-slice decision words (in the control block's allocation)
+  uint32_t n_slices = 0;
   bool clc = false;                  // FLEP_KFLAG_CLC: hardware work queue, resume = clear (R25)
   bool sw = false;                   // FLEP_KFLAG_SCHED_WARP: scheduling-warp worker (R26)
   bool relay = false;                // FLEP_KFLAG_HOST_RELAY: one request-relay CTA (R28)
@@ -327,6 +331,7 @@ flep_status materialize(flep_rt rt, Launch& L) {
   if (L.gen0 + 2 * kEvEpochs >= kCtrlGenMask) return fail(FLEP_ERR_NOMEM, "control block generation space exhausted");
   L.cb = (ControlBlock*)L.dmem;
   L.ev = (WorkerEvent*)((char*)L.dmem + sizeof(ControlBlock));
+  L.slice_dec = (uint32_t*)((char*)L.dmem + sizeof(ControlBlock) + (size_t)kEvEpochs * rt->max_workers * sizeof(WorkerEvent));
   tm[3] = now_ns();
   const uint32_t N = L.n_blocks;
   if (L.want_cov) {
@@ -343,12 +348,14 @@ flep_status materialize(flep_rt rt, Launch& L) {
     // per-worker partial-tile records and fp32 accumulator spill slots; no reset needed (the
     // first epoch's workers clear their records)
     const size_t need = partial_bytes(L.workers);
-    for (size_t i = 0; i < rt->free_partial.size(); ++i) {
-      if (rt->free_partial[i].second >= need) {
-        L.partial = rt->free_partial[i].first; L.partial_cap = rt->free_partial[i].second;
-        rt->free_partial.erase(rt->free_partial.begin() + i);
-        break;
-      }
+    size_t best = rt->free_partial.size();
+    for (size_t i = 0; i < rt->free_partial.size(); ++i)
+      if (rt->free_partial[i].second >= need &&
+          (best == rt->free_partial.size() || rt->free_partial[i].second < rt->free_partial[best].second))
+        best = i;
+    if (best < rt->free_partial.size()) {
+      L.partial = rt->free_partial[best].first; L.partial_cap = rt->free_partial[best].second;
+      rt->free_partial.erase(rt->free_partial.begin() + best);
     }
     if (!L.partial) { L.partial_cap = need; CUDA_TRY(cudaMalloc(&L.partial, need)); }
   }
@@ -364,6 +371,7 @@ flep_status materialize(flep_rt rt, Launch& L) {
   if (s) return s;
   if (L.cov) CUDA_TRY(cudaMemsetAsync(L.cov, 0, (size_t)N * 4, L.exec));
   if (fresh_cb) CUDA_TRY(cudaMemsetAsync(L.dmem, 0, sizeof(ControlBlock), L.exec));
+  if (L.slice_dev) CUDA_TRY(cudaMemsetAsync(L.slice_dec, 0, (size_t)L.n_slices * 4, L.exec));   // R31
   tm[5] = now_ns();
   if (slow_threshold_ns() >= 0 && tm[5] - tm[0] > slow_threshold_ns())
     fprintf(stderr, "[flep] materialize launch %lld: stream %.1f wait %.1f block %.1f bufs %.1f event %.1f us\n",
@@ -390,6 +398,22 @@ flep_status start_epoch(flep_rt rt, Launch& L) {
                 (long long)L.id, L.body, L.epoch, (b - a) / 1e3, fresh ? " (first)" : "", (c - b) / 1e3);
     }
   } slow_report{L, t_a, t_b, fresh};
+  if (L.sliced && L.slice_dev) {
+    // R31: every remaining slice goes on the stream now; each decides at its entry
+    L.epoch++;
+    SliceParams sp{&L.cb->ctrl, L.slice_dec, 0, gen_of(L)};
+    for (uint64_t off = L.next_block; off < L.n_blocks; off += L.slice_blocks) {
+      sp.slice = (uint32_t)(off / L.slice_blocks);
+      const uint32_t cnt = (uint32_t)std::min<uint64_t>(L.slice_blocks, L.n_blocks - off);
+      CUDA_TRY(L.ops->sliced(L.args.data(), L.grid, (uint32_t)off, cnt, sp, L.exec));
+    }
+    CUDA_TRY(cudaEventRecord(L.fin_ev, L.exec));
+    L.state = FLEP_STATE_RUNNING;
+    L.n_yield = 0;
+    if (L.t_first_start < 0) L.t_first_start = now_ns();
+    mark_active(rt, L);
+    return FLEP_OK;
+  }
   if (L.sliced) {
     L.epoch++;
     L.state = FLEP_STATE_RUNNING;
@@ -456,6 +480,46 @@ bool refresh(flep_rt rt, Launch& L) {
   if (L.state != FLEP_STATE_RUNNING && L.state != FLEP_STATE_YIELDING && L.state != FLEP_STATE_PARTIAL &&
       !(L.clc && L.state == FLEP_STATE_PREEMPTED))   // a preempted CLC grid still completes (R25)
     return false;
+  if (L.sliced && L.slice_dev) {
+    // R31: the epoch's slices have all run or been skipped once its last grid completed; the
+    // skipped ones are a suffix (a request stays in force until the resume), found from the
+    // decision words
+    if (!(L.fin_ev && cudaEventQuery(L.fin_ev) == cudaSuccess)) return false;
+    const uint32_t j0 = (uint32_t)(L.next_block / L.slice_blocks);
+    std::vector<uint32_t> dec(L.n_slices - j0);
+    if (!dec.empty()) {
+      if (cudaMemcpyAsync(dec.data(), L.slice_dec + j0, dec.size() * 4, cudaMemcpyDeviceToHost, rt->aux) != cudaSuccess ||
+          cudaStreamSynchronize(rt->aux) != cudaSuccess)
+        return false;
+    }
+    // progress = the first slice not run in any epoch (a resume issued before this epoch's end
+    // was seen starts from the older bound; its slices that already ran skip themselves)
+    uint64_t next = L.n_blocks;
+    for (size_t i = 0; i < dec.size(); ++i)
+      if ((dec[i] & 3u) != kSliceRun) {
+        next = (uint64_t)(j0 + i) * L.slice_blocks;
+        break;
+      }
+    if (slow_threshold_ns() >= 0) {
+      fprintf(stderr, "[flep] slice epoch end: launch %lld gen %u j0 %u slices %u next %llu dec:", (long long)L.id,
+              gen_of(L), j0, L.n_slices, (unsigned long long)next);
+      for (size_t i = 0; i < dec.size() && i < 80; ++i) fprintf(stderr, " %u:%u", dec[i] >> 2, dec[i] & 3u);
+      fprintf(stderr, "\n");
+    }
+    L.next_block = next;
+    L.slice_done = next;
+    L.last_done = (uint32_t)next;
+    L.last_ctr = (uint32_t)next;
+    if (next >= L.n_blocks) {
+      L.state = FLEP_STATE_DONE;
+      L.t_finish = L.t_seen > 0 ? L.t_seen : now_ns();
+      L.t_seen = 0;
+      return true;
+    }
+    L.state = FLEP_STATE_PREEMPTED;
+    L.t_last_drain = now_ns();
+    return false;
+  }
   if (L.sliced) {
     while (!L.inflight.empty() && cudaEventQuery(L.inflight.front().first) == cudaSuccess) {
       L.slice_done += L.inflight.front().second;
@@ -545,7 +609,12 @@ void apply_decisions(flep_rt rt) {
     Launch& L = *it->second;
     if (x.action == kPreempt) {
       const bool spatial = x.n_sms < (int64_t)rt->num_sms;
-      if (L.sliced && L.state == FLEP_STATE_RUNNING) {   // slicing: stop issuing sub-kernels
+      if (L.sliced && L.slice_dev && L.state == FLEP_STATE_RUNNING) {
+        // R31: the slices not yet entered skip themselves once the request is in force
+        write_ctrl(rt, L, ctrl_word(L, kCtrlAll));
+        L.state = FLEP_STATE_YIELDING;
+        L.n_yield = (uint32_t)x.n_sms;
+      } else if (L.sliced && L.state == FLEP_STATE_RUNNING) {   // slicing: stop issuing sub-kernels
         L.t_last_request = now_ns();
         L.state = FLEP_STATE_YIELDING;
         L.n_yield = (uint32_t)x.n_sms;
@@ -706,8 +775,9 @@ void monitor_loop(flep_rt rt) {
       auto it = snap.find(id);
       const bool running = L->state == FLEP_STATE_RUNNING || L->state == FLEP_STATE_YIELDING ||
                            L->state == FLEP_STATE_PARTIAL || (L->clc && L->state == FLEP_STATE_PREEMPTED);
-      watch.push_back({wp, it != snap.end() ? it->second : ~0ull, L->sliced, id,
-                       (running && !L->sliced) ? L->fin_ev : nullptr});
+      const bool host_sliced = L->sliced && !L->slice_dev;    // host-issued slices: every pass
+      watch.push_back({wp, it != snap.end() ? it->second : ~0ull, host_sliced, id,
+                       (running && !host_sliced) ? L->fin_ev : nullptr});
     }
     deadline = rt->policy->epoch_end();
     pending_release = !rt->to_release.empty();
@@ -750,7 +820,7 @@ flep_status flep_init(int device, const flep_options* opts, flep_rt* out) {
   if (opts) rt->opt = *opts;
   if (rt->opt.default_chunk == 0) rt->opt.default_chunk = 8;
   if (rt->opt.default_poll == 0) rt->opt.default_poll = 1;
-  if (rt->opt.policy < FLEP_POLICY_MANUAL || rt->opt.policy > FLEP_POLICY_REORDER)
+  if (rt->opt.policy < FLEP_POLICY_MANUAL || rt->opt.policy > FLEP_POLICY_SLICE_DEVICE)
     return fail(FLEP_ERR_INVALID, "bad policy %d", rt->opt.policy);
   if (rt->opt.spatial && rt->opt.policy != FLEP_POLICY_HPF)
     return fail(FLEP_ERR_INVALID, "spatial decisions need the HPF policy");
@@ -782,7 +852,8 @@ flep_status flep_init(int device, const flep_options* opts, flep_rt* out) {
   CUDA_TRY(cudaHostGetDevicePointer(&rt->d_slots, rt->h_slots, 0));
   for (int i = kMaxSlots - 1; i >= 0; --i) rt->free_slots.push_back(i);
   rt->max_workers = rt->num_sms * kMaxWorkersPerSm;
-  rt->dmem_bytes = sizeof(ControlBlock) + (size_t)kEvEpochs * rt->max_workers * sizeof(WorkerEvent);
+  rt->dmem_bytes = sizeof(ControlBlock) + (size_t)kEvEpochs * rt->max_workers * sizeof(WorkerEvent) +
+                  (size_t)kMaxSlices * sizeof(uint32_t);
   for (int i = 0; i < 16; ++i) {             // warm pool: no allocation on the launch path
     void* p = nullptr;
     CUDA_TRY(cudaMalloc(&p, rt->dmem_bytes));
@@ -806,7 +877,8 @@ flep_status flep_init(int device, const flep_options* opts, flep_rt* out) {
     }
   }
   if (rt->opt.policy != FLEP_POLICY_MANUAL) {
-    rt->policy.reset(new Policy(rt->opt.policy == FLEP_POLICY_SLICE ? (int32_t)kPolicyHPF : rt->opt.policy,
+    const bool slicing = rt->opt.policy == FLEP_POLICY_SLICE || rt->opt.policy == FLEP_POLICY_SLICE_DEVICE;
+    rt->policy.reset(new Policy(slicing ? (int32_t)kPolicyHPF : rt->opt.policy,
                                 rt->num_sms, rt->opt.max_overhead_ppm ? rt->opt.max_overhead_ppm : 100000));
     // spatial decisions (R29): HPF on the persistent-worker mechanism only (a sliced kernel has no
     // per-SM yield)
@@ -833,6 +905,23 @@ flep_status flep_register_kernel(flep_rt rt, const flep_kernel_desc* d, flep_ker
   if ((d->flags & FLEP_KFLAG_IN_TILE) && (d->flags & FLEP_KFLAG_PREFETCH))
     return fail(FLEP_ERR_UNSUPPORTED, "in-tile preemption does not combine with chunk prefetch");
   ApiLock lk(rt);
+  if (d->flags & FLEP_KFLAG_IN_TILE) {
+    // in-tile records + accumulator spill slots for the largest worker grid this kernel can have,
+    // allocated here (a cudaMalloc on the launch path took 3-50 ms while kernels ran, stalling
+    // the monitor): keep three in the pool
+    int kk = 0;
+    flep_status s = occupancy(rt, body_ops(d->body), (rt->opt.debug_coverage & 1u) != 0, &kk);
+    if (s) return s;
+    if (d->ctas_per_sm && (int)d->ctas_per_sm < kk) kk = (int)d->ctas_per_sm;
+    const size_t need = partial_bytes(std::min<uint32_t>((uint32_t)kk * rt->num_sms, rt->max_workers));
+    size_t have = 0;
+    for (auto& f : rt->free_partial) if (f.second >= need) ++have;
+    for (; have < 3; ++have) {
+      void* p = nullptr;
+      CUDA_TRY(cudaMalloc(&p, need));
+      rt->free_partial.push_back({p, need});
+    }
+  }
   KernelReg k;
   k.name = d->name ? d->name : "";
   k.body = d->body;
@@ -881,7 +970,8 @@ flep_status flep_launch(flep_rt rt, flep_kernel kid, flep_dim3 grid, const void*
   const bool sw = (kr.flags & FLEP_KFLAG_SCHED_WARP) && !(kr.flags & FLEP_KFLAG_CLC);
   if (sw && !ops->worker_sw) return fail(FLEP_ERR_UNSUPPORTED, "body %d has no scheduling-warp worker", kr.body);
   // R30: warp tasks (not under SLICE, whose sub-kernels are the unwrapped original grid)
-  const bool warp = (kr.flags & FLEP_KFLAG_WARP_TASKS) && rt->opt.policy != FLEP_POLICY_SLICE;
+  const bool slicing = rt->opt.policy == FLEP_POLICY_SLICE || rt->opt.policy == FLEP_POLICY_SLICE_DEVICE;
+  const bool warp = (kr.flags & FLEP_KFLAG_WARP_TASKS) && !slicing;
   if (warp && (!ops->warp_worker || !ops->warp_tasks))
     return fail(FLEP_ERR_UNSUPPORTED, "body %d has no warp-task worker", kr.body);
   if (warp && (sw || (kr.flags & (FLEP_KFLAG_CLC | FLEP_KFLAG_IN_TILE))))
@@ -912,7 +1002,7 @@ flep_status flep_launch(flep_rt rt, flep_kernel kid, flep_dim3 grid, const void*
   L.sw = sw;
   if (kr.flags & FLEP_KFLAG_CLC) {
     if (!ops->clc) return fail(FLEP_ERR_UNSUPPORTED, "body %d has no CLC variant", kr.body);
-    if (rt->opt.policy == FLEP_POLICY_SLICE) return fail(FLEP_ERR_UNSUPPORTED, "CLC kernels cannot be sliced");
+    if (slicing) return fail(FLEP_ERR_UNSUPPORTED, "CLC kernels cannot be sliced");
     L.clc = true;                                    // CTA i of the CLC grid = chunk i (C blocks)
   }
   if (kr.ctas_per_sm && (int)kr.ctas_per_sm < k) k = (int)kr.ctas_per_sm;
@@ -937,10 +1027,17 @@ flep_status flep_launch(flep_rt rt, flep_kernel kid, flep_dim3 grid, const void*
     const uint64_t ctas = L.clc ? std::min<uint64_t>(need, wmax) : (uint64_t)L.ctas + (L.relay ? 1u : 0u);
     L.sms_need = (int64_t)std::min<uint64_t>(rt->num_sms, (ctas + (uint64_t)k - 1) / (uint64_t)k);
   }
-  if (rt->opt.policy == FLEP_POLICY_SLICE) {
+  if (slicing) {
     L.sliced = true;                                  // R16: one slice = one wave of W*C*K blocks
     L.slice_blocks = rt->opt.slice_blocks ? rt->opt.slice_blocks
                                           : (uint32_t)std::min<uint64_t>(wmax * L.chunk * L.poll, 0x7fffffff);
+    if (rt->opt.policy == FLEP_POLICY_SLICE_DEVICE) {
+      if (!ops->sliced) return fail(FLEP_ERR_UNSUPPORTED, "body %d has no device-checked slice kernel", kr.body);
+      L.slice_dev = true;
+      // at most kMaxSlices decision words: larger slices for very large grids
+      L.slice_blocks = std::max<uint32_t>(L.slice_blocks, (uint32_t)((N + kMaxSlices - 1) / kMaxSlices));
+      L.n_slices = (uint32_t)((N + L.slice_blocks - 1) / L.slice_blocks);
+    }
   }
   L.t_arrive = now_ns();
   L.t_e = flep_model_predict_ns(kr.model, (double)N, (double)ops->threads, (double)N, 0.0);
@@ -955,7 +1052,7 @@ flep_status flep_launch(flep_rt rt, flep_kernel kid, flep_dim3 grid, const void*
   // queue can hold hundreds of intercepted launches, and only running or preempted ones need them.
   L.exec_level = stream_level(rt, priority);
   L.want_cov = cov;
-  if (rt->opt.exec_on_user_stream && rt->opt.policy == FLEP_POLICY_MANUAL) {
+  if (rt->opt.exec_on_user_stream) {
     L.exec = L.user;
     L.exec_level = -1000;
   } else {
@@ -1402,8 +1499,8 @@ flep_status flep_policy_set_max_overhead(flep_policy_t p, uint32_t ppm) {
 
 flep_status flep_policy_create(int32_t kind, uint32_t num_sms, flep_policy_t* out) {
   if (!out) return fail(FLEP_ERR_INVALID, "out is NULL");
-  if (kind < kPolicyFIFO || kind > kPolicyREORDER) return fail(FLEP_ERR_INVALID, "bad policy kind %d", kind);
-  *out = new flep_policy_s(kind == kPolicySLICE ? kPolicyHPF : kind, num_sms);
+  if (kind < kPolicyFIFO || kind > kPolicyREORDER + 1) return fail(FLEP_ERR_INVALID, "bad policy kind %d", kind);
+  *out = new flep_policy_s((kind == kPolicySLICE || kind == kPolicyREORDER + 1) ? kPolicyHPF : kind, num_sms);
   return FLEP_OK;
 }
 flep_status flep_policy_destroy(flep_policy_t p) { delete p; return FLEP_OK; }

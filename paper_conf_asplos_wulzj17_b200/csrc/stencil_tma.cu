@@ -78,4 +78,11 @@ cudaError_t stencil_tma_clc_launch(const void* user, const WorkerParams& p, uint
 
 cudaError_t stencil_tma_occupancy(int* k, bool cov) { return occupancy_raw<Stencil5TmaBody>(k, cov); }
 
+cudaError_t stencil_tma_slice_launch(const void* user, dim3 grid, uint32_t offset, uint32_t count,
+                               const SliceParams& sp, cudaStream_t s) {
+  StencilTmaArgsDev d;
+  if (!to_dev(user, &d)) return cudaErrorInvalidValue;
+  return launch_slice_raw<Stencil5TmaBody>(d, grid, offset, count, sp, s);
+}
+
 }  // namespace flep

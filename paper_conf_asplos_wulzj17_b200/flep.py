@@ -14,6 +14,7 @@ LIB_PATH = os.environ.get("FLEP_LIB_PATH") or os.path.join(HERE, "libflep.so")  
 
 OK, ERR_INVALID, ERR_STATE, ERR_CUDA, ERR_NOMEM, ERR_TIMEOUT, ERR_UNSUPPORTED = 0, -1, -2, -3, -4, -5, -6
 POLICY_MANUAL, POLICY_FIFO, POLICY_HPF, POLICY_SLICE, POLICY_FFS, POLICY_REORDER = 0, 1, 2, 3, 4, 5
+POLICY_SLICE_DEVICE = 6
 FLAG_STREAM_MEMOP, FLAG_HOST_MAPPED = 0, 1
 BODY_SAXPY_I32, BODY_SAXPY_F32, BODY_SPMV_CSR_F32, BODY_STENCIL5_F32, BODY_STENCIL5_I32, BODY_GEMM_BF16 = 1, 2, 3, 4, 5, 6
 BODY_STENCIL5_F32_TMA = 7

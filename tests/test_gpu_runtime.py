@@ -410,3 +410,55 @@ def test_managed_cancel_releases_the_policy():
             assert np.array_equal(y2d.cpu().numpy(), W.saxpy_i32(11, x2, y2))
     finally:
         rt.close()
+
+
+@pytest.mark.parametrize("stream_exec", [False, True])
+def test_slice_device_preempts_at_slice_boundaries(stream_exec):
+    """Kernel slicing with every slice enqueued and the device check at slice entry (R31): the
+    high-priority arrival makes the remaining slices skip themselves; the victim resumes at the
+    first skipped slice; results bit-exact; decisions = HPF's, replayed by the oracle."""
+    f = flep_mod()
+    import torch
+    rt = f.Runtime(policy=f.POLICY_SLICE_DEVICE, slice_blocks=4096, exec_on_user_stream=stream_exec)
+    try:
+        n_lp, n_hp = 1 << 26, 1 << 16
+        x, y = gen.saxpy_i32_inputs(n_lp, seed=81)
+        x2, y2 = gen.saxpy_i32_inputs(n_hp, seed=82)
+        xd, yd, x2d, y2d = t(x), t(y), t(x2), t(y2)
+        k_lp = rt.register_kernel(f.BODY_SAXPY_I32, chunk=1, poll=1, model=(0, 0, 0, 0, 2_000_000))
+        k_hp = rt.register_kernel(f.BODY_SAXPY_I32, chunk=1, poll=1, model=(0, 0, 0, 0, 5_000))
+        sA, sB = torch.cuda.Stream(), torch.cuda.Stream()
+        h_lp = rt.launch(k_lp, f.saxpy_grid(n_lp), f.saxpy_i32_args(yd, xd, 7), priority=0, stream=sA)
+        h_hp = rt.launch(k_hp, f.saxpy_grid(n_hp), f.saxpy_i32_args(y2d, x2d, 9), priority=1, stream=sB)
+        rt.sync(h_hp, timeout_ns=10_000_000_000)
+        rt.sync(h_lp, timeout_ns=10_000_000_000)
+        torch.cuda.synchronize()
+        assert np.array_equal(yd.cpu().numpy(), W.saxpy_i32(7, x, y))
+        assert np.array_equal(y2d.cpu().numpy(), W.saxpy_i32(9, x2, y2))
+        dec = rt.decision_log()
+        acts = [f.ACTION_NAMES[d[1]] for d in dec]
+        assert acts == ["LAUNCH", "PREEMPT", "LAUNCH", "RESUME"]
+        info = rt.query(h_lp)
+        assert info.epoch == 2 and info.state == f.STATE_DONE
+        assert dec == _replay_from_runtime(rt, des.HPF)
+    finally:
+        rt.close()
+
+
+def test_slice_device_never_preempted_exact():
+    f = flep_mod()
+    import torch
+    rt = f.Runtime(policy=f.POLICY_SLICE_DEVICE)
+    try:
+        for n in (3, 1000, 4096):
+            a = gen.stencil_i32_input(n, seed=83)
+            ind = t(a)
+            outd = torch.empty_like(ind)
+            k = rt.register_kernel(f.BODY_STENCIL5_I32, chunk=1, poll=1)
+            h = rt.launch(k, f.stencil_grid(n), f.stencil_args(outd, ind))
+            rt.sync(h, timeout_ns=10_000_000_000)
+            torch.cuda.synchronize()
+            assert np.array_equal(outd.cpu().numpy(), W.stencil5_i32(a))
+            assert rt.query(h).epoch == 1
+    finally:
+        rt.close()
