@@ -1055,14 +1055,16 @@ def run_tune(args, rank, world, local):
     g.manual_seed(21 + rank)
     cases = {}
     x, y = gen.saxpy_i32_inputs(1 << 20, seed=1)
-    cases["saxpy_i32_2^20 (configs[0] LP)"] = (F.BODY_SAXPY_I32, F.saxpy_grid(1 << 20), F.saxpy_i32_args(T(y), T(x), 3))
+    keep = [T(y), T(x)]                  # device tensors must outlive the args structs (raw pointers)
+    cases["saxpy_i32_2^20 (configs[0] LP)"] = (F.BODY_SAXPY_I32, F.saxpy_grid(1 << 20), F.saxpy_i32_args(keep[0], keep[1], 3))
     xs = torch.ones(1 << 28, dtype=torch.int32, device="cuda")
     ys = torch.ones(1 << 28, dtype=torch.int32, device="cuda")
     cases["saxpy_i32_2^28"] = (F.BODY_SAXPY_I32, F.saxpy_grid(1 << 28), F.saxpy_i32_args(ys, xs, 3))
     rp, col, val, xv = gen.csr_inputs(1 << 20, seed=2)
     yv = torch.zeros(1 << 20, device="cuda")
+    keep += [T(rp), T(col), T(val), T(xv)]
     cases["spmv_2^20 (configs[1] LP)"] = (F.BODY_SPMV_CSR_F32, F.spmv_grid(1 << 20),
-                                          F.spmv_args(yv, T(rp), T(col), T(val), T(xv)))
+                                          F.spmv_args(yv, *keep[2:6]))
     st = T(gen.stencil_f32_input(4096, seed=3))
     so = torch.empty_like(st)
     cases["stencil_4096^2 (configs[1] HP)"] = (F.BODY_STENCIL5_F32, F.stencil_grid(4096), F.stencil_args(so, st))

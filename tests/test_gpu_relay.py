@@ -61,7 +61,8 @@ def test_relay_host_request_preempts_and_resumes(rt):
     import torch
     y = torch.zeros(rows, device="cuda")
     k = rt.register_kernel(f.BODY_SPMV_CSR_F32, chunk=1, poll=1, host_relay=True, started_hint=True)
-    h = rt.launch(k, f.spmv_grid(rows), f.spmv_args(y, t(rp), t(col), t(val), t(xv)))
+    keep = (t(rp), t(col), t(val), t(xv))       # outlive the args struct (raw pointers)
+    h = rt.launch(k, f.spmv_grid(rows), f.spmv_args(y, *keep))
     t0 = time.perf_counter()
     while rt.query(h).started_epoch < 1 and time.perf_counter() - t0 < 1:
         pass
@@ -95,7 +96,8 @@ def test_relay_leaves_a_released_sm(rt, seed):
     k = rt.register_kernel(f.BODY_SPMV_CSR_F32, chunk=1, poll=1, host_relay=True, started_hint=True)
     g = gen.rng(4000 + seed)
     n = int(g.integers(1, rt.num_sms))
-    h = rt.launch(k, f.spmv_grid(rows), f.spmv_args(y, t(rp), t(col), t(val), t(xv)))
+    keep = (t(rp), t(col), t(val), t(xv))       # outlive the args struct (raw pointers)
+    h = rt.launch(k, f.spmv_grid(rows), f.spmv_args(y, *keep))
     t0 = time.perf_counter()
     while rt.query(h).started_epoch < 1 and time.perf_counter() - t0 < 1:
         pass

@@ -26,7 +26,8 @@ def main():
             T = lambda a: torch.from_numpy(a).cuda()  # noqa: E731
             yv = torch.zeros(rows, device="cuda")
             k = rt.register_kernel(F.BODY_SPMV_CSR_F32, chunk=1, poll=1, started_hint=True)
-            grid, kargs = F.spmv_grid(rows), F.spmv_args(yv, T(rp), T(col), T(val), T(xv))
+            keep = (T(rp), T(col), T(val), T(xv))   # outlive the args struct (raw pointers)
+            grid, kargs = F.spmv_grid(rows), F.spmv_args(yv, *keep)
         else:
             n = 1 << 28
             x = torch.ones(n, dtype=torch.int32, device="cuda")

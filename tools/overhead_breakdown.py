@@ -32,9 +32,10 @@ def main():
     st = T(gen.stencil_f32_input(4096, seed=3))
     out = torch.empty_like(st)
     rp, col, val, x = gen.csr_inputs(1 << 20, seed=2)
+    dev = (T(rp), T(col), T(val), T(x))   # outlive the args structs (raw pointers)
     y = torch.zeros(1 << 20, device="cuda")
     cases = [("stencil", F.BODY_STENCIL5_F32, F.stencil_grid(4096), F.stencil_args(out, st)),
-             ("spmv", F.BODY_SPMV_CSR_F32, F.spmv_grid(1 << 20), F.spmv_args(y, T(rp), T(col), T(val), T(x)))]
+             ("spmv", F.BODY_SPMV_CSR_F32, F.spmv_grid(1 << 20), F.spmv_args(y, *dev))]
     s = torch.cuda.current_stream()
     reps = 30
 

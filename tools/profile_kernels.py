@@ -35,8 +35,9 @@ def main():
     if "spmv" in a.kernels:
         rp, col, val, x = gen.csr_inputs(1 << 20, seed=2)
         y = torch.zeros(1 << 20, device="cuda")
-        args = F.spmv_args(y, T(rp), T(col), T(val), T(x))
-        jobs.append(("spmv", F.BODY_SPMV_CSR_F32, F.spmv_grid(1 << 20), args, (rp, col, val, x)))
+        dev = (T(rp), T(col), T(val), T(x))        # kept alive: the args struct holds raw pointers
+        args = F.spmv_args(y, *dev)
+        jobs.append(("spmv", F.BODY_SPMV_CSR_F32, F.spmv_grid(1 << 20), args, dev + (y,)))
     if "stencil" in a.kernels:
         st = T(gen.stencil_f32_input(4096, seed=3))
         out = torch.empty_like(st)

@@ -32,7 +32,8 @@ def main():
     rp, col, val, xv = gen.csr_inputs(2000, 2)
     yv = torch.zeros(2000, device="cuda")
     k2 = rt.register_kernel(F.BODY_SPMV_CSR_F32, chunk=2, poll=1, prefetch=True)
-    rt.sync(rt.launch(k2, F.spmv_grid(2000), F.spmv_args(yv, T(rp), T(col), T(val), T(xv))))
+    keep = (T(rp), T(col), T(val), T(xv))       # outlive the args struct (raw pointers)
+    rt.sync(rt.launch(k2, F.spmv_grid(2000), F.spmv_args(yv, *keep)))
     st = T(gen.stencil_f32_input(200, 3))
     out = torch.empty_like(st)
     k3 = rt.register_kernel(F.BODY_STENCIL5_F32, chunk=1, poll=1)

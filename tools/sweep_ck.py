@@ -36,16 +36,18 @@ def main():
     flush = L2Flush(torch)
     T = lambda x: torch.from_numpy(np.ascontiguousarray(x)).cuda()  # noqa: E731
     jobs = {}
-    if "spmv" in a.bodies:
+    if "spmv" in a.bodies.split(","):
         rp, col, val, x = gen.csr_inputs(1 << 20, seed=2)
         y = torch.zeros(1 << 20, device="cuda")
-        jobs["spmv"] = (F.BODY_SPMV_CSR_F32, F.spmv_grid(1 << 20), F.spmv_args(y, T(rp), T(col), T(val), T(x)),
-                        8 * int(rp[-1]) + 12 * (1 << 20), (rp, col, val, x, y))
+        dev = (T(rp), T(col), T(val), T(x))        # kept alive: the args struct holds raw pointers
+        jobs["spmv"] = (F.BODY_SPMV_CSR_F32, F.spmv_grid(1 << 20), F.spmv_args(y, *dev),
+                        8 * int(rp[-1]) + 12 * (1 << 20), dev + (y,))
     if "spmvvec" in a.bodies:
         rp, col, val, x = gen.csr_inputs(1 << 20, seed=2)
         y = torch.zeros(1 << 20, device="cuda")
-        jobs["spmvvec"] = (F.BODY_SPMV_CSR_F32_VEC, F.spmv_grid(1 << 20), F.spmv_args(y, T(rp), T(col), T(val), T(x)),
-                           8 * int(rp[-1]) + 12 * (1 << 20), (rp, col, val, x, y))
+        dev2 = (T(rp), T(col), T(val), T(x))
+        jobs["spmvvec"] = (F.BODY_SPMV_CSR_F32_VEC, F.spmv_grid(1 << 20), F.spmv_args(y, *dev2),
+                           8 * int(rp[-1]) + 12 * (1 << 20), dev2 + (y,))
     if "stencil" in a.bodies.split(","):
         st = T(gen.stencil_f32_input(4096, seed=3))
         out = torch.empty_like(st)
