@@ -357,7 +357,10 @@ def run_temporal(args, rank, world, local):
     gather_roofline = {"bound": "l1_gather", "kernel": "flep_worker<spmv>", "achieved": float(f"{g_ach:.4g}"),
                        "peak": gpk, "unit": "gathers/s", "frac": round(g_ach / gpk, 4) if gpk else None,
                        "unwrapped_frac": round(wl.nnz / (kern["spmv"]["unwrapped_us"] * 1e-6) / gpk, 4) if gpk else None,
-                       "peak_source": "measured: probes/probe6.cu (profiles/r01_probe_gather_ceiling.jsonl)"}
+                       "peak_source": "measured: probes/probe6.cu (profiles/r0[12]_probe_gather_ceiling.jsonl)",
+                       "limiter": "L1TEX->XBAR miss-request interface (one request per cycle per SM): probe 6 runs it at 83 % "
+                                  "of peak (elapsed), the SpMV worker at 61 %, unwrapped 67 % (profiles/r02_probe6_limiter.json, "
+                                  "r02_ncu_full_summary.json); every x gather that misses L1 (95 %) is one request"}
     roofline = {"bound": "hbm", "achieved": round(achieved, 1), "peak": hbm, "unit": "GB/s",
                 "frac": round(achieved / hbm, 4), "traffic": prof_traffic, "kernel": f"flep_worker<{dom}>",
                 "algorithmic_bytes": algo, "peak_source": peak_src}
@@ -465,7 +468,14 @@ def kernel_timings(rt, F, torch, wl, flush, A, kLP, kHP, lp_args, hp_args, lp_gr
                 if r >= 2:
                     (tw if mode == "w" else tu).append(e0.elapsed_time(e1) * 1e3)
         w_us, u_us = event_mean_us(tw), event_mean_us(tu)
+        # 95 % confidence half-width of the overhead ratio (delta method on the sample means)
+        aw, au = np.asarray(tw), np.asarray(tu)
+        mw, mu = float(aw.mean()), float(au.mean())
+        var_r = aw.var(ddof=1) / len(aw) / mu ** 2 + mw ** 2 * au.var(ddof=1) / len(au) / mu ** 4
         res[name] = {"stat": "trimmed mean (middle 80 %) of dithered CUDA-event durations",
+                     "overhead_pct_mean": round((mw / mu - 1.0) * 100.0, 2),
+                     "overhead_pct_ci95": round(1.96 * float(np.sqrt(var_r)) * 100.0, 2),
+                     "samples": [len(tw), len(tu)],
                      "wrapped_us": round(w_us, 3), "unwrapped_us": round(u_us, 3),
                      "wrapped_min_us": round(min(tw), 3), "unwrapped_min_us": round(min(tu), 3),
                      "wrapped_gbs": round(nbytes / (w_us * 1e-6) / 1e9, 1),
@@ -477,12 +487,15 @@ def kernel_timings(rt, F, torch, wl, flush, A, kLP, kHP, lp_args, hp_args, lp_gr
 
 def load_gather_peak():
     """Measured random-gather ceiling (gathers/s) of probes/probe6.cu, committed under profiles/."""
-    p = os.path.join(ROOT, "profiles", "r01_probe_gather_ceiling.jsonl")
-    try:
-        with open(p) as f:
-            return max(json.loads(l)["gathers_per_s"] for l in f if l.strip())
-    except Exception:
-        return None
+    best = None
+    for name in ("r01_probe_gather_ceiling.jsonl", "r02_probe6_gather_ceiling.jsonl"):
+        try:
+            with open(os.path.join(ROOT, "profiles", name)) as f:
+                v = max(json.loads(l)["gathers_per_s"] for l in f if l.strip())
+            best = v if best is None else max(best, v)
+        except Exception:
+            pass
+    return best
 
 
 def load_traffic(dom):

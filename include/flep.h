@@ -94,9 +94,14 @@ typedef enum {
   FLEP_BODY_STENCIL5_F32_TMA = 7, /* STENCIL5_F32 with the tile and its halo staged in shared memory
                                   by the TMA unit and the output tile written back by a bulk
                                   tensor store; same args; n % 4 == 0, 16-byte aligned in/out */
-  FLEP_BODY_SPMV_CSR_F32_VEC = 8 /* y = A x, CSR fp32, CSR-vector form (4 lanes per row, shuffle
+  FLEP_BODY_SPMV_CSR_F32_VEC = 8, /* y = A x, CSR fp32, CSR-vector form (4 lanes per row, shuffle
                                   reduction, no shared memory); same args; 128 rows per block,
                                   each warp owns 16 of them (warp-task capable, R30) */
+  FLEP_BODY_GEMM_BF16_2SM = 9  /* GEMM_BF16 on CTA pairs (cluster of 2, tcgen05.mma.cta_group::2):
+                                  256x256 output tile per block, grid (N/256, M/256, 1),
+                                  M % 256 == N % 256 == K % 64 == 0; the worker is the pair
+                                  (flep_launch_info.workers = pairs), tile-granular preemption, a
+                                  spatial request releases a pair iff it names either SM (R32) */
 } flep_body;
 
 /* Per-body argument structs (copied by value at launch). All pointers are device pointers. */
@@ -294,6 +299,12 @@ flep_status flep_launch_unwrapped(flep_rt rt, int32_t body, flep_dim3 grid, cons
 /* Kernel slicing (K8): ceil(N/slice_blocks) back-to-back sub-kernels of slice_blocks. */
 flep_status flep_launch_sliced(flep_rt rt, int32_t body, flep_dim3 grid, const void* args,
                                size_t args_size, uint32_t slice_blocks, flep_stream_t stream);
+/* The static persistent twin (U1): the body's resident CTAs (pairs for GEMM_BF16_2SM) take chunks
+   of `chunk` blocks in a fixed round-robin order, with no counter, no poll, no exit accounting:
+   persistence without the FLEP wrapper, the baseline that isolates the wrapper's own cost.
+   FLEP_ERR_UNSUPPORTED for bodies without it (the TMA stencil). */
+flep_status flep_launch_static(flep_rt rt, int32_t body, flep_dim3 grid, const void* args,
+                               size_t args_size, uint32_t chunk, flep_stream_t stream);
 /* Worker grid size W (= resident CTAs per SM x SMs) for a body / chunk. */
 flep_status flep_workers_for(flep_rt rt, int32_t body, uint32_t* ctas_per_sm, uint32_t* workers);
 

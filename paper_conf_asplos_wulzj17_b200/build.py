@@ -9,8 +9,9 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libflep.so")
-SOURCES = ["kernels.cu", "gemm_tcgen05.cu", "stencil_tma.cu", "runtime.cu"]
-HEADERS = ["flep_device.cuh", "bodies.cuh", "gemm_tcgen05.cuh", "stencil_tma.cuh", "kernels.hpp", "policy.hpp"]
+SOURCES = ["kernels.cu", "gemm_tcgen05.cu", "gemm2_tcgen05.cu", "stencil_tma.cu", "runtime.cu"]
+HEADERS = ["flep_device.cuh", "bodies.cuh", "gemm_tcgen05.cuh", "gemm2_tcgen05.cuh", "stencil_tma.cuh", "kernels.hpp",
+           "policy.hpp"]
 
 NVCC_FLAGS = [
     "-gencode", "arch=compute_100a,code=sm_100a",

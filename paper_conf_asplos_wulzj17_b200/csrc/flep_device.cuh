@@ -113,6 +113,8 @@ struct WorkerParams {
   uint32_t ctrl_sys;       // 1: `ctrl` is a CPU-written mapped host word (FLEP_FLAG_HOST_MAPPED):
                            //    polled with a system-scope load (a gpu-scope load is not
                            //    guaranteed to observe a CPU store)
+  uint32_t static_sched;   // 1: the static persistent twin (U1, flep_static): worker i takes chunks
+                           //    i, i + W, i + 2W, ... with no counter, no poll, no exit accounting
   void* partial;           // in-tile preemption (FLEP_KFLAG_IN_TILE, GEMM): W partial-tile records
                            // then W accumulator spill slots (layout: partial_bytes below), or nullptr
 #ifdef FLEP_TRACE
@@ -251,6 +253,7 @@ struct SchedState {
   bool have_seen = false;            // async poll: a copy of the control word is in flight
   bool stopping = false;             // a request named this SM; drain the held chunk
   bool first = true;                 // first step of this worker
+  uint32_t snext = 0xffffffffu;      // static twin (U1): the next chunk base of this worker
 };
 
 // pull_task. In the first epoch of a launch the counter hands out blocks after the W
@@ -297,7 +300,17 @@ __device__ __forceinline__ void note_exit_event(const WorkerParams& p, WorkerSha
 }
 
 __device__ __forceinline__ uint32_t next_chunk(const WorkerParams& p, SchedState& st, WorkerShared& ws,
-                                               uint32_t wid = blockIdx.x) {
+                                               uint32_t wid = blockIdx.x, uint32_t yield_sm = 0xffffffffu) {
+  // the SM whose rank a spatial request is checked against (a CTA pair passes its lower-ranked SM)
+  const auto my_sm = [&]() { return yield_sm != 0xffffffffu ? yield_sm : smid_reg(); };
+  if (p.static_sched) {              // U1 twin: a fixed schedule, nothing shared, never preempted
+    if (st.snext == 0xffffffffu) st.snext = wid * p.chunk;
+    const uint32_t b = st.snext;
+    st.snext += p.workers * p.chunk;
+    if (b >= p.n_blocks) { ws.reason = kReasonExhausted; return 0xffffffffu; }
+    ws.blocks += min(p.chunk, p.n_blocks - b);
+    return b;
+  }
   uint32_t base = 0xffffffffu;
   bool have = false;
   if (st.first) {
@@ -315,13 +328,13 @@ __device__ __forceinline__ uint32_t next_chunk(const WorkerParams& p, SchedState
       const uint32_t c = poll_ctrl(p);
       const uint32_t dg = ld_relaxed_gpu(&p.cb->done_gen);
       if (dg >= p.gen_first) { ws.reason = kReasonExhausted; return 0xffffffffu; }
-      if (should_yield(c, p, smid_reg())) { ws.reason = kReasonYield; return 0xffffffffu; }
+      if (should_yield(c, p, my_sm())) { ws.reason = kReasonYield; return 0xffffffffu; }
     }
   } else if (st.k == 0 && !st.stopping) {            // amortised poll (Fig. 4(b))
     // async poll (FLEP_KFLAG_ASYNC_POLL, reading R22): use the word loaded at the previous step,
     // so no round trip sits between two chunks; a request is then acted on one chunk later
     const uint32_t c = (p.async_poll && st.have_seen) ? poll_consume(ws) : poll_ctrl(p);
-    if (should_yield(c, p, smid_reg())) { st.stopping = true; ws.reason = kReasonYield; }
+    if (should_yield(c, p, my_sm())) { st.stopping = true; ws.reason = kReasonYield; }
   }
 #ifdef FLEP_TRACE
   ws.t_poll = gtimer();
@@ -778,6 +791,25 @@ flep_slice(const __grid_constant__ typename Body::Args args, uint32_t gx, uint32
   const uint32_t b = block_offset + blockIdx.x + gx * (blockIdx.y + gy * blockIdx.z);
   Body::setup(args);
   Body::run(args, b, b + 1, gx, gy);
+  Body::teardown(args);
+}
+
+// The static persistent twin (U1): W resident CTAs, CTA i runs chunks i, i + W, ...
+// of C original blocks with no counter, no poll and no exit accounting: the cost of persistence
+// alone, the baseline that separates it from the FLEP wrapper's own overhead.
+template <class Body>
+__global__ void __launch_bounds__(Body::kThreads, Body::kMinBlocks)
+flep_static(const __grid_constant__ typename Body::Args args, const WorkerParams p) {
+  __shared__ WorkerShared ws;
+  Body::setup(args);
+  if constexpr (Body::kPersistent) {
+    Body::persistent(args, p, ws);
+  } else {
+    for (uint32_t b0 = blockIdx.x * p.chunk; b0 < p.n_blocks; b0 += gridDim.x * p.chunk) {
+      Body::run(args, b0, min(b0 + p.chunk, p.n_blocks), p.gx, p.gy);
+      __syncthreads();               // the next chunk reuses the body's shared memory
+    }
+  }
   Body::teardown(args);
 }
 

@@ -74,6 +74,12 @@ cudaError_t gemm_unwrapped_launch(const void* user, dim3 grid, uint32_t offset, 
 
 cudaError_t gemm_occupancy(int* k, bool cov) { return occupancy_raw<GemmBody>(k, cov); }
 
+cudaError_t gemm_static_launch(const void* user, dim3 grid, uint32_t ctas, uint32_t chunk, cudaStream_t s) {
+  GemmArgsDev d;
+  if (!to_dev(user, &d)) return cudaErrorInvalidValue;
+  return launch_static_raw<GemmBody>(d, grid, ctas, chunk, s);
+}
+
 cudaError_t gemm_slice_launch(const void* user, dim3 grid, uint32_t offset, uint32_t count,
                                const SliceParams& sp, cudaStream_t s) {
   GemmArgsDev d;

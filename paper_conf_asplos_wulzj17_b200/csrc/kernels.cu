@@ -61,6 +61,18 @@ struct Ops {
     flep_slice<Body><<<count, Body::kThreads, Body::kDynSmem, s>>>(a, grid.x, grid.y, offset, sp);
     return cudaGetLastError();
   }
+  static cudaError_t static_launch(const void* args, dim3 grid, uint32_t ctas, uint32_t chunk, cudaStream_t s) {
+    const typename Body::Args& a = *reinterpret_cast<const typename Body::Args*>(args);
+    WorkerParams p{};
+    p.static_sched = 1u;
+    p.n_blocks = grid.x * grid.y * grid.z;
+    p.chunk = chunk ? chunk : 1u;
+    p.workers = ctas;
+    p.gx = grid.x;
+    p.gy = grid.y;
+    flep_static<Body><<<ctas, Body::kThreads, Body::kDynSmem, s>>>(a, p);
+    return cudaGetLastError();
+  }
   static cudaError_t occupancy(int* k, bool cov) {
     cudaError_t e;
     if (Body::kDynSmem > 48 * 1024) {
@@ -139,6 +151,23 @@ cudaError_t launch_slice_raw(const typename Body::Args& a, dim3 grid, uint32_t o
   return cudaGetLastError();
 }
 template <class Body>
+cudaError_t launch_static_raw(const typename Body::Args& a, dim3 grid, uint32_t ctas, uint32_t chunk, cudaStream_t s) {
+  const size_t sm = smem_for<Body>(chunk ? chunk : 1u);
+  if (sm > 48 * 1024) {
+    cudaError_t e = cudaFuncSetAttribute(flep_static<Body>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    if (e) return e;
+  }
+  WorkerParams p{};
+  p.static_sched = 1u;
+  p.n_blocks = grid.x * grid.y * grid.z;
+  p.chunk = chunk ? chunk : 1u;
+  p.workers = ctas;
+  p.gx = grid.x;
+  p.gy = grid.y;
+  flep_static<Body><<<ctas, Body::kThreads, sm, s>>>(a, p);
+  return cudaGetLastError();
+}
+template <class Body>
 cudaError_t launch_clc_raw(const typename Body::Args& a, const WorkerParams& p, uint32_t N, cudaStream_t s, bool cov) {
   const size_t sm = smem_for<Body>(p.chunk);
   if (cov) flep_clc_worker<Body, true><<<N, Body::kThreads, sm, s>>>(a, p);
@@ -152,6 +181,7 @@ template cudaError_t occupancy_raw<Stencil5TmaBody>(int*, bool);
 template cudaError_t launch_worker_raw<GemmBody>(const GemmBody::Args&, const WorkerParams&, uint32_t, cudaStream_t, bool);
 template cudaError_t launch_unwrapped_raw<GemmBody>(const GemmBody::Args&, dim3, uint32_t, uint32_t, cudaStream_t);
 template cudaError_t occupancy_raw<GemmBody>(int*, bool);
+template cudaError_t launch_static_raw<GemmBody>(const GemmBody::Args&, dim3, uint32_t, uint32_t, cudaStream_t);
 template cudaError_t launch_slice_raw<GemmBody>(const GemmBody::Args&, dim3, uint32_t, uint32_t, const SliceParams&, cudaStream_t);
 template cudaError_t launch_slice_raw<Stencil5TmaBody>(const Stencil5TmaBody::Args&, dim3, uint32_t, uint32_t, const SliceParams&, cudaStream_t);
 
@@ -168,31 +198,34 @@ const BodyOps kOps[] = {
     {0, 0, 0, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr},
     {FLEP_BODY_SAXPY_I32, SaxpyI32::kThreads, sizeof(flep_saxpy_i32_args), &Ops<SaxpyI32>::worker,
      &Ops<SaxpyI32>::unwrapped, &Ops<SaxpyI32>::occupancy, nullptr, &Ops<SaxpyI32>::clc,
-     &Ops<SaxpyI32>::worker_sw, &Ops<SaxpyI32>::occupancy_sw, nullptr, nullptr, 0, &Ops<SaxpyI32>::sliced},
+     &Ops<SaxpyI32>::worker_sw, &Ops<SaxpyI32>::occupancy_sw, nullptr, nullptr, 0, &Ops<SaxpyI32>::sliced, &Ops<SaxpyI32>::static_launch, nullptr},
     {FLEP_BODY_SAXPY_F32, SaxpyF32::kThreads, sizeof(flep_saxpy_f32_args), &Ops<SaxpyF32>::worker,
      &Ops<SaxpyF32>::unwrapped, &Ops<SaxpyF32>::occupancy, nullptr, &Ops<SaxpyF32>::clc,
-     &Ops<SaxpyF32>::worker_sw, &Ops<SaxpyF32>::occupancy_sw, nullptr, nullptr, 0, &Ops<SaxpyF32>::sliced},
+     &Ops<SaxpyF32>::worker_sw, &Ops<SaxpyF32>::occupancy_sw, nullptr, nullptr, 0, &Ops<SaxpyF32>::sliced, &Ops<SaxpyF32>::static_launch, nullptr},
     {FLEP_BODY_SPMV_CSR_F32, Spmv::kThreads, sizeof(flep_spmv_args), &Ops<Spmv>::worker,
      &Ops<Spmv>::unwrapped, &Ops<Spmv>::occupancy, nullptr, &Ops<Spmv>::clc,
-     &Ops<Spmv>::worker_sw, &Ops<Spmv>::occupancy_sw, nullptr, nullptr, 0, &Ops<Spmv>::sliced},
+     &Ops<Spmv>::worker_sw, &Ops<Spmv>::occupancy_sw, nullptr, nullptr, 0, &Ops<Spmv>::sliced, &Ops<Spmv>::static_launch, nullptr},
     {FLEP_BODY_STENCIL5_F32, StencilF32::kThreads, sizeof(flep_stencil_args), &Ops<StencilF32>::worker,
      &Ops<StencilF32>::unwrapped, &Ops<StencilF32>::occupancy, nullptr, &Ops<StencilF32>::clc,
      &Ops<StencilF32>::worker_sw, &Ops<StencilF32>::occupancy_sw, &Ops<StencilF32>::warp_worker,
-     &Ops<StencilF32>::occupancy_warp, StencilF32::kWarpTasks, &Ops<StencilF32>::sliced},
+     &Ops<StencilF32>::occupancy_warp, StencilF32::kWarpTasks, &Ops<StencilF32>::sliced, &Ops<StencilF32>::static_launch, nullptr},
     {FLEP_BODY_STENCIL5_I32, StencilI32::kThreads, sizeof(flep_stencil_args), &Ops<StencilI32>::worker,
      &Ops<StencilI32>::unwrapped, &Ops<StencilI32>::occupancy, nullptr, &Ops<StencilI32>::clc,
      &Ops<StencilI32>::worker_sw, &Ops<StencilI32>::occupancy_sw, &Ops<StencilI32>::warp_worker,
-     &Ops<StencilI32>::occupancy_warp, StencilI32::kWarpTasks, &Ops<StencilI32>::sliced},
+     &Ops<StencilI32>::occupancy_warp, StencilI32::kWarpTasks, &Ops<StencilI32>::sliced, &Ops<StencilI32>::static_launch, nullptr},
     {FLEP_BODY_GEMM_BF16, GemmBody::kThreads, sizeof(flep_gemm_args), &gemm_worker_launch,
      &gemm_unwrapped_launch, &gemm_occupancy, &gemm_validate, nullptr, nullptr, nullptr, nullptr, nullptr, 0,
-     &gemm_slice_launch},
+     &gemm_slice_launch, &gemm_static_launch, nullptr},
     {FLEP_BODY_STENCIL5_F32_TMA, Stencil5TmaBody::kThreads, sizeof(flep_stencil_args), &stencil_tma_worker_launch,
      &stencil_tma_unwrapped_launch, &stencil_tma_occupancy, &stencil_tma_validate, &stencil_tma_clc_launch,
      nullptr, nullptr, nullptr, nullptr, 0, &stencil_tma_slice_launch},
     {FLEP_BODY_SPMV_CSR_F32_VEC, SpmvVec::kThreads, sizeof(flep_spmv_args), &Ops<SpmvVec>::worker,
      &Ops<SpmvVec>::unwrapped, &Ops<SpmvVec>::occupancy, nullptr, &Ops<SpmvVec>::clc,
      &Ops<SpmvVec>::worker_sw, &Ops<SpmvVec>::occupancy_sw, &Ops<SpmvVec>::warp_worker,
-     &Ops<SpmvVec>::occupancy_warp, SpmvVec::kWarpTasks, &Ops<SpmvVec>::sliced},
+     &Ops<SpmvVec>::occupancy_warp, SpmvVec::kWarpTasks, &Ops<SpmvVec>::sliced, &Ops<SpmvVec>::static_launch, nullptr},
+    {FLEP_BODY_GEMM_BF16_2SM, 256 /* Gemm2::kThreads (gemm2_tcgen05.cuh, its own TU) */, sizeof(flep_gemm_args), &gemm2_worker_launch,
+     &gemm2_unwrapped_launch, &gemm2_occupancy, &gemm2_validate, nullptr, nullptr, nullptr, nullptr, nullptr, 0,
+     nullptr, &gemm2_static_launch, &gemm2_max_pairs},
 };
 
 }  // namespace
@@ -204,7 +237,7 @@ cudaError_t set_unwrapped_trace(uint64_t* p) {
 #endif
 
 const BodyOps* body_ops(int32_t body) {
-  if (body < 1 || body > FLEP_BODY_SPMV_CSR_F32_VEC) return nullptr;
+  if (body < 1 || body > FLEP_BODY_GEMM_BF16_2SM) return nullptr;
   return &kOps[body];
 }
 

@@ -35,10 +35,21 @@ struct BodyOps {
   // kernel slicing with the device check (flep_slice<Body>, R31): blocks [offset, offset+count)
   cudaError_t (*sliced)(const void* args, dim3 grid, uint32_t offset, uint32_t count, const SliceParams& sp,
                         cudaStream_t s);
+  // the static persistent twin (flep_static<Body>, U1): `ctas` resident CTAs, chunks of C blocks
+  cudaError_t (*static_launch)(const void* args, dim3 grid, uint32_t ctas, uint32_t chunk, cudaStream_t s);
+  // CTA-pair bodies (R32): the worker is a cluster of 2 CTAs; max resident pairs
+  cudaError_t (*max_pairs)(int* pairs, bool cov);
 };
 
 const BodyOps* body_ops(int32_t body);
-// GEMM body (gemm_tcgen05.cu)
+// GEMM bodies (gemm_tcgen05.cu, gemm2_tcgen05.cu)
+cudaError_t gemm_static_launch(const void* user, dim3 grid, uint32_t ctas, uint32_t chunk, cudaStream_t s);
+cudaError_t gemm2_worker_launch(const void* user, const WorkerParams& p, uint32_t ctas, cudaStream_t s, bool cov);
+cudaError_t gemm2_unwrapped_launch(const void* user, dim3 grid, uint32_t offset, uint32_t count, cudaStream_t s);
+cudaError_t gemm2_static_launch(const void* user, dim3 grid, uint32_t ctas, uint32_t chunk, cudaStream_t s);
+cudaError_t gemm2_occupancy(int* k, bool cov);
+cudaError_t gemm2_max_pairs(int* pairs, bool cov);
+const char* gemm2_validate(const void* user, dim3 grid);
 cudaError_t gemm_slice_launch(const void* user, dim3 grid, uint32_t offset, uint32_t count,
                               const SliceParams& sp, cudaStream_t s);
 #ifdef FLEP_TRACE
@@ -51,6 +62,8 @@ template <class Body>
 cudaError_t launch_unwrapped_raw(const typename Body::Args& a, dim3 grid, uint32_t offset, uint32_t count, cudaStream_t s);
 template <class Body>
 cudaError_t occupancy_raw(int* k, bool cov);
+template <class Body>
+cudaError_t launch_static_raw(const typename Body::Args& a, dim3 grid, uint32_t ctas, uint32_t chunk, cudaStream_t s);
 template <class Body>
 cudaError_t launch_slice_raw(const typename Body::Args& a, dim3 grid, uint32_t offset, uint32_t count,
                              const SliceParams& sp, cudaStream_t s);

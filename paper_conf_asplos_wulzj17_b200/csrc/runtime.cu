@@ -465,6 +465,7 @@ flep_status start_epoch(flep_rt rt, Launch& L) {
   cudaError_t e = L.clc ? L.ops->clc(L.args.data(), p, (L.n_blocks + L.chunk - 1) / L.chunk, L.exec, L.cov != nullptr)
                  : L.sw ? L.ops->worker_sw(L.args.data(), p, L.workers, L.exec, L.cov != nullptr)
                  : L.warp ? L.ops->warp_worker(L.args.data(), p, L.ctas + (L.relay ? 1u : 0u), L.exec, L.cov != nullptr)
+                 : L.ops->max_pairs ? L.ops->worker(L.args.data(), p, L.ctas, L.exec, L.cov != nullptr)
                         : L.ops->worker(L.args.data(), p, L.workers + (L.relay ? 1u : 0u), L.exec, L.cov != nullptr);
   if (e != cudaSuccess) return fail(FLEP_ERR_CUDA, "worker launch failed: %s", cudaGetErrorString(e));
   CUDA_TRY(cudaEventRecord(L.fin_ev, L.exec));
@@ -946,6 +947,11 @@ flep_status flep_workers_for(flep_rt rt, int32_t body, uint32_t* ctas_per_sm, ui
   if (s) return s;
   if (ctas_per_sm) *ctas_per_sm = (uint32_t)k;
   if (workers) *workers = (uint32_t)k * rt->num_sms;
+  if (ops->max_pairs && workers) {                    // R32: workers are CTA pairs
+    int pairs = 0;
+    CUDA_TRY(ops->max_pairs(&pairs, rt->opt.debug_coverage & 1u));
+    *workers = (uint32_t)pairs;
+  }
   return FLEP_OK;
 }
 
@@ -1011,7 +1017,15 @@ flep_status flep_launch(flep_rt rt, flep_kernel kid, flep_dim3 grid, const void*
   // R28: the relay CTA takes one resident slot (plain counter worker, stream-memop transport)
   L.relay = (kr.flags & FLEP_KFLAG_HOST_RELAY) && !L.sw && !L.clc && !ops->validate &&
             rt->opt.flag != FLEP_FLAG_HOST_MAPPED && wmax > 1;
-  if (warp) {
+  if (ops->max_pairs) {
+    // R32: CTA-pair body: the worker is a cluster of 2 CTAs
+    int pairs = 0;
+    CUDA_TRY(ops->max_pairs(&pairs, cov));
+    if (pairs <= 0) return fail(FLEP_ERR_UNSUPPORTED, "body %d: no CTA pair can be resident", kr.body);
+    L.workers = (uint32_t)std::min<uint64_t>((uint64_t)pairs, need);
+    L.ctas = 2 * L.workers;
+    L.relay = false;
+  } else if (warp) {
     // R30: worker CTAs of threads/32 warp workers each
     const uint64_t wpc = (uint64_t)ops->threads / 32u;
     const uint64_t g_need = (need + wpc - 1) / wpc;
@@ -1025,6 +1039,7 @@ flep_status flep_launch(flep_rt rt, flep_kernel kid, flep_dim3 grid, const void*
     // SMs that host every CTA of this launch (A9: n = ceil(grid / k)): the workers
     // (+ the relay CTA), or the CLC grid's resident part
     const uint64_t ctas = L.clc ? std::min<uint64_t>(need, wmax) : (uint64_t)L.ctas + (L.relay ? 1u : 0u);
+    // (a CTA-pair body: ctas = 2 x pairs, one CTA per SM)
     L.sms_need = (int64_t)std::min<uint64_t>(rt->num_sms, (ctas + (uint64_t)k - 1) / (uint64_t)k);
   }
   if (slicing) {
@@ -1322,6 +1337,36 @@ flep_status flep_launch_unwrapped(flep_rt rt, int32_t body, flep_dim3 grid, cons
   if (ops->validate) { const char* m = ops->validate(args, g); if (m) return fail(FLEP_ERR_INVALID, "%s", m); }
   { int k; ApiLock lk(rt); s = occupancy(rt, ops, false, &k); if (s) return s; }
   CUDA_TRY(ops->unwrapped(args, g, 0, 0, (cudaStream_t)stream));
+  return FLEP_OK;
+}
+
+flep_status flep_launch_static(flep_rt rt, int32_t body, flep_dim3 grid, const void* args,
+                               size_t args_size, uint32_t chunk, flep_stream_t stream) {
+  if (!rt || !args) return fail(FLEP_ERR_INVALID, "NULL argument");
+  const BodyOps* ops = body_ops(body);
+  if (!ops) return fail(FLEP_ERR_INVALID, "unknown body %d", body);
+  if (!ops->static_launch) return fail(FLEP_ERR_UNSUPPORTED, "body %d has no static persistent twin", body);
+  if (args_size != ops->args_size) return fail(FLEP_ERR_INVALID, "args_size mismatch");
+  uint64_t N = 0;
+  flep_status s = validate_grid(grid, &N);
+  if (s) return s;
+  dim3 g(grid.x, grid.y, grid.z);
+  if (ops->validate) { const char* m = ops->validate(args, g); if (m) return fail(FLEP_ERR_INVALID, "%s", m); }
+  uint32_t ctas = 0;
+  {
+    ApiLock lk(rt);
+    int k = 0;
+    s = occupancy(rt, ops, false, &k);
+    if (s) return s;
+    if (ops->max_pairs) {
+      int pairs = 0;
+      CUDA_TRY(ops->max_pairs(&pairs, false));
+      ctas = 2u * (uint32_t)std::max(pairs, 1);
+    } else {
+      ctas = (uint32_t)k * rt->num_sms;
+    }
+  }
+  CUDA_TRY(ops->static_launch(args, g, ctas, chunk ? chunk : 1u, (cudaStream_t)stream));
   return FLEP_OK;
 }
 

@@ -19,6 +19,7 @@ FLAG_STREAM_MEMOP, FLAG_HOST_MAPPED = 0, 1
 BODY_SAXPY_I32, BODY_SAXPY_F32, BODY_SPMV_CSR_F32, BODY_STENCIL5_F32, BODY_STENCIL5_I32, BODY_GEMM_BF16 = 1, 2, 3, 4, 5, 6
 BODY_STENCIL5_F32_TMA = 7
 BODY_SPMV_CSR_F32_VEC = 8
+BODY_GEMM_BF16_2SM = 9
 STATE_QUEUED, STATE_RUNNING, STATE_YIELDING, STATE_PREEMPTED, STATE_PARTIAL, STATE_DONE = 0, 1, 2, 3, 4, 5
 STATE_NAMES = {0: "QUEUED", 1: "RUNNING", 2: "YIELDING", 3: "PREEMPTED", 4: "PARTIAL", 5: "DONE"}
 REASON_YIELD, REASON_EXHAUSTED = 1, 2
@@ -97,7 +98,7 @@ class EpochInfo(C.Structure):
 
 ARGS_FOR_BODY = {BODY_SAXPY_I32: SaxpyI32Args, BODY_SAXPY_F32: SaxpyF32Args, BODY_SPMV_CSR_F32: SpmvArgs,
                  BODY_STENCIL5_F32: StencilArgs, BODY_STENCIL5_I32: StencilArgs, BODY_GEMM_BF16: GemmArgs,
-                 BODY_STENCIL5_F32_TMA: StencilArgs, BODY_SPMV_CSR_F32_VEC: SpmvArgs}
+                 BODY_STENCIL5_F32_TMA: StencilArgs, BODY_SPMV_CSR_F32_VEC: SpmvArgs, BODY_GEMM_BF16_2SM: GemmArgs}
 
 # exported symbols: name -> (restype, argtypes)
 _P = C.c_void_p
@@ -116,6 +117,7 @@ _SIG = {
     "flep_wait_epoch": (C.c_int, [_P, C.c_int64, C.c_int64]),
     "flep_launch_unwrapped": (C.c_int, [_P, C.c_int32, Dim3, _P, C.c_size_t, _P]),
     "flep_launch_sliced": (C.c_int, [_P, C.c_int32, Dim3, _P, C.c_size_t, C.c_uint32, _P]),
+    "flep_launch_static": (C.c_int, [_P, C.c_int32, Dim3, _P, C.c_size_t, C.c_uint32, _P]),
     "flep_workers_for": (C.c_int, [_P, C.c_int32, C.POINTER(C.c_uint32), C.POINTER(C.c_uint32)]),
     "flep_debug_trigger_at": (C.c_int, [_P, C.c_int64, C.c_uint64, C.c_uint32]),
     "flep_debug_arm_next_trigger": (C.c_int, [_P, C.c_uint64, C.c_uint32]),
@@ -268,6 +270,10 @@ class Runtime:
     def launch_sliced(self, body, grid, args, slice_blocks, stream=None):
         check(self.L.flep_launch_sliced(self.h, body, dim3(grid), C.byref(args), C.sizeof(args),
                                         slice_blocks, _stream_ptr(stream)), "flep_launch_sliced")
+
+    def launch_static(self, body, grid, args, chunk=1, stream=None):
+        check(self.L.flep_launch_static(self.h, body, dim3(grid), C.byref(args), C.sizeof(args), chunk,
+                                        _stream_ptr(stream)), "flep_launch_static")
 
     def workers_for(self, body):
         k, w = C.c_uint32(), C.c_uint32()
@@ -424,3 +430,8 @@ def stencil_grid(n):
 
 def gemm_grid(m, n):
     return (n // 256, m // 128, 1)
+
+
+def gemm2_grid(m, n):
+    """Original grid of the CTA-pair GEMM body: one 256x256 tile per block."""
+    return (n // 256, m // 256, 1)

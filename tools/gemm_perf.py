@@ -1,0 +1,70 @@
+"""GEMM 8192^3 (configs[3]'s largest): cuBLAS (torch.matmul) vs the 1-CTA body (unwrapped,
+static persistent U1, FLEP worker) vs the CTA-pair body (unwrapped, U1, FLEP worker), interleaved
+round-robin, CUDA events, clocks sampled during the run. One JSON line per variant."""
+import json
+import os
+import sys
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+
+def main():
+    import torch
+    from paper_conf_asplos_wulzj17_b200 import build, flep as F
+    from bench import ClockSampler
+    build.build()
+    M = int(os.environ.get("GEMM_M", "8192"))
+    reps = int(os.environ.get("GEMM_REPS", "12"))
+    g = torch.Generator(device="cuda")
+    g.manual_seed(5)
+    A = (torch.rand(M, M, device="cuda", generator=g) * 2 - 1).to(torch.bfloat16)
+    B = (torch.rand(M, M, device="cuda", generator=g) * 2 - 1).to(torch.bfloat16)
+    C = torch.empty(M, M, device="cuda", dtype=torch.bfloat16)
+    rt = F.Runtime(exec_on_user_stream=True)
+    s = torch.cuda.current_stream()
+    args = F.gemm_args(C, A, B)
+    g1, g2 = F.gemm_grid(M, M), F.gemm2_grid(M, M)
+    k1 = {c: rt.register_kernel(F.BODY_GEMM_BF16, chunk=c, poll=1) for c in (1, 2)}
+    k1t = rt.register_kernel(F.BODY_GEMM_BF16, chunk=2, poll=1, in_tile=True)
+    k2 = {c: rt.register_kernel(F.BODY_GEMM_BF16_2SM, chunk=c, poll=1) for c in (1, 2)}
+    variants = {
+        "cublas": lambda: (torch.matmul(A, B.t(), out=C), None)[1],
+        "gemm1_unwrapped": lambda: rt.launch_unwrapped(F.BODY_GEMM_BF16, g1, args, stream=s),
+        "gemm1_static_u1": lambda: rt.launch_static(F.BODY_GEMM_BF16, g1, args, chunk=1, stream=s),
+        "gemm1_flep_c1": lambda: rt.launch(k1[1], g1, args, stream=s),
+        "gemm1_flep_c2": lambda: rt.launch(k1[2], g1, args, stream=s),
+        "gemm1_flep_c2_intile": lambda: rt.launch(k1t, g1, args, stream=s),
+        "gemm2_unwrapped": lambda: rt.launch_unwrapped(F.BODY_GEMM_BF16_2SM, g2, args, stream=s),
+        "gemm2_static_u1": lambda: rt.launch_static(F.BODY_GEMM_BF16_2SM, g2, args, stream=s),
+        "gemm2_flep_c1": lambda: rt.launch(k2[1], g2, args, stream=s),
+        "gemm2_flep_c2": lambda: rt.launch(k2[2], g2, args, stream=s),
+    }
+    ts = {k: [] for k in variants}
+    with ClockSampler(0) as clk:
+        for r in range(reps + 2):
+            for name, fn in variants.items():
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record(s)
+                h = fn()
+                e1.record(s)
+                e1.synchronize()
+                if isinstance(h, int):
+                    rt.sync(h)
+                if r >= 2:
+                    ts[name].append(e0.elapsed_time(e1) * 1e3)
+    clocks = clk.summary()
+    flop = 2.0 * M ** 3
+    cub = float(np.median(ts["cublas"]))
+    for name, v in ts.items():
+        us = float(np.median(v))
+        print(json.dumps({"gemm": f"{M}^3 bf16", "variant": name, "us_p50": round(us, 2), "us_min": round(min(v), 2),
+                          "tflops": round(flop / us / 1e6, 1), "vs_cublas": round(cub / us, 3), "clocks": clocks}),
+              flush=True)
+    rt.close()
+
+
+if __name__ == "__main__":
+    main()
