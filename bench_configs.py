@@ -1459,7 +1459,7 @@ def run_slicing_overhead(args, rank, world, local):
             k_s = rt_s.register_kernel(body, chunk=C, poll=1)
             cps, w = rt_m.workers_for(body)
             slice_blocks = w * C                                     # one wave of W*C*K blocks (A20)
-            t = {m: [] for m in ("unwrapped", "flep_tuned", "flep_c1", "slice_device", "slice_plain")}
+            t = {m: [] for m in ("unwrapped", "static_u1", "flep_tuned", "flep_c1", "slice_device", "slice_plain")}
             for r in range(reps + 2):
                 for m in t:
                     with torch.cuda.stream(S):
@@ -1470,6 +1470,8 @@ def run_slicing_overhead(args, rank, world, local):
                     h = None
                     if m == "unwrapped":
                         rt_m.launch_unwrapped(body, grid, a, stream=S)
+                    elif m == "static_u1":
+                        rt_m.launch_static(body, grid, a, chunk=C, stream=S)
                     elif m == "flep_tuned":
                         h = (rt_m, rt_m.launch(k_t, grid, a, stream=S))
                     elif m == "flep_c1":
@@ -1488,12 +1490,48 @@ def run_slicing_overhead(args, rank, world, local):
             nb = grid[0] * grid[1]
             row = {"kernel": f"{key[0]}-{key[1]}", "blocks": nb, "slice_blocks": slice_blocks,
                    "slices": -(-nb // slice_blocks), "unwrapped_us": round(u, 2)}
-            for m in ("flep_tuned", "flep_c1", "slice_device", "slice_plain"):
+            for m in ("static_u1", "flep_tuned", "flep_c1", "slice_device", "slice_plain"):
                 v = event_mean_us(t[m])
                 row[m + "_us"] = round(v, 2)
                 row[m + "_overhead_pct"] = round((v / u - 1) * 100, 2)
+            row["flep_tuned_over_static_pct"] = round((row["flep_tuned_us"] / row["static_u1_us"] - 1) * 100, 2)
             row["tuned_chunk"] = C
             rows.append(row)
+        # the CTA-pair GEMM (R32) at the largest size: cuBLAS, unwrapped, U1 and the FLEP pair
+        # workers, interleaved
+        A8, B8, C8 = inst[("gemm_bf16", 2)][3]
+        a8 = F.gemm_args(C8, A8, B8)
+        g2 = F.gemm2_grid(C8.shape[0], C8.shape[1])
+        k2 = {c: rt_m.register_kernel(F.BODY_GEMM_BF16_2SM, chunk=c, poll=1) for c in (1, 2)}
+        tg = {m: [] for m in ("cublas", "unwrapped", "static_u1", "flep_c1", "flep_c2")}
+        for r in range(max(6, reps // 2) + 2):
+            for m in tg:
+                with torch.cuda.stream(S):
+                    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                    e0.record(S)
+                    h = None
+                    if m == "cublas":
+                        torch.matmul(A8, B8.t(), out=C8)
+                    elif m == "unwrapped":
+                        rt_m.launch_unwrapped(F.BODY_GEMM_BF16_2SM, g2, a8, stream=S)
+                    elif m == "static_u1":
+                        rt_m.launch_static(F.BODY_GEMM_BF16_2SM, g2, a8, stream=S)
+                    else:
+                        h = rt_m.launch(k2[1 if m == "flep_c1" else 2], g2, a8, stream=S)
+                    e1.record(S)
+                e1.synchronize()
+                if h is not None:
+                    rt_m.sync(h)
+                if r >= 2:
+                    tg[m].append(e0.elapsed_time(e1) * 1e3)
+        gm = {m: float(np.median(v)) for m, v in tg.items()}
+        flop = 2.0 * C8.shape[0] * C8.shape[1] * A8.shape[1]
+        gemm2 = {"size": f"{C8.shape[0]}x{C8.shape[1]}x{A8.shape[1]} bf16", "stat": "median, interleaved",
+                 **{m + "_us": round(v, 2) for m, v in gm.items()},
+                 **{m + "_tflops": round(flop / v / 1e6, 1) for m, v in gm.items()},
+                 "flep_c2_vs_cublas": round(gm["cublas"] / gm["flep_c2"], 3),
+                 "flep_c2_over_static_pct": round((gm["flep_c2"] / gm["static_u1"] - 1) * 100, 2),
+                 "flep_c1_over_static_pct": round((gm["flep_c1"] / gm["static_u1"] - 1) * 100, 2)}
     rt_m.close()
     rt_s.close()
     big = [r for r in rows if r["kernel"].endswith("-2")]
@@ -1504,10 +1542,10 @@ def run_slicing_overhead(args, rank, world, local):
            "dtype": "mixed", "data": "synthetic (seeded)",
            "config": {"workload": "E13: the configs[3] queue's 12 kernel instances run alone, never preempted",
                       "reps": reps, "l2": "flushed between samples"},
-           "mean_overhead_pct": {k: mean(k + "_overhead_pct", rows) for k in ("flep_tuned", "flep_c1", "slice_device", "slice_plain")},
-           "mean_overhead_pct_large": {k: mean(k + "_overhead_pct", big) for k in ("flep_tuned", "flep_c1", "slice_device", "slice_plain")},
+           "mean_overhead_pct": {k: mean(k + "_overhead_pct", rows) for k in ("static_u1", "flep_tuned", "flep_c1", "slice_device", "slice_plain")},
+           "mean_overhead_pct_large": {k: mean(k + "_overhead_pct", big) for k in ("static_u1", "flep_tuned", "flep_c1", "slice_device", "slice_plain")},
            "paper": "FLEP 2.5 % vs kernel slicing 8 % at the same preemption granularity (P:391, K40)",
-           "kernels": rows, "clocks": clk.summary()}
+           "kernels": rows, "gemm_2sm_8192": gemm2, "clocks": clk.summary()}
     _emit(out, rank, args)
     barrier(world)
     return out
