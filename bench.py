@@ -118,11 +118,17 @@ def dist_setup(dry_run=False):
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    # FLEP_SHARE_GPU=1 (functional test of the N > 1 path on a one-GPU box): every rank uses the
+    # visible GPUs round-robin and the process group runs on gloo (NCCL refuses a shared GPU);
+    # the numbers of such a run are not scaling measurements
+    share = os.environ.get("FLEP_SHARE_GPU") == "1"
     if world > 1:
         import torch
         import torch.distributed as dist
+        if share and torch.cuda.is_available():
+            local = local % max(1, torch.cuda.device_count())
         if not dist.is_initialized():
-            if dry_run or not torch.cuda.is_available():
+            if dry_run or share or not torch.cuda.is_available():
                 dist.init_process_group("gloo")
             else:
                 torch.cuda.set_device(local)
