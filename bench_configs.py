@@ -344,8 +344,25 @@ def run_corun1(args, rank, world, local):
     B = torch.cuda.Stream(priority=0)
     nb = n_lp // 256
     rng = gen.rng(3000 + rank)
-    lat, drain, hpt, bad, pre = [], [], [], 0, 0
+    lat, drain, hpt, bad, pre, hpt_fifo = [], [], [], 0, 0, []
     with ClockSampler(physical_gpu_index(local)) as clk:
+        # FIFO reference (no preemption): the same arrival point is only stamped (trigger width 0),
+        # the HP kernel waits behind the persistent LP workers
+        for i in range(args.warmup + args.steps):
+            yd.copy_(y0)
+            y2d.copy_(y20)
+            flush.zero_()
+            torch.cuda.synchronize()
+            tstar = int(rng.integers(nb // 4, 3 * nb // 4))
+            rt.arm_next_trigger(tstar, 0)
+            h = rt.launch(k_lp, F.saxpy_grid(n_lp), F.saxpy_i32_args(yd, xd, a_lp), priority=0, stream=A)
+            h2 = rt.launch(k_hp, F.saxpy_grid(n_hp), F.saxpy_i32_args(y2d, x2d, a_hp), priority=1, stream=B)
+            rt.sync(h, timeout_ns=10_000_000_000)
+            rt.sync(h2, timeout_ns=10_000_000_000)
+            ep = rt.epoch_info(h, 1)
+            if i >= args.warmup and ep.t_trigger:
+                hpt_fifo.append((_span(rt.events(h2, 1))[1] - ep.t_trigger) / 1e3)
+        rng = gen.rng(3000 + rank)
         for i in range(args.warmup + args.steps):
             yd.copy_(y0)
             y2d.copy_(y20)
@@ -384,6 +401,9 @@ def run_corun1(args, rank, world, local):
            "preempted_steps": pre, "wrong_results": bad,
            "waiting_start_us_p50": round(float(np.median(lat)), 3) if lat else None,
            "hp_turnaround_us_p50": round(float(np.median(hpt)), 3) if hpt else None,
+           "hp_turnaround_fifo_us_p50": round(float(np.median(hpt_fifo)), 3) if hpt_fifo else None,
+           "hp_speedup_vs_fifo": (round(float(np.median(hpt_fifo)) / float(np.median(hpt)), 2)
+                                  if hpt and hpt_fifo else None),
            "drain_us_max": round(float(np.max(drain)), 3) if drain else None,
            "clocks": clk.summary()}
     _emit(out, rank, args)
