@@ -84,8 +84,46 @@ def main():
     if rt.query(h).state == F.STATE_PREEMPTED:
         rt.resume(h)
     rt.sync(h)
+    # round 2: warp-task workers (SpMV vector body, stencil) with a temporal preempt/resume cycle,
+    # the static persistent twin, the CTA-pair GEMM (unwrapped, static, worker with a preemption)
+    # and device-checked slicing with a preemption
+    k9 = rt.register_kernel(F.BODY_SPMV_CSR_F32_VEC, chunk=2, poll=1, warp_tasks=True)
+    rt.arm_next_trigger(4, rt.num_sms)
+    h = rt.launch(k9, F.spmv_grid(2000), F.spmv_args(yv, *keep))
+    rt.wait_epoch(h)
+    if rt.query(h).state == F.STATE_PREEMPTED:
+        rt.resume(h)
+    rt.sync(h)
+    k10 = rt.register_kernel(F.BODY_STENCIL5_F32, chunk=1, poll=1, warp_tasks=True)
+    rt.sync(rt.launch(k10, F.stencil_grid(200), F.stencil_args(out, st)))
+    rt.launch_static(F.BODY_SPMV_CSR_F32, F.spmv_grid(2000), F.spmv_args(yv, *keep), chunk=2)
+    a_bits, b_bits = gen.gemm_bf16_inputs(512, 512, 256, 8)
+    A2 = torch.from_numpy(a_bits.view(np.int16)).cuda().view(torch.bfloat16)
+    B2 = torch.from_numpy(b_bits.view(np.int16)).cuda().view(torch.bfloat16)
+    C2 = torch.empty(512, 512, dtype=torch.bfloat16, device="cuda")
+    g2 = F.gemm2_grid(512, 512)
+    rt.launch_unwrapped(F.BODY_GEMM_BF16_2SM, g2, F.gemm_args(C2, A2, B2))
+    rt.launch_static(F.BODY_GEMM_BF16_2SM, g2, F.gemm_args(C2, A2, B2))
+    k11 = rt.register_kernel(F.BODY_GEMM_BF16_2SM, chunk=1, poll=1)
+    rt.arm_next_trigger(1, rt.num_sms)
+    h = rt.launch(k11, g2, F.gemm_args(C2, A2, B2))
+    rt.wait_epoch(h)
+    if rt.query(h).state == F.STATE_PREEMPTED:
+        rt.resume(h)
+    rt.sync(h)
     torch.cuda.synchronize()
     rt.close()
+    rs = F.Runtime(policy=F.POLICY_SLICE_DEVICE, slice_blocks=8)
+    kl = rs.register_kernel(F.BODY_SAXPY_I32, chunk=1, poll=1, model=(0, 0, 0, 0, 1_000_000))
+    kh = rs.register_kernel(F.BODY_SAXPY_I32, chunk=1, poll=1, model=(0, 0, 0, 0, 1_000))
+    x3, y3 = gen.saxpy_i32_inputs(256, 3)
+    x3d, y3d = T(x3), T(y3)
+    h1 = rs.launch(kl, F.saxpy_grid(n), F.saxpy_i32_args(yd, xd, 3), priority=0)
+    h2 = rs.launch(kh, F.saxpy_grid(256), F.saxpy_i32_args(y3d, x3d, 5), priority=1)
+    rs.sync(h2)
+    rs.sync(h1)
+    torch.cuda.synchronize()
+    rs.close()
     print("sanitizer case done")
 
 
