@@ -72,6 +72,19 @@ def run_spatial(args, rank, world, local):
         alone(k_v, v_grid, v_args)
     t_v = float(np.median([alone(k_v, v_grid, v_args) for _ in range(5)]))
     rng = gen.rng(2000 + rank)
+    check_rows = sorted(set(int(r) for r in gen.rng(2050 + rank).integers(1, n_st - 1, 6)))
+    slabs = {r: v_in[r - 1:r + 2].cpu().numpy() for r in check_rows}
+    import bench_check as BC
+
+    def victim_rows_err():
+        """Sampled output rows of the last victim run against NumPy fp64 (3-row slabs)."""
+        worst = 0.0
+        for r in check_rows:
+            ref, den = BC.stencil5_f32(slabs[r])
+            got = v_out[r].cpu().numpy()
+            d = np.maximum(np.abs(ref[1]), den[1])
+            worst = max(worst, float(np.max(np.abs(got - ref[1]) / np.where(d > 0, d, 1))))
+        return worst
     rows = []
     with ClockSampler(physical_gpu_index(local)) as clk:
         for n in widths:
@@ -125,7 +138,8 @@ def run_spatial(args, rank, world, local):
                 tflep.append((max(v1, w1) - v0) / 1e3)
                 ok += 1
             t_org = t_v + t_w
-            rows.append({"n_sms": n, "trials": ok, "yield_latency_us_p50": round(float(np.median(lat)), 3) if lat else None,
+            verr = victim_rows_err()
+            rows.append({"n_sms": n, "trials": ok, "victim_rows_max_rel": verr, "victim_parity_ok": bool(verr <= 1e-5), "yield_latency_us_p50": round(float(np.median(lat)), 3) if lat else None,
                          "yield_latency_us_max": round(float(np.max(lat)), 3) if lat else None,
                          "waiting_start_us_p50": round(float(np.median(start)), 3),
                          "t_flep_us": round(float(np.median(tflep)), 2), "t_org_us": round(t_org, 2),
@@ -156,6 +170,7 @@ def run_spatial(args, rank, world, local):
                                   "with n*k_wait blocks (waiting kernel) for n in {8,16,32,74} and 148 (temporal)",
                       "victim_chunk": 1, "poll": 1, "l2": "flushed between trials"},
            "per_width": rows,
+           "victim_parity_ok": all(r["victim_parity_ok"] for r in rows),
            "spatial_cheaper_than_full": all((r["overhead_with_refill"] if r["overhead_with_refill"] is not None
                                              else 1e9) < temporal["overhead"] for r in rows[:-1]),
            "spatial_yield_latency_lower_than_full": all(
