@@ -203,6 +203,13 @@ typedef struct {
    block index are in tasks (flep_launch_info.tasks_per_block = 8; the trigger index given in
    blocks is converted); worker records are per warp. */
 #define FLEP_KFLAG_WARP_TASKS 128u
+/* In-chunk stop (R33; the counter worker of the memory-bound bodies, not with prefetch,
+   CLC, the scheduling warp, warp tasks or in-tile): chunks of C blocks per fetch, and a poll
+   between the blocks of a chunk (async, R22), so a request is acted on after one block whatever
+   C is. A worker stopped mid-chunk leaves the rest of its chunk in a per-worker record that the
+   worker with the same index runs first in the next epoch (a preempted epoch's coverage is then
+   not a prefix of the counter). Costs W x 16 B of runtime-owned device memory. */
+#define FLEP_KFLAG_IN_CHUNK 256u
 
 typedef enum {
   FLEP_STATE_QUEUED = 0,     /* intercepted, waiting for a scheduling decision (S2) */

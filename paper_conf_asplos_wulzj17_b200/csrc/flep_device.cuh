@@ -520,6 +520,100 @@ flep_worker(const __grid_constant__ typename Body::Args args, const WorkerParams
   if (tid == 0) worker_exit(p, ws);
 }
 
+// ---- in-chunk stop (FLEP_KFLAG_IN_CHUNK, reading R33) --------------------------------------------
+// The counter worker with C > 1 blocks per fetch (the atomic, not the poll, is what a chunk
+// boundary costs) and a poll between the blocks of a chunk, so that a request is acted on after
+// ONE block: the worker that stops mid-chunk leaves the rest of its chunk [b, b_end) in its
+// record (the chunk-rest record of R21, without an accumulator), counted in the exit word's
+// partial bits (R23, the epoch cannot complete while a record is valid); the worker with the same
+// index in the next epoch runs that rest before it fetches. The poll between blocks is the async
+// poll of R22 (copied during the block, tested after it) and one CTA barrier carries the decision.
+template <class Body, bool kCoverage>
+__global__ void __launch_bounds__(Body::kThreads, Body::kMinBlocks)
+flep_worker_ic(const __grid_constant__ typename Body::Args args, const WorkerParams p) {
+  __shared__ uint32_t s_rng[2][2];   // chunk [b0, b1) broadcast, double-buffered
+  __shared__ uint32_t s_stop[2];     // per-block stop decision, double-buffered
+  __shared__ WorkerShared ws;
+  constexpr uint32_t STOP = 0xffffffffu;
+  const uint32_t tid = threadIdx.x;
+  if (blockIdx.x == p.relay_block) { request_relay(p); return; }   // R28: not a worker
+  if (tid == 0) {
+    ws.sm = smid_reg(); ws.t_entry = gtimer(); ws.blocks = 0; ws.reason = 0;
+    ws.counted = 0; ws.last = 0; ws.ev_raw = 0; ws.ev_part = 0; ws.partial = 0;
+    if (blockIdx.x == 0 && p.started_hint && p.status) st_relaxed_sys(&p.status->started, p.epoch);
+  }
+  Body::setup(args);
+  PartialTile* mine = reinterpret_cast<PartialTile*>(p.partial) + blockIdx.x;
+  SchedState st;
+  bool restore = true;
+  uint32_t par = 0, spar = 0;
+  while (true) {
+    if (tid == 0) {
+      uint32_t b0 = STOP, b1 = 0;
+      bool leave = false;
+      if (restore) {                                   // the rest of a chunk stopped last epoch
+        restore = false;
+        if (p.epoch == p.gen_first) {
+          mine->valid = 0;                             // no record survives from another launch
+        } else {
+          const PartialTile e = *mine;                 // written by the previous grid
+          if (e.valid) {
+            st.first = false;                          // (the launch is not complete)
+            if (should_yield(poll_ctrl(p), p, smid_reg())) {   // entry check (a2)
+              ws.reason = kReasonYield;                // the record stays for a later epoch
+              ws.partial = e.b_end - e.b;
+              leave = true;
+            } else {
+              b0 = e.b; b1 = e.b_end;
+              mine->valid = 0;
+              ws.blocks += b1 - b0;
+            }
+          }
+        }
+      }
+      if (!leave && b0 == STOP) {
+        b0 = next_chunk(p, st, ws);
+        b1 = b0 == STOP ? 0u : min(b0 + p.chunk, p.n_blocks);
+      }
+      s_rng[par][0] = leave ? STOP : b0;
+      s_rng[par][1] = b1;
+    }
+    __syncthreads();
+    const uint32_t b0 = s_rng[par][0], b1 = s_rng[par][1];
+    par ^= 1u;
+    if (b0 == STOP) break;
+    bool stopped = false;
+    for (uint32_t b = b0; b < b1; ++b) {
+      const bool more = b + 1 < b1;
+      // async poll (device word), tested after this block; a CPU-written mapped word is read at
+      // the decision point instead (cp.async is for device memory)
+      if (tid == 0 && more && !p.ctrl_sys) poll_issue(ws, p.ctrl);
+      Body::run(args, b, b + 1, p.gx, p.gy);
+      if (kCoverage && tid == 0) atomicAdd(&p.cov[b], 1u);
+      if (more) {
+        if (tid == 0) {
+          const uint32_t c = p.ctrl_sys ? poll_ctrl(p) : poll_consume(ws);
+          const bool stop = should_yield(c, p, smid_reg());
+          s_stop[spar] = stop ? 1u : 0u;
+          if (stop) {
+            mine->b = b + 1; mine->kb = 0; mine->b_end = b1; mine->valid = 1;
+            ws.blocks -= b1 - (b + 1);
+            ws.reason = kReasonYield;
+            ws.partial = b1 - (b + 1);                 // the epoch cannot complete (R23)
+          }
+        }
+        __syncthreads();
+        stopped = s_stop[spar] != 0u;
+        spar ^= 1u;
+        if (stopped) break;
+      }
+    }
+    if (stopped) break;
+  }
+  Body::teardown(args);
+  if (tid == 0) worker_exit(p, ws);
+}
+
 // ---- scheduling-warp worker (FLEP_KFLAG_SCHED_WARP, reading R26) ------------------------------
 // The same protocol as flep_worker, with the scheduling step (poll, fetch, exit accounting) run by
 // one extra warp instead of thread 0 of the body: the scheduler fills a two-slot ring in shared

@@ -44,6 +44,16 @@ struct Ops {
     else flep_warp_worker<Body, false><<<G, Body::kThreads, Body::kDynSmem, s>>>(a, p);
     return cudaGetLastError();
   }
+  static cudaError_t worker_ic(const void* args, const WorkerParams& p, uint32_t W, cudaStream_t s, bool cov) {
+    const typename Body::Args& a = *reinterpret_cast<const typename Body::Args*>(args);
+    if (cov) flep_worker_ic<Body, true><<<W, Body::kThreads, Body::kDynSmem, s>>>(a, p);
+    else flep_worker_ic<Body, false><<<W, Body::kThreads, Body::kDynSmem, s>>>(a, p);
+    return cudaGetLastError();
+  }
+  static cudaError_t occupancy_ic(int* k, bool cov) {
+    if (cov) return cudaOccupancyMaxActiveBlocksPerMultiprocessor(k, flep_worker_ic<Body, true>, Body::kThreads, Body::kDynSmem);
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(k, flep_worker_ic<Body, false>, Body::kThreads, Body::kDynSmem);
+  }
   static cudaError_t occupancy_warp(int* k, bool cov) {
     if (cov) return cudaOccupancyMaxActiveBlocksPerMultiprocessor(k, flep_warp_worker<Body, true>, Body::kThreads, Body::kDynSmem);
     return cudaOccupancyMaxActiveBlocksPerMultiprocessor(k, flep_warp_worker<Body, false>, Body::kThreads, Body::kDynSmem);
@@ -198,21 +208,21 @@ const BodyOps kOps[] = {
     {0, 0, 0, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr},
     {FLEP_BODY_SAXPY_I32, SaxpyI32::kThreads, sizeof(flep_saxpy_i32_args), &Ops<SaxpyI32>::worker,
      &Ops<SaxpyI32>::unwrapped, &Ops<SaxpyI32>::occupancy, nullptr, &Ops<SaxpyI32>::clc,
-     &Ops<SaxpyI32>::worker_sw, &Ops<SaxpyI32>::occupancy_sw, nullptr, nullptr, 0, &Ops<SaxpyI32>::sliced, &Ops<SaxpyI32>::static_launch, nullptr},
+     &Ops<SaxpyI32>::worker_sw, &Ops<SaxpyI32>::occupancy_sw, nullptr, nullptr, 0, &Ops<SaxpyI32>::sliced, &Ops<SaxpyI32>::static_launch, nullptr, &Ops<SaxpyI32>::worker_ic, &Ops<SaxpyI32>::occupancy_ic},
     {FLEP_BODY_SAXPY_F32, SaxpyF32::kThreads, sizeof(flep_saxpy_f32_args), &Ops<SaxpyF32>::worker,
      &Ops<SaxpyF32>::unwrapped, &Ops<SaxpyF32>::occupancy, nullptr, &Ops<SaxpyF32>::clc,
-     &Ops<SaxpyF32>::worker_sw, &Ops<SaxpyF32>::occupancy_sw, nullptr, nullptr, 0, &Ops<SaxpyF32>::sliced, &Ops<SaxpyF32>::static_launch, nullptr},
+     &Ops<SaxpyF32>::worker_sw, &Ops<SaxpyF32>::occupancy_sw, nullptr, nullptr, 0, &Ops<SaxpyF32>::sliced, &Ops<SaxpyF32>::static_launch, nullptr, &Ops<SaxpyF32>::worker_ic, &Ops<SaxpyF32>::occupancy_ic},
     {FLEP_BODY_SPMV_CSR_F32, Spmv::kThreads, sizeof(flep_spmv_args), &Ops<Spmv>::worker,
      &Ops<Spmv>::unwrapped, &Ops<Spmv>::occupancy, nullptr, &Ops<Spmv>::clc,
-     &Ops<Spmv>::worker_sw, &Ops<Spmv>::occupancy_sw, nullptr, nullptr, 0, &Ops<Spmv>::sliced, &Ops<Spmv>::static_launch, nullptr},
+     &Ops<Spmv>::worker_sw, &Ops<Spmv>::occupancy_sw, nullptr, nullptr, 0, &Ops<Spmv>::sliced, &Ops<Spmv>::static_launch, nullptr, &Ops<Spmv>::worker_ic, &Ops<Spmv>::occupancy_ic},
     {FLEP_BODY_STENCIL5_F32, StencilF32::kThreads, sizeof(flep_stencil_args), &Ops<StencilF32>::worker,
      &Ops<StencilF32>::unwrapped, &Ops<StencilF32>::occupancy, nullptr, &Ops<StencilF32>::clc,
      &Ops<StencilF32>::worker_sw, &Ops<StencilF32>::occupancy_sw, &Ops<StencilF32>::warp_worker,
-     &Ops<StencilF32>::occupancy_warp, StencilF32::kWarpTasks, &Ops<StencilF32>::sliced, &Ops<StencilF32>::static_launch, nullptr},
+     &Ops<StencilF32>::occupancy_warp, StencilF32::kWarpTasks, &Ops<StencilF32>::sliced, &Ops<StencilF32>::static_launch, nullptr, &Ops<StencilF32>::worker_ic, &Ops<StencilF32>::occupancy_ic},
     {FLEP_BODY_STENCIL5_I32, StencilI32::kThreads, sizeof(flep_stencil_args), &Ops<StencilI32>::worker,
      &Ops<StencilI32>::unwrapped, &Ops<StencilI32>::occupancy, nullptr, &Ops<StencilI32>::clc,
      &Ops<StencilI32>::worker_sw, &Ops<StencilI32>::occupancy_sw, &Ops<StencilI32>::warp_worker,
-     &Ops<StencilI32>::occupancy_warp, StencilI32::kWarpTasks, &Ops<StencilI32>::sliced, &Ops<StencilI32>::static_launch, nullptr},
+     &Ops<StencilI32>::occupancy_warp, StencilI32::kWarpTasks, &Ops<StencilI32>::sliced, &Ops<StencilI32>::static_launch, nullptr, &Ops<StencilI32>::worker_ic, &Ops<StencilI32>::occupancy_ic},
     {FLEP_BODY_GEMM_BF16, GemmBody::kThreads, sizeof(flep_gemm_args), &gemm_worker_launch,
      &gemm_unwrapped_launch, &gemm_occupancy, &gemm_validate, nullptr, nullptr, nullptr, nullptr, nullptr, 0,
      &gemm_slice_launch, &gemm_static_launch, nullptr},
@@ -222,7 +232,7 @@ const BodyOps kOps[] = {
     {FLEP_BODY_SPMV_CSR_F32_VEC, SpmvVec::kThreads, sizeof(flep_spmv_args), &Ops<SpmvVec>::worker,
      &Ops<SpmvVec>::unwrapped, &Ops<SpmvVec>::occupancy, nullptr, &Ops<SpmvVec>::clc,
      &Ops<SpmvVec>::worker_sw, &Ops<SpmvVec>::occupancy_sw, &Ops<SpmvVec>::warp_worker,
-     &Ops<SpmvVec>::occupancy_warp, SpmvVec::kWarpTasks, &Ops<SpmvVec>::sliced, &Ops<SpmvVec>::static_launch, nullptr},
+     &Ops<SpmvVec>::occupancy_warp, SpmvVec::kWarpTasks, &Ops<SpmvVec>::sliced, &Ops<SpmvVec>::static_launch, nullptr, &Ops<SpmvVec>::worker_ic, &Ops<SpmvVec>::occupancy_ic},
     {FLEP_BODY_GEMM_BF16_2SM, 256 /* Gemm2::kThreads (gemm2_tcgen05.cuh, its own TU) */, sizeof(flep_gemm_args), &gemm2_worker_launch,
      &gemm2_unwrapped_launch, &gemm2_occupancy, &gemm2_validate, nullptr, nullptr, nullptr, nullptr, nullptr, 0,
      nullptr, &gemm2_static_launch, &gemm2_max_pairs},

@@ -39,6 +39,9 @@ struct BodyOps {
   cudaError_t (*static_launch)(const void* args, dim3 grid, uint32_t ctas, uint32_t chunk, cudaStream_t s);
   // CTA-pair bodies (R32): the worker is a cluster of 2 CTAs; max resident pairs
   cudaError_t (*max_pairs)(int* pairs, bool cov);
+  // in-chunk stop worker (flep_worker_ic<Body>, R33) and its occupancy
+  cudaError_t (*worker_ic)(const void* args, const WorkerParams& p, uint32_t W, cudaStream_t s, bool cov);
+  cudaError_t (*occupancy_ic)(int* ctas_per_sm, bool cov);
 };
 
 const BodyOps* body_ops(int32_t body);

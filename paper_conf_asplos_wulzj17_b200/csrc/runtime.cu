@@ -132,6 +132,7 @@ struct Launch {
   bool sw = false;                   // FLEP_KFLAG_SCHED_WARP: scheduling-warp worker (R26)
   bool relay = false;                // FLEP_KFLAG_HOST_RELAY: one request-relay CTA (R28)
   bool warp = false;                 // FLEP_KFLAG_WARP_TASKS: warp workers, counts in tasks (R30)
+  bool ic = false;                   // FLEP_KFLAG_IN_CHUNK: poll between the blocks of a chunk (R33)
   uint32_t tasks_per_block = 1;
   uint32_t ctas = 0;                 // worker CTAs per epoch (= workers, or workers / warps per CTA)
   uint32_t slice_blocks = 0;
@@ -216,12 +217,14 @@ struct ApiLock {
   }
 };
 
-flep_status occupancy(flep_rt rt, const BodyOps* ops, bool cov, int* k, bool sw = false, bool warp = false) {
-  auto key = std::make_pair(ops->body * 4 + (sw ? 1 : 0) + (warp ? 2 : 0), cov);
+flep_status occupancy(flep_rt rt, const BodyOps* ops, bool cov, int* k, bool sw = false, bool warp = false,
+                      bool ic = false) {
+  auto key = std::make_pair(ops->body * 8 + (sw ? 1 : 0) + (warp ? 2 : 0) + (ic ? 4 : 0), cov);
   auto it = rt->occ_cache.find(key);
   if (it != rt->occ_cache.end()) { *k = it->second; return FLEP_OK; }
   if (sw) CUDA_TRY(ops->occupancy_sw(k, cov));
   else if (warp) CUDA_TRY(ops->occupancy_warp(k, cov));
+  else if (ic) CUDA_TRY(ops->occupancy_ic(k, cov));
   else CUDA_TRY(ops->occupancy(k, cov));
   if (*k <= 0) return fail(FLEP_ERR_UNSUPPORTED, "body %d cannot be resident", ops->body);
   rt->occ_cache[key] = *k;
@@ -344,10 +347,10 @@ flep_status materialize(flep_rt rt, Launch& L) {
     }
     if (!L.cov) { L.cov_cap = std::max<size_t>(N, 4096); CUDA_TRY(cudaMalloc(&L.cov, L.cov_cap * 4)); }
   }
-  if (L.flags & FLEP_KFLAG_IN_TILE) {
-    // per-worker partial-tile records and fp32 accumulator spill slots; no reset needed (the
-    // first epoch's workers clear their records)
-    const size_t need = partial_bytes(L.workers);
+  if (L.flags & (FLEP_KFLAG_IN_TILE | FLEP_KFLAG_IN_CHUNK)) {
+    // per-worker partial-tile records (and, in-tile, fp32 accumulator spill slots); no reset
+    // needed (the first epoch's workers clear their records)
+    const size_t need = (L.flags & FLEP_KFLAG_IN_TILE) ? partial_bytes(L.workers) : partial_header_bytes(L.workers);
     size_t best = rt->free_partial.size();
     for (size_t i = 0; i < rt->free_partial.size(); ++i)
       if (rt->free_partial[i].second >= need &&
@@ -450,7 +453,7 @@ flep_status start_epoch(flep_rt rt, Launch& L) {
   p.trigger_n = L.trig_n;
   // no prefetch with in-tile preemption: a worker whose exhausted prefetch already counted its
   // exit must not later leave a partial tile (R23)
-  p.prefetch = ((L.flags & FLEP_KFLAG_PREFETCH) && !(L.flags & FLEP_KFLAG_IN_TILE)) ? 1u : 0u;
+  p.prefetch = ((L.flags & FLEP_KFLAG_PREFETCH) && !(L.flags & (FLEP_KFLAG_IN_TILE | FLEP_KFLAG_IN_CHUNK))) ? 1u : 0u;
   p.gen_first = L.gen0 + 1;
   p.started_hint = (L.flags & FLEP_KFLAG_STARTED_HINT) ? 1u : 0u;
   p.relay_block = L.relay ? L.ctas : 0xffffffffu;
@@ -466,6 +469,7 @@ flep_status start_epoch(flep_rt rt, Launch& L) {
                  : L.sw ? L.ops->worker_sw(L.args.data(), p, L.workers, L.exec, L.cov != nullptr)
                  : L.warp ? L.ops->warp_worker(L.args.data(), p, L.ctas + (L.relay ? 1u : 0u), L.exec, L.cov != nullptr)
                  : L.ops->max_pairs ? L.ops->worker(L.args.data(), p, L.ctas, L.exec, L.cov != nullptr)
+                 : L.ic ? L.ops->worker_ic(L.args.data(), p, L.workers + (L.relay ? 1u : 0u), L.exec, L.cov != nullptr)
                         : L.ops->worker(L.args.data(), p, L.workers + (L.relay ? 1u : 0u), L.exec, L.cov != nullptr);
   if (e != cudaSuccess) return fail(FLEP_ERR_CUDA, "worker launch failed: %s", cudaGetErrorString(e));
   CUDA_TRY(cudaEventRecord(L.fin_ev, L.exec));
@@ -905,6 +909,15 @@ flep_status flep_register_kernel(flep_rt rt, const flep_kernel_desc* d, flep_ker
     return fail(FLEP_ERR_UNSUPPORTED, "in-tile preemption is implemented for the GEMM body only");
   if ((d->flags & FLEP_KFLAG_IN_TILE) && (d->flags & FLEP_KFLAG_PREFETCH))
     return fail(FLEP_ERR_UNSUPPORTED, "in-tile preemption does not combine with chunk prefetch");
+  if (d->flags & FLEP_KFLAG_IN_CHUNK) {
+    const BodyOps* o = body_ops(d->body);
+    if (!o->worker_ic)
+      return fail(FLEP_ERR_UNSUPPORTED, "body %d has no in-chunk-stop worker", d->body);
+    if (d->flags & (FLEP_KFLAG_PREFETCH | FLEP_KFLAG_CLC | FLEP_KFLAG_SCHED_WARP | FLEP_KFLAG_WARP_TASKS |
+                    FLEP_KFLAG_IN_TILE))
+      return fail(FLEP_ERR_UNSUPPORTED, "in-chunk stop does not combine with prefetch, CLC, the scheduling warp, "
+                                        "warp tasks or in-tile preemption");
+  }
   ApiLock lk(rt);
   if (d->flags & FLEP_KFLAG_IN_TILE) {
     // in-tile records + accumulator spill slots for the largest worker grid this kernel can have,
@@ -984,8 +997,9 @@ flep_status flep_launch(flep_rt rt, flep_kernel kid, flep_dim3 grid, const void*
     return fail(FLEP_ERR_UNSUPPORTED, "warp tasks do not combine with CLC, the scheduling warp or in-tile preemption");
   const uint32_t tpb = warp ? ops->warp_tasks : 1u;
   if (N * tpb >= (1ull << 31)) return fail(FLEP_ERR_INVALID, "grid too large for warp tasks");
+  const bool ic = (kr.flags & FLEP_KFLAG_IN_CHUNK) && !slicing;
   int k = 0;
-  s = occupancy(rt, ops, cov, &k, sw, warp);
+  s = occupancy(rt, ops, cov, &k, sw, warp, ic);
   if (s) return s;
   if (rt->free_slots.empty()) return fail(FLEP_ERR_NOMEM, "out of status slots");
 
@@ -998,6 +1012,7 @@ flep_status flep_launch(flep_rt rt, flep_kernel kid, flep_dim3 grid, const void*
   L.args.assign((const uint8_t*)args, (const uint8_t*)args + args_size);
   L.grid = g;
   L.warp = warp;
+  L.ic = ic;
   L.tasks_per_block = tpb;
   L.n_blocks = (uint32_t)(N * tpb);          // the runtime's unit: tasks (= blocks unless R30)
   L.prio = priority;

@@ -5,7 +5,7 @@ of the workers (first entry -> last exit, %globaltimer) so that launch / teardow
 span is visible.
 
   FLEP_LIB_PATH=build_variants/x.so python tools/ab_overhead.py [case,...]
-case = body:C:K[:pf[:clc[:warp]]]
+case = body:C:K[:pf[:clc[:warp[:in_chunk]]]]
 """
 import json
 import os
@@ -53,8 +53,10 @@ def main():
         f = c.split(":")
         name, C, K = f[0], int(f[1]), int(f[2])
         pf, clc, warp = (int(f[3]) if len(f) > 3 else 0), (int(f[4]) if len(f) > 4 else 0), (int(f[5]) if len(f) > 5 else 0)
+        ic = int(f[6]) if len(f) > 6 else 0
         body, grid, args = bodies[name]
-        k = rt.register_kernel(body, chunk=C, poll=K, prefetch=bool(pf), clc=bool(clc), warp_tasks=bool(warp))
+        k = rt.register_kernel(body, chunk=C, poll=K, prefetch=bool(pf), clc=bool(clc), warp_tasks=bool(warp),
+                               in_chunk=bool(ic))
         tw, tu, span, uspan = [], [], [], []
         for r in range(reps + 3):
             for mode in ("w", "u"):
