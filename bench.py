@@ -269,14 +269,15 @@ def run_temporal(args, rank, world, local):
     n_lp = lp_grid[0]
     g = gen.rng(1000 + rank)
 
-    def step():
+    def step(k_lp=None):
+        k_lp = kLP if k_lp is None else k_lp
         tstar = int(g.integers(n_lp // 4, 3 * n_lp // 4))
         with torch.cuda.stream(A):
             flush.zero_()
             e0 = torch.cuda.Event(enable_timing=True)
             e0.record(A)
         rt.arm_next_trigger(tstar, num_sms)
-        h_lp = rt.launch(kLP, lp_grid, lp_args, priority=0, stream=A)
+        h_lp = rt.launch(k_lp, lp_grid, lp_args, priority=0, stream=A)
         B.wait_event(e0)
         h_hp = rt.launch(kHP, hp_grid, hp_args, priority=1, stream=B)
         rt.wait_epoch(h_lp, timeout_ns=10_000_000_000)
@@ -371,6 +372,22 @@ def run_temporal(args, rank, world, local):
                 "frac": round(achieved / hbm, 4), "traffic": prof_traffic, "kernel": f"flep_worker<{dom}>",
                 "algorithmic_bytes": algo, "peak_source": peak_src}
 
+    # the throughput operating point of the same co-run (SURVEY §8(d) "(C, K) sweep"): the victim
+    # fetches C = 2 blocks per atomic, so its drain is up to two blocks and its overhead is paid
+    # per 256 rows; measured with the same steps, the same kernel timing protocol
+    op2 = None
+    if args.lp_chunk == 1 and args.op2:
+        kLP2 = rt.register_kernel(F.BODY_SPMV_CSR_F32, chunk=2, poll=args.lp_poll, name="spmv-c2")
+        for _ in range(args.warmup):
+            step(kLP2)
+        r2 = [step(kLP2) for _ in range(args.steps)]
+        d2 = [r["drain_us"] for r in r2 if r["preempted"]]
+        kt2 = kernel_timings(rt, F, torch, wl, flush, A, kLP2, kHP, lp_args, hp_args, lp_grid, hp_grid, args.reps,
+                             only=("spmv",))
+        op2 = {"lp_chunk": 2, "drain_us": {"p50": round(float(np.median(d2)), 3) if d2 else None,
+                                           "p99": round(float(np.percentile(d2, 99)), 3) if d2 else None,
+                                           "max": round(max(d2), 3) if d2 else None, "preempted_steps": len(d2)},
+               "spmv": kt2["spmv"]}
     e2e = run_e2e(F, torch, wl, local, args.e2e_steps, args)
     _diag = run_e2e(F, torch, wl, local, args.e2e_steps, args, diag=True)
     e2e["breakdown_us_p50"] = _diag.get("breakdown_us_p50")
@@ -408,6 +425,11 @@ def run_temporal(args, rank, world, local):
         "target_20us_met": bool(drain) and max(drain) < 20.0,
         "latency_budget": latency_budget,
         "wrapper_overhead_pct": {k: v["overhead_pct"] for k, v in kern.items()},
+        "operating_points": {"latency (victim C = 1, the headline)": {
+                                 "lp_chunk": args.lp_chunk, "drain_us_p50": round(d50, 3),
+                                 "spmv_overhead_pct": kern["spmv"]["overhead_pct"],
+                                 "spmv_overhead_pct_ci95": kern["spmv"].get("overhead_pct_ci95")},
+                             "throughput (victim C = 2)": op2},
         "kernels": kern,
         "roofline": roofline,
         "gather_roofline": gather_roofline,
@@ -451,10 +473,13 @@ def spot_parity(wl, torch):
             "ok": bool(worst <= 1e-5 and worst_st <= 1e-5)}
 
 
-def kernel_timings(rt, F, torch, wl, flush, A, kLP, kHP, lp_args, hp_args, lp_grid, hp_grid, reps):
+def kernel_timings(rt, F, torch, wl, flush, A, kLP, kHP, lp_args, hp_args, lp_grid, hp_grid, reps,
+                   only=("spmv", "stencil")):
     res = {}
     for name, k, body, a, grid, nbytes in (("spmv", kLP, F.BODY_SPMV_CSR_F32, lp_args, lp_grid, wl.spmv_bytes),
                                            ("stencil", kHP, F.BODY_STENCIL5_F32, hp_args, hp_grid, wl.st_bytes)):
+        if name not in only:
+            continue
         tw, tu = [], []
         for r in range(reps + 2):
             for mode in ("w", "u"):
@@ -712,6 +737,7 @@ def main():
     ap.add_argument("--dry-run", action="store_true",
                     help="configs[4] launcher and control flow without CUDA (CPU, gloo); one JSON line")
     ap.add_argument("--sub", type=int, default=1, help="default run: add the configs[0,2,3,4] sub-records")
+    ap.add_argument("--op2", type=int, default=1, help="default run: also measure the C = 2 operating point")
     ap.add_argument("--sub-steps", type=int, default=12, help="timed trials per sub-record case")
     ap.add_argument("--skip-sub", default="", help="comma list of sub-record names to skip")
     ap.add_argument("--scale-kernels", type=int, default=512)
