@@ -6,6 +6,7 @@ workers' %globaltimer event log; all inputs are seeded (synth/gen.py)."""
 from __future__ import annotations
 
 import json
+import os
 import time
 
 import numpy as np
@@ -819,7 +820,9 @@ def _queue_instances(torch, F, seed):
                 A = (torch.rand(sz, sz, device="cuda", generator=g) * 2 - 1).to(torch.bfloat16)
                 B = (torch.rand(sz, sz, device="cuda", generator=g) * 2 - 1).to(torch.bfloat16)
                 C = torch.empty(sz, sz, device="cuda", dtype=torch.bfloat16)
-                inst[(ty, cls)] = (F.BODY_GEMM_BF16, F.gemm_grid(sz, sz), F.gemm_args(C, A, B), (A, B, C),
+                pair = os.environ.get("FLEP_QUEUE_GEMM", "1") == "2"   # the CTA-pair body (R32)
+                inst[(ty, cls)] = ((F.BODY_GEMM_BF16_2SM, F.gemm2_grid(sz, sz)) if pair else
+                                   (F.BODY_GEMM_BF16, F.gemm_grid(sz, sz))) + (F.gemm_args(C, A, B), (A, B, C),
                                    2 * sz ** 3)
     return inst
 

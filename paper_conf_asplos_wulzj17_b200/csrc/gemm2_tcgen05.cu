@@ -97,6 +97,16 @@ cudaError_t gemm2_static_launch(const void* user, dim3 grid, uint32_t ctas, uint
   return cudaGetLastError();
 }
 
+cudaError_t gemm2_slice_launch(const void* user, dim3 grid, uint32_t offset, uint32_t count, const SliceParams& sp,
+                               cudaStream_t s) {
+  Gemm2Args d;
+  if (!to_dev(user, &d)) return cudaErrorInvalidValue;
+  cudaError_t e = smem_attr(flep_gemm2_slice);
+  if (e) return e;
+  flep_gemm2_slice<<<2 * count, Gemm2::kThreads, Gemm2::kDynSmem, s>>>(d, grid.x, grid.y, offset, sp);
+  return cudaGetLastError();
+}
+
 cudaError_t gemm2_occupancy(int* k, bool cov) {
   // one CTA per SM; the runtime sizes the grid in pairs (gemm2_max_pairs)
   cudaError_t e = cov ? smem_attr(flep_gemm2_worker<true>) : smem_attr(flep_gemm2_worker<false>);

@@ -335,6 +335,42 @@ flep_gemm2_unwrapped(const __grid_constant__ Gemm2Args g, uint32_t gx, uint32_t 
   Gemm2::teardown();
 }
 
+// Kernel slicing with the device check (R31): one pair per tile of the slice; every CTA follows
+// the slice's one decision (taken by the first CTA of the slice that gets there), so both CTAs of
+// a pair agree.
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Gemm2::kThreads, 1)
+flep_gemm2_slice(const __grid_constant__ Gemm2Args g, uint32_t gx, uint32_t gy, uint32_t offset, const SliceParams sp) {
+  __shared__ uint32_t s_go;
+  if (threadIdx.x == 0) {
+    uint32_t* dp = sp.decision + sp.slice;
+    uint32_t d = ld_relaxed_gpu(dp);
+    bool go;
+    if ((d >> 2) == slice_tag(sp.gen)) {
+      go = (d & 3u) == kSliceRun;
+    } else if ((d & 3u) == kSliceRun) {
+      go = false;
+    } else {
+      const uint32_t c = ld_relaxed_gpu(sp.ctrl);
+      const bool stop = ctrl_gen(c) == (sp.gen & kCtrlGenMask) && ctrl_n(c) > 0;
+      const uint32_t want = (slice_tag(sp.gen) << 2) | (stop ? kSliceSkip : kSliceRun);
+      const uint32_t old = atomicCAS(dp, d, want);
+      go = ((old == d) ? want : old) == ((slice_tag(sp.gen) << 2) | kSliceRun);
+    }
+    s_go = go ? 1u : 0u;
+  }
+  __syncthreads();
+  if (!s_go) return;                   // both CTAs of the pair leave (same decision)
+  Gemm2::setup();
+  const uint32_t b = offset + (blockIdx.x >> 1);
+  bool given = false;
+  Gemm2::pipeline(g, gx, gy, [&](uint32_t& b0, uint32_t& b1) {
+    if (given) return false;
+    given = true; b0 = b; b1 = b + 1;
+    return true;
+  });
+  Gemm2::teardown();
+}
+
 // Static persistent twin (U1): the same pairs, tiles pair, pair + P, pair + 2P, ... with no
 // counter and no poll (the FLEP worker's overhead baseline).
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Gemm2::kThreads, 1)

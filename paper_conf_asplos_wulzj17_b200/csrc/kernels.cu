@@ -235,7 +235,7 @@ const BodyOps kOps[] = {
      &Ops<SpmvVec>::occupancy_warp, SpmvVec::kWarpTasks, &Ops<SpmvVec>::sliced, &Ops<SpmvVec>::static_launch, nullptr, &Ops<SpmvVec>::worker_ic, &Ops<SpmvVec>::occupancy_ic},
     {FLEP_BODY_GEMM_BF16_2SM, 256 /* Gemm2::kThreads (gemm2_tcgen05.cuh, its own TU) */, sizeof(flep_gemm_args), &gemm2_worker_launch,
      &gemm2_unwrapped_launch, &gemm2_occupancy, &gemm2_validate, nullptr, nullptr, nullptr, nullptr, nullptr, 0,
-     nullptr, &gemm2_static_launch, &gemm2_max_pairs},
+     &gemm2_slice_launch, &gemm2_static_launch, &gemm2_max_pairs},
 };
 
 }  // namespace

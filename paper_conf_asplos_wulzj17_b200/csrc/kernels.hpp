@@ -51,6 +51,8 @@ cudaError_t gemm2_worker_launch(const void* user, const WorkerParams& p, uint32_
 cudaError_t gemm2_unwrapped_launch(const void* user, dim3 grid, uint32_t offset, uint32_t count, cudaStream_t s);
 cudaError_t gemm2_static_launch(const void* user, dim3 grid, uint32_t ctas, uint32_t chunk, cudaStream_t s);
 cudaError_t gemm2_occupancy(int* k, bool cov);
+cudaError_t gemm2_slice_launch(const void* user, dim3 grid, uint32_t offset, uint32_t count, const SliceParams& sp,
+                               cudaStream_t s);
 cudaError_t gemm2_max_pairs(int* pairs, bool cov);
 const char* gemm2_validate(const void* user, dim3 grid);
 cudaError_t gemm_slice_launch(const void* user, dim3 grid, uint32_t offset, uint32_t count,

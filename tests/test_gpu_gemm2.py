@@ -127,3 +127,35 @@ def test_gemm2_8192_sampled_vs_oracle(rt):
     got = C[rows].float().cpu().numpy().astype(np.float64)
     rms = float(np.sqrt(np.mean(ref ** 2)))
     assert np.all(np.abs(got - ref) <= TOL * (np.abs(ref) + rms))
+
+
+def test_gemm2_sliced_with_device_check_preempted():
+    """Kernel slicing with the device check (R31) on the pair body: a higher-priority arrival
+    makes the remaining slices skip; the resumed run is bit-identical to the unwrapped grid."""
+    import torch
+    f = flep_mod()
+    rs = f.Runtime(policy=f.POLICY_SLICE_DEVICE, slice_blocks=16)
+    try:
+        m, n, k = 8192, 4096, 2048                 # ~0.1 ms: the arrival lands while it runs
+        a_bits, b_bits = gen.gemm_bf16_inputs(m, n, k, seed=172)
+        A, B = _bf16(a_bits), _bf16(b_bits)
+        grid = f.gemm2_grid(m, n)
+        C0 = torch.empty((m, n), dtype=torch.bfloat16, device="cuda")
+        rs.launch_unwrapped(f.BODY_GEMM_BF16_2SM, grid, f.gemm_args(C0, A, B))
+        torch.cuda.synchronize()
+        C1 = torch.empty((m, n), dtype=torch.bfloat16, device="cuda")
+        kl = rs.register_kernel(f.BODY_GEMM_BF16_2SM, chunk=1, poll=1, model=(0, 0, 0, 0, 2_000_000))
+        kh = rs.register_kernel(f.BODY_SAXPY_I32, chunk=1, poll=1, model=(0, 0, 0, 0, 5_000))
+        x, y = gen.saxpy_i32_inputs(1 << 16, seed=173)
+        xd, yd = torch.from_numpy(x).cuda(), torch.from_numpy(y).cuda()
+        h1 = rs.launch(kl, grid, f.gemm_args(C1, A, B), priority=0)
+        h2 = rs.launch(kh, f.saxpy_grid(1 << 16), f.saxpy_i32_args(yd, xd, 3), priority=1)
+        rs.sync(h2, timeout_ns=20_000_000_000)
+        rs.sync(h1, timeout_ns=20_000_000_000)
+        torch.cuda.synchronize()
+        assert torch.equal(C1, C0)
+        assert np.array_equal(yd.cpu().numpy(), W.saxpy_i32(3, x, y))
+        acts = [f.ACTION_NAMES[d[1]] for d in rs.decision_log()]
+        assert acts[:3] == ["LAUNCH", "PREEMPT", "LAUNCH"]
+    finally:
+        rs.close()
