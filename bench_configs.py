@@ -449,9 +449,12 @@ def run_gemm_preempt(args, rank, world, local):
     st_in = torch.rand(4096, 4096, device="cuda", generator=g)
     st_out = torch.empty_like(st_in)
     in_tile = bool(args.gemm_in_tile)
-    k_lp = rt.register_kernel(F.BODY_GEMM_BF16, chunk=1, poll=1, name="gemm", in_tile=in_tile)
+    pair = bool(getattr(args, "gemm_pair", 0))            # the CTA-pair body (R32)
+    body = F.BODY_GEMM_BF16_2SM if pair else F.BODY_GEMM_BF16
+    k_lp = rt.register_kernel(body, chunk=1, poll=1, name="gemm", in_tile=in_tile)
     k_hp = rt.register_kernel(F.BODY_STENCIL5_F32, chunk=2, poll=1, prefetch=True, name="stencil")
-    lp_args, lp_grid = F.gemm_args(C_, A_, B_), F.gemm_grid(M, N)
+    lp_args = F.gemm_args(C_, A_, B_)
+    lp_grid = F.gemm2_grid(M, N) if pair else F.gemm_grid(M, N)
     hp_args, hp_grid = F.stencil_args(st_out, st_in), F.stencil_grid(4096)
     nb = lp_grid[0] * lp_grid[1]
     flush = L2Flush(torch)
@@ -511,8 +514,9 @@ def run_gemm_preempt(args, rank, world, local):
                                "last GEMM CTA gone, p50",
            "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "higher_is_better": False,
            "scaling": "weak", "vs_baseline": None, "dtype": "bf16", "data": "synthetic (seeded)",
-           "config": {"workload": "LP GEMM bf16 8192^3 (tcgen05, 128x256 tiles) preempted by HP stencil5 4096^2",
-                      "chunk": 1, "poll": 1, "in_tile": in_tile},
+           "config": {"workload": ("LP GEMM bf16 8192^3 (tcgen05 cta_group::2, 256x256 tiles on CTA pairs)" if pair else
+                                   "LP GEMM bf16 8192^3 (tcgen05, 128x256 tiles)") + " preempted by HP stencil5 4096^2",
+                      "chunk": 1, "poll": 1, "in_tile": in_tile, "pair": pair},
            "preempted_steps": pre, "not_bit_identical_to_uninterrupted": bad,
            "sample_max_rel": worst, "tol": 2e-2,
            "drain_us": {"p50": round(float(np.median(drain)), 3) if drain else None,
@@ -835,7 +839,7 @@ def _run_trace(F, torch, local, policy, trace, inst, t_alone, overhead_ns, strea
         C, pf = QUEUE_CHUNK[key[0]]
         kid[key] = rt.register_kernel(body, chunk=C, poll=1, prefetch=pf, name=f"{key[0]}-{key[1]}",
                                       model=(0, 0, 0, 0, float(t_alone[key])), overhead_ns=int(overhead_ns),
-                                      in_tile=body == F.BODY_GEMM_BF16)
+                                      in_tile=body in (F.BODY_GEMM_BF16, F.BODY_GEMM_BF16_2SM))
     hs = []
     call_ns = []
     t0 = F.now_ns() + 2_000_000
@@ -888,7 +892,7 @@ def run_queue(args, rank, world, local):
     rt = F.Runtime(device=local, policy=F.POLICY_FIFO)
     for key, (body, grid, a, keep, _) in inst.items():
         C, pf = QUEUE_CHUNK[key[0]]
-        k = rt.register_kernel(body, chunk=C, poll=1, prefetch=pf, in_tile=body == F.BODY_GEMM_BF16)
+        k = rt.register_kernel(body, chunk=C, poll=1, prefetch=pf, in_tile=body in (F.BODY_GEMM_BF16, F.BODY_GEMM_BF16_2SM))
         ts = []
         for r in range(4):
             flush.zero_()                      # cold L2: the queue interleaves working sets
@@ -1200,7 +1204,7 @@ def run_scale_queue(args, rank, world, local):
     rt_m = F.Runtime(device=local, exec_on_user_stream=True)
     for key, (body, grid, a, keep, _) in sorted(inst.items()):
         C, pf = QUEUE_CHUNK[key[0]]
-        k = rt.register_kernel(body, chunk=C, poll=1, prefetch=pf, in_tile=body == F.BODY_GEMM_BF16)
+        k = rt.register_kernel(body, chunk=C, poll=1, prefetch=pf, in_tile=body in (F.BODY_GEMM_BF16, F.BODY_GEMM_BF16_2SM))
         ts = []
         for r in range(3):
             flush.zero_()
@@ -1211,7 +1215,7 @@ def run_scale_queue(args, rank, world, local):
             if r:
                 ts.append(info.t_finish - info.t_arrive)
         t_alone[key] = int(np.median(ts))
-        km = rt_m.register_kernel(body, chunk=C, poll=1, prefetch=pf, in_tile=body == F.BODY_GEMM_BF16)
+        km = rt_m.register_kernel(body, chunk=C, poll=1, prefetch=pf, in_tile=body in (F.BODY_GEMM_BF16, F.BODY_GEMM_BF16_2SM))
         tw, tu = [], []
         for r in range(4):
             for mode in ("w", "u"):
@@ -1492,8 +1496,8 @@ def run_slicing_overhead(args, rank, world, local):
         for key in sorted(inst):
             body, grid, a, keep, _ = inst[key]
             C, pf = QUEUE_CHUNK[key[0]]
-            k_t = rt_m.register_kernel(body, chunk=C, poll=1, prefetch=pf, in_tile=body == F.BODY_GEMM_BF16)
-            k_1 = rt_m.register_kernel(body, chunk=1, poll=1, in_tile=body == F.BODY_GEMM_BF16)
+            k_t = rt_m.register_kernel(body, chunk=C, poll=1, prefetch=pf, in_tile=body in (F.BODY_GEMM_BF16, F.BODY_GEMM_BF16_2SM))
+            k_1 = rt_m.register_kernel(body, chunk=1, poll=1, in_tile=body in (F.BODY_GEMM_BF16, F.BODY_GEMM_BF16_2SM))
             k_s = rt_s.register_kernel(body, chunk=C, poll=1)
             cps, w = rt_m.workers_for(body)
             slice_blocks = w * C                                     # one wave of W*C*K blocks (A20)

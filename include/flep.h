@@ -162,11 +162,13 @@ typedef struct {
    (flep_launch_info.started_epoch). Off by default: the system-scope store it needs delays the
    grid's completion by about a microsecond. */
 #define FLEP_KFLAG_STARTED_HINT 2u
-/* In-tile preemption (GEMM body only; not with FLEP_KFLAG_PREFETCH): workers also poll inside a
+/* In-tile preemption (GEMM bodies only; not with FLEP_KFLAG_PREFETCH): workers also poll inside a
    tile (every 4 k-steps) and, when asked to leave, spill the fp32 accumulator of the tile in
    progress to a per-worker slot; the next epoch's worker with the same index restores it and
    continues the k-loop. The result stays bit-identical to an uninterrupted run. Costs
-   W x (16 B + 128 KiB) of device memory per launch (runtime-owned, pooled).
+   W x (16 B + 128 KiB) of device memory per launch (runtime-owned, pooled); for the CTA-pair
+   body (FLEP_BODY_GEMM_BF16_2SM) one record per pair and one 128 KiB slot per CTA (each CTA
+   spills its 128-row half of the 256x256 tile).
    flep_register_kernel returns FLEP_ERR_UNSUPPORTED for other bodies or with prefetch. */
 #define FLEP_KFLAG_IN_TILE 4u
 /* Asynchronous poll: the control word a worker tests at a poll point was loaded at its previous

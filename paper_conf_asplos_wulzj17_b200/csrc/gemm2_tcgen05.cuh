@@ -21,9 +21,10 @@
 //   warps 4..7           : epilogue of the CTA's 128 rows: tcgen05.ld -> bf16 -> global; then
 //                          a (remote, for the peer) arrive on the leader's accumulator-empty
 //                          barrier
-// Preemption granularity: one tile (the pair polls between chunks; no in-tile spill here, the
-// 1-CTA GEMM body keeps that). A spatial request releases a pair iff it names either of its SMs
-// (a pair cannot split), R32.
+// Preemption granularity: one tile (the pair polls between chunks), or — registered with
+// FLEP_KFLAG_IN_TILE — a few k-steps: the pair stops inside a tile and spills both 128-row halves
+// of its accumulator (worker_pipeline below, R21 + R32). A spatial request releases a pair iff it
+// names either of its SMs (a pair cannot split), R32.
 #pragma once
 #include <cuda.h>
 #include <cuda_bf16.h>
@@ -53,12 +54,18 @@ struct Gemm2 {
   static constexpr uint32_t kQConsumers = 10;                  // leader: MMA + 4 epilogue warps; peer: producer + 4
   static constexpr size_t kDynSmem = 1024 + STAGES * kStage + 1024;
   static constexpr uint32_t STOP = 0xffffffffu;
+  static constexpr uint32_t STOP_PARTIAL = 0xfffffffeu;         // in-tile: the last tile was stopped
 
   struct State {
     uint64_t full[STAGES], empty[STAGES];
     uint64_t tfull[2], tempty[2];
     uint64_t qfull[QDEPTH], qempty[QDEPTH];
+    uint64_t trest[2];                // in-tile: both CTAs restored a spilled half (leader's, count 8)
     uint32_t tile_q[QDEPTH];
+    uint32_t tile_kb0[QDEPTH];        // in-tile: first k-step of the tile (> 0: continue a spill)
+    uint32_t stage_stop[STAGES];      // in-tile: this stage is a stop marker (leader)
+    uint32_t lic;                     // in-tile (peer): k-step loads the leader has licensed
+    uint32_t stop_at;                 // in-tile (peer): the licence count at which loads stop
     uint32_t tmem_base;
     uint32_t smid;
   };
@@ -128,6 +135,10 @@ struct Gemm2 {
       for (uint32_t i = 0; i < STAGES; ++i) { mbar_init(&s->full[i], 1); mbar_init(&s->empty[i], 1); }
       for (uint32_t i = 0; i < 2; ++i) { mbar_init(&s->tfull[i], 1); mbar_init(&s->tempty[i], 8); }
       for (uint32_t i = 0; i < QDEPTH; ++i) { mbar_init(&s->qfull[i], 1); mbar_init(&s->qempty[i], kQConsumers); }
+      // in-tile: trest counts one arrive per epilogue warp of both CTAs
+      for (uint32_t i = 0; i < 2; ++i) mbar_init(&s->trest[i], 8);
+      for (uint32_t i = 0; i < STAGES; ++i) s->stage_stop[i] = 0;
+      s->lic = 0; s->stop_at = 0xffffffffu;
       s->smid = smid_reg();
       asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
@@ -284,6 +295,317 @@ struct Gemm2 {
       }
     }
   }
+
+  // ---- the FLEP worker's pipeline with in-tile preemption (R32 + R21) --------------------------
+  // As `pipeline`, plus: the leader's producer polls the control word every kInTilePoll k-steps
+  // inside a tile; the peer's producer issues a k-step's loads only once the leader has licensed
+  // it (a running licence count, kLicSlack ahead of the leader's own loads, written into the
+  // peer's shared memory), so at a stop both CTAs load exactly the same k-steps: the leader tells
+  // the peer the last licensed count, loads up to it itself, sends a stop
+  // marker through its stage ring, the MMA commits the partial accumulator and publishes the
+  // k-steps it holds to both CTAs, both epilogues spill their 128-row halves to the pair's slots,
+  // and the leader records {tile, next k-step, chunk end}. The pair with the same index in the
+  // next epoch restores both halves (tcgen05.st) and continues the k-loop: every k-step of every
+  // tile is accumulated once, in order (bit-identical to an uninterrupted run).
+  static constexpr uint32_t kInTilePoll = 4, kMinLeft = 4;
+  // the peer may run kLicSlack loads ahead of the leader; a stop then lets the leader catch up to
+  // the licensed count (kLicSlack more k-steps, < kMinLeft so they are in the same tile)
+#ifndef FLEP_GEMM2_LIC_SLACK
+#define FLEP_GEMM2_LIC_SLACK 2
+#endif
+  static constexpr uint32_t kLicSlack = FLEP_GEMM2_LIC_SLACK;
+  static_assert(kLicSlack <= kMinLeft, "the catch-up loads must stay inside the tile");
+  __device__ static float4* spill_slot(const WorkerParams& p, uint32_t wid, uint32_t r) {
+    return reinterpret_cast<float4*>(reinterpret_cast<uint8_t*>(p.partial) + partial_header_bytes(2 * p.workers) +
+                                     (size_t)(2 * wid + r) * kSpillBytes);
+  }
+  template <bool kCov, class Fetch>
+  __device__ static void worker_pipeline(const Gemm2Args& g, const WorkerParams& p, WorkerShared& ws,
+                                         uint32_t wid, uint32_t yield_sm, Fetch fetch) {
+    State* s = state();
+    uint8_t* base = ring();
+    const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31u;
+    const uint32_t r = rank();
+    const bool leader = r == 0;
+    const uint32_t nk = g.k / BK;
+    const bool in_tile = p.partial != nullptr;
+    const uint32_t gx = p.gx, gy = p.gy;
+    if (warp == 0 && lane == 0) {                       // ---- scheduler (leader) + TMA producers
+      uint32_t qi = 0, qph = 0, st = 0, ph = 0, q = 0;  // q: k-step loads issued (licence count)
+      const uint32_t full0 = peer_addr(&s->full[0], 0);
+      if (leader) {
+        const uint32_t lic_peer = peer_addr(&s->lic, 1), stop_peer = peer_addr(&s->stop_at, 1);
+        auto push = [&](uint32_t tile, uint32_t kb0) {
+          wait(&s->qempty[qi], qph ^ 1u);
+          s->tile_q[qi] = tile;
+          s->tile_kb0[qi] = kb0;
+          asm volatile("st.shared::cluster.u32 [%0], %1;" :: "r"(peer_addr(&s->tile_q[qi], 1)), "r"(tile) : "memory");
+          asm volatile("st.shared::cluster.u32 [%0], %1;" :: "r"(peer_addr(&s->tile_kb0[qi], 1)), "r"(kb0) : "memory");
+          arrive_local(&s->qfull[qi]);
+          arrive_remote(peer_addr(&s->qfull[qi], 1));
+          if (++qi == QDEPTH) { qi = 0; qph ^= 1u; }
+        };
+        PartialTile* mine = in_tile ? reinterpret_cast<PartialTile*>(p.partial) + wid : nullptr;
+        uint32_t rb0 = STOP, rb1 = 0, rkb = 0, q_stop = 0;
+        bool leave = false, stopping = false, stopped_in_tile = false;
+        SchedState sch;
+        if (in_tile) asm volatile("st.relaxed.cluster.shared::cluster.u32 [%0], %1;" :: "r"(lic_peer), "r"(kLicSlack) : "memory");
+        if (in_tile) {
+          if (p.epoch == p.gen_first) {
+            mine->valid = 0;
+          } else {
+            const PartialTile e = *mine;
+            if (e.valid) {
+              sch.first = false;
+              if (should_yield(poll_ctrl(p), p, yield_sm)) {      // entry check (a2)
+                ws.reason = kReasonYield;
+                ws.partial = e.b_end - e.b;
+                leave = true;
+              } else {
+                rb0 = e.b; rb1 = e.b_end; rkb = e.kb;
+                mine->valid = 0;
+                ws.blocks += e.b_end - e.b;
+              }
+            }
+          }
+        }
+        while (!leave) {
+          uint32_t b0, b1, kbs = 0;
+          bool restoring = false;
+          if (rb0 != STOP) {
+            b0 = rb0; b1 = rb1; kbs = rkb; restoring = true; rb0 = STOP;
+          } else {
+            if (!fetch(sch, b0, b1)) break;
+          }
+          for (uint32_t b = b0; b < b1; ++b) {
+            const uint32_t kb0 = (restoring && b == b0) ? kbs : 0u;
+            push(b, kb0);
+            if (kCov && !restoring) atomicAdd(&p.cov[b], 1u);
+            int32_t tm, tn;
+            tile_coords(b, gx, gy, tm, tn);
+            uint32_t kb = kb0, pend = 0;
+            bool pend_valid = false, stop = false;
+            for (; kb < nk; ++kb) {
+              if (in_tile) {
+                if (stopping) {                        // catching up to the licensed count
+                  if (q == q_stop) { stop = true; break; }
+                } else {                               // amortised in-tile poll (as GemmBody)
+                  const uint32_t j = kb - kb0;
+                  if (pend_valid && j % kInTilePoll == kInTilePoll / 2) {
+                    pend_valid = false;
+                    if (nk - kb > kMinLeft && should_yield(pend, p, yield_sm)) {
+                      // the peer loads nothing from licence q_stop on
+                      stopping = true;
+                      q_stop = q + kLicSlack;
+                      asm volatile("st.relaxed.cluster.shared::cluster.u32 [%0], %1;" :: "r"(stop_peer), "r"(q_stop) : "memory");
+                      if (q == q_stop) { stop = true; break; }
+                    }
+                  }
+#ifndef FLEP_X_NO_POLL
+                  if (j % kInTilePoll == 0 && j > 0) { pend = poll_ctrl(p); pend_valid = true; }
+#endif
+                }
+              }
+              wait(&s->empty[st], ph ^ 1u);
+              s->stage_stop[st] = 0u;
+              uint8_t* sa = base + st * kStage;
+              expect_tx(&s->full[st], 2 * kStage);
+              const uint32_t fb = full0 + st * 8u;
+              tma_2sm(&g.tma_a, sa, fb, (int32_t)(kb * BK), tm * (int32_t)TM);
+              tma_2sm(&g.tma_b, sa + kBytesA, fb, (int32_t)(kb * BK), tn * (int32_t)BN);
+              ++q;
+              // the licence orders nothing else (relaxed: a release here fences every k-step)
+              if (in_tile && !stopping)
+                asm volatile("st.relaxed.cluster.shared::cluster.u32 [%0], %1;" :: "r"(lic_peer), "r"(q + kLicSlack) : "memory");
+              if (++st == STAGES) { st = 0; ph ^= 1u; }
+            }
+            if (stop) {
+              // both CTAs loaded k-steps < kb; a data-less stop marker ends the MMA's tile
+              wait(&s->empty[st], ph ^ 1u);
+              s->stage_stop[st] = 1u;
+              arrive_local(&s->full[st]);
+              if (++st == STAGES) { st = 0; ph ^= 1u; }
+              mine->b = b; mine->kb = kb; mine->b_end = b1; mine->valid = 1;
+              if (kCov && !restoring)
+                for (uint32_t bb = b + 1; bb < b1; ++bb) atomicAdd(&p.cov[bb], 1u);
+              ws.blocks -= b1 - b;
+              ws.reason = kReasonYield;
+              ws.partial = b1 - b;
+              leave = stopped_in_tile = true;
+              break;
+            }
+          }
+        }
+        push(stopped_in_tile ? STOP_PARTIAL : STOP, 0);
+      } else {                                         // peer producer
+        while (true) {
+          wait(&s->qfull[qi], qph);
+          const uint32_t tile = s->tile_q[qi];
+          const uint32_t kb0 = s->tile_kb0[qi];
+          arrive_remote(peer_addr(&s->qempty[qi], 0));
+          if (++qi == QDEPTH) { qi = 0; qph ^= 1u; }
+          if (tile >= STOP_PARTIAL) break;
+          int32_t tm, tn;
+          tile_coords(tile, gx, gy, tm, tn);
+          bool stopped = false;
+          for (uint32_t kb = kb0; kb < nk; ++kb) {
+#ifndef FLEP_X_NO_LIC
+            if (in_tile) {                             // wait for the licence of load q (or a stop)
+              while (true) {
+                uint32_t l, sa_;
+                asm volatile("ld.relaxed.cluster.shared::cta.u32 %0, [%1];" : "=r"(l) : "r"(su32(&s->lic)) : "memory");
+                if (l > q) break;
+                asm volatile("ld.relaxed.cluster.shared::cta.u32 %0, [%1];" : "=r"(sa_) : "r"(su32(&s->stop_at)) : "memory");
+                if (sa_ == q) { stopped = true; break; }
+              }
+              if (stopped) break;
+            }
+#endif
+            wait(&s->empty[st], ph ^ 1u);
+            uint8_t* sa = base + st * kStage;
+            const uint32_t fb = full0 + st * 8u;
+            tma_2sm(&g.tma_a, sa, fb, (int32_t)(kb * BK), tm * (int32_t)TM + (int32_t)BM);
+            tma_2sm(&g.tma_b, sa + kBytesA, fb, (int32_t)(kb * BK), tn * (int32_t)BN + (int32_t)(BN / 2));
+            ++q;
+            if (++st == STAGES) { st = 0; ph ^= 1u; }
+          }
+          // after a stop the leader pushes STOP next: the loop ends there (the leader's ring is one
+          // stage ahead, the stop marker; the pair leaves, so the rings are not used again)
+        }
+      }
+    } else if (warp == 1 && lane == 0 && leader) {      // ---- MMA issuer (leader only)
+      uint32_t qi = 0, qph = 0, st = 0, ph = 0, acc = 0, aph = 0;
+      uint32_t rph[2] = {0u, 0u};
+      const uint32_t tmem0 = s->tmem_base;
+      while (true) {
+        wait(&s->qfull[qi], qph);
+        const uint32_t tile = s->tile_q[qi];
+        const uint32_t kb0 = s->tile_kb0[qi];
+        arrive_local(&s->qempty[qi]);
+        if (++qi == QDEPTH) { qi = 0; qph ^= 1u; }
+        if (tile >= STOP_PARTIAL) break;
+        wait(&s->tempty[acc], aph ^ 1u);
+        if (kb0 > 0) { wait(&s->trest[acc], rph[acc]); rph[acc] ^= 1u; }   // both halves restored
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        const uint32_t tmem = tmem0 + acc * BN;
+        uint32_t kb = kb0;
+        for (; kb < nk; ++kb) {
+          wait(&s->full[st], ph);
+          if (s->stage_stop[st]) {                     // stop marker (the pair leaves: the rings
+            arrive_local(&s->empty[st]);               // are not used again)
+            if (++st == STAGES) { st = 0; ph ^= 1u; }
+            break;
+          }
+          asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+          const uint32_t sa = su32(base + st * kStage), sb = sa + kBytesA;
+#pragma unroll
+          for (uint32_t k = 0; k < BK / UMMA_K; ++k) {
+            const uint64_t da = sdesc(sa + k * UMMA_K * 2), db = sdesc(sb + k * UMMA_K * 2);
+            const uint32_t accum = (kb | k) ? 1u : 0u;
+            asm volatile(
+                "{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n"
+                " tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n}\n"
+                :: "r"(tmem), "l"(da), "l"(db), "r"(kIdesc), "r"(accum) : "memory");
+          }
+          asm volatile("tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;"
+                       :: "r"(su32(&s->empty[st])), "h"((uint16_t)3) : "memory");
+          if (++st == STAGES) { st = 0; ph ^= 1u; }
+        }
+        asm volatile("tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;"
+                     :: "r"(su32(&s->tfull[acc])), "h"((uint16_t)3) : "memory");
+        if (++acc == 2) { acc = 0; aph ^= 1u; }
+      }
+    } else if (warp >= 4) {                              // ---- epilogue: this CTA's 128 rows
+      const uint32_t qw = warp - 4;
+      const uint32_t rl = qw * 32u + lane;
+      uint32_t qi = 0, qph = 0, acc = 0, aph = 0;
+      const uint32_t tempty0 = peer_addr(&s->tempty[0], 0), trest0 = peer_addr(&s->trest[0], 0);
+      while (true) {
+        wait(&s->qfull[qi], qph);
+        const uint32_t tile = s->tile_q[qi];
+        const uint32_t kb0 = s->tile_kb0[qi];
+        __syncwarp();
+        if (lane == 0) {
+          if (leader) arrive_local(&s->qempty[qi]);
+          else arrive_remote(peer_addr(&s->qempty[qi], 0));
+        }
+        if (++qi == QDEPTH) { qi = 0; qph ^= 1u; }
+        if (tile >= STOP_PARTIAL) break;
+        int32_t tm, tn;
+        tile_coords(tile, gx, gy, tm, tn);
+        const uint32_t tmem = s->tmem_base + acc * BN + ((qw * 32u) << 16);
+        if (kb0 > 0) {                                   // restore this CTA's spilled half
+          const float4* src = spill_slot(p, wid, r);     // layout [col/4][row]: coalesced
+#pragma unroll 1
+          for (uint32_t c0 = 0; c0 < BN; c0 += 32) {
+            uint32_t v[32];
+#pragma unroll
+            for (int j = 0; j < 8; ++j) {
+              const float4 f = __ldcs(src + (size_t)(c0 / 4 + j) * BM + rl);
+              v[4 * j] = __float_as_uint(f.x); v[4 * j + 1] = __float_as_uint(f.y);
+              v[4 * j + 2] = __float_as_uint(f.z); v[4 * j + 3] = __float_as_uint(f.w);
+            }
+            GemmBody::tmem_st32(tmem + c0, v);
+          }
+          asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+          asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+          __syncwarp();
+          if (lane == 0) {
+            if (leader) arrive_local(&s->trest[acc]);
+            else arrive_remote(trest0 + acc * 8u);
+          }
+        }
+        wait(&s->tfull[acc], aph);
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        // stopped inside the tile iff the queue's next entry is STOP_PARTIAL (a stop is always
+        // the pair's last tile; the leader pushes the next entry before this tile's MMAs end, so
+        // the peek costs nothing; a remote publish from the MMA thread would fence its pipeline)
+#ifndef FLEP_X_NO_PEEK
+        wait(&s->qfull[qi], qph);
+        if (s->tile_q[qi] == STOP_PARTIAL) {
+#else
+        if (false) {
+#endif
+          float4* dst = spill_slot(p, wid, r);
+#pragma unroll 1
+          for (uint32_t c0 = 0; c0 < BN; c0 += 32) {
+            uint32_t v[32];
+            GemmBody::tmem_ld32(tmem + c0, v);
+#pragma unroll
+            for (int j = 0; j < 8; ++j)
+              __stcs(dst + (size_t)(c0 / 4 + j) * BM + rl,
+                     make_float4(__uint_as_float(v[4 * j]), __uint_as_float(v[4 * j + 1]),
+                                 __uint_as_float(v[4 * j + 2]), __uint_as_float(v[4 * j + 3])));
+          }
+        } else {
+          const uint32_t row = (uint32_t)tm * TM + r * BM + rl;
+          __nv_bfloat16* crow = g.c + (size_t)row * g.n + (size_t)tn * BN;
+#pragma unroll 1
+          for (uint32_t c0 = 0; c0 < BN; c0 += 32) {
+            uint32_t v[32];
+            GemmBody::tmem_ld32(tmem + c0, v);
+            uint4 o[4];
+            uint32_t* ow = reinterpret_cast<uint32_t*>(o);
+#pragma unroll
+            for (int i = 0; i < 16; ++i) {
+              __nv_bfloat162 h = __floats2bfloat162_rn(__uint_as_float(v[2 * i]), __uint_as_float(v[2 * i + 1]));
+              ow[i] = *reinterpret_cast<uint32_t*>(&h);
+            }
+            uint4* dst = reinterpret_cast<uint4*>(crow + c0);
+#pragma unroll
+            for (int i = 0; i < 4; ++i) dst[i] = o[i];
+          }
+        }
+        asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+        __syncwarp();
+        if (lane == 0) {
+          if (leader) arrive_local(&s->tempty[acc]);
+          else arrive_remote(tempty0 + acc * 8u);
+        }
+        if (++acc == 2) { acc = 0; aph ^= 1u; }
+      }
+    }
+  }
 };
 
 // Worker (the PAIR is the FLEP worker: wid = cluster index, W = pairs). The leader runs the
@@ -308,15 +630,24 @@ flep_gemm2_worker(const __grid_constant__ Gemm2Args g, const WorkerParams p) {
     yield_sm = p.rank[peer_sm] < p.rank[ws.sm] ? peer_sm : ws.sm;
     ws.sm = yield_sm;                                  // the worker record names the deciding SM
   }
-  SchedState st;
-  Gemm2::pipeline(g, p.gx, p.gy, [&](uint32_t& b0, uint32_t& b1) {
-    b0 = next_chunk(p, st, ws, wid, yield_sm);
-    if (b0 == 0xffffffffu) return false;
-    b1 = min(b0 + p.chunk, p.n_blocks);
-    if (kCoverage)
-      for (uint32_t b = b0; b < b1; ++b) atomicAdd(&p.cov[b], 1u);
-    return true;
-  });
+  if (p.partial) {                                     // in-tile preemption (R21 on the pair)
+    Gemm2::worker_pipeline<kCoverage>(g, p, ws, wid, yield_sm, [&](SchedState& st, uint32_t& b0, uint32_t& b1) {
+      b0 = next_chunk(p, st, ws, wid, yield_sm);
+      if (b0 == 0xffffffffu) return false;
+      b1 = min(b0 + p.chunk, p.n_blocks);
+      return true;
+    });
+  } else {
+    SchedState st;
+    Gemm2::pipeline(g, p.gx, p.gy, [&](uint32_t& b0, uint32_t& b1) {
+      b0 = next_chunk(p, st, ws, wid, yield_sm);
+      if (b0 == 0xffffffffu) return false;
+      b1 = min(b0 + p.chunk, p.n_blocks);
+      if (kCoverage)
+        for (uint32_t b = b0; b < b1; ++b) atomicAdd(&p.cov[b], 1u);
+      return true;
+    });
+  }
   Gemm2::teardown();
   if (leader && threadIdx.x == 0) worker_exit(p, ws, wid);
 }

@@ -350,7 +350,9 @@ flep_status materialize(flep_rt rt, Launch& L) {
   if (L.flags & (FLEP_KFLAG_IN_TILE | FLEP_KFLAG_IN_CHUNK)) {
     // per-worker partial-tile records (and, in-tile, fp32 accumulator spill slots); no reset
     // needed (the first epoch's workers clear their records)
-    const size_t need = (L.flags & FLEP_KFLAG_IN_TILE) ? partial_bytes(L.workers) : partial_header_bytes(L.workers);
+    // (a CTA pair spills two 128-row halves: one record per pair, one slot per CTA)
+    const uint32_t slots = L.ops->max_pairs ? 2 * L.workers : L.workers;
+    const size_t need = (L.flags & FLEP_KFLAG_IN_TILE) ? partial_bytes(slots) : partial_header_bytes(L.workers);
     size_t best = rt->free_partial.size();
     for (size_t i = 0; i < rt->free_partial.size(); ++i)
       if (rt->free_partial[i].second >= need &&
@@ -905,8 +907,8 @@ flep_status flep_device_info(flep_rt rt, uint32_t* num_sms, uint32_t* nsmid) {
 flep_status flep_register_kernel(flep_rt rt, const flep_kernel_desc* d, flep_kernel* out) {
   if (!rt || !d || !out) return fail(FLEP_ERR_INVALID, "NULL argument");
   if (!body_ops(d->body)) return fail(FLEP_ERR_INVALID, "unknown body %d", d->body);
-  if ((d->flags & FLEP_KFLAG_IN_TILE) && d->body != FLEP_BODY_GEMM_BF16)
-    return fail(FLEP_ERR_UNSUPPORTED, "in-tile preemption is implemented for the GEMM body only");
+  if ((d->flags & FLEP_KFLAG_IN_TILE) && d->body != FLEP_BODY_GEMM_BF16 && d->body != FLEP_BODY_GEMM_BF16_2SM)
+    return fail(FLEP_ERR_UNSUPPORTED, "in-tile preemption is implemented for the GEMM bodies only");
   if ((d->flags & FLEP_KFLAG_IN_TILE) && (d->flags & FLEP_KFLAG_PREFETCH))
     return fail(FLEP_ERR_UNSUPPORTED, "in-tile preemption does not combine with chunk prefetch");
   if (d->flags & FLEP_KFLAG_IN_CHUNK) {

@@ -2,7 +2,8 @@
 against the oracle (fp64 from the same bf16 inputs): the unwrapped pair-per-tile grid, the static
 persistent twin and the FLEP pair workers give bit-identical C; preempt/resume cycles (temporal
 and spatial) stay bit-identical with every tile run once; a spatial request releases exactly the
-pairs that have a named SM."""
+pairs that have a named SM; with in-tile preemption (R21 + R32) the pair stops inside a tile,
+spills both accumulator halves and the next epoch's pair continues it, bit-identically."""
 import numpy as np
 import pytest
 
@@ -159,3 +160,71 @@ def test_gemm2_sliced_with_device_check_preempted():
         assert acts[:3] == ["LAUNCH", "PREEMPT", "LAUNCH"]
     finally:
         rs.close()
+
+
+@pytest.mark.parametrize("chunk", [1, 2])
+def test_gemm2_in_tile_random_schedules_bitexact(rt, chunk):
+    """In-tile preemption on the CTA pair: random temporal/spatial schedules stop pairs inside
+    tiles (both 128-row halves spilled, restored by the pair with the same index next epoch).
+    Every schedule: every tile once, C bit-identical to the unwrapped grid, and some epochs
+    really ended with tiles stopped mid-way."""
+    import torch
+    f = flep_mod()
+    m, n, k = 2048, 2048, 4096                      # 64 tiles of 256x256, 64 k-steps each
+    a_bits, b_bits = gen.gemm_bf16_inputs(m, n, k, seed=175 + chunk)
+    A, B = _bf16(a_bits), _bf16(b_bits)
+    grid = f.gemm2_grid(m, n)
+    ntiles = grid[0] * grid[1]
+    C0 = torch.empty((m, n), dtype=torch.bfloat16, device="cuda")
+    rt.launch_unwrapped(f.BODY_GEMM_BF16_2SM, grid, f.gemm_args(C0, A, B))
+    torch.cuda.synchronize()
+    _check(C0, W.gemm_bf16(a_bits, b_bits))
+    kk = rt.register_kernel(f.BODY_GEMM_BF16_2SM, chunk=chunk, poll=1, in_tile=True)
+    C1 = torch.empty((m, n), dtype=torch.bfloat16, device="cuda")
+    stats, bad = {}, []
+    for i in range(24):
+        s = gen.preempt_schedule(1800 + 50 * chunk + i, ntiles, rt.num_sms)
+        C1.fill_(float("nan"))
+        h, npre, viol = run_manual_schedule(rt, kk, grid, f.gemm_args(C1, A, B), ntiles, s, rt.num_sms,
+                                            check_prefix=False, stats=stats)
+        if not np.all(rt.coverage_np(h, ntiles) == 1):
+            viol.append("I1: coverage != 1")
+        if not torch.equal(C0.view(torch.int16), C1.view(torch.int16)):
+            viol.append("C differs from the uninterrupted run")
+        if viol:
+            bad.append((i, s, viol))
+    assert not bad, bad[:3]
+    assert stats.get("partial_epochs", 0) > 3       # tiles really were stopped mid-way
+
+
+def test_gemm2_in_tile_latency_below_tile_time(rt):
+    """A temporal request drains the in-tile pair GEMM in far less than one tile's compute time
+    (k = 8192: 128 k-steps per 256x256 tile)."""
+    import torch
+    f = flep_mod()
+    m = n = 4096
+    k = 8192
+    a_bits, b_bits = gen.gemm_bf16_inputs(m, n, k, seed=178)
+    A, B = _bf16(a_bits), _bf16(b_bits)
+    grid = f.gemm2_grid(m, n)
+    C0 = torch.empty((m, n), dtype=torch.bfloat16, device="cuda")
+    rt.launch_unwrapped(f.BODY_GEMM_BF16_2SM, grid, f.gemm_args(C0, A, B))
+    torch.cuda.synchronize()
+    _, pairs = rt.workers_for(f.BODY_GEMM_BF16_2SM)
+    C = torch.empty((m, n), dtype=torch.bfloat16, device="cuda")
+    out = {}
+    for in_tile in (False, True):
+        kk = rt.register_kernel(f.BODY_GEMM_BF16_2SM, chunk=1, poll=1, in_tile=in_tile)
+        lat = []
+        for rep in range(3):
+            rt.arm_next_trigger(pairs + 10, rt.num_sms)   # after the static first wave
+            h = rt.launch(kk, grid, f.gemm_args(C, A, B))
+            rt.wait_epoch(h, timeout_ns=20_000_000_000)
+            assert rt.query(h).state == f.STATE_PREEMPTED
+            ep = rt.epoch_info(h, 1)
+            lat.append((ep.t_end - ep.t_trigger) / 1e3)
+            rt.resume(h)
+            rt.sync(h, timeout_ns=20_000_000_000)
+            assert torch.equal(C, C0)
+        out[in_tile] = float(np.median(lat))
+    assert out[True] < 0.5 * out[False], out

@@ -30,6 +30,7 @@ def main():
     k1 = {c: rt.register_kernel(F.BODY_GEMM_BF16, chunk=c, poll=1) for c in (1, 2)}
     k1t = rt.register_kernel(F.BODY_GEMM_BF16, chunk=2, poll=1, in_tile=True)
     k2 = {c: rt.register_kernel(F.BODY_GEMM_BF16_2SM, chunk=c, poll=1) for c in (1, 2)}
+    k2t = rt.register_kernel(F.BODY_GEMM_BF16_2SM, chunk=1, poll=1, in_tile=True)
     variants = {
         "cublas": lambda: (torch.matmul(A, B.t(), out=C), None)[1],
         "gemm1_unwrapped": lambda: rt.launch_unwrapped(F.BODY_GEMM_BF16, g1, args, stream=s),
@@ -41,7 +42,11 @@ def main():
         "gemm2_static_u1": lambda: rt.launch_static(F.BODY_GEMM_BF16_2SM, g2, args, stream=s),
         "gemm2_flep_c1": lambda: rt.launch(k2[1], g2, args, stream=s),
         "gemm2_flep_c2": lambda: rt.launch(k2[2], g2, args, stream=s),
+        "gemm2_flep_c1_intile": lambda: rt.launch(k2t, g2, args, stream=s),
     }
+    only = os.environ.get("GEMM_ONLY")                 # comma list: a subset of the variants
+    if only:
+        variants = {k: v for k, v in variants.items() if k in only.split(",") or k == "cublas"}
     ts = {k: [] for k in variants}
     with ClockSampler(0) as clk:
         for r in range(reps + 2):

@@ -85,7 +85,7 @@ def main():
         rt.resume(h)
     rt.sync(h)
     # round 2: warp-task workers (SpMV vector body, stencil) with a temporal preempt/resume cycle,
-    # the static persistent twin, the CTA-pair GEMM (unwrapped, static, worker with a preemption)
+    # the static persistent twin, the CTA-pair GEMM (unwrapped, static, worker with a preemption, in-tile worker)
     # and device-checked slicing with a preemption
     k9 = rt.register_kernel(F.BODY_SPMV_CSR_F32_VEC, chunk=2, poll=1, warp_tasks=True)
     rt.arm_next_trigger(4, rt.num_sms)
@@ -107,6 +107,17 @@ def main():
     k11 = rt.register_kernel(F.BODY_GEMM_BF16_2SM, chunk=1, poll=1)
     rt.arm_next_trigger(1, rt.num_sms)
     h = rt.launch(k11, g2, F.gemm_args(C2, A2, B2))
+    rt.wait_epoch(h)
+    if rt.query(h).state == F.STATE_PREEMPTED:
+        rt.resume(h)
+    rt.sync(h)
+    k12 = rt.register_kernel(F.BODY_GEMM_BF16_2SM, chunk=1, poll=1, in_tile=True)
+    a_bits, b_bits = gen.gemm_bf16_inputs(512, 512, 1024, 9)
+    A3 = torch.from_numpy(a_bits.view(np.int16)).cuda().view(torch.bfloat16)
+    B3 = torch.from_numpy(b_bits.view(np.int16)).cuda().view(torch.bfloat16)
+    C3 = torch.empty(512, 512, dtype=torch.bfloat16, device="cuda")
+    rt.arm_next_trigger(1, rt.num_sms)
+    h = rt.launch(k12, g2, F.gemm_args(C3, A3, B3))
     rt.wait_epoch(h)
     if rt.query(h).state == F.STATE_PREEMPTED:
         rt.resume(h)
