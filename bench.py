@@ -255,8 +255,10 @@ def run_temporal(args, rank, world, local):
     B = torch.cuda.Stream(priority=0)
     rt = F.Runtime(device=local, exec_on_user_stream=True)
     num_sms = rt.num_sms
+    # the victim fetches speculatively (R34): poll and fetch in one round trip, a fetched chunk is
+    # returned through the worker's record on a stop
     kLP = rt.register_kernel(F.BODY_SPMV_CSR_F32, chunk=args.lp_chunk, poll=args.lp_poll, name="spmv",
-                             prefetch=bool(args.prefetch))
+                             prefetch=bool(args.prefetch), spec_fetch=bool(args.lp_spec))
     # the waiting (high-priority) kernel is never preempted here: it is tuned for throughput (CLC
     # task fetch, C = 1, K = 4: 4.6 % over the unwrapped grid vs 19 % for the counter worker,
     # profiles/r01_bench_clc.json), the victim for latency (atomic counter, C = K = 1)
@@ -377,7 +379,8 @@ def run_temporal(args, rank, world, local):
     # per 256 rows; measured with the same steps, the same kernel timing protocol
     op2 = None
     if args.lp_chunk == 1 and args.op2:
-        kLP2 = rt.register_kernel(F.BODY_SPMV_CSR_F32, chunk=2, poll=args.lp_poll, name="spmv-c2")
+        kLP2 = rt.register_kernel(F.BODY_SPMV_CSR_F32, chunk=2, poll=args.lp_poll, name="spmv-c2",
+                                  spec_fetch=bool(args.lp_spec))
         for _ in range(args.warmup):
             step(kLP2)
         r2 = [step(kLP2) for _ in range(args.steps)]
@@ -411,7 +414,7 @@ def run_temporal(args, rank, world, local):
                                f"{wl.nnz} nnz, low priority) by stencil5 fp32 4096^2 (high priority)",
                    "lp_chunk": args.lp_chunk, "lp_poll": args.lp_poll, "hp_chunk": args.hp_chunk, "hp_poll": args.hp_poll, "hp_clc": bool(args.hp_clc), "hp_prefetch": bool(args.hp_prefetch),
                    "hp_async_poll": bool(args.hp_async),
-                   "prefetch": bool(args.prefetch),
+                   "prefetch": bool(args.prefetch), "lp_spec_fetch": bool(args.lp_spec),
                    "flag": "stream_memop (device self-trigger for the request)",
                    "l2": "flushed between steps (write of 2x L2 bytes)", "parallelism": f"replicas x{world}"},
         "value_definition": "full-GPU preemption latency (device %globaltimer): request visible on the GPU -> "
@@ -547,7 +550,7 @@ def run_e2e(F, torch, wl, local, steps, args, diag=False):
     rt = F.Runtime(device=local, policy=F.POLICY_HPF)
     kLP = rt.register_kernel(F.BODY_SPMV_CSR_F32, chunk=args.lp_chunk, poll=args.lp_poll, name="spmv",
                              model=(0, 0, 0, 0, 70_000), prefetch=bool(args.prefetch), started_hint=True,
-                             host_relay=bool(args.e2e_relay))
+                             host_relay=bool(args.e2e_relay), spec_fetch=bool(args.lp_spec))
     kHP = rt.register_kernel(F.BODY_STENCIL5_F32, chunk=args.hp_chunk, poll=args.hp_poll, name="stencil",
                              model=(0, 0, 0, 0, 30_000), prefetch=bool(args.hp_prefetch), async_poll=bool(args.hp_async),
                              clc=bool(args.hp_clc))
@@ -756,6 +759,7 @@ def main():
     ap.add_argument("--hp-prefetch", type=int, default=0)
     ap.add_argument("--hp-async", type=int, default=0, help="waiting kernel: async poll (R22)")
     ap.add_argument("--lp-poll", type=int, default=1)
+    ap.add_argument("--lp-spec", type=int, default=1, help="victim: speculative fetch (R34)")
     ap.add_argument("--reps", type=int, default=40)
     ap.add_argument("--e2e-relay", type=int, default=1, help="e2e victim with the request-relay CTA (R28)")
     ap.add_argument("--e2e-overlap-copy", type=int, default=0, help="e2e: let the HP's input copy overlap the co-run")

@@ -254,6 +254,7 @@ struct SchedState {
   bool stopping = false;             // a request named this SM; drain the held chunk
   bool first = true;                 // first step of this worker
   uint32_t snext = 0xffffffffu;      // static twin (U1): the next chunk base of this worker
+  bool want_fetch = false;           // R34 with prefetch: issue the next fetch after the barrier
 };
 
 // pull_task. In the first epoch of a launch the counter hands out blocks after the W
@@ -299,8 +300,26 @@ __device__ __forceinline__ void note_exit_event(const WorkerParams& p, WorkerSha
   ws.ev_part = (uint32_t)(old >> 48) + own_partial;
 }
 
+// A worker that must leave holding a fetched, unstarted chunk (speculative fetch, R34): an
+// exhausted fetch is its exit event (R23); otherwise the chunk goes to the worker's record, run
+// first by the worker with the same index next epoch (the chunk-rest record of R33).
+__device__ __forceinline__ void return_chunk(const WorkerParams& p, WorkerShared& ws, PartialTile* rec,
+                                             unsigned long long w) {
+  const uint32_t b = (uint32_t)w + ctr_offset(p);
+  if (b >= p.n_blocks) {
+    note_exit_event(p, ws, w, p.chunk, 0u);
+    ws.reason = kReasonExhausted;
+  } else {
+    const uint32_t e = min(b + p.chunk, p.n_blocks);
+    rec->b = b; rec->kb = 0; rec->b_end = e; rec->valid = 1;
+    ws.partial = e - b;                              // the epoch cannot complete (R23)
+    ws.reason = kReasonYield;
+  }
+}
+
 __device__ __forceinline__ uint32_t next_chunk(const WorkerParams& p, SchedState& st, WorkerShared& ws,
-                                               uint32_t wid = blockIdx.x, uint32_t yield_sm = 0xffffffffu) {
+                                               uint32_t wid = blockIdx.x, uint32_t yield_sm = 0xffffffffu,
+                                               PartialTile* rec = nullptr) {
   // the SM whose rank a spatial request is checked against (a CTA pair passes its lower-ranked SM)
   const auto my_sm = [&]() { return yield_sm != 0xffffffffu ? yield_sm : smid_reg(); };
   if (p.static_sched) {              // U1 twin: a fixed schedule, nothing shared, never preempted
@@ -331,16 +350,39 @@ __device__ __forceinline__ uint32_t next_chunk(const WorkerParams& p, SchedState
       if (should_yield(c, p, my_sm())) { ws.reason = kReasonYield; return 0xffffffffu; }
     }
   } else if (st.k == 0 && !st.stopping) {            // amortised poll (Fig. 4(b))
-    // async poll (FLEP_KFLAG_ASYNC_POLL, reading R22): use the word loaded at the previous step,
-    // so no round trip sits between two chunks; a request is then acted on one chunk later
-    const uint32_t c = (p.async_poll && st.have_seen) ? poll_consume(ws) : poll_ctrl(p);
-    if (should_yield(c, p, my_sm())) { st.stopping = true; ws.reason = kReasonYield; }
+#ifndef FLEP_NO_SPEC_FETCH
+    if (rec && !p.async_poll && st.held == ~0ull) {
+      // speculative fetch (reading R34): the fetch and the poll are in flight together, one
+      // round trip instead of two back to back; a chunk fetched by a worker that must leave is
+      // not run but returned through its record (the chunk-rest record of R33), which the worker
+      // with the same index runs first in the next epoch, so a request still costs one chunk
+      const unsigned long long w = fetch_chunk(p);
+      const uint32_t c = poll_ctrl(p);
+      if (should_yield(c, p, my_sm())) {
+        st.stopping = true;
+        return_chunk(p, ws, rec, w);
+        return 0xffffffffu;
+      }
+      st.held = w;                                   // consumed just below
+    } else
+#endif
+    {
+      // async poll (FLEP_KFLAG_ASYNC_POLL, reading R22): use the word loaded at the previous step,
+      // so no round trip sits between two chunks; a request is then acted on one chunk later
+      const uint32_t c = (p.async_poll && st.have_seen) ? poll_consume(ws) : poll_ctrl(p);
+      if (should_yield(c, p, my_sm())) { st.stopping = true; ws.reason = kReasonYield; }
+    }
   }
 #ifdef FLEP_TRACE
   ws.t_poll = gtimer();
 #endif
   if (!have) {
     unsigned long long w = ~0ull;
+    if (st.held != ~0ull && st.stopping && rec) {    // R34 with prefetch: return the held chunk
+      return_chunk(p, ws, rec, st.held);
+      st.held = ~0ull;
+      return 0xffffffffu;
+    }
     if (st.held != ~0ull) {                          // a fetched chunk is always processed (A4)
       w = st.held;
       st.held = ~0ull;
@@ -359,7 +401,10 @@ __device__ __forceinline__ uint32_t next_chunk(const WorkerParams& p, SchedState
 #endif
   if (base != 0xffffffffu) {
     ws.blocks += min(p.chunk, p.n_blocks - base);
-    if (p.prefetch && !st.stopping) st.held = fetch_chunk(p);   // overlaps the body
+    if (p.prefetch && !st.stopping) {                // overlaps the body
+      if (rec) st.want_fetch = true;                 // R34: issued after the chunk barrier
+      else st.held = fetch_chunk(p);
+    }
     if (p.trigger_block - base < p.chunk) {          // device self-trigger inside this chunk
       const uint32_t e = p.epoch % kEvEpochs;
       p.cb->ep_t_trigger[e] = gtimer();
@@ -456,6 +501,26 @@ __device__ __forceinline__ void request_relay(const WorkerParams& p) {
   p.cb->ep_relay_t[e] = gtimer();
 }
 
+// A chunk returned through the worker's record by the previous epoch (speculative fetch, R34):
+// returns its first block, kRestLeave if the entry check says leave at once (the record stays),
+// or 0xffffffff if there is none (the first epoch clears the record).
+constexpr uint32_t kRestLeave = 0xfffffffeu;
+__device__ __forceinline__ uint32_t take_rest(const WorkerParams& p, SchedState& st, WorkerShared& ws,
+                                              PartialTile* rec) {
+  if (p.epoch == p.gen_first) { rec->valid = 0; return 0xffffffffu; }
+  const PartialTile e = *rec;                          // written by the previous grid
+  if (!e.valid) return 0xffffffffu;
+  st.first = false;                                    // (the launch is not complete)
+  if (should_yield(poll_ctrl(p), p, smid_reg())) {     // entry check (a2)
+    ws.reason = kReasonYield;
+    ws.partial = e.b_end - e.b;
+    return kRestLeave;
+  }
+  rec->valid = 0;
+  ws.blocks += e.b_end - e.b;
+  return e.b;
+}
+
 // The worker. Body contract:
 //   Body::kThreads               CTA size of the original kernel
 //   Body::kMinBlocks             resident CTAs per SM the register budget is sized for
@@ -486,6 +551,11 @@ flep_worker(const __grid_constant__ typename Body::Args args, const WorkerParams
   } else {
     SchedState st;
     uint32_t parity = 0;
+    // speculative fetch (FLEP_KFLAG_SPEC_FETCH, reading R34): a chunk returned by the previous
+    // epoch's worker with this index is run first (after the entry check)
+    PartialTile* rec = p.partial ? reinterpret_cast<PartialTile*>(p.partial) + blockIdx.x : nullptr;
+    uint32_t rest = 0xffffffffu;
+    if (rec && tid == 0) rest = take_rest(p, st, ws, rec);
 #ifdef FLEP_TRACE
     uint32_t nchunk = 0;
 #endif
@@ -495,7 +565,10 @@ flep_worker(const __grid_constant__ typename Body::Args args, const WorkerParams
       // body done), when the poll decision was taken, when the step returned (fetch done) and
       // when the chunk barrier released it (the slowest warp of the previous body)
       const uint64_t ta = (tid == 0 && p.trace) ? gtimer() : 0;
-      if (tid == 0) s_slot[parity] = next_chunk(p, st, ws);
+      if (tid == 0) {
+        if (rest != 0xffffffffu) { s_slot[parity] = rest == kRestLeave ? 0xffffffffu : rest; rest = 0xffffffffu; }
+        else s_slot[parity] = next_chunk(p, st, ws, blockIdx.x, 0xffffffffu, rec);
+      }
       const uint64_t tb = (tid == 0 && p.trace) ? gtimer() : 0;
       __syncthreads();
       if (tid == 0 && p.trace && nchunk < kTraceChunks) {
@@ -504,12 +577,16 @@ flep_worker(const __grid_constant__ typename Body::Args args, const WorkerParams
       }
       ++nchunk;
 #else
-      if (tid == 0) s_slot[parity] = next_chunk(p, st, ws);
+      if (tid == 0) {
+        if (rest != 0xffffffffu) { s_slot[parity] = rest == kRestLeave ? 0xffffffffu : rest; rest = 0xffffffffu; }
+        else s_slot[parity] = next_chunk(p, st, ws, blockIdx.x, 0xffffffffu, rec);
+      }
       __syncthreads();
 #endif
       const uint32_t b0 = s_slot[parity];
       parity ^= 1u;
       if (b0 == 0xffffffffu) break;
+      if (tid == 0 && st.want_fetch) { st.held = fetch_chunk(p); st.want_fetch = false; }
       const uint32_t b1 = min(b0 + p.chunk, p.n_blocks);
       Body::run(args, b0, b1, p.gx, p.gy);
       if (kCoverage && tid == 0)
@@ -572,7 +649,7 @@ flep_worker_ic(const __grid_constant__ typename Body::Args args, const WorkerPar
         }
       }
       if (!leave && b0 == STOP) {
-        b0 = next_chunk(p, st, ws);
+        b0 = next_chunk(p, st, ws, blockIdx.x, 0xffffffffu, mine);
         b1 = b0 == STOP ? 0u : min(b0 + p.chunk, p.n_blocks);
       }
       s_rng[par][0] = leave ? STOP : b0;

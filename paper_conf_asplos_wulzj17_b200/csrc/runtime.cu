@@ -347,7 +347,7 @@ flep_status materialize(flep_rt rt, Launch& L) {
     }
     if (!L.cov) { L.cov_cap = std::max<size_t>(N, 4096); CUDA_TRY(cudaMalloc(&L.cov, L.cov_cap * 4)); }
   }
-  if (L.flags & (FLEP_KFLAG_IN_TILE | FLEP_KFLAG_IN_CHUNK)) {
+  if (L.flags & (FLEP_KFLAG_IN_TILE | FLEP_KFLAG_IN_CHUNK | FLEP_KFLAG_SPEC_FETCH)) {
     // per-worker partial-tile records (and, in-tile, fp32 accumulator spill slots); no reset
     // needed (the first epoch's workers clear their records)
     // (a CTA pair spills two 128-row halves: one record per pair, one slot per CTA)
@@ -919,6 +919,14 @@ flep_status flep_register_kernel(flep_rt rt, const flep_kernel_desc* d, flep_ker
                     FLEP_KFLAG_IN_TILE))
       return fail(FLEP_ERR_UNSUPPORTED, "in-chunk stop does not combine with prefetch, CLC, the scheduling warp, "
                                         "warp tasks or in-tile preemption");
+  }
+  if (d->flags & FLEP_KFLAG_SPEC_FETCH) {
+    if (d->body == FLEP_BODY_GEMM_BF16 || d->body == FLEP_BODY_GEMM_BF16_2SM)
+      return fail(FLEP_ERR_UNSUPPORTED, "the speculative fetch is for the counter worker of the memory-bound bodies");
+    if (d->flags & (FLEP_KFLAG_ASYNC_POLL | FLEP_KFLAG_CLC | FLEP_KFLAG_SCHED_WARP | FLEP_KFLAG_WARP_TASKS |
+                    FLEP_KFLAG_IN_TILE))
+      return fail(FLEP_ERR_UNSUPPORTED, "the speculative fetch does not combine with async poll, CLC, "
+                                        "the scheduling warp, warp tasks or in-tile preemption");
   }
   ApiLock lk(rt);
   if (d->flags & FLEP_KFLAG_IN_TILE) {

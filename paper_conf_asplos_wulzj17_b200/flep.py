@@ -35,6 +35,7 @@ KFLAG_SCHED_WARP = 32
 KFLAG_HOST_RELAY = 64
 KFLAG_WARP_TASKS = 128
 KFLAG_IN_CHUNK = 256
+KFLAG_SPEC_FETCH = 512
 WARP_TASKS_PER_BLOCK = 8
 
 
@@ -224,12 +225,13 @@ class Runtime:
 
     def register_kernel(self, body, chunk=0, poll=0, name="", model=(0, 0, 0, 0, 1), overhead_ns=0,
                         prefetch=False, ctas_per_sm=0, started_hint=False, in_tile=False, async_poll=False,
-                        clc=False, sched_warp=False, host_relay=False, warp_tasks=False, in_chunk=False):
+                        clc=False, sched_warp=False, host_relay=False, warp_tasks=False, in_chunk=False,
+                        spec_fetch=False):
         flags = ((KFLAG_PREFETCH if prefetch else 0) | (KFLAG_STARTED_HINT if started_hint else 0)
                  | (KFLAG_IN_TILE if in_tile else 0) | (KFLAG_ASYNC_POLL if async_poll else 0)
                  | (KFLAG_CLC if clc else 0) | (KFLAG_SCHED_WARP if sched_warp else 0)
                  | (KFLAG_HOST_RELAY if host_relay else 0) | (KFLAG_WARP_TASKS if warp_tasks else 0)
-                 | (KFLAG_IN_CHUNK if in_chunk else 0))
+                 | (KFLAG_IN_CHUNK if in_chunk else 0) | (KFLAG_SPEC_FETCH if spec_fetch else 0))
         d = KernelDesc(name.encode(), body, chunk, poll, (C.c_double * 5)(*model), overhead_ns,
                        flags, ctas_per_sm)
         k = C.c_int32()

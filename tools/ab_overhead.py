@@ -5,7 +5,8 @@ of the workers (first entry -> last exit, %globaltimer) so that launch / teardow
 span is visible.
 
   FLEP_LIB_PATH=build_variants/x.so python tools/ab_overhead.py [case,...]
-case = body:C:K[:pf[:clc[:warp[:in_chunk]]]]
+case = body:C:K[:pf[:clc[:warp[:in_chunk[:static[:async_poll[:spec_fetch]]]]]]]   (static = 1: the static
+       persistent twin U1 with chunk C instead of the FLEP worker)
 """
 import json
 import os
@@ -54,9 +55,12 @@ def main():
         name, C, K = f[0], int(f[1]), int(f[2])
         pf, clc, warp = (int(f[3]) if len(f) > 3 else 0), (int(f[4]) if len(f) > 4 else 0), (int(f[5]) if len(f) > 5 else 0)
         ic = int(f[6]) if len(f) > 6 else 0
+        u1 = int(f[7]) if len(f) > 7 else 0
+        ap = int(f[8]) if len(f) > 8 else 0
+        sp = int(f[9]) if len(f) > 9 else 0
         body, grid, args = bodies[name]
         k = rt.register_kernel(body, chunk=C, poll=K, prefetch=bool(pf), clc=bool(clc), warp_tasks=bool(warp),
-                               in_chunk=bool(ic))
+                               in_chunk=bool(ic), async_poll=bool(ap), spec_fetch=bool(sp))
         tw, tu, span, uspan = [], [], [], []
         for r in range(reps + 3):
             for mode in ("w", "u"):
@@ -66,13 +70,16 @@ def main():
                     torch.cuda._sleep(gate)      # GPU busy while the host submits e0 + the kernel
                 e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                 e0.record(s)
-                if mode == "w":
+                if mode == "w" and u1:
+                    rt.launch_static(body, grid, args, chunk=C, stream=s)
+                    h = None
+                elif mode == "w":
                     h = rt.launch(k, grid, args, stream=s)
                 else:
                     rt.launch_unwrapped(body, grid, args, stream=s)
                 e1.record(s)
                 e1.synchronize()
-                if mode == "w":
+                if mode == "w" and h is not None:
                     rt.sync(h)
                 if r >= 3:
                     (tw if mode == "w" else tu).append(e0.elapsed_time(e1) * 1e3)
@@ -80,7 +87,7 @@ def main():
                         nb = grid[0] * grid[1]
                         tr = utrace[:2 * nb].view(nb, 2)
                         uspan.append(float((tr[:, 1].max() - tr[:, 0].min()).item()) / 1e3)
-                    if mode == "w" and not clc:
+                    if mode == "w" and not clc and h is not None:
                         ev = [e for e in rt.events(h, 1) if e.t_entry > 0]
                         if ev:
                             a0, a1 = min(e.t_entry for e in ev), max(e.t_exit for e in ev)
