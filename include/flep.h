@@ -217,10 +217,7 @@ typedef struct {
    scheduling step instead of two back to back). A worker that must leave after fetching returns
    the unstarted chunk through its per-worker record (as FLEP_KFLAG_IN_CHUNK), which the worker
    with the same index runs first in the next epoch: a request still costs at most one chunk.
-   With FLEP_KFLAG_PREFETCH the next chunk's fetch is issued right after the chunk barrier and
-   consumed at the next step (only the poll's round trip stays on the step), and a worker that
-   must leave returns the prefetched chunk the same way instead of running it.
-   Not with FLEP_KFLAG_ASYNC_POLL, FLEP_KFLAG_CLC, FLEP_KFLAG_SCHED_WARP,
+   Not with FLEP_KFLAG_PREFETCH, FLEP_KFLAG_ASYNC_POLL, FLEP_KFLAG_CLC, FLEP_KFLAG_SCHED_WARP,
    FLEP_KFLAG_WARP_TASKS or FLEP_KFLAG_IN_TILE (FLEP_KFLAG_IN_CHUNK workers always fetch this way);
    flep_register_kernel returns FLEP_ERR_UNSUPPORTED otherwise. Costs W x 16 B of runtime-owned
    device memory; a preempted epoch's coverage is then not a prefix of the counter. */

@@ -254,7 +254,6 @@ struct SchedState {
   bool stopping = false;             // a request named this SM; drain the held chunk
   bool first = true;                 // first step of this worker
   uint32_t snext = 0xffffffffu;      // static twin (U1): the next chunk base of this worker
-  bool want_fetch = false;           // R34 with prefetch: issue the next fetch after the barrier
 };
 
 // pull_task. In the first epoch of a launch the counter hands out blocks after the W
@@ -378,11 +377,6 @@ __device__ __forceinline__ uint32_t next_chunk(const WorkerParams& p, SchedState
 #endif
   if (!have) {
     unsigned long long w = ~0ull;
-    if (st.held != ~0ull && st.stopping && rec) {    // R34 with prefetch: return the held chunk
-      return_chunk(p, ws, rec, st.held);
-      st.held = ~0ull;
-      return 0xffffffffu;
-    }
     if (st.held != ~0ull) {                          // a fetched chunk is always processed (A4)
       w = st.held;
       st.held = ~0ull;
@@ -401,10 +395,7 @@ __device__ __forceinline__ uint32_t next_chunk(const WorkerParams& p, SchedState
 #endif
   if (base != 0xffffffffu) {
     ws.blocks += min(p.chunk, p.n_blocks - base);
-    if (p.prefetch && !st.stopping) {                // overlaps the body
-      if (rec) st.want_fetch = true;                 // R34: issued after the chunk barrier
-      else st.held = fetch_chunk(p);
-    }
+    if (p.prefetch && !st.stopping) st.held = fetch_chunk(p);   // overlaps the body
     if (p.trigger_block - base < p.chunk) {          // device self-trigger inside this chunk
       const uint32_t e = p.epoch % kEvEpochs;
       p.cb->ep_t_trigger[e] = gtimer();
@@ -586,7 +577,6 @@ flep_worker(const __grid_constant__ typename Body::Args args, const WorkerParams
       const uint32_t b0 = s_slot[parity];
       parity ^= 1u;
       if (b0 == 0xffffffffu) break;
-      if (tid == 0 && st.want_fetch) { st.held = fetch_chunk(p); st.want_fetch = false; }
       const uint32_t b1 = min(b0 + p.chunk, p.n_blocks);
       Body::run(args, b0, b1, p.gx, p.gy);
       if (kCoverage && tid == 0)

@@ -455,7 +455,8 @@ flep_status start_epoch(flep_rt rt, Launch& L) {
   p.trigger_n = L.trig_n;
   // no prefetch with in-tile preemption: a worker whose exhausted prefetch already counted its
   // exit must not later leave a partial tile (R23)
-  p.prefetch = ((L.flags & FLEP_KFLAG_PREFETCH) && !(L.flags & (FLEP_KFLAG_IN_TILE | FLEP_KFLAG_IN_CHUNK))) ? 1u : 0u;
+  p.prefetch = ((L.flags & FLEP_KFLAG_PREFETCH) &&
+                !(L.flags & (FLEP_KFLAG_IN_TILE | FLEP_KFLAG_IN_CHUNK | FLEP_KFLAG_SPEC_FETCH))) ? 1u : 0u;
   p.gen_first = L.gen0 + 1;
   p.started_hint = (L.flags & FLEP_KFLAG_STARTED_HINT) ? 1u : 0u;
   p.relay_block = L.relay ? L.ctas : 0xffffffffu;
@@ -923,9 +924,11 @@ flep_status flep_register_kernel(flep_rt rt, const flep_kernel_desc* d, flep_ker
   if (d->flags & FLEP_KFLAG_SPEC_FETCH) {
     if (d->body == FLEP_BODY_GEMM_BF16 || d->body == FLEP_BODY_GEMM_BF16_2SM)
       return fail(FLEP_ERR_UNSUPPORTED, "the speculative fetch is for the counter worker of the memory-bound bodies");
-    if (d->flags & (FLEP_KFLAG_ASYNC_POLL | FLEP_KFLAG_CLC | FLEP_KFLAG_SCHED_WARP | FLEP_KFLAG_WARP_TASKS |
-                    FLEP_KFLAG_IN_TILE))
-      return fail(FLEP_ERR_UNSUPPORTED, "the speculative fetch does not combine with async poll, CLC, "
+    // (with prefetch the next fetch would be in flight at every poll; measured slower anyway:
+    // issuing it after the chunk barrier delayed the scheduling warp's own body)
+    if (d->flags & (FLEP_KFLAG_PREFETCH | FLEP_KFLAG_ASYNC_POLL | FLEP_KFLAG_CLC | FLEP_KFLAG_SCHED_WARP |
+                    FLEP_KFLAG_WARP_TASKS | FLEP_KFLAG_IN_TILE))
+      return fail(FLEP_ERR_UNSUPPORTED, "the speculative fetch does not combine with prefetch, async poll, CLC, "
                                         "the scheduling warp, warp tasks or in-tile preemption");
   }
   ApiLock lk(rt);

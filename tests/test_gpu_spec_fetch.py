@@ -3,8 +3,7 @@ task-fetch atomic and the poll load are in flight together; a worker that must l
 chunk it fetched through its record, and the worker with the same index runs it first in the next
 epoch. Checked: every block exactly once under random preempt/resume schedules (temporal and
 spatial, I3), outputs bit-identical to uninterrupted runs and to the oracle, a yielding worker runs
-nothing after the request (its fetched or prefetched chunk is returned whole), and the flag's
-exclusions."""
+nothing after the request (its fetched chunk is returned whole), and the flag's exclusions."""
 import numpy as np
 import pytest
 
@@ -34,10 +33,10 @@ def test_spec_fetch_random_schedules_saxpy(rt):
     kern, bad = {}, []
     for i in range(600):
         s = gen.preempt_schedule(7000 + i, nb, rt.num_sms)
-        key = (s["C"], s["K"], i % 3, i % 2)
+        key = (s["C"], s["K"], i % 3)
         if key not in kern:
             kern[key] = rt.register_kernel(f.BODY_SAXPY_I32, chunk=s["C"], poll=s["K"], spec_fetch=True,
-                                           ctas_per_sm=(1, 2, 8)[i % 3], prefetch=bool(i % 2))
+                                           ctas_per_sm=(1, 2, 8)[i % 3])
         yd.copy_(y0)
         h, npre, viol = run_manual_schedule(rt, kern[key], f.saxpy_grid(n), f.saxpy_i32_args(yd, xd, a), nb,
                                             s, rt.num_sms, check_prefix=False)
@@ -71,8 +70,8 @@ def test_spec_fetch_preempt_resume_bitexact(rt, body):
     rt.launch_unwrapped(bid, grid, args)
     torch.cuda.synchronize()
     base = out.clone()
-    for C, pf in ((1, False), (1, True), (2, False), (4, True)):
-        k = rt.register_kernel(bid, chunk=C, poll=1, spec_fetch=True, prefetch=pf)
+    for C, K in ((1, 1), (1, 3), (2, 1), (4, 2)):
+        k = rt.register_kernel(bid, chunk=C, poll=K, spec_fetch=True)
         for cyc in range(4):
             out.zero_()
             sched = gen.preempt_schedule(8000 + 10 * C + cyc, nb, rt.num_sms)
@@ -87,8 +86,7 @@ def test_spec_fetch_preempt_resume_bitexact(rt, body):
         assert float(np.max(np.abs(got - ref) / np.where(d > 0, d, 1))) <= 1e-5
 
 
-@pytest.mark.parametrize("pf", [False, True])
-def test_spec_fetch_returns_whole_chunks(rt, pf):
+def test_spec_fetch_returns_whole_chunks(rt):
     """C = 8, temporal request: the drained epoch ran the counter's blocks except the returned
     chunks; each hole is a whole fetched chunk [b, b + 8) (nothing of it ran), at most one per
     yielding worker; the resume runs them exactly once."""
@@ -98,7 +96,7 @@ def test_spec_fetch_returns_whole_chunks(rt, pf):
     C = 8
     x, y = gen.saxpy_i32_inputs(n, seed=53)
     xd, yd = t(x), t(y)
-    k = rt.register_kernel(f.BODY_SAXPY_I32, chunk=C, poll=1, spec_fetch=True, prefetch=pf)
+    k = rt.register_kernel(f.BODY_SAXPY_I32, chunk=C, poll=1, spec_fetch=True)
     rt.arm_next_trigger(nb // 2, rt.num_sms)
     h = rt.launch(k, f.saxpy_grid(n), f.saxpy_i32_args(yd, xd, 3))
     rt.wait_epoch(h, timeout_ns=10_000_000_000)
@@ -123,7 +121,7 @@ def test_spec_fetch_returns_whole_chunks(rt, pf):
 
 def test_spec_fetch_exclusions(rt):
     f = flep_mod()
-    for kw in ({"async_poll": True}, {"clc": True}, {"sched_warp": True},
+    for kw in ({"prefetch": True}, {"async_poll": True}, {"clc": True}, {"sched_warp": True},
                {"warp_tasks": True}):
         with pytest.raises(f.FlepError):
             rt.register_kernel(f.BODY_SAXPY_I32, chunk=1, poll=1, spec_fetch=True, **kw)

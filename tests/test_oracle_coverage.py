@@ -56,8 +56,8 @@ def test_refill_without_done_marker_double_executes():
     orig = m.successors
 
     def no_marker(cfg, st):
-        st2 = st[:9] + ((st[9][0], 0, st[9][2]),)   # pretend no epoch ever recorded completion
-        return [(lab, s[:9] + ((s[9][0], 0, s[9][2]),)) for lab, s in orig(cfg, st2)]
+        st2 = st[:9] + ((st[9][0], 0, st[9][2]) + st[9][3:],)   # pretend no epoch ever recorded completion
+        return [(lab, s[:9] + ((s[9][0], 0, s[9][2]) + s[9][3:],)) for lab, s in orig(cfg, st2)]
     m.successors = no_marker
     try:
         r = cv.explore(_cfg(n_blocks=3, chunk=1, poll=1, worker_sm=(0, 1), preempt_widths=(1,),
@@ -284,3 +284,56 @@ def test_planted_double_count_is_caught():
     for pf in (False, True):
         cfg = _cfg(n_blocks=5, chunk=1, poll=1, worker_sm=(0, 0, 1), prefetch=pf, bug_count_twice=True)
         assert cv.explore(cfg).violations
+
+
+# ---- speculative fetch (R34): fetch + poll together, a fetched chunk returned -----------
+
+@pytest.mark.parametrize("n,c,k,sms,extra", [
+    (4, 1, 1, (0, 1), {}), (5, 2, 1, (0, 1), {}), (6, 1, 1, (0, 1, 1), {}),
+    (6, 1, 1, (0, 1, 1), {"allow_clear": True}), (6, 1, 1, (0, 1, 1), {"allow_refill": True}),
+    (5, 1, 2, (0, 0, 1), {}),
+])
+def test_spec_fetch_exhaustive(n, c, k, sms, extra):
+    cfg = cv.Config(n_blocks=n, chunk=c, poll=k, worker_sm=sms, num_sms=2, preempt_widths=(1, 2),
+                    max_events=3, static_first=True, spec_fetch=True, **extra)
+    r = cv.explore(cfg)
+    assert r.violations == set()
+    assert r.preempted_epoch_ends > 0
+
+
+@pytest.mark.parametrize("bug", ["bug_spec_drop", "bug_spec_publish"])
+def test_spec_fetch_planted_bugs_caught(bug):
+    cfg = cv.Config(n_blocks=4, chunk=1, poll=1, worker_sm=(0, 1), num_sms=2, preempt_widths=(1, 2),
+                    max_events=2, static_first=True, spec_fetch=True, **{bug: True})
+    r = cv.explore(cfg)
+    assert any(v.startswith("I1") for v in r.violations)
+
+
+def test_spec_fetch_hand_trace():
+    """N = 4, C = 1, two workers on SMs 0 and 1 (R20 static first chunks 0 and 1, counter at 2).
+    w0 runs block 0, fetches block 2 speculatively, a temporal request lands, w0's poll sees it:
+    block 2 goes to w0's record and w0 leaves; w1 (holding its static block 1) runs it, then its
+    poll step sees the request and leaves. The drained epoch covered {0, 1}: the prefix [0, 3)
+    minus the record. On resume, worker 0 runs block 2 from its record first (after its entry
+    check), then both fetch; every block once."""
+    cfg = cv.Config(n_blocks=4, chunk=1, poll=1, worker_sm=(0, 1), num_sms=2, preempt_widths=(2,),
+                    max_events=1, static_first=True, spec_fetch=True)
+    st = cv.initial_state(cfg)
+    for lab in ["w0.fetch", "w0.proc", "w0.spec_fetch", "preempt(2)", "w0.spec_yield", "w0.exit",
+                "w1.fetch", "w1.proc", "w1.spec_fetch", "w1.spec_yield", "w1.exit"]:
+        st = dict(cv.successors(cfg, st))[lab]
+    assert st[6] == cv.ST_PREEMPTED
+    assert st[4] == (1, 1, 0, 0)
+    assert st[9][3] == (2, 3)                          # both fetched chunks were returned
+    assert st[0] == 4                                  # counter: 2 static + 2 speculative fetches
+    assert cv.check_state(cfg, st) == set()
+    st = dict(cv.successors(cfg, st))["resume"]
+    for lab in ["w0.take_rest", "w0.proc", "w1.take_rest", "w1.proc"]:
+        st = dict(cv.successors(cfg, st))[lab]
+    assert st[4] == (1, 1, 1, 1) and st[9][3] == (cv.NOCHUNK, cv.NOCHUNK)
+    while True:                                        # the rest: exhausted fetches and exits
+        succ = cv.successors(cfg, st)
+        if not succ:
+            break
+        st = succ[0][1]
+    assert st[6] == cv.ST_DONE and st[4] == (1, 1, 1, 1)
