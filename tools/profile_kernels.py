@@ -21,7 +21,7 @@ def main():
     ap.add_argument("--chunk", type=int, default=1)
     ap.add_argument("--prefetch", type=int, default=1)
     ap.add_argument("--poll", type=int, default=1)
-    ap.add_argument("--combos", default="", help="C:K:prefetch[:async[:clc]][,...] wrapped variants (overrides --chunk/--poll/--prefetch)")
+    ap.add_argument("--combos", default="", help="C:K:prefetch[:async[:clc[:spec]]][,...] wrapped variants (overrides --chunk/--poll/--prefetch)")
     a = ap.parse_args()
     import torch
     from paper_conf_asplos_wulzj17_b200 import build, flep as F
@@ -54,11 +54,12 @@ def main():
         Cg = torch.empty(M, M, device="cuda", dtype=torch.bfloat16)
         jobs.append(("gemm", F.BODY_GEMM_BF16, F.gemm_grid(M, M), F.gemm_args(Cg, A, B), (A, B, Cg)))
     s = torch.cuda.current_stream()
-    combos = [(tuple(map(int, c.split(":"))) + (0, 0))[:5] for c in a.combos.split(",")] if a.combos \
-        else [(a.chunk, a.poll, a.prefetch, 0, 0)]
+    combos = [(tuple(map(int, c.split(":"))) + (0, 0, 0))[:6] for c in a.combos.split(",")] if a.combos \
+        else [(a.chunk, a.poll, a.prefetch, 0, 0, 0)]
     for name, body, grid, args, keep in jobs:
-        ks = [rt.register_kernel(body, chunk=C, poll=K, prefetch=bool(pf), async_poll=bool(ap), clc=bool(clc))
-              for C, K, pf, ap, clc in combos]
+        ks = [rt.register_kernel(body, chunk=C, poll=K, prefetch=bool(pf), async_poll=bool(ap), clc=bool(clc),
+                                 spec_fetch=bool(sp))
+              for C, K, pf, ap, clc, sp in combos]
         for _ in range(a.reps):
             flush.zero_()
             rt.launch_unwrapped(body, grid, args, stream=s)

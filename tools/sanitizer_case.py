@@ -86,7 +86,7 @@ def main():
     rt.sync(h)
     # round 2: warp-task workers (SpMV vector body, stencil) with a temporal preempt/resume cycle,
     # the static persistent twin, the CTA-pair GEMM (unwrapped, static, worker with a preemption, in-tile worker)
-    # and device-checked slicing with a preemption
+    # device-checked slicing with a preemption and the speculative fetch with a preemption
     k9 = rt.register_kernel(F.BODY_SPMV_CSR_F32_VEC, chunk=2, poll=1, warp_tasks=True)
     rt.arm_next_trigger(4, rt.num_sms)
     h = rt.launch(k9, F.spmv_grid(2000), F.spmv_args(yv, *keep))
@@ -107,6 +107,14 @@ def main():
     k11 = rt.register_kernel(F.BODY_GEMM_BF16_2SM, chunk=1, poll=1)
     rt.arm_next_trigger(1, rt.num_sms)
     h = rt.launch(k11, g2, F.gemm_args(C2, A2, B2))
+    rt.wait_epoch(h)
+    if rt.query(h).state == F.STATE_PREEMPTED:
+        rt.resume(h)
+    rt.sync(h)
+    # speculative fetch (R34): a preempt/resume cycle that returns fetched chunks through records
+    k13 = rt.register_kernel(F.BODY_SPMV_CSR_F32, chunk=1, poll=1, spec_fetch=True)
+    rt.arm_next_trigger(4, rt.num_sms)
+    h = rt.launch(k13, F.spmv_grid(2000), F.spmv_args(yv, *keep))
     rt.wait_epoch(h)
     if rt.query(h).state == F.STATE_PREEMPTED:
         rt.resume(h)
