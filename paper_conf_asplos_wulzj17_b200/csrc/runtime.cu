@@ -199,6 +199,7 @@ struct flep_rt_s {
   std::atomic<int> waiters{0};      // API threads waiting for `mu`
   std::vector<int64_t> active_ids;  // managed mode: launches whose state the monitor must poll
   std::atomic<uint64_t> active_gen{0};   // bumped whenever active_ids grows (wakes the monitor)
+  int64_t mon_t_hit = 0, mon_t_locked = 0;   // FLEP_DEBUG_SLOW diagnostics of the monitor's pass
 };
 
 namespace {
@@ -568,6 +569,12 @@ bool refresh(flep_rt rt, Launch& L) {
   L.ctr_known = true;
   // the monitor stamps the moment it saw the word move (before taking the lock)
   const int64_t t_obs = L.t_seen > 0 ? L.t_seen : now_ns();
+  if (slow_threshold_ns() >= 0 && (w & 0xffu) != kStateDone)
+    fprintf(stderr, "[flep] monitor: launch %lld preempted: request +0, word seen %+.3f us (%s), pass hit %+.3f, "
+                    "locked %+.3f, now %+.3f\n", (long long)L.id,
+            L.t_seen > 0 ? (L.t_seen - L.t_last_request) / 1e3 : -1.0, L.t_seen > 0 ? "spin" : "pass",
+            (rt->mon_t_hit - L.t_last_request) / 1e3, (rt->mon_t_locked - L.t_last_request) / 1e3,
+            (now_ns() - L.t_last_request) / 1e3);
   L.t_seen = 0;
   if ((w & 0xffu) == kStateDone) {
     L.state = FLEP_STATE_DONE;
@@ -723,26 +730,30 @@ void monitor_pass(flep_rt rt) {
 // never starved by it.
 void monitor_loop(flep_rt rt) {
   cudaSetDevice(rt->device);
-  struct Watch { const uint64_t* word; uint64_t seen; bool sliced; int64_t id; cudaEvent_t ev; };
+  struct Watch { const uint64_t* word; uint64_t seen; bool sliced; int64_t id; cudaEvent_t ev; bool stamped; };
   std::vector<std::pair<int64_t, int64_t>> moved;     // (launch, host time seen)
   std::vector<Watch> watch;
   int64_t deadline = -1;
   bool pending_release = false;
   uint64_t gen_seen = ~0ull;
   uint32_t spin = 0;
+  bool yielding = false;             // a request is pending on some watched launch
+  int64_t t_last_busy = now_ns();    // last pass with a watched launch
   while (!rt->stop.load(std::memory_order_relaxed)) {
     bool hit = false;
     if (gen_seen != rt->active_gen.load(std::memory_order_acquire)) hit = true;   // new work
     moved.clear();
     // the pinned words every pass (a plain load); the completion events of silent DONE epochs
     // (R24) every 8th pass: cudaEventQuery takes a driver lock that the application's launches
-    // also need, and the PREEMPTED word is the latency-critical notification
-    const bool query_events = (++spin & 7u) == 0;
-    for (const Watch& w : watch) {
+    // also need, and the PREEMPTED word is the latency-critical notification. While a request is
+    // pending no event is queried at all: a query that waits behind the application's driver
+    // call (the waiting kernel's launch, ~10 us) delayed seeing the drained word by as much
+    const bool query_events = !yielding && (++spin & 7u) == 0;
+    for (Watch& w : watch) {
       if (w.sliced) { hit = true; continue; }
       if (__atomic_load_n(w.word, __ATOMIC_ACQUIRE) != w.seen ||
           (query_events && w.ev && cudaEventQuery(w.ev) == cudaSuccess)) {
-        hit = true; moved.push_back({w.id, now_ns()});
+        hit = true; moved.push_back({w.id, now_ns()}); w.stamped = true;
       }
     }
     if (deadline >= 0 && now_ns() >= deadline) hit = true;
@@ -750,7 +761,11 @@ void monitor_loop(flep_rt rt) {
     // lock is what application threads need; a release is never latency-critical)
     if (pending_release && (spin & 63u) == 0) hit = true;
     if (!hit) {
-      if (watch.empty() && deadline < 0) {
+      // idle: sleep only after 50 ms without any watched launch. A sleeping monitor is woken by
+      // the next flep_launch's notify, and a futex wake-up took 5-15 us: when the next launch is
+      // preempted right after it starts (the bench's e2e step), the drained epoch was then seen
+      // late by that much
+      if (watch.empty() && deadline < 0 && now_ns() - t_last_busy > 50'000'000) {
         std::unique_lock<std::mutex> lk(rt->mu);
         rt->cv.wait_for(lk, std::chrono::milliseconds(1));
       } else {
@@ -761,7 +776,20 @@ void monitor_loop(flep_rt rt) {
     // API threads announce themselves before taking the lock (ApiLock): let them in first, for a
     // bounded time (a thread that calls the API in a loop must not starve the monitor either)
     for (int i = 0; i < 256 && rt->waiters.load(std::memory_order_relaxed) > 0; ++i) __builtin_ia32_pause();
-    std::unique_lock<std::mutex> lk(rt->mu);
+    // while an API call holds the lock (a managed launch that preempts holds it ~10 us for its
+    // driver calls), keep watching the pinned words: a drained epoch is stamped when its word
+    // moves, not when the monitor gets the lock
+    const int64_t t_hit = now_ns();
+    std::unique_lock<std::mutex> lk(rt->mu, std::defer_lock);
+    while (!lk.try_lock()) {
+      for (Watch& w : watch)
+        if (!w.sliced && !w.stamped && __atomic_load_n(w.word, __ATOMIC_ACQUIRE) != w.seen) {
+          moved.push_back({w.id, now_ns()}); w.stamped = true;
+        }
+      for (int i = 0; i < 32; ++i) __builtin_ia32_pause();
+    }
+    rt->mon_t_hit = t_hit;
+    rt->mon_t_locked = now_ns();
     for (auto& m : moved) {
       Launch* L = find(rt, m.first);
       if (L) L->t_seen = m.second;
@@ -776,19 +804,22 @@ void monitor_loop(flep_rt rt) {
     }
     monitor_pass(rt);
     watch.clear();
+    yielding = false;
     for (int64_t id : rt->active_ids) {
       Launch* L = find(rt, id);
       if (!L || !L->hs) continue;
+      if (L->state == FLEP_STATE_YIELDING) yielding = true;
       const uint64_t* wp = reinterpret_cast<const uint64_t*>(&L->hs->word);
       auto it = snap.find(id);
       const bool running = L->state == FLEP_STATE_RUNNING || L->state == FLEP_STATE_YIELDING ||
                            L->state == FLEP_STATE_PARTIAL || (L->clc && L->state == FLEP_STATE_PREEMPTED);
       const bool host_sliced = L->sliced && !L->slice_dev;    // host-issued slices: every pass
       watch.push_back({wp, it != snap.end() ? it->second : ~0ull, host_sliced, id,
-                       (running && !host_sliced) ? L->fin_ev : nullptr});
+                       (running && !host_sliced) ? L->fin_ev : nullptr, false});
     }
     deadline = rt->policy->epoch_end();
     pending_release = !rt->to_release.empty();
+    t_last_busy = now_ns();
   }
 }
 
