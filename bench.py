@@ -547,7 +547,7 @@ def run_e2e(F, torch, wl, local, steps, args, diag=False):
     copies the inputs from pinned host memory, the HP arrival is an intercepted flep_launch that
     makes the runtime preempt the running LP, and the outputs are read back. Latency = host
     clock from the runtime's preemption request to its observation of the drained epoch."""
-    rt = F.Runtime(device=local, policy=F.POLICY_HPF)
+    rt = F.Runtime(device=local, policy=F.POLICY_HPF, keep_logs=diag)
     kLP = rt.register_kernel(F.BODY_SPMV_CSR_F32, chunk=args.lp_chunk, poll=args.lp_poll, name="spmv",
                              model=(0, 0, 0, 0, 70_000), prefetch=bool(args.prefetch), started_hint=True,
                              host_relay=bool(args.e2e_relay), spec_fetch=bool(args.lp_spec))
@@ -584,15 +584,6 @@ def run_e2e(F, torch, wl, local, steps, args, diag=False):
         h_hp = rt.launch(kHP, F.stencil_grid(STENCIL_N), hp_args, priority=1, stream=B)
         t_l1 = F.now_ns()
         ev = []
-        if diag:      # read the victim's first-epoch worker log while it is preempted (before release)
-            t_d = time.perf_counter()
-            while rt.query(h_lp).state not in (F.STATE_PREEMPTED, F.STATE_DONE) and time.perf_counter() - t_d < 1.0:
-                pass
-            if rt.query(h_lp).state == F.STATE_PREEMPTED:
-                try:
-                    ev = rt.events(h_lp, 1)
-                except F.FlepError:
-                    ev = []
         rt.sync(h_hp, timeout_ns=10_000_000_000)
         rt.sync(h_lp, timeout_ns=10_000_000_000)
         with torch.cuda.stream(A):
@@ -603,6 +594,8 @@ def run_e2e(F, torch, wl, local, steps, args, diag=False):
         B.synchronize()
         dt = (time.perf_counter() - t0) * 1e3
         info = rt.query(h_lp)
+        if diag and info.epoch >= 2:  # the victim's first-epoch worker log, kept (keep_logs): read
+            ev = rt.events(h_lp, 1)   # after the step, so the host thread waits in flep_sync as usual
         if i >= 2:
             step_ms.append(dt)
             if info.epoch >= 2 and info.t_last_drain > 0:
@@ -638,8 +631,10 @@ def run_e2e(F, torch, wl, local, steps, args, diag=False):
             "breakdown_us_p50": ({"request_to_first_yield": round(float(np.median([a for a, _, _ in dev])), 3),
                                   "yield_spread": round(float(np.median([b for _, b, _ in dev])), 3),
                                   "last_yield_to_host_seen": round(float(np.median([c for _, _, c in dev])), 3),
-                                  "note": "device times mapped to the host clock through the started hint "
-                                          "(error ~ one PCIe write + one poll)"} if dev else None)}
+                                  "note": "device times mapped to the host clock through the started hint: "
+                                          "the host sees that hint one PCIe write + one poll late, so every "
+                                          "mapped device time reads late by that much (the last leg can read "
+                                          "negative); the logs are read after the step (keep_logs)"} if dev else None)}
 
 
 def cpu_baseline(wl):

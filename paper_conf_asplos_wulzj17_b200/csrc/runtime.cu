@@ -745,10 +745,9 @@ void monitor_loop(flep_rt rt) {
     moved.clear();
     // the pinned words every pass (a plain load); the completion events of silent DONE epochs
     // (R24) every 8th pass: cudaEventQuery takes a driver lock that the application's launches
-    // also need, and the PREEMPTED word is the latency-critical notification. While a request is
-    // pending no event is queried at all: a query that waits behind the application's driver
-    // call (the waiting kernel's launch, ~10 us) delayed seeing the drained word by as much
-    const bool query_events = !yielding && (++spin & 7u) == 0;
+    // also need, and the PREEMPTED word is the latency-critical notification (while a request is
+    // pending, every 32nd pass: a yielding launch may still end DONE, which only its event shows)
+    const bool query_events = (++spin & (yielding ? 31u : 7u)) == 0;
     for (Watch& w : watch) {
       if (w.sliced) { hit = true; continue; }
       if (__atomic_load_n(w.word, __ATOMIC_ACQUIRE) != w.seen ||
