@@ -401,9 +401,7 @@ struct Gemm2 {
                       if (q == q_stop) { stop = true; break; }
                     }
                   }
-#ifndef FLEP_X_NO_POLL
                   if (j % kInTilePoll == 0 && j > 0) { pend = poll_ctrl(p); pend_valid = true; }
-#endif
                 }
               }
               wait(&s->empty[st], ph ^ 1u);
@@ -449,7 +447,6 @@ struct Gemm2 {
           tile_coords(tile, gx, gy, tm, tn);
           bool stopped = false;
           for (uint32_t kb = kb0; kb < nk; ++kb) {
-#ifndef FLEP_X_NO_LIC
             if (in_tile) {                             // wait for the licence of load q (or a stop)
               while (true) {
                 uint32_t l, sa_;
@@ -460,7 +457,6 @@ struct Gemm2 {
               }
               if (stopped) break;
             }
-#endif
             wait(&s->empty[st], ph ^ 1u);
             uint8_t* sa = base + st * kStage;
             const uint32_t fb = full0 + st * 8u;
@@ -560,12 +556,8 @@ struct Gemm2 {
         // stopped inside the tile iff the queue's next entry is STOP_PARTIAL (a stop is always
         // the pair's last tile; the leader pushes the next entry before this tile's MMAs end, so
         // the peek costs nothing; a remote publish from the MMA thread would fence its pipeline)
-#ifndef FLEP_X_NO_PEEK
         wait(&s->qfull[qi], qph);
         if (s->tile_q[qi] == STOP_PARTIAL) {
-#else
-        if (false) {
-#endif
           float4* dst = spill_slot(p, wid, r);
 #pragma unroll 1
           for (uint32_t c0 = 0; c0 < BN; c0 += 32) {
