@@ -241,11 +241,13 @@ def test_managed_ffs_share_and_replay():
         rt.close()
 
 
+@pytest.mark.parametrize("spec", [False, True])
 @pytest.mark.parametrize("tail", [False, True])
-def test_spatial_refill_exactly_once(tail):
+def test_spatial_refill_exactly_once(tail, spec):
     """Spatial yield, then refill: the victim is re-spread over all SMs. With the
     trigger near the end, the running epoch usually completes the launch before the refill epoch
-    starts; that epoch must not re-run anything (the control block was already reset)."""
+    starts; that epoch must not re-run anything (the control block was already reset). With the
+    speculative fetch (R34) the yielded workers' returned chunks are run by the refill epoch."""
     f = flep_mod()
     rt = f.Runtime(coverage=True)
     try:
@@ -254,7 +256,7 @@ def test_spatial_refill_exactly_once(tail):
         x, y = gen.saxpy_i32_inputs(n, seed=81)
         ref = W.saxpy_i32(13, x, y)
         xd, y0 = t(x), t(y)
-        k = rt.register_kernel(f.BODY_SAXPY_I32, chunk=1, poll=1)
+        k = rt.register_kernel(f.BODY_SAXPY_I32, chunk=1, poll=1, spec_fetch=spec)
         for rep in range(20):
             yd = y0.clone()
             tstar = nb - 40 if tail else nb // 4
@@ -331,8 +333,9 @@ def _replay_ex(rt, spatial):
     return [(t_, acts[a], i, n) for (t_, a, i, n) in des.replay(des.HPF, evs, num_sms=rt.num_sms, spatial=spatial)]
 
 
+@pytest.mark.parametrize("spec", [False, True])
 @pytest.mark.parametrize("n_sms", [5, 16, 74])
-def test_managed_spatial_hpf_decides_how_far(n_sms):
+def test_managed_spatial_hpf_decides_how_far(n_sms, spec):
     """Spatial HPF (R29): a high-priority SAXPY-int32 whose workers fit on n SMs
     arrives while an int32 stencil 8192^2 runs; the runtime yields exactly n SMs (rank < n), runs
     the waiting kernel beside the victim, refills the victim at its end. Checked: decision list
@@ -346,7 +349,8 @@ def test_managed_spatial_hpf_decides_how_far(n_sms):
         a = gen.stencil_i32_input(nst, seed=61)
         ind = t(a)
         outd = torch.empty_like(ind)
-        k_v = rt.register_kernel(f.BODY_STENCIL5_I32, chunk=1, poll=1, model=(0, 0, 0, 0, 400_000))
+        k_v = rt.register_kernel(f.BODY_STENCIL5_I32, chunk=1, poll=1, model=(0, 0, 0, 0, 400_000),
+                                 spec_fetch=spec)
         cps, _ = rt.workers_for(f.BODY_SAXPY_I32)
         n_hp = n_sms * cps * 256 - 77                      # ragged tail, still n_sms * cps blocks
         x2, y2 = gen.saxpy_i32_inputs(n_hp, seed=62)
