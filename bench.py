@@ -52,17 +52,51 @@ def peaks():
 
 # ------------------------------------------------------------------------------------------
 class ClockSampler:
-    """nvidia-smi clocks / throttle reasons sampled DURING the timed region."""
+    """SM clocks and clock-event (throttle) reasons sampled DURING the timed region: an NVML
+    thread every ~2 ms (the timed region of the default run is tens of ms, too short for
+    nvidia-smi's 50 ms loop, which also starts ~100 ms late); nvidia-smi if NVML is missing."""
 
     FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
               "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
               "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+    NAMES = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
 
-    def __init__(self, gpu_index):
+    def __init__(self, gpu_index, period_s=0.002):
         self.idx = gpu_index
+        self.period = period_s
         self.p = None
+        self.nv = None
+        self.samples = []            # (sm_mhz, max_mhz, set(reasons))
+        self.out = ""
+
+    def _nvml_loop(self):
+        import pynvml as N
+        bits = {"hw_slowdown": N.nvmlClocksEventReasonHwSlowdown,
+                "hw_thermal_slowdown": N.nvmlClocksEventReasonHwThermalSlowdown,
+                "sw_thermal_slowdown": N.nvmlClocksEventReasonSwThermalSlowdown,
+                "sw_power_cap": N.nvmlClocksEventReasonSwPowerCap}
+        while not self.stop.is_set():
+            try:
+                sm = N.nvmlDeviceGetClockInfo(self.nv, N.NVML_CLOCK_SM)
+                mx = N.nvmlDeviceGetMaxClockInfo(self.nv, N.NVML_CLOCK_SM)
+                r = N.nvmlDeviceGetCurrentClocksEventReasons(self.nv)
+                self.samples.append((float(sm), float(mx), {k for k, b in bits.items() if r & b}))
+            except Exception:
+                pass
+            time.sleep(self.period)
 
     def __enter__(self):
+        import threading
+        try:
+            import pynvml as N
+            N.nvmlInit()
+            self.nv = N.nvmlDeviceGetHandleByIndex(int(self.idx))
+            self.stop = threading.Event()
+            self.th = threading.Thread(target=self._nvml_loop, daemon=True)
+            self.th.start()
+            return self
+        except Exception:
+            self.nv = None
         try:
             self.p = subprocess.Popen(["nvidia-smi", "-i", str(self.idx), f"--query-gpu={self.FIELDS}",
                                        "--format=csv,noheader,nounits", "-lms", "50"],
@@ -72,7 +106,10 @@ class ClockSampler:
         return self
 
     def __exit__(self, *a):
-        self.out = ""
+        if self.nv is not None:
+            self.stop.set()
+            self.th.join(timeout=2)
+            return
         if self.p is not None:
             self.p.terminate()
             try:
@@ -82,7 +119,10 @@ class ClockSampler:
 
     def summary(self):
         sm, mx, reasons = [], 0.0, set()
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for s_, m_, r_ in self.samples:
+            sm.append(s_)
+            mx = max(mx, m_)
+            reasons |= r_
         for line in (self.out or "").splitlines():
             f = [x.strip() for x in line.split(",")]
             if len(f) < 9:
@@ -92,12 +132,13 @@ class ClockSampler:
                 mx = max(mx, float(f[2]))
             except ValueError:
                 continue
-            for nm, v in zip(names, f[5:9]):
+            for nm, v in zip(self.NAMES, f[5:9]):
                 if v.lower() == "active":
                     reasons.add(nm)
         load = [s for s in sm if s > 300] or sm
         return {"sm_mhz": statistics.median(load) if load else None, "sm_max_mhz": mx or None,
-                "reasons": sorted(reasons), "samples": len(sm)}
+                "reasons": sorted(reasons), "samples": len(sm),
+                "source": "nvml" if self.nv is not None else "nvidia-smi"}
 
 
 def physical_gpu_index(local_rank):
