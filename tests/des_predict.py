@@ -1,5 +1,6 @@
 """DES prediction vs the B200 measurement for the configs[3] queue (SURVEY §8(c) O3 simulate mode,
-§8(d) C4 "DES-predicted vs measured ANTT"). Test/report infrastructure: imports the oracle.
+§8(d) C4 "DES-predicted vs measured ANTT"). Test infrastructure (it imports the oracle, so it
+lives under tests/; run by tests/test_oracle_des.py, or directly to print the report).
 
 Input: the per-kernel record of one queue run (tests/golden/queue_debug_r02.json: name, host
 arrival, first start, finish, epochs, standalone time, per policy) and that run's measured ANTT.

@@ -260,11 +260,11 @@ def test_reordering_baseline_triplet():
 def test_des_predicts_the_b200_queue_run():
     """Simulate mode vs a measured B200 run (SURVEY §8(d) C4 "DES-predicted vs measured ANTT"):
     the oracle DES fed with the run's own arrivals and standalone times predicts each policy's
-    ANTT within 30 % and the same ordering HPF < REORDER < FIFO (tools/des_predict.py; a model
+    ANTT within 30 % and the same ordering HPF < REORDER < FIFO (tests/des_predict.py; a model
     check, reported rather than pinned: the simulation ignores co-run interference)."""
     import os
     import sys
-    sys.path.insert(0, os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "tools"))
+    sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
     import des_predict
     out = des_predict.main()
     for k, v in out["policies"].items():
