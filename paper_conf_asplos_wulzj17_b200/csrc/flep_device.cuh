@@ -844,16 +844,21 @@ flep_clc_worker(const __grid_constant__ typename Body::Args args, const WorkerPa
   // on its own chunk (launched by the hardware)
   uint32_t b = blockIdx.x;
   uint32_t k = 0, phase = 0, parity = 0;
+  bool have_seen = false;            // async poll: a copy of the control word is in flight
   while (true) {
     bool pending = false;
     if (tid == 0) {
       // amortised poll (every K blocks) before asking for more work; a request that names this
-      // SM ends the persistence after the block in hand
+      // SM ends the persistence after the block in hand. With FLEP_KFLAG_ASYNC_POLL (R22) the
+      // word was copied into shared memory one block earlier (no round trip here; a request is
+      // then seen up to one block later)
       bool stop = false;
       if (++k == p.poll) {
         k = 0;
-        stop = should_yield(poll_ctrl(p), p, smid_reg());
+        const uint32_t c = (p.async_poll && have_seen) ? poll_consume(ws) : poll_ctrl(p);
+        stop = should_yield(c, p, smid_reg());
       }
+      if (p.async_poll && !stop && k == p.poll - 1) { poll_issue(ws, p.ctrl); have_seen = true; }
       if (!stop) { clc_try_cancel(resp, mbar); pending = true; }   // overlaps the body
       else ws.reason = kReasonYield;
       if (p.trigger_block - b * p.chunk < p.chunk) {     // device self-trigger (test/bench hook)
