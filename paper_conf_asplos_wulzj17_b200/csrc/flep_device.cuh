@@ -243,8 +243,9 @@ __device__ __forceinline__ uint32_t poll_consume(const WorkerShared& ws) {
 // poll every K chunks, then the task fetch (pull_task) — or the chunk fetched
 // ahead by the previous step when prefetching. Returns the base block of the chunk to run, or
 // 0xffffffff when the worker must leave (yield on request, or counter exhausted). Never returns
-// "leave" while a fetched chunk is held (exactly-once, reading A4). Also fires the device
-// self-trigger of the test/bench hooks.
+// "leave" while a fetched chunk is held (exactly-once, reading A4) — except with the speculative
+// fetch (R34, `rec` given), which returns such a chunk through the worker's record first. Also
+// fires the device self-trigger of the test/bench hooks.
 struct SchedState {
   uint32_t k = 0;                    // chunk index within the current poll period
   unsigned long long held = ~0ull;   // prefetched counter word not yet handed out (raw: the
