@@ -802,7 +802,7 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=10)
     ap.add_argument("--tune-bound", type=float, default=0.04, help="config tune: overhead bound (P:166: 4 %%)")
     ap.add_argument("--gemm-in-tile", type=int, default=1, help="config gemm: in-tile preemption (1) or tile granularity (0)")
-    ap.add_argument("--gemm-pair", type=int, default=0, help="config gemm: the CTA-pair body (1) or the 1-CTA body (0)")
+    ap.add_argument("--gemm-pair", type=int, default=0, help="config gemm: the 1-CTA body (0), the CTA-pair body (1) or its 256x512 tile (2)")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     args.skip_sub = [x.strip() for x in args.skip_sub.split(",") if x.strip()]

@@ -449,12 +449,12 @@ def run_gemm_preempt(args, rank, world, local):
     st_in = torch.rand(4096, 4096, device="cuda", generator=g)
     st_out = torch.empty_like(st_in)
     in_tile = bool(args.gemm_in_tile)
-    pair = bool(getattr(args, "gemm_pair", 0))            # the CTA-pair body (R32)
-    body = F.BODY_GEMM_BF16_2SM if pair else F.BODY_GEMM_BF16
+    pair = int(getattr(args, "gemm_pair", 0))             # 1: the CTA-pair body (R32), 2: its wide tile
+    body = {0: F.BODY_GEMM_BF16, 1: F.BODY_GEMM_BF16_2SM, 2: F.BODY_GEMM_BF16_2SM_W}[pair]
     k_lp = rt.register_kernel(body, chunk=1, poll=1, name="gemm", in_tile=in_tile)
     k_hp = rt.register_kernel(F.BODY_STENCIL5_F32, chunk=2, poll=1, prefetch=True, name="stencil")
     lp_args = F.gemm_args(C_, A_, B_)
-    lp_grid = F.gemm2_grid(M, N) if pair else F.gemm_grid(M, N)
+    lp_grid = {0: F.gemm_grid, 1: F.gemm2_grid, 2: F.gemm2w_grid}[pair](M, N)
     hp_args, hp_grid = F.stencil_args(st_out, st_in), F.stencil_grid(4096)
     nb = lp_grid[0] * lp_grid[1]
     flush = L2Flush(torch)
@@ -514,8 +514,10 @@ def run_gemm_preempt(args, rank, world, local):
                                "last GEMM CTA gone, p50",
            "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "higher_is_better": False,
            "scaling": "weak", "vs_baseline": None, "dtype": "bf16", "data": "synthetic (seeded)",
-           "config": {"workload": ("LP GEMM bf16 8192^3 (tcgen05 cta_group::2, 256x256 tiles on CTA pairs)" if pair else
-                                   "LP GEMM bf16 8192^3 (tcgen05, 128x256 tiles)") + " preempted by HP stencil5 4096^2",
+           "config": {"workload": {0: "LP GEMM bf16 8192^3 (tcgen05, 128x256 tiles)",
+                                   1: "LP GEMM bf16 8192^3 (tcgen05 cta_group::2, 256x256 tiles on CTA pairs)",
+                                   2: "LP GEMM bf16 8192^3 (tcgen05 cta_group::2, 256x512 tiles on CTA pairs)"}[pair]
+                                  + " preempted by HP stencil5 4096^2",
                       "chunk": 1, "poll": 1, "in_tile": in_tile, "pair": pair},
            "preempted_steps": pre, "not_bit_identical_to_uninterrupted": bad,
            "sample_max_rel": worst, "tol": 2e-2,
@@ -824,10 +826,12 @@ def _queue_instances(torch, F, seed):
                 A = (torch.rand(sz, sz, device="cuda", generator=g) * 2 - 1).to(torch.bfloat16)
                 B = (torch.rand(sz, sz, device="cuda", generator=g) * 2 - 1).to(torch.bfloat16)
                 C = torch.empty(sz, sz, device="cuda", dtype=torch.bfloat16)
-                pair = os.environ.get("FLEP_QUEUE_GEMM", "1") == "2"   # the CTA-pair body (R32)
-                inst[(ty, cls)] = ((F.BODY_GEMM_BF16_2SM, F.gemm2_grid(sz, sz)) if pair else
-                                   (F.BODY_GEMM_BF16, F.gemm_grid(sz, sz))) + (F.gemm_args(C, A, B), (A, B, C),
-                                   2 * sz ** 3)
+                # FLEP_QUEUE_GEMM: 1 the 1-CTA body, 2 the CTA-pair body (R32), 3 its wide tile
+                which = os.environ.get("FLEP_QUEUE_GEMM", "1")
+                inst[(ty, cls)] = {"1": (F.BODY_GEMM_BF16, F.gemm_grid(sz, sz)),
+                                   "2": (F.BODY_GEMM_BF16_2SM, F.gemm2_grid(sz, sz)),
+                                   "3": (F.BODY_GEMM_BF16_2SM_W, F.gemm2w_grid(sz, sz))}[which] + (
+                                       F.gemm_args(C, A, B), (A, B, C), 2 * sz ** 3)
     return inst
 
 
@@ -839,7 +843,7 @@ def _run_trace(F, torch, local, policy, trace, inst, t_alone, overhead_ns, strea
         C, pf = QUEUE_CHUNK[key[0]]
         kid[key] = rt.register_kernel(body, chunk=C, poll=1, prefetch=pf, name=f"{key[0]}-{key[1]}",
                                       model=(0, 0, 0, 0, float(t_alone[key])), overhead_ns=int(overhead_ns),
-                                      in_tile=body in (F.BODY_GEMM_BF16, F.BODY_GEMM_BF16_2SM))
+                                      in_tile=body in (F.BODY_GEMM_BF16, F.BODY_GEMM_BF16_2SM, F.BODY_GEMM_BF16_2SM_W))
     hs = []
     call_ns = []
     t0 = F.now_ns() + 2_000_000
@@ -892,7 +896,7 @@ def run_queue(args, rank, world, local):
     rt = F.Runtime(device=local, policy=F.POLICY_FIFO)
     for key, (body, grid, a, keep, _) in inst.items():
         C, pf = QUEUE_CHUNK[key[0]]
-        k = rt.register_kernel(body, chunk=C, poll=1, prefetch=pf, in_tile=body in (F.BODY_GEMM_BF16, F.BODY_GEMM_BF16_2SM))
+        k = rt.register_kernel(body, chunk=C, poll=1, prefetch=pf, in_tile=body in (F.BODY_GEMM_BF16, F.BODY_GEMM_BF16_2SM, F.BODY_GEMM_BF16_2SM_W))
         ts = []
         for r in range(4):
             flush.zero_()                      # cold L2: the queue interleaves working sets
@@ -1204,7 +1208,7 @@ def run_scale_queue(args, rank, world, local):
     rt_m = F.Runtime(device=local, exec_on_user_stream=True)
     for key, (body, grid, a, keep, _) in sorted(inst.items()):
         C, pf = QUEUE_CHUNK[key[0]]
-        k = rt.register_kernel(body, chunk=C, poll=1, prefetch=pf, in_tile=body in (F.BODY_GEMM_BF16, F.BODY_GEMM_BF16_2SM))
+        k = rt.register_kernel(body, chunk=C, poll=1, prefetch=pf, in_tile=body in (F.BODY_GEMM_BF16, F.BODY_GEMM_BF16_2SM, F.BODY_GEMM_BF16_2SM_W))
         ts = []
         for r in range(3):
             flush.zero_()
@@ -1215,7 +1219,7 @@ def run_scale_queue(args, rank, world, local):
             if r:
                 ts.append(info.t_finish - info.t_arrive)
         t_alone[key] = int(np.median(ts))
-        km = rt_m.register_kernel(body, chunk=C, poll=1, prefetch=pf, in_tile=body in (F.BODY_GEMM_BF16, F.BODY_GEMM_BF16_2SM))
+        km = rt_m.register_kernel(body, chunk=C, poll=1, prefetch=pf, in_tile=body in (F.BODY_GEMM_BF16, F.BODY_GEMM_BF16_2SM, F.BODY_GEMM_BF16_2SM_W))
         tw, tu = [], []
         for r in range(4):
             for mode in ("w", "u"):
@@ -1496,8 +1500,8 @@ def run_slicing_overhead(args, rank, world, local):
         for key in sorted(inst):
             body, grid, a, keep, _ = inst[key]
             C, pf = QUEUE_CHUNK[key[0]]
-            k_t = rt_m.register_kernel(body, chunk=C, poll=1, prefetch=pf, in_tile=body in (F.BODY_GEMM_BF16, F.BODY_GEMM_BF16_2SM))
-            k_1 = rt_m.register_kernel(body, chunk=1, poll=1, in_tile=body in (F.BODY_GEMM_BF16, F.BODY_GEMM_BF16_2SM))
+            k_t = rt_m.register_kernel(body, chunk=C, poll=1, prefetch=pf, in_tile=body in (F.BODY_GEMM_BF16, F.BODY_GEMM_BF16_2SM, F.BODY_GEMM_BF16_2SM_W))
+            k_1 = rt_m.register_kernel(body, chunk=1, poll=1, in_tile=body in (F.BODY_GEMM_BF16, F.BODY_GEMM_BF16_2SM, F.BODY_GEMM_BF16_2SM_W))
             k_s = rt_s.register_kernel(body, chunk=C, poll=1)
             cps, w = rt_m.workers_for(body)
             slice_blocks = w * C                                     # one wave of W*C*K blocks (A20)
@@ -1545,7 +1549,10 @@ def run_slicing_overhead(args, rank, world, local):
         a8 = F.gemm_args(C8, A8, B8)
         g2 = F.gemm2_grid(C8.shape[0], C8.shape[1])
         k2 = {c: rt_m.register_kernel(F.BODY_GEMM_BF16_2SM, chunk=c, poll=1) for c in (1, 2)}
-        tg = {m: [] for m in ("cublas", "unwrapped", "static_u1", "flep_c1", "flep_c2")}
+        g2w = F.gemm2w_grid(C8.shape[0], C8.shape[1])          # the 256x512 pair tile
+        k2w = rt_m.register_kernel(F.BODY_GEMM_BF16_2SM_W, chunk=1, poll=1)
+        tg = {m: [] for m in ("cublas", "unwrapped", "static_u1", "flep_c1", "flep_c2",
+                              "wide_unwrapped", "wide_static_u1", "wide_flep_c1")}
         for r in range(max(6, reps // 2) + 2):
             for m in tg:
                 with torch.cuda.stream(S):
@@ -1558,6 +1565,12 @@ def run_slicing_overhead(args, rank, world, local):
                         rt_m.launch_unwrapped(F.BODY_GEMM_BF16_2SM, g2, a8, stream=S)
                     elif m == "static_u1":
                         rt_m.launch_static(F.BODY_GEMM_BF16_2SM, g2, a8, stream=S)
+                    elif m == "wide_unwrapped":
+                        rt_m.launch_unwrapped(F.BODY_GEMM_BF16_2SM_W, g2w, a8, stream=S)
+                    elif m == "wide_static_u1":
+                        rt_m.launch_static(F.BODY_GEMM_BF16_2SM_W, g2w, a8, stream=S)
+                    elif m == "wide_flep_c1":
+                        h = rt_m.launch(k2w, g2w, a8, stream=S)
                     else:
                         h = rt_m.launch(k2[1 if m == "flep_c1" else 2], g2, a8, stream=S)
                     e1.record(S)
@@ -1573,7 +1586,9 @@ def run_slicing_overhead(args, rank, world, local):
                  **{m + "_tflops": round(flop / v / 1e6, 1) for m, v in gm.items()},
                  "flep_c2_vs_cublas": round(gm["cublas"] / gm["flep_c2"], 3),
                  "flep_c2_over_static_pct": round((gm["flep_c2"] / gm["static_u1"] - 1) * 100, 2),
-                 "flep_c1_over_static_pct": round((gm["flep_c1"] / gm["static_u1"] - 1) * 100, 2)}
+                 "flep_c1_over_static_pct": round((gm["flep_c1"] / gm["static_u1"] - 1) * 100, 2),
+                 "wide_flep_c1_vs_cublas": round(gm["cublas"] / gm["wide_flep_c1"], 3),
+                 "wide_flep_c1_over_static_pct": round((gm["wide_flep_c1"] / gm["wide_static_u1"] - 1) * 100, 2)}
     rt_m.close()
     rt_s.close()
     big = [r for r in rows if r["kernel"].endswith("-2")]

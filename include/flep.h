@@ -97,11 +97,17 @@ typedef enum {
   FLEP_BODY_SPMV_CSR_F32_VEC = 8, /* y = A x, CSR fp32, CSR-vector form (4 lanes per row, shuffle
                                   reduction, no shared memory); same args; 128 rows per block,
                                   each warp owns 16 of them (warp-task capable, R30) */
-  FLEP_BODY_GEMM_BF16_2SM = 9  /* GEMM_BF16 on CTA pairs (cluster of 2, tcgen05.mma.cta_group::2):
+  FLEP_BODY_GEMM_BF16_2SM = 9, /* GEMM_BF16 on CTA pairs (cluster of 2, tcgen05.mma.cta_group::2):
                                   256x256 output tile per block, grid (N/256, M/256, 1),
                                   M % 256 == N % 256 == K % 64 == 0; the worker is the pair
                                   (flep_launch_info.workers = pairs), tile-granular preemption, a
                                   spatial request releases a pair iff it names either SM (R32) */
+  FLEP_BODY_GEMM_BF16_2SM_W = 10 /* GEMM_BF16_2SM with a 256x512 output tile per block (two
+                                  N = 256 MMAs per k-slice into one 512-column TMEM accumulator):
+                                  grid (N/512, M/256, 1), M % 256 == N % 512 == K % 64 == 0;
+                                  a quarter less L2 -> SM operand traffic per flop than the
+                                  256x256 tile, no overlap of one tile's epilogue with the next
+                                  tile's MMAs; in-tile preemption spills 256 KiB per CTA */
 } flep_body;
 
 /* Per-body argument structs (copied by value at launch). All pointers are device pointers. */

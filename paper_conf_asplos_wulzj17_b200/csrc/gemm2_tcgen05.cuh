@@ -40,19 +40,38 @@ namespace flep {
 struct Gemm2Args {
   CUtensorMap tma_a;           // A [M,K] bf16, box {64, 128}, SWIZZLE_128B
   CUtensorMap tma_b;           // B [N,K] bf16, box {64, 128}, SWIZZLE_128B
+  CUtensorMap tma_c;           // C [M,N] bf16, box {64, 32}, SWIZZLE_128B (epilogue bulk stores)
   __nv_bfloat16* c;            // C [M,N] bf16 row-major
   uint32_t m, n, k;
 };
 
-struct Gemm2 {
+template <uint32_t kBN>
+struct Gemm2T {
   static constexpr int kThreads = 256;
-  static constexpr uint32_t BM = 128, BN = 256, BK = 64, UMMA_K = 16, STAGES = 6;
+  // BN = 256: the 256x256 pair tile, two TMEM accumulators (the epilogue of one tile overlaps the
+  // next tile's MMAs), 6 stages of 32 KB. BN = 512 (the wide tile, FLEP_BODY_GEMM_BF16_2SM_W): a
+  // 256x512 pair tile as two N = 256 MMAs per k-slice into one 512-column accumulator, 4 stages of
+  // 48 KB: per k-step each SM loads 16 KB of A and 32 KB of B for twice the MMA work, so L2 -> SM
+  // operand traffic per flop drops by a quarter more (the tensor pipe is ~96 % active in both
+  // shapes at 8192^3; the wide tile's lower fabric traffic is what keeps the clock up under the
+  // power cap).
+  static constexpr uint32_t BM = 128, BN = kBN, BK = 64, UMMA_K = 16, MMA_N = 256;
+  static constexpr uint32_t NH = BN / MMA_N;                   // MMAs per k-slice (B halves of 128 rows per CTA)
+  static constexpr uint32_t NACC = 512 / BN;                   // TMEM accumulators (512 columns in all)
+  static constexpr uint32_t STAGES = NH == 1 ? 6 : 4;
+  static_assert(NH == 1 || NH == 2, "BN is 256 or 512");
   static constexpr uint32_t TM = 2 * BM;                       // tile rows of the pair
-  static constexpr uint32_t kBytesA = BM * BK * 2, kBytesB = (BN / 2) * BK * 2, kStage = kBytesA + kBytesB;
-  static constexpr uint32_t kTmemCols = 512;                   // two 128-lane x 256-column accumulators
+  static constexpr uint32_t kHalfB = 128 * BK * 2;             // one 128-row B box (16 KB)
+  static constexpr uint32_t kBytesA = BM * BK * 2, kBytesB = NH * kHalfB, kStage = kBytesA + kBytesB;
+  static constexpr uint32_t kTmemCols = 512;                   // NACC accumulators of 128 lanes x BN columns
+  static constexpr size_t kSpill = kSpillBytes * NH;           // one CTA's fp32 128 x BN half
   static constexpr uint32_t QDEPTH = 4;
   static constexpr uint32_t kQConsumers = 10;                  // leader: MMA + 4 epilogue warps; peer: producer + 4
-  static constexpr size_t kDynSmem = 1024 + STAGES * kStage + 1024;
+  // epilogue staging: per epilogue warp two 4 KB buffers of 32 rows x 64 bf16 columns (128-B
+  // rows, SWIZZLE_128B) that a bulk tensor store writes to C
+  static constexpr uint32_t kEpiBuf = 32 * 128;
+  static constexpr size_t kDynSmem = 1024 + STAGES * kStage + 1024 + 4 * 2 * kEpiBuf;
+  static_assert(kDynSmem <= 232448, "shared memory per block");
   static constexpr uint32_t STOP = 0xffffffffu;
   static constexpr uint32_t STOP_PARTIAL = 0xfffffffeu;         // in-tile: the last tile was stopped
 
@@ -76,6 +95,9 @@ struct Gemm2 {
     return dsmem + (((a + 1023u) & ~1023u) - a);
   }
   __device__ static State* state() { return reinterpret_cast<State*>(ring() + STAGES * kStage); }
+  __device__ static uint8_t* epi_buf(uint32_t q, uint32_t bi) {
+    return ring() + STAGES * kStage + 1024 + (2 * q + bi) * kEpiBuf;
+  }
   __device__ static uint32_t su32(const void* p) { return static_cast<uint32_t>(__cvta_generic_to_shared(p)); }
   __device__ static uint32_t rank() { uint32_t r; asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r)); return r; }
   // shared::cluster address of `local` in CTA `r` of the cluster
@@ -93,6 +115,13 @@ struct Gemm2 {
     asm volatile(
         "{\n .reg .pred p;\n W: mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 p, [%0], %1;\n"
         " @!p bra W;\n}\n" :: "r"(su32(b)), "r"(parity) : "memory");
+  }
+  __device__ static bool test_wait(uint64_t* b, uint32_t parity) {
+    uint32_t ok;
+    asm volatile(
+        "{\n .reg .pred p;\n mbarrier.test_wait.parity.acquire.cluster.shared::cta.b64 p, [%1], %2;\n"
+        " selp.u32 %0, 1, 0, p;\n}\n" : "=r"(ok) : "r"(su32(b)), "r"(parity) : "memory");
+    return ok != 0;
   }
   __device__ static void arrive_local(uint64_t* b) {
     asm volatile("mbarrier.arrive.release.cta.shared::cta.b64 _, [%0];" :: "r"(su32(b)) : "memory");
@@ -115,7 +144,48 @@ struct Gemm2 {
            ((uint64_t)1u << 46) | ((uint64_t)2u << 61);
   }
   // kind::f16, D f32, A/B bf16 K-major, N = 256, M = 256 (the pair)
-  static constexpr uint32_t kIdesc = (1u << 4) | (1u << 7) | (1u << 10) | ((BN >> 3) << 17) | ((TM >> 4) << 24);
+  static constexpr uint32_t kIdesc = (1u << 4) | (1u << 7) | (1u << 10) | ((MMA_N >> 3) << 17) | ((TM >> 4) << 24);
+  // this CTA's B rows of a k-step: for MMA h, rows tn*BN + 256h + 128r .. +127 (a cta_group::2
+  // MMA with N = 256 takes B rows 0..127 from the leader's and 128..255 from the peer's smem)
+  __device__ static void load_b(const Gemm2Args& g, uint8_t* sb, uint32_t fb, uint32_t kb, int32_t tn, uint32_t r) {
+#pragma unroll
+    for (uint32_t h = 0; h < NH; ++h)
+      tma_2sm(&g.tma_b, sb + h * kHalfB, fb, (int32_t)(kb * BK), tn * (int32_t)BN + (int32_t)(h * MMA_N + r * 128));
+  }
+  // the MMAs of one k-step for column half h of the wide tile (B box h)
+  __device__ static void mma_half(uint32_t tmem_h, uint32_t sa, uint32_t kb, uint32_t h) {
+    const uint32_t sb = sa + kBytesA + h * kHalfB;
+#pragma unroll
+    for (uint32_t k = 0; k < BK / UMMA_K; ++k) {
+      const uint64_t da = sdesc(sa + k * UMMA_K * 2), db = sdesc(sb + k * UMMA_K * 2);
+      const uint32_t accum = (kb | k) ? 1u : 0u;
+      asm volatile(
+          "{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n"
+          " tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n}\n"
+          :: "r"(tmem_h), "l"(da), "l"(db), "r"(kIdesc), "r"(accum) : "memory");
+    }
+  }
+  __device__ static void commit_multicast(uint64_t* b) {   // arrives on b in both CTAs of the pair
+    asm volatile("tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;"
+                 :: "r"(su32(b)), "h"((uint16_t)3) : "memory");
+  }
+  // the MMAs of one k-step (stage at sa: A, then the NH B boxes)
+  __device__ static void mma_kstep(uint32_t tmem, uint32_t sa, uint32_t kb) {
+    const uint32_t sb = sa + kBytesA;
+#pragma unroll
+    for (uint32_t k = 0; k < BK / UMMA_K; ++k) {
+      const uint64_t da = sdesc(sa + k * UMMA_K * 2);
+      const uint32_t accum = (kb | k) ? 1u : 0u;
+#pragma unroll
+      for (uint32_t h = 0; h < NH; ++h) {
+        const uint64_t db = sdesc(sb + h * kHalfB + k * UMMA_K * 2);
+        asm volatile(
+            "{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n"
+            " tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n}\n"
+            :: "r"(tmem + h * MMA_N), "l"(da), "l"(db), "r"(kIdesc), "r"(accum) : "memory");
+      }
+    }
+  }
 
   // original block b -> 256x256 tile (tm, tn): bands of GROUP tile-rows, column-major inside
   static constexpr uint32_t GROUP = 8;
@@ -162,6 +232,54 @@ struct Gemm2 {
       asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" :: "r"(s->tmem_base), "r"(kTmemCols) : "memory");
   }
 
+  // Epilogue of one warp's 32 accumulator rows, columns [c_begin, c_end) (multiples of 64):
+  // TMEM -> bf16 -> this warp's staging buffer (row = lane, 16-B chunk c at c ^ (lane & 7), the
+  // SWIZZLE_128B layout) -> one bulk tensor store of 32 x 64 per 64 columns, issued by lane 0;
+  // two buffers per warp, so the store of one chunk overlaps the next chunk's TMEM loads. `it`
+  // counts this warp's stores (buffer = it & 1); the caller ends with bulk_wait_all().
+  __device__ static void store_cols(const Gemm2Args& g, uint32_t tmem_w, uint32_t c_begin, uint32_t c_end,
+                                    int32_t x0, int32_t y0, uint32_t q, uint32_t lane, uint32_t& it) {
+#pragma unroll 1
+    for (uint32_t c0 = c_begin; c0 < c_end; c0 += 64) {
+      uint32_t o[32];
+#pragma unroll
+      for (uint32_t hh = 0; hh < 2; ++hh) {
+        uint32_t v[32];
+        GemmBody::tmem_ld32(tmem_w + c0 + 32 * hh, v);
+#pragma unroll
+        for (int i = 0; i < 16; ++i) {
+          __nv_bfloat162 hv = __floats2bfloat162_rn(__uint_as_float(v[2 * i]), __uint_as_float(v[2 * i + 1]));
+          o[16 * hh + i] = *reinterpret_cast<uint32_t*>(&hv);
+        }
+      }
+      const uint32_t bi = it & 1u;
+      if (it >= 2) {                                   // the store that used this buffer has read it
+        if (lane == 0) asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
+        __syncwarp();
+      }
+      uint8_t* buf = epi_buf(q, bi);
+      const uint32_t rowb = su32(buf) + lane * 128u;
+#pragma unroll
+      for (uint32_t c = 0; c < 8; ++c)
+        asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};"
+                     :: "r"(rowb + ((c ^ (lane & 7u)) << 4)), "r"(o[4 * c]), "r"(o[4 * c + 1]), "r"(o[4 * c + 2]),
+                        "r"(o[4 * c + 3]) : "memory");
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // visible to the bulk store
+      __syncwarp();
+      if (lane == 0) {
+        asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];"
+                     :: "l"(reinterpret_cast<uint64_t>(&g.tma_c)), "r"(su32(buf)), "r"(x0 + (int32_t)c0), "r"(y0)
+                     : "memory");
+        asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+      }
+      ++it;
+    }
+  }
+  __device__ static void bulk_wait_all(uint32_t lane) {     // this warp's stores complete
+    if (lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+    __syncwarp();
+  }
+
   // The pair's pipeline. Next(b0, b1) is called by the leader's scheduling thread: it returns
   // false when the pair must stop, else the next chunk [b0, b1) of tiles. Returns after both
   // CTAs drained every tile handed out.
@@ -185,7 +303,7 @@ struct Gemm2 {
           if (leader) expect_tx(&s->full[st], 2 * kStage);
           const uint32_t fb = full0 + st * 8u;
           tma_2sm(&g.tma_a, sa, fb, (int32_t)(kb * BK), tm * (int32_t)TM + (int32_t)(r * BM));
-          tma_2sm(&g.tma_b, sa + kBytesA, fb, (int32_t)(kb * BK), tn * (int32_t)BN + (int32_t)(r * (BN / 2)));
+          load_b(g, sa + kBytesA, fb, kb, tn, r);
           if (++st == STAGES) { st = 0; ph ^= 1u; }
         }
       };
@@ -222,36 +340,56 @@ struct Gemm2 {
         arrive_local(&s->qempty[qi]);
         if (++qi == QDEPTH) { qi = 0; qph ^= 1u; }
         if (tile == STOP) break;
-        wait(&s->tempty[acc], aph ^ 1u);                 // both CTAs' epilogues drained this half
-        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-        const uint32_t tmem = tmem0 + acc * BN;
-        for (uint32_t kb = 0; kb < nk; ++kb) {
-          wait(&s->full[st], ph);
+        if constexpr (NH == 1) {
+          wait(&s->tempty[acc], aph ^ 1u);               // both CTAs' epilogues drained this accumulator
           asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-          const uint32_t sa = su32(base + st * kStage), sb = sa + kBytesA;
-#pragma unroll
-          for (uint32_t k = 0; k < BK / UMMA_K; ++k) {
-            const uint64_t da = sdesc(sa + k * UMMA_K * 2), db = sdesc(sb + k * UMMA_K * 2);
-            const uint32_t accum = (kb | k) ? 1u : 0u;
-            asm volatile(
-                "{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n"
-                " tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n}\n"
-                :: "r"(tmem), "l"(da), "l"(db), "r"(kIdesc), "r"(accum) : "memory");
+          const uint32_t tmem = tmem0 + acc * BN;
+          for (uint32_t kb = 0; kb < nk; ++kb) {
+            wait(&s->full[st], ph);
+            asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+            mma_kstep(tmem, su32(base + st * kStage), kb);
+            commit_multicast(&s->empty[st]);             // frees stage st in both CTAs
+            if (++st == STAGES) { st = 0; ph ^= 1u; }
           }
-          // frees stage st in both CTAs
-          asm volatile("tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;"
-                       :: "r"(su32(&s->empty[st])), "h"((uint16_t)3) : "memory");
-          if (++st == STAGES) { st = 0; ph ^= 1u; }
+        } else {
+          // Wide tile, one accumulator: tempty[h] says column half h is drained. The MMAs of
+          // half 0 start as soon as half 0 is drained and run up to STAGES k-steps ahead of
+          // half 1's while the epilogue still drains half 1 (a stage is freed once both halves
+          // consumed it); each half still accumulates its k-steps in order (bit-identical).
+          wait(&s->tempty[0], aph ^ 1u);
+          asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+          uint32_t kb0 = 0, kb1 = 0, st0 = st, ph0 = ph;
+          bool h1 = false;
+          while (kb1 < nk) {
+            if (!h1 && test_wait(&s->tempty[1], aph ^ 1u)) {
+              h1 = true;
+              asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+            }
+            if (h1 && kb1 < kb0) {
+              mma_half(tmem0 + MMA_N, su32(base + st * kStage), kb1, 1);
+              commit_multicast(&s->empty[st]);
+              if (++st == STAGES) { st = 0; ph ^= 1u; }
+              ++kb1;
+            } else if (kb0 < nk && kb0 - kb1 < STAGES) {
+              wait(&s->full[st0], ph0);
+              asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+              mma_half(tmem0, su32(base + st0 * kStage), kb0, 0);
+              if (++st0 == STAGES) { st0 = 0; ph0 ^= 1u; }
+              ++kb0;
+            } else {
+              wait(&s->tempty[1], aph ^ 1u);
+              h1 = true;
+              asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+            }
+          }
         }
-        // the accumulator half is complete in both CTAs' TMEM
-        asm volatile("tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;"
-                     :: "r"(su32(&s->tfull[acc])), "h"((uint16_t)3) : "memory");
-        if (++acc == 2) { acc = 0; aph ^= 1u; }
+        // the accumulator is complete in both CTAs' TMEM
+        commit_multicast(&s->tfull[NH == 1 ? acc : 0u]);
+        if (++acc == NACC) { acc = 0; aph ^= 1u; }
       }
     } else if (warp >= 4) {                              // ---- epilogue: this CTA's 128 rows
       const uint32_t q = warp - 4;
-      const uint32_t rl = q * 32u + lane;
-      uint32_t qi = 0, qph = 0, acc = 0, aph = 0;
+      uint32_t qi = 0, qph = 0, acc = 0, aph = 0, it = 0;
       const uint32_t tempty0 = peer_addr(&s->tempty[0], 0);
       while (true) {
         wait(&s->qfull[qi], qph);
@@ -268,31 +406,22 @@ struct Gemm2 {
         wait(&s->tfull[acc], aph);
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
         const uint32_t tmem = s->tmem_base + acc * BN + ((q * 32u) << 16);
-        const uint32_t row = (uint32_t)tm * TM + r * BM + rl;
-        __nv_bfloat16* crow = g.c + (size_t)row * g.n + (size_t)tn * BN;
+        const int32_t x0 = tn * (int32_t)BN, y0 = tm * (int32_t)TM + (int32_t)(r * BM + q * 32u);
+        // NH == 1: one arrive on tempty[acc] after the whole tile; NH == 2: one per column half
 #pragma unroll 1
-        for (uint32_t c0 = 0; c0 < BN; c0 += 32) {
-          uint32_t v[32];
-          GemmBody::tmem_ld32(tmem + c0, v);
-          uint4 o[4];
-          uint32_t* ow = reinterpret_cast<uint32_t*>(o);
-#pragma unroll
-          for (int i = 0; i < 16; ++i) {
-            __nv_bfloat162 h = __floats2bfloat162_rn(__uint_as_float(v[2 * i]), __uint_as_float(v[2 * i + 1]));
-            ow[i] = *reinterpret_cast<uint32_t*>(&h);
+        for (uint32_t h = 0; h < NH; ++h) {
+          store_cols(g, tmem, h * MMA_N, (h + 1) * MMA_N, x0, y0, q, lane, it);
+          asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+          __syncwarp();
+          const uint32_t e = NH == 1 ? acc : h;
+          if (lane == 0) {
+            if (leader) arrive_local(&s->tempty[e]);
+            else arrive_remote(tempty0 + e * 8u);
           }
-          uint4* dst = reinterpret_cast<uint4*>(crow + c0);
-#pragma unroll
-          for (int i = 0; i < 4; ++i) dst[i] = o[i];
         }
-        asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
-        __syncwarp();
-        if (lane == 0) {
-          if (leader) arrive_local(&s->tempty[acc]);
-          else arrive_remote(tempty0 + acc * 8u);
-        }
-        if (++acc == 2) { acc = 0; aph ^= 1u; }
+        if (++acc == NACC) { acc = 0; aph ^= 1u; }
       }
+      bulk_wait_all(lane);
     }
   }
 
@@ -317,7 +446,7 @@ struct Gemm2 {
   static_assert(kLicSlack <= kMinLeft, "the catch-up loads must stay inside the tile");
   __device__ static float4* spill_slot(const WorkerParams& p, uint32_t wid, uint32_t r) {
     return reinterpret_cast<float4*>(reinterpret_cast<uint8_t*>(p.partial) + partial_header_bytes(2 * p.workers) +
-                                     (size_t)(2 * wid + r) * kSpillBytes);
+                                     (size_t)(2 * wid + r) * kSpill);
   }
   template <bool kCov, class Fetch>
   __device__ static void worker_pipeline(const Gemm2Args& g, const WorkerParams& p, WorkerShared& ws,
@@ -410,7 +539,7 @@ struct Gemm2 {
               expect_tx(&s->full[st], 2 * kStage);
               const uint32_t fb = full0 + st * 8u;
               tma_2sm(&g.tma_a, sa, fb, (int32_t)(kb * BK), tm * (int32_t)TM);
-              tma_2sm(&g.tma_b, sa + kBytesA, fb, (int32_t)(kb * BK), tn * (int32_t)BN);
+              load_b(g, sa + kBytesA, fb, kb, tn, 0);
               ++q;
               // the licence orders nothing else (relaxed: a release here fences every k-step)
               if (in_tile && !stopping)
@@ -461,7 +590,7 @@ struct Gemm2 {
             uint8_t* sa = base + st * kStage;
             const uint32_t fb = full0 + st * 8u;
             tma_2sm(&g.tma_a, sa, fb, (int32_t)(kb * BK), tm * (int32_t)TM + (int32_t)BM);
-            tma_2sm(&g.tma_b, sa + kBytesA, fb, (int32_t)(kb * BK), tn * (int32_t)BN + (int32_t)(BN / 2));
+            load_b(g, sa + kBytesA, fb, kb, tn, 1);
             ++q;
             if (++st == STAGES) { st = 0; ph ^= 1u; }
           }
@@ -481,6 +610,7 @@ struct Gemm2 {
         if (++qi == QDEPTH) { qi = 0; qph ^= 1u; }
         if (tile >= STOP_PARTIAL) break;
         wait(&s->tempty[acc], aph ^ 1u);
+        if constexpr (NH == 2) wait(&s->tempty[1], aph ^ 1u);   // wide tile: both column halves drained
         if (kb0 > 0) { wait(&s->trest[acc], rph[acc]); rph[acc] ^= 1u; }   // both halves restored
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
         const uint32_t tmem = tmem0 + acc * BN;
@@ -493,28 +623,19 @@ struct Gemm2 {
             break;
           }
           asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-          const uint32_t sa = su32(base + st * kStage), sb = sa + kBytesA;
-#pragma unroll
-          for (uint32_t k = 0; k < BK / UMMA_K; ++k) {
-            const uint64_t da = sdesc(sa + k * UMMA_K * 2), db = sdesc(sb + k * UMMA_K * 2);
-            const uint32_t accum = (kb | k) ? 1u : 0u;
-            asm volatile(
-                "{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n"
-                " tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n}\n"
-                :: "r"(tmem), "l"(da), "l"(db), "r"(kIdesc), "r"(accum) : "memory");
-          }
+          mma_kstep(tmem, su32(base + st * kStage), kb);
           asm volatile("tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;"
                        :: "r"(su32(&s->empty[st])), "h"((uint16_t)3) : "memory");
           if (++st == STAGES) { st = 0; ph ^= 1u; }
         }
         asm volatile("tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;"
                      :: "r"(su32(&s->tfull[acc])), "h"((uint16_t)3) : "memory");
-        if (++acc == 2) { acc = 0; aph ^= 1u; }
+        if (++acc == NACC) { acc = 0; aph ^= 1u; }
       }
     } else if (warp >= 4) {                              // ---- epilogue: this CTA's 128 rows
       const uint32_t qw = warp - 4;
       const uint32_t rl = qw * 32u + lane;
-      uint32_t qi = 0, qph = 0, acc = 0, aph = 0;
+      uint32_t qi = 0, qph = 0, acc = 0, aph = 0, it = 0;
       const uint32_t tempty0 = peer_addr(&s->tempty[0], 0), trest0 = peer_addr(&s->trest[0], 0);
       while (true) {
         wait(&s->qfull[qi], qph);
@@ -570,60 +691,51 @@ struct Gemm2 {
                                  __uint_as_float(v[4 * j + 2]), __uint_as_float(v[4 * j + 3])));
           }
         } else {
-          const uint32_t row = (uint32_t)tm * TM + r * BM + rl;
-          __nv_bfloat16* crow = g.c + (size_t)row * g.n + (size_t)tn * BN;
-#pragma unroll 1
-          for (uint32_t c0 = 0; c0 < BN; c0 += 32) {
-            uint32_t v[32];
-            GemmBody::tmem_ld32(tmem + c0, v);
-            uint4 o[4];
-            uint32_t* ow = reinterpret_cast<uint32_t*>(o);
-#pragma unroll
-            for (int i = 0; i < 16; ++i) {
-              __nv_bfloat162 h = __floats2bfloat162_rn(__uint_as_float(v[2 * i]), __uint_as_float(v[2 * i + 1]));
-              ow[i] = *reinterpret_cast<uint32_t*>(&h);
-            }
-            uint4* dst = reinterpret_cast<uint4*>(crow + c0);
-#pragma unroll
-            for (int i = 0; i < 4; ++i) dst[i] = o[i];
-          }
+          store_cols(g, tmem, 0, BN, tn * (int32_t)BN, tm * (int32_t)TM + (int32_t)(r * BM + qw * 32u), qw, lane, it);
         }
         asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
         __syncwarp();
         if (lane == 0) {
           if (leader) arrive_local(&s->tempty[acc]);
           else arrive_remote(tempty0 + acc * 8u);
+          if constexpr (NH == 2) {                       // wide tile: tempty[1] = column half 1
+            if (leader) arrive_local(&s->tempty[1]);
+            else arrive_remote(tempty0 + 8u);
+          }
         }
-        if (++acc == 2) { acc = 0; aph ^= 1u; }
+        if (++acc == NACC) { acc = 0; aph ^= 1u; }
       }
+      bulk_wait_all(lane);
     }
   }
 };
+using Gemm2 = Gemm2T<256>;
+using Gemm2W = Gemm2T<512>;
 
 // Worker (the PAIR is the FLEP worker: wid = cluster index, W = pairs). The leader runs the
 // scheduling step of flep_worker (next_chunk: poll every K chunks, fetch C tiles, exit event);
 // the spatial check uses the pair's lower-ranked SM so that a request naming either SM releases it.
-template <bool kCoverage>
-__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Gemm2::kThreads, 1)
+template <class G, bool kCoverage>
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(256, 1)
 flep_gemm2_worker(const __grid_constant__ Gemm2Args g, const WorkerParams p) {
   __shared__ WorkerShared ws;
   const uint32_t wid = blockIdx.x >> 1;
-  const bool leader = Gemm2::rank() == 0;
+  const bool leader = G::rank() == 0;
   if (threadIdx.x == 0) {
     ws.sm = smid_reg(); ws.t_entry = gtimer(); ws.blocks = 0; ws.reason = 0;
     ws.counted = 0; ws.last = 0; ws.ev_raw = 0; ws.ev_part = 0; ws.partial = 0;
     if (wid == 0 && leader && p.started_hint && p.status) st_relaxed_sys(&p.status->started, p.epoch);
   }
-  Gemm2::setup();
+  G::setup();
   uint32_t yield_sm = 0;
   if (leader && threadIdx.x == 0) {                    // the pair's SM with the lower rank (spatial)
     uint32_t peer_sm;
-    asm volatile("ld.shared::cluster.u32 %0, [%1];" : "=r"(peer_sm) : "r"(Gemm2::peer_addr(&Gemm2::state()->smid, 1)) : "memory");
+    asm volatile("ld.shared::cluster.u32 %0, [%1];" : "=r"(peer_sm) : "r"(G::peer_addr(&G::state()->smid, 1)) : "memory");
     yield_sm = p.rank[peer_sm] < p.rank[ws.sm] ? peer_sm : ws.sm;
     ws.sm = yield_sm;                                  // the worker record names the deciding SM
   }
   if (p.partial) {                                     // in-tile preemption (R21 on the pair)
-    Gemm2::worker_pipeline<kCoverage>(g, p, ws, wid, yield_sm, [&](SchedState& st, uint32_t& b0, uint32_t& b1) {
+    G::template worker_pipeline<kCoverage>(g, p, ws, wid, yield_sm, [&](SchedState& st, uint32_t& b0, uint32_t& b1) {
       b0 = next_chunk(p, st, ws, wid, yield_sm);
       if (b0 == 0xffffffffu) return false;
       b1 = min(b0 + p.chunk, p.n_blocks);
@@ -631,7 +743,7 @@ flep_gemm2_worker(const __grid_constant__ Gemm2Args g, const WorkerParams p) {
     });
   } else {
     SchedState st;
-    Gemm2::pipeline(g, p.gx, p.gy, [&](uint32_t& b0, uint32_t& b1) {
+    G::pipeline(g, p.gx, p.gy, [&](uint32_t& b0, uint32_t& b1) {
       b0 = next_chunk(p, st, ws, wid, yield_sm);
       if (b0 == 0xffffffffu) return false;
       b1 = min(b0 + p.chunk, p.n_blocks);
@@ -640,28 +752,30 @@ flep_gemm2_worker(const __grid_constant__ Gemm2Args g, const WorkerParams p) {
       return true;
     });
   }
-  Gemm2::teardown();
+  G::teardown();
   if (leader && threadIdx.x == 0) worker_exit(p, ws, wid);
 }
 
 // The original kernel (unwrapped twin): one pair per tile.
-__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Gemm2::kThreads, 1)
+template <class G>
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(256, 1)
 flep_gemm2_unwrapped(const __grid_constant__ Gemm2Args g, uint32_t gx, uint32_t gy, uint32_t offset) {
-  Gemm2::setup();
+  G::setup();
   const uint32_t b = offset + (blockIdx.x >> 1) + (gridDim.x >> 1) * blockIdx.y;
   bool given = false;
-  Gemm2::pipeline(g, gx, gy, [&](uint32_t& b0, uint32_t& b1) {
+  G::pipeline(g, gx, gy, [&](uint32_t& b0, uint32_t& b1) {
     if (given) return false;
     given = true; b0 = b; b1 = b + 1;
     return true;
   });
-  Gemm2::teardown();
+  G::teardown();
 }
 
 // Kernel slicing with the device check (R31): one pair per tile of the slice; every CTA follows
 // the slice's one decision (taken by the first CTA of the slice that gets there), so both CTAs of
 // a pair agree.
-__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Gemm2::kThreads, 1)
+template <class G>
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(256, 1)
 flep_gemm2_slice(const __grid_constant__ Gemm2Args g, uint32_t gx, uint32_t gy, uint32_t offset, const SliceParams sp) {
   __shared__ uint32_t s_go;
   if (threadIdx.x == 0) {
@@ -683,30 +797,31 @@ flep_gemm2_slice(const __grid_constant__ Gemm2Args g, uint32_t gx, uint32_t gy, 
   }
   __syncthreads();
   if (!s_go) return;                   // both CTAs of the pair leave (same decision)
-  Gemm2::setup();
+  G::setup();
   const uint32_t b = offset + (blockIdx.x >> 1);
   bool given = false;
-  Gemm2::pipeline(g, gx, gy, [&](uint32_t& b0, uint32_t& b1) {
+  G::pipeline(g, gx, gy, [&](uint32_t& b0, uint32_t& b1) {
     if (given) return false;
     given = true; b0 = b; b1 = b + 1;
     return true;
   });
-  Gemm2::teardown();
+  G::teardown();
 }
 
 // Static persistent twin (U1): the same pairs, tiles pair, pair + P, pair + 2P, ... with no
 // counter and no poll (the FLEP worker's overhead baseline).
-__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Gemm2::kThreads, 1)
+template <class G>
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(256, 1)
 flep_gemm2_static(const __grid_constant__ Gemm2Args g, uint32_t gx, uint32_t gy, uint32_t n_tiles) {
-  Gemm2::setup();
+  G::setup();
   const uint32_t pair = blockIdx.x >> 1, pairs = gridDim.x >> 1;
   uint32_t next = pair;
-  Gemm2::pipeline(g, gx, gy, [&](uint32_t& b0, uint32_t& b1) {
+  G::pipeline(g, gx, gy, [&](uint32_t& b0, uint32_t& b1) {
     if (next >= n_tiles) return false;
     b0 = next; b1 = next + 1; next += pairs;
     return true;
   });
-  Gemm2::teardown();
+  G::teardown();
 }
 
 

@@ -236,6 +236,9 @@ const BodyOps kOps[] = {
     {FLEP_BODY_GEMM_BF16_2SM, 256 /* Gemm2::kThreads (gemm2_tcgen05.cuh, its own TU) */, sizeof(flep_gemm_args), &gemm2_worker_launch,
      &gemm2_unwrapped_launch, &gemm2_occupancy, &gemm2_validate, nullptr, nullptr, nullptr, nullptr, nullptr, 0,
      &gemm2_slice_launch, &gemm2_static_launch, &gemm2_max_pairs},
+    {FLEP_BODY_GEMM_BF16_2SM_W, 256 /* Gemm2W::kThreads */, sizeof(flep_gemm_args), &gemm2w_worker_launch,
+     &gemm2w_unwrapped_launch, &gemm2w_occupancy, &gemm2w_validate, nullptr, nullptr, nullptr, nullptr, nullptr, 0,
+     &gemm2w_slice_launch, &gemm2w_static_launch, &gemm2w_max_pairs, nullptr, nullptr, 2},
 };
 
 }  // namespace
@@ -247,7 +250,7 @@ cudaError_t set_unwrapped_trace(uint64_t* p) {
 #endif
 
 const BodyOps* body_ops(int32_t body) {
-  if (body < 1 || body > FLEP_BODY_GEMM_BF16_2SM) return nullptr;
+  if (body < 1 || body > FLEP_BODY_GEMM_BF16_2SM_W) return nullptr;
   return &kOps[body];
 }
 

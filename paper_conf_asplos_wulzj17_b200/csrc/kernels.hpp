@@ -42,6 +42,8 @@ struct BodyOps {
   // in-chunk stop worker (flep_worker_ic<Body>, R33) and its occupancy
   cudaError_t (*worker_ic)(const void* args, const WorkerParams& p, uint32_t W, cudaStream_t s, bool cov);
   cudaError_t (*occupancy_ic)(int* ctas_per_sm, bool cov);
+  // in-tile accumulator spill slots of kSpillBytes per CTA (0 = 1; the wide pair tile: 2)
+  uint32_t spill_per_cta;
 };
 
 const BodyOps* body_ops(int32_t body);
@@ -55,6 +57,15 @@ cudaError_t gemm2_slice_launch(const void* user, dim3 grid, uint32_t offset, uin
                                cudaStream_t s);
 cudaError_t gemm2_max_pairs(int* pairs, bool cov);
 const char* gemm2_validate(const void* user, dim3 grid);
+// the wide pair tile (256x512, FLEP_BODY_GEMM_BF16_2SM_W): same signatures
+cudaError_t gemm2w_worker_launch(const void* user, const WorkerParams& p, uint32_t ctas, cudaStream_t s, bool cov);
+cudaError_t gemm2w_unwrapped_launch(const void* user, dim3 grid, uint32_t offset, uint32_t count, cudaStream_t s);
+cudaError_t gemm2w_static_launch(const void* user, dim3 grid, uint32_t ctas, uint32_t chunk, cudaStream_t s);
+cudaError_t gemm2w_occupancy(int* k, bool cov);
+cudaError_t gemm2w_slice_launch(const void* user, dim3 grid, uint32_t offset, uint32_t count, const SliceParams& sp,
+                                cudaStream_t s);
+cudaError_t gemm2w_max_pairs(int* pairs, bool cov);
+const char* gemm2w_validate(const void* user, dim3 grid);
 cudaError_t gemm_slice_launch(const void* user, dim3 grid, uint32_t offset, uint32_t count,
                               const SliceParams& sp, cudaStream_t s);
 #ifdef FLEP_TRACE

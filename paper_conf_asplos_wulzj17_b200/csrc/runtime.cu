@@ -352,7 +352,8 @@ flep_status materialize(flep_rt rt, Launch& L) {
     // per-worker partial-tile records (and, in-tile, fp32 accumulator spill slots); no reset
     // needed (the first epoch's workers clear their records)
     // (a CTA pair spills two 128-row halves: one record per pair, one slot per CTA)
-    const uint32_t slots = L.ops->max_pairs ? 2 * L.workers : L.workers;
+    // (the wide pair tile: two slots per CTA, spill_per_cta)
+    const uint32_t slots = (L.ops->max_pairs ? 2 * L.workers : L.workers) * std::max<uint32_t>(1u, L.ops->spill_per_cta);
     const size_t need = (L.flags & FLEP_KFLAG_IN_TILE) ? partial_bytes(slots) : partial_header_bytes(L.workers);
     size_t best = rt->free_partial.size();
     for (size_t i = 0; i < rt->free_partial.size(); ++i)
@@ -938,7 +939,8 @@ flep_status flep_device_info(flep_rt rt, uint32_t* num_sms, uint32_t* nsmid) {
 flep_status flep_register_kernel(flep_rt rt, const flep_kernel_desc* d, flep_kernel* out) {
   if (!rt || !d || !out) return fail(FLEP_ERR_INVALID, "NULL argument");
   if (!body_ops(d->body)) return fail(FLEP_ERR_INVALID, "unknown body %d", d->body);
-  if ((d->flags & FLEP_KFLAG_IN_TILE) && d->body != FLEP_BODY_GEMM_BF16 && d->body != FLEP_BODY_GEMM_BF16_2SM)
+  if ((d->flags & FLEP_KFLAG_IN_TILE) && d->body != FLEP_BODY_GEMM_BF16 && d->body != FLEP_BODY_GEMM_BF16_2SM &&
+      d->body != FLEP_BODY_GEMM_BF16_2SM_W)
     return fail(FLEP_ERR_UNSUPPORTED, "in-tile preemption is implemented for the GEMM bodies only");
   if ((d->flags & FLEP_KFLAG_IN_TILE) && (d->flags & FLEP_KFLAG_PREFETCH))
     return fail(FLEP_ERR_UNSUPPORTED, "in-tile preemption does not combine with chunk prefetch");
@@ -952,7 +954,7 @@ flep_status flep_register_kernel(flep_rt rt, const flep_kernel_desc* d, flep_ker
                                         "warp tasks or in-tile preemption");
   }
   if (d->flags & FLEP_KFLAG_SPEC_FETCH) {
-    if (d->body == FLEP_BODY_GEMM_BF16 || d->body == FLEP_BODY_GEMM_BF16_2SM)
+    if (d->body == FLEP_BODY_GEMM_BF16 || d->body == FLEP_BODY_GEMM_BF16_2SM || d->body == FLEP_BODY_GEMM_BF16_2SM_W)
       return fail(FLEP_ERR_UNSUPPORTED, "the speculative fetch is for the counter worker of the memory-bound bodies");
     // (with prefetch the next fetch would be in flight at every poll; measured slower anyway:
     // issuing it after the chunk barrier delayed the scheduling warp's own body)
@@ -970,7 +972,8 @@ flep_status flep_register_kernel(flep_rt rt, const flep_kernel_desc* d, flep_ker
     flep_status s = occupancy(rt, body_ops(d->body), (rt->opt.debug_coverage & 1u) != 0, &kk);
     if (s) return s;
     if (d->ctas_per_sm && (int)d->ctas_per_sm < kk) kk = (int)d->ctas_per_sm;
-    const size_t need = partial_bytes(std::min<uint32_t>((uint32_t)kk * rt->num_sms, rt->max_workers));
+    const uint32_t per_cta = std::max<uint32_t>(1u, body_ops(d->body)->spill_per_cta);
+    const size_t need = partial_bytes(per_cta * std::min<uint32_t>((uint32_t)kk * rt->num_sms, rt->max_workers));
     size_t have = 0;
     for (auto& f : rt->free_partial) if (f.second >= need) ++have;
     for (; have < 3; ++have) {

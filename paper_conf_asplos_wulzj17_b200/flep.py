@@ -20,6 +20,7 @@ BODY_SAXPY_I32, BODY_SAXPY_F32, BODY_SPMV_CSR_F32, BODY_STENCIL5_F32, BODY_STENC
 BODY_STENCIL5_F32_TMA = 7
 BODY_SPMV_CSR_F32_VEC = 8
 BODY_GEMM_BF16_2SM = 9
+BODY_GEMM_BF16_2SM_W = 10
 STATE_QUEUED, STATE_RUNNING, STATE_YIELDING, STATE_PREEMPTED, STATE_PARTIAL, STATE_DONE = 0, 1, 2, 3, 4, 5
 STATE_NAMES = {0: "QUEUED", 1: "RUNNING", 2: "YIELDING", 3: "PREEMPTED", 4: "PARTIAL", 5: "DONE"}
 REASON_YIELD, REASON_EXHAUSTED = 1, 2
@@ -100,7 +101,8 @@ class EpochInfo(C.Structure):
 
 ARGS_FOR_BODY = {BODY_SAXPY_I32: SaxpyI32Args, BODY_SAXPY_F32: SaxpyF32Args, BODY_SPMV_CSR_F32: SpmvArgs,
                  BODY_STENCIL5_F32: StencilArgs, BODY_STENCIL5_I32: StencilArgs, BODY_GEMM_BF16: GemmArgs,
-                 BODY_STENCIL5_F32_TMA: StencilArgs, BODY_SPMV_CSR_F32_VEC: SpmvArgs, BODY_GEMM_BF16_2SM: GemmArgs}
+                 BODY_STENCIL5_F32_TMA: StencilArgs, BODY_SPMV_CSR_F32_VEC: SpmvArgs, BODY_GEMM_BF16_2SM: GemmArgs,
+                 BODY_GEMM_BF16_2SM_W: GemmArgs}
 
 # exported symbols: name -> (restype, argtypes)
 _P = C.c_void_p
@@ -439,3 +441,8 @@ def gemm_grid(m, n):
 def gemm2_grid(m, n):
     """Original grid of the CTA-pair GEMM body: one 256x256 tile per block."""
     return (n // 256, m // 256, 1)
+
+
+def gemm2w_grid(m, n):
+    """Original grid of the wide CTA-pair GEMM body: one 256x512 tile per block."""
+    return (n // 512, m // 256, 1)
