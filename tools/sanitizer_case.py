@@ -130,6 +130,22 @@ def main():
     if rt.query(h).state == F.STATE_PREEMPTED:
         rt.resume(h)
     rt.sync(h)
+    # the wide pair tile (256x512): unwrapped, static, worker preempted tile-granular and in-tile
+    a_bits, b_bits = gen.gemm_bf16_inputs(512, 1024, 1024, 10)
+    A4 = torch.from_numpy(a_bits.view(np.int16)).cuda().view(torch.bfloat16)
+    B4 = torch.from_numpy(b_bits.view(np.int16)).cuda().view(torch.bfloat16)
+    C4 = torch.empty(512, 1024, dtype=torch.bfloat16, device="cuda")
+    g2w = F.gemm2w_grid(512, 1024)
+    rt.launch_unwrapped(F.BODY_GEMM_BF16_2SM_W, g2w, F.gemm_args(C4, A4, B4))
+    rt.launch_static(F.BODY_GEMM_BF16_2SM_W, g2w, F.gemm_args(C4, A4, B4))
+    for in_tile in (False, True):
+        k14 = rt.register_kernel(F.BODY_GEMM_BF16_2SM_W, chunk=1, poll=1, in_tile=in_tile)
+        rt.arm_next_trigger(1, rt.num_sms)
+        h = rt.launch(k14, g2w, F.gemm_args(C4, A4, B4))
+        rt.wait_epoch(h)
+        if rt.query(h).state == F.STATE_PREEMPTED:
+            rt.resume(h)
+        rt.sync(h)
     torch.cuda.synchronize()
     rt.close()
     rs = F.Runtime(policy=F.POLICY_SLICE_DEVICE, slice_blocks=8)
