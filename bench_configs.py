@@ -788,6 +788,21 @@ def _agree_t_alone(t_alone, world, torch):
 
 
 QUEUE_CHUNK = {"saxpy_f32": (8, False), "spmv": (2, True), "stencil_f32": (2, True), "gemm_bf16": (1, False)}
+# FLEP_QUEUE_FETCH=spec (the default): SpMV and stencil fetch their C-block chunks speculatively
+# (R34) instead of prefetching them: a prefetching worker runs the chunk it holds before it yields
+# (A4), which doubles its drain; a speculative fetch hands that chunk back through the worker's
+# record. Measured on configs[4] (profiles/r02_queue_fetch_spec.jsonl): preemption latency p99
+# 45-46 -> 27.7 us (SpMV 2^23 victims p50 38 -> 22-24 us), same throughput and overheads.
+# FLEP_QUEUE_FETCH=prefetch restores the round-1/2 setting (QUEUE_CHUNK).
+QUEUE_CHUNK_SPEC = {"saxpy_f32": (8, False), "spmv": (2, False), "stencil_f32": (2, False), "gemm_bf16": (1, False)}
+
+
+def _qopts(F, ty, body):
+    """register_kernel options of a queue kernel of type `ty` (configs[3], configs[4], E13)."""
+    spec = os.environ.get("FLEP_QUEUE_FETCH", "spec") == "spec"
+    C, pf = (QUEUE_CHUNK_SPEC if spec else QUEUE_CHUNK)[ty]
+    gemm = body in (F.BODY_GEMM_BF16, F.BODY_GEMM_BF16_2SM, F.BODY_GEMM_BF16_2SM_W)
+    return dict(chunk=C, poll=1, prefetch=pf, spec_fetch=spec and not gemm and ty != "saxpy_f32", in_tile=gemm)
 
 
 def _queue_instances(torch, F, seed):
@@ -840,12 +855,11 @@ def _run_trace(F, torch, local, policy, trace, inst, t_alone, overhead_ns, strea
     rt = F.Runtime(device=local, policy=policy, slice_blocks=slice_blocks)
     kid = {}
     for key, (body, grid, a, keep, _) in inst.items():
-        C, pf = QUEUE_CHUNK[key[0]]
-        kid[key] = rt.register_kernel(body, chunk=C, poll=1, prefetch=pf, name=f"{key[0]}-{key[1]}",
-                                      model=(0, 0, 0, 0, float(t_alone[key])), overhead_ns=int(overhead_ns),
-                                      in_tile=body in (F.BODY_GEMM_BF16, F.BODY_GEMM_BF16_2SM, F.BODY_GEMM_BF16_2SM_W))
+        kid[key] = rt.register_kernel(body, name=f"{key[0]}-{key[1]}", model=(0, 0, 0, 0, float(t_alone[key])),
+                                      overhead_ns=int(overhead_ns), **_qopts(F, key[0], body))
     hs = []
     call_ns = []
+    _run_trace.lat_keys = []           # victim kernel of each latency sample (want_lat)
     t0 = F.now_ns() + 2_000_000
     for i, job in enumerate(trace):
         key = (job["type"], job["size_class"])
@@ -867,6 +881,7 @@ def _run_trace(F, torch, local, policy, trace, inst, t_alone, overhead_ns, strea
         # host-observed preemption latency of the last drained epoch (request -> drained status)
         if info.epoch >= 2 and info.t_last_drain > 0 and info.t_last_request > 0:
             lat.append((info.t_last_drain - info.t_last_request) / 1e3)
+            _run_trace.lat_keys.append(f"{key[0]}-{key[1]}")
     dec = rt.decision_log()
     evl = rt.event_log()
     rt.close()
@@ -895,8 +910,7 @@ def run_queue(args, rank, world, local):
     flush = L2Flush(torch)
     rt = F.Runtime(device=local, policy=F.POLICY_FIFO)
     for key, (body, grid, a, keep, _) in inst.items():
-        C, pf = QUEUE_CHUNK[key[0]]
-        k = rt.register_kernel(body, chunk=C, poll=1, prefetch=pf, in_tile=body in (F.BODY_GEMM_BF16, F.BODY_GEMM_BF16_2SM, F.BODY_GEMM_BF16_2SM_W))
+        k = rt.register_kernel(body, **_qopts(F, key[0], body))
         ts = []
         for r in range(4):
             flush.zero_()                      # cold L2: the queue interleaves working sets
@@ -1207,8 +1221,7 @@ def run_scale_queue(args, rank, world, local):
     rt = F.Runtime(device=local, policy=F.POLICY_FIFO)
     rt_m = F.Runtime(device=local, exec_on_user_stream=True)
     for key, (body, grid, a, keep, _) in sorted(inst.items()):
-        C, pf = QUEUE_CHUNK[key[0]]
-        k = rt.register_kernel(body, chunk=C, poll=1, prefetch=pf, in_tile=body in (F.BODY_GEMM_BF16, F.BODY_GEMM_BF16_2SM, F.BODY_GEMM_BF16_2SM_W))
+        k = rt.register_kernel(body, **_qopts(F, key[0], body))
         ts = []
         for r in range(3):
             flush.zero_()
@@ -1219,7 +1232,7 @@ def run_scale_queue(args, rank, world, local):
             if r:
                 ts.append(info.t_finish - info.t_arrive)
         t_alone[key] = int(np.median(ts))
-        km = rt_m.register_kernel(body, chunk=C, poll=1, prefetch=pf, in_tile=body in (F.BODY_GEMM_BF16, F.BODY_GEMM_BF16_2SM, F.BODY_GEMM_BF16_2SM_W))
+        km = rt_m.register_kernel(body, **_qopts(F, key[0], body))
         tw, tu = [], []
         for r in range(4):
             for mode in ("w", "u"):
@@ -1255,7 +1268,8 @@ def run_scale_queue(args, rank, world, local):
                                              want_lat=True)
             res[name] = {"turn": [int(t[0]) for t in turn], "alone": [int(t_alone[t[1]]) for t in turn],
                          "makespan_ns": int(max(t[4] for t in turn)) if turn else 0,
-                         "preemptions": sum(1 for d in dec if d[1] == 2), "lat_us": lat}
+                         "preemptions": sum(1 for d in dec if d[1] == 2), "lat_us": lat,
+                         "lat_keys": list(_run_trace.lat_keys)}
     rec = {"rank": rank, "kernels": len(mine), "res": res, "clocks": clk.summary(), "overhead_pct": over}
     allr = gather_objects(rec, world)
     out = None
@@ -1278,6 +1292,12 @@ def run_scale_queue(args, rank, world, local):
                             "antt_fifo": round(M.antt(r["res"]["FIFO"]["turn"], r["res"]["FIFO"]["alone"]), 3) if r["kernels"] else None,
                             "clocks": r["clocks"]})
         all_lat = [x for r in allr for x in r["res"]["HPF"]["lat_us"]]
+        by_kernel = {}                 # the latency distribution per victim kernel (type-size class)
+        for r in allr:
+            for x, k in zip(r["res"]["HPF"]["lat_us"], r["res"]["HPF"].get("lat_keys", [])):
+                by_kernel.setdefault(k, []).append(x)
+        by_kernel = {k: {"p50": round(float(np.median(v)), 2), "max": round(float(np.max(v)), 2), "n": len(v)}
+                     for k, v in sorted(by_kernel.items())}
         gain = agg["FIFO"]["antt"] / agg["HPF"]["antt"]
         out = {"metric": METRIC, "value": round(gain, 3), "unit": "x (ANTT_FIFO / ANTT_FLEP)",
                "value_definition": "NATT gain of FLEP-HPF over FIFO over all kernels of the shared job queue",
@@ -1291,6 +1311,7 @@ def run_scale_queue(args, rank, world, local):
                "preempt_latency_us_all": ({"p50": round(float(np.median(all_lat)), 2),
                                            "p99": round(float(np.percentile(all_lat, 99)), 2),
                                            "max": round(float(np.max(all_lat)), 2), "n": len(all_lat)} if all_lat else None),
+               "preempt_latency_us_by_victim": by_kernel,
                "wrapper_overhead_pct_rank0": allr[0]["overhead_pct"],
                "wrapper_overhead_pct_max_over_gpus": {k: max(r["overhead_pct"][k] for r in allr)
                                                       for k in allr[0]["overhead_pct"]}}
@@ -1499,8 +1520,8 @@ def run_slicing_overhead(args, rank, world, local):
     with ClockSampler(physical_gpu_index(local)) as clk:
         for key in sorted(inst):
             body, grid, a, keep, _ = inst[key]
-            C, pf = QUEUE_CHUNK[key[0]]
-            k_t = rt_m.register_kernel(body, chunk=C, poll=1, prefetch=pf, in_tile=body in (F.BODY_GEMM_BF16, F.BODY_GEMM_BF16_2SM, F.BODY_GEMM_BF16_2SM_W))
+            C = _qopts(F, key[0], body)["chunk"]
+            k_t = rt_m.register_kernel(body, **_qopts(F, key[0], body))
             k_1 = rt_m.register_kernel(body, chunk=1, poll=1, in_tile=body in (F.BODY_GEMM_BF16, F.BODY_GEMM_BF16_2SM, F.BODY_GEMM_BF16_2SM_W))
             k_s = rt_s.register_kernel(body, chunk=C, poll=1)
             cps, w = rt_m.workers_for(body)
