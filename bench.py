@@ -772,7 +772,8 @@ def main():
     ap.add_argument("--impl", default="flep", choices=["flep", "reference"])
     ap.add_argument("--config", default="temporal", choices=["temporal", "corun1", "spatial", "spatial_managed", "queue",
                                                              "scale", "ffs", "model", "gemm", "tune", "clc", "delay",
-                                                             "spatial_f1", "slicing"])
+                                                             "spatial_f1", "slicing", "coruns"])
+    ap.add_argument("--corun-reps", type=int, default=3, help="config coruns: runs per case and policy")
     ap.add_argument("--dry-run", action="store_true",
                     help="configs[4] launcher and control flow without CUDA (CPU, gloo); one JSON line")
     ap.add_argument("--sub", type=int, default=1, help="default run: add the configs[0,2,3,4] sub-records")
@@ -832,7 +833,8 @@ def main():
               "tune": bench_configs.run_tune, "ffs": bench_configs.run_ffs, "model": bench_configs.run_model,
               "clc": bench_configs.run_clc, "delay": bench_configs.run_delay,
               "spatial_f1": bench_configs.run_spatial_f1, "queue": bench_configs.run_queue,
-              "scale": bench_configs.run_scale_queue, "slicing": bench_configs.run_slicing_overhead}[args.config]
+              "scale": bench_configs.run_scale_queue, "slicing": bench_configs.run_slicing_overhead,
+              "coruns": bench_configs.run_coruns}[args.config]
         fn(args, rank, world, local)
 
 

@@ -854,7 +854,10 @@ def _run_trace(F, torch, local, policy, trace, inst, t_alone, overhead_ns, strea
                want_lat=False):
     rt = F.Runtime(device=local, policy=policy, slice_blocks=slice_blocks)
     kid = {}
+    used = {(j["type"], j["size_class"]) for j in trace}
     for key, (body, grid, a, keep, _) in inst.items():
+        if key not in used:
+            continue
         kid[key] = rt.register_kernel(body, name=f"{key[0]}-{key[1]}", model=(0, 0, 0, 0, float(t_alone[key])),
                                       overhead_ns=int(overhead_ns), **_qopts(F, key[0], body))
     hs = []
@@ -891,6 +894,30 @@ def _run_trace(F, torch, local, policy, trace, inst, t_alone, overhead_ns, strea
     return turn, dec, evl
 
 
+def _measure_t_alone(F, torch, local, inst):
+    """Standalone turnaround (ns) of every queue instance through the same runtime path (FIFO, idle
+    GPU, L2 flushed: the queue interleaves working sets); median of 3 after one warm-up."""
+    from bench import L2Flush
+    flush = L2Flush(torch)
+    t_alone = {}
+    rt = F.Runtime(device=local, policy=F.POLICY_FIFO)
+    for key, (body, grid, a, keep, _) in inst.items():
+        k = rt.register_kernel(body, **_qopts(F, key[0], body))
+        ts = []
+        for r in range(4):
+            flush.zero_()
+            torch.cuda.synchronize()
+            h = rt.launch(k, grid, a)
+            rt.sync(h)
+            info = rt.query(h)
+            if r:
+                ts.append(info.t_finish - info.t_arrive)
+        t_alone[key] = int(np.median(ts))
+    rt.close()
+    del flush
+    return t_alone
+
+
 def run_queue(args, rank, world, local):
     """configs[3] (and configs[4] at N > 1): same-priority mixed queue of 64 kernels (SAXPY-f32,
     SpMV, stencil5, bf16 GEMM up to 8192^3) with Poisson arrivals at offered load rho; ANTT and
@@ -904,25 +931,7 @@ def run_queue(args, rank, world, local):
     torch.cuda.set_device(local)
     inst = _queue_instances(torch, F, seed=5)
     streams = [torch.cuda.Stream() for _ in range(4)]
-    # standalone turnaround of every instance through the same runtime path (FIFO, idle GPU)
-    t_alone = {}
-    from bench import L2Flush
-    flush = L2Flush(torch)
-    rt = F.Runtime(device=local, policy=F.POLICY_FIFO)
-    for key, (body, grid, a, keep, _) in inst.items():
-        k = rt.register_kernel(body, **_qopts(F, key[0], body))
-        ts = []
-        for r in range(4):
-            flush.zero_()                      # cold L2: the queue interleaves working sets
-            torch.cuda.synchronize()
-            h = rt.launch(k, grid, a)
-            rt.sync(h)
-            info = rt.query(h)
-            if r:
-                ts.append(info.t_finish - info.t_arrive)
-        t_alone[key] = int(np.median(ts))
-    rt.close()
-    t_alone = _agree_t_alone(t_alone, world, torch)
+    t_alone = _agree_t_alone(_measure_t_alone(F, torch, local, inst), world, torch)
     n_total = args.queue_kernels * world
     mean_alone = float(np.mean([t_alone[(j["type"], j["size_class"])]
                                 for j in gen.queue_trace(5, n_total, 1)]))
@@ -992,6 +1001,118 @@ def run_queue(args, rank, world, local):
 
 
 # ------------------------------------------------------------------------------------------
+CORUN_TYPES = ("saxpy_f32", "spmv", "stencil_f32", "gemm_bf16")
+CORUN_SHORT = {"saxpy_f32": "VA", "spmv": "SPMV", "stencil_f32": "ST", "gemm_bf16": "MM"}
+
+
+def corun_cases(seed=7, n_triplets=28, gap_ns=20_000):
+    """The paper's co-run experiments as job traces over the queue instances (large = class 2,
+    small = class 1): E4 (Fig. 8) every large low-priority kernel with every small
+    high-priority kernel launched right after it; E6/E7 (Figs. 10-11) the same pairs at
+    equal priority; E8 (Fig. 12) 28 seeded triplets A_B_C, A large then B and C small
+    (B != C). Returns [(experiment, name, trace)]."""
+    cases = []
+    for lp in CORUN_TYPES:
+        for hp in CORUN_TYPES:
+            for exp, prio in (("E4", 1), ("E6", 0)):
+                cases.append((exp, f"{CORUN_SHORT[lp]}_{CORUN_SHORT[hp]}", [
+                    {"id": 0, "type": lp, "size_class": 2, "priority": 0, "arrival_ns": 0},
+                    {"id": 1, "type": hp, "size_class": 1, "priority": prio, "arrival_ns": gap_ns}]))
+    # the paper's named triplet VA_SPMV_MM (P:349) and n_triplets - 1 seeded others
+    named = ("saxpy_f32", "spmv", "gemm_bf16")
+    trip = [(a, b, c) for a in CORUN_TYPES for b in CORUN_TYPES for c in CORUN_TYPES if b != c and (a, b, c) != named]
+    g = gen.rng(seed)
+    pick = [trip[i] for i in g.choice(len(trip), size=n_triplets - 1, replace=False).tolist()] + [named]
+    for a, b, c in sorted(pick, key=lambda t: tuple(CORUN_TYPES.index(x) for x in t)):
+        cases.append(("E8", f"{CORUN_SHORT[a]}_{CORUN_SHORT[b]}_{CORUN_SHORT[c]}", [
+            {"id": 0, "type": a, "size_class": 2, "priority": 0, "arrival_ns": 0},
+            {"id": 1, "type": b, "size_class": 1, "priority": 0, "arrival_ns": gap_ns},
+            {"id": 2, "type": c, "size_class": 1, "priority": 0, "arrival_ns": 2 * gap_ns}]))
+    return cases
+
+
+def run_coruns(args, rank, world, local):
+    """The paper's co-run matrices on one B200 through the managed runtime: E4 high-priority
+    speedup (Fig. 8: HP turnaround under the FIFO / MPS-like default co-run over FLEP-HPF), E6
+    ANTT gain and E7 STP degradation of equal-priority pairs (Figs. 10-11), E8 ANTT gain of 28
+    triplets and of non-preemptive reordering (Fig. 12). Median of `reps` runs per case and
+    policy; the runtime's event and decision logs of the first run of every case are written to
+    FLEP_EVIDENCE_DIR (corun_logs.json) for the oracle replay test."""
+    import os
+    import torch
+    import bench_check as M
+    from bench import ClockSampler, barrier, physical_gpu_index
+    from paper_conf_asplos_wulzj17_b200 import flep as F
+    torch.cuda.set_device(local)
+    inst = _queue_instances(torch, F, seed=5)
+    inst = {k: v for k, v in inst.items() if k[1] >= 1}          # small and large classes only
+    streams = [torch.cuda.Stream() for _ in range(4)]
+    t_alone = _measure_t_alone(F, torch, local, inst)
+    overhead_ns = 20_000
+    reps = max(1, int(getattr(args, "corun_reps", 3)))
+    cases = corun_cases()
+    pols = {"E4": (("FIFO", F.POLICY_FIFO), ("HPF", F.POLICY_HPF)),
+            "E6": (("FIFO", F.POLICY_FIFO), ("HPF", F.POLICY_HPF)),
+            "E8": (("FIFO", F.POLICY_FIFO), ("HPF", F.POLICY_HPF), ("REORDER", F.POLICY_REORDER))}
+    _run_trace(F, torch, local, F.POLICY_HPF, cases[0][2], inst, t_alone, overhead_ns, streams)   # warm-up
+    rows, logs = [], {}
+    with ClockSampler(physical_gpu_index(local)) as clk:
+        for exp, name, trace in cases:
+            row = {"exp": exp, "case": name}
+            for pname, pol in pols[exp]:
+                turns = []
+                for r in range(reps):
+                    turn, dec, evl = _run_trace(F, torch, local, pol, trace, inst, t_alone, overhead_ns, streams)
+                    turns.append([t[0] for t in turn])
+                    if r == 0:
+                        logs[f"{exp}/{name}/{pname}"] = {"events": [list(map(int, e)) for e in evl],
+                                                         "decisions": [list(map(int, d_)) for d_ in dec]}
+                tt = [int(np.median([t[i] for t in turns])) for i in range(len(trace))]
+                al = [t_alone[(j["type"], j["size_class"])] for j in trace]
+                row[pname] = {"turn_us": [round(x / 1e3, 1) for x in tt], "antt": round(M.antt(tt, al), 3),
+                              "stp": round(M.stp(tt, al), 3)}
+            al = [t_alone[(j["type"], j["size_class"])] for j in trace]
+            if exp == "E4":
+                row["hp_speedup"] = round(row["FIFO"]["turn_us"][1] / row["HPF"]["turn_us"][1], 2)
+                # a non-preemptive co-run makes the HP wait for the rest of the LP (P:321's bound)
+                row["hp_speedup_bound"] = round((al[0] - trace[1]["arrival_ns"] + al[1]) / al[1], 2)
+            else:
+                row["antt_gain"] = round(row["FIFO"]["antt"] / row["HPF"]["antt"], 2)
+                row["stp_degradation"] = round(1 - row["HPF"]["stp"] / row["FIFO"]["stp"], 4)
+                if exp == "E8":
+                    row["reorder_gain"] = round(row["FIFO"]["antt"] / row["REORDER"]["antt"], 3)
+            rows.append(row)
+    ev_dir = os.environ.get("FLEP_EVIDENCE_DIR")
+    if ev_dir and rank == 0:
+        with open(os.path.join(ev_dir, "corun_logs.json"), "w") as fh:
+            json.dump({"workload": "co-run matrices E4/E6/E8 over the queue instances (seed 5)", "logs": logs}, fh)
+
+    def summ(exp, key):
+        v = [r[key] for r in rows if r["exp"] == exp]
+        return {"mean": round(float(np.mean(v)), 3), "min": round(float(np.min(v)), 3),
+                "max": round(float(np.max(v)), 3), "n": len(v),
+                "argmax": max((r for r in rows if r["exp"] == exp), key=lambda r: r[key])["case"]}
+    out = {"metric": METRIC, "value": summ("E6", "antt_gain")["mean"], "unit": "x (ANTT_FIFO / ANTT_FLEP)",
+           "value_definition": "mean ANTT gain of FLEP-HPF over the FIFO (MPS-like) co-run over the 16 "
+                               "equal-priority pairs (E6, Fig. 10)",
+           "n_gpus": world, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+           "dtype": "mixed (f32, bf16->f32)", "data": "synthetic (seeded)",
+           "config": {"workload": "co-runs of the configs[3] instances: large = class 2 (SAXPY 2^28, SpMV 2^23 rows, "
+                                  "stencil 16384^2, GEMM 8192^3), small = class 1 (2^24, 2^20 rows, 4096^2, 4096^3); "
+                                  "the second (and third) kernel arrives 20 (40) us after the first",
+                      "reps": reps, "overhead_estimate_ns": overhead_ns},
+           "E4_hp_speedup": summ("E4", "hp_speedup"), "E6_antt_gain": summ("E6", "antt_gain"),
+           "E7_stp_degradation": summ("E6", "stp_degradation"), "E8_antt_gain": summ("E8", "antt_gain"),
+           "E8_reorder_gain": summ("E8", "reorder_gain"),
+           "paper": "K40: E4 10.1x mean / 24.2x max / 4.1x min; E6 8x mean, 27x max; E7 5.4 %; E8 6.6x mean, "
+                    "20.2x max (VA_SPMV_MM); reordering 2.3 % (P:321, P:329, P:343, P:349-351)",
+           "t_alone_us": {f"{k[0]}-{k[1]}": round(v / 1e3, 1) for k, v in sorted(t_alone.items())},
+           "cases": rows, "clocks": clk.summary()}
+    _emit(out, rank, args)
+    barrier(world)
+    return out
+
+
 def run_ffs(args, rank, world, local):
     """FFS experiment (Figs. 13-14): two applications keep invoking the
     same long kernel (SAXPY-int32 over 2^30 elements, ~2 ms) in a loop, priorities 1 and 0 (weights

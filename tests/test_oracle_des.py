@@ -271,3 +271,21 @@ def test_des_predicts_the_b200_queue_run():
         assert 0.7 <= v["ratio"] <= 1.3, (k, v)
     p = {k: v["predicted_antt"] for k, v in out["policies"].items()}
     assert p["HPF"] < p["REORDER"] < p["FIFO"]
+
+
+def test_des_predicts_the_b200_corun_matrices():
+    """Simulate mode vs the measured B200 co-run matrices (E4 / E6 / E8, Figs. 8, 10, 12;
+    tests/des_predict_coruns.py on tests/golden/coruns_measured_r02.json): every case's HP speedup
+    or ANTT gain predicted within 30 % and each experiment's mean within 20 % (a model check: the
+    simulation has no co-run interference and one drain for every victim)."""
+    import os
+    import sys
+    sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
+    import des_predict_coruns
+    out = des_predict_coruns.main()
+    assert len(out["cases"]) == 60
+    for r in out["cases"]:
+        assert 0.7 <= r["ratio"] <= 1.3, r
+        assert r["pred"] > 1.0                   # preemption helps every case in the model too
+    for exp, s in out["summary"].items():
+        assert 0.8 <= s["pred_mean"] / s["meas_mean"] <= 1.2, (exp, s)

@@ -178,3 +178,26 @@ def test_b200_managed_spatial_log_replays_exactly():
     widths = sorted({x[3] for x in d["decisions"] if x[1] == ACT["PREEMPT"]})
     assert widths == [8, 16, 32, 74, 148]
     assert sum(1 for x in d["decisions"] if x[1] == ACT["REFILL"]) >= 40
+
+
+def test_b200_corun_matrix_logs_replay_exactly():
+    """The co-run matrices on the B200 (bench.py --config coruns: E4 high-priority pairs, E6
+    equal-priority pairs, E8 triplets, Figs. 8 / 10 / 12; tests/golden/corun_logs_r02.json): every
+    case's event log under FIFO, FLEP-HPF and REORDER replayed through the oracle DES gives the
+    runtime's decision list bit for bit; every HPF case preempts its large first kernel."""
+    import json
+    import os
+    path = os.path.join(os.path.dirname(__file__), "golden", "corun_logs_r02.json")
+    with open(path) as fh:
+        logs = json.load(fh)["logs"]
+    kinds = {"FIFO": des.FIFO, "HPF": des.HPF, "REORDER": des.REORDER}
+    seen = {"E4": 0, "E6": 0, "E8": 0}
+    for key, lg in logs.items():
+        exp, case, pol = key.split("/")
+        evs = [(t, "ARRIVE", des.KernelSpec(i, t, p, te, o)) if ty == 0 else (t, "FINISH", i)
+               for (t, ty, i, p, te, o) in lg["events"]]
+        assert as_tuples(des.replay(kinds[pol], evs)) == [tuple(d) for d in lg["decisions"]], key
+        if pol == "HPF":
+            seen[exp] += 1
+            assert any(d[1] == ACT["PREEMPT"] for d in lg["decisions"]), key
+    assert seen == {"E4": 16, "E6": 16, "E8": 28}
