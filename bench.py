@@ -739,8 +739,9 @@ def sub_records(args, rank, world, local):
     configs[0] (SAXPY-int co-run, exactness), configs[2] (spatial yield per width: the manual
     device-triggered sweep and the managed spatial-HPF decision path, victim checked against a
     NumPy reference), configs[3] (64-kernel same-priority queue: ANTT/STP, decision logs),
-    configs[4] (one 512-kernel job queue over the N GPUs of this run) and E13 (never-preempted
-    overhead of FLEP vs kernel slicing)."""
+    configs[4] (one 512-kernel job queue over the N GPUs of this run), E13 (never-preempted
+    overhead of FLEP vs kernel slicing) and the co-run matrices (E4 / E6 / E8: Figs. 8,
+    10, 12)."""
     import copy
     import bench_configs as BCF
     a = copy.copy(args)
@@ -749,7 +750,8 @@ def sub_records(args, rank, world, local):
     out, timing = {}, {}
     for name, fn in (("configs[0]", BCF.run_corun1), ("configs[2]", BCF.run_spatial),
                      ("configs[2]_managed", BCF.run_spatial_managed), ("configs[3]", BCF.run_queue),
-                     ("configs[4]", BCF.run_scale_queue), ("E13_never_preempted", BCF.run_slicing_overhead)):
+                     ("configs[4]", BCF.run_scale_queue), ("E13_never_preempted", BCF.run_slicing_overhead),
+                     ("coruns_E4_E6_E8", BCF.run_coruns)):
         if name in args.skip_sub:
             continue
         t0 = time.perf_counter()

@@ -22,7 +22,7 @@ def test_bench_two_ranks_one_line():
     env["FLEP_SHARE_GPU"] = "1"
     r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "2", "--steps", "3", "--warmup", "3",
                         "--reps", "4", "--e2e-steps", "2", "--sub-steps", "3",
-                        "--skip-sub", "configs[2],configs[2]_managed,configs[3],E13_never_preempted"],
+                        "--skip-sub", "configs[2],configs[2]_managed,configs[3],E13_never_preempted,coruns_E4_E6_E8"],
                        capture_output=True, text=True, env=env, timeout=900, cwd=ROOT)
     assert r.returncode == 0, r.stderr[-3000:]
     lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
