@@ -720,6 +720,7 @@ def run_reference(args, rank, world):
         if i >= args.warmup:
             lats.append((t1 - t0) * 1e6)
     v = float(np.median(lats))
+    extra = oracle_timings()
     out = {"impl": "reference", "metric": METRIC, "value": round(v, 1), "unit": "us", "n_gpus": world,
            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(float(np.mean(lats)) / 1e3, 3),
            "higher_is_better": False, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
@@ -730,8 +731,42 @@ def run_reference(args, rank, world):
                             "sample": "per step: oracle SpMV over the LP rows after a seeded t* (what a "
                                       "non-preemptive program must finish before the HP starts); ms_per_step is the "
                                       "mean of these timed steps"},
-           "e2e": {"value": round(v, 1), "unit": "us", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+           "e2e": {"value": round(v, 1), "unit": "us", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+           "oracle_timings": extra}
     print(json.dumps(out), flush=True)
+
+
+def oracle_timings():
+    """SURVEY §8(d) oracle-timing protocol beside the reference arm: the host (model, cores, BLAS
+    threads), the fp64 GEMM oracle on a bounded sample (2048^3, all cores; 8192^3 extrapolated by
+    the flop ratio) and the DES per trace (configs[3]: 64 kernels, configs[4]: 512)."""
+    import platform
+    from oracle import des, workloads as W
+    info = {"cpu_count": os.cpu_count(), "machine": platform.machine()}
+    try:
+        with open("/proc/cpuinfo") as fh:
+            info["cpu_model"] = next((l.split(":", 1)[1].strip() for l in fh if l.startswith("model name")), None)
+    except OSError:
+        info["cpu_model"] = None
+    try:
+        from threadpoolctl import threadpool_info
+        info["blas"] = [{"api": d.get("internal_api"), "threads": d.get("num_threads")} for d in threadpool_info()]
+    except Exception:
+        info["blas"] = None
+    a_bits, b_bits = gen.gemm_bf16_inputs(2048, 2048, 2048, seed=60)
+    t0 = time.perf_counter()
+    W.gemm_bf16(a_bits, b_bits)
+    t_g = time.perf_counter() - t0
+    info["gemm_fp64_2048cubed_s"] = round(t_g, 3)
+    info["gemm_fp64_8192cubed_s_extrapolated"] = round(t_g * 64, 2)
+    for name, n in (("configs[3]", 64), ("configs[4]", 512)):
+        tr = gen.queue_trace(5 if n == 64 else 6, n, 200_000)
+        ks = [des.KernelSpec(j["id"], j["arrival_ns"], 0, 100_000 * (1 + j["size_class"] * 10), 20_000,
+                             100_000 * (1 + j["size_class"] * 10)) for j in tr]
+        t0 = time.perf_counter()
+        des.simulate(des.HPF, ks)
+        info[f"des_hpf_{name}_{n}_kernels_ms"] = round((time.perf_counter() - t0) * 1e3, 2)
+    return info
 
 
 def sub_records(args, rank, world, local):
