@@ -28,6 +28,9 @@
 #ifndef FLEP_SPMV_AU
 #define FLEP_SPMV_AU 8               // gathers in flight per thread in the cp.async body
 #endif
+#ifndef FLEP_SPMV_TILE
+#define FLEP_SPMV_TILE 2048          // SpMV CSR-stream: nonzeros per shared-memory product tile
+#endif
 #ifndef FLEP_SPMV_ROWS
 #define FLEP_SPMV_ROWS 128           // rows per original block (flep.py SPMV_ROWS_PER_BLOCK)
 #endif
@@ -111,7 +114,7 @@ struct SpmvBody : NoResources {
   static constexpr int kThreads = 256;
   static constexpr int kMinBlocks = 8;
   static constexpr uint32_t kRowsPerBlock = FLEP_SPMV_ROWS;
-  static constexpr uint32_t kTile = 2048;
+  static constexpr uint32_t kTile = FLEP_SPMV_TILE;     // products staged per tile (smem)
   using Args = flep_spmv_args;
 
   static constexpr uint32_t kGroupRows = 256;     // rows streamed together (2 blocks of a chunk)
