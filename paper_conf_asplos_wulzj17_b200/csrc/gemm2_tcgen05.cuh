@@ -232,53 +232,14 @@ struct Gemm2T {
       asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" :: "r"(s->tmem_base), "r"(kTmemCols) : "memory");
   }
 
-  // Epilogue of one warp's 32 accumulator rows, columns [c_begin, c_end) (multiples of 64):
-  // TMEM -> bf16 -> this warp's staging buffer (row = lane, 16-B chunk c at c ^ (lane & 7), the
-  // SWIZZLE_128B layout) -> one bulk tensor store of 32 x 64 per 64 columns, issued by lane 0;
-  // two buffers per warp, so the store of one chunk overlaps the next chunk's TMEM loads. `it`
-  // counts this warp's stores (buffer = it & 1); the caller ends with bulk_wait_all().
+  // Epilogue of one warp's 32 accumulator rows, columns [c_begin, c_end): GemmBody::store_bulk
+  // (TMEM -> bf16 -> the warp's two SWIZZLE_128B staging buffers -> bulk tensor stores of C)
   __device__ static void store_cols(const Gemm2Args& g, uint32_t tmem_w, uint32_t c_begin, uint32_t c_end,
                                     int32_t x0, int32_t y0, uint32_t q, uint32_t lane, uint32_t& it) {
-#pragma unroll 1
-    for (uint32_t c0 = c_begin; c0 < c_end; c0 += 64) {
-      uint32_t o[32];
-#pragma unroll
-      for (uint32_t hh = 0; hh < 2; ++hh) {
-        uint32_t v[32];
-        GemmBody::tmem_ld32(tmem_w + c0 + 32 * hh, v);
-#pragma unroll
-        for (int i = 0; i < 16; ++i) {
-          __nv_bfloat162 hv = __floats2bfloat162_rn(__uint_as_float(v[2 * i]), __uint_as_float(v[2 * i + 1]));
-          o[16 * hh + i] = *reinterpret_cast<uint32_t*>(&hv);
-        }
-      }
-      const uint32_t bi = it & 1u;
-      if (it >= 2) {                                   // the store that used this buffer has read it
-        if (lane == 0) asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
-        __syncwarp();
-      }
-      uint8_t* buf = epi_buf(q, bi);
-      const uint32_t rowb = su32(buf) + lane * 128u;
-#pragma unroll
-      for (uint32_t c = 0; c < 8; ++c)
-        asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};"
-                     :: "r"(rowb + ((c ^ (lane & 7u)) << 4)), "r"(o[4 * c]), "r"(o[4 * c + 1]), "r"(o[4 * c + 2]),
-                        "r"(o[4 * c + 3]) : "memory");
-      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // visible to the bulk store
-      __syncwarp();
-      if (lane == 0) {
-        asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];"
-                     :: "l"(reinterpret_cast<uint64_t>(&g.tma_c)), "r"(su32(buf)), "r"(x0 + (int32_t)c0), "r"(y0)
-                     : "memory");
-        asm volatile("cp.async.bulk.commit_group;" ::: "memory");
-      }
-      ++it;
-    }
+    static_assert(kEpiBuf == GemmBody::kEpiBuf, "staging buffer size");
+    GemmBody::store_bulk(&g.tma_c, epi_buf(q, 0), tmem_w, c_begin, c_end, x0, y0, lane, it);
   }
-  __device__ static void bulk_wait_all(uint32_t lane) {     // this warp's stores complete
-    if (lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
-    __syncwarp();
-  }
+  __device__ static void bulk_wait_all(uint32_t lane) { GemmBody::bulk_wait_all(lane); }
 
   // The pair's pipeline. Next(b0, b1) is called by the leader's scheduling thread: it returns
   // false when the pair must stop, else the next chunk [b0, b1) of tiles. Returns after both

@@ -42,7 +42,8 @@ bool to_dev(const void* user, GemmArgsDev* d) {
   const flep_gemm_args& u = *reinterpret_cast<const flep_gemm_args*>(user);
   d->c = reinterpret_cast<__nv_bfloat16*>(u.c);
   d->m = u.m; d->n = u.n; d->k = u.k;
-  return make_map(&d->tma_a, u.a, u.m, u.k, GemmBody::BM) && make_map(&d->tma_b, u.b, u.n, u.k, GemmBody::BN);
+  return make_map(&d->tma_a, u.a, u.m, u.k, GemmBody::BM) && make_map(&d->tma_b, u.b, u.n, u.k, GemmBody::BN) &&
+         make_map(&d->tma_c, u.c, u.m, u.n, 32);     // epilogue: 32 rows x 64 columns per bulk store
 }
 
 }  // namespace

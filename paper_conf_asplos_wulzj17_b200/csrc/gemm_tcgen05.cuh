@@ -43,6 +43,7 @@ namespace flep {
 struct GemmArgsDev {
   CUtensorMap tma_a;           // A [M,K] bf16, box {64, 128}, SWIZZLE_128B
   CUtensorMap tma_b;           // B [N,K] bf16, box {64, 256}, SWIZZLE_128B
+  CUtensorMap tma_c;           // C [M,N] bf16, box {64, 32}, SWIZZLE_128B (epilogue bulk stores)
   __nv_bfloat16* c;            // C [M,N] bf16 row-major
   uint32_t m, n, k;
 };
@@ -54,7 +55,11 @@ struct GemmBody {
   static constexpr uint32_t kBytesA = BM * BK * 2, kBytesB = BN * BK * 2, kStage = kBytesA + kBytesB;
   static constexpr uint32_t kTmemCols = 512;           // two 128x256 fp32 accumulators
   static constexpr uint32_t QDEPTH = 4;                // tile queue: scheduler -> MMA / epilogue
-  static constexpr size_t kDynSmem = 1024 + STAGES * kStage + 512;
+  // epilogue staging after the state block: per epilogue warp two 4 KB buffers (32 rows x 64
+  // bf16 columns, SWIZZLE_128B) written to C by bulk tensor stores (store_bulk)
+  static constexpr uint32_t kEpiBuf = 32 * 128;
+  static constexpr size_t kDynSmem = 1024 + STAGES * kStage + 1024 + 4 * 2 * kEpiBuf;
+  static_assert(kDynSmem <= 232448, "shared memory per block");
   static constexpr bool kPersistent = true;
   using Args = GemmArgsDev;
 
@@ -82,6 +87,7 @@ struct GemmBody {
   }
   __device__ static State* state() { return reinterpret_cast<State*>(ring() + STAGES * kStage); }
   __device__ static uint32_t smem_u32(const void* p) { return static_cast<uint32_t>(__cvta_generic_to_shared(p)); }
+  __device__ static uint8_t* epi_buf(uint32_t q) { return ring() + STAGES * kStage + 1024 + 2 * q * kEpiBuf; }
 
   __device__ static void mbar_init(uint64_t* b, uint32_t n) {
     asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" :: "r"(smem_u32(b)), "r"(n) : "memory");
@@ -212,43 +218,19 @@ struct GemmBody {
       }
     } else if (warp >= 4) {                                // ---- epilogue (128 threads)
       const uint32_t q = warp - 4;                         // TMEM lanes [32q, 32q+32)
-      uint32_t acc = s->e_acc[q];
+      uint32_t acc = s->e_acc[q], it = 0;
       const uint32_t tmem = s->tmem_base + ((q * 32u) << 16);
       for (uint32_t b = b0; b < b1; ++b) {
         int32_t tm, tn;
         tile_coords(b, gx, p_gy(g), tm, tn);
         mbar_wait(&s->tmem_full, acc);
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-        const uint32_t row = tm * BM + q * 32u + lane;
-        __nv_bfloat16* crow = g.c + (size_t)row * g.n + (size_t)tn * BN;
-#pragma unroll 1
-        for (uint32_t c0 = 0; c0 < BN; c0 += 32) {
-          uint32_t r[32];
-          asm volatile(
-              "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
-              "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
-              : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
-                "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]),
-                "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]),
-                "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
-              : "r"(tmem + c0));
-          asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
-          uint4 o[4];
-          uint32_t* ow = reinterpret_cast<uint32_t*>(o);
-#pragma unroll
-          for (int i = 0; i < 16; ++i) {
-            __nv_bfloat162 h = __floats2bfloat162_rn(__uint_as_float(r[2 * i]), __uint_as_float(r[2 * i + 1]));
-            ow[i] = *reinterpret_cast<uint32_t*>(&h);
-          }
-          uint4* dst = reinterpret_cast<uint4*>(crow + c0);
-#pragma unroll
-          for (int i = 0; i < 4; ++i) dst[i] = o[i];
-        }
+        store_bulk(&g.tma_c, epi_buf(q), tmem, 0, BN, tn * (int32_t)BN, tm * (int32_t)BM + (int32_t)(q * 32u), lane, it);
         asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
         mbar_arrive(&s->tmem_empty);
         acc ^= 1u;
       }
-      __syncwarp();
+      bulk_wait_all(lane);
       if (lane == 0) s->e_acc[q] = acc;
     }
   }
@@ -281,6 +263,55 @@ struct GemmBody {
            "r"(r[16]), "r"(r[17]), "r"(r[18]), "r"(r[19]), "r"(r[20]), "r"(r[21]), "r"(r[22]), "r"(r[23]),
            "r"(r[24]), "r"(r[25]), "r"(r[26]), "r"(r[27]), "r"(r[28]), "r"(r[29]), "r"(r[30]), "r"(r[31])
         : "memory");
+  }
+
+  // Epilogue store of one warp's 32 accumulator rows (TMEM lanes of tmem_w), columns
+  // [c_begin, c_end) in steps of 64: TMEM -> bf16 -> one of the warp's two staging buffers (row =
+  // lane, 16-B chunk c at c ^ (lane & 7): the SWIZZLE_128B layout of the C tensor map) -> one bulk
+  // tensor store of 32 x 64 issued by lane 0 at (x0 + c, y0), so the store of one chunk overlaps
+  // the next chunk's TMEM loads and C is written in full 128-B lines (the per-lane row stores it
+  // replaces issued one 16-B request per row). `it` counts the warp's stores (buffer it & 1);
+  // the warp ends with bulk_wait_all() before the CTA can exit. Used by both GEMM bodies.
+  __device__ static void store_bulk(const CUtensorMap* tmc, uint8_t* bufs, uint32_t tmem_w, uint32_t c_begin,
+                                    uint32_t c_end, int32_t x0, int32_t y0, uint32_t lane, uint32_t& it) {
+#pragma unroll 1
+    for (uint32_t c0 = c_begin; c0 < c_end; c0 += 64) {
+      uint32_t o[32];
+#pragma unroll
+      for (uint32_t hh = 0; hh < 2; ++hh) {
+        uint32_t v[32];
+        tmem_ld32(tmem_w + c0 + 32 * hh, v);
+#pragma unroll
+        for (int i = 0; i < 16; ++i) {
+          __nv_bfloat162 hv = __floats2bfloat162_rn(__uint_as_float(v[2 * i]), __uint_as_float(v[2 * i + 1]));
+          o[16 * hh + i] = *reinterpret_cast<uint32_t*>(&hv);
+        }
+      }
+      if (it >= 2) {                                   // the store that used this buffer has read it
+        if (lane == 0) asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
+        __syncwarp();
+      }
+      uint8_t* buf = bufs + (it & 1u) * kEpiBuf;
+      const uint32_t rowb = smem_u32(buf) + lane * 128u;
+#pragma unroll
+      for (uint32_t c = 0; c < 8; ++c)
+        asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};"
+                     :: "r"(rowb + ((c ^ (lane & 7u)) << 4)), "r"(o[4 * c]), "r"(o[4 * c + 1]), "r"(o[4 * c + 2]),
+                        "r"(o[4 * c + 3]) : "memory");
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // visible to the bulk store
+      __syncwarp();
+      if (lane == 0) {
+        asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];"
+                     :: "l"(reinterpret_cast<uint64_t>(tmc)), "r"(smem_u32(buf)), "r"(x0 + (int32_t)c0), "r"(y0)
+                     : "memory");
+        asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+      }
+      ++it;
+    }
+  }
+  __device__ static void bulk_wait_all(uint32_t lane) {    // this warp's bulk stores are complete
+    if (lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+    __syncwarp();
   }
 
   // ---- persistent FLEP worker loop (warp-specialised; chunk boundaries do not drain the
@@ -439,7 +470,7 @@ struct GemmBody {
     } else if (warp >= 4) {                                // ---- epilogue (128 threads)
       const uint32_t q = warp - 4;
       const uint32_t rl = q * 32u + lane;                  // tile row (TMEM lane) of this thread
-      uint32_t qi = 0, qph = 0, acc = 0, aph = 0;
+      uint32_t qi = 0, qph = 0, acc = 0, aph = 0, it = 0;
       while (true) {
         mbar_wait(&s->qfull[qi], qph);
         const uint32_t b = s->tile_q[qi];
@@ -483,28 +514,13 @@ struct GemmBody {
                                  __uint_as_float(r[4 * j + 2]), __uint_as_float(r[4 * j + 3])));
           }
         } else {
-          const uint32_t row = tm * BM + rl;
-          __nv_bfloat16* crow = g.c + (size_t)row * g.n + (size_t)tn * BN;
-#pragma unroll 1
-          for (uint32_t c0 = 0; c0 < BN; c0 += 32) {
-            uint32_t r[32];
-            tmem_ld32(tmem + c0, r);
-            uint4 o[4];
-            uint32_t* ow = reinterpret_cast<uint32_t*>(o);
-#pragma unroll
-            for (int i = 0; i < 16; ++i) {
-              __nv_bfloat162 h = __floats2bfloat162_rn(__uint_as_float(r[2 * i]), __uint_as_float(r[2 * i + 1]));
-              ow[i] = *reinterpret_cast<uint32_t*>(&h);
-            }
-            uint4* dst = reinterpret_cast<uint4*>(crow + c0);
-#pragma unroll
-            for (int i = 0; i < 4; ++i) dst[i] = o[i];
-          }
+          store_bulk(&g.tma_c, epi_buf(q), tmem, 0, BN, tn * (int32_t)BN, tm * (int32_t)BM + (int32_t)(q * 32u), lane, it);
         }
         asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
         mbar_arrive(&s->tempty[acc]);
         if (++acc == 2) { acc = 0; aph ^= 1u; }
       }
+      bulk_wait_all(lane);
     }
     __syncthreads();
   }
