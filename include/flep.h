@@ -174,7 +174,8 @@ typedef struct {
    continues the k-loop. The result stays bit-identical to an uninterrupted run. Costs
    W x (16 B + 128 KiB) of device memory per launch (runtime-owned, pooled); for the CTA-pair
    body (FLEP_BODY_GEMM_BF16_2SM) one record per pair and one 128 KiB slot per CTA (each CTA
-   spills its 128-row half of the 256x256 tile).
+   spills its 128-row half of the 256x256 tile); for the wide pair body
+   (FLEP_BODY_GEMM_BF16_2SM_W) two 128 KiB slots per CTA (its 128x512 half).
    flep_register_kernel returns FLEP_ERR_UNSUPPORTED for other bodies or with prefetch. */
 #define FLEP_KFLAG_IN_TILE 4u
 /* Asynchronous poll: the control word a worker tests at a poll point was loaded at its previous
