@@ -1731,6 +1731,15 @@ def run_slicing_overhead(args, rank, world, local):
                  "flep_c1_over_static_pct": round((gm["flep_c1"] / gm["static_u1"] - 1) * 100, 2),
                  "wide_flep_c1_vs_cublas": round(gm["cublas"] / gm["wide_flep_c1"], 3),
                  "wide_flep_c1_over_static_pct": round((gm["wide_flep_c1"] / gm["wide_static_u1"] - 1) * 100, 2)}
+        # the wrapped tensor-core kernel against the tensor roofline (burst peak: a kernel timed
+        # alone between others, MEASURED_PEAKS.json)
+        from bench import peaks
+        _, pk_burst, pk_sus, pk_src = peaks()
+        ach = flop / gm["wide_flep_c1"] / 1e6
+        gemm2["roofline"] = {"bound": "tensor", "kernel": "flep_gemm2_worker<Gemm2T<512>> C = 1",
+                             "achieved": round(ach, 1), "peak": pk_burst, "unit": "TFLOP/s",
+                             "frac": round(ach / pk_burst, 4), "peak_source": pk_src + " (burst)",
+                             "frac_of_sustained_peak": round(ach / pk_sus, 4)}
     rt_m.close()
     rt_s.close()
     big = [r for r in rows if r["kernel"].endswith("-2")]
