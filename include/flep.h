@@ -288,6 +288,37 @@ flep_status flep_shutdown(flep_rt rt);
 /* num_sms = multiprocessor count; nsmid = %nsmid upper bound of %smid values. */
 flep_status flep_device_info(flep_rt rt, uint32_t* num_sms, uint32_t* nsmid);
 
+/* ---- user-defined bodies (extension; the paper transforms any kernel) ------------
+   A body written in the caller's own .cu against include/flep_body.cuh (a struct with Args,
+   kThreads, kMinBlocks and `run(args, b0, b1, gx, gy)` running original blocks [b0, b1), plus
+   setup/teardown) gets the FLEP worker, the original (unwrapped) grid and the static twin
+   instantiated there by FLEP_DEFINE_BODY(sym, Body), which also defines `sym_ops(flep_body_ops*)`.
+   flep_register_body copies the table and returns a body id (>= FLEP_BODY_USER_FIRST) usable in
+   flep_kernel_desc.body like a built-in one: counter worker (chunk C, poll K), temporal and
+   spatial preemption, resume, managed policies. Not available to user bodies: CLC, the
+   scheduling-warp / warp-task / in-chunk workers, in-tile preemption, slicing with the device
+   check. The caller's .cu must be compiled against the same flep headers as libflep.so
+   (abi_version), for sm_100a, and its module must stay loaded while the runtime uses the body.
+   Errors: FLEP_ERR_INVALID for NULL or incomplete tables, a zero or > 1024 thread count, a
+   mismatched abi_version; FLEP_ERR_NOMEM when FLEP_BODY_USER_MAX bodies are registered. */
+#define FLEP_BODY_USER_FIRST 64
+#define FLEP_BODY_USER_MAX 16
+#define FLEP_BODY_ABI_VERSION 1u
+typedef struct {
+  uint32_t abi_version;        /* FLEP_BODY_ABI_VERSION */
+  uint32_t threads;            /* CTA size of the body (Body::kThreads) */
+  size_t args_size;            /* sizeof(Body::Args): flep_launch's args_size must match */
+  const char* name;
+  /* cudaError_t-valued launchers (0 = success) generated by FLEP_DEFINE_BODY: W worker CTAs with
+     the runtime's (opaque) worker parameters; the original grid or its 1-D slice
+     [offset, offset + count); the static persistent twin; resident worker CTAs per SM */
+  int (*worker)(const void* args, const void* worker_params, uint32_t ctas, flep_stream_t stream, int coverage);
+  int (*unwrapped)(const void* args, flep_dim3 grid, uint32_t offset, uint32_t count, flep_stream_t stream);
+  int (*static_launch)(const void* args, flep_dim3 grid, uint32_t ctas, uint32_t chunk, flep_stream_t stream);
+  int (*occupancy)(int* ctas_per_sm, int coverage);
+} flep_body_ops;
+flep_status flep_register_body(flep_rt rt, const flep_body_ops* ops, int32_t* body_out);
+
 /* ---- kernels and launches ------------------------------------------------------------- */
 flep_status flep_register_kernel(flep_rt rt, const flep_kernel_desc* desc, flep_kernel* out);
 /* Intercepted launch: `grid` is the ORIGINAL grid in blocks; `args` points to the

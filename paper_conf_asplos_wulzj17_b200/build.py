@@ -56,5 +56,21 @@ def build(force: bool = False, verbose: bool = False) -> str:
     return LIB
 
 
+def build_user_body(src: str, out: str, force: bool = False) -> str:
+    """Compile a user-defined body (a .cu using include/flep_body.cuh and FLEP_DEFINE_BODY) into
+    its own shared library with the flags and headers libflep.so was built with."""
+    deps = [src, os.path.join(ROOT, "include", "flep_body.cuh"), os.path.join(ROOT, "include", "flep.h"),
+            os.path.join(CSRC, "flep_device.cuh")]
+    if not force and os.path.exists(out) and all(os.path.getmtime(d) <= os.path.getmtime(out) for d in deps):
+        return out
+    os.makedirs(os.path.dirname(os.path.abspath(out)), exist_ok=True)
+    cmd = [_nvcc()] + NVCC_FLAGS + ["-I", os.path.join(ROOT, "include"), "-o", out + ".tmp", src]
+    r = subprocess.run(cmd, capture_output=True, text=True)
+    if r.returncode != 0:
+        raise RuntimeError("nvcc failed for the user body:\n" + r.stdout + r.stderr)
+    os.replace(out + ".tmp", out)
+    return out
+
+
 if __name__ == "__main__":
     print(build(force="--force" in sys.argv, verbose=True))

@@ -9,6 +9,9 @@
 #include "stencil_tma.cuh"
 #include "kernels.hpp"
 
+#include <mutex>
+#include <utility>
+
 namespace flep {
 
 namespace {
@@ -249,7 +252,67 @@ cudaError_t set_unwrapped_trace(uint64_t* p) {
 }
 #endif
 
+// ---- user-defined bodies (flep_register_body): a fixed table of FLEP_BODY_USER_MAX slots whose
+// BodyOps entries are thunks into the caller's C launchers (plain function pointers, no captures)
+namespace {
+flep_body_ops g_user_tab[FLEP_BODY_USER_MAX];
+BodyOps g_user_ops[FLEP_BODY_USER_MAX];
+int g_user_n = 0;
+std::mutex g_user_mu;
+
+template <int I>
+cudaError_t u_worker(const void* a, const WorkerParams& p, uint32_t W, cudaStream_t s, bool cov) {
+  return static_cast<cudaError_t>(g_user_tab[I].worker(a, &p, W, static_cast<flep_stream_t>(s), cov ? 1 : 0));
+}
+template <int I>
+cudaError_t u_unwrapped(const void* a, dim3 g, uint32_t offset, uint32_t count, cudaStream_t s) {
+  const flep_dim3 d = {g.x, g.y, g.z};
+  return static_cast<cudaError_t>(g_user_tab[I].unwrapped(a, d, offset, count, static_cast<flep_stream_t>(s)));
+}
+template <int I>
+cudaError_t u_static(const void* a, dim3 g, uint32_t ctas, uint32_t chunk, cudaStream_t s) {
+  const flep_dim3 d = {g.x, g.y, g.z};
+  return static_cast<cudaError_t>(g_user_tab[I].static_launch(a, d, ctas, chunk, static_cast<flep_stream_t>(s)));
+}
+template <int I>
+cudaError_t u_occupancy(int* k, bool cov) {
+  return static_cast<cudaError_t>(g_user_tab[I].occupancy(k, cov ? 1 : 0));
+}
+template <int I>
+void make_user_ops(BodyOps& o) {
+  o = BodyOps{};
+  o.body = FLEP_BODY_USER_FIRST + I;
+  o.threads = static_cast<int>(g_user_tab[I].threads);
+  o.args_size = g_user_tab[I].args_size;
+  o.worker = &u_worker<I>;
+  o.unwrapped = &u_unwrapped<I>;
+  o.occupancy = &u_occupancy<I>;
+  o.static_launch = g_user_tab[I].static_launch ? &u_static<I> : nullptr;
+}
+template <int... I>
+void make_user_ops_at(int slot, std::integer_sequence<int, I...>) {
+  ((slot == I ? make_user_ops<I>(g_user_ops[I]) : void()), ...);
+}
+}  // namespace
+
+int32_t register_user_body(const flep_body_ops* o, const char** why) {
+  if (!o || !o->worker || !o->unwrapped || !o->occupancy) { *why = "incomplete flep_body_ops"; return -1; }
+  if (o->abi_version != FLEP_BODY_ABI_VERSION) { *why = "abi_version mismatch"; return -1; }
+  if (o->threads == 0 || o->threads > 1024 || o->args_size == 0) { *why = "threads / args_size out of range"; return -1; }
+  std::lock_guard<std::mutex> lk(g_user_mu);
+  if (g_user_n >= FLEP_BODY_USER_MAX) { *why = "all FLEP_BODY_USER_MAX user body slots are taken"; return -2; }
+  const int slot = g_user_n;
+  g_user_tab[slot] = *o;
+  make_user_ops_at(slot, std::make_integer_sequence<int, FLEP_BODY_USER_MAX>{});
+  g_user_n = slot + 1;                     // published after the entry is complete
+  return FLEP_BODY_USER_FIRST + slot;
+}
+
 const BodyOps* body_ops(int32_t body) {
+  if (body >= FLEP_BODY_USER_FIRST && body < FLEP_BODY_USER_FIRST + FLEP_BODY_USER_MAX) {
+    std::lock_guard<std::mutex> lk(g_user_mu);
+    return body - FLEP_BODY_USER_FIRST < g_user_n ? &g_user_ops[body - FLEP_BODY_USER_FIRST] : nullptr;
+  }
   if (body < 1 || body > FLEP_BODY_GEMM_BF16_2SM_W) return nullptr;
   return &kOps[body];
 }

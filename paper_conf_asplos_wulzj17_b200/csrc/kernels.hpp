@@ -47,6 +47,8 @@ struct BodyOps {
 };
 
 const BodyOps* body_ops(int32_t body);
+// user-defined bodies: the id (>= FLEP_BODY_USER_FIRST), -1 invalid table, -2 no slot left
+int32_t register_user_body(const flep_body_ops* ops, const char** why);
 // GEMM bodies (gemm_tcgen05.cu, gemm2_tcgen05.cu)
 cudaError_t gemm_static_launch(const void* user, dim3 grid, uint32_t ctas, uint32_t chunk, cudaStream_t s);
 cudaError_t gemm2_worker_launch(const void* user, const WorkerParams& p, uint32_t ctas, cudaStream_t s, bool cov);

@@ -929,6 +929,16 @@ flep_status flep_init(int device, const flep_options* opts, flep_rt* out) {
   return FLEP_OK;
 }
 
+flep_status flep_register_body(flep_rt rt, const flep_body_ops* ops, int32_t* body_out) {
+  if (!rt || !ops || !body_out) return fail(FLEP_ERR_INVALID, "NULL argument");
+  const char* why = "";
+  const int32_t id = register_user_body(ops, &why);
+  if (id == -2) return fail(FLEP_ERR_NOMEM, "flep_register_body: %s", why);
+  if (id < 0) return fail(FLEP_ERR_INVALID, "flep_register_body: %s", why);
+  *body_out = id;
+  return FLEP_OK;
+}
+
 flep_status flep_device_info(flep_rt rt, uint32_t* num_sms, uint32_t* nsmid) {
   if (!rt) return fail(FLEP_ERR_INVALID, "rt is NULL");
   if (num_sms) *num_sms = rt->num_sms;

@@ -93,6 +93,16 @@ class WorkerEvent(C.Structure):
                 ("epoch", C.c_uint32), ("t_entry", C.c_uint64), ("t_exit", C.c_uint64)]
 
 
+class BodyOps(C.Structure):
+    """flep_body_ops (include/flep.h): filled by a user body library's `<sym>_ops` function."""
+    _fields_ = [("abi_version", C.c_uint32), ("threads", C.c_uint32), ("args_size", C.c_size_t),
+                ("name", C.c_char_p), ("worker", C.c_void_p), ("unwrapped", C.c_void_p),
+                ("static_launch", C.c_void_p), ("occupancy", C.c_void_p)]
+
+
+BODY_USER_FIRST = 64
+
+
 class EpochInfo(C.Structure):
     _fields_ = [("t_trigger", C.c_uint64), ("t_end", C.c_uint64), ("trigger_block", C.c_uint32),
                 ("done", C.c_uint32), ("counter", C.c_uint32), ("state", C.c_uint32),
@@ -111,6 +121,7 @@ _SIG = {
     "flep_shutdown": (C.c_int, [_P]),
     "flep_device_info": (C.c_int, [_P, C.POINTER(C.c_uint32), C.POINTER(C.c_uint32)]),
     "flep_register_kernel": (C.c_int, [_P, C.POINTER(KernelDesc), C.POINTER(C.c_int32)]),
+    "flep_register_body": (C.c_int, [_P, C.POINTER(BodyOps), C.POINTER(C.c_int32)]),
     "flep_launch": (C.c_int, [_P, C.c_int32, Dim3, _P, C.c_size_t, C.c_int32, _P, C.POINTER(C.c_int64)]),
     "flep_preempt": (C.c_int, [_P, C.c_int64, C.c_uint32]),
     "flep_resume": (C.c_int, [_P, C.c_int64]),
@@ -151,6 +162,9 @@ _SIG = {
 }
 
 _lib = None
+
+
+_user_libs = {}                       # user body libraries, loaded once and never unloaded
 
 
 def lib():
@@ -239,6 +253,21 @@ class Runtime:
         k = C.c_int32()
         check(self.L.flep_register_kernel(self.h, C.byref(d), C.byref(k)), "flep_register_kernel")
         return k.value
+
+    def register_body(self, lib_path, sym):
+        """Register a user-defined body (include/flep_body.cuh): load its library (kept loaded
+        for the process), fill the ops table through `<sym>_ops` and return the body id."""
+        ul = _user_libs.get(lib_path)
+        if ul is None:
+            ul = _user_libs[lib_path] = C.CDLL(lib_path)
+        fill = getattr(ul, sym + "_ops")
+        fill.restype = None
+        fill.argtypes = [C.POINTER(BodyOps)]
+        ops = BodyOps()
+        fill(C.byref(ops))
+        body = C.c_int32()
+        check(self.L.flep_register_body(self.h, C.byref(ops), C.byref(body)), "flep_register_body")
+        return body.value
 
     def launch(self, kernel, grid, args, priority=0, stream=None):
         out = C.c_int64()
