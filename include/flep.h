@@ -295,9 +295,9 @@ flep_status flep_device_info(flep_rt rt, uint32_t* num_sms, uint32_t* nsmid);
    instantiated there by FLEP_DEFINE_BODY(sym, Body), which also defines `sym_ops(flep_body_ops*)`.
    flep_register_body copies the table and returns a body id (>= FLEP_BODY_USER_FIRST) usable in
    flep_kernel_desc.body like a built-in one: counter worker (chunk C, poll K), temporal and
-   spatial preemption, resume, managed policies. Not available to user bodies: CLC, the
-   scheduling-warp / warp-task / in-chunk workers, in-tile preemption, slicing with the device
-   check. The caller's .cu must be compiled against the same flep headers as libflep.so
+   spatial preemption, resume, managed policies, the CLC fetch and slicing with the device
+   check. Not available to user bodies: the scheduling-warp / warp-task / in-chunk workers and
+   in-tile preemption. The caller's .cu must be compiled against the same flep headers as libflep.so
    (abi_version), for sm_100a, and its module must stay loaded while the runtime uses the body.
    Errors: FLEP_ERR_INVALID for NULL or incomplete tables, a zero or > 1024 thread count, a
    mismatched abi_version; FLEP_ERR_NOMEM when FLEP_BODY_USER_MAX bodies are registered. */
@@ -316,6 +316,12 @@ typedef struct {
   int (*unwrapped)(const void* args, flep_dim3 grid, uint32_t offset, uint32_t count, flep_stream_t stream);
   int (*static_launch)(const void* args, flep_dim3 grid, uint32_t ctas, uint32_t chunk, flep_stream_t stream);
   int (*occupancy)(int* ctas_per_sm, int coverage);
+  /* optional (NULL = unsupported): the CLC worker over the original grid in chunks
+     (FLEP_KFLAG_CLC), and the device-checked slice kernel (FLEP_POLICY_SLICE_DEVICE) with the
+     runtime's (opaque) slice parameters */
+  int (*clc)(const void* args, const void* worker_params, uint32_t ctas, flep_stream_t stream, int coverage);
+  int (*sliced)(const void* args, flep_dim3 grid, uint32_t offset, uint32_t count, const void* slice_params,
+                flep_stream_t stream);
 } flep_body_ops;
 flep_status flep_register_body(flep_rt rt, const flep_body_ops* ops, int32_t* body_out);
 

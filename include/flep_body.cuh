@@ -7,7 +7,9 @@
 //     from the launch's counter, poll the control word every K chunks and yield (temporal or
 //     spatial), exactly-once across preempt/resume;
 //   * the original kernel (flep_unwrapped<Body>): one CTA per original block;
-//   * the static persistent twin (flep_static<Body>): the overhead baseline.
+//   * the static persistent twin (flep_static<Body>): the overhead baseline;
+//   * the CLC worker (flep_clc_worker<Body>, FLEP_KFLAG_CLC) and the device-checked slice kernel
+//     (flep_slice<Body>, FLEP_POLICY_SLICE_DEVICE).
 //
 // A body is a struct with
 //   using Args = <trivially copyable argument struct, passed by value to the grids>;
@@ -73,6 +75,24 @@ int user_occupancy(int* k, int cov) {
 }
 
 template <class Body>
+int user_clc_launch(const void* a, const void* wp, uint32_t N, flep_stream_t s, int cov) {
+  const auto& args = *static_cast<const typename Body::Args*>(a);
+  const auto& p = *static_cast<const WorkerParams*>(wp);
+  const cudaStream_t st = static_cast<cudaStream_t>(s);
+  if (cov) flep_clc_worker<Body, true><<<N, Body::kThreads, 0, st>>>(args, p);
+  else flep_clc_worker<Body, false><<<N, Body::kThreads, 0, st>>>(args, p);
+  return static_cast<int>(cudaGetLastError());
+}
+
+template <class Body>
+int user_slice_launch(const void* a, flep_dim3 g, uint32_t offset, uint32_t count, const void* sp, flep_stream_t s) {
+  const auto& args = *static_cast<const typename Body::Args*>(a);
+  flep_slice<Body><<<count, Body::kThreads, 0, static_cast<cudaStream_t>(s)>>>(
+      args, g.x, g.y, offset, *static_cast<const SliceParams*>(sp));
+  return static_cast<int>(cudaGetLastError());
+}
+
+template <class Body>
 void user_body_ops(flep_body_ops* o, const char* name) {
   static_assert(!Body::kPersistent, "user bodies run original blocks (kPersistent = false)");
   o->abi_version = FLEP_BODY_ABI_VERSION;
@@ -83,6 +103,8 @@ void user_body_ops(flep_body_ops* o, const char* name) {
   o->unwrapped = &user_unwrapped_launch<Body>;
   o->static_launch = &user_static_launch<Body>;
   o->occupancy = &user_occupancy<Body>;
+  o->clc = &user_clc_launch<Body>;
+  o->sliced = &user_slice_launch<Body>;
 }
 
 }  // namespace flep

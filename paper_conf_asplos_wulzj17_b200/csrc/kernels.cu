@@ -275,6 +275,15 @@ cudaError_t u_static(const void* a, dim3 g, uint32_t ctas, uint32_t chunk, cudaS
   return static_cast<cudaError_t>(g_user_tab[I].static_launch(a, d, ctas, chunk, static_cast<flep_stream_t>(s)));
 }
 template <int I>
+cudaError_t u_clc(const void* a, const WorkerParams& p, uint32_t N, cudaStream_t s, bool cov) {
+  return static_cast<cudaError_t>(g_user_tab[I].clc(a, &p, N, static_cast<flep_stream_t>(s), cov ? 1 : 0));
+}
+template <int I>
+cudaError_t u_sliced(const void* a, dim3 g, uint32_t offset, uint32_t count, const SliceParams& sp, cudaStream_t s) {
+  const flep_dim3 d = {g.x, g.y, g.z};
+  return static_cast<cudaError_t>(g_user_tab[I].sliced(a, d, offset, count, &sp, static_cast<flep_stream_t>(s)));
+}
+template <int I>
 cudaError_t u_occupancy(int* k, bool cov) {
   return static_cast<cudaError_t>(g_user_tab[I].occupancy(k, cov ? 1 : 0));
 }
@@ -288,6 +297,8 @@ void make_user_ops(BodyOps& o) {
   o.unwrapped = &u_unwrapped<I>;
   o.occupancy = &u_occupancy<I>;
   o.static_launch = g_user_tab[I].static_launch ? &u_static<I> : nullptr;
+  o.clc = g_user_tab[I].clc ? &u_clc<I> : nullptr;
+  o.sliced = g_user_tab[I].sliced ? &u_sliced<I> : nullptr;
 }
 template <int... I>
 void make_user_ops_at(int slot, std::integer_sequence<int, I...>) {

@@ -97,7 +97,8 @@ class BodyOps(C.Structure):
     """flep_body_ops (include/flep.h): filled by a user body library's `<sym>_ops` function."""
     _fields_ = [("abi_version", C.c_uint32), ("threads", C.c_uint32), ("args_size", C.c_size_t),
                 ("name", C.c_char_p), ("worker", C.c_void_p), ("unwrapped", C.c_void_p),
-                ("static_launch", C.c_void_p), ("occupancy", C.c_void_p)]
+                ("static_launch", C.c_void_p), ("occupancy", C.c_void_p), ("clc", C.c_void_p),
+                ("sliced", C.c_void_p)]
 
 
 BODY_USER_FIRST = 64

@@ -137,3 +137,59 @@ def test_args_size_mismatch_is_rejected(env):
     k = rt.register_kernel(body, chunk=1, poll=1)
     with pytest.raises(f.FlepError):                 # a 24-byte SAXPY struct for a 32-byte body
         rt.launch(k, (4, 1, 1), f.SaxpyI32Args(0, 0, 1, 0))
+
+
+@pytest.mark.parametrize("chunk", [1, 4])
+def test_clc_worker_of_a_user_body(env, chunk):
+    """The CLC fetch (hardware work queue, R25) instantiated for the user body: exact result,
+    every block once, also across host-issued preempt/resume cycles."""
+    import time
+    import torch
+    f, rt, body = env
+    n = 1 << 24
+    x, xd, yd, args = _case(n, seed=970 + chunk)
+    grid = (-(-n // PER), 1, 1)
+    k = rt.register_kernel(body, chunk=chunk, poll=1, clc=True)
+    h = rt.launch(k, grid, args)
+    g = gen.rng(971 + chunk)
+    try:
+        for _ in range(3):
+            time.sleep(float(g.uniform(5e-6, 40e-6)))
+            rt.preempt(h, rt.num_sms if g.random() < 0.5 else int(g.integers(1, rt.num_sms)))
+            time.sleep(float(g.uniform(5e-6, 40e-6)))
+            rt.resume(h)
+    except f.FlepError:                              # the grid completed between two requests
+        assert rt.query(h).state == f.STATE_DONE
+    rt.sync(h, timeout_ns=20_000_000_000)
+    torch.cuda.synchronize()
+    assert np.all(rt.coverage_np(h, grid[0]) == 1)
+    assert np.array_equal(yd.cpu().numpy(), affine_rev_ref(x, 1664525, 1013904223))
+
+
+def test_device_checked_slicing_of_a_user_body():
+    """FLEP_POLICY_SLICE_DEVICE (R31) with the user body's slice kernel: a higher-priority arrival
+    makes the remaining slices skip, the resumed slices finish the grid, results exact."""
+    import torch
+    from paper_conf_asplos_wulzj17_b200 import build
+    f = flep_mod()
+    rs = f.Runtime(policy=f.POLICY_SLICE_DEVICE, slice_blocks=2048)
+    try:
+        body = rs.register_body(build.build_user_body(SRC, OUT), "affine_rev")
+        n = 1 << 26
+        x, xd, yd, args = _case(n, seed=980)
+        grid = (-(-n // PER), 1, 1)
+        kl = rs.register_kernel(body, chunk=1, poll=1, model=(0, 0, 0, 0, 5_000_000))
+        kh = rs.register_kernel(f.BODY_SAXPY_I32, chunk=1, poll=1, model=(0, 0, 0, 0, 5_000))
+        x2, y2 = gen.saxpy_i32_inputs(1 << 16, seed=981)
+        x2d, y2d = torch.from_numpy(x2).cuda(), torch.from_numpy(y2).cuda()
+        h1 = rs.launch(kl, grid, args, priority=0)
+        h2 = rs.launch(kh, f.saxpy_grid(1 << 16), f.saxpy_i32_args(y2d, x2d, 5), priority=1)
+        rs.sync(h2, timeout_ns=20_000_000_000)
+        rs.sync(h1, timeout_ns=20_000_000_000)
+        torch.cuda.synchronize()
+        assert np.array_equal(yd.cpu().numpy(), affine_rev_ref(x, 1664525, 1013904223))
+        assert np.array_equal(y2d.cpu().numpy(), W.saxpy_i32(5, x2, y2))
+        acts = [f.ACTION_NAMES[d[1]] for d in rs.decision_log()]
+        assert acts[:3] == ["LAUNCH", "PREEMPT", "LAUNCH"]
+    finally:
+        rs.close()

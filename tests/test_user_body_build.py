@@ -31,7 +31,8 @@ def test_user_body_compiles_and_fills_its_ops(libs):
     assert ops.threads == 128
     assert ops.args_size == 32                      # {int32_t* y; const int32_t* x; int32_t a, c; uint32_t n}
     assert ops.name == b"affine_rev"
-    assert all(getattr(ops, f) for f in ("worker", "unwrapped", "static_launch", "occupancy"))
+    assert ops.clc and ops.sliced
+    assert all(getattr(ops, f) for f in ("worker", "unwrapped", "static_launch", "occupancy", "clc", "sliced"))
 
 
 def test_register_body_is_exported_and_checks_arguments(libs):
