@@ -14,7 +14,9 @@
 // A body is a struct with
 //   using Args = <trivially copyable argument struct, passed by value to the grids>;
 //   static constexpr int kThreads;      // CTA size
-//   static constexpr int kMinBlocks;    // __launch_bounds__ min blocks per SM
+//   static constexpr int kMinBlocks;    // __launch_bounds__ min blocks per SM: give the original
+//                                       // grid's occupancy, so that the worker (which holds more
+//                                       // state) is register-capped to the same CTAs per SM
 //   __device__ static void run(const Args&, uint32_t b0, uint32_t b1, uint32_t gx, uint32_t gy);
 //                                       // run original blocks [b0, b1) of a gx x gy grid; every
 //                                       // thread of the CTA calls it; a block's result must not

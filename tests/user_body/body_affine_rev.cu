@@ -17,7 +17,7 @@ struct AffineRevArgs {
 struct AffineRevBody : flep::UserBody {
   using Args = AffineRevArgs;
   static constexpr int kThreads = 128;
-  static constexpr int kMinBlocks = 8;
+  static constexpr int kMinBlocks = 16;    // the original grid's 2048 threads per SM: the worker keeps them
   static constexpr uint32_t kPer = 512;
   __device__ static void run(const Args& g, uint32_t b0, uint32_t b1, uint32_t, uint32_t) {
     __shared__ int32_t s[kPer];
