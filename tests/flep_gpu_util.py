@@ -29,15 +29,6 @@ def saxpy_i32_case(n, seed):
     return x, y
 
 
-def check_yield_events(rt, h, epoch, num_sms):
-    """I3 on the device log: a worker exits with YIELD only on a requested SM."""
-    f = flep_mod()
-    info = rt.query(h)
-    ev = rt.events(h, epoch)
-    ep = rt.epoch_info(h, epoch)
-    return ev, ep
-
-
 def run_manual_schedule(rt, kernel, grid, args, n_blocks, schedule, num_sms, check_prefix=True,
                         priority=0, stats=None):
     """Execute one manual-mode preempt/resume schedule driven by device self-triggers.
