@@ -28,6 +28,9 @@
 #ifndef FLEP_SPMV_AU
 #define FLEP_SPMV_AU 8               // gathers in flight per thread in the cp.async body
 #endif
+#ifndef FLEP_SPMV_MINB
+#define FLEP_SPMV_MINB 8             // SpMV CSR-stream: __launch_bounds__ min blocks (8 -> 32 registers)
+#endif
 #ifndef FLEP_SPMV_TILE
 #define FLEP_SPMV_TILE 2048          // SpMV CSR-stream: nonzeros per shared-memory product tile
 #endif
@@ -112,7 +115,7 @@ struct SaxpyBody : NoResources {
 // unwrapped, preempted and resumed) gives bit-identical results.
 struct SpmvBody : NoResources {
   static constexpr int kThreads = 256;
-  static constexpr int kMinBlocks = 8;
+  static constexpr int kMinBlocks = FLEP_SPMV_MINB;   // resident CTAs per SM the register budget is sized for
   static constexpr uint32_t kRowsPerBlock = FLEP_SPMV_ROWS;
   static constexpr uint32_t kTile = FLEP_SPMV_TILE;     // products staged per tile (smem)
   using Args = flep_spmv_args;
