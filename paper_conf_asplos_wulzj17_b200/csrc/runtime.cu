@@ -991,6 +991,22 @@ flep_status flep_register_kernel(flep_rt rt, const flep_kernel_desc* d, flep_ker
       CUDA_TRY(cudaMalloc(&p, need));
       rt->free_partial.push_back({p, need});
     }
+  } else if (d->flags & (FLEP_KFLAG_SPEC_FETCH | FLEP_KFLAG_IN_CHUNK)) {
+    // the per-worker chunk records of the speculative fetch / in-chunk stop (16 B per worker),
+    // also allocated here and not on the launch path; a preempted launch keeps its buffer until
+    // it completes, so a queue can hold several at once: keep eight in the pool
+    int kk = 0;
+    flep_status s = occupancy(rt, body_ops(d->body), (rt->opt.debug_coverage & 1u) != 0, &kk);
+    if (s) return s;
+    if (d->ctas_per_sm && (int)d->ctas_per_sm < kk) kk = (int)d->ctas_per_sm;
+    const size_t need = partial_header_bytes(std::min<uint32_t>((uint32_t)kk * rt->num_sms, rt->max_workers));
+    size_t have = 0;
+    for (auto& f : rt->free_partial) if (f.second >= need) ++have;
+    for (; have < 8; ++have) {
+      void* p = nullptr;
+      CUDA_TRY(cudaMalloc(&p, need));
+      rt->free_partial.push_back({p, need});
+    }
   }
   KernelReg k;
   k.name = d->name ? d->name : "";
