@@ -893,7 +893,9 @@ flep_status flep_init(int device, const flep_options* opts, flep_rt* out) {
   rt->max_workers = rt->num_sms * kMaxWorkersPerSm;
   rt->dmem_bytes = sizeof(ControlBlock) + (size_t)kEvEpochs * rt->max_workers * sizeof(WorkerEvent) +
                   (size_t)kMaxSlices * sizeof(uint32_t);
-  for (int i = 0; i < 16; ++i) {             // warm pool: no allocation on the launch path
+  // warm pool: no allocation on the launch path (a managed queue holds one block per running or
+  // preempted launch; nested SRPT preemptions can stack a dozen or more; 48 x ~2.4 MB)
+  for (int i = 0; i < 48; ++i) {
     void* p = nullptr;
     CUDA_TRY(cudaMalloc(&p, rt->dmem_bytes));
     CUDA_TRY(cudaMemset(p, 0, sizeof(ControlBlock)));
