@@ -168,6 +168,11 @@ struct flep_rt_s {
   cudaStream_t ctl = nullptr;              // highest-priority control stream
   cudaStream_t aux = nullptr;              // debug copies of launches whose stream went back to the pool
   uint16_t* d_rank = nullptr;
+  char* cb_slab = nullptr;           // the warm control-block pool, one allocation
+  size_t cb_slab_bytes = 0;
+  bool in_slab(const void* p) const {
+    return cb_slab && (const char*)p >= cb_slab && (const char*)p < cb_slab + cb_slab_bytes;
+  }
   HostStatus* h_slots = nullptr;
   HostStatus* d_slots = nullptr;
   std::vector<int> free_slots;
@@ -894,13 +899,18 @@ flep_status flep_init(int device, const flep_options* opts, flep_rt* out) {
   rt->dmem_bytes = sizeof(ControlBlock) + (size_t)kEvEpochs * rt->max_workers * sizeof(WorkerEvent) +
                   (size_t)kMaxSlices * sizeof(uint32_t);
   // warm pool: no allocation on the launch path (a managed queue holds one block per running or
-  // preempted launch; nested SRPT preemptions can stack a dozen or more; 48 x ~2.4 MB)
-  for (int i = 0; i < 48; ++i) {
-    void* p = nullptr;
-    CUDA_TRY(cudaMalloc(&p, rt->dmem_bytes));
-    CUDA_TRY(cudaMemset(p, 0, sizeof(ControlBlock)));
-    rt->cb_gen[p] = 0;
-    rt->free_dmem.push_back(p);
+  // preempted launch; nested SRPT preemptions can stack a dozen or more): 48 x ~2.4 MB carved from
+  // one allocation with one memset (48 separate ones made every runtime's start ~0.2 s slower)
+  {
+    constexpr int kWarm = 48;
+    rt->cb_slab_bytes = (size_t)kWarm * rt->dmem_bytes;
+    CUDA_TRY(cudaMalloc(&rt->cb_slab, rt->cb_slab_bytes));
+    CUDA_TRY(cudaMemset(rt->cb_slab, 0, rt->cb_slab_bytes));
+    for (int i = 0; i < kWarm; ++i) {
+      void* p = rt->cb_slab + (size_t)i * rt->dmem_bytes;
+      rt->cb_gen[p] = 0;
+      rt->free_dmem.push_back(p);
+    }
   }
   if (rt->opt.debug_coverage) {              // debug runtimes retain 64 launches' logs: warm more
     // (coverage buffers only with bit 0)
@@ -1395,13 +1405,14 @@ flep_status flep_shutdown(flep_rt rt) {
     for (cudaEvent_t e : L.evpool) cudaEventDestroy(e);
     for (auto& e : L.inflight) cudaEventDestroy(e.first);
     if (!L.released) {
-      if (L.dmem) cudaFree(L.dmem);
+      if (L.dmem && !rt->in_slab(L.dmem)) cudaFree(L.dmem);
       if (L.cov) cudaFree(L.cov);
       if (L.partial) cudaFree(L.partial);
     }
   }
   for (cudaEvent_t e : rt->event_pool) cudaEventDestroy(e);
-  for (void* p : rt->free_dmem) cudaFree(p);
+  for (void* p : rt->free_dmem) if (!rt->in_slab(p)) cudaFree(p);
+  if (rt->cb_slab) cudaFree(rt->cb_slab);
   for (auto& c : rt->free_cov) cudaFree(c.first);
   for (auto& c : rt->free_partial) cudaFree(c.first);
   for (cudaStream_t s : rt->all_streams) cudaStreamDestroy(s);
