@@ -984,6 +984,9 @@ def run_queue(args, rank, world, local):
            "replay_parity": "checked on CPU: tests/test_policy_replay.py replays the committed logs (tests/golden/queue_logs_r01.json) through the oracle DES",
            "makespan_ms": {k: v["makespan_ms"] for k, v in res.items()},
            "launch_call_us": {k: v["launch_call_us"] for k, v in res.items()},
+           "launch_call_note": "host time of the flep_launch call; SLICE_DEVICE enqueues every slice in that call "
+                               "(up to ~110 kernel launches, ~4 us each), which is its max; FLEP_DEBUG_SLOW=<us> "
+                               "prints any slower epoch start with its materialize/launch split",
            "t_alone_us": {f"{k[0]}-{k[1]}": round(v / 1e3, 1) for k, v in sorted(t_alone.items())}}
     if world > 1:
         from bench import allreduce_max
