@@ -299,7 +299,7 @@ def run_temporal(args, rank, world, local):
     # the victim fetches speculatively (R34): poll and fetch in one round trip, a fetched chunk is
     # returned through the worker's record on a stop
     kLP = rt.register_kernel(F.BODY_SPMV_CSR_F32, chunk=args.lp_chunk, poll=args.lp_poll, name="spmv",
-                             prefetch=bool(args.prefetch), spec_fetch=bool(args.lp_spec))
+                             prefetch=bool(args.prefetch), spec_fetch=bool(args.lp_spec), ctas_per_sm=args.lp_cps)
     # the waiting (high-priority) kernel is never preempted here: it is tuned for throughput (CLC
     # task fetch, C = 1, K = 4: 4.6 % over the unwrapped grid vs 19 % for the counter worker,
     # profiles/r01_bench_clc.json), the victim for latency (atomic counter, C = K = 1)
@@ -396,6 +396,8 @@ def run_temporal(args, rank, world, local):
     # its next poll, i.e. after the chunk it is running: at C = K = 1 the drain is bounded by one
     # chunk's execution time plus the exit), with the chunk time from the standalone wrapped run
     _, w_lp = rt.workers_for(F.BODY_SPMV_CSR_F32)
+    if args.lp_cps:
+        w_lp = min(w_lp, args.lp_cps * num_sms)
     chunk_us = kern["spmv"]["wrapped_us"] * w_lp * args.lp_chunk / n_lp
     latency_budget = {"drain_p50_us": round(d50, 3), "victim_chunk_us": round(chunk_us, 3),
                       "drain_over_chunk": round(d50 / chunk_us, 3) if chunk_us else None,
@@ -421,7 +423,7 @@ def run_temporal(args, rank, world, local):
     op2 = None
     if args.lp_chunk == 1 and args.op2:
         kLP2 = rt.register_kernel(F.BODY_SPMV_CSR_F32, chunk=2, poll=args.lp_poll, name="spmv-c2",
-                                  spec_fetch=bool(args.lp_spec))
+                                  spec_fetch=bool(args.lp_spec), ctas_per_sm=args.lp_cps)
         for _ in range(args.warmup):
             step(kLP2)
         r2 = [step(kLP2) for _ in range(args.steps)]
@@ -456,6 +458,7 @@ def run_temporal(args, rank, world, local):
                    "lp_chunk": args.lp_chunk, "lp_poll": args.lp_poll, "hp_chunk": args.hp_chunk, "hp_poll": args.hp_poll, "hp_clc": bool(args.hp_clc), "hp_prefetch": bool(args.hp_prefetch),
                    "hp_async_poll": bool(args.hp_async),
                    "prefetch": bool(args.prefetch), "lp_spec_fetch": bool(args.lp_spec),
+                   "lp_ctas_per_sm": args.lp_cps or w_lp // num_sms,
                    "flag": "stream_memop (device self-trigger for the request)",
                    "l2": "flushed between steps (write of 2x L2 bytes)", "parallelism": f"replicas x{world}"},
         "value_definition": "full-GPU preemption latency (device %globaltimer): request visible on the GPU -> "
@@ -591,7 +594,7 @@ def run_e2e(F, torch, wl, local, steps, args, diag=False):
     rt = F.Runtime(device=local, policy=F.POLICY_HPF, keep_logs=diag)
     kLP = rt.register_kernel(F.BODY_SPMV_CSR_F32, chunk=args.lp_chunk, poll=args.lp_poll, name="spmv",
                              model=(0, 0, 0, 0, 70_000), prefetch=bool(args.prefetch), started_hint=True,
-                             host_relay=bool(args.e2e_relay), spec_fetch=bool(args.lp_spec))
+                             host_relay=bool(args.e2e_relay), spec_fetch=bool(args.lp_spec), ctas_per_sm=args.lp_cps)
     kHP = rt.register_kernel(F.BODY_STENCIL5_F32, chunk=args.hp_chunk, poll=args.hp_poll, name="stencil",
                              model=(0, 0, 0, 0, 30_000), prefetch=bool(args.hp_prefetch), async_poll=bool(args.hp_async),
                              clc=bool(args.hp_clc))
@@ -834,6 +837,7 @@ def main():
     ap.add_argument("--hp-async", type=int, default=0, help="waiting kernel: async poll (R22)")
     ap.add_argument("--lp-poll", type=int, default=1)
     ap.add_argument("--lp-spec", type=int, default=1, help="victim: speculative fetch (R34)")
+    ap.add_argument("--lp-cps", type=int, default=0, help="victim: resident workers per SM (0 = occupancy, P:128)")
     ap.add_argument("--reps", type=int, default=40)
     ap.add_argument("--e2e-relay", type=int, default=1, help="e2e victim with the request-relay CTA (R28)")
     ap.add_argument("--e2e-overlap-copy", type=int, default=0, help="e2e: let the HP's input copy overlap the co-run")
