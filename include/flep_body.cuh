@@ -22,7 +22,9 @@
 //                                       // thread of the CTA calls it; a block's result must not
 //                                       // depend on which CTA or SM runs it
 // and setup/teardown/kPersistent, inherited from flep::UserBody for bodies without per-worker
-// resources. Then, at namespace scope:
+// resources. A body whose run() uses no shared memory and no CTA barrier may declare
+//   static constexpr uint32_t kWarpTasks = kThreads / 32;
+// and then runs, with the CLC fetch at K = 1, without a CTA barrier between blocks (flep_clc_ring). Then, at namespace scope:
 //   FLEP_DEFINE_BODY(my_body, MyBody)
 // defines extern "C" void my_body_ops(flep_body_ops* out), which fills the table that
 // flep_register_body(rt, &ops, &body_id) takes; body_id is then used in flep_kernel_desc.body.
@@ -81,6 +83,13 @@ int user_clc_launch(const void* a, const void* wp, uint32_t N, flep_stream_t s, 
   const auto& args = *static_cast<const typename Body::Args*>(a);
   const auto& p = *static_cast<const WorkerParams*>(wp);
   const cudaStream_t st = static_cast<cudaStream_t>(s);
+  if constexpr (ClcRing<Body>::value) {
+    if (clc_use_ring<Body>(p.poll)) {
+      if (cov) flep_clc_ring<Body, true><<<N, Body::kThreads, 0, st>>>(args, p);
+      else flep_clc_ring<Body, false><<<N, Body::kThreads, 0, st>>>(args, p);
+      return static_cast<int>(cudaGetLastError());
+    }
+  }
   if (cov) flep_clc_worker<Body, true><<<N, Body::kThreads, 0, st>>>(args, p);
   else flep_clc_worker<Body, false><<<N, Body::kThreads, 0, st>>>(args, p);
   return static_cast<int>(cudaGetLastError());

@@ -824,6 +824,125 @@ __device__ __forceinline__ uint32_t clc_response(uint32_t resp, uint32_t mbar, u
   return ok ? x : 0xffffffffu;
 }
 
+// A body whose run() uses no shared memory and no CTA barrier (the warp-task bodies: they define
+// kWarpTasks) lets the CLC worker's warps drift between blocks like the warps of separate CTAs:
+// the cancel response is broadcast through an mbarrier ring instead of a CTA barrier (below).
+template <class B, class = void> struct ClcRing { static constexpr bool value = false; };
+template <class B> struct ClcRing<B, decltype((void)B::kWarpTasks)> {
+#ifdef FLEP_NO_CLC_RING
+  static constexpr bool value = false;
+#else
+  static constexpr bool value = true;
+#endif
+};
+
+// CLC worker without a per-block CTA barrier (reading R38, flep_clc_ring): two response slots, each with a
+// "full" mbarrier (one arrival: the try_cancel's complete_tx, or thread 0's plain arrive when it
+// stops cancelling, with s_stop set) and an "empty" mbarrier (one arrival per warp once its lanes
+// have read the slot). Thread 0 reuses a slot only after every warp released it, so a warp that
+// lags a block behind still reads its own response; every warp leaves after the response that
+// says "no block" (exactly-once is unchanged: a cancelled CTA's block is run by all warps of the
+// canceller, each warp its share).
+template <class Body, bool kCoverage>
+__device__ __forceinline__ void clc_worker_ring(const typename Body::Args& args, const WorkerParams& p,
+                                                WorkerShared& ws) {
+  constexpr uint32_t kWarps = Body::kThreads / 32;
+  __shared__ alignas(16) uint32_t s_resp[2][4];
+  __shared__ alignas(8) uint64_t s_full[2], s_empty[2];
+  __shared__ uint32_t s_stop[2];
+  const uint32_t tid = threadIdx.x, lane = tid & 31u;
+  const uint32_t full0 = static_cast<uint32_t>(__cvta_generic_to_shared(&s_full[0]));
+  const uint32_t empty0 = static_cast<uint32_t>(__cvta_generic_to_shared(&s_empty[0]));
+  const uint32_t resp0 = static_cast<uint32_t>(__cvta_generic_to_shared(&s_resp[0][0]));
+  if (tid == 0) {
+    for (uint32_t j = 0; j < 2; ++j) {
+      asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" :: "r"(full0 + 8u * j) : "memory");
+      asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" :: "r"(empty0 + 8u * j), "r"(kWarps) : "memory");
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();                   // the only CTA barrier: the ring is initialised
+  Body::setup(args);
+  uint32_t b = blockIdx.x, k = 0;
+  bool have_seen = false;
+  for (uint32_t i = 0;; ++i) {
+    const uint32_t j = i & 1u, use = i >> 1;          // slot, and how often it was used before
+    if (tid == 0) {
+      bool stop = false;
+      if (++k == p.poll) {
+        k = 0;
+        const uint32_t c = (p.async_poll && have_seen) ? poll_consume(ws) : poll_ctrl(p);
+        stop = should_yield(c, p, smid_reg());
+      }
+      if (p.async_poll && !stop && k == p.poll - 1) { poll_issue(ws, p.ctrl); have_seen = true; }
+      if (use > 0) {                                 // every warp has read this slot's last response
+        uint32_t done = 0;
+        while (!done)
+          asm volatile("{ .reg .pred q; mbarrier.try_wait.parity.shared::cta.b64 q, [%1], %2; selp.u32 %0, 1, 0, q; }"
+                       : "=r"(done) : "r"(empty0 + 8u * j), "r"((use - 1u) & 1u) : "memory");
+      }
+      s_stop[j] = stop ? 1u : 0u;
+      if (!stop) clc_try_cancel(resp0 + 16u * j, full0 + 8u * j);   // overlaps the body
+      else {
+        ws.reason = kReasonYield;
+        asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" :: "r"(full0 + 8u * j) : "memory");
+      }
+      if (p.trigger_block - b * p.chunk < p.chunk) {   // device self-trigger (test/bench hook)
+        const uint32_t e = p.epoch % kEvEpochs;
+        p.cb->ep_t_trigger[e] = gtimer();
+        p.cb->ep_trigger_block[e] = p.trigger_block;
+        store_ctrl(p, ctrl_word(p.epoch, p.trigger_n));
+      }
+    }
+    const uint32_t b0 = b * p.chunk, b1 = min(b0 + p.chunk, p.n_blocks);
+    Body::run(args, b0, b1, p.gx, p.gy);
+    if (tid == 0) {
+      if (kCoverage)
+        for (uint32_t bb = b0; bb < b1; ++bb) atomicAdd(&p.cov[bb], 1u);
+      ws.blocks += b1 - b0;
+    }
+    uint32_t nb = 0xffffffffu;
+    {
+      uint32_t done = 0;
+      while (!done)
+        asm volatile("{ .reg .pred q; mbarrier.try_wait.parity.shared::cta.b64 q, [%1], %2; selp.u32 %0, 1, 0, q; }"
+                     : "=r"(done) : "r"(full0 + 8u * j), "r"(use & 1u) : "memory");
+      if (!s_stop[j]) {
+        uint32_t ok, x;
+        asm volatile("{ .reg .pred q; .reg .b128 r; ld.shared.b128 r, [%2];"
+                     " clusterlaunchcontrol.query_cancel.is_canceled.pred.b128 q, r; selp.u32 %0, 1, 0, q;"
+                     " @q clusterlaunchcontrol.query_cancel.get_first_ctaid::x.b32.b128 %1, r; }"
+                     : "=r"(ok), "=r"(x) : "r"(resp0 + 16u * j) : "memory");
+        if (ok) nb = x;
+      }
+      __syncwarp();
+      if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" :: "r"(empty0 + 8u * j) : "memory");
+    }
+    b = nb;
+    if (b == 0xffffffffu) break;
+  }
+  Body::teardown(args);
+}
+
+template <class Body, bool kCoverage>
+__global__ void __launch_bounds__(Body::kThreads, Body::kMinBlocks)
+flep_clc_ring(const __grid_constant__ typename Body::Args args, const WorkerParams p) {
+  __shared__ WorkerShared ws;
+  if (threadIdx.x == 0) { ws.sm = smid_reg(); ws.t_entry = gtimer(); ws.blocks = 0; ws.reason = kReasonExhausted; }
+  clc_worker_ring<Body, kCoverage>(args, p, ws);
+  if (threadIdx.x == 0 && blockIdx.x < p.workers) {    // event log, as in flep_clc_worker
+    WorkerEvent& e = p.ev[(p.epoch % kEvEpochs) * p.workers + blockIdx.x];
+    e.smid = ws.sm; e.reason = ws.reason; e.n_blocks = ws.blocks; e.epoch = p.epoch;
+    e.t_entry = ws.t_entry; e.t_exit = gtimer();
+  }
+}
+// The ring form is chosen when the worker polls at every block (K = 1): the barrier form then
+// holds every warp behind thread 0's poll round trip at each block (measured: stencil 4096² C = K = 1
+// +18 % -> +9-10 %, SpMV-vector +6.7 % -> +3.7 %); at K >= 2 the barrier form is as fast or faster
+// (the warps of one CTA stay on one block: better L1 reuse of the stencil's halos).
+template <class Body>
+__host__ __device__ constexpr bool clc_use_ring(uint32_t poll) { return ClcRing<Body>::value && poll == 1u; }
+
 template <class Body, bool kCoverage>
 __global__ void __launch_bounds__(Body::kThreads, Body::kMinBlocks)
 flep_clc_worker(const __grid_constant__ typename Body::Args args, const WorkerParams p) {

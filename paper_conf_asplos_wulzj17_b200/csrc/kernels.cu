@@ -27,6 +27,13 @@ struct Ops {
   }
   static cudaError_t clc(const void* args, const WorkerParams& p, uint32_t N, cudaStream_t s, bool cov) {
     const typename Body::Args& a = *reinterpret_cast<const typename Body::Args*>(args);
+    if constexpr (ClcRing<Body>::value) {
+      if (clc_use_ring<Body>(p.poll)) {
+        if (cov) flep_clc_ring<Body, true><<<N, Body::kThreads, Body::kDynSmem, s>>>(a, p);
+        else flep_clc_ring<Body, false><<<N, Body::kThreads, Body::kDynSmem, s>>>(a, p);
+        return cudaGetLastError();
+      }
+    }
     if (cov) flep_clc_worker<Body, true><<<N, Body::kThreads, Body::kDynSmem, s>>>(a, p);
     else flep_clc_worker<Body, false><<<N, Body::kThreads, Body::kDynSmem, s>>>(a, p);
     return cudaGetLastError();

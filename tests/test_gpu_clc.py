@@ -3,6 +3,7 @@ CTAs are the work queue (clusterlaunchcontrol.try_cancel) instead of the atomic 
 Every original block must run exactly once (coverage == 1) with outputs equal to the oracle's,
 uninterrupted, under temporal and spatial requests and under random preempt/resume cycles; a
 preempted CLC victim hands its SMs to a higher-priority waiting kernel."""
+import os
 import time
 
 import numpy as np
@@ -213,3 +214,100 @@ def test_clc_rejected_for_gemm(rt):
     C = torch.empty((128, 256), dtype=torch.bfloat16, device="cuda")
     with pytest.raises(f.FlepError):
         rt.launch(k, f.gemm_grid(128, 256), f.gemm_args(C, A, B))
+
+
+# ---- barrier-free CLC form (flep_clc_ring, reading R38): warp-task bodies at K = 1 ----------------
+
+def test_clc_ring_and_barrier_forms_agree_bitwise(rt, torch_mod):
+    """K = 1 selects the mbarrier-ring form for the stencil and SpMV-vector bodies, K = 2 the
+    barrier form: the same blocks, so identical outputs (and the oracle's within fp32 tolerance)."""
+    f = flep_mod()
+    n = 4096 + 37                                        # ragged tiles
+    a = gen.stencil_f32_input(n, seed=41)
+    ind = t(a)
+    outs = []
+    for poll in (1, 2):
+        k = rt.register_kernel(f.BODY_STENCIL5_F32, chunk=1, poll=poll, clc=True)
+        o = torch_mod.empty_like(ind)
+        h = rt.launch(k, f.stencil_grid(n), f.stencil_args(o, ind))
+        rt.sync(h, timeout_ns=10_000_000_000)
+        g = f.stencil_grid(n)
+        assert np.all(rt.coverage_np(h, g[0] * g[1]) == 1)
+        outs.append(o)
+    assert torch_mod.equal(outs[0].view(torch_mod.int32), outs[1].view(torch_mod.int32))
+    ref, absum = W.stencil5_f32(a)
+    assert _rel_err(outs[0].cpu().numpy(), ref, absum) <= REL_FP32
+    rows = (1 << 16) + 5
+    rp, col, val, x = gen.csr_inputs(rows, seed=42)
+    args_in = (t(rp), t(col), t(val), t(x))
+    ys = []
+    for poll in (1, 2):
+        k = rt.register_kernel(f.BODY_SPMV_CSR_F32_VEC, chunk=1, poll=poll, clc=True)
+        y = torch_mod.zeros(rows, device="cuda")
+        h = rt.launch(k, f.spmv_grid(rows), f.spmv_args(y, *args_in))
+        rt.sync(h, timeout_ns=10_000_000_000)
+        assert np.all(rt.coverage_np(h, f.spmv_grid(rows)[0]) == 1)
+        ys.append(y)
+    assert torch_mod.equal(ys[0].view(torch_mod.int32), ys[1].view(torch_mod.int32))
+    ref, absum = W.spmv_csr(rp, col, val, x)
+    assert _rel_err(ys[0].cpu().numpy(), ref, absum) <= REL_FP32
+
+
+@pytest.mark.parametrize("seed", range(int(os.environ.get("FLEP_RING_SEEDS", "4"))))
+def test_clc_ring_random_preempt_resume_exactly_once(rt, torch_mod, seed):
+    """The ring form under random temporal/spatial requests and resumes: a stencil-i32 16384²
+    victim (65536 tiles) runs every tile once, output bit-exact against the oracle's closed form."""
+    f = flep_mod()
+    g = gen.rng(900 + seed)
+    n = 16384
+    a = gen.stencil_i32_input(n, seed=50 + seed)
+    ind = t(a)
+    outd = torch_mod.empty_like(ind)
+    k = rt.register_kernel(f.BODY_STENCIL5_I32, chunk=1, poll=1, clc=True)
+    h = rt.launch(k, f.stencil_grid(n), f.stencil_args(outd, ind), priority=0)
+    requests = []
+    try:
+        for _ in range(int(g.integers(1, 5))):
+            time.sleep(float(g.uniform(5e-6, 80e-6)))
+            nsm = rt.num_sms if g.random() < 0.5 else int(g.integers(1, rt.num_sms))
+            rt.preempt(h, nsm)
+            requests.append(nsm)
+            time.sleep(float(g.uniform(5e-6, 80e-6)))
+            rt.resume(h)
+    except f.FlepError:                 # the grid completed between two requests
+        assert rt.query(h).state == f.STATE_DONE
+    rt.sync(h, timeout_ns=20_000_000_000)
+    gr = f.stencil_grid(n)
+    assert np.all(rt.coverage_np(h, gr[0] * gr[1]) == 1)
+    assert np.array_equal(outd.cpu().numpy(), W.stencil5_i32(a))
+    if len(requests) == 1 and requests[0] < rt.num_sms:  # I3 when the one request was spatial
+        for e in rt.events(h, 1):
+            if e.reason == f.REASON_YIELD:
+                assert e.smid < requests[0]
+
+
+def test_clc_ring_temporal_preempt_releases_sms(rt, torch_mod):
+    """A temporal request on a ring-form victim: first-wave workers yield, the waiting kernel runs,
+    the resumed victim completes exactly once."""
+    f = flep_mod()
+    n = 16384
+    a = gen.stencil_i32_input(n, seed=60)
+    ind = t(a)
+    outd = torch_mod.empty_like(ind)
+    x2, y2 = gen.saxpy_i32_inputs(1 << 20, seed=61)
+    x2d, y2d = t(x2), t(y2)
+    k = rt.register_kernel(f.BODY_STENCIL5_I32, chunk=1, poll=1, clc=True)
+    k_hp = rt.register_kernel(f.BODY_SAXPY_I32, chunk=4, poll=1)
+    h = rt.launch(k, f.stencil_grid(n), f.stencil_args(outd, ind), priority=0)
+    time.sleep(30e-6)
+    rt.preempt(h, rt.num_sms)
+    h2 = rt.launch(k_hp, f.saxpy_grid(1 << 20), f.saxpy_i32_args(y2d, x2d, 5), priority=1)
+    rt.sync(h2, timeout_ns=10_000_000_000)
+    _resume_unless_done(rt, f, h)
+    rt.sync(h, timeout_ns=20_000_000_000)
+    torch_mod.cuda.synchronize()
+    gr = f.stencil_grid(n)
+    assert np.all(rt.coverage_np(h, gr[0] * gr[1]) == 1)
+    assert np.array_equal(outd.cpu().numpy(), W.stencil5_i32(a))
+    assert np.array_equal(y2d.cpu().numpy(), W.saxpy_i32(5, x2, y2))
+    assert any(e.reason == f.REASON_YIELD for e in rt.events(h, 1)), "no first-wave worker yielded"
