@@ -802,6 +802,9 @@ def _qopts(F, ty, body):
     spec = os.environ.get("FLEP_QUEUE_FETCH", "spec") == "spec"
     C, pf = (QUEUE_CHUNK_SPEC if spec else QUEUE_CHUNK)[ty]
     gemm = body in (F.BODY_GEMM_BF16, F.BODY_GEMM_BF16_2SM, F.BODY_GEMM_BF16_2SM_W)
+    if ty == "stencil_f32" and os.environ.get("FLEP_QUEUE_STENCIL") == "clc":
+        # experiment: the stencil victims on the CLC fetch at C = K = 1 (the barrier-free form, R38)
+        return dict(chunk=1, poll=1, clc=True)
     return dict(chunk=C, poll=1, prefetch=pf, spec_fetch=spec and not gemm and ty != "saxpy_f32", in_tile=gemm)
 
 
