@@ -936,12 +936,15 @@ flep_clc_ring(const __grid_constant__ typename Body::Args args, const WorkerPara
     e.t_entry = ws.t_entry; e.t_exit = gtimer();
   }
 }
-// The ring form is chosen when the worker polls at every block (K = 1): the barrier form then
-// holds every warp behind thread 0's poll round trip at each block (measured: stencil 4096² C = K = 1
-// +18 % -> +9-10 %, SpMV-vector +6.7 % -> +3.7 %); at K >= 2 the barrier form is as fast or faster
-// (the warps of one CTA stay on one block: better L1 reuse of the stencil's halos).
+// The ring form is chosen when the worker polls at every block or every other block (K <= 2): the
+// barrier form then holds every warp behind thread 0's poll round trip (measured: stencil 4096²
+// C = K = 1 +18 % -> +9-10 %, SpMV-vector K = 1 +6.7 % -> +3.7 %, K = 2 61.0 -> 59.1 µs); at K = 4
+// the barrier form is faster (stencil 24.3 vs 24.6 µs).
+#ifndef FLEP_CLC_RING_MAXK
+#define FLEP_CLC_RING_MAXK 2         // the largest K that takes the ring form (build knob)
+#endif
 template <class Body>
-__host__ __device__ constexpr bool clc_use_ring(uint32_t poll) { return ClcRing<Body>::value && poll == 1u; }
+__host__ __device__ constexpr bool clc_use_ring(uint32_t poll) { return ClcRing<Body>::value && poll <= FLEP_CLC_RING_MAXK; }
 
 template <class Body, bool kCoverage>
 __global__ void __launch_bounds__(Body::kThreads, Body::kMinBlocks)

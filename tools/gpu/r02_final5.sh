@@ -1,6 +1,7 @@
 #!/bin/bash
 # Final validation after R38: the whole GPU suite, smoke, the default bench line and the reference arm.
 mkdir -p gpurun_out/f6
+rm -f gpurun_out/f6/*
 timeout 1500 python -m pytest tests -m gpu -q > gpurun_out/f6/pytest_gpu.log 2>&1; echo "pytest rc=$?" >> gpurun_out/f6/pytest_gpu.log
 tail -3 gpurun_out/f6/pytest_gpu.log
 timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/f6/smoke.log 2>&1; echo "smoke rc=$?"; tail -1 gpurun_out/f6/smoke.log
