@@ -24,7 +24,7 @@
 // and setup/teardown/kPersistent, inherited from flep::UserBody for bodies without per-worker
 // resources. A body whose run() uses no shared memory and no CTA barrier may declare
 //   static constexpr uint32_t kWarpTasks = kThreads / 32;
-// and then runs, with the CLC fetch at K = 1, without a CTA barrier between blocks (flep_clc_ring). Then, at namespace scope:
+// and then runs, with the CLC fetch at K <= 2, without a CTA barrier between blocks (flep_clc_ring). Then, at namespace scope:
 //   FLEP_DEFINE_BODY(my_body, MyBody)
 // defines extern "C" void my_body_ops(flep_body_ops* out), which fills the table that
 // flep_register_body(rt, &ops, &body_id) takes; body_id is then used in flep_kernel_desc.body.
